@@ -1,0 +1,798 @@
+// engine.cpp -- host orchestration of the hot path.
+//
+//   grid_build      a1-a4 on every device of the context (each holds the full
+//                   point set and its grid).
+//   neighbor_table  a5 sampled count + plan (Sec. VI, Eq. 1 P:736-741,
+//                   buffer rule P:812-823), query shards (devices x processes),
+//                   a6 exact count, a7 scan, the "final gather of counts" that
+//                   gives every shard its base offset, a8 batched write kernels
+//                   round-robin over n_streams streams with each
+//                   batch DMA'd straight into the host table (a9/a10: the
+//                   paper's T_i^min/max + B layout, without the
+//                   pinned->pageable staging copy), or a device-resident table.
+#include <algorithm>
+#include <chrono>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <exception>
+#include <memory>
+#include <thread>
+
+#include "internal.h"
+
+namespace hdb {
+
+// ------------------------------------------------------------------ errors
+static thread_local std::string g_err;
+
+void set_error(const char* fmt, ...) {
+    char buf[1024];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    g_err = buf;
+}
+
+void fail(hdb_status st, const char* fmt, ...) {
+    char buf[1024];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    g_err = buf;
+    throw Error{st};
+}
+
+const char* last_error() { return g_err.c_str(); }
+
+int resolve_threads(int req) {
+    if (req > 0) return req;
+    unsigned h = std::thread::hardware_concurrency();
+    return h ? (int)h : 1;
+}
+
+// ------------------------------------------------------------------ pools
+void* PinnedPool::acquire(size_t bytes, size_t* got) {
+    std::lock_guard<std::mutex> lk(m);
+    if (bytes == 0) bytes = 64;
+    auto it = free_blocks.lower_bound(bytes);
+    if (it != free_blocks.end() && it->first <= 2 * bytes + (64u << 20)) {
+        void* p = it->second;
+        *got = it->first;
+        free_blocks.erase(it);
+        return p;
+    }
+    size_t sz = (bytes + (2u << 20) - 1) & ~(size_t)((2u << 20) - 1);
+    void* p = nullptr;
+    cudaError_t e = cudaHostAlloc(&p, sz, cudaHostAllocPortable);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        for (auto& kv : free_blocks) {
+            cudaFreeHost(kv.second);
+            bytes_total -= kv.first;
+        }
+        free_blocks.clear();
+        e = cudaHostAlloc(&p, sz, cudaHostAllocPortable);
+        if (e != cudaSuccess) {
+            cudaGetLastError();
+            fail(HDB_ENOMEM, "pinned host allocation of %zu bytes failed: %s", sz, cudaGetErrorString(e));
+        }
+    }
+    bytes_total += sz;
+    ++grows;
+    *got = sz;
+    return p;
+}
+
+void PinnedPool::release(void* p, size_t bytes) {
+    if (!p) return;
+    std::lock_guard<std::mutex> lk(m);
+    free_blocks.emplace(bytes, p);
+}
+
+PinnedPool::~PinnedPool() {
+    for (auto& kv : free_blocks) cudaFreeHost(kv.second);
+}
+
+// ------------------------------------------------------------------ helpers
+namespace {
+
+struct DeviceGuard {
+    int prev = -1;
+    explicit DeviceGuard(int d) {
+        cudaGetDevice(&prev);
+        if (prev != d) HDB_CUDA(cudaSetDevice(d));
+    }
+    ~DeviceGuard() {
+        if (prev >= 0) cudaSetDevice(prev);
+    }
+};
+
+// stream-ordered device buffer, freed at scope exit unless released
+struct DBuf {
+    void* p = nullptr;
+    cudaStream_t s = nullptr;
+    DBuf() = default;
+    DBuf(size_t bytes, cudaStream_t st) : s(st) {
+        if (bytes == 0) bytes = 16;
+        cudaError_t e = cudaMallocAsync(&p, bytes, st);
+        if (e != cudaSuccess) {
+            cudaGetLastError();
+            p = nullptr;
+            fail(HDB_ENOMEM, "device allocation of %zu bytes failed: %s", bytes, cudaGetErrorString(e));
+        }
+    }
+    DBuf(const DBuf&) = delete;
+    DBuf& operator=(const DBuf&) = delete;
+    DBuf(DBuf&& o) noexcept : p(o.p), s(o.s) { o.p = nullptr; }
+    DBuf& operator=(DBuf&& o) noexcept {
+        reset();
+        p = o.p;
+        s = o.s;
+        o.p = nullptr;
+        return *this;
+    }
+    ~DBuf() { reset(); }
+    void reset() {
+        if (p) cudaFreeAsync(p, s);
+        p = nullptr;
+    }
+    void* release() {
+        void* q = p;
+        p = nullptr;
+        return q;
+    }
+    template <typename T>
+    T* as() const {
+        return (T*)p;
+    }
+};
+
+struct Event {
+    cudaEvent_t e = nullptr;
+    Event() { HDB_CUDA(cudaEventCreate(&e)); }
+    ~Event() {
+        if (e) cudaEventDestroy(e);
+    }
+    Event(const Event&) = delete;
+    Event& operator=(const Event&) = delete;
+};
+
+float elapsed(const Event& a, const Event& b) {
+    float ms = 0;
+    HDB_CUDA(cudaEventElapsedTime(&ms, a.e, b.e));
+    return ms;
+}
+
+constexpr uint64_t kMaxCellsAbs = 1ull << 30;
+
+enum class Loc { Host, Device };
+
+struct PtrInfo {
+    Loc loc = Loc::Host;
+    int device = -1;
+};
+
+PtrInfo classify(const void* p) {
+    PtrInfo r;
+    if (!p) return r;
+    cudaPointerAttributes a{};
+    cudaError_t e = cudaPointerGetAttributes(&a, p);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        return r;
+    }
+    if (a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged) {
+        r.loc = Loc::Device;
+        r.device = a.device;
+    }
+    return r;
+}
+
+void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t n, hdb_dtype dt, double eps,
+               DevGrid& g) {
+    DeviceGuard dg(dc.device);
+    cudaStream_t s = dc.main;
+    const size_t esz = dt == HDB_F64 ? 16 : 8;
+    g.device = dc.device;
+    g.dtype = dt;
+    g.n = n;
+    g.stream = s;
+    Event ev0, ev1;
+    HDB_CUDA(cudaEventRecord(ev0.e, s));
+
+    // ---- a1: ingest + bbox + validation
+    DBuf xin_owned;
+    const void* xin = xy;
+    if (n > 0) {
+        if (where.loc == Loc::Host) {
+            xin_owned = DBuf(n * esz, s);
+            HDB_CUDA(cudaMemcpyAsync(xin_owned.p, xy, n * esz, cudaMemcpyHostToDevice, s));
+            ctx->stats.bytes_h2d += n * esz;
+            xin = xin_owned.p;
+        } else if (where.device != dc.device) {
+            xin_owned = DBuf(n * esz, s);
+            HDB_CUDA(cudaMemcpyPeerAsync(xin_owned.p, dc.device, xy, where.device, n * esz, s));
+            xin = xin_owned.p;
+        }
+    }
+    DBuf misc(256, s);
+    unsigned long long* bb = misc.as<unsigned long long>();          // [0..3] bbox, [4] nonempty
+    unsigned int* bad = (unsigned int*)(bb + 5);
+    launch_bbox_init(bb, bad, s);
+    HDB_CUDA(cudaMemsetAsync(bb + 4, 0, 8, s));
+    launch_bbox(xin, n, dt, bb, bad, s);
+    HDB_LAUNCH_CHECK();
+    unsigned long long hb[6];
+    HDB_CUDA(cudaMemcpyAsync(hb, bb, sizeof hb, cudaMemcpyDeviceToHost, s));
+    HDB_CUDA(cudaStreamSynchronize(s));
+    if ((unsigned int)hb[5] != 0) fail(HDB_EINVAL, "%u non-finite coordinate(s)", (unsigned)hb[5]);
+
+    double eps_used = eps;
+    if (dt == HDB_F32) {
+        float ef = (float)eps;
+        if (!(ef > 0.0f) || !std::isfinite(ef)) fail(HDB_EINVAL, "eps=%g is not a positive finite float", eps);
+        eps_used = (double)ef;
+        g.e2_f = ef * ef;               // fl32(eps_f * eps_f)
+    }
+    g.e2_d = eps_used * eps_used;       // fl64(eps * eps)
+    g.eps = eps_used;
+    g.w = eps_used * (1.0 + 0x1p-19);   // reading R9
+    g.inv_w = 1.0 / g.w;
+    if (n > 0) {
+        g.xmin = bbox_decode(hb[0], false);
+        g.ymin = bbox_decode(hb[1], false);
+        g.xmax = bbox_decode(hb[2], true);
+        g.ymax = bbox_decode(hb[3], true);
+    }
+    const double ex = (g.xmax - g.xmin) * g.inv_w;   // same rounded ops as the key kernel
+    const double ey = (g.ymax - g.ymin) * g.inv_w;
+    if (!(ex <= 0x1p30) || !(ey <= 0x1p30))
+        fail(HDB_ERANGE, "extent/eps too large (%g x %g cells > 2^30)", ex, ey);
+    g.nx = (uint32_t)std::floor(ex) + 1;
+    g.ny = (uint32_t)std::floor(ey) + 1;
+    g.n_cells = (uint64_t)g.nx * g.ny;
+    const uint64_t cell_cap = std::min<uint64_t>(kMaxCellsAbs, 64 * n + (1ull << 24));
+    if (g.n_cells > cell_cap)
+        fail(HDB_ERANGE, "grid of %u x %u = %llu cells exceeds the dense-grid limit %llu", g.nx, g.ny,
+             (unsigned long long)g.n_cells, (unsigned long long)cell_cap);
+    const uint64_t C = g.n_cells;
+
+    // ---- a2: keys
+    DBuf k0(4 * n, s), v0(4 * n, s), k1(4 * n, s), v1(4 * n, s);
+    launch_keys(xin, n, dt, g.xmin, g.ymin, g.inv_w, g.nx, g.ny, k0.as<uint32_t>(), v0.as<uint32_t>(), s);
+    HDB_LAUNCH_CHECK();
+    // ---- a3: stable radix sort by key
+    int bits = 1;
+    while (bits < 32 && (1ull << bits) < C) ++bits;
+    size_t tb = std::max(radix_sort_temp_bytes(n), scan_temp_bytes(std::max<uint64_t>(n, C) + 1));
+    DBuf temp(tb, s);
+    int which = radix_sort_pairs(k0.as<uint32_t>(), v0.as<uint32_t>(), k1.as<uint32_t>(), v1.as<uint32_t>(), n,
+                                 bits, temp.p, s);
+    HDB_LAUNCH_CHECK();
+    DBuf keys = which ? std::move(k1) : std::move(k0);
+    DBuf ids = which ? std::move(v1) : std::move(v0);
+    k0.reset();
+    k1.reset();
+    v0.reset();
+    v1.reset();
+    DBuf xy_s(n * esz, s);
+    launch_gather_points(xin, ids.as<uint32_t>(), n, dt, xy_s.p, s);
+    HDB_LAUNCH_CHECK();
+    xin_owned.reset();
+    // ---- a4: per-cell counts -> exclusive scan -> G
+    DBuf cnt(4 * C, s);
+    HDB_CUDA(cudaMemsetAsync(cnt.p, 0, 4 * C, s));
+    launch_cell_counts(keys.as<uint32_t>(), n, cnt.as<uint32_t>(), bb + 4, s);
+    DBuf start(4 * (C + 1), s);
+    scan_u32_to_u32(cnt.as<uint32_t>(), start.as<uint32_t>(), C, temp.p, s);
+    cnt.reset();
+    // ---- query groups
+    DBuf flags(4 * n, s), pos(4 * (n + 1), s);
+    launch_group_flags(keys.as<uint32_t>(), start.as<uint32_t>(), n, flags.as<uint32_t>(), s);
+    scan_u32_to_u32(flags.as<uint32_t>(), pos.as<uint32_t>(), n, temp.p, s);
+    HDB_LAUNCH_CHECK();
+    uint32_t hng = 0;
+    HDB_CUDA(cudaMemcpyAsync(&hng, pos.as<uint32_t>() + n, 4, cudaMemcpyDeviceToHost, s));
+    HDB_CUDA(cudaMemcpyAsync(hb, bb + 4, 8, cudaMemcpyDeviceToHost, s));
+    HDB_CUDA(cudaStreamSynchronize(s));
+    g.n_groups = hng;
+    g.n_nonempty = hb[0];
+    DBuf gstart(4 * (g.n_groups + 1), s);
+    launch_group_scatter(flags.as<uint32_t>(), pos.as<uint32_t>(), n, gstart.as<uint32_t>(), s);
+    HDB_LAUNCH_CHECK();
+    flags.reset();
+    pos.reset();
+    temp.reset();
+    misc.reset();
+    HDB_CUDA(cudaEventRecord(ev1.e, s));
+    HDB_CUDA(cudaEventSynchronize(ev1.e));
+    g.ms_build = elapsed(ev0, ev1);
+    g.xy_s = xy_s.release();
+    g.ids = (uint32_t*)ids.release();
+    g.keys = (uint32_t*)keys.release();
+    g.start = (uint32_t*)start.release();
+    g.gstart = (uint32_t*)gstart.release();
+}
+
+void free_dev_grid(DevGrid& g) {
+    if (!g.stream) return;
+    DeviceGuard dg(g.device);
+    for (void* p : {(void*)g.xy_s, (void*)g.ids, (void*)g.keys, (void*)g.start, (void*)g.gstart})
+        if (p) cudaFreeAsync(p, g.stream);
+    g.xy_s = nullptr;
+    g.ids = g.keys = g.start = g.gstart = nullptr;
+    cudaStreamSynchronize(g.stream);
+}
+
+}  // namespace
+
+// ------------------------------------------------------------------ grid
+void grid_build(hdb_ctx* ctx, const void* xy, uint64_t n, hdb_dtype dt, double eps, hdb_grid** out) {
+    if (dt != HDB_F64 && dt != HDB_F32) fail(HDB_EINVAL, "unknown dtype %d", (int)dt);
+    if (!std::isfinite(eps) || !(eps > 0)) fail(HDB_EINVAL, "eps=%g must be finite and > 0", eps);
+    if (n >= 0xffffffffull) fail(HDB_ERANGE, "n=%llu >= 2^32-1", (unsigned long long)n);
+    if (n > 0 && !xy) fail(HDB_EINVAL, "xy is NULL with n=%llu", (unsigned long long)n);
+    PtrInfo where = classify(xy);
+    uint64_t launches0 = g_kernel_launches.load();
+    auto* g = new hdb_grid;
+    g->ctx = ctx;
+    g->dev.resize(ctx->dev.size());
+    try {
+        for (size_t d = 0; d < ctx->dev.size(); ++d) build_dev(ctx, ctx->dev[d], xy, where, n, dt, eps, g->dev[d]);
+    } catch (...) {
+        for (auto& dg : g->dev) free_dev_grid(dg);
+        delete g;
+        throw;
+    }
+    const DevGrid& g0 = g->dev[0];
+    ctx->stats.n = n;
+    ctx->stats.n_cells = g0.n_cells;
+    ctx->stats.n_nonempty = g0.n_nonempty;
+    ctx->stats.n_groups = g0.n_groups;
+    ctx->stats.ms_grid = g0.ms_build;
+    ctx->stats.kernel_launches = (uint32_t)(g_kernel_launches.load() - launches0);
+    ctx->live_objects++;
+    *out = g;
+}
+
+void grid_free(hdb_grid* g) {
+    if (!g) return;
+    for (auto& dg : g->dev) free_dev_grid(dg);
+    if (g->ctx) g->ctx->live_objects--;
+    delete g;
+}
+
+// ------------------------------------------------------------------ table
+namespace {
+
+struct ShardRange {
+    uint64_t g0 = 0, g1 = 0;   // query groups
+    uint64_t q0 = 0, q1 = 0;   // sorted query positions
+};
+
+struct ShardState {
+    ShardRange r;
+    DBuf cnt, off;
+    uint64_t pairs = 0;
+    uint64_t tests = 0;
+    uint64_t base = 0;   // global offset of this shard's first pair
+    float ms_count = 0, ms_scan = 0, ms_write = 0;
+    uint32_t write_launches = 0;
+    uint64_t n_batches = 0, max_batch = 0, d2h = 0;
+};
+
+// Sorted position -> group boundaries for `parts` shards balanced by the sampled counts.
+std::vector<uint64_t> shard_cuts(const DevGrid& g, DevCtx& dc, const std::vector<uint32_t>& samp, uint64_t stride,
+                                 uint32_t parts) {
+    std::vector<uint64_t> cuts(parts + 1, 0);
+    cuts[parts] = g.n_groups;
+    if (parts <= 1) return cuts;
+    std::vector<uint64_t> pre(samp.size() + 1, 0);
+    for (size_t j = 0; j < samp.size(); ++j) pre[j + 1] = pre[j] + samp[j];
+    std::vector<uint64_t> scut(parts + 1);
+    hdb_balanced_cuts(pre.data(), samp.size(), parts, scut.data());
+    std::vector<uint64_t> posv(parts - 1);
+    for (uint32_t k = 1; k < parts; ++k) posv[k - 1] = std::min<uint64_t>(scut[k] * stride, g.n);
+    cudaStream_t s = dc.main;
+    DBuf dpos(8 * posv.size(), s), dgrp(8 * posv.size(), s);
+    HDB_CUDA(cudaMemcpyAsync(dpos.p, posv.data(), 8 * posv.size(), cudaMemcpyHostToDevice, s));
+    launch_pos_to_group(g.gstart, g.n_groups, dpos.as<uint64_t>(), (uint32_t)posv.size(), dgrp.as<uint64_t>(), s);
+    std::vector<uint64_t> grp(posv.size());
+    HDB_CUDA(cudaMemcpyAsync(grp.data(), dgrp.p, 8 * grp.size(), cudaMemcpyDeviceToHost, s));
+    HDB_CUDA(cudaStreamSynchronize(s));
+    for (uint32_t k = 1; k < parts; ++k) cuts[k] = std::max(cuts[k - 1], grp[k - 1]);
+    return cuts;
+}
+
+uint32_t read_u32(const uint32_t* d, cudaStream_t s) {
+    uint32_t v = 0;
+    HDB_CUDA(cudaMemcpyAsync(&v, d, 4, cudaMemcpyDeviceToHost, s));
+    HDB_CUDA(cudaStreamSynchronize(s));
+    return v;
+}
+
+// a6 + a7 on one device for one shard
+void count_phase(hdb_ctx* ctx, DevCtx& dc, const DevGrid& g, ShardState& st) {
+    DeviceGuard dg(dc.device);
+    cudaStream_t s = dc.main;
+    const uint64_t n = g.n;
+    if (st.r.g1 > st.r.g0) {
+        st.r.q0 = read_u32(g.gstart + st.r.g0, s);
+        st.r.q1 = read_u32(g.gstart + st.r.g1, s);
+    } else {
+        st.r.q0 = st.r.q1 = 0;
+    }
+    st.cnt = DBuf(4 * (n ? n : 1), s);
+    st.off = DBuf(8 * (n + 1), s);
+    DBuf tests(8, s);
+    HDB_CUDA(cudaMemsetAsync(tests.p, 0, 8, s));
+    Event e0, e1, e2;
+    HDB_CUDA(cudaEventRecord(e0.e, s));
+    launch_count(g, st.r.g0, st.r.g1, st.cnt.as<uint32_t>(), tests.as<unsigned long long>(), ctx->opts.search_kernel,
+                 s);
+    HDB_LAUNCH_CHECK();
+    HDB_CUDA(cudaEventRecord(e1.e, s));
+    const uint64_t len = st.r.q1 - st.r.q0;
+    DBuf temp(scan_temp_bytes(len + 1), s);
+    scan_u32_to_u64(st.cnt.as<uint32_t>() + st.r.q0, st.off.as<uint64_t>() + st.r.q0, len, temp.p, s);
+    HDB_LAUNCH_CHECK();
+    HDB_CUDA(cudaEventRecord(e2.e, s));
+    uint64_t h[2] = {0, 0};
+    HDB_CUDA(cudaMemcpyAsync(&h[0], st.off.as<uint64_t>() + st.r.q1, 8, cudaMemcpyDeviceToHost, s));
+    HDB_CUDA(cudaMemcpyAsync(&h[1], tests.p, 8, cudaMemcpyDeviceToHost, s));
+    HDB_CUDA(cudaStreamSynchronize(s));
+    st.pairs = h[0];
+    st.tests = h[1];
+    st.ms_count = elapsed(e0, e1);
+    st.ms_scan = elapsed(e1, e2);
+}
+
+void ensure_batch_buf(DevCtx& dc, size_t si, size_t pairs, uint64_t* grows) {
+    if (dc.batch_buf.size() <= si) {
+        dc.batch_buf.resize(si + 1, nullptr);
+        dc.batch_cap.resize(si + 1, 0);
+    }
+    if (dc.batch_cap[si] >= pairs && dc.batch_buf[si]) return;
+    if (dc.batch_buf[si]) {
+        HDB_CUDA(cudaStreamSynchronize(dc.streams[si]));
+        cudaFree(dc.batch_buf[si]);
+        dc.batch_buf[si] = nullptr;
+        dc.batch_cap[si] = 0;
+    }
+    size_t cap = std::max<size_t>(pairs, 1024);
+    cap += cap / 8;
+    void* p = nullptr;
+    cudaError_t e = cudaMalloc(&p, cap * 4);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        fail(HDB_ENOMEM, "device batch buffer of %zu pairs: %s", cap, cudaGetErrorString(e));
+    }
+    dc.batch_buf[si] = (uint32_t*)p;
+    dc.batch_cap[si] = cap;
+    ++*grows;
+}
+
+// a8 + a9 for one shard: batches cut on exact counts, round-robin on streams,
+// each batch written into a per-stream device buffer and DMA'd into the host
+// table at its final offset.
+void write_phase_host(hdb_ctx* ctx, DevCtx& dc, const DevGrid& g, ShardState& st, uint32_t* h_nbrs,
+                      uint64_t batch_pairs, uint64_t* grows) {
+    DeviceGuard dg(dc.device);
+    if (st.pairs == 0) return;
+    cudaStream_t s = dc.main;
+    const uint32_t S = (uint32_t)dc.streams.size();
+    uint64_t nb = (st.pairs + batch_pairs - 1) / batch_pairs;
+    nb = std::max<uint64_t>(nb, 1);
+    nb = std::min<uint64_t>(nb, std::max<uint64_t>(1, st.r.g1 - st.r.g0));
+    DBuf dcut(8 * (nb + 1) * 2, s);
+    uint64_t* gcut = dcut.as<uint64_t>();
+    uint64_t* pcut = gcut + (nb + 1);
+    // offsets are relative to the shard start: off[q0] == 0
+    launch_batch_cuts(g.gstart, st.off.as<uint64_t>(), st.r.g0, st.r.g1, (uint32_t)nb, gcut, pcut, s);
+    HDB_LAUNCH_CHECK();
+    std::vector<uint64_t> hc(2 * (nb + 1));
+    HDB_CUDA(cudaMemcpyAsync(hc.data(), dcut.p, 8 * hc.size(), cudaMemcpyDeviceToHost, s));
+    HDB_CUDA(cudaStreamSynchronize(s));
+    const uint64_t* hg = hc.data();
+    const uint64_t* hp = hc.data() + (nb + 1);
+    uint64_t maxb = 0;
+    for (uint64_t b = 0; b < nb; ++b) maxb = std::max(maxb, hp[b + 1] - hp[b]);
+    for (uint32_t i = 0; i < S && i < nb; ++i) ensure_batch_buf(dc, i, maxb, grows);
+    Event ready;
+    HDB_CUDA(cudaEventRecord(ready.e, s));
+    std::vector<Event> evs(2 * nb);
+    for (uint64_t b = 0; b < nb; ++b) {
+        const uint32_t si = (uint32_t)(b % S);
+        cudaStream_t ss = dc.streams[si];
+        const uint64_t pairs_b = hp[b + 1] - hp[b];
+        if (b < S) HDB_CUDA(cudaStreamWaitEvent(ss, ready.e, 0));
+        HDB_CUDA(cudaEventRecord(evs[2 * b].e, ss));
+        launch_write(g, hg[b], hg[b + 1], st.off.as<uint64_t>(), hp[b], dc.batch_buf[si], ctx->opts.search_kernel,
+                     ss);
+        HDB_LAUNCH_CHECK();
+        HDB_CUDA(cudaEventRecord(evs[2 * b + 1].e, ss));
+        if (pairs_b)
+            HDB_CUDA(cudaMemcpyAsync(h_nbrs + st.base + hp[b], dc.batch_buf[si], 4 * pairs_b, cudaMemcpyDeviceToHost,
+                                     ss));
+        st.d2h += 4 * pairs_b;
+    }
+    for (uint32_t i = 0; i < S; ++i) HDB_CUDA(cudaStreamSynchronize(dc.streams[i]));
+    for (uint64_t b = 0; b < nb; ++b) st.ms_write += elapsed(evs[2 * b], evs[2 * b + 1]);
+    st.write_launches += (uint32_t)nb;
+    st.n_batches = nb;
+    st.max_batch = maxb;
+}
+
+template <typename F>
+void run_parallel(size_t k, F&& f) {
+    if (k == 1) {
+        f(0);
+        return;
+    }
+    std::vector<std::exception_ptr> errs(k);
+    std::vector<std::string> msgs(k);
+    std::vector<std::thread> th;
+    for (size_t i = 0; i < k; ++i)
+        th.emplace_back([&, i] {
+            try {
+                f(i);
+            } catch (...) {
+                errs[i] = std::current_exception();
+                msgs[i] = last_error();
+            }
+        });
+    for (auto& t : th) t.join();
+    for (size_t i = 0; i < k; ++i)
+        if (errs[i]) {
+            g_err = msgs[i];
+            std::rethrow_exception(errs[i]);
+        }
+}
+
+template <typename T>
+T* pool_get(hdb_table* t, size_t count, size_t* cap) {
+    return (T*)t->pool->acquire(count * sizeof(T), cap);
+}
+
+}  // namespace
+
+void table_free(hdb_table* t) {
+    if (!t) return;
+    if (t->on_device) {
+        DeviceGuard dg(t->device);
+        for (void* p : {(void*)t->begin, (void*)t->count, (void*)t->nbrs})
+            if (p) cudaFreeAsync(p, t->dstream);
+        cudaStreamSynchronize(t->dstream);
+    } else if (t->pool) {
+        t->pool->release(t->begin, t->cap_begin);
+        t->pool->release(t->count, t->cap_count);
+        t->pool->release(t->nbrs, t->cap_nbrs);
+    } else if (t->malloced) {
+        free(t->begin);
+        free(t->count);
+        free(t->nbrs);
+    }
+    if (t->ctx) t->ctx->live_objects--;
+    delete t;
+}
+
+void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hdb_table** out) {
+    auto t_wall0 = std::chrono::steady_clock::now();
+    const uint64_t launches0 = g_kernel_launches.load();
+    hdb_stats& S = ctx->stats;
+    const DevGrid& G0 = grid->dev[0];
+    const uint64_t n = G0.n;
+    S.n = n;
+    S.n_cells = G0.n_cells;
+    S.n_nonempty = G0.n_nonempty;
+    S.n_groups = G0.n_groups;
+    S.bytes_d2h = 0;
+    S.pool_grows = 0;
+    S.n_streams = ctx->opts.n_streams;
+    const uint32_t R_proc = ctx->opts.shard_count > 0 ? (uint32_t)ctx->opts.shard_count : 1;
+    const uint32_t rank = ctx->opts.shard_count > 0 ? (uint32_t)ctx->opts.shard_rank : 0;
+    const size_t ndev = device_resident ? 1 : grid->dev.size();
+    S.n_devices = (int)ndev;
+
+    auto* t = new hdb_table;
+    t->n = n;
+    t->eps = G0.eps;
+    t->dtype = G0.dtype;
+    t->host_threads = ctx->opts.host_threads;
+    std::vector<ShardState> sh(ndev);
+    try {
+        // ---- a5: sampled count + plan (device 0)
+        DevCtx& dc0 = ctx->dev[0];
+        DeviceGuard dg0(dc0.device);
+        const double f = ctx->opts.sample_fraction;
+        const uint64_t stride = std::max<uint64_t>(1, (uint64_t)std::floor(1.0 / f));
+        const uint64_t ns = n ? (n + stride - 1) / stride : 0;
+        std::vector<uint32_t> samp(ns);
+        {
+            cudaStream_t s = dc0.main;
+            DBuf dsamp(4 * (ns ? ns : 1), s), dsum(8, s);
+            HDB_CUDA(cudaMemsetAsync(dsum.p, 0, 8, s));
+            Event e0, e1;
+            HDB_CUDA(cudaEventRecord(e0.e, s));
+            launch_sample_count(G0, stride, ns, dsamp.as<uint32_t>(), dsum.as<unsigned long long>(), s);
+            HDB_LAUNCH_CHECK();
+            HDB_CUDA(cudaEventRecord(e1.e, s));
+            uint64_t eb = 0;
+            HDB_CUDA(cudaMemcpyAsync(&eb, dsum.p, 8, cudaMemcpyDeviceToHost, s));
+            if (ns) HDB_CUDA(cudaMemcpyAsync(samp.data(), dsamp.p, 4 * ns, cudaMemcpyDeviceToHost, s));
+            HDB_CUDA(cudaStreamSynchronize(s));
+            S.sample_size = ns;
+            S.sample_pairs = eb;
+            S.est_pairs = eb * stride;   // a_b = e_b / f  (reading R15)
+            S.ms_sample = elapsed(e0, e1);
+        }
+        double bb_plan = 0;
+        uint64_t nb_plan = 0;
+        hdb_plan_batches((double)S.est_pairs, ctx->opts.alpha, ctx->opts.n_streams, &bb_plan, &nb_plan);
+        uint64_t batch_pairs = ctx->opts.batch_pairs ? ctx->opts.batch_pairs : (uint64_t)std::ceil(bb_plan);
+        batch_pairs = std::max<uint64_t>(batch_pairs, 1);
+        S.planned_batch_pairs = batch_pairs;
+        S.planned_batches = ctx->opts.batch_pairs
+                                ? (uint64_t)std::ceil((1.0 + ctx->opts.alpha) * (double)S.est_pairs / (double)batch_pairs)
+                                : nb_plan;
+
+        // ---- query shards: processes x devices, balanced by sampled counts
+        const uint32_t parts = R_proc * (uint32_t)ndev;
+        std::vector<uint64_t> cuts = shard_cuts(G0, dc0, samp, stride, parts);
+        for (size_t d = 0; d < ndev; ++d) {
+            const uint32_t k = rank * (uint32_t)ndev + (uint32_t)d;
+            sh[d].r.g0 = cuts[k];
+            sh[d].r.g1 = cuts[k + 1];
+        }
+        // ---- a6/a7 on every device
+        run_parallel(ndev, [&](size_t d) { count_phase(ctx, ctx->dev[d], grid->dev[d], sh[d]); });
+        // ---- the final gather of counts: shard bases
+        uint64_t P = 0;
+        for (size_t d = 0; d < ndev; ++d) {
+            sh[d].base = P;
+            P += sh[d].pairs;
+        }
+        S.npairs = P;
+        S.candidate_tests = 0;
+        S.ms_count = S.ms_scan = 0;
+        for (auto& st : sh) {
+            S.candidate_tests += st.tests;
+            S.ms_count = std::max(S.ms_count, (double)st.ms_count);
+            S.ms_scan = std::max(S.ms_scan, (double)st.ms_scan);
+        }
+        if (ctx->opts.host_budget_bytes && 4 * P > ctx->opts.host_budget_bytes && !device_resident)
+            fail(HDB_ENOMEM, "table needs %llu bytes (P=%llu) > host budget %llu", (unsigned long long)(4 * P),
+                 (unsigned long long)P, (unsigned long long)ctx->opts.host_budget_bytes);
+        t->npairs = P;
+        const bool whole = (parts == 1);
+        t->first_query = whole ? 0 : sh[0].r.q0;
+        t->end_query = whole ? n : sh[ndev - 1].r.q1;
+
+        if (device_resident) {
+            // ---- a8 into a device-resident table
+            DevCtx& dc = ctx->dev[0];
+            const DevGrid& g = grid->dev[0];
+            ShardState& st = sh[0];
+            cudaStream_t s = dc.main;
+            t->on_device = true;
+            t->device = dc.device;
+            t->dstream = s;
+            DBuf nb(4 * (P ? P : 1), s), beg(8 * (n ? n : 1), s), cnt(4 * (n ? n : 1), s);
+            if (!whole) {
+                HDB_CUDA(cudaMemsetAsync(beg.p, 0, 8 * (n ? n : 1), s));
+                HDB_CUDA(cudaMemsetAsync(cnt.p, 0, 4 * (n ? n : 1), s));
+            }
+            Event e0, e1;
+            HDB_CUDA(cudaEventRecord(e0.e, s));
+            launch_write(g, st.r.g0, st.r.g1, st.off.as<uint64_t>(), 0, nb.as<uint32_t>(), ctx->opts.search_kernel, s);
+            HDB_LAUNCH_CHECK();
+            HDB_CUDA(cudaEventRecord(e1.e, s));
+            launch_scatter_rows(g.ids, st.off.as<uint64_t>(), st.cnt.as<uint32_t>(), st.r.q0, st.r.q1, 0,
+                                beg.as<uint64_t>(), cnt.as<uint32_t>(), s);
+            HDB_LAUNCH_CHECK();
+            HDB_CUDA(cudaStreamSynchronize(s));
+            st.ms_write = elapsed(e0, e1);
+            st.write_launches = 1;
+            st.n_batches = 1;
+            st.max_batch = P;
+            t->nbrs = (uint32_t*)nb.release();
+            t->begin = (uint64_t*)beg.release();
+            t->count = (uint32_t*)cnt.release();
+        } else {
+            // ---- a8/a9/a10 into the host table
+            t->pool = ctx->pinned;
+            uint64_t grows0 = ctx->pinned->grows;
+            t->nbrs = pool_get<uint32_t>(t, P ? P : 1, &t->cap_nbrs);
+            t->begin = pool_get<uint64_t>(t, n ? n : 1, &t->cap_begin);
+            t->count = pool_get<uint32_t>(t, n ? n : 1, &t->cap_count);
+            if (!whole) {
+                memset(t->begin, 0, 8 * (n ? n : 1));
+                memset(t->count, 0, 4 * (n ? n : 1));
+            }
+            std::vector<uint64_t> dev_grows(ndev, 0);
+            run_parallel(ndev, [&](size_t d) {
+                write_phase_host(ctx, ctx->dev[d], grid->dev[d], sh[d], t->nbrs, batch_pairs, &dev_grows[d]);
+            });
+            // begin/count by original id
+            if (whole) {
+                DevCtx& dc = ctx->dev[0];
+                DeviceGuard dg(dc.device);
+                cudaStream_t s = dc.main;
+                DBuf beg(8 * (n ? n : 1), s), cnt(4 * (n ? n : 1), s);
+                launch_scatter_rows(grid->dev[0].ids, sh[0].off.as<uint64_t>(), sh[0].cnt.as<uint32_t>(), 0, n, 0,
+                                    beg.as<uint64_t>(), cnt.as<uint32_t>(), s);
+                HDB_LAUNCH_CHECK();
+                if (n) {
+                    HDB_CUDA(cudaMemcpyAsync(t->begin, beg.p, 8 * n, cudaMemcpyDeviceToHost, s));
+                    HDB_CUDA(cudaMemcpyAsync(t->count, cnt.p, 4 * n, cudaMemcpyDeviceToHost, s));
+                }
+                HDB_CUDA(cudaStreamSynchronize(s));
+                S.bytes_d2h += 12 * n;
+            } else {
+                run_parallel(ndev, [&](size_t d) {
+                    ShardState& st = sh[d];
+                    const uint64_t len = st.r.q1 - st.r.q0;
+                    if (!len) return;
+                    DeviceGuard dg(ctx->dev[d].device);
+                    cudaStream_t s = ctx->dev[d].main;
+                    std::vector<uint32_t> ids(len), cnt(len);
+                    std::vector<uint64_t> off(len);
+                    HDB_CUDA(cudaMemcpyAsync(ids.data(), grid->dev[d].ids + st.r.q0, 4 * len, cudaMemcpyDeviceToHost, s));
+                    HDB_CUDA(cudaMemcpyAsync(cnt.data(), st.cnt.as<uint32_t>() + st.r.q0, 4 * len,
+                                             cudaMemcpyDeviceToHost, s));
+                    HDB_CUDA(cudaMemcpyAsync(off.data(), st.off.as<uint64_t>() + st.r.q0, 8 * len,
+                                             cudaMemcpyDeviceToHost, s));
+                    HDB_CUDA(cudaStreamSynchronize(s));
+                    for (uint64_t i = 0; i < len; ++i) {
+                        t->begin[ids[i]] = off[i] + st.base;
+                        t->count[ids[i]] = cnt[i];
+                    }
+                    st.d2h += 16 * len;
+                });
+            }
+            for (size_t d = 0; d < ndev; ++d) S.pool_grows += dev_grows[d];
+            S.pool_grows += ctx->pinned->grows - grows0;
+            if (ctx->opts.sort_lists) {
+                const int T = resolve_threads(ctx->opts.host_threads);
+                run_parallel((size_t)T, [&](size_t k) {
+                    for (uint64_t p = k; p < n; p += (uint64_t)T)
+                        std::sort(t->nbrs + t->begin[p], t->nbrs + t->begin[p] + t->count[p]);
+                });
+            }
+        }
+        S.n_batches = S.max_batch_pairs = 0;
+        S.ms_write_kernel = 0;
+        S.write_launches = 0;
+        for (auto& st : sh) {
+            S.n_batches += st.n_batches;
+            S.max_batch_pairs = std::max(S.max_batch_pairs, st.max_batch);
+            S.ms_write_kernel += st.ms_write;
+            S.write_launches += st.write_launches;
+            S.bytes_d2h += st.d2h;
+        }
+    } catch (...) {
+        for (auto& st : sh) {
+            st.cnt.reset();
+            st.off.reset();
+        }
+        table_free(t);
+        throw;
+    }
+    for (size_t d = 0; d < ndev; ++d) {
+        DeviceGuard dg(ctx->dev[d].device);
+        sh[d].cnt.reset();
+        sh[d].off.reset();
+    }
+    S.kernel_launches = (uint32_t)(g_kernel_launches.load() - launches0);
+    S.ms_table_wall =
+        std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_wall0).count();
+    t->ctx = ctx;
+    ctx->live_objects++;
+    *out = t;
+}
+
+}  // namespace hdb

@@ -1,0 +1,194 @@
+// internal.h -- shared declarations of libhdb (kernels + host orchestration).
+// Not part of the public ABI (include/hdb.h is).
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <atomic>
+#include <map>
+#include <memory>
+#include <mutex>
+#include <string>
+#include <vector>
+
+#include "hdb.h"
+
+namespace hdb {
+
+// ---------------------------------------------------------------- errors
+extern std::atomic<uint64_t> g_kernel_launches;   // kernels launched by this process
+void set_error(const char* fmt, ...);
+struct Error {
+    hdb_status st;
+};
+[[noreturn]] void fail(hdb_status st, const char* fmt, ...);
+#define HDB_CUDA(call)                                                                      \
+    do {                                                                                    \
+        cudaError_t e_ = (call);                                                            \
+        if (e_ != cudaSuccess)                                                              \
+            ::hdb::fail(e_ == cudaErrorMemoryAllocation ? HDB_ENOMEM : HDB_ECUDA,           \
+                        "%s failed: %s (%s:%d)", #call, cudaGetErrorString(e_), __FILE__,   \
+                        __LINE__);                                                          \
+    } while (0)
+#define HDB_LAUNCH_CHECK() HDB_CUDA(cudaGetLastError())
+
+// Warps per search CTA and queries per group (one warp's query tile).
+constexpr int kGroup = 32;
+constexpr int kSearchThreads = 256;
+
+// ---------------------------------------------------------------- grid
+// One device's copy of the grid (Fig. 1 re-laid out).
+struct DevGrid {
+    int device = 0;
+    hdb_dtype dtype = HDB_F64;
+    uint64_t n = 0;
+    double eps = 0, w = 0, inv_w = 0;
+    double e2_d = 0;     // fl(eps*eps) in f64
+    float e2_f = 0;      // fl(eps_f*eps_f) in f32
+    double xmin = 0, ymin = 0, xmax = 0, ymax = 0;
+    uint32_t nx = 1, ny = 1;
+    uint64_t n_cells = 0, n_nonempty = 0, n_groups = 0;
+    void* xy_s = nullptr;          // [n] double2 / float2, cell order
+    uint32_t* ids = nullptr;       // [n] sorted pos -> original id  (A)
+    uint32_t* keys = nullptr;      // [n] cell key per sorted pos
+    uint32_t* start = nullptr;     // [n_cells+1] cell start            (G)
+    uint32_t* gstart = nullptr;    // [n_groups+1] first sorted pos of each query group
+    cudaStream_t stream = nullptr; // stream the buffers were allocated on
+    float ms_build = 0;
+};
+
+// Kernel-side view (passed by value).
+template <typename T>
+struct GridArgs {
+    const void* xy;   // T2*
+    const uint32_t* ids;
+    const uint32_t* keys;
+    const uint32_t* start;
+    const uint32_t* gstart;
+    uint32_t nx, ny;
+    uint32_t n;
+    T e2;
+};
+
+// ---------------------------------------------------------------- kernels
+// grid build (kernels_grid.cu)
+void launch_bbox_init(unsigned long long* bb, unsigned int* bad, cudaStream_t s);
+void launch_bbox(const void* xy, uint64_t n, hdb_dtype dt, unsigned long long* bb, unsigned int* bad,
+                 cudaStream_t s);
+double bbox_decode(unsigned long long v, bool is_max);
+void launch_keys(const void* xy, uint64_t n, hdb_dtype dt, double xmin, double ymin, double inv_w,
+                 uint32_t nx, uint32_t ny, uint32_t* keys, uint32_t* vals, cudaStream_t s);
+size_t radix_sort_temp_bytes(uint64_t n);
+// Stable LSD radix sort of (keys, vals) on the low `bits` bits.  Ping-pongs
+// between (k0,v0) and (k1,v1); returns 0 if the result is in (k0,v0), 1 else.
+int radix_sort_pairs(uint32_t* k0, uint32_t* v0, uint32_t* k1, uint32_t* v1, uint64_t n, int bits,
+                     void* temp, cudaStream_t s);
+void launch_gather_points(const void* xy_in, const uint32_t* ids, uint64_t n, hdb_dtype dt, void* xy_s,
+                          cudaStream_t s);
+void launch_cell_counts(const uint32_t* keys_sorted, uint64_t n, uint32_t* cell_cnt,
+                        unsigned long long* n_nonempty, cudaStream_t s);
+void launch_group_flags(const uint32_t* keys_sorted, const uint32_t* start, uint64_t n, uint32_t* flags,
+                        cudaStream_t s);
+void launch_group_scatter(const uint32_t* flags, const uint32_t* pos, uint64_t n, uint32_t* gstart,
+                          cudaStream_t s);
+
+// scans (kernels_scan.cu): exclusive scan of in[0..n) into out[0..n], out[n] = total
+size_t scan_temp_bytes(uint64_t n);
+void scan_u32_to_u32(const uint32_t* in, uint32_t* out, uint64_t n, void* temp, cudaStream_t s);
+void scan_u32_to_u64(const uint32_t* in, uint64_t* out, uint64_t n, void* temp, cudaStream_t s);
+
+// search (kernels_search.cu)
+// Sampled count (a5): sum of |N_eps| over sorted positions j*stride, j < n_sample;
+// per-sample counts to samp_cnt (may be null).
+void launch_sample_count(const DevGrid& g, uint64_t stride, uint64_t n_sample, uint32_t* samp_cnt,
+                         unsigned long long* sum, cudaStream_t s);
+// Exact count (a6) over query groups [g0, g1): cnt[sorted pos].
+void launch_count(const DevGrid& g, uint64_t g0, uint64_t g1, uint32_t* cnt, unsigned long long* tests,
+                  int variant, cudaStream_t s);
+// Write (a8) over groups [g0, g1): out[off[q] - out_base + k] = k-th neighbour id of q.
+void launch_write(const DevGrid& g, uint64_t g0, uint64_t g1, const uint64_t* off, uint64_t out_base,
+                  uint32_t* out, int variant, cudaStream_t s);
+// cuts: for b in 0..nb, gcut[b] = first group g in [g0,g1] with off[gstart[g]] >= target_b,
+// target_b = off[gstart[g0]] + b * span / nb (gcut[0] = g0, gcut[nb] = g1); pcut[b] = off[gstart[gcut[b]]]
+void launch_batch_cuts(const uint32_t* gstart, const uint64_t* off, uint64_t g0, uint64_t g1, uint32_t nb,
+                       uint64_t* gcut, uint64_t* pcut, cudaStream_t s);
+// map sorted positions -> the group containing them (binary search in gstart)
+void launch_pos_to_group(const uint32_t* gstart, uint64_t n_groups, const uint64_t* pos, uint32_t m,
+                         uint64_t* grp, cudaStream_t s);
+// T assembly by original id: begin[ids[q]] = off[q] + base, count[ids[q]] = cnt[q], q in [q0,q1)
+void launch_scatter_rows(const uint32_t* ids, const uint64_t* off, const uint32_t* cnt, uint64_t q0,
+                         uint64_t q1, uint64_t base, uint64_t* begin, uint32_t* count, cudaStream_t s);
+// per-list ascending sort (segmented, in place), lists by sorted query [q0,q1)
+void launch_sort_lists(const uint64_t* off, const uint32_t* cnt, uint64_t q0, uint64_t q1, uint64_t out_base,
+                       uint32_t* out, cudaStream_t s);
+
+// ---------------------------------------------------------------- pools
+struct PinnedPool {
+    std::mutex m;
+    std::multimap<size_t, void*> free_blocks;
+    size_t bytes_total = 0;
+    uint64_t grows = 0;
+    void* acquire(size_t bytes, size_t* got);
+    void release(void* p, size_t bytes);
+    ~PinnedPool();
+};
+
+struct DevCtx {
+    int device = 0;
+    cudaStream_t main = nullptr;
+    bool own_main = true;
+    std::vector<cudaStream_t> streams;     // write + D2H streams
+    std::vector<cudaEvent_t> ev_pool;
+    // cached per-stream device batch buffers (reused across calls)
+    std::vector<uint32_t*> batch_buf;
+    std::vector<size_t> batch_cap;
+};
+
+}  // namespace hdb
+
+struct hdb_ctx {
+    hdb_opts opts{};
+    std::vector<int> device_list;
+    std::vector<hdb::DevCtx> dev;
+    std::shared_ptr<hdb::PinnedPool> pinned;
+    std::recursive_mutex mu;
+    hdb_stats stats{};
+    std::atomic<int> live_objects{0};
+};
+
+struct hdb_grid {
+    hdb_ctx* ctx = nullptr;
+    std::vector<hdb::DevGrid> dev;   // one per ctx device (same content)
+};
+
+struct hdb_table {
+    uint64_t n = 0, npairs = 0;
+    double eps = 0;
+    hdb_dtype dtype = HDB_F64;
+    bool on_device = false;
+    int device = 0;
+    uint64_t first_query = 0, end_query = 0;
+    uint64_t* begin = nullptr;
+    uint32_t* count = nullptr;
+    uint32_t* nbrs = nullptr;
+    // ownership
+    std::shared_ptr<hdb::PinnedPool> pool;   // non-null: begin/count/nbrs are pinned pool blocks
+    size_t cap_begin = 0, cap_count = 0, cap_nbrs = 0;
+    bool malloced = false;                   // begin/count/nbrs from malloc
+    cudaStream_t dstream = nullptr;          // device-resident: stream for cudaFreeAsync
+    int host_threads = 0;
+    hdb_ctx* ctx = nullptr;
+};
+
+namespace hdb {
+int resolve_threads(int requested);
+// engine.cpp
+void grid_build(hdb_ctx* ctx, const void* xy, uint64_t n, hdb_dtype dt, double eps, hdb_grid** out);
+void grid_free(hdb_grid* g);
+void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hdb_table** out);
+void table_free(hdb_table* t);
+// dbscan.cpp
+uint32_t dbscan_host(const hdb_table* t, uint32_t minpts, int n_threads, int32_t* labels, uint8_t* core);
+void canonicalize(hdb_table* t);
+}  // namespace hdb

@@ -22,3 +22,21 @@ def pytest_collection_modifyitems(config, items):
     for it in items:
         if "slow" in it.keywords:
             it.add_marker(skip)
+
+
+def _ensure_lib():
+    """Build libhdb.so in-tree if missing (nvcc cross-compiles without a GPU)."""
+    import paper_conf_ipps_gowanlockrblp17_b200 as pkg
+    if not os.path.exists(pkg.LIB_PATH):
+        pkg.build()
+
+
+_ensure_lib()
+
+
+def cuda_available():
+    try:
+        import torch
+        return torch.cuda.is_available()
+    except Exception:
+        return False

@@ -1,0 +1,399 @@
+"""GPU parity: the CUDA path (through the C-ABI) against the CPU oracle.
+
+Neighbour tables must be bit-exact after per-row sorting (counts first, then
+lists); DBSCAN core flags, noise and labels must be equal (the library emits
+the canonical labelling, so labels are simply equal).  Inputs are the seeded
+generators of datagen/ at sizes the oracle finishes in seconds (several tiles,
+ragged tails) plus sampled rows at the bench's full sizes.
+"""
+import math
+
+import numpy as np
+import pytest
+
+import datagen
+import oracle
+from paper_conf_ipps_gowanlockrblp17_b200 import hdb
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def torch_cuda():
+    import torch
+    assert torch.cuda.is_available(), "GPU tests need a CUDA device"
+    return torch
+
+
+def _ctx(**opts):
+    return hdb.hdb_ctx_create(**opts)
+
+
+def _canon(begin, count, nbrs):
+    """rows in id order, lists ascending -> (off, flat)"""
+    n = count.size
+    off = np.zeros(n + 1, np.uint64)
+    np.cumsum(count.astype(np.uint64), out=off[1:])
+    rows = np.repeat(np.arange(n, dtype=np.int64), count.astype(np.int64))
+    src = (np.repeat(begin.astype(np.int64), count.astype(np.int64))
+           + (np.arange(rows.size, dtype=np.int64) - np.repeat(off[:-1].astype(np.int64), count.astype(np.int64))))
+    vals = nbrs[src] if rows.size else np.zeros(0, np.uint32)
+    order = np.lexsort((vals, rows))
+    return off, vals[order]
+
+
+def lib_table(xy, eps, device=False, ctx=None, **opts):
+    own = ctx is None
+    if own:
+        ctx = _ctx(**opts)
+    try:
+        g = hdb.hdb_grid_build(ctx, xy, eps)
+        try:
+            t = (hdb.hdb_neighbor_table_device if device else hdb.hdb_neighbor_table)(ctx, g)
+        finally:
+            hdb.hdb_grid_free(g)
+        try:
+            b, c, v = hdb.hdb_table_copy_to_host(t)
+            view = hdb.hdb_table_view_get(t)
+        finally:
+            hdb.hdb_table_free(t)
+        stats = hdb.hdb_stats_get(ctx)
+    finally:
+        if own:
+            hdb.hdb_ctx_destroy(ctx)
+    return b, c, v, view, stats
+
+
+def assert_table_equal(xy, eps, b, c, v, dtype="f64"):
+    off, nbr = oracle.eps_join(xy, eps, dtype=dtype)
+    want_cnt = np.diff(off.astype(np.int64))
+    assert np.array_equal(c.astype(np.int64), want_cnt), \
+        f"count mismatch at rows {np.nonzero(c.astype(np.int64) != want_cnt)[0][:10]}"
+    loff, lnbr = _canon(b, c, v)
+    assert np.array_equal(lnbr, nbr)
+
+
+# ------------------------------------------------------------------ tables
+@pytest.mark.parametrize("device", [False, True])
+@pytest.mark.parametrize("dtype", ["f64", "f32"])
+def test_c1_full_table(torch_cuda, device, dtype):
+    xy = datagen.c1()
+    if dtype == "f32":
+        xy = xy.astype(np.float32)
+    b, c, v, view, st = lib_table(xy, datagen.C1_EPS, device=device)
+    assert view.npairs == c.astype(np.int64).sum() == v.size
+    assert st["npairs"] == view.npairs
+    assert_table_equal(xy, datagen.C1_EPS, b, c, v, dtype)
+
+
+@pytest.mark.parametrize("name,gen,eps_list", [
+    ("tec", lambda: datagen.subsample(datagen.tec_like(), 40_000, seed=1), (0.15, 0.45, 1.40, 3.0)),
+    ("sdss", lambda: datagen.subsample(datagen.sdss_like(), 40_000, seed=2), (0.07, 0.2, 0.6, 2.0)),
+    ("skew", lambda: datagen.dense_skew(30_000, seed=7), (0.5, 4.0, 15.0)),
+])
+def test_workload_subsets(torch_cuda, name, gen, eps_list):
+    xy = gen()
+    for eps in eps_list:
+        b, c, v, view, st = lib_table(xy, eps, device=True)
+        assert_table_equal(xy, eps, b, c, v)
+
+
+def test_input_from_device_tensor(torch_cuda):
+    torch = torch_cuda
+    xy = datagen.subsample(datagen.tec_like(), 20_000, seed=3)
+    b, c, v, _, _ = lib_table(torch.from_numpy(xy).cuda(), 0.45, device=True)
+    assert_table_equal(xy, 0.45, b, c, v)
+
+
+@pytest.mark.parametrize("dtype", ["f64", "f32"])
+def test_near_ties_adversarial(torch_cuda, dtype):
+    for eps in (0.45, 0.1, 1.4, 0.07):
+        xy = datagen.near_ties(4000, eps, seed=int(eps * 100))
+        if dtype == "f32":
+            xy = xy.astype(np.float32)
+        b, c, v, _, _ = lib_table(xy, eps, device=True)
+        assert_table_equal(xy, eps, b, c, v, dtype)
+
+
+def test_lattice_ties(torch_cuda):
+    for k, eps in ((40, 1.0), (40, math.sqrt(2.0)), (33, 0.5), (20, 2.0)):
+        xy = datagen.lattice(k, spacing=1.0 if eps >= 1 else 0.5, origin=(-7.25, 3.5))
+        b, c, v, _, _ = lib_table(xy, eps)
+        assert_table_equal(xy, eps, b, c, v)
+
+
+def test_decimal_steps_on_a_line(torch_cuda):
+    # points k*eps apart: membership decided by the rounded arithmetic
+    x = np.array([k * 0.1 for k in range(3000)])
+    xy = np.stack([x, np.zeros_like(x)], axis=1)
+    for eps in (0.1, 0.2, 0.30000000000000004, 0.3):
+        b, c, v, _, _ = lib_table(xy, eps)
+        assert_table_equal(xy, eps, b, c, v)
+
+
+def test_edge_cases(torch_cuda):
+    # n = 0
+    b, c, v, view, _ = lib_table(np.zeros((0, 2)), 1.0)
+    assert view.n == 0 and view.npairs == 0
+    # n = 1
+    b, c, v, view, _ = lib_table(np.array([[3.0, -2.0]]), 0.5)
+    assert c.tolist() == [1] and v.tolist() == [0]
+    # duplicates, identical points -> P = n^2
+    same = np.tile([[1.5, 2.5]], (700, 1))
+    b, c, v, view, _ = lib_table(same, 0.01)
+    assert view.npairs == 700 * 700 and np.all(c == 700)
+    # all in one cell; negative coordinates; points on the bbox max
+    xy = np.array([[-1.0, -1.0], [-0.9, -1.0], [-1.0, -0.95], [5.0, 5.0], [4.5, 5.0], [5.0, 4.5]])
+    b, c, v, _, _ = lib_table(xy, 0.5)
+    assert_table_equal(xy, 0.5, b, c, v)
+    # ragged: 33 points in a single cell with one isolated far point
+    rng = np.random.default_rng(1)
+    xy = np.concatenate([rng.uniform(0, 0.1, (33, 2)), [[50.0, 50.0]]])
+    b, c, v, _, _ = lib_table(xy, 0.2)
+    assert_table_equal(xy, 0.2, b, c, v)
+
+
+def test_dense_cell_bigger_than_group(torch_cuda):
+    rng = np.random.default_rng(5)
+    xy = np.concatenate([rng.normal(0, 0.05, (5000, 2)), rng.uniform(-5, 5, (3000, 2))])
+    b, c, v, _, _ = lib_table(xy, 0.3, device=True)
+    assert_table_equal(xy, 0.3, b, c, v)
+
+
+def test_errors(torch_cuda):
+    ctx = _ctx()
+    try:
+        for bad_eps in (0.0, -1.0, float("nan"), float("inf")):
+            with pytest.raises(hdb.HdbError) as e:
+                hdb.hdb_grid_build(ctx, datagen.c1(), bad_eps)
+            assert e.value.status == hdb.HDB_EINVAL
+        for bad in (float("nan"), float("inf"), -float("inf")):
+            xy = datagen.c1()
+            xy[17, 1] = bad
+            with pytest.raises(hdb.HdbError) as e:
+                hdb.hdb_grid_build(ctx, xy, 0.5)
+            assert e.value.status == hdb.HDB_EINVAL
+        xy = np.array([[-1e9, 0.0], [1e9, 1.0]])
+        with pytest.raises(hdb.HdbError) as e:
+            hdb.hdb_grid_build(ctx, xy, 1e-3)
+        assert e.value.status == hdb.HDB_ERANGE
+    finally:
+        hdb.hdb_ctx_destroy(ctx)
+
+
+# ------------------------------------------------------------------ grid structure
+def test_grid_structure_fig1(torch_cuda):
+    """Fig. 1: G holds per-cell ranges into A, |A| = |D|, the ids of
+    a cell are contiguous in A; here also: cells in key order, stable (ids
+    ascending inside a cell), keys = floor((x - xmin) / w)."""
+    xy = datagen.subsample(datagen.tec_like(), 50_000, seed=4)
+    eps = 0.45
+    ctx = _ctx()
+    try:
+        g = hdb.hdb_grid_build(ctx, xy, eps)
+        gg = hdb.hdb_grid_copy_to_host(g)
+        hdb.hdb_grid_free(g)
+    finally:
+        hdb.hdb_ctx_destroy(ctx)
+    v = gg["view"]
+    ids, keys, start = gg["ids"], gg["keys"], gg["cell_start"]
+    n = xy.shape[0]
+    assert np.array_equal(np.sort(ids), np.arange(n))                 # |A| = |D|, a permutation
+    assert np.all(np.diff(keys.astype(np.int64)) >= 0)                 # sorted by cell
+    assert start[0] == 0 and start[-1] == n and np.all(np.diff(start.astype(np.int64)) >= 0)
+    w = eps * (1 + 2.0 ** -19)
+    assert v.cell_w == w
+    inv = 1.0 / w
+    cx = np.floor((xy[:, 0] - xy[:, 0].min()) * inv).astype(np.int64)
+    cy = np.floor((xy[:, 1] - xy[:, 1].min()) * inv).astype(np.int64)
+    assert v.nx == cx.max() + 1 and v.ny == cy.max() + 1
+    want_key = cy * v.nx + cx
+    assert np.array_equal(keys.astype(np.int64), want_key[ids])
+    assert np.array_equal(gg["xy_sorted"], xy[ids])
+    # cell h holds exactly the sorted positions [start[h], start[h+1])
+    h = keys.astype(np.int64)
+    pos = np.arange(n)
+    assert np.all(start[h] <= pos) and np.all(pos < start[h + 1])
+    # stable: ids ascending inside each cell
+    same = h[1:] == h[:-1]
+    assert np.all(ids[1:][same] > ids[:-1][same])
+    assert v.n_nonempty == np.unique(h).size
+
+
+# ------------------------------------------------------------------ batching / streams / shards
+def test_batching_fault_injection(torch_cuda):
+    xy = datagen.subsample(datagen.tec_like(), 30_000, seed=5)
+    eps = 0.8
+    off, nbr = oracle.eps_join(xy, eps)
+    P = int(off[-1])
+    ref = None
+    configs = [dict(), dict(batch_pairs=997), dict(batch_pairs=P // 7 + 1, n_streams=1),
+               dict(batch_pairs=50_000, n_streams=5), dict(sample_fraction=1.0), dict(sample_fraction=0.5),
+               dict(batch_pairs=1)]
+    for cfg in configs:
+        b, c, v, view, st = lib_table(xy, eps, **cfg)
+        assert_table_equal(xy, eps, b, c, v)
+        assert st["npairs"] == P
+        if "batch_pairs" in cfg and cfg["batch_pairs"] < P:
+            assert st["n_batches"] > 1
+        lo, lv = _canon(b, c, v)
+        if ref is None:
+            ref = lv
+        assert np.array_equal(lv, ref)
+
+
+def test_host_budget_enomem(torch_cuda):
+    xy = datagen.subsample(datagen.tec_like(), 20_000, seed=6)
+    with pytest.raises(hdb.HdbError) as e:
+        lib_table(xy, 0.8, host_budget_bytes=1000)
+    assert e.value.status == hdb.HDB_ENOMEM
+
+
+def test_estimate_and_plan_stats(torch_cuda):
+    xy = datagen.subsample(datagen.tec_like(), 200_000, seed=8)
+    b, c, v, view, st = lib_table(xy, 0.45, device=True)
+    assert st["sample_size"] == math.ceil(xy.shape[0] / 100)
+    assert st["est_pairs"] == st["sample_pairs"] * 100
+    bb, nb = hdb.hdb_plan_batches(st["est_pairs"], 0.05, 3)
+    assert st["planned_batches"] == nb
+    # the strided sample of the cell-sorted order is a decent estimator
+    assert abs(st["est_pairs"] - view.npairs) / view.npairs < 0.25
+    assert st["candidate_tests"] >= view.npairs
+
+
+def test_virtual_devices_in_one_context(torch_cuda):
+    """Several 'devices' mapped to GPU 0: exercises the multi-device shard
+    driver (sampled cuts, per-shard count/scan, gather of counts, per-shard
+    D2H at global bases, host scatter of T) on one GPU."""
+    xy = datagen.subsample(datagen.dense_skew(2_000_000, seed=5), 60_000, seed=1)
+    eps = 3.0
+    ref = lib_table(xy, eps)
+    for devs in ([0, 0], [0, 0, 0, 0]):
+        b, c, v, view, st = lib_table(xy, eps, devices=devs, batch_pairs=100_000)
+        assert st["n_devices"] == len(devs)
+        assert np.array_equal(c, ref[1])
+        assert np.array_equal(_canon(b, c, v)[1], _canon(*ref[:3])[1])
+    assert_table_equal(xy, eps, *ref[:3])
+
+
+@pytest.mark.parametrize("R", [2, 3, 8])
+def test_process_shards_partition_the_table(torch_cuda, R):
+    """shard_rank/shard_count (torchrun mode): the R partial tables cover
+    disjoint, contiguous ranges of the cell-sorted queries, their pair
+    counts sum to P, and together they are the full table."""
+    xy = datagen.subsample(datagen.sdss_like(), 50_000, seed=3)
+    eps = 0.5
+    full = lib_table(xy, eps, device=True)
+    n = xy.shape[0]
+    count = np.zeros(n, np.int64)
+    rows_seen = np.zeros(n, np.int64)
+    total = 0
+    ranges = []
+    for r in range(R):
+        for device in (True, False):
+            b, c, v, view, st = lib_table(xy, eps, device=device, shard_rank=r, shard_count=R)
+            if device:
+                ranges.append((view.first_query, view.end_query))
+                total += view.npairs
+                mine = c > 0
+                rows_seen += mine
+                count[mine] = c[mine]
+                # each present row equals the full table's row
+                fb, fc, fv = full[:3]
+                for p in np.nonzero(mine)[0][:200]:
+                    a = np.sort(v[b[p]:b[p] + c[p]])
+                    bref = np.sort(fv[fb[p]:fb[p] + fc[p]])
+                    assert np.array_equal(a, bref)
+    assert ranges[0][0] == 0 and ranges[-1][1] == n
+    assert all(ranges[i][1] == ranges[i + 1][0] for i in range(R - 1))
+    assert total == full[3].npairs
+    assert np.all(rows_seen == 1)
+    assert np.array_equal(count, full[1].astype(np.int64))
+
+
+def test_deterministic(torch_cuda):
+    xy = datagen.subsample(datagen.tec_like(), 30_000, seed=9)
+    a = lib_table(xy, 0.45)
+    b = lib_table(xy, 0.45)
+    for x, y in zip(a[:3], b[:3]):
+        assert np.array_equal(x, y)
+
+
+def test_sort_lists_option(torch_cuda):
+    xy = datagen.subsample(datagen.tec_like(), 10_000, seed=2)
+    b, c, v, _, _ = lib_table(xy, 0.6, sort_lists=1)
+    for p in range(0, 10_000, 97):
+        lst = v[b[p]:b[p] + c[p]]
+        assert np.all(np.diff(lst.astype(np.int64)) > 0)
+
+
+# ------------------------------------------------------------------ DBSCAN end to end
+@pytest.mark.parametrize("threads", [1, 8])
+def test_dbscan_end_to_end(torch_cuda, threads):
+    for xy, eps, minpts in ((datagen.c1(), 0.5, 4),
+                            (datagen.subsample(datagen.tec_like(), 30_000, seed=1), 0.45, 4),
+                            (datagen.subsample(datagen.sdss_like(), 30_000, seed=1), 0.3, 8),
+                            (datagen.subsample(datagen.tec_like(), 20_000, seed=2), 0.3, 1)):
+        want = oracle.dbscan(*oracle.eps_join(xy, eps), minpts)
+        ctx = _ctx()
+        try:
+            g = hdb.hdb_grid_build(ctx, xy, eps)
+            t = hdb.hdb_neighbor_table(ctx, g)
+            hdb.hdb_grid_free(g)
+            lab, core, k = hdb.hdb_dbscan(t, minpts, n_threads=threads)
+            hdb.hdb_table_free(t)
+        finally:
+            hdb.hdb_ctx_destroy(ctx)
+        assert k == want[2]
+        assert np.array_equal(core, want[1])
+        assert np.array_equal(lab, want[0])
+
+
+def test_sweep_matches_oracle(torch_cuda):
+    xy = datagen.subsample(datagen.tec_like(), 20_000, seed=11)
+    eps_list = (0.15, 0.3, 0.45, 1.0)
+    mp = (4, 8, 16)
+    ctx = _ctx()
+    try:
+        labels, k = hdb.hdb_sweep(ctx, xy, eps_list, mp)
+    finally:
+        hdb.hdb_ctx_destroy(ctx)
+    for i, eps in enumerate(eps_list):
+        off, nbr = oracle.eps_join(xy, eps)
+        for j, m in enumerate(mp):
+            want = oracle.dbscan(off, nbr, m)
+            assert k[i, j] == want[2]
+            assert np.array_equal(labels[i, j], want[0])
+
+
+# ------------------------------------------------------------------ full-size sampled rows
+def _sampled_rows_check(xy, eps, m_rows=1500, seed=0, **opts):
+    b, c, v, view, st = lib_table(xy, eps, device=True, **opts)
+    n = xy.shape[0]
+    assert view.npairs == c.astype(np.int64).sum()
+    rng = np.random.default_rng(seed)
+    rows = rng.choice(n, size=m_rows, replace=False)
+    # plus the rows with the largest lists (dense-cell stress)
+    rows = np.unique(np.concatenate([rows, np.argsort(c)[-50:]]))
+    roff, rnbr = oracle.eps_join_rows(xy, eps, rows)
+    for i, p in enumerate(rows):
+        got = np.sort(v[b[p]:b[p] + c[p]])
+        assert np.array_equal(got, rnbr[roff[i]:roff[i + 1]]), p
+    # symmetry on the sampled rows
+    for p in rows[:300]:
+        for q in v[b[p]:b[p] + c[p]][:50]:
+            lst = v[b[q]:b[q] + c[q]]
+            assert p in lst
+    return view, st
+
+
+def test_c2_full_size_sampled_rows(torch_cuda):
+    xy = datagen.tec_like()
+    view, st = _sampled_rows_check(xy, 0.45)
+    assert 1.0e9 < view.npairs < 2.0e9
+
+
+def test_c3_full_size_sampled_rows(torch_cuda):
+    xy = datagen.sdss_like()
+    for eps in datagen.C3_EPS:
+        _sampled_rows_check(xy, eps, m_rows=800, seed=int(eps * 100))
