@@ -1,0 +1,305 @@
+#!/usr/bin/env python
+"""bench.py -- HYBRID-DBSCAN hot path on B200: eps-neighbour pairs/s.
+
+One step = one pass of the whole device hot path over the workload: grid build
+(bbox, keys, radix sort, cell offsets, groups), sampled count + plan, exact
+count, scan, neighbour write into a device-resident table.
+``value`` = pairs/s with the points resident in HBM; ``e2e`` = the same metric
+through the C-ABI from pinned HOST points to a HOST table plus the host DBSCAN
+(a1-a11), with the H2D/D2H copies inside the timed region.
+
+Workload (default): C2, the TEC-like set of SW1's size (1,864,620 points,
+P:828-829), eps = 0.45, minpts = 4 (BASELINE.json configs[1]).
+
+Multi-GPU (torchrun): every rank holds the full point set and its grid and
+computes the table for its shard of the cell-sorted queries;
+the only collective is an all_gather of the per-shard pair counts.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+import datagen  # noqa: E402
+
+WORKLOADS = {
+    "C2-eps0.45": dict(gen=datagen.tec_like, eps=0.45, desc="TEC-like n=1,864,620 eps=0.45 minpts=4"),
+    "C2-eps0.15": dict(gen=datagen.tec_like, eps=0.15, desc="TEC-like n=1,864,620 eps=0.15 minpts=4"),
+    "C2-eps1.40": dict(gen=datagen.tec_like, eps=1.40, desc="TEC-like n=1,864,620 eps=1.40 minpts=4"),
+    "C3-eps0.20": dict(gen=datagen.sdss_like, eps=0.20, desc="SDSS-like n=2,000,000 eps=0.20 minpts=4"),
+    "C3L-eps0.20": dict(gen=lambda: datagen.sdss_like(datagen.C3_N_LARGE, seed=4), eps=0.20,
+                        desc="SDSS-like n=5,000,000 eps=0.20 minpts=4"),
+    "C5-eps0.5": dict(gen=datagen.dense_skew, eps=0.5, desc="dense-skew n=50,000,000 eps=0.5 minpts=4"),
+}
+MINPTS = 4
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured"
+    return 6650.0, "fallback"
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+    Q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.rows = []
+        self.proc = None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            parts = [x.strip() for x in line.split(",")]
+            if len(parts) == 6:
+                self.rows.append(parts)
+
+    def __exit__(self, *a):
+        if self.proc is not None:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+            self.t.join(timeout=2)
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"], "samples": 0}
+        sm = [float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in self.rows for i in range(4) if r[2 + i].lower() == "active"})
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(self.rows)}
+
+
+def dist_env():
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return ws, rank, local
+
+
+def cpu_baseline_run(xy, eps, budget_s=12.0, rows=None):
+    """The oracle as it stands (brute-force rows, OpenMP) on a bounded sample."""
+    import oracle
+    n = xy.shape[0]
+    if rows is None:
+        # calibrate on a small sample, then size the sample to ~budget_s
+        probe = np.arange(0, n, max(1, n // 64))[:64]
+        t0 = time.perf_counter()
+        oracle.eps_join_rowhash(xy, eps, probe)
+        dt = max(time.perf_counter() - t0, 1e-3)
+        m = int(min(n, max(64, 64 * budget_s / dt)))
+        rows = np.linspace(0, n - 1, m).astype(np.int64)
+    t0 = time.perf_counter()
+    cnt, _ = oracle.eps_join_rowhash(xy, eps, rows)
+    dt = time.perf_counter() - t0
+    pairs = int(cnt.sum())
+    return dict(value=pairs / dt, unit="pairs/s", cores=oracle.threads(), kind="oracle",
+                sample=f"{rows.size} evenly spaced query rows x all {n} points, brute force "
+                       f"({pairs} pairs, {rows.size * n:.3g} tests, {dt:.2f} s)"), rows
+
+
+def run_reference(args, wl, ws, rank):
+    if rank != 0:
+        return
+    xy = wl["gen"]()
+    K, W = args.steps, args.warmup
+    res, rows = cpu_baseline_run(xy, wl["eps"], budget_s=max(2.0, 60.0 / max(K + W, 1)))
+    for _ in range(W):
+        cpu_baseline_run(xy, wl["eps"], rows=rows)
+    vals = []
+    t_all = time.perf_counter()
+    for _ in range(K):
+        r, _ = cpu_baseline_run(xy, wl["eps"], rows=rows)
+        vals.append(r["value"])
+    t_all = time.perf_counter() - t_all
+    v = float(np.median(vals))
+    line = {"impl": "reference", "metric": "eps_neighbor_pairs_per_sec", "value": v, "unit": "pairs/s",
+            "n_gpus": ws, "steps": K, "warmup": W, "ms_per_step": 1000 * t_all / max(K, 1),
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic", "config": {"workload": args.workload, "desc": wl["desc"]},
+            "cpu_baseline": dict(res, value=v),
+            "e2e": {"value": v, "unit": "pairs/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="hdb", choices=["hdb", "reference"])
+    ap.add_argument("--workload", default="C2-eps0.45", choices=sorted(WORKLOADS))
+    ap.add_argument("--dtype", default="f64", choices=["f64", "f32"])
+    ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--kernel", type=int, default=0, help="search kernel variant (hdb_opts.search_kernel)")
+    args = ap.parse_args()
+    wl = WORKLOADS[args.workload]
+    ws, rank, local = dist_env()
+    if args.impl == "reference":
+        return run_reference(args, wl, ws, rank)
+
+    import torch
+    import torch.distributed as dist
+    from paper_conf_ipps_gowanlockrblp17_b200 import hdb
+
+    assert torch.cuda.is_available(), "bench.py needs a GPU"
+    torch.cuda.set_device(local)
+    if ws > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    dev = torch.device("cuda", local)
+    xy_np = wl["gen"]()
+    if args.dtype == "f32":
+        xy_np = xy_np.astype(np.float32)
+    n = xy_np.shape[0]
+    eps = wl["eps"]
+    xy_dev = torch.from_numpy(xy_np).to(dev)
+    stream = torch.cuda.current_stream(dev)
+    opts = dict(shard_rank=rank, shard_count=ws) if ws > 1 else {}
+    ctx = hdb.hdb_ctx_create(search_kernel=args.kernel, **opts)
+    hdb.hdb_ctx_set_stream(ctx, stream.cuda_stream)
+
+    def step():
+        g = hdb.hdb_grid_build(ctx, xy_dev, eps)
+        t = hdb.hdb_neighbor_table_device(ctx, g)
+        st = hdb.hdb_stats_get(ctx)
+        v = hdb.hdb_table_view_get(t)
+        hdb.hdb_table_free(t)
+        hdb.hdb_grid_free(g)
+        return st, v
+
+    for _ in range(max(args.warmup, 0)):
+        step()
+    torch.cuda.synchronize()
+    if ws > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    write_ms, pairs_local, launches = [], 0, 0
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    l0 = hdb.hdb_kernel_launches()
+    with ClockSampler(local) as clk:
+        ev0.record(stream)
+        for _ in range(args.steps):
+            st, v = step()
+            write_ms.append(st["ms_write_kernel"])
+            pairs_local += v.npairs
+        ev1.record(stream)
+        torch.cuda.synchronize()
+    launches = hdb.hdb_kernel_launches() - l0
+    ms = ev0.elapsed_time(ev1)
+    if ws > 1:
+        t = torch.tensor([ms], device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+        # the "final gather of counts": per-shard pair totals
+        c = torch.tensor([pairs_local], dtype=torch.int64, device=dev)
+        allc = [torch.zeros_like(c) for _ in range(ws)]
+        dist.all_gather(allc, c)
+        pairs_total = int(sum(int(x.item()) for x in allc))
+    else:
+        pairs_total = pairs_local
+    P = pairs_total // max(args.steps, 1)
+    value = pairs_total / (ms / 1000.0)
+
+    # roofline of the dominant kernel (the neighbour write kernel, a8)
+    hbm, peak_kind = load_peaks()
+    esz = 16 if args.dtype == "f64" else 8
+    n_shard = (v.end_query - v.first_query) if ws > 1 else n
+    alg_bytes = 4 * v.npairs + (esz + 4 + 8) * n_shard   # 4 B/pair + sorted xy, id map, offsets per query
+    wms = float(np.mean(write_ms))
+    achieved = alg_bytes / (wms / 1000.0) / 1e9
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(tp):
+        with open(tp) as f:
+            traffic = json.load(f).get(f"{args.workload}-{args.dtype}-k{args.kernel}")
+
+    line = {"metric": "eps_neighbor_pairs_per_sec", "value": value, "unit": "pairs/s", "n_gpus": ws,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms / args.steps,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": args.dtype,
+            "data": "synthetic",
+            "config": {"workload": args.workload, "desc": wl["desc"], "n": n, "eps": eps,
+                       "pairs_per_step": P, "parallelism": f"query-shard{ws}",
+                       "l2": "not flushed: each step writes a %.1f GB table (>> 126 MB L2)" % (4 * P / 1e9),
+                       "step": "grid build + sampled count + count + scan + write (device-resident table)"},
+            "gpu_launches": launches,
+            "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
+                         "frac": achieved / hbm, "traffic": traffic, "peak_kind": peak_kind,
+                         "kernel": "k_search<write>", "kernel_ms": wms, "alg_bytes": alg_bytes},
+            "clocks": clk.summary(),
+            "stats": {k: st[k] for k in ("n_nonempty", "n_groups", "candidate_tests", "ms_grid", "ms_sample",
+                                         "ms_count", "ms_scan", "ms_write_kernel", "kernel_launches")}}
+
+    # ---- e2e: host points -> host table -> host DBSCAN, through the C-ABI
+    if rank == 0 and ws == 1 and args.e2e_steps > 0:
+        hdb.hdb_ctx_set_stream(ctx, None)
+        xy_pin = torch.from_numpy(xy_np).pin_memory()
+        labels = np.empty(n, np.int32)
+        core = np.empty(n, np.uint8)
+
+        def e2e_step():
+            g = hdb.hdb_grid_build(ctx, xy_pin, eps)
+            t = hdb.hdb_neighbor_table(ctx, g)
+            hdb.hdb_grid_free(g)
+            _, _, k = hdb.hdb_dbscan(t, MINPTS, labels=labels, is_core=core)
+            v = hdb.hdb_table_view_get(t)
+            hdb.hdb_table_free(t)
+            return v.npairs, k
+
+        e2e_step()   # warm the pinned pool and device buffers
+        ts, tt = [], []
+        for _ in range(args.e2e_steps):
+            t0 = time.perf_counter()
+            Pe, k = e2e_step()
+            ts.append(time.perf_counter() - t0)
+            tt.append(hdb.hdb_stats_get(ctx)["ms_table_wall"] / 1000.0)
+        te = float(np.median(ts))
+        line["e2e"] = {"value": Pe / te, "unit": "pairs/s", "h2d_bytes_per_step": esz * n,
+                       "d2h_bytes_per_step": 4 * Pe + 12 * n, "s_per_step": te,
+                       "points_clustered_per_sec": n / te, "table_to_host_pairs_per_sec": Pe / float(np.median(tt)),
+                       "n_clusters": k, "includes": "H2D points, grid, count, batched write + D2H on 3 streams, "
+                                                    "host T, host DBSCAN (minpts=4, all host cores)"}
+    else:
+        line["e2e"] = None
+    if rank == 0 and not args.no_cpu_baseline:
+        line["cpu_baseline"], _ = cpu_baseline_run(xy_np.astype(np.float64) if args.dtype == "f64" else xy_np,
+                                                   eps) if args.dtype == "f64" else (None, None)
+    hdb.hdb_ctx_destroy(ctx)
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if ws > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

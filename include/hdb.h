@@ -104,7 +104,8 @@ typedef struct {
 } hdb_table_view;
 
 /* Borrowed view of a grid (Fig. 1, re-laid out: A is the sorted
- * position -> original id map, G is the dense half-open cell-start array).
+ * position -> original id map; G keeps only the NON-EMPTY cells, as ascending
+ * keys h = cy*nx + cx with half-open start offsets into A).
  * All pointers are DEVICE pointers on `device`. */
 typedef struct {
     uint64_t n;
@@ -113,15 +114,15 @@ typedef struct {
     double xmin, ymin, xmax, ymax;   /* bounding box of the data (reading R10)               */
     double cell_w;                   /* w = eps_F * (1 + 2^-19) (reading R9)                  */
     uint32_t nx, ny;                 /* cells per axis; cell key h = cy * nx + cx             */
-    uint64_t n_cells;                /* nx * ny                                               */
+    uint64_t n_cells;                /* nx * ny (cells of the full grid, most may be empty)   */
     uint64_t n_nonempty;             /* non-empty cells (Table II's block count)   */
     uint64_t n_groups;               /* query groups (<= 32 queries of one cell)              */
     int device;
     const void* xy_sorted;           /* [n] double2 / float2 in cell order                    */
     const uint32_t* ids;             /* [n] A: sorted position -> original id                 */
-    const uint32_t* keys_sorted;     /* [n] cell key of each sorted position                  */
-    const uint32_t* cell_start;      /* [n_cells + 1] G: cell h = sorted positions
-                                        [cell_start[h], cell_start[h+1])                      */
+    const uint64_t* cell_keys;       /* [n_nonempty] key h of each non-empty cell, ascending  */
+    const uint32_t* cell_start;      /* [n_nonempty + 1] G: non-empty cell c holds the sorted
+                                        positions [cell_start[c], cell_start[c+1])            */
 } hdb_grid_view;
 
 /* Per-call statistics of the last hdb_neighbor_table* / hdb_grid_build on a context. */
@@ -164,8 +165,9 @@ hdb_status  hdb_grid_build(hdb_ctx* ctx, const void* xy, uint64_t n, hdb_dtype d
 void        hdb_grid_free(hdb_grid* grid);
 hdb_status  hdb_grid_view_get(const hdb_grid* grid, hdb_grid_view* out);   /* first device */
 /* Copy the first device's grid arrays to caller buffers (any may be NULL):
- * ids[n] (A), keys[n], cell_start[n_cells+1] (G), xy_sorted[2n] of the grid's dtype. */
-hdb_status  hdb_grid_copy_to_host(const hdb_grid* grid, uint32_t* ids, uint32_t* keys, uint32_t* cell_start,
+ * ids[n] (A), cell_keys[n_nonempty], cell_start[n_nonempty+1] (G),
+ * xy_sorted[2n] of the grid's dtype. */
+hdb_status  hdb_grid_copy_to_host(const hdb_grid* grid, uint32_t* ids, uint64_t* cell_keys, uint32_t* cell_start,
                                   void* xy_sorted);
 
 /* ---- (2) neighbour table ----------------------------------------------- */

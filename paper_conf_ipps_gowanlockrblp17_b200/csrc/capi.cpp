@@ -219,12 +219,12 @@ hdb_status hdb_grid_view_get(const hdb_grid* g, hdb_grid_view* v) {
     v->device = d.device;
     v->xy_sorted = d.xy_s;
     v->ids = d.ids;
-    v->keys_sorted = d.keys;
-    v->cell_start = d.start;
+    v->cell_keys = d.ckey;
+    v->cell_start = d.cstart;
     return HDB_OK;
 }
 
-hdb_status hdb_grid_copy_to_host(const hdb_grid* g, uint32_t* ids, uint32_t* keys, uint32_t* cell_start,
+hdb_status hdb_grid_copy_to_host(const hdb_grid* g, uint32_t* ids, uint64_t* cell_keys, uint32_t* cell_start,
                                  void* xy_sorted) {
     if (!g) {
         set_error("grid is NULL");
@@ -237,8 +237,9 @@ hdb_status hdb_grid_copy_to_host(const hdb_grid* g, uint32_t* ids, uint32_t* key
     HDB_CUDA(cudaSetDevice(d.device));
     const size_t esz = d.dtype == HDB_F64 ? 16 : 8;
     if (ids && d.n) HDB_CUDA(cudaMemcpy(ids, d.ids, 4 * d.n, cudaMemcpyDeviceToHost));
-    if (keys && d.n) HDB_CUDA(cudaMemcpy(keys, d.keys, 4 * d.n, cudaMemcpyDeviceToHost));
-    if (cell_start) HDB_CUDA(cudaMemcpy(cell_start, d.start, 4 * (d.n_cells + 1), cudaMemcpyDeviceToHost));
+    if (cell_keys && d.n_nonempty)
+        HDB_CUDA(cudaMemcpy(cell_keys, d.ckey, 8 * d.n_nonempty, cudaMemcpyDeviceToHost));
+    if (cell_start) HDB_CUDA(cudaMemcpy(cell_start, d.cstart, 4 * (d.n_nonempty + 1), cudaMemcpyDeviceToHost));
     if (xy_sorted && d.n) HDB_CUDA(cudaMemcpy(xy_sorted, d.xy_s, esz * d.n, cudaMemcpyDeviceToHost));
     cudaSetDevice(prev);
     HDB_GUARD_END

@@ -192,6 +192,42 @@ PtrInfo classify(const void* p) {
     return r;
 }
 
+// f64 mode: bound on |t_f32 - (d2_f64 - e2_f64)| for the search kernel's f32
+// filter.  Filter coordinates are X = fl32(fl64(x - o))
+// with o the bbox centre; every candidate lies in the 3x3 stencil, so
+// |x_p - x_q| < Dmax = 2w.  With u = 2^-24:
+//   E     = R (u + 2^-52)                    (|X - (x - o)|, R = max |fl64(x - o)|)
+//   delta = 2E + (Dmax + 2E) u               (|fl32(X_p - X_q) - (x_p - x_q)|)
+//   |t - S| <= 2 delta (2 Dmax + delta)      (the two squares)
+//            + u (e2 + (Dmax^2 + e2) + (2 Dmax^2 + e2)) (1 + 2^-20)   (e2 rounding, 2 fma roundings)
+//            + 2^-49 Dmax^2                  (the f64 predicate's own rounding)
+// and the kernel uses band = 2x that bound (rounded up): |t| > band => sign(t)
+// is the exact f64 decision.  The filter is disabled (exact f64 kernel) when
+// float overflow is possible or the band would cover a large part of eps^2.
+void set_filter_bound(DevGrid& g) {
+    g.filter = false;
+    g.band = 0;
+    if (g.dtype != HDB_F64) return;
+    g.ox = 0.5 * g.xmin + 0.5 * g.xmax;
+    g.oy = 0.5 * g.ymin + 0.5 * g.ymax;
+    const double R = std::max(std::max(std::fabs(g.xmax - g.ox), std::fabs(g.xmin - g.ox)),
+                              std::max(std::fabs(g.ymax - g.oy), std::fabs(g.ymin - g.oy)));
+    const double u = 0x1p-24;
+    const double Dmax = 2.0 * g.w * (1.0 + 0x1p-18);   // cell rounding: <= 2^-21 cell widths
+    const double E = R * (u + 0x1p-52);
+    const double delta = 2 * E + (Dmax + 2 * E) * u;
+    const double e2 = g.e2_d;
+    const double bound = 2 * delta * (2 * Dmax + delta) + u * (3 * e2 + 3 * Dmax * Dmax) * (1 + 0x1p-20) +
+                         0x1p-49 * Dmax * Dmax;
+    const double band = 2.0 * bound;
+    g.e2_f = (float)e2;
+    if (!(R < 1e15) || !(Dmax < 1e15) || !(e2 > 1e-30) || !(band < 0.25 * e2)) return;
+    float bf = (float)band;
+    if ((double)bf < band) bf = std::nextafter(bf, INFINITY);
+    g.band = bf;
+    g.filter = true;
+}
+
 void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t n, hdb_dtype dt, double eps,
                DevGrid& g) {
     DeviceGuard dg(dc.device);
@@ -254,23 +290,19 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
         fail(HDB_ERANGE, "extent/eps too large (%g x %g cells > 2^30)", ex, ey);
     g.nx = (uint32_t)std::floor(ex) + 1;
     g.ny = (uint32_t)std::floor(ey) + 1;
-    g.n_cells = (uint64_t)g.nx * g.ny;
-    const uint64_t cell_cap = std::min<uint64_t>(kMaxCellsAbs, 64 * n + (1ull << 24));
-    if (g.n_cells > cell_cap)
-        fail(HDB_ERANGE, "grid of %u x %u = %llu cells exceeds the dense-grid limit %llu", g.nx, g.ny,
-             (unsigned long long)g.n_cells, (unsigned long long)cell_cap);
-    const uint64_t C = g.n_cells;
+    g.n_cells = (uint64_t)g.nx * g.ny;   // < 2^61: only the non-empty ones are stored
+    set_filter_bound(g);
 
     // ---- a2: keys
-    DBuf k0(4 * n, s), v0(4 * n, s), k1(4 * n, s), v1(4 * n, s);
-    launch_keys(xin, n, dt, g.xmin, g.ymin, g.inv_w, g.nx, g.ny, k0.as<uint32_t>(), v0.as<uint32_t>(), s);
+    DBuf k0(8 * n, s), v0(4 * n, s), k1(8 * n, s), v1(4 * n, s);
+    launch_keys(xin, n, dt, g.xmin, g.ymin, g.inv_w, g.nx, g.ny, k0.as<uint64_t>(), v0.as<uint32_t>(), s);
     HDB_LAUNCH_CHECK();
-    // ---- a3: stable radix sort by key
+    // ---- a3: stable radix sort by key (only the bits the key range needs)
     int bits = 1;
-    while (bits < 32 && (1ull << bits) < C) ++bits;
-    size_t tb = std::max(radix_sort_temp_bytes(n), scan_temp_bytes(std::max<uint64_t>(n, C) + 1));
+    while (bits < 64 && (1ull << bits) < g.n_cells) ++bits;
+    size_t tb = std::max(radix_sort_temp_bytes(n), scan_temp_bytes(n + 1));
     DBuf temp(tb, s);
-    int which = radix_sort_pairs(k0.as<uint32_t>(), v0.as<uint32_t>(), k1.as<uint32_t>(), v1.as<uint32_t>(), n,
+    int which = radix_sort_pairs(k0.as<uint64_t>(), v0.as<uint32_t>(), k1.as<uint64_t>(), v1.as<uint32_t>(), n,
                                  bits, temp.p, s);
     HDB_LAUNCH_CHECK();
     DBuf keys = which ? std::move(k1) : std::move(k0);
@@ -280,51 +312,71 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
     v0.reset();
     v1.reset();
     DBuf xy_s(n * esz, s);
-    launch_gather_points(xin, ids.as<uint32_t>(), n, dt, xy_s.p, s);
+    DBuf xf;
+    if (dt == HDB_F64) xf = DBuf(8 * n, s);
+    launch_gather_points(xin, ids.as<uint32_t>(), n, dt, xy_s.p, xf.as<float2>(), g.ox, g.oy, s);
     HDB_LAUNCH_CHECK();
     xin_owned.reset();
-    // ---- a4: per-cell counts -> exclusive scan -> G
-    DBuf cnt(4 * C, s);
-    HDB_CUDA(cudaMemsetAsync(cnt.p, 0, 4 * C, s));
-    launch_cell_counts(keys.as<uint32_t>(), n, cnt.as<uint32_t>(), bb + 4, s);
-    DBuf start(4 * (C + 1), s);
-    scan_u32_to_u32(cnt.as<uint32_t>(), start.as<uint32_t>(), C, temp.p, s);
-    cnt.reset();
-    // ---- query groups
+    // ---- a4: run boundaries -> scan -> (key, start) of the non-empty cells
     DBuf flags(4 * n, s), pos(4 * (n + 1), s);
-    launch_group_flags(keys.as<uint32_t>(), start.as<uint32_t>(), n, flags.as<uint32_t>(), s);
+    launch_cell_flags(keys.as<uint64_t>(), n, flags.as<uint32_t>(), s);
     scan_u32_to_u32(flags.as<uint32_t>(), pos.as<uint32_t>(), n, temp.p, s);
     HDB_LAUNCH_CHECK();
-    uint32_t hng = 0;
-    HDB_CUDA(cudaMemcpyAsync(&hng, pos.as<uint32_t>() + n, 4, cudaMemcpyDeviceToHost, s));
-    HDB_CUDA(cudaMemcpyAsync(hb, bb + 4, 8, cudaMemcpyDeviceToHost, s));
+    uint32_t hne = 0;
+    HDB_CUDA(cudaMemcpyAsync(&hne, pos.as<uint32_t>() + n, 4, cudaMemcpyDeviceToHost, s));
     HDB_CUDA(cudaStreamSynchronize(s));
-    g.n_groups = hng;
-    g.n_nonempty = hb[0];
-    DBuf gstart(4 * (g.n_groups + 1), s);
-    launch_group_scatter(flags.as<uint32_t>(), pos.as<uint32_t>(), n, gstart.as<uint32_t>(), s);
+    g.n_nonempty = hne;
+    const uint64_t nne = hne;
+    DBuf ckey(8 * nne, s), cstart(4 * (nne + 1), s);
+    launch_cell_scatter(keys.as<uint64_t>(), flags.as<uint32_t>(), pos.as<uint32_t>(), n, ckey.as<uint64_t>(),
+                        cstart.as<uint32_t>(), s);
     HDB_LAUNCH_CHECK();
     flags.reset();
     pos.reset();
+    keys.reset();
+    // ---- stencil row spans per non-empty cell + query groups
+    DBuf cspan(24 * nne, s), gcount(4 * (nne + 1), s), gofs(4 * (nne + 1), s);
+    launch_cell_spans(ckey.as<uint64_t>(), cstart.as<uint32_t>(), nne, g.nx, g.ny, cspan.as<uint2>(),
+                      gcount.as<uint32_t>(), s);
+    scan_u32_to_u32(gcount.as<uint32_t>(), gofs.as<uint32_t>(), nne, temp.p, s);
+    HDB_LAUNCH_CHECK();
+    uint32_t hng = 0;
+    HDB_CUDA(cudaMemcpyAsync(&hng, gofs.as<uint32_t>() + nne, 4, cudaMemcpyDeviceToHost, s));
+    HDB_CUDA(cudaStreamSynchronize(s));
+    g.n_groups = hng;
+    DBuf gstart(4 * (g.n_groups + 1), s), gcell(4 * (g.n_groups + 1), s);
+    launch_group_build(cstart.as<uint32_t>(), gofs.as<uint32_t>(), nne, n, gstart.as<uint32_t>(),
+                       gcell.as<uint32_t>(), s);
+    HDB_LAUNCH_CHECK();
+    gcount.reset();
+    gofs.reset();
     temp.reset();
     misc.reset();
     HDB_CUDA(cudaEventRecord(ev1.e, s));
     HDB_CUDA(cudaEventSynchronize(ev1.e));
     g.ms_build = elapsed(ev0, ev1);
     g.xy_s = xy_s.release();
+    g.xf = dt == HDB_F64 ? (float2*)xf.release() : (float2*)g.xy_s;
     g.ids = (uint32_t*)ids.release();
-    g.keys = (uint32_t*)keys.release();
-    g.start = (uint32_t*)start.release();
+    g.ckey = (uint64_t*)ckey.release();
+    g.cstart = (uint32_t*)cstart.release();
+    g.cspan = (uint2*)cspan.release();
     g.gstart = (uint32_t*)gstart.release();
+    g.gcell = (uint32_t*)gcell.release();
 }
 
 void free_dev_grid(DevGrid& g) {
     if (!g.stream) return;
     DeviceGuard dg(g.device);
-    for (void* p : {(void*)g.xy_s, (void*)g.ids, (void*)g.keys, (void*)g.start, (void*)g.gstart})
+    void* xf = (g.dtype == HDB_F64) ? (void*)g.xf : nullptr;
+    for (void* p : {(void*)g.xy_s, xf, (void*)g.ids, (void*)g.ckey, (void*)g.cstart, (void*)g.cspan,
+                    (void*)g.gstart, (void*)g.gcell})
         if (p) cudaFreeAsync(p, g.stream);
     g.xy_s = nullptr;
-    g.ids = g.keys = g.start = g.gstart = nullptr;
+    g.xf = nullptr;
+    g.ids = g.cstart = g.gstart = g.gcell = nullptr;
+    g.ckey = nullptr;
+    g.cspan = nullptr;
     cudaStreamSynchronize(g.stream);
 }
 

@@ -38,37 +38,33 @@ constexpr int kGroup = 32;
 constexpr int kSearchThreads = 256;
 
 // ---------------------------------------------------------------- grid
-// One device's copy of the grid (Fig. 1 re-laid out).
+// One device's copy of the grid (Fig. 1 re-laid out):
+// points sorted by cell key h = cy*nx + cx; only NON-EMPTY cells are stored
+// (key, start), so sparse extents cost nothing; every non-empty cell carries
+// its three stencil row spans (contiguous ranges of sorted positions).
 struct DevGrid {
     int device = 0;
     hdb_dtype dtype = HDB_F64;
     uint64_t n = 0;
     double eps = 0, w = 0, inv_w = 0;
     double e2_d = 0;     // fl(eps*eps) in f64
-    float e2_f = 0;      // fl(eps_f*eps_f) in f32
+    float e2_f = 0;      // fl(eps_f*eps_f) in f32 (f32 mode) / fl32(e2_d) (f64 filter)
+    float band = 0;      // f64 mode: |t| <= band => decide in exact f64
+    bool filter = false; // f64 mode with a useful f32 filter
     double xmin = 0, ymin = 0, xmax = 0, ymax = 0;
+    double ox = 0, oy = 0;  // f64 mode: origin of the f32 filter coordinates
     uint32_t nx = 1, ny = 1;
     uint64_t n_cells = 0, n_nonempty = 0, n_groups = 0;
-    void* xy_s = nullptr;          // [n] double2 / float2, cell order
+    void* xy_s = nullptr;          // [n] double2 / float2, cell order (exact coordinates)
+    float2* xf = nullptr;          // [n] f32 filter coordinates (f64 mode; == xy_s in f32 mode)
     uint32_t* ids = nullptr;       // [n] sorted pos -> original id  (A)
-    uint32_t* keys = nullptr;      // [n] cell key per sorted pos
-    uint32_t* start = nullptr;     // [n_cells+1] cell start            (G)
+    uint64_t* ckey = nullptr;      // [n_nonempty] cell key of each non-empty cell (ascending)
+    uint32_t* cstart = nullptr;    // [n_nonempty+1] first sorted pos of each non-empty cell (G)
+    uint2* cspan = nullptr;        // [3*n_nonempty] stencil row spans [lo,hi) per non-empty cell
     uint32_t* gstart = nullptr;    // [n_groups+1] first sorted pos of each query group
+    uint32_t* gcell = nullptr;     // [n_groups] non-empty cell index of each query group
     cudaStream_t stream = nullptr; // stream the buffers were allocated on
     float ms_build = 0;
-};
-
-// Kernel-side view (passed by value).
-template <typename T>
-struct GridArgs {
-    const void* xy;   // T2*
-    const uint32_t* ids;
-    const uint32_t* keys;
-    const uint32_t* start;
-    const uint32_t* gstart;
-    uint32_t nx, ny;
-    uint32_t n;
-    T e2;
 };
 
 // ---------------------------------------------------------------- kernels
@@ -78,20 +74,22 @@ void launch_bbox(const void* xy, uint64_t n, hdb_dtype dt, unsigned long long* b
                  cudaStream_t s);
 double bbox_decode(unsigned long long v, bool is_max);
 void launch_keys(const void* xy, uint64_t n, hdb_dtype dt, double xmin, double ymin, double inv_w,
-                 uint32_t nx, uint32_t ny, uint32_t* keys, uint32_t* vals, cudaStream_t s);
+                 uint32_t nx, uint32_t ny, uint64_t* keys, uint32_t* vals, cudaStream_t s);
 size_t radix_sort_temp_bytes(uint64_t n);
 // Stable LSD radix sort of (keys, vals) on the low `bits` bits.  Ping-pongs
 // between (k0,v0) and (k1,v1); returns 0 if the result is in (k0,v0), 1 else.
-int radix_sort_pairs(uint32_t* k0, uint32_t* v0, uint32_t* k1, uint32_t* v1, uint64_t n, int bits,
+int radix_sort_pairs(uint64_t* k0, uint32_t* v0, uint64_t* k1, uint32_t* v1, uint64_t n, int bits,
                      void* temp, cudaStream_t s);
+// gather sorted points; f64 mode also writes the f32 filter coordinates (x-ox, y-oy)
 void launch_gather_points(const void* xy_in, const uint32_t* ids, uint64_t n, hdb_dtype dt, void* xy_s,
-                          cudaStream_t s);
-void launch_cell_counts(const uint32_t* keys_sorted, uint64_t n, uint32_t* cell_cnt,
-                        unsigned long long* n_nonempty, cudaStream_t s);
-void launch_group_flags(const uint32_t* keys_sorted, const uint32_t* start, uint64_t n, uint32_t* flags,
-                        cudaStream_t s);
-void launch_group_scatter(const uint32_t* flags, const uint32_t* pos, uint64_t n, uint32_t* gstart,
-                          cudaStream_t s);
+                          float2* xf, double ox, double oy, cudaStream_t s);
+void launch_cell_flags(const uint64_t* keys_sorted, uint64_t n, uint32_t* flags, cudaStream_t s);
+void launch_cell_scatter(const uint64_t* keys_sorted, const uint32_t* flags, const uint32_t* pos, uint64_t n,
+                         uint64_t* ckey, uint32_t* cstart, cudaStream_t s);
+void launch_cell_spans(const uint64_t* ckey, const uint32_t* cstart, uint64_t nne, uint32_t nx, uint32_t ny,
+                       uint2* cspan, uint32_t* gcount, cudaStream_t s);
+void launch_group_build(const uint32_t* cstart, const uint32_t* gofs, uint64_t nne, uint64_t n, uint32_t* gstart,
+                        uint32_t* gcell, cudaStream_t s);
 
 // scans (kernels_scan.cu): exclusive scan of in[0..n) into out[0..n], out[n] = total
 size_t scan_temp_bytes(uint64_t n);
@@ -99,8 +97,7 @@ void scan_u32_to_u32(const uint32_t* in, uint32_t* out, uint64_t n, void* temp, 
 void scan_u32_to_u64(const uint32_t* in, uint64_t* out, uint64_t n, void* temp, cudaStream_t s);
 
 // search (kernels_search.cu)
-// Sampled count (a5): sum of |N_eps| over sorted positions j*stride, j < n_sample;
-// per-sample counts to samp_cnt (may be null).
+// Sampled count (a5): |N_eps| of sorted positions j*stride, j < n_sample -> samp_cnt, sum.
 void launch_sample_count(const DevGrid& g, uint64_t stride, uint64_t n_sample, uint32_t* samp_cnt,
                          unsigned long long* sum, cudaStream_t s);
 // Exact count (a6) over query groups [g0, g1): cnt[sorted pos].
@@ -113,15 +110,12 @@ void launch_write(const DevGrid& g, uint64_t g0, uint64_t g1, const uint64_t* of
 // target_b = off[gstart[g0]] + b * span / nb (gcut[0] = g0, gcut[nb] = g1); pcut[b] = off[gstart[gcut[b]]]
 void launch_batch_cuts(const uint32_t* gstart, const uint64_t* off, uint64_t g0, uint64_t g1, uint32_t nb,
                        uint64_t* gcut, uint64_t* pcut, cudaStream_t s);
-// map sorted positions -> the group containing them (binary search in gstart)
+// map sorted positions -> the first group starting at or after them (binary search in gstart)
 void launch_pos_to_group(const uint32_t* gstart, uint64_t n_groups, const uint64_t* pos, uint32_t m,
                          uint64_t* grp, cudaStream_t s);
-// T assembly by original id: begin[ids[q]] = off[q] + base, count[ids[q]] = cnt[q], q in [q0,q1)
+// T assembly by original id: begin[ids[q]] = off[q] - off[q0] + base, count[ids[q]] = cnt[q], q in [q0,q1)
 void launch_scatter_rows(const uint32_t* ids, const uint64_t* off, const uint32_t* cnt, uint64_t q0,
                          uint64_t q1, uint64_t base, uint64_t* begin, uint32_t* count, cudaStream_t s);
-// per-list ascending sort (segmented, in place), lists by sorted query [q0,q1)
-void launch_sort_lists(const uint64_t* off, const uint32_t* cnt, uint64_t q0, uint64_t q1, uint64_t out_base,
-                       uint32_t* out, cudaStream_t s);
 
 // ---------------------------------------------------------------- pools
 struct PinnedPool {

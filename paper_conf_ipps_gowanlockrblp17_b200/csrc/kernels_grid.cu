@@ -10,8 +10,13 @@
 //   a3  sort      -- stable LSD radix sort of (h, id) -> A (sorted pos -> id) and
 //                    the points permuted into cell order (the paper's locality
 //                    pre-sort, is subsumed)
-//   a4  offsets   -- per-cell counts from run boundaries of the sorted keys, then a
-//                    warp-shuffle exclusive scan -> dense half-open G (reading R11)
+//   a4  offsets   -- run boundaries of the sorted keys + a warp-shuffle exclusive
+//                    scan -> G restricted to the NON-EMPTY cells: (key, start) pairs,
+//                    half-open (reading R11); sparse extents cost nothing
+//   +   spans     -- for every non-empty cell, its three stencil row spans: with
+//                    row-major keys the cells (cx-1..cx+1, y') are consecutive in
+//                    key order, so each stencil row is one contiguous range of
+//                    sorted positions (found by binary search over the keys)
 //   +   groups    -- query groups: <= 32 consecutive sorted queries of one cell,
 //                    the unit of work of the search kernels.
 #include <cuda_runtime.h>
@@ -94,15 +99,15 @@ __global__ void __launch_bounds__(256) k_bbox(const typename V2<T>::type* __rest
 template <typename T>
 __global__ void __launch_bounds__(256) k_keys(const typename V2<T>::type* __restrict__ xy, uint64_t n,
                                               double xmin, double ymin, double inv_w, uint32_t nx,
-                                              uint32_t ny, uint32_t* __restrict__ keys,
+                                              uint32_t ny, uint64_t* __restrict__ keys,
                                               uint32_t* __restrict__ vals) {
     for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n;
          i += (uint64_t)gridDim.x * blockDim.x) {
         auto p = xy[i];
         double tx = floor(__dmul_rn(__dsub_rn((double)p.x, xmin), inv_w));
         double ty = floor(__dmul_rn(__dsub_rn((double)p.y, ymin), inv_w));
-        uint32_t cx = (uint32_t)fmin(fmax(tx, 0.0), (double)(nx - 1));
-        uint32_t cy = (uint32_t)fmin(fmax(ty, 0.0), (double)(ny - 1));
+        uint64_t cx = (uint64_t)fmin(fmax(tx, 0.0), (double)(nx - 1));
+        uint64_t cy = (uint64_t)fmin(fmax(ty, 0.0), (double)(ny - 1));
         keys[i] = cy * nx + cx;
         vals[i] = (uint32_t)i;
     }
@@ -116,7 +121,7 @@ constexpr int RS_TILE = RS_THREADS * RS_ITEMS;       // 4096 keys per CTA
 constexpr int RS_BITS = 8;
 constexpr int RS_BINS = 1 << RS_BITS;
 
-__global__ void __launch_bounds__(RS_THREADS) k_radix_hist(const uint32_t* __restrict__ keys, uint64_t n,
+__global__ void __launch_bounds__(RS_THREADS) k_radix_hist(const uint64_t* __restrict__ keys, uint64_t n,
                                                            int shift, uint32_t* __restrict__ hist,
                                                            uint32_t nblocks) {
     __shared__ uint32_t h[RS_BINS];
@@ -129,7 +134,7 @@ __global__ void __launch_bounds__(RS_THREADS) k_radix_hist(const uint32_t* __res
     for (int r = 0; r < RS_ITEMS; ++r) {
         uint64_t idx = base + (uint64_t)r * RS_THREADS + tid;
         bool valid = idx < n;
-        uint32_t d = valid ? ((keys[idx] >> shift) & (RS_BINS - 1)) : (0x100u + lane);
+        uint32_t d = valid ? (uint32_t)((keys[idx] >> shift) & (RS_BINS - 1)) : (0x100u + lane);
         unsigned peers = __match_any_sync(FULL, d);
         if (valid && lane == __ffs(peers) - 1) atomicAdd(&h[d], __popc(peers));
     }
@@ -141,9 +146,9 @@ __global__ void __launch_bounds__(RS_THREADS) k_radix_hist(const uint32_t* __res
 // 16 rounds of 32 consecutive keys; the rank of a key is the number of earlier
 // keys of the same digit in (earlier warps of the tile, earlier rounds of this
 // warp, lower lanes of this round) plus the digit's global base for the tile.
-__global__ void __launch_bounds__(RS_THREADS) k_radix_scatter(const uint32_t* __restrict__ kin,
+__global__ void __launch_bounds__(RS_THREADS) k_radix_scatter(const uint64_t* __restrict__ kin,
                                                               const uint32_t* __restrict__ vin,
-                                                              uint32_t* __restrict__ kout,
+                                                              uint64_t* __restrict__ kout,
                                                               uint32_t* __restrict__ vout, uint64_t n,
                                                               int shift, const uint32_t* __restrict__ hscan,
                                                               uint32_t nblocks) {
@@ -156,14 +161,15 @@ __global__ void __launch_bounds__(RS_THREADS) k_radix_scatter(const uint32_t* __
     __syncthreads();
     const uint64_t base = (uint64_t)blockIdx.x * RS_TILE + (uint64_t)w * (RS_ITEMS * 32);
     const unsigned lt = (1u << lane) - 1u;
-    uint32_t key[RS_ITEMS], val[RS_ITEMS], rank[RS_ITEMS];
+    uint64_t key[RS_ITEMS];
+    uint32_t val[RS_ITEMS], rank[RS_ITEMS];
 #pragma unroll
     for (int r = 0; r < RS_ITEMS; ++r) {
         uint64_t idx = base + (uint64_t)r * 32 + lane;
         bool valid = idx < n;
-        key[r] = valid ? kin[idx] : 0u;
+        key[r] = valid ? kin[idx] : 0ull;
         val[r] = valid ? vin[idx] : 0u;
-        uint32_t d = valid ? ((key[r] >> shift) & (RS_BINS - 1)) : (0x100u + lane);
+        uint32_t d = valid ? (uint32_t)((key[r] >> shift) & (RS_BINS - 1)) : (0x100u + lane);
         unsigned peers = __match_any_sync(FULL, d);
         uint32_t before = valid ? wcnt[w][d] : 0u;
         rank[r] = before + __popc(peers & lt);
@@ -186,7 +192,7 @@ __global__ void __launch_bounds__(RS_THREADS) k_radix_scatter(const uint32_t* __
     for (int r = 0; r < RS_ITEMS; ++r) {
         uint64_t idx = base + (uint64_t)r * 32 + lane;
         if (idx < n) {
-            uint32_t d = (key[r] >> shift) & (RS_BINS - 1);
+            uint32_t d = (uint32_t)((key[r] >> shift) & (RS_BINS - 1));
             uint32_t pos = gbase[d] + wcnt[w][d] + rank[r];
             kout[pos] = key[r];
             vout[pos] = val[r];
@@ -197,50 +203,103 @@ __global__ void __launch_bounds__(RS_THREADS) k_radix_scatter(const uint32_t* __
 template <typename T>
 __global__ void __launch_bounds__(256) k_gather(const typename V2<T>::type* __restrict__ in,
                                                 const uint32_t* __restrict__ ids, uint64_t n,
-                                                typename V2<T>::type* __restrict__ out) {
-    for (uint64_t s = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; s < n;
-         s += (uint64_t)gridDim.x * blockDim.x)
-        out[s] = in[ids[s]];
-}
-
-// a4 histogram from run boundaries of the sorted keys: one atomic per
-// (warp, run) -- dense cells cost one atomic per 32 points.
-__global__ void __launch_bounds__(256) k_cell_counts(const uint32_t* __restrict__ keys, uint64_t n,
-                                                     uint32_t* __restrict__ cnt,
-                                                     unsigned long long* __restrict__ nonempty) {
-    const int lane = threadIdx.x & 31;
-    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
-    // uniform trip count per warp so that __match_any_sync sees all lanes
-    for (uint64_t base = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) - lane; base < n;
-         base += stride) {
-        uint64_t s = base + lane;
-        bool valid = s < n;
-        uint32_t k = valid ? keys[s] : 0xffffffffu;
-        unsigned peers = __match_any_sync(FULL, k);
-        if (valid && lane == __ffs(peers) - 1) atomicAdd(&cnt[k], (uint32_t)__popc(peers));
-        bool first = valid && (s == 0 || keys[s - 1] != k);
-        unsigned fm = __ballot_sync(FULL, first);
-        if (lane == 0 && fm) atomicAdd(nonempty, (unsigned long long)__popc(fm));
-    }
-}
-
-__global__ void __launch_bounds__(256) k_group_flags(const uint32_t* __restrict__ keys,
-                                                     const uint32_t* __restrict__ start, uint64_t n,
-                                                     uint32_t* __restrict__ flags) {
+                                                typename V2<T>::type* __restrict__ out, float2* __restrict__ xf,
+                                                double ox, double oy) {
     for (uint64_t s = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; s < n;
          s += (uint64_t)gridDim.x * blockDim.x) {
-        uint32_t c0 = start[keys[s]];
-        flags[s] = ((uint32_t)s - c0) % (uint32_t)kGroup == 0 ? 1u : 0u;
+        auto p = in[ids[s]];
+        out[s] = p;
+        if (xf) xf[s] = make_float2((float)__dsub_rn((double)p.x, ox), (float)__dsub_rn((double)p.y, oy));
     }
 }
 
-__global__ void __launch_bounds__(256) k_group_scatter(const uint32_t* __restrict__ flags,
-                                                       const uint32_t* __restrict__ pos, uint64_t n,
-                                                       uint32_t* __restrict__ gstart) {
+// a4: run boundaries of the sorted keys
+__global__ void __launch_bounds__(256) k_cell_flags(const uint64_t* __restrict__ keys, uint64_t n,
+                                                    uint32_t* __restrict__ flags) {
     for (uint64_t s = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; s < n;
          s += (uint64_t)gridDim.x * blockDim.x)
-        if (flags[s]) gstart[pos[s]] = (uint32_t)s;
-    if (blockIdx.x == 0 && threadIdx.x == 0) gstart[pos[n]] = (uint32_t)n;
+        flags[s] = (s == 0 || keys[s] != keys[s - 1]) ? 1u : 0u;
+}
+
+__global__ void __launch_bounds__(256) k_cell_scatter(const uint64_t* __restrict__ keys,
+                                                      const uint32_t* __restrict__ flags,
+                                                      const uint32_t* __restrict__ pos, uint64_t n,
+                                                      uint64_t* __restrict__ ckey, uint32_t* __restrict__ cstart) {
+    for (uint64_t s = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; s < n;
+         s += (uint64_t)gridDim.x * blockDim.x)
+        if (flags[s]) {
+            ckey[pos[s]] = keys[s];
+            cstart[pos[s]] = (uint32_t)s;
+        }
+    if (blockIdx.x == 0 && threadIdx.x == 0) cstart[pos[n]] = (uint32_t)n;
+}
+
+// first index i in [lo, hi) with ckey[i] >= k (hi if none)
+__device__ __forceinline__ uint64_t lower_bound_u64(const uint64_t* __restrict__ a, uint64_t lo, uint64_t hi,
+                                                    uint64_t k) {
+    while (lo < hi) {
+        uint64_t mid = (lo + hi) >> 1;
+        if (__ldg(&a[mid]) < k)
+            lo = mid + 1;
+        else
+            hi = mid;
+    }
+    return lo;
+}
+
+// Stencil row spans of every non-empty cell c (cx, cy): for y' in cy-1..cy+1,
+// the sorted positions of cells (max(cx-1,0) .. min(cx+1,nx-1), y').  The own
+// row uses the neighbouring entries directly; the rows above/below are binary
+// searches over the keys (the cells of row cy-1 precede c, of row cy+1 follow).
+// Also gcount[c] = number of 32-query groups of the cell.
+__global__ void __launch_bounds__(256) k_cell_spans(const uint64_t* __restrict__ ckey,
+                                                    const uint32_t* __restrict__ cstart, uint64_t nne,
+                                                    uint32_t nx, uint32_t ny, uint2* __restrict__ cspan,
+                                                    uint32_t* __restrict__ gcount) {
+    for (uint64_t c = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; c < nne;
+         c += (uint64_t)gridDim.x * blockDim.x) {
+        const uint64_t key = ckey[c];
+        const uint64_t cy = key / nx, cx = key - cy * nx;
+        const uint64_t xl = cx > 0 ? cx - 1 : 0;
+        const uint64_t xh = cx + 1 < nx ? cx + 1 : nx - 1;
+        // own row
+        uint64_t a = c, b = c + 1;
+        if (cx > 0 && c > 0 && ckey[c - 1] == key - 1) a = c - 1;
+        if (cx + 1 < nx && c + 1 < nne && ckey[c + 1] == key + 1) b = c + 2;
+        uint2 own = make_uint2(cstart[a], cstart[b]);
+        uint2 lo_row = make_uint2(0, 0), hi_row = make_uint2(0, 0);
+        if (cy > 0) {
+            const uint64_t rb = (cy - 1) * nx;
+            uint64_t i0 = lower_bound_u64(ckey, 0, c, rb + xl);
+            uint64_t i1 = lower_bound_u64(ckey, i0, c, rb + xh + 1);
+            lo_row = make_uint2(cstart[i0], cstart[i1]);
+        }
+        if (cy + 1 < ny) {
+            const uint64_t rb = (cy + 1) * nx;
+            uint64_t i0 = lower_bound_u64(ckey, c + 1, nne, rb + xl);
+            uint64_t i1 = lower_bound_u64(ckey, i0, nne, rb + xh + 1);
+            hi_row = make_uint2(cstart[i0], cstart[i1]);
+        }
+        cspan[3 * c + 0] = lo_row;
+        cspan[3 * c + 1] = own;
+        cspan[3 * c + 2] = hi_row;
+        gcount[c] = (cstart[c + 1] - cstart[c] + (uint32_t)kGroup - 1) / (uint32_t)kGroup;
+    }
+}
+
+__global__ void __launch_bounds__(256) k_group_build(const uint32_t* __restrict__ cstart,
+                                                     const uint32_t* __restrict__ gofs, uint64_t nne, uint64_t n,
+                                                     uint32_t* __restrict__ gstart, uint32_t* __restrict__ gcell) {
+    for (uint64_t c = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; c < nne;
+         c += (uint64_t)gridDim.x * blockDim.x) {
+        const uint32_t s0 = cstart[c], s1 = cstart[c + 1];
+        uint32_t g = gofs[c];
+        for (uint32_t s = s0; s < s1; s += kGroup, ++g) {
+            gstart[g] = s;
+            gcell[g] = (uint32_t)c;
+        }
+    }
+    if (blockIdx.x == 0 && threadIdx.x == 0) gstart[gofs[nne]] = (uint32_t)n;
 }
 
 inline unsigned grid_for(uint64_t n, int threads = 256, unsigned cap = 148u * 16u) {
@@ -274,7 +333,7 @@ void launch_bbox(const void* xy, uint64_t n, hdb_dtype dt, unsigned long long* b
 }
 
 void launch_keys(const void* xy, uint64_t n, hdb_dtype dt, double xmin, double ymin, double inv_w,
-                 uint32_t nx, uint32_t ny, uint32_t* keys, uint32_t* vals, cudaStream_t s) {
+                 uint32_t nx, uint32_t ny, uint64_t* keys, uint32_t* vals, cudaStream_t s) {
     if (n == 0) return;
     if (dt == HDB_F64)
         k_keys<double><<<grid_for(n), 256, 0, s>>>((const double2*)xy, n, xmin, ymin, inv_w, nx, ny, keys, vals);
@@ -289,7 +348,7 @@ size_t radix_sort_temp_bytes(uint64_t n) {
     return (m + 1) * sizeof(uint32_t) * 2 + scan_temp_bytes(m) + 256;
 }
 
-int radix_sort_pairs(uint32_t* k0, uint32_t* v0, uint32_t* k1, uint32_t* v1, uint64_t n, int bits, void* temp,
+int radix_sort_pairs(uint64_t* k0, uint32_t* v0, uint64_t* k1, uint32_t* v1, uint64_t n, int bits, void* temp,
                      cudaStream_t s) {
     if (n <= 1 || bits <= 0) return 0;
     uint32_t nblocks = (uint32_t)((n + RS_TILE - 1) / RS_TILE);
@@ -299,9 +358,9 @@ int radix_sort_pairs(uint32_t* k0, uint32_t* v0, uint32_t* k1, uint32_t* v1, uin
     void* stemp = (void*)(((uintptr_t)(hscan + m + 1) + 255) & ~(uintptr_t)255);
     int cur = 0;
     for (int shift = 0; shift < bits; shift += RS_BITS) {
-        uint32_t* ki = cur ? k1 : k0;
+        uint64_t* ki = cur ? k1 : k0;
         uint32_t* vi = cur ? v1 : v0;
-        uint32_t* ko = cur ? k0 : k1;
+        uint64_t* ko = cur ? k0 : k1;
         uint32_t* vo = cur ? v0 : v1;
         k_radix_hist<<<nblocks, RS_THREADS, 0, s>>>(ki, n, shift, hist, nblocks);
         ++g_kernel_launches;
@@ -313,33 +372,38 @@ int radix_sort_pairs(uint32_t* k0, uint32_t* v0, uint32_t* k1, uint32_t* v1, uin
     return cur;
 }
 
-void launch_gather_points(const void* xy_in, const uint32_t* ids, uint64_t n, hdb_dtype dt, void* xy_s,
-                          cudaStream_t s) {
+void launch_gather_points(const void* xy_in, const uint32_t* ids, uint64_t n, hdb_dtype dt, void* xy_s, float2* xf,
+                          double ox, double oy, cudaStream_t s) {
     if (n == 0) return;
     if (dt == HDB_F64)
-        k_gather<double><<<grid_for(n), 256, 0, s>>>((const double2*)xy_in, ids, n, (double2*)xy_s);
+        k_gather<double><<<grid_for(n), 256, 0, s>>>((const double2*)xy_in, ids, n, (double2*)xy_s, xf, ox, oy);
     else
-        k_gather<float><<<grid_for(n), 256, 0, s>>>((const float2*)xy_in, ids, n, (float2*)xy_s);
+        k_gather<float><<<grid_for(n), 256, 0, s>>>((const float2*)xy_in, ids, n, (float2*)xy_s, nullptr, 0, 0);
     ++g_kernel_launches;
 }
 
-void launch_cell_counts(const uint32_t* keys_sorted, uint64_t n, uint32_t* cell_cnt,
-                        unsigned long long* n_nonempty, cudaStream_t s) {
+void launch_cell_flags(const uint64_t* keys_sorted, uint64_t n, uint32_t* flags, cudaStream_t s) {
     if (n == 0) return;
-    k_cell_counts<<<grid_for(n), 256, 0, s>>>(keys_sorted, n, cell_cnt, n_nonempty);
+    k_cell_flags<<<grid_for(n), 256, 0, s>>>(keys_sorted, n, flags);
     ++g_kernel_launches;
 }
 
-void launch_group_flags(const uint32_t* keys_sorted, const uint32_t* start, uint64_t n, uint32_t* flags,
-                        cudaStream_t s) {
-    if (n == 0) return;
-    k_group_flags<<<grid_for(n), 256, 0, s>>>(keys_sorted, start, n, flags);
+void launch_cell_scatter(const uint64_t* keys_sorted, const uint32_t* flags, const uint32_t* pos, uint64_t n,
+                         uint64_t* ckey, uint32_t* cstart, cudaStream_t s) {
+    k_cell_scatter<<<grid_for(n), 256, 0, s>>>(keys_sorted, flags, pos, n, ckey, cstart);
     ++g_kernel_launches;
 }
 
-void launch_group_scatter(const uint32_t* flags, const uint32_t* pos, uint64_t n, uint32_t* gstart,
-                          cudaStream_t s) {
-    k_group_scatter<<<grid_for(n), 256, 0, s>>>(flags, pos, n, gstart);
+void launch_cell_spans(const uint64_t* ckey, const uint32_t* cstart, uint64_t nne, uint32_t nx, uint32_t ny,
+                       uint2* cspan, uint32_t* gcount, cudaStream_t s) {
+    if (nne == 0) return;
+    k_cell_spans<<<grid_for(nne), 256, 0, s>>>(ckey, cstart, nne, nx, ny, cspan, gcount);
+    ++g_kernel_launches;
+}
+
+void launch_group_build(const uint32_t* cstart, const uint32_t* gofs, uint64_t nne, uint64_t n, uint32_t* gstart,
+                        uint32_t* gcell, cudaStream_t s) {
+    k_group_build<<<grid_for(nne), 256, 0, s>>>(cstart, gofs, nne, n, gstart, gcell);
     ++g_kernel_launches;
 }
 

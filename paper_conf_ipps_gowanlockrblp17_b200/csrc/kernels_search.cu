@@ -6,18 +6,25 @@
 //
 //  * Row spans.  Keys are row-major (h = cy*nx + cx) and points are sorted by
 //    key, so the 3 cells (cx-1..cx+1, y') of one stencil row are ONE contiguous
-//    span of sorted positions: [G[h(cx-1,y')], G[h(cx+1,y')+1]).  A query's
-//    candidates are 3 contiguous spans (reading R8 of Alg. 2 lines 8-10).
+//    span of sorted positions (reading R8 of Alg. 2 lines 8-10); the grid
+//    stores the 3 spans of every non-empty cell.
 //  * Query groups.  A warp owns <= 32 consecutive queries of one cell (they share
-//    the 3 spans); lane j streams candidate j of a 32-wide chunk with one
-//    coalesced 16-B (f64) / 8-B (f32) load, and every query of the group is
-//    tested against the chunk: hit = pred(q_i, c_j); ballot; popc.
-//  * Count -> scan -> write (a6-a8): the count pass stores |N_eps(q)|, an exclusive
-//    scan gives each query's offset, and the write pass stores the ballot-
-//    compacted hits contiguously into the query's CSR segment (no atomics, no
-//    overflow, no key/value sort -- Alg. 4 line 7's Thrust sort is unnecessary).
-//  * Exact predicate: fl(fl(dx*dx)+fl(dy*dy)) <= fl(eps^2) with __d*_rn / __f*_rn
-//    intrinsics, which nvcc never contracts into FMA (reading R2).
+//    the 3 spans).  Candidates stream through the warp in chunks of 64: lane j
+//    holds candidates j and j+32 as one packed f32x2 pair, and every query of
+//    the group is tested against the chunk with FADD2/FFMA2 (two tests per
+//    instruction); ballot + popc give counts and the compacted write positions.
+//  * Exact predicate, fast.  The paper fixes only dist <= eps; the
+//    contract here is the f64 no-FMA predicate of the oracle (reading R1/R2).
+//    f64 mode evaluates t = (dx^2 - e2) + dy^2 in f32 on coordinates relative to
+//    the bbox centre; whenever |t| > band (a rigorous bound on the f32 error,
+//    computed on the host -- DESIGN.md "filter bound") sign(t) IS the exact f64
+//    decision; the rare |t| <= band tests are re-done in exact f64 with
+//    __dsub_rn/__dmul_rn/__dadd_rn (never contracted to FMA).  f32 mode
+//    evaluates the f32 predicate itself exactly (sub/mul/add .rn f32x2).
+//  * Count -> scan -> write (a6-a8): the count pass stores |N_eps(q)|, an
+//    exclusive scan gives each query's offset, and the write pass stores the
+//    ballot-compacted hits contiguously into the query's CSR segment (no
+//    atomics, no overflow, no key/value sort -- Alg. 4 line 7 is unnecessary).
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -25,146 +32,249 @@
 
 namespace hdb {
 
-extern std::atomic<uint64_t> g_kernel_launches;
-
 namespace {
 
 constexpr unsigned FULL = 0xffffffffu;
+constexpr int kWarps = kSearchThreads / 32;
 
-template <typename T>
-struct V2;
-template <>
-struct V2<double> {
-    using type = double2;
-};
-template <>
-struct V2<float> {
-    using type = float2;
+struct SArgs {
+    const float2* xf;      // f32 coordinates: filter coords (f64 mode) / exact coords (f32 mode)
+    const double2* xd;     // exact f64 coordinates (f64 mode)
+    const uint32_t* ids;
+    const uint32_t* cstart;
+    const uint2* cspan;
+    const uint32_t* gstart;
+    const uint32_t* gcell;
+    float e2f;             // f32 mode: fl32(eps^2); f64 mode: fl32(e2_d)
+    float band;            // f64 mode: decide in exact f64 when |t| <= band
+    double e2d;            // fl64(eps^2)
 };
 
-// O1 predicate, exact: no FMA contraction possible with explicit _rn ops.
-__device__ __forceinline__ bool pred(double xp, double yp, double xq, double yq, double e2) {
+typedef unsigned long long u64x;
+
+__device__ __forceinline__ u64x pack2(float a, float b) {
+    u64x r;
+    asm("mov.b64 %0, {%1,%2};" : "=l"(r) : "f"(a), "f"(b));
+    return r;
+}
+__device__ __forceinline__ float2 unpack2(u64x v) {
+    float2 r;
+    asm("mov.b64 {%0,%1}, %2;" : "=f"(r.x), "=f"(r.y) : "l"(v));
+    return r;
+}
+__device__ __forceinline__ u64x sub2(u64x a, u64x b) {
+    u64x r;
+    asm("sub.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(a), "l"(b));
+    return r;
+}
+__device__ __forceinline__ u64x mul2(u64x a, u64x b) {
+    u64x r;
+    asm("mul.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(a), "l"(b));
+    return r;
+}
+__device__ __forceinline__ u64x add2(u64x a, u64x b) {
+    u64x r;
+    asm("add.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(a), "l"(b));
+    return r;
+}
+__device__ __forceinline__ u64x fma2(u64x a, u64x b, u64x c) {
+    u64x r;
+    asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(r) : "l"(a), "l"(b), "l"(c));
+    return r;
+}
+
+// O1 predicate in exact f64: no FMA contraction possible with explicit _rn ops.
+__device__ __forceinline__ bool pred_f64(double xp, double yp, double xq, double yq, double e2) {
     double dx = __dsub_rn(xp, xq);
     double dy = __dsub_rn(yp, yq);
     return __dadd_rn(__dmul_rn(dx, dx), __dmul_rn(dy, dy)) <= e2;
 }
-__device__ __forceinline__ bool pred(float xp, float yp, float xq, float yq, float e2) {
+__device__ __forceinline__ bool pred_f32(float xp, float yp, float xq, float yq, float e2) {
     float dx = __fsub_rn(xp, xq);
     float dy = __fsub_rn(yp, yq);
     return __fadd_rn(__fmul_rn(dx, dx), __fmul_rn(dy, dy)) <= e2;
 }
 
-__device__ __forceinline__ double far_coord(double) { return 1e300; }
-__device__ __forceinline__ float far_coord(float) { return 3e38f; }
+constexpr float kFar = 1e30f;   // padding coordinate: never a neighbour (t ~ 1e60 -> inf > band)
 
-// Stencil row spans of cell `key`: span r = [lo[r], hi[r]) (empty if out of grid).
-__device__ __forceinline__ void row_spans(const uint32_t* __restrict__ start, uint32_t key, uint32_t nx,
-                                          uint32_t ny, uint32_t lo[3], uint32_t hi[3]) {
-    uint32_t cy = key / nx, cx = key - cy * nx;
-    uint32_t xl = cx > 0 ? cx - 1 : 0;
-    uint32_t xh = cx + 1 < nx ? cx + 1 : nx - 1;
-#pragma unroll
-    for (int r = 0; r < 3; ++r) {
-        int yy = (int)cy + r - 1;
-        if (yy < 0 || yy >= (int)ny) {
-            lo[r] = hi[r] = 0;
-        } else {
-            uint32_t rowb = (uint32_t)yy * nx;
-            lo[r] = __ldg(&start[rowb + xl]);
-            hi[r] = __ldg(&start[rowb + xh + 1]);
-        }
+// Kernel modes: f32 input (exact f32 predicate), f64 input with the f32
+// filter + exact f64 fallback, f64 input tested in exact f64 only (used when
+// the filter bound is useless, e.g. extent/eps near 2^30 or huge coordinates).
+enum Mode { kF32 = 0, kF64Filter = 1, kF64Exact = 2 };
+
+// Tests of query q (broadcast) against the lane's two candidates (packed).
+// Returns the two hit predicates via in0/in1.
+template <int MODE>
+__device__ __forceinline__ void test_pair(const SArgs& a, float4 q, u64x X, u64x Y, bool v0, bool v1, uint32_t j0,
+                                          uint32_t j1, const double2& qd, const double2& c0, const double2& c1,
+                                          bool& in0, bool& in1) {
+    if (MODE == kF64Exact) {
+        in0 = v0 && pred_f64(qd.x, qd.y, c0.x, c0.y, a.e2d);
+        in1 = v1 && pred_f64(qd.x, qd.y, c1.x, c1.y, a.e2d);
+        return;
     }
-}
-
-// a5: thread per sampled query (the paper's estimator kernel).
-template <typename T>
-__global__ void __launch_bounds__(256) k_sample_count(GridArgs<T> g, uint64_t stride, uint64_t ns,
-                                                      uint32_t* __restrict__ samp_cnt,
-                                                      unsigned long long* __restrict__ sum) {
-    using V = typename V2<T>::type;
-    const V* __restrict__ xy = (const V*)g.xy;
-    uint64_t j = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
-    uint32_t c = 0;
-    if (j < ns) {
-        uint64_t s = j * stride;
-        V q = xy[s];
-        uint32_t lo[3], hi[3];
-        row_spans(g.start, g.keys[s], g.nx, g.ny, lo, hi);
-        for (int r = 0; r < 3; ++r)
-            for (uint32_t k = lo[r]; k < hi[r]; ++k) {
-                V p = xy[k];
-                c += pred(q.x, q.y, p.x, p.y, g.e2) ? 1u : 0u;
+    const u64x qx = pack2(q.x, q.y);   // {qx, qx}
+    const u64x qy = pack2(q.z, q.w);   // {qy, qy}
+    const u64x dx = sub2(qx, X);
+    const u64x dy = sub2(qy, Y);
+    if (MODE == kF64Filter) {
+        const u64x ne2 = pack2(-a.e2f, -a.e2f);
+        const float2 t = unpack2(fma2(dy, dy, fma2(dx, dx, ne2)));   // (dx^2 - e2) + dy^2
+        in0 = v0 && t.x < 0.f;
+        in1 = v1 && t.y < 0.f;
+        const bool b0 = v0 && fabsf(t.x) <= a.band;
+        const bool b1 = v1 && fabsf(t.y) <= a.band;
+        if (__any_sync(FULL, b0 || b1)) {   // rare: decide in exact f64
+            if (b0) {
+                const double2 p = a.xd[j0];
+                in0 = pred_f64(qd.x, qd.y, p.x, p.y, a.e2d);
             }
-        if (samp_cnt) samp_cnt[j] = c;
+            if (b1) {
+                const double2 p = a.xd[j1];
+                in1 = pred_f64(qd.x, qd.y, p.x, p.y, a.e2d);
+            }
+        }
+    } else {
+        const float2 d2 = unpack2(add2(mul2(dx, dx), mul2(dy, dy)));  // fl(fl(dx^2) + fl(dy^2))
+        in0 = v0 && d2.x <= a.e2f;
+        in1 = v1 && d2.y <= a.e2f;
     }
-    unsigned long long t = c;
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) t += __shfl_xor_sync(FULL, t, o);
-    if ((threadIdx.x & 31) == 0 && t) atomicAdd(sum, t);
 }
 
-// a6 / a8: warp per query group, lane per candidate.
-template <typename T, bool WRITE>
-__global__ void __launch_bounds__(kSearchThreads) k_search(GridArgs<T> g, uint32_t g0, uint32_t g1,
+// a6 / a8: warp per query group, two candidates per lane per chunk.
+template <int MODE, bool WRITE>
+__global__ void __launch_bounds__(kSearchThreads) k_search(SArgs a, uint32_t g0, uint32_t g1,
                                                            uint32_t* __restrict__ cnt,
                                                            unsigned long long* __restrict__ tests_out,
                                                            const uint64_t* __restrict__ off, uint64_t out_base,
                                                            uint32_t* __restrict__ out) {
-    using V = typename V2<T>::type;
-    const V* __restrict__ xy = (const V*)g.xy;
+    constexpr bool F64 = MODE != kF32;
+    __shared__ float4 sq[kWarps][32];              // {qx, qx, qy, qy}
+    __shared__ double2 sqd[F64 ? kWarps : 1][32];  // exact query coordinates (f64 modes)
     const int lane = threadIdx.x & 31;
+    const int w = threadIdx.x >> 5;
     const unsigned lt = (1u << lane) - 1u;
     const uint32_t wid = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const uint32_t nw = (gridDim.x * blockDim.x) >> 5;
     unsigned long long tests = 0;
     for (uint32_t gi = g0 + wid; gi < g1; gi += nw) {
-        const uint32_t qs = __ldg(&g.gstart[gi]);
-        const uint32_t key = __ldg(&g.keys[qs]);
-        const uint32_t cend = __ldg(&g.start[key + 1]);
-        const uint32_t nq = min((uint32_t)kGroup, cend - qs);
-        V q;
-        q.x = far_coord(T(0));
-        q.y = far_coord(T(0));
-        if ((uint32_t)lane < nq) q = xy[qs + lane];
-        uint64_t cur = 0;     // write: this lane's query's next output slot
-        uint32_t c = 0;       // count: this lane's query's count
-        if (WRITE && (uint32_t)lane < nq) cur = off[qs + lane] - out_base;
-        uint32_t lo[3], hi[3];
-        row_spans(g.start, key, g.nx, g.ny, lo, hi);
+        const uint32_t qs = __ldg(&a.gstart[gi]);
+        const uint32_t c = __ldg(&a.gcell[gi]);
+        const uint32_t nq = min((uint32_t)kGroup, __ldg(&a.cstart[c + 1]) - qs);
+        __syncwarp();
+        if ((uint32_t)lane < nq) {
+            if (MODE != kF64Exact) {
+                const float2 p = a.xf[qs + lane];
+                sq[w][lane] = make_float4(p.x, p.x, p.y, p.y);
+            }
+            if (F64) sqd[F64 ? w : 0][lane] = a.xd[qs + lane];
+        }
+        uint32_t my = 0;        // count: this lane's query's count; write: its offset within the group
+        uint32_t* gout = nullptr;
+        if (WRITE) {
+            const uint64_t gb = off[qs];
+            gout = out + (gb - out_base);
+            if ((uint32_t)lane < nq) my = (uint32_t)(off[qs + lane] - gb);
+        }
+        __syncwarp();
 #pragma unroll 1
         for (int r = 0; r < 3; ++r) {
+            const uint2 sp = __ldg(&a.cspan[3 * c + r]);
+            const uint32_t hi = sp.y;
 #pragma unroll 1
-            for (uint32_t c0 = lo[r]; c0 < hi[r]; c0 += 32) {
-                const uint32_t j = c0 + lane;
-                const bool valid = j < hi[r];
-                V p;
-                p.x = far_coord(T(0));
-                p.y = far_coord(T(0));
-                uint32_t id = 0;
-                if (valid) {
-                    p = xy[j];
-                    if (WRITE) id = __ldg(&g.ids[j]);
+            for (uint32_t c0 = sp.x; c0 < hi; c0 += 64) {
+                const uint32_t j0 = c0 + lane, j1 = c0 + 32 + lane;
+                const bool v0 = j0 < hi, v1 = j1 < hi;
+                float2 p0 = make_float2(kFar, kFar), p1 = make_float2(kFar, kFar);
+                double2 c0d = make_double2(0, 0), c1d = make_double2(0, 0);
+                if (MODE == kF64Exact) {
+                    if (v0) c0d = a.xd[j0];
+                    if (v1) c1d = a.xd[j1];
+                } else {
+                    if (v0) p0 = a.xf[j0];
+                    if (v1) p1 = a.xf[j1];
                 }
-                if (!WRITE) tests += (unsigned long long)nq * min(32u, hi[r] - c0);
-#pragma unroll 4
+                const u64x X = pack2(p0.x, p1.x);
+                const u64x Y = pack2(p0.y, p1.y);
+                uint32_t id0 = 0, id1 = 0;
+                if (WRITE) {
+                    if (v0) id0 = __ldg(&a.ids[j0]);
+                    if (v1) id1 = __ldg(&a.ids[j1]);
+                }
+                if (!WRITE) tests += (unsigned long long)nq * min(64u, hi - c0);
+#pragma unroll 2
                 for (uint32_t i = 0; i < nq; ++i) {
-                    const T qx = __shfl_sync(FULL, q.x, i);
-                    const T qy = __shfl_sync(FULL, q.y, i);
-                    const bool hit = valid && pred(qx, qy, p.x, p.y, g.e2);
-                    const unsigned m = __ballot_sync(FULL, hit);
+                    float4 q = make_float4(0, 0, 0, 0);
+                    if (MODE != kF64Exact) q = sq[w][i];
+                    double2 qd = make_double2(0, 0);
+                    if (F64) qd = sqd[F64 ? w : 0][i];
+                    bool in0, in1;
+                    test_pair<MODE>(a, q, X, Y, v0, v1, j0, j1, qd, c0d, c1d, in0, in1);
+                    const unsigned m0 = __ballot_sync(FULL, in0);
+                    const unsigned m1 = __ballot_sync(FULL, in1);
+                    const uint32_t n0 = __popc(m0);
                     if (WRITE) {
-                        const uint64_t b = __shfl_sync(FULL, cur, i);
-                        if (hit) out[b + __popc(m & lt)] = id;
-                        if ((uint32_t)lane == i) cur += __popc(m);
-                    } else {
-                        if ((uint32_t)lane == i) c += __popc(m);
+                        const uint32_t b = __shfl_sync(FULL, my, i);
+                        if (in0) gout[b + __popc(m0 & lt)] = id0;
+                        if (in1) gout[b + n0 + __popc(m1 & lt)] = id1;
                     }
+                    if ((uint32_t)lane == i) my += n0 + __popc(m1);
                 }
             }
         }
-        if (!WRITE && (uint32_t)lane < nq) cnt[qs + lane] = c;
+        if (!WRITE && (uint32_t)lane < nq) cnt[qs + lane] = my;
     }
     if (!WRITE && tests_out && lane == 0 && tests) atomicAdd(tests_out, tests);
+}
+
+// a5: warp per sampled query (the paper's estimator kernel),
+// exact predicate, lanes over candidates.
+template <bool F64>
+__global__ void __launch_bounds__(256) k_sample_count(SArgs a, uint64_t nne, uint64_t stride, uint64_t ns,
+                                                      uint32_t* __restrict__ samp_cnt,
+                                                      unsigned long long* __restrict__ sum) {
+    const int lane = threadIdx.x & 31;
+    const uint64_t wid = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
+    const uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+    unsigned long long tot = 0;
+    for (uint64_t j = wid; j < ns; j += nw) {
+        const uint64_t s = j * stride;
+        // cell of sorted position s: last c with cstart[c] <= s
+        uint64_t lo = 0, hi = nne;
+        while (hi - lo > 1) {
+            uint64_t mid = (lo + hi) >> 1;
+            if (__ldg(&a.cstart[mid]) <= s)
+                lo = mid;
+            else
+                hi = mid;
+        }
+        const uint64_t c = lo;
+        uint32_t cntv = 0;
+        if (F64) {
+            const double2 q = a.xd[s];
+            for (int r = 0; r < 3; ++r) {
+                const uint2 sp = a.cspan[3 * c + r];
+                for (uint32_t k = sp.x + lane; k < sp.y; k += 32) {
+                    const double2 p = a.xd[k];
+                    cntv += pred_f64(q.x, q.y, p.x, p.y, a.e2d) ? 1u : 0u;
+                }
+            }
+        } else {
+            const float2 q = a.xf[s];
+            for (int r = 0; r < 3; ++r) {
+                const uint2 sp = a.cspan[3 * c + r];
+                for (uint32_t k = sp.x + lane; k < sp.y; k += 32) {
+                    const float2 p = a.xf[k];
+                    cntv += pred_f32(q.x, q.y, p.x, p.y, a.e2f) ? 1u : 0u;
+                }
+            }
+        }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) cntv += __shfl_xor_sync(FULL, cntv, o);
+        if (lane == 0 && samp_cnt) samp_cnt[j] = cntv;
+        tot += cntv;
+    }
+    if (lane == 0 && tot) atomicAdd(sum, tot);
 }
 
 __global__ void k_batch_cuts(const uint32_t* __restrict__ gstart, const uint64_t* __restrict__ off, uint64_t g0,
@@ -179,7 +289,6 @@ __global__ void k_batch_cuts(const uint32_t* __restrict__ gstart, const uint64_t
     } else if (b == nb) {
         g = g1;
     } else {
-        // target pair offset of cut b (128-bit safe: span < 2^64 / nb for any sane P)
         const uint64_t target = p0 + (uint64_t)(((unsigned __int128)(p1 - p0) * b) / nb);
         uint64_t lo = g0, hi = g1;   // first g in [g0, g1] with off[gstart[g]] >= target
         while (lo < hi) {
@@ -200,8 +309,7 @@ __global__ void k_pos_to_group(const uint32_t* __restrict__ gstart, uint64_t ng,
     uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= m) return;
     uint64_t p = pos[i];
-    // first group whose start is >= p  (so a shard boundary never splits a group)
-    uint64_t lo = 0, hi = ng;
+    uint64_t lo = 0, hi = ng;   // first group whose start is >= p
     while (lo < hi) {
         uint64_t mid = (lo + hi) >> 1;
         if ((uint64_t)gstart[mid] >= p)
@@ -217,38 +325,54 @@ __global__ void __launch_bounds__(256) k_scatter_rows(const uint32_t* __restrict
                                                       const uint32_t* __restrict__ cnt, uint64_t q0, uint64_t q1,
                                                       uint64_t base, uint64_t* __restrict__ begin,
                                                       uint32_t* __restrict__ count) {
+    const uint64_t o0 = off[q0];
     for (uint64_t q = q0 + blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; q < q1;
          q += (uint64_t)gridDim.x * blockDim.x) {
         uint32_t id = ids[q];
-        begin[id] = off[q] - off[q0] + base;
+        begin[id] = off[q] - o0 + base;
         count[id] = cnt[q];
     }
 }
 
-template <typename T>
-GridArgs<T> args_of(const DevGrid& g) {
-    GridArgs<T> a;
-    a.xy = g.xy_s;
+SArgs args_of(const DevGrid& g) {
+    SArgs a;
+    a.xf = g.xf;
+    a.xd = (const double2*)g.xy_s;
     a.ids = g.ids;
-    a.keys = g.keys;
-    a.start = g.start;
+    a.cstart = g.cstart;
+    a.cspan = g.cspan;
     a.gstart = g.gstart;
-    a.nx = g.nx;
-    a.ny = g.ny;
-    a.n = (uint32_t)g.n;
-    if constexpr (sizeof(T) == 8)
-        a.e2 = g.e2_d;
-    else
-        a.e2 = g.e2_f;
+    a.gcell = g.gcell;
+    a.e2f = g.e2_f;
+    a.band = g.band;
+    a.e2d = g.e2_d;
     return a;
 }
 
 unsigned search_grid(uint64_t ngroups) {
-    const uint64_t warps_per_cta = kSearchThreads / 32;
-    uint64_t ctas = (ngroups + warps_per_cta - 1) / warps_per_cta;
+    uint64_t ctas = (ngroups + kWarps - 1) / kWarps;
     const uint64_t cap = 148ull * 8ull;   // 8 CTAs x 8 warps = 64 warps per SM
     if (ctas > cap) ctas = cap;
     return (unsigned)(ctas ? ctas : 1);
+}
+
+template <bool WRITE>
+void launch_search(const DevGrid& g, uint64_t g0, uint64_t g1, uint32_t* cnt, unsigned long long* tests,
+                   const uint64_t* off, uint64_t out_base, uint32_t* out, bool force_exact, cudaStream_t s) {
+    if (g1 <= g0) return;
+    const unsigned grid = search_grid(g1 - g0);
+    const SArgs a = args_of(g);
+    const int mode = g.dtype == HDB_F32 ? kF32 : (g.filter && !force_exact ? kF64Filter : kF64Exact);
+    if (mode == kF64Filter)
+        k_search<kF64Filter, WRITE><<<grid, kSearchThreads, 0, s>>>(a, (uint32_t)g0, (uint32_t)g1, cnt, tests, off,
+                                                                     out_base, out);
+    else if (mode == kF64Exact)
+        k_search<kF64Exact, WRITE><<<grid, kSearchThreads, 0, s>>>(a, (uint32_t)g0, (uint32_t)g1, cnt, tests, off,
+                                                                    out_base, out);
+    else
+        k_search<kF32, WRITE><<<grid, kSearchThreads, 0, s>>>(a, (uint32_t)g0, (uint32_t)g1, cnt, tests, off,
+                                                               out_base, out);
+    ++g_kernel_launches;
 }
 
 }  // namespace
@@ -256,38 +380,26 @@ unsigned search_grid(uint64_t ngroups) {
 void launch_sample_count(const DevGrid& g, uint64_t stride, uint64_t n_sample, uint32_t* samp_cnt,
                          unsigned long long* sum, cudaStream_t s) {
     if (n_sample == 0) return;
-    unsigned blocks = (unsigned)((n_sample + 255) / 256);
+    uint64_t blocks = (n_sample + 7) / 8;
+    if (blocks > 148 * 16) blocks = 148 * 16;
     if (g.dtype == HDB_F64)
-        k_sample_count<double><<<blocks, 256, 0, s>>>(args_of<double>(g), stride, n_sample, samp_cnt, sum);
+        k_sample_count<true><<<(unsigned)blocks, 256, 0, s>>>(args_of(g), g.n_nonempty, stride, n_sample, samp_cnt,
+                                                              sum);
     else
-        k_sample_count<float><<<blocks, 256, 0, s>>>(args_of<float>(g), stride, n_sample, samp_cnt, sum);
+        k_sample_count<false><<<(unsigned)blocks, 256, 0, s>>>(args_of(g), g.n_nonempty, stride, n_sample, samp_cnt,
+                                                               sum);
     ++g_kernel_launches;
 }
 
-void launch_count(const DevGrid& g, uint64_t g0, uint64_t g1, uint32_t* cnt, unsigned long long* tests, int,
-                  cudaStream_t s) {
-    if (g1 <= g0) return;
-    unsigned grid = search_grid(g1 - g0);
-    if (g.dtype == HDB_F64)
-        k_search<double, false><<<grid, kSearchThreads, 0, s>>>(args_of<double>(g), (uint32_t)g0, (uint32_t)g1,
-                                                                cnt, tests, nullptr, 0, nullptr);
-    else
-        k_search<float, false><<<grid, kSearchThreads, 0, s>>>(args_of<float>(g), (uint32_t)g0, (uint32_t)g1,
-                                                               cnt, tests, nullptr, 0, nullptr);
-    ++g_kernel_launches;
+// variant (hdb_opts.search_kernel): 0 = default, 1 = force the exact-f64-only kernel
+void launch_count(const DevGrid& g, uint64_t g0, uint64_t g1, uint32_t* cnt, unsigned long long* tests,
+                  int variant, cudaStream_t s) {
+    launch_search<false>(g, g0, g1, cnt, tests, nullptr, 0, nullptr, variant == 1, s);
 }
 
 void launch_write(const DevGrid& g, uint64_t g0, uint64_t g1, const uint64_t* off, uint64_t out_base,
-                  uint32_t* out, int, cudaStream_t s) {
-    if (g1 <= g0) return;
-    unsigned grid = search_grid(g1 - g0);
-    if (g.dtype == HDB_F64)
-        k_search<double, true><<<grid, kSearchThreads, 0, s>>>(args_of<double>(g), (uint32_t)g0, (uint32_t)g1,
-                                                               nullptr, nullptr, off, out_base, out);
-    else
-        k_search<float, true><<<grid, kSearchThreads, 0, s>>>(args_of<float>(g), (uint32_t)g0, (uint32_t)g1,
-                                                              nullptr, nullptr, off, out_base, out);
-    ++g_kernel_launches;
+                  uint32_t* out, int variant, cudaStream_t s) {
+    launch_search<true>(g, g0, g1, nullptr, nullptr, off, out_base, out, variant == 1, s);
 }
 
 void launch_batch_cuts(const uint32_t* gstart, const uint64_t* off, uint64_t g0, uint64_t g1, uint32_t nb,

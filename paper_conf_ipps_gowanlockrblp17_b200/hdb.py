@@ -47,7 +47,7 @@ class hdb_grid_view(ctypes.Structure):
     _fields_ = [("n", _u64), ("eps", _dbl), ("dtype", _int), ("xmin", _dbl), ("ymin", _dbl), ("xmax", _dbl),
                 ("ymax", _dbl), ("cell_w", _dbl), ("nx", _u32), ("ny", _u32), ("n_cells", _u64),
                 ("n_nonempty", _u64), ("n_groups", _u64), ("device", _int), ("xy_sorted", _vp), ("ids", _vp),
-                ("keys_sorted", _vp), ("cell_start", _vp)]
+                ("cell_keys", _vp), ("cell_start", _vp)]
 
 
 class hdb_stats(ctypes.Structure):
@@ -205,11 +205,11 @@ def hdb_grid_view_get(grid) -> hdb_grid_view:
 def hdb_grid_copy_to_host(grid):
     v = hdb_grid_view_get(grid)
     ids = np.empty(v.n, np.uint32)
-    keys = np.empty(v.n, np.uint32)
-    start = np.empty(v.n_cells + 1, np.uint32)
+    keys = np.empty(v.n_nonempty, np.uint64)
+    start = np.empty(v.n_nonempty + 1, np.uint32)
     xy = np.empty((v.n, 2), np.float64 if v.dtype == HDB_F64 else np.float32)
     _check(lib.hdb_grid_copy_to_host(grid, _ptr(ids), _ptr(keys), _ptr(start), _ptr(xy)), "hdb_grid_copy_to_host")
-    return dict(ids=ids, keys=keys, cell_start=start, xy_sorted=xy, view=v)
+    return dict(ids=ids, cell_keys=keys, cell_start=start, xy_sorted=xy, view=v)
 
 
 def hdb_neighbor_table(ctx, grid):

@@ -196,11 +196,12 @@ def test_grid_structure_fig1(torch_cuda):
     finally:
         hdb.hdb_ctx_destroy(ctx)
     v = gg["view"]
-    ids, keys, start = gg["ids"], gg["keys"], gg["cell_start"]
+    ids, ckeys, start = gg["ids"], gg["cell_keys"], gg["cell_start"]
     n = xy.shape[0]
     assert np.array_equal(np.sort(ids), np.arange(n))                 # |A| = |D|, a permutation
-    assert np.all(np.diff(keys.astype(np.int64)) >= 0)                 # sorted by cell
-    assert start[0] == 0 and start[-1] == n and np.all(np.diff(start.astype(np.int64)) >= 0)
+    assert np.all(np.diff(ckeys.astype(np.int64)) > 0)                 # non-empty cells, ascending keys
+    assert start[0] == 0 and start[-1] == n and np.all(np.diff(start.astype(np.int64)) > 0)
+    keys = np.repeat(ckeys, np.diff(start.astype(np.int64)))           # key of every sorted position
     w = eps * (1 + 2.0 ** -19)
     assert v.cell_w == w
     inv = 1.0 / w
@@ -210,14 +211,23 @@ def test_grid_structure_fig1(torch_cuda):
     want_key = cy * v.nx + cx
     assert np.array_equal(keys.astype(np.int64), want_key[ids])
     assert np.array_equal(gg["xy_sorted"], xy[ids])
-    # cell h holds exactly the sorted positions [start[h], start[h+1])
-    h = keys.astype(np.int64)
-    pos = np.arange(n)
-    assert np.all(start[h] <= pos) and np.all(pos < start[h + 1])
     # stable: ids ascending inside each cell
+    h = keys.astype(np.int64)
     same = h[1:] == h[:-1]
     assert np.all(ids[1:][same] > ids[:-1][same])
-    assert v.n_nonempty == np.unique(h).size
+    assert v.n_nonempty == np.unique(want_key).size == ckeys.size
+    assert v.n_groups == int(np.sum((np.diff(start.astype(np.int64)) + 31) // 32))
+
+
+def test_sparse_extent_compact_grid(torch_cuda):
+    """A few points spread over a huge extent: 10^12 grid cells, only the
+    non-empty ones are stored (dense grids would not fit)."""
+    rng = np.random.default_rng(3)
+    centers = rng.uniform(-5e5, 5e5, (50, 2))
+    xy = (centers[:, None, :] + rng.normal(0, 0.5, (50, 40, 2))).reshape(-1, 2)
+    b, c, v, view, st = lib_table(xy, 1.0)
+    assert st["n_cells"] > 10 ** 11
+    assert_table_equal(xy, 1.0, b, c, v)
 
 
 # ------------------------------------------------------------------ batching / streams / shards
@@ -397,3 +407,22 @@ def test_c3_full_size_sampled_rows(torch_cuda):
     xy = datagen.sdss_like()
     for eps in datagen.C3_EPS:
         _sampled_rows_check(xy, eps, m_rows=800, seed=int(eps * 100))
+
+
+def test_exact_f64_kernel_variant(torch_cuda):
+    """search_kernel=1 forces the exact-f64-only kernel; both kernels must equal the oracle."""
+    xy = datagen.subsample(datagen.tec_like(), 30_000, seed=12)
+    for eps in (0.15, 0.45):
+        for k in (0, 1):
+            b, c, v, _, _ = lib_table(xy, eps, search_kernel=k)
+            assert_table_equal(xy, eps, b, c, v)
+
+
+def test_filter_disabled_for_huge_extent(torch_cuda):
+    """Extent/eps so large that the f32 filter bound is useless: the library
+    falls back to exact f64 and stays exact."""
+    rng = np.random.default_rng(8)
+    base = rng.uniform(-1e7, 1e7, (300, 2))
+    xy = np.concatenate([base, base + rng.normal(0, 0.02, base.shape)])
+    b, c, v, _, _ = lib_table(xy, 0.05)
+    assert_table_equal(xy, 0.05, b, c, v)
