@@ -15,6 +15,7 @@
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <exception>
 #include <memory>
@@ -99,6 +100,33 @@ PinnedPool::~PinnedPool() {
 
 // ------------------------------------------------------------------ helpers
 namespace {
+
+// HDB_TRACE=1: host wall-clock marks of the phases of each call, to stderr.
+struct Trace {
+    bool on = false;
+    const char* what;
+    std::chrono::steady_clock::time_point t0, last;
+    std::string buf;
+    explicit Trace(const char* w) : what(w) {
+        const char* e = getenv("HDB_TRACE");
+        on = e && *e == '1';
+        t0 = last = std::chrono::steady_clock::now();
+    }
+    void mark(const char* name) {
+        if (!on) return;
+        auto t = std::chrono::steady_clock::now();
+        char b[96];
+        snprintf(b, sizeof b, " %s=%.3f", name, std::chrono::duration<double, std::milli>(t - last).count());
+        buf += b;
+        last = t;
+    }
+    ~Trace() {
+        if (on)
+            fprintf(stderr, "[hdb trace] %s total=%.3f ms:%s\n", what,
+                    std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count(),
+                    buf.c_str());
+    }
+};
 
 struct DeviceGuard {
     int prev = -1;
@@ -240,6 +268,7 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
     Event ev0, ev1;
     HDB_CUDA(cudaEventRecord(ev0.e, s));
 
+    Trace tr("grid_build");
     // ---- a1: ingest + bbox + validation
     DBuf xin_owned;
     const void* xin = xy;
@@ -293,8 +322,11 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
     g.n_cells = (uint64_t)g.nx * g.ny;   // < 2^61: only the non-empty ones are stored
     set_filter_bound(g);
 
+    tr.mark("bbox+sync");
     // ---- a2: keys
-    DBuf k0(8 * n, s), v0(4 * n, s), k1(8 * n, s), v1(4 * n, s);
+    // ids and points are padded by 2 entries: the search kernels load candidate
+    // pairs (2k, 2k+1) with one vector load and mask the invalid half
+    DBuf k0(8 * n, s), v0(4 * (n + 2), s), k1(8 * n, s), v1(4 * (n + 2), s);
     launch_keys(xin, n, dt, g.xmin, g.ymin, g.inv_w, g.nx, g.ny, k0.as<uint64_t>(), v0.as<uint32_t>(), s);
     HDB_LAUNCH_CHECK();
     // ---- a3: stable radix sort by key (only the bits the key range needs)
@@ -311,12 +343,17 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
     k1.reset();
     v0.reset();
     v1.reset();
-    DBuf xy_s(n * esz, s);
-    DBuf xf;
-    if (dt == HDB_F64) xf = DBuf(8 * n, s);
-    launch_gather_points(xin, ids.as<uint32_t>(), n, dt, xy_s.p, xf.as<float2>(), g.ox, g.oy, s);
+    DBuf xy_s((n + 2) * esz, s);
+    DBuf xp(16 * (n / 2 + 2), s);
+    DBuf counters(4 * kCounterSlots, s);
+    HDB_CUDA(cudaMemsetAsync(xy_s.as<char>() + n * esz, 0, 2 * esz, s));
+    HDB_CUDA(cudaMemsetAsync(ids.as<uint32_t>() + n, 0, 8, s));
+    HDB_CUDA(cudaMemsetAsync(xp.p, 0, 16 * (n / 2 + 2), s));
+    HDB_CUDA(cudaMemsetAsync(counters.p, 0, 4 * kCounterSlots, s));
+    launch_gather_points(xin, ids.as<uint32_t>(), n, dt, xy_s.p, xp.as<float4>(), g.ox, g.oy, s);
     HDB_LAUNCH_CHECK();
     xin_owned.reset();
+    tr.mark("keys+sort+gather(enqueue)");
     // ---- a4: run boundaries -> scan -> (key, start) of the non-empty cells
     DBuf flags(4 * n, s), pos(4 * (n + 1), s);
     launch_cell_flags(keys.as<uint64_t>(), n, flags.as<uint32_t>(), s);
@@ -334,6 +371,7 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
     flags.reset();
     pos.reset();
     keys.reset();
+    tr.mark("cells+sync");
     // ---- stencil row spans per non-empty cell + query groups
     DBuf cspan(24 * nne, s), gcount(4 * (nne + 1), s), gofs(4 * (nne + 1), s);
     launch_cell_spans(ckey.as<uint64_t>(), cstart.as<uint32_t>(), nne, g.nx, g.ny, cspan.as<uint2>(),
@@ -355,26 +393,40 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
     HDB_CUDA(cudaEventRecord(ev1.e, s));
     HDB_CUDA(cudaEventSynchronize(ev1.e));
     g.ms_build = elapsed(ev0, ev1);
+    tr.mark("groups+sync");
     g.xy_s = xy_s.release();
-    g.xf = dt == HDB_F64 ? (float2*)xf.release() : (float2*)g.xy_s;
+    g.xp = (float4*)xp.release();
+    g.counters = (unsigned int*)counters.release();
     g.ids = (uint32_t*)ids.release();
     g.ckey = (uint64_t*)ckey.release();
     g.cstart = (uint32_t*)cstart.release();
     g.cspan = (uint2*)cspan.release();
     g.gstart = (uint32_t*)gstart.release();
     g.gcell = (uint32_t*)gcell.release();
+    // hit-mask table layout of the two-pass search (count stores, write replays)
+    {
+        DBuf words(4 * (g.n_groups + 1), s), mtemp(scan_temp_bytes(g.n_groups + 1), s), moff(8 * (g.n_groups + 1), s);
+        launch_mask_words(g, words.as<uint32_t>(), s);
+        scan_u32_to_u64(words.as<uint32_t>(), moff.as<uint64_t>(), g.n_groups, mtemp.p, s);
+        HDB_LAUNCH_CHECK();
+        HDB_CUDA(cudaMemcpyAsync(&g.mask_words, moff.as<uint64_t>() + g.n_groups, 8, cudaMemcpyDeviceToHost, s));
+        HDB_CUDA(cudaStreamSynchronize(s));
+        g.moff = (uint64_t*)moff.release();
+    }
+    tr.mark("mask-layout+sync");
 }
 
 void free_dev_grid(DevGrid& g) {
     if (!g.stream) return;
     DeviceGuard dg(g.device);
-    void* xf = (g.dtype == HDB_F64) ? (void*)g.xf : nullptr;
-    for (void* p : {(void*)g.xy_s, xf, (void*)g.ids, (void*)g.ckey, (void*)g.cstart, (void*)g.cspan,
-                    (void*)g.gstart, (void*)g.gcell})
-        if (p) cudaFreeAsync(p, g.stream);
+    for (void* p : {(void*)g.xy_s, (void*)g.xp, (void*)g.counters, (void*)g.ids, (void*)g.ckey, (void*)g.cstart,
+                    (void*)g.cspan, (void*)g.gstart, (void*)g.gcell, (void*)g.moff})
+        if (p) cudaFreeAsync(p, g.stream);   // stream-ordered: no host sync needed
     g.xy_s = nullptr;
-    g.xf = nullptr;
+    g.xp = nullptr;
+    g.counters = nullptr;
     g.ids = g.cstart = g.gstart = g.gcell = nullptr;
+    g.moff = nullptr;
     g.ckey = nullptr;
     g.cspan = nullptr;
     cudaStreamSynchronize(g.stream);
@@ -429,6 +481,8 @@ struct ShardRange {
 struct ShardState {
     ShardRange r;
     DBuf cnt, off;
+    DBuf masks;              // hit masks of the shard's groups (null: write pass recomputes)
+    uint2* mask_base = nullptr;   // masks - moff[g0]/2, indexed by the grid-wide layout
     uint64_t pairs = 0;
     uint64_t tests = 0;
     uint64_t base = 0;   // global offset of this shard's first pair
@@ -460,21 +514,23 @@ std::vector<uint64_t> shard_cuts(const DevGrid& g, DevCtx& dc, const std::vector
     return cuts;
 }
 
-uint32_t read_u32(const uint32_t* d, cudaStream_t s) {
-    uint32_t v = 0;
-    HDB_CUDA(cudaMemcpyAsync(&v, d, 4, cudaMemcpyDeviceToHost, s));
-    HDB_CUDA(cudaStreamSynchronize(s));
-    return v;
-}
-
 // a6 + a7 on one device for one shard
 void count_phase(hdb_ctx* ctx, DevCtx& dc, const DevGrid& g, ShardState& st) {
     DeviceGuard dg(dc.device);
+    Trace tr("count_phase");
     cudaStream_t s = dc.main;
     const uint64_t n = g.n;
-    if (st.r.g1 > st.r.g0) {
-        st.r.q0 = read_u32(g.gstart + st.r.g0, s);
-        st.r.q1 = read_u32(g.gstart + st.r.g1, s);
+    const bool whole = st.r.g0 == 0 && st.r.g1 == g.n_groups;   // no syncs needed for the full range
+    if (whole) {
+        st.r.q0 = 0;
+        st.r.q1 = n;
+    } else if (st.r.g1 > st.r.g0) {
+        uint32_t q[2] = {0, 0};
+        HDB_CUDA(cudaMemcpyAsync(&q[0], g.gstart + st.r.g0, 4, cudaMemcpyDeviceToHost, s));
+        HDB_CUDA(cudaMemcpyAsync(&q[1], g.gstart + st.r.g1, 4, cudaMemcpyDeviceToHost, s));
+        HDB_CUDA(cudaStreamSynchronize(s));
+        st.r.q0 = q[0];
+        st.r.q1 = q[1];
     } else {
         st.r.q0 = st.r.q1 = 0;
     }
@@ -482,10 +538,29 @@ void count_phase(hdb_ctx* ctx, DevCtx& dc, const DevGrid& g, ShardState& st) {
     st.off = DBuf(8 * (n + 1), s);
     DBuf tests(8, s);
     HDB_CUDA(cudaMemsetAsync(tests.p, 0, 8, s));
+    // mask table for the shard's groups (search_kernel == 2 asks for the recompute
+    // write pass; an allocation failure falls back to it as well)
+    if (st.r.g1 > st.r.g0 && ctx->opts.search_kernel != 2) {
+        uint64_t mo[2] = {0, g.mask_words};
+        if (!whole) {
+            HDB_CUDA(cudaMemcpyAsync(&mo[0], g.moff + st.r.g0, 8, cudaMemcpyDeviceToHost, s));
+            HDB_CUDA(cudaMemcpyAsync(&mo[1], g.moff + st.r.g1, 8, cudaMemcpyDeviceToHost, s));
+            HDB_CUDA(cudaStreamSynchronize(s));
+        }
+        const size_t bytes = 4 * (mo[1] - mo[0]);
+        void* p = nullptr;
+        if (cudaMallocAsync(&p, bytes ? bytes : 16, s) == cudaSuccess) {
+            st.masks.p = p;
+            st.masks.s = s;
+            st.mask_base = (uint2*)p - (mo[0] >> 1);
+        } else {
+            cudaGetLastError();
+        }
+    }
     Event e0, e1, e2;
     HDB_CUDA(cudaEventRecord(e0.e, s));
     launch_count(g, st.r.g0, st.r.g1, st.cnt.as<uint32_t>(), tests.as<unsigned long long>(), ctx->opts.search_kernel,
-                 s);
+                 0, st.mask_base, s);
     HDB_LAUNCH_CHECK();
     HDB_CUDA(cudaEventRecord(e1.e, s));
     const uint64_t len = st.r.q1 - st.r.q0;
@@ -499,6 +574,7 @@ void count_phase(hdb_ctx* ctx, DevCtx& dc, const DevGrid& g, ShardState& st) {
     HDB_CUDA(cudaStreamSynchronize(s));
     st.pairs = h[0];
     st.tests = h[1];
+    tr.mark("count+scan+sync");
     st.ms_count = elapsed(e0, e1);
     st.ms_scan = elapsed(e1, e2);
 }
@@ -564,7 +640,7 @@ void write_phase_host(hdb_ctx* ctx, DevCtx& dc, const DevGrid& g, ShardState& st
         if (b < S) HDB_CUDA(cudaStreamWaitEvent(ss, ready.e, 0));
         HDB_CUDA(cudaEventRecord(evs[2 * b].e, ss));
         launch_write(g, hg[b], hg[b + 1], st.off.as<uint64_t>(), hp[b], dc.batch_buf[si], ctx->opts.search_kernel,
-                     ss);
+                     1 + (int)si, st.mask_base, ss);
         HDB_LAUNCH_CHECK();
         HDB_CUDA(cudaEventRecord(evs[2 * b + 1].e, ss));
         if (pairs_b)
@@ -617,8 +693,7 @@ void table_free(hdb_table* t) {
     if (t->on_device) {
         DeviceGuard dg(t->device);
         for (void* p : {(void*)t->begin, (void*)t->count, (void*)t->nbrs})
-            if (p) cudaFreeAsync(p, t->dstream);
-        cudaStreamSynchronize(t->dstream);
+            if (p) cudaFreeAsync(p, t->dstream);   // stream-ordered: no host sync needed
     } else if (t->pool) {
         t->pool->release(t->begin, t->cap_begin);
         t->pool->release(t->count, t->cap_count);
@@ -657,6 +732,7 @@ void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hd
     t->host_threads = ctx->opts.host_threads;
     std::vector<ShardState> sh(ndev);
     try {
+        Trace tr("neighbor_table");
         // ---- a5: sampled count + plan (device 0)
         DevCtx& dc0 = ctx->dev[0];
         DeviceGuard dg0(dc0.device);
@@ -692,6 +768,7 @@ void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hd
                                 ? (uint64_t)std::ceil((1.0 + ctx->opts.alpha) * (double)S.est_pairs / (double)batch_pairs)
                                 : nb_plan;
 
+        tr.mark("sample+sync");
         // ---- query shards: processes x devices, balanced by sampled counts
         const uint32_t parts = R_proc * (uint32_t)ndev;
         std::vector<uint64_t> cuts = shard_cuts(G0, dc0, samp, stride, parts);
@@ -702,6 +779,7 @@ void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hd
         }
         // ---- a6/a7 on every device
         run_parallel(ndev, [&](size_t d) { count_phase(ctx, ctx->dev[d], grid->dev[d], sh[d]); });
+        tr.mark("count_phase");
         // ---- the final gather of counts: shard bases
         uint64_t P = 0;
         for (size_t d = 0; d < ndev; ++d) {
@@ -740,7 +818,8 @@ void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hd
             }
             Event e0, e1;
             HDB_CUDA(cudaEventRecord(e0.e, s));
-            launch_write(g, st.r.g0, st.r.g1, st.off.as<uint64_t>(), 0, nb.as<uint32_t>(), ctx->opts.search_kernel, s);
+            launch_write(g, st.r.g0, st.r.g1, st.off.as<uint64_t>(), 0, nb.as<uint32_t>(), ctx->opts.search_kernel, 1,
+                         st.mask_base, s);
             HDB_LAUNCH_CHECK();
             HDB_CUDA(cudaEventRecord(e1.e, s));
             launch_scatter_rows(g.ids, st.off.as<uint64_t>(), st.cnt.as<uint32_t>(), st.r.q0, st.r.q1, 0,
@@ -748,6 +827,7 @@ void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hd
             HDB_LAUNCH_CHECK();
             HDB_CUDA(cudaStreamSynchronize(s));
             st.ms_write = elapsed(e0, e1);
+            tr.mark("alloc+write+scatter+sync");
             st.write_launches = 1;
             st.n_batches = 1;
             st.max_batch = P;
@@ -830,6 +910,7 @@ void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hd
         for (auto& st : sh) {
             st.cnt.reset();
             st.off.reset();
+            st.masks.reset();
         }
         table_free(t);
         throw;
@@ -838,6 +919,7 @@ void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hd
         DeviceGuard dg(ctx->dev[d].device);
         sh[d].cnt.reset();
         sh[d].off.reset();
+        sh[d].masks.reset();
     }
     S.kernel_launches = (uint32_t)(g_kernel_launches.load() - launches0);
     S.ms_table_wall =

@@ -36,6 +36,7 @@ struct Error {
 // Warps per search CTA and queries per group (one warp's query tile).
 constexpr int kGroup = 32;
 constexpr int kSearchThreads = 256;
+constexpr int kCounterSlots = 64;   // slot 0: count pass; 1 + stream index: write passes
 
 // ---------------------------------------------------------------- grid
 // One device's copy of the grid (Fig. 1 re-laid out):
@@ -56,13 +57,17 @@ struct DevGrid {
     uint32_t nx = 1, ny = 1;
     uint64_t n_cells = 0, n_nonempty = 0, n_groups = 0;
     void* xy_s = nullptr;          // [n] double2 / float2, cell order (exact coordinates)
-    float2* xf = nullptr;          // [n] f32 filter coordinates (f64 mode; == xy_s in f32 mode)
+    float4* xp = nullptr;          // [n/2+1] paired-SoA f32 coords {x_2k, x_2k+1, y_2k, y_2k+1}: the
+                                   // filter coords x-ox, y-oy (f64 mode) / the exact coords (f32 mode)
+    unsigned int* counters = nullptr;  // [kCounterSlots] work counters of the search kernels
     uint32_t* ids = nullptr;       // [n] sorted pos -> original id  (A)
     uint64_t* ckey = nullptr;      // [n_nonempty] cell key of each non-empty cell (ascending)
     uint32_t* cstart = nullptr;    // [n_nonempty+1] first sorted pos of each non-empty cell (G)
     uint2* cspan = nullptr;        // [3*n_nonempty] stencil row spans [lo,hi) per non-empty cell
     uint32_t* gstart = nullptr;    // [n_groups+1] first sorted pos of each query group
     uint32_t* gcell = nullptr;     // [n_groups] non-empty cell index of each query group
+    uint64_t* moff = nullptr;      // [n_groups+1] first 32-bit word of each group's hit masks
+    uint64_t mask_words = 0;       // moff[n_groups]
     cudaStream_t stream = nullptr; // stream the buffers were allocated on
     float ms_build = 0;
 };
@@ -82,7 +87,7 @@ int radix_sort_pairs(uint64_t* k0, uint32_t* v0, uint64_t* k1, uint32_t* v1, uin
                      void* temp, cudaStream_t s);
 // gather sorted points; f64 mode also writes the f32 filter coordinates (x-ox, y-oy)
 void launch_gather_points(const void* xy_in, const uint32_t* ids, uint64_t n, hdb_dtype dt, void* xy_s,
-                          float2* xf, double ox, double oy, cudaStream_t s);
+                          float4* xp, double ox, double oy, cudaStream_t s);
 void launch_cell_flags(const uint64_t* keys_sorted, uint64_t n, uint32_t* flags, cudaStream_t s);
 void launch_cell_scatter(const uint64_t* keys_sorted, const uint32_t* flags, const uint32_t* pos, uint64_t n,
                          uint64_t* ckey, uint32_t* cstart, cudaStream_t s);
@@ -101,11 +106,15 @@ void scan_u32_to_u64(const uint32_t* in, uint64_t* out, uint64_t n, void* temp, 
 void launch_sample_count(const DevGrid& g, uint64_t stride, uint64_t n_sample, uint32_t* samp_cnt,
                          unsigned long long* sum, cudaStream_t s);
 // Exact count (a6) over query groups [g0, g1): cnt[sorted pos].
+// masks (optional): the hit-mask table (see k_emit), laid out by g.moff.
 void launch_count(const DevGrid& g, uint64_t g0, uint64_t g1, uint32_t* cnt, unsigned long long* tests,
-                  int variant, cudaStream_t s);
+                  int variant, int slot, uint2* masks, cudaStream_t s);
 // Write (a8) over groups [g0, g1): out[off[q] - out_base + k] = k-th neighbour id of q.
+// masks != null: emit from the stored hit masks; null: recompute the tests.
 void launch_write(const DevGrid& g, uint64_t g0, uint64_t g1, const uint64_t* off, uint64_t out_base,
-                  uint32_t* out, int variant, cudaStream_t s);
+                  uint32_t* out, int variant, int slot, const uint2* masks, cudaStream_t s);
+// words[g] = 32-bit words of group g's hit masks (scan -> g.moff)
+void launch_mask_words(const DevGrid& g, uint32_t* words, cudaStream_t s);
 // cuts: for b in 0..nb, gcut[b] = first group g in [g0,g1] with off[gstart[g]] >= target_b,
 // target_b = off[gstart[g0]] + b * span / nb (gcut[0] = g0, gcut[nb] = g1); pcut[b] = off[gstart[gcut[b]]]
 void launch_batch_cuts(const uint32_t* gstart, const uint64_t* off, uint64_t g0, uint64_t g1, uint32_t nb,

@@ -203,13 +203,26 @@ __global__ void __launch_bounds__(RS_THREADS) k_radix_scatter(const uint64_t* __
 template <typename T>
 __global__ void __launch_bounds__(256) k_gather(const typename V2<T>::type* __restrict__ in,
                                                 const uint32_t* __restrict__ ids, uint64_t n,
-                                                typename V2<T>::type* __restrict__ out, float2* __restrict__ xf,
+                                                typename V2<T>::type* __restrict__ out, float4* __restrict__ xp,
                                                 double ox, double oy) {
+    // xp: paired-SoA f32 copy {x_2k, x_2k+1, y_2k, y_2k+1} -- f64 input: filter
+    // coordinates fl32(fl64(x - ox)); f32 input: the exact coordinates
+    float* xpf = (float*)xp;
     for (uint64_t s = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; s < n;
          s += (uint64_t)gridDim.x * blockDim.x) {
         auto p = in[ids[s]];
         out[s] = p;
-        if (xf) xf[s] = make_float2((float)__dsub_rn((double)p.x, ox), (float)__dsub_rn((double)p.y, oy));
+        float fx, fy;
+        if (sizeof(p.x) == 8) {
+            fx = (float)__dsub_rn((double)p.x, ox);
+            fy = (float)__dsub_rn((double)p.y, oy);
+        } else {
+            fx = (float)p.x;
+            fy = (float)p.y;
+        }
+        const uint64_t k = s >> 1, o = s & 1;
+        xpf[4 * k + o] = fx;
+        xpf[4 * k + 2 + o] = fy;
     }
 }
 
@@ -372,13 +385,13 @@ int radix_sort_pairs(uint64_t* k0, uint32_t* v0, uint64_t* k1, uint32_t* v1, uin
     return cur;
 }
 
-void launch_gather_points(const void* xy_in, const uint32_t* ids, uint64_t n, hdb_dtype dt, void* xy_s, float2* xf,
+void launch_gather_points(const void* xy_in, const uint32_t* ids, uint64_t n, hdb_dtype dt, void* xy_s, float4* xp,
                           double ox, double oy, cudaStream_t s) {
     if (n == 0) return;
     if (dt == HDB_F64)
-        k_gather<double><<<grid_for(n), 256, 0, s>>>((const double2*)xy_in, ids, n, (double2*)xy_s, xf, ox, oy);
+        k_gather<double><<<grid_for(n), 256, 0, s>>>((const double2*)xy_in, ids, n, (double2*)xy_s, xp, ox, oy);
     else
-        k_gather<float><<<grid_for(n), 256, 0, s>>>((const float2*)xy_in, ids, n, (float2*)xy_s, nullptr, 0, 0);
+        k_gather<float><<<grid_for(n), 256, 0, s>>>((const float2*)xy_in, ids, n, (float2*)xy_s, xp, 0, 0);
     ++g_kernel_launches;
 }
 

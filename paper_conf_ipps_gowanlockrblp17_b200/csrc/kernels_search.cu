@@ -28,6 +28,8 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <algorithm>
+
 #include "internal.h"
 
 namespace hdb {
@@ -38,7 +40,9 @@ constexpr unsigned FULL = 0xffffffffu;
 constexpr int kWarps = kSearchThreads / 32;
 
 struct SArgs {
-    const float2* xf;      // f32 coordinates: filter coords (f64 mode) / exact coords (f32 mode)
+    const float4* xp;      // paired-SoA f32 coordinates {x_2k, x_2k+1, y_2k, y_2k+1}: filter coords (f64
+                           // mode) / exact coords (f32 mode)
+    const float2* xs;      // f32 mode: exact coordinates (sorted)
     const double2* xd;     // exact f64 coordinates (f64 mode)
     const uint32_t* ids;
     const uint32_t* cstart;
@@ -77,6 +81,14 @@ __device__ __forceinline__ u64x add2(u64x a, u64x b) {
     asm("add.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(a), "l"(b));
     return r;
 }
+// predicated global store (keeps the st.global space after the pointer is laundered).
+// No "memory" clobber: nothing in the kernels reads the output, and a clobber
+// would pin every later shared/global load behind the store (serialising the
+// emission loop on LDS latency).
+__device__ __forceinline__ void stg_if(uint32_t* p, uint32_t v, bool f) {
+    asm volatile("{ .reg .pred q; setp.ne.b32 q, %2, 0; @q st.global.u32 [%0], %1; }" ::"l"(p), "r"(v),
+                 "r"((uint32_t)f));
+}
 __device__ __forceinline__ u64x fma2(u64x a, u64x b, u64x c) {
     u64x r;
     asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(r) : "l"(a), "l"(b), "l"(c));
@@ -95,136 +107,324 @@ __device__ __forceinline__ bool pred_f32(float xp, float yp, float xq, float yq,
     return __fadd_rn(__fmul_rn(dx, dx), __fmul_rn(dy, dy)) <= e2;
 }
 
-constexpr float kFar = 1e30f;   // padding coordinate: never a neighbour (t ~ 1e60 -> inf > band)
-
 // Kernel modes: f32 input (exact f32 predicate), f64 input with the f32
 // filter + exact f64 fallback, f64 input tested in exact f64 only (used when
 // the filter bound is useless, e.g. extent/eps near 2^30 or huge coordinates).
 enum Mode { kF32 = 0, kF64Filter = 1, kF64Exact = 2 };
 
-// Tests of query q (broadcast) against the lane's two candidates (packed).
-// Returns the two hit predicates via in0/in1.
-template <int MODE>
-__device__ __forceinline__ void test_pair(const SArgs& a, float4 q, u64x X, u64x Y, bool v0, bool v1, uint32_t j0,
-                                          uint32_t j1, const double2& qd, const double2& c0, const double2& c1,
-                                          bool& in0, bool& in1) {
-    if (MODE == kF64Exact) {
-        in0 = v0 && pred_f64(qd.x, qd.y, c0.x, c0.y, a.e2d);
-        in1 = v1 && pred_f64(qd.x, qd.y, c1.x, c1.y, a.e2d);
-        return;
-    }
-    const u64x qx = pack2(q.x, q.y);   // {qx, qx}
-    const u64x qy = pack2(q.z, q.w);   // {qy, qy}
-    const u64x dx = sub2(qx, X);
-    const u64x dy = sub2(qy, Y);
-    if (MODE == kF64Filter) {
-        const u64x ne2 = pack2(-a.e2f, -a.e2f);
-        const float2 t = unpack2(fma2(dy, dy, fma2(dx, dx, ne2)));   // (dx^2 - e2) + dy^2
-        in0 = v0 && t.x < 0.f;
-        in1 = v1 && t.y < 0.f;
-        const bool b0 = v0 && fabsf(t.x) <= a.band;
-        const bool b1 = v1 && fabsf(t.y) <= a.band;
-        if (__any_sync(FULL, b0 || b1)) {   // rare: decide in exact f64
-            if (b0) {
-                const double2 p = a.xd[j0];
-                in0 = pred_f64(qd.x, qd.y, p.x, p.y, a.e2d);
-            }
-            if (b1) {
-                const double2 p = a.xd[j1];
-                in1 = pred_f64(qd.x, qd.y, p.x, p.y, a.e2d);
-            }
-        }
-    } else {
-        const float2 d2 = unpack2(add2(mul2(dx, dx), mul2(dy, dy)));  // fl(fl(dx^2) + fl(dy^2))
-        in0 = v0 && d2.x <= a.e2f;
-        in1 = v1 && d2.y <= a.e2f;
-    }
+// Dynamic work distribution: warps grab `chunk` consecutive query groups at a
+// time from a global counter (heavy-tailed group costs: dense cells have up
+// to ~60x the candidates of sparse ones, C2/C5).
+__device__ __forceinline__ uint32_t grab(unsigned int* ctr, uint32_t chunk, int lane) {
+    uint32_t v = 0;
+    if (lane == 0) v = atomicAdd(ctr, chunk);
+    return __shfl_sync(FULL, v, 0);
 }
 
-// a6 / a8: warp per query group, two candidates per lane per chunk.
+// Hit-mask table (count pass -> write pass).  Per group, chunks are grouped in
+// windows of kWin; window v holds, for each query i, its kWin chunk masks
+// contiguously: masks[v][i][kk] (uint2 = even / odd candidate halves).  The
+// write pass then emits query by query inside a window, i.e. in runs of
+// ~kWin * 27 consecutive ids per query (long sequential store streams).
+constexpr int kWin = 8;
+
+__device__ __forceinline__ void flush_window(uint2 (*swin)[kWin], uint2* gmask, uint32_t v, uint32_t nq,
+                                             int lane) {
+    __syncwarp();
+    if ((uint32_t)lane < nq) {
+        const uint4* src = (const uint4*)swin[lane];
+        uint4* dst = (uint4*)(gmask + ((size_t)v * nq + lane) * kWin);
+#pragma unroll
+        for (int u = 0; u < kWin / 2; ++u) dst[u] = src[u];
+    }
+    __syncwarp();
+#pragma unroll
+    for (int kk = 0; kk < kWin; ++kk) swin[lane][kk] = make_uint2(0, 0);   // next window starts empty
+    __syncwarp();
+}
+
+// a6 / a8: warp per query group; lane j holds the candidate PAIR (2k, 2k+1)
+// of the chunk (one 16-B load of the paired-SoA layout {x0, x1, y0, y1} gives
+// the packed operands X = {x0, x1}, Y = {y0, y1} directly); each query is
+// tested against 64 candidates with FADD2/FFMA2 and two ballots.
 template <int MODE, bool WRITE>
-__global__ void __launch_bounds__(kSearchThreads) k_search(SArgs a, uint32_t g0, uint32_t g1,
+__global__ void __launch_bounds__(kSearchThreads) k_search(SArgs a, uint32_t g0, uint32_t g1, uint32_t chunk,
+                                                           unsigned int* __restrict__ ctr,
                                                            uint32_t* __restrict__ cnt,
                                                            unsigned long long* __restrict__ tests_out,
                                                            const uint64_t* __restrict__ off, uint64_t out_base,
-                                                           uint32_t* __restrict__ out) {
+                                                           uint32_t* __restrict__ out, uint2* __restrict__ masks,
+                                                           const uint64_t* __restrict__ moff) {
     constexpr bool F64 = MODE != kF32;
-    __shared__ float4 sq[kWarps][32];              // {qx, qx, qy, qy}
+    __shared__ uint2 swin[WRITE ? 1 : kWarps][32][kWin];   // count pass: masks of the current window
+    __shared__ ulonglong2 sq[kWarps][32];          // {{qx, qx}, {qy, qy}} packed f32 pairs
     __shared__ double2 sqd[F64 ? kWarps : 1][32];  // exact query coordinates (f64 modes)
     const int lane = threadIdx.x & 31;
     const int w = threadIdx.x >> 5;
     const unsigned lt = (1u << lane) - 1u;
-    const uint32_t wid = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    const uint32_t nw = (gridDim.x * blockDim.x) >> 5;
+    const ulonglong2* __restrict__ xp = (const ulonglong2*)a.xp;
+    if (!WRITE) {
+#pragma unroll
+        for (int kk = 0; kk < kWin; ++kk) swin[WRITE ? 0 : w][lane][kk] = make_uint2(0, 0);
+    }
+    const u64x NE2 = pack2(-a.e2f, -a.e2f);
+    const float band = a.band;
     unsigned long long tests = 0;
-    for (uint32_t gi = g0 + wid; gi < g1; gi += nw) {
+    uint32_t gi = g0 + grab(ctr, chunk, lane), gend = min(gi + chunk, g1);
+    while (gi < g1) {
         const uint32_t qs = __ldg(&a.gstart[gi]);
         const uint32_t c = __ldg(&a.gcell[gi]);
         const uint32_t nq = min((uint32_t)kGroup, __ldg(&a.cstart[c + 1]) - qs);
         __syncwarp();
         if ((uint32_t)lane < nq) {
-            if (MODE != kF64Exact) {
-                const float2 p = a.xf[qs + lane];
-                sq[w][lane] = make_float4(p.x, p.x, p.y, p.y);
-            }
-            if (F64) sqd[F64 ? w : 0][lane] = a.xd[qs + lane];
+            const uint32_t q = qs + lane;
+            const float4 P = a.xp[q >> 1];
+            const float qx = (q & 1) ? P.y : P.x, qy = (q & 1) ? P.w : P.z;
+            sq[w][lane] = make_ulonglong2(pack2(qx, qx), pack2(qy, qy));
+            if (F64) sqd[F64 ? w : 0][lane] = a.xd[q];
         }
         uint32_t my = 0;        // count: this lane's query's count; write: its offset within the group
         uint32_t* gout = nullptr;
         if (WRITE) {
             const uint64_t gb = off[qs];
             gout = out + (gb - out_base);
+            // materialise the group's base pointer so that every store address is one
+            // IMAD.WIDE (32-bit index), not a 64-bit add chain re-derived from out_base
+            asm volatile("mov.b64 %0, %0;" : "+l"(gout));
             if ((uint32_t)lane < nq) my = (uint32_t)(off[qs + lane] - gb);
         }
+        // count pass: the hit masks of chunk k for query i go to masks[moff[gi]/2 + k*nq + i]
+        uint2* gmask = (!WRITE && masks) ? masks + (__ldg(&moff[gi]) >> 1) : nullptr;
+        uint32_t k = 0;
         __syncwarp();
 #pragma unroll 1
         for (int r = 0; r < 3; ++r) {
             const uint2 sp = __ldg(&a.cspan[3 * c + r]);
-            const uint32_t hi = sp.y;
+            const uint32_t lo = sp.x, hi = sp.y;
+            if (lo >= hi) continue;   // empty span: no chunk (the mask layout counts none)
 #pragma unroll 1
-            for (uint32_t c0 = sp.x; c0 < hi; c0 += 64) {
-                const uint32_t j0 = c0 + lane, j1 = c0 + 32 + lane;
-                const bool v0 = j0 < hi, v1 = j1 < hi;
-                float2 p0 = make_float2(kFar, kFar), p1 = make_float2(kFar, kFar);
-                double2 c0d = make_double2(0, 0), c1d = make_double2(0, 0);
-                if (MODE == kF64Exact) {
-                    if (v0) c0d = a.xd[j0];
-                    if (v1) c1d = a.xd[j1];
-                } else {
-                    if (v0) p0 = a.xf[j0];
-                    if (v1) p1 = a.xf[j1];
+            for (uint32_t c0 = lo & ~1u; c0 < hi; c0 += 64, ++k) {
+                uint2 mk = make_uint2(0, 0);   // count pass: lane i keeps query i's masks
+                const uint32_t s0 = c0 + 2 * lane, s1 = s0 + 1;
+                const bool v0 = s0 >= lo && s0 < hi, v1 = s1 >= lo && s1 < hi;
+                ulonglong2 P = make_ulonglong2(0, 0);
+                double2 d0 = make_double2(0, 0), d1 = make_double2(0, 0);
+                if (v0 || v1) {
+                    if (MODE == kF64Exact) {
+                        d0 = a.xd[s0];
+                        d1 = a.xd[s1];
+                    } else {
+                        P = xp[s0 >> 1];
+                    }
                 }
-                const u64x X = pack2(p0.x, p1.x);
-                const u64x Y = pack2(p0.y, p1.y);
-                uint32_t id0 = 0, id1 = 0;
-                if (WRITE) {
-                    if (v0) id0 = __ldg(&a.ids[j0]);
-                    if (v1) id1 = __ldg(&a.ids[j1]);
-                }
-                if (!WRITE) tests += (unsigned long long)nq * min(64u, hi - c0);
+                uint2 id = make_uint2(0, 0);
+                if (WRITE && (v0 || v1)) id = *(const uint2*)(a.ids + s0);
+                if (!WRITE) tests += (unsigned long long)nq * (min(c0 + 64, hi) - max(c0, lo));
 #pragma unroll 2
                 for (uint32_t i = 0; i < nq; ++i) {
-                    float4 q = make_float4(0, 0, 0, 0);
-                    if (MODE != kF64Exact) q = sq[w][i];
-                    double2 qd = make_double2(0, 0);
-                    if (F64) qd = sqd[F64 ? w : 0][i];
-                    bool in0, in1;
-                    test_pair<MODE>(a, q, X, Y, v0, v1, j0, j1, qd, c0d, c1d, in0, in1);
-                    const unsigned m0 = __ballot_sync(FULL, in0);
-                    const unsigned m1 = __ballot_sync(FULL, in1);
-                    const uint32_t n0 = __popc(m0);
-                    if (WRITE) {
-                        const uint32_t b = __shfl_sync(FULL, my, i);
-                        if (in0) gout[b + __popc(m0 & lt)] = id0;
-                        if (in1) gout[b + n0 + __popc(m1 & lt)] = id1;
+                    unsigned m0, m1;
+                    if (MODE == kF64Exact) {
+                        const double2 qd = sqd[F64 ? w : 0][i];
+                        m0 = __ballot_sync(FULL, v0 && pred_f64(qd.x, qd.y, d0.x, d0.y, a.e2d));
+                        m1 = __ballot_sync(FULL, v1 && pred_f64(qd.x, qd.y, d1.x, d1.y, a.e2d));
+                    } else {
+                        const ulonglong2 Q = sq[w][i];
+                        const u64x dx = sub2(Q.x, P.x);
+                        const u64x dy = sub2(Q.y, P.y);
+                        if (MODE == kF64Filter) {
+                            const float2 t = unpack2(fma2(dy, dy, fma2(dx, dx, NE2)));   // (dx^2 - e2) + dy^2
+                            m0 = __ballot_sync(FULL, v0 && t.x < 0.f);
+                            m1 = __ballot_sync(FULL, v1 && t.y < 0.f);
+                            const bool b0 = v0 & (fabsf(t.x) <= band);
+                            const bool b1 = v1 & (fabsf(t.y) <= band);
+                            if (__any_sync(FULL, b0 | b1)) {   // rare: decide these tests in exact f64
+                                const double2 qd = sqd[F64 ? w : 0][i];
+                                bool e0 = false, e1 = false;
+                                if (b0) {
+                                    const double2 p = a.xd[s0];
+                                    e0 = pred_f64(qd.x, qd.y, p.x, p.y, a.e2d);
+                                }
+                                if (b1) {
+                                    const double2 p = a.xd[s1];
+                                    e1 = pred_f64(qd.x, qd.y, p.x, p.y, a.e2d);
+                                }
+                                m0 = (m0 & ~__ballot_sync(FULL, b0)) | __ballot_sync(FULL, e0);
+                                m1 = (m1 & ~__ballot_sync(FULL, b1)) | __ballot_sync(FULL, e1);
+                            }
+                        } else {
+                            // fl(fl(dx^2) + fl(dy^2)).  The sum is two scalar add.rn: ptxas fuses
+                            // mul.rn.f32x2 + add.rn.f32x2 into FFMA2 (observed in SASS, even with
+                            // --fmad=false), which would break the no-FMA contract (reading R2).
+                            const float2 px = unpack2(mul2(dx, dx));
+                            const float2 py = unpack2(mul2(dy, dy));
+                            m0 = __ballot_sync(FULL, v0 && __fadd_rn(px.x, py.x) <= a.e2f);
+                            m1 = __ballot_sync(FULL, v1 && __fadd_rn(px.y, py.y) <= a.e2f);
+                        }
                     }
-                    if ((uint32_t)lane == i) my += n0 + __popc(m1);
+                    if (WRITE) {
+                        // addresses computed by every lane, stores predicated (no branches)
+                        const uint32_t n0 = __popc(m0);
+                        const uint32_t b = __shfl_sync(FULL, my, i);
+                        uint32_t* p0 = gout + (b + __popc(m0 & lt));
+                        uint32_t* p1 = gout + (b + n0 + __popc(m1 & lt));
+                        stg_if(p0, id.x, (m0 >> lane) & 1u);
+                        stg_if(p1, id.y, (m1 >> lane) & 1u);
+                        const uint32_t nn = n0 + __popc(m1);
+                        my += ((uint32_t)lane == i) ? nn : 0u;
+                    } else if ((uint32_t)lane == i) {
+                        mk = make_uint2(m0, m1);
+                    }
+                }
+                if (!WRITE) {
+                    my += __popc(mk.x) + __popc(mk.y);
+                    if (gmask) {
+                        if ((uint32_t)lane < nq) swin[WRITE ? 0 : w][lane][k % kWin] = mk;
+                        if (k % kWin == kWin - 1) flush_window(swin[WRITE ? 0 : w], gmask, k / kWin, nq, lane);
+                    }
                 }
             }
         }
+        if (!WRITE && gmask && (k % kWin) != 0) flush_window(swin[WRITE ? 0 : w], gmask, k / kWin, nq, lane);
         if (!WRITE && (uint32_t)lane < nq) cnt[qs + lane] = my;
+        if (++gi >= gend) {
+            gi = g0 + grab(ctr, chunk, lane);
+            gend = min(gi + chunk, g1);
+        }
     }
     if (!WRITE && tests_out && lane == 0 && tests) atomicAdd(tests_out, tests);
+}
+
+// a8 (mask path): emission only.  The count pass stored every query's hit
+// masks per 64-candidate chunk (windowed layout above); this kernel replays the
+// chunk order without any distance arithmetic.  Per window of kWin chunks the
+// masks are staged in shared memory by cp.async (double-buffered, the next
+// window's copy overlaps this window's stores), then the warp emits query by
+// query: for query i the window's hits are one contiguous run of its CSR
+// segment, written by ballot-free popc prefixes with all 32 lanes (lane j owns
+// candidate pair (2j, 2j+1) of each chunk).  Long per-warp store streams keep
+// L2 lines whole -- interleaving 32 query lists per chunk halved the store rate.
+__device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
+    const uint32_t sa = (uint32_t)__cvta_generic_to_shared(smem);
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(sa), "l"(gmem));
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() {
+    asm volatile("cp.async.wait_group %0;" ::"n"(N));
+}
+
+__global__ void __launch_bounds__(kSearchThreads) k_emit(SArgs a, uint32_t g0, uint32_t g1, uint32_t chunk,
+                                                         unsigned int* __restrict__ ctr,
+                                                         const uint64_t* __restrict__ off, uint64_t out_base,
+                                                         uint32_t* __restrict__ out, const uint2* __restrict__ masks,
+                                                         const uint64_t* __restrict__ moff) {
+    __shared__ uint2 wm[kWarps][2][32][kWin];   // double-buffered window masks [query][chunk]
+    const int lane = threadIdx.x & 31;
+    const int w = threadIdx.x >> 5;
+    const unsigned lt = (1u << lane) - 1u;
+    uint32_t gi = g0 + grab(ctr, chunk, lane), gend = min(gi + chunk, g1);
+    while (gi < g1) {
+        const uint32_t qs = __ldg(&a.gstart[gi]);
+        const uint32_t c = __ldg(&a.gcell[gi]);
+        const uint32_t nq = min((uint32_t)kGroup, __ldg(&a.cstart[c + 1]) - qs);
+        const uint64_t m_a = __ldg(&moff[gi]), m_b = __ldg(&moff[gi + 1]);
+        const uint32_t nwin = (uint32_t)((m_b - m_a) / (2ull * nq * kWin));
+        const uint2* gmask = masks + (m_a >> 1);
+        const uint64_t gb = off[qs];
+        uint32_t* gout = out + (gb - out_base);
+        asm volatile("mov.b64 %0, %0;" : "+l"(gout));
+        uint32_t my = 0;
+        if ((uint32_t)lane < nq) my = (uint32_t)(off[qs + lane] - gb);
+        const uint2 S0 = __ldg(&a.cspan[3 * c]), S1 = __ldg(&a.cspan[3 * c + 1]), S2 = __ldg(&a.cspan[3 * c + 2]);
+        // chunk iterator (same order as the count pass)
+        int r = S0.x < S0.y ? 0 : (S1.x < S1.y ? 1 : 2);   // the own-row span is never empty
+        uint2 sp = r == 0 ? S0 : (r == 1 ? S1 : S2);
+        uint32_t c0 = sp.x & ~1u, hi = sp.y;
+        __syncwarp();   // the previous group's window buffers are no longer read
+        // prefetch window 0: lane i copies its 64-B mask row
+        if ((uint32_t)lane < nq) {
+            const uint4* src = (const uint4*)(gmask + (size_t)lane * kWin);
+#pragma unroll
+            for (int u = 0; u < kWin / 2; ++u) cp_async16(&wm[w][0][lane][2 * u], src + u);
+        }
+        cp_async_commit();
+#pragma unroll 1
+        for (uint32_t v = 0; v < nwin; ++v) {
+            // chunk starts of this window (registers, fully unrolled) and advance the iterator
+            uint32_t cst[kWin];
+#pragma unroll
+            for (int kk = 0; kk < kWin; ++kk) {
+                cst[kk] = c0;
+                if (r < 3) {
+                    c0 += 64;
+                    if (c0 >= hi) {
+                        ++r;
+                        while (r < 3) {
+                            sp = r == 1 ? S1 : S2;
+                            if (sp.x < sp.y) break;
+                            ++r;
+                        }
+                        if (r < 3) {
+                            c0 = sp.x & ~1u;
+                            hi = sp.y;
+                        }
+                    }
+                }
+            }
+            // prefetch window v+1 into the other buffer
+            if (v + 1 < nwin && (uint32_t)lane < nq) {
+                const uint4* src = (const uint4*)(gmask + ((size_t)(v + 1) * nq + lane) * kWin);
+#pragma unroll
+                for (int u = 0; u < kWin / 2; ++u) cp_async16(&wm[w][(v + 1) & 1][lane][2 * u], src + u);
+            }
+            cp_async_commit();
+            cp_async_wait<1>();
+            __syncwarp();
+            uint2 (*M)[kWin] = wm[w][v & 1];
+#pragma unroll 1
+            for (uint32_t i = 0; i < nq; ++i) {
+                uint32_t b = __shfl_sync(FULL, my, i);
+#pragma unroll
+                for (int kk = 0; kk < kWin; ++kk) {
+                    const uint2 m = M[i][kk];   // broadcast; unused window slots are never set (zero-filled)
+                    const uint32_t n0 = __popc(m.x), nn = n0 + __popc(m.y);
+                    if (nn) {
+                        const bool h0 = (m.x >> lane) & 1u, h1 = (m.y >> lane) & 1u;
+                        uint2 id = make_uint2(0, 0);
+                        if (h0 | h1) id = __ldg((const uint2*)(a.ids + cst[kk] + 2 * lane));
+                        stg_if(gout + (b + __popc(m.x & lt)), id.x, h0);
+                        stg_if(gout + (b + n0 + __popc(m.y & lt)), id.y, h1);
+                        b += nn;
+                    }
+                }
+            }
+            if ((uint32_t)lane < nq) {
+#pragma unroll
+                for (int kk = 0; kk < kWin; ++kk) my += __popc(M[lane][kk].x) + __popc(M[lane][kk].y);
+            }
+            __syncwarp();   // buffer v&1 is refilled by the prefetch of window v+2
+        }
+        cp_async_wait<0>();
+        if (++gi >= gend) {
+            gi = g0 + grab(ctr, chunk, lane);
+            gend = min(gi + chunk, g1);
+        }
+    }
+}
+
+// Mask-table layout: words of group g = 2 * nq * (number of 64-candidate chunks of its 3 spans)
+__global__ void __launch_bounds__(256) k_mask_words(SArgs a, uint64_t ng, uint32_t* __restrict__ words) {
+    for (uint64_t g = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; g < ng;
+         g += (uint64_t)gridDim.x * blockDim.x) {
+        const uint32_t qs = a.gstart[g], c = a.gcell[g];
+        const uint32_t nq = min((uint32_t)kGroup, a.cstart[c + 1] - qs);
+        uint32_t ch = 0;
+        for (int r = 0; r < 3; ++r) {
+            const uint2 sp = a.cspan[3 * c + r];
+            if (sp.y > sp.x) ch += (sp.y - (sp.x & ~1u) + 63) / 64;
+        }
+        words[g] = 2 * nq * kWin * ((ch + kWin - 1) / kWin);
+    }
 }
 
 // a5: warp per sampled query (the paper's estimator kernel),
@@ -260,11 +460,11 @@ __global__ void __launch_bounds__(256) k_sample_count(SArgs a, uint64_t nne, uin
                 }
             }
         } else {
-            const float2 q = a.xf[s];
+            const float2 q = a.xs[s];
             for (int r = 0; r < 3; ++r) {
                 const uint2 sp = a.cspan[3 * c + r];
                 for (uint32_t k = sp.x + lane; k < sp.y; k += 32) {
-                    const float2 p = a.xf[k];
+                    const float2 p = a.xs[k];
                     cntv += pred_f32(q.x, q.y, p.x, p.y, a.e2f) ? 1u : 0u;
                 }
             }
@@ -336,7 +536,8 @@ __global__ void __launch_bounds__(256) k_scatter_rows(const uint32_t* __restrict
 
 SArgs args_of(const DevGrid& g) {
     SArgs a;
-    a.xf = g.xf;
+    a.xp = g.xp;
+    a.xs = (const float2*)g.xy_s;
     a.xd = (const double2*)g.xy_s;
     a.ids = g.ids;
     a.cstart = g.cstart;
@@ -349,29 +550,53 @@ SArgs args_of(const DevGrid& g) {
     return a;
 }
 
-unsigned search_grid(uint64_t ngroups) {
-    uint64_t ctas = (ngroups + kWarps - 1) / kWarps;
-    const uint64_t cap = 148ull * 8ull;   // 8 CTAs x 8 warps = 64 warps per SM
-    if (ctas > cap) ctas = cap;
-    return (unsigned)(ctas ? ctas : 1);
+// One wave of resident CTAs; warps grab `chunk` groups at a time (~32 grabs
+// per resident warp keeps the tail short while bounding counter atomics).
+template <typename K>
+void launch_groups(K kern, int& blocks_per_sm, uint64_t ng, uint32_t& chunk, unsigned& ctas) {
+    if (!blocks_per_sm) {
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks_per_sm, kern, kSearchThreads, 0);
+        if (blocks_per_sm < 1) blocks_per_sm = 1;
+    }
+    int dev = 0, nsm = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    const uint64_t wave_warps = (uint64_t)nsm * blocks_per_sm * kWarps;
+    ctas = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>((ng + kWarps - 1) / kWarps, (uint64_t)nsm * blocks_per_sm));
+    chunk = (uint32_t)std::max<uint64_t>(1, ng / (wave_warps * 32));
+}
+
+template <int MODE, bool WRITE>
+void launch_mode(const SArgs& a, uint64_t g0, uint64_t g1, unsigned int* ctr, uint32_t* cnt,
+                 unsigned long long* tests, const uint64_t* off, uint64_t out_base, uint32_t* out, uint2* masks,
+                 const uint64_t* moff, cudaStream_t s) {
+    static int bps = 0;
+    uint32_t chunk;
+    unsigned ctas;
+    launch_groups(k_search<MODE, WRITE>, bps, g1 - g0, chunk, ctas);
+    k_search<MODE, WRITE><<<ctas, kSearchThreads, 0, s>>>(a, (uint32_t)g0, (uint32_t)g1, chunk, ctr, cnt, tests, off,
+                                                          out_base, out, masks, moff);
+}
+
+int mode_of(const DevGrid& g, bool force_exact) {
+    return g.dtype == HDB_F32 ? kF32 : (g.filter && !force_exact ? kF64Filter : kF64Exact);
 }
 
 template <bool WRITE>
 void launch_search(const DevGrid& g, uint64_t g0, uint64_t g1, uint32_t* cnt, unsigned long long* tests,
-                   const uint64_t* off, uint64_t out_base, uint32_t* out, bool force_exact, cudaStream_t s) {
+                   const uint64_t* off, uint64_t out_base, uint32_t* out, bool force_exact, int slot, uint2* masks,
+                   cudaStream_t s) {
     if (g1 <= g0) return;
-    const unsigned grid = search_grid(g1 - g0);
     const SArgs a = args_of(g);
-    const int mode = g.dtype == HDB_F32 ? kF32 : (g.filter && !force_exact ? kF64Filter : kF64Exact);
+    unsigned int* ctr = g.counters + (slot % kCounterSlots);
+    cudaMemsetAsync(ctr, 0, sizeof(unsigned int), s);
+    const int mode = mode_of(g, force_exact);
     if (mode == kF64Filter)
-        k_search<kF64Filter, WRITE><<<grid, kSearchThreads, 0, s>>>(a, (uint32_t)g0, (uint32_t)g1, cnt, tests, off,
-                                                                     out_base, out);
+        launch_mode<kF64Filter, WRITE>(a, g0, g1, ctr, cnt, tests, off, out_base, out, masks, g.moff, s);
     else if (mode == kF64Exact)
-        k_search<kF64Exact, WRITE><<<grid, kSearchThreads, 0, s>>>(a, (uint32_t)g0, (uint32_t)g1, cnt, tests, off,
-                                                                    out_base, out);
+        launch_mode<kF64Exact, WRITE>(a, g0, g1, ctr, cnt, tests, off, out_base, out, masks, g.moff, s);
     else
-        k_search<kF32, WRITE><<<grid, kSearchThreads, 0, s>>>(a, (uint32_t)g0, (uint32_t)g1, cnt, tests, off,
-                                                               out_base, out);
+        launch_mode<kF32, WRITE>(a, g0, g1, ctr, cnt, tests, off, out_base, out, masks, g.moff, s);
     ++g_kernel_launches;
 }
 
@@ -393,13 +618,35 @@ void launch_sample_count(const DevGrid& g, uint64_t stride, uint64_t n_sample, u
 
 // variant (hdb_opts.search_kernel): 0 = default, 1 = force the exact-f64-only kernel
 void launch_count(const DevGrid& g, uint64_t g0, uint64_t g1, uint32_t* cnt, unsigned long long* tests,
-                  int variant, cudaStream_t s) {
-    launch_search<false>(g, g0, g1, cnt, tests, nullptr, 0, nullptr, variant == 1, s);
+                  int variant, int slot, uint2* masks, cudaStream_t s) {
+    launch_search<false>(g, g0, g1, cnt, tests, nullptr, 0, nullptr, variant == 1, slot, masks, s);
 }
 
+// masks != null: emission from the count pass's hit masks (k_emit); else the
+// write pass recomputes the distance tests (k_search<WRITE>).
 void launch_write(const DevGrid& g, uint64_t g0, uint64_t g1, const uint64_t* off, uint64_t out_base,
-                  uint32_t* out, int variant, cudaStream_t s) {
-    launch_search<true>(g, g0, g1, nullptr, nullptr, off, out_base, out, variant == 1, s);
+                  uint32_t* out, int variant, int slot, const uint2* masks, cudaStream_t s) {
+    if (!masks) {
+        launch_search<true>(g, g0, g1, nullptr, nullptr, off, out_base, out, variant == 1, slot, nullptr, s);
+        return;
+    }
+    if (g1 <= g0) return;
+    unsigned int* ctr = g.counters + (slot % kCounterSlots);
+    cudaMemsetAsync(ctr, 0, sizeof(unsigned int), s);
+    static int bps = 0;
+    uint32_t chunk;
+    unsigned ctas;
+    launch_groups(k_emit, bps, g1 - g0, chunk, ctas);
+    k_emit<<<ctas, kSearchThreads, 0, s>>>(args_of(g), (uint32_t)g0, (uint32_t)g1, chunk, ctr, off, out_base, out,
+                                           masks, g.moff);
+    ++g_kernel_launches;
+}
+
+void launch_mask_words(const DevGrid& g, uint32_t* words, cudaStream_t s) {
+    if (g.n_groups == 0) return;
+    unsigned blocks = (unsigned)std::min<uint64_t>((g.n_groups + 255) / 256, 148 * 16);
+    k_mask_words<<<blocks, 256, 0, s>>>(args_of(g), g.n_groups, words);
+    ++g_kernel_launches;
 }
 
 void launch_batch_cuts(const uint32_t* gstart, const uint64_t* off, uint64_t g0, uint64_t g1, uint32_t nb,

@@ -410,10 +410,12 @@ def test_c3_full_size_sampled_rows(torch_cuda):
 
 
 def test_exact_f64_kernel_variant(torch_cuda):
-    """search_kernel=1 forces the exact-f64-only kernel; both kernels must equal the oracle."""
+    """search_kernel=1 forces the exact-f64-only kernel, 2 the write pass that
+    recomputes the tests instead of replaying stored hit masks; all must equal
+    the oracle, host- and device-resident."""
     xy = datagen.subsample(datagen.tec_like(), 30_000, seed=12)
     for eps in (0.15, 0.45):
-        for k in (0, 1):
+        for k in (0, 1, 2):
             b, c, v, _, _ = lib_table(xy, eps, search_kernel=k)
             assert_table_equal(xy, eps, b, c, v)
 

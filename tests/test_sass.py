@@ -1,0 +1,60 @@
+"""SASS-level checks of the exact-arithmetic contract (reading R2, no FMA in
+the predicate): no DFMA anywhere in libhdb; the f32-mode search kernels
+contain no FFMA/FFMA2 (ptxas fuses mul.rn.f32x2 + add.rn.f32x2 otherwise);
+the f64 filter kernels use FFMA2 (the filter is allowed to, its error bound
+covers it); the exact-f64 kernels none.  CPU only (cuobjdump)."""
+import os
+import re
+import shutil
+import subprocess
+
+import pytest
+
+from paper_conf_ipps_gowanlockrblp17_b200 import LIB_PATH
+
+CUOBJDUMP = shutil.which("cuobjdump") or "/usr/local/cuda/bin/cuobjdump"
+
+
+@pytest.fixture(scope="module")
+def sass():
+    if not os.path.exists(CUOBJDUMP):
+        pytest.skip("cuobjdump not available")
+    out = subprocess.run([CUOBJDUMP, "-sass", LIB_PATH], capture_output=True, text=True, check=True).stdout
+    funcs = {}
+    for chunk in re.split(r"\n\s*Function : ", out)[1:]:
+        name, body = chunk.split("\n", 1)
+        funcs[name.strip()] = body
+    assert funcs
+    return funcs
+
+
+def _mode_kernels(sass, mode):
+    return {k: v for k, v in sass.items() if re.search(rf"k_searchILi{mode}ELb[01]E", k)}
+
+
+def test_sm100a_code_present(sass):
+    out = subprocess.run([CUOBJDUMP, "-lelf", LIB_PATH], capture_output=True, text=True).stdout
+    assert "sm_100a" in out
+
+
+def test_no_dfma_anywhere(sass):
+    for name, body in sass.items():
+        assert "DFMA" not in body, name
+
+
+def test_f32_mode_has_no_ffma(sass):
+    ks = _mode_kernels(sass, 0)
+    assert len(ks) == 2
+    for name, body in ks.items():
+        assert "FFMA" not in body, name          # neither FFMA nor FFMA2
+        assert "FMUL2" in body and "FADD2" in body, name
+
+
+def test_filter_and_exact_kernels(sass):
+    filt = _mode_kernels(sass, 1)
+    exact = _mode_kernels(sass, 2)
+    assert len(filt) == 2 and len(exact) == 2
+    for name, body in filt.items():
+        assert "FFMA2" in body and "DMUL" in body, name   # f32 filter + exact f64 fallback
+    for name, body in exact.items():
+        assert "FFMA" not in body and "DMUL" in body, name
