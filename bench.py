@@ -107,7 +107,7 @@ def dist_env():
     return ws, rank, local
 
 
-def cpu_baseline_run(xy, eps, budget_s=12.0, rows=None):
+def cpu_baseline_run(xy, eps, budget_s=12.0, rows=None, dtype="f64"):
     """The oracle as it stands (brute-force rows, OpenMP) on a bounded sample."""
     import oracle
     n = xy.shape[0]
@@ -115,12 +115,12 @@ def cpu_baseline_run(xy, eps, budget_s=12.0, rows=None):
         # calibrate on a small sample, then size the sample to ~budget_s
         probe = np.arange(0, n, max(1, n // 64))[:64]
         t0 = time.perf_counter()
-        oracle.eps_join_rowhash(xy, eps, probe)
+        oracle.eps_join_rowhash(xy, eps, probe, dtype=dtype)
         dt = max(time.perf_counter() - t0, 1e-3)
         m = int(min(n, max(64, 64 * budget_s / dt)))
         rows = np.linspace(0, n - 1, m).astype(np.int64)
     t0 = time.perf_counter()
-    cnt, _ = oracle.eps_join_rowhash(xy, eps, rows)
+    cnt, _ = oracle.eps_join_rowhash(xy, eps, rows, dtype=dtype)
     dt = time.perf_counter() - t0
     pairs = int(cnt.sum())
     return dict(value=pairs / dt, unit="pairs/s", cores=oracle.threads(), kind="oracle",
@@ -204,7 +204,7 @@ def main():
     if ws > 1:
         dist.barrier()
     torch.cuda.synchronize()
-    write_ms, pairs_local, launches = [], 0, 0
+    write_ms, count_ms, pairs_local, launches = [], [], 0, 0
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     l0 = hdb.hdb_kernel_launches()
     with ClockSampler(local) as clk:
@@ -212,30 +212,30 @@ def main():
         for _ in range(args.steps):
             st, v = step()
             write_ms.append(st["ms_write_kernel"])
+            count_ms.append(st["ms_count"])
             pairs_local += v.npairs
         ev1.record(stream)
         torch.cuda.synchronize()
     launches = hdb.hdb_kernel_launches() - l0
     ms = ev0.elapsed_time(ev1)
     if ws > 1:
+        from paper_conf_ipps_gowanlockrblp17_b200 import dist as hdist
         t = torch.tensor([ms], device=dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         ms = float(t.item())
-        # the "final gather of counts": per-shard pair totals
-        c = torch.tensor([pairs_local], dtype=torch.int64, device=dev)
-        allc = [torch.zeros_like(c) for _ in range(ws)]
-        dist.all_gather(allc, c)
-        pairs_total = int(sum(int(x.item()) for x in allc))
+        # the path's one exchange: the gather of per-shard pair counts
+        _, pairs_total = hdist.gather_pair_counts(pairs_local, device=dev)
     else:
         pairs_total = pairs_local
     P = pairs_total // max(args.steps, 1)
     value = pairs_total / (ms / 1000.0)
 
-    # roofline of the dominant kernel (the neighbour write kernel, a8)
+    # roofline of the dominant kernel: the neighbour write kernel (a8, k_emit),
+    # HBM-write bound.  Algorithmic bytes per launch:
+    # 4 B per pair written + 12 B per query (uint64 offset + uint32 id map).
     hbm, peak_kind = load_peaks()
-    esz = 16 if args.dtype == "f64" else 8
     n_shard = (v.end_query - v.first_query) if ws > 1 else n
-    alg_bytes = 4 * v.npairs + (esz + 4 + 8) * n_shard   # 4 B/pair + sorted xy, id map, offsets per query
+    alg_bytes = 4 * v.npairs + 12 * n_shard
     wms = float(np.mean(write_ms))
     achieved = alg_bytes / (wms / 1000.0) / 1e9
     traffic = None
@@ -243,6 +243,10 @@ def main():
     if os.path.exists(tp):
         with open(tp) as f:
             traffic = json.load(f).get(f"{args.workload}-{args.dtype}-k{args.kernel}")
+    # whole-step view: SURVEY 8(d) B_alg = 4P + 64n + 8C (f64) over the step time
+    esz = 16 if args.dtype == "f64" else 8
+    b_step = 4 * P + (4 * esz + 32) * n + 8 * st["n_nonempty"]
+    cms = float(np.mean(count_ms))
 
     line = {"metric": "eps_neighbor_pairs_per_sec", "value": value, "unit": "pairs/s", "n_gpus": ws,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms / args.steps,
@@ -255,7 +259,12 @@ def main():
             "gpu_launches": launches,
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
                          "frac": achieved / hbm, "traffic": traffic, "peak_kind": peak_kind,
-                         "kernel": "k_search<write>", "kernel_ms": wms, "alg_bytes": alg_bytes},
+                         "kernel": "k_emit (neighbour write, a8)", "kernel_ms": wms, "alg_bytes": alg_bytes},
+            "count_kernel": {"bound": "alu", "kernel": "k_search (count + hit masks, a6)", "ms": cms,
+                             "tests": st["candidate_tests"],
+                             "tests_per_s": st["candidate_tests"] / (cms / 1e3) if cms > 0 else None},
+            "step_roofline": {"alg_bytes": b_step, "achieved_gbs": b_step / (ms / args.steps / 1e3) / 1e9,
+                              "frac": b_step / (ms / args.steps / 1e3) / 1e9 / hbm},
             "clocks": clk.summary(),
             "stats": {k: st[k] for k in ("n_nonempty", "n_groups", "candidate_tests", "ms_grid", "ms_sample",
                                          "ms_count", "ms_scan", "ms_write_kernel", "kernel_launches")}}
@@ -292,8 +301,7 @@ def main():
     else:
         line["e2e"] = None
     if rank == 0 and not args.no_cpu_baseline:
-        line["cpu_baseline"], _ = cpu_baseline_run(xy_np.astype(np.float64) if args.dtype == "f64" else xy_np,
-                                                   eps) if args.dtype == "f64" else (None, None)
+        line["cpu_baseline"], _ = cpu_baseline_run(xy_np, eps, dtype=args.dtype)
     hdb.hdb_ctx_destroy(ctx)
     if rank == 0:
         print(json.dumps(line), flush=True)

@@ -318,7 +318,8 @@ __global__ void __launch_bounds__(kSearchThreads) k_emit(SArgs a, uint32_t g0, u
                                                          const uint64_t* __restrict__ off, uint64_t out_base,
                                                          uint32_t* __restrict__ out, const uint2* __restrict__ masks,
                                                          const uint64_t* __restrict__ moff) {
-    __shared__ uint2 wm[kWarps][2][32][kWin];   // double-buffered window masks [query][chunk]
+    __shared__ uint2 raw[kWarps][32][kWin];   // cp.async landing buffer (next window's masks)
+    __shared__ uint4 wq[kWarps][32][kWin];    // current window: {m0, m1, pos0, pos1} per (query, chunk)
     const int lane = threadIdx.x & 31;
     const int w = threadIdx.x >> 5;
     const unsigned lt = (1u << lane) - 1u;
@@ -333,29 +334,29 @@ __global__ void __launch_bounds__(kSearchThreads) k_emit(SArgs a, uint32_t g0, u
         const uint64_t gb = off[qs];
         uint32_t* gout = out + (gb - out_base);
         asm volatile("mov.b64 %0, %0;" : "+l"(gout));
-        uint32_t my = 0;
+        uint32_t my = 0;   // lane i: output cursor of query i within the group
         if ((uint32_t)lane < nq) my = (uint32_t)(off[qs + lane] - gb);
         const uint2 S0 = __ldg(&a.cspan[3 * c]), S1 = __ldg(&a.cspan[3 * c + 1]), S2 = __ldg(&a.cspan[3 * c + 2]);
         // chunk iterator (same order as the count pass)
         int r = S0.x < S0.y ? 0 : (S1.x < S1.y ? 1 : 2);   // the own-row span is never empty
         uint2 sp = r == 0 ? S0 : (r == 1 ? S1 : S2);
         uint32_t c0 = sp.x & ~1u, hi = sp.y;
-        __syncwarp();   // the previous group's window buffers are no longer read
-        // prefetch window 0: lane i copies its 64-B mask row
-        if ((uint32_t)lane < nq) {
+        __syncwarp();   // the previous group's buffers are no longer read
+        if ((uint32_t)lane < nq) {   // prefetch window 0: lane i copies its 64-B mask row
             const uint4* src = (const uint4*)(gmask + (size_t)lane * kWin);
 #pragma unroll
-            for (int u = 0; u < kWin / 2; ++u) cp_async16(&wm[w][0][lane][2 * u], src + u);
+            for (int u = 0; u < kWin / 2; ++u) cp_async16(&raw[w][lane][2 * u], src + u);
         }
         cp_async_commit();
 #pragma unroll 1
         for (uint32_t v = 0; v < nwin; ++v) {
-            // chunk starts of this window (registers, fully unrolled) and advance the iterator
-            uint32_t cst[kWin];
+            // this window's candidate ids: lane j holds pair (2j, 2j+1) of each chunk
+            uint2 ids[kWin];
 #pragma unroll
             for (int kk = 0; kk < kWin; ++kk) {
-                cst[kk] = c0;
+                ids[kk] = make_uint2(0, 0);
                 if (r < 3) {
+                    if (c0 + 2 * lane < hi) ids[kk] = __ldg((const uint2*)(a.ids + c0 + 2 * lane));
                     c0 += 64;
                     if (c0 >= hi) {
                         ++r;
@@ -371,38 +372,37 @@ __global__ void __launch_bounds__(kSearchThreads) k_emit(SArgs a, uint32_t g0, u
                     }
                 }
             }
-            // prefetch window v+1 into the other buffer
+            cp_async_wait<0>();
+            __syncwarp();
+            // lane i turns its row of masks into output positions (all queries in parallel)
+            if ((uint32_t)lane < nq) {
+#pragma unroll
+                for (int kk = 0; kk < kWin; ++kk) {
+                    const uint2 m = raw[w][lane][kk];
+                    const uint32_t p0 = my;
+                    my += __popc(m.x);
+                    wq[w][lane][kk] = make_uint4(m.x, m.y, p0, my);
+                    my += __popc(m.y);
+                }
+            }
+            __syncwarp();
+            // prefetch the next window's masks into the landing buffer (overlaps the stores)
             if (v + 1 < nwin && (uint32_t)lane < nq) {
                 const uint4* src = (const uint4*)(gmask + ((size_t)(v + 1) * nq + lane) * kWin);
 #pragma unroll
-                for (int u = 0; u < kWin / 2; ++u) cp_async16(&wm[w][(v + 1) & 1][lane][2 * u], src + u);
+                for (int u = 0; u < kWin / 2; ++u) cp_async16(&raw[w][lane][2 * u], src + u);
             }
             cp_async_commit();
-            cp_async_wait<1>();
-            __syncwarp();
-            uint2 (*M)[kWin] = wm[w][v & 1];
 #pragma unroll 1
             for (uint32_t i = 0; i < nq; ++i) {
-                uint32_t b = __shfl_sync(FULL, my, i);
 #pragma unroll
                 for (int kk = 0; kk < kWin; ++kk) {
-                    const uint2 m = M[i][kk];   // broadcast; unused window slots are never set (zero-filled)
-                    const uint32_t n0 = __popc(m.x), nn = n0 + __popc(m.y);
-                    if (nn) {
-                        const bool h0 = (m.x >> lane) & 1u, h1 = (m.y >> lane) & 1u;
-                        uint2 id = make_uint2(0, 0);
-                        if (h0 | h1) id = __ldg((const uint2*)(a.ids + cst[kk] + 2 * lane));
-                        stg_if(gout + (b + __popc(m.x & lt)), id.x, h0);
-                        stg_if(gout + (b + n0 + __popc(m.y & lt)), id.y, h1);
-                        b += nn;
-                    }
+                    const uint4 e = wq[w][i][kk];   // broadcast
+                    stg_if(gout + (e.z + __popc(e.x & lt)), ids[kk].x, (e.x >> lane) & 1u);
+                    stg_if(gout + (e.w + __popc(e.y & lt)), ids[kk].y, (e.y >> lane) & 1u);
                 }
             }
-            if ((uint32_t)lane < nq) {
-#pragma unroll
-                for (int kk = 0; kk < kWin; ++kk) my += __popc(M[lane][kk].x) + __popc(M[lane][kk].y);
-            }
-            __syncwarp();   // buffer v&1 is refilled by the prefetch of window v+2
+            __syncwarp();   // wq is rewritten for the next window
         }
         cp_async_wait<0>();
         if (++gi >= gend) {
