@@ -220,40 +220,63 @@ PtrInfo classify(const void* p) {
     return r;
 }
 
-// f64 mode: bound on |t_f32 - (d2_f64 - e2_f64)| for the search kernel's f32
+// f64 mode: bound on |t_f32 - (d2_f64 - e2_f64)| for the search kernels' f32
 // filter.  Filter coordinates are X = fl32(fl64(x - o))
-// with o the bbox centre; every candidate lies in the 3x3 stencil, so
-// |x_p - x_q| < Dmax = 2w.  With u = 2^-24:
-//   E     = R (u + 2^-52)                    (|X - (x - o)|, R = max |fl64(x - o)|)
+// for an origin o with |x - o| <= R; every candidate lies in the 3x3 stencil,
+// so |x_p - x_q| < Dmax = 2w.  With u = 2^-24:
+//   E     = R (u + 2^-52)                    (|X - (x - o)|)
 //   delta = 2E + (Dmax + 2E) u               (|fl32(X_p - X_q) - (x_p - x_q)|)
 //   |t - S| <= 2 delta (2 Dmax + delta)      (the two squares)
 //            + u (e2 + (Dmax^2 + e2) + (2 Dmax^2 + e2)) (1 + 2^-20)   (e2 rounding, 2 fma roundings)
 //            + 2^-49 Dmax^2                  (the f64 predicate's own rounding)
-// and the kernel uses band = 2x that bound (rounded up): |t| > band => sign(t)
-// is the exact f64 decision.  The filter is disabled (exact f64 kernel) when
-// float overflow is possible or the band would cover a large part of eps^2.
+// and the kernels use band = 2x that bound (rounded up): |t| > band => sign(t)
+// is the exact f64 decision.  Two origins are used:
+//   * count pass (k_count): o = the group's first query, R = Dmax (local, tiny band,
+//     so band tests are detected per chunk, ~1e-3 of chunks);
+//   * recompute write variant: o = bbox centre, R = bbox half-extent.
+// A filter is disabled (exact f64 kernel) when float overflow is possible or its
+// band would cover a large part of eps^2.
+static double filter_band(double R, double Dmax, double e2) {
+    const double u = 0x1p-24;
+    const double E = R * (u + 0x1p-52);
+    const double delta = 2 * E + (Dmax + 2 * E) * u;
+    const double bound = 2 * delta * (2 * Dmax + delta) + u * (3 * e2 + 3 * Dmax * Dmax) * (1 + 0x1p-20) +
+                         0x1p-49 * Dmax * Dmax;
+    return 2.0 * bound;
+}
+
+static float round_up_f(double v) {
+    float f = (float)v;
+    if ((double)f < v) f = std::nextafter(f, INFINITY);
+    return f;
+}
+
 void set_filter_bound(DevGrid& g) {
-    g.filter = false;
-    g.band = 0;
+    g.filter = g.filter_l = false;
+    g.band = g.band_l = 0;
+    g.nb2_l = 0;
     if (g.dtype != HDB_F64) return;
     g.ox = 0.5 * g.xmin + 0.5 * g.xmax;
     g.oy = 0.5 * g.ymin + 0.5 * g.ymax;
     const double R = std::max(std::max(std::fabs(g.xmax - g.ox), std::fabs(g.xmin - g.ox)),
                               std::max(std::fabs(g.ymax - g.oy), std::fabs(g.ymin - g.oy)));
-    const double u = 0x1p-24;
     const double Dmax = 2.0 * g.w * (1.0 + 0x1p-18);   // cell rounding: <= 2^-21 cell widths
-    const double E = R * (u + 0x1p-52);
-    const double delta = 2 * E + (Dmax + 2 * E) * u;
     const double e2 = g.e2_d;
-    const double bound = 2 * delta * (2 * Dmax + delta) + u * (3 * e2 + 3 * Dmax * Dmax) * (1 + 0x1p-20) +
-                         0x1p-49 * Dmax * Dmax;
-    const double band = 2.0 * bound;
     g.e2_f = (float)e2;
-    if (!(R < 1e15) || !(Dmax < 1e15) || !(e2 > 1e-30) || !(band < 0.25 * e2)) return;
-    float bf = (float)band;
-    if ((double)bf < band) bf = std::nextafter(bf, INFINITY);
-    g.band = bf;
-    g.filter = true;
+    if (!(Dmax < 1e15) || !(e2 > 1e-30)) return;
+    const double band = filter_band(R, Dmax, e2);
+    if (R < 1e15 && band < 0.25 * e2) {
+        g.band = round_up_f(band);
+        g.filter = true;
+    }
+    const double band_l = filter_band(Dmax, Dmax, e2);
+    if (band_l < 0.25 * e2) {
+        // flag test in the kernel: fma(t, t, -B^2) < 0 with B = band_l (1 + 2^-20) covers |t| <= band_l
+        const double B = band_l * (1.0 + 0x1p-20);
+        g.band_l = round_up_f(band_l);
+        g.nb2_l = -round_up_f(B * B);
+        g.filter_l = true;
+    }
 }
 
 void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t n, hdb_dtype dt, double eps,

@@ -50,8 +50,11 @@ struct DevGrid {
     double eps = 0, w = 0, inv_w = 0;
     double e2_d = 0;     // fl(eps*eps) in f64
     float e2_f = 0;      // fl(eps_f*eps_f) in f32 (f32 mode) / fl32(e2_d) (f64 filter)
-    float band = 0;      // f64 mode: |t| <= band => decide in exact f64
-    bool filter = false; // f64 mode with a useful f32 filter
+    float band = 0;      // f64 mode, bbox-centre filter: |t| <= band => decide in exact f64
+    bool filter = false; // f64 mode: bbox-centre filter usable (recompute write variant)
+    float band_l = 0;    // f64 mode, group-local filter (count pass)
+    float nb2_l = 0;     //   -(band_l (1 + 2^-20))^2, rounded away from zero
+    bool filter_l = false;
     double xmin = 0, ymin = 0, xmax = 0, ymax = 0;
     double ox = 0, oy = 0;  // f64 mode: origin of the f32 filter coordinates
     uint32_t nx = 1, ny = 1;

@@ -50,7 +50,9 @@ struct SArgs {
     const uint32_t* gstart;
     const uint32_t* gcell;
     float e2f;             // f32 mode: fl32(eps^2); f64 mode: fl32(e2_d)
-    float band;            // f64 mode: decide in exact f64 when |t| <= band
+    float band;            // f64 mode, bbox-centre filter: decide in exact f64 when |t| <= band
+    float band_l;          // f64 mode, group-local filter (count pass)
+    float nb2_l;           //   -(band_l (1 + 2^-20))^2
     double e2d;            // fl64(eps^2)
 };
 
@@ -128,14 +130,18 @@ __device__ __forceinline__ uint32_t grab(unsigned int* ctr, uint32_t chunk, int 
 // ~kWin * 27 consecutive ids per query (long sequential store streams).
 constexpr int kWin = 8;
 
-__device__ __forceinline__ void flush_window(uint2 (*swin)[kWin], uint2* gmask, uint32_t v, uint32_t nq,
+constexpr int kWinPad = kWin + 1;   // padded smem rows: 72-B stride, conflict-free per-lane access
+
+__device__ __forceinline__ void flush_window(uint2 (*swin)[kWinPad], uint2* gmask, uint32_t v, uint32_t nq,
                                              int lane) {
     __syncwarp();
     if ((uint32_t)lane < nq) {
-        const uint4* src = (const uint4*)swin[lane];
         uint4* dst = (uint4*)(gmask + ((size_t)v * nq + lane) * kWin);
 #pragma unroll
-        for (int u = 0; u < kWin / 2; ++u) dst[u] = src[u];
+        for (int u = 0; u < kWin / 2; ++u) {
+            const uint2 a = swin[lane][2 * u], b = swin[lane][2 * u + 1];
+            dst[u] = make_uint4(a.x, a.y, b.x, b.y);
+        }
     }
     __syncwarp();
 #pragma unroll
@@ -143,7 +149,162 @@ __device__ __forceinline__ void flush_window(uint2 (*swin)[kWin], uint2* gmask, 
     __syncwarp();
 }
 
-// a6 / a8: warp per query group; lane j holds the candidate PAIR (2k, 2k+1)
+// a6: the count pass.  Warp per query group; lane j holds the candidate PAIR
+// (2k, 2k+1) of a 64-candidate chunk of the group's row spans (packed f32x2
+// operands X = {x0, x1}, Y = {y0, y1}); every query of the group (broadcast
+// from shared memory) is tested against the pair with FADD2/FFMA2, two
+// ballots give the chunk's hit masks (lane 0 stores them to the window
+// buffer), and at the end of the chunk lane i adds query i's popcounts.
+// f64 mode: coordinates relative to the group's first query (|x - o| < 2w),
+// so the f32 error band is ~1e-6 of eps^2; the band flag is accumulated per
+// lane with one LOP3 (sign bit of fma(t, t, -B^2)) and checked once per chunk;
+// the rare flagged chunk is replayed with the band tests in exact f64.
+// Invalid candidate slots carry far coordinates (t = +inf): never hits, never flagged.
+constexpr float kFarF = 1e30f;
+constexpr double kFarD = 1e300;
+
+template <int MODE>
+__global__ void __launch_bounds__(kSearchThreads) k_count(SArgs a, uint32_t g0, uint32_t g1, uint32_t chunk,
+                                                          unsigned int* __restrict__ ctr, uint32_t* __restrict__ cnt,
+                                                          unsigned long long* __restrict__ tests_out,
+                                                          uint2* __restrict__ masks, const uint64_t* __restrict__ moff) {
+    constexpr bool F64 = MODE != kF32;
+    __shared__ uint2 swin[kWarps][32][kWinPad];   // masks of the current window [query][chunk]
+    __shared__ ulonglong2 sq[kWarps][32];           // {{qx, qx}, {qy, qy}} packed f32 pairs
+    __shared__ double2 sqd[F64 ? kWarps : 1][32];   // exact query coordinates (f64 modes)
+    const int lane = threadIdx.x & 31;
+    const int w = threadIdx.x >> 5;
+    const ulonglong2* __restrict__ xp = (const ulonglong2*)a.xp;
+#pragma unroll
+    for (int kk = 0; kk < kWin; ++kk) swin[w][lane][kk] = make_uint2(0, 0);
+    const u64x NE2 = pack2(-a.e2f, -a.e2f);
+    const u64x NB2 = pack2(a.nb2_l, a.nb2_l);
+    unsigned long long tests = 0;
+    uint32_t gi = g0 + grab(ctr, chunk, lane), gend = min(gi + chunk, g1);
+    while (gi < g1) {
+        const uint32_t qs = __ldg(&a.gstart[gi]);
+        const uint32_t c = __ldg(&a.gcell[gi]);
+        const uint32_t nq = min((uint32_t)kGroup, __ldg(&a.cstart[c + 1]) - qs);
+        double2 o = make_double2(0, 0);
+        if (MODE == kF64Filter) o = a.xd[qs];
+        __syncwarp();
+        if ((uint32_t)lane < nq) {
+            const uint32_t q = qs + lane;
+            if (MODE == kF32) {
+                const float2 p = a.xs[q];
+                sq[w][lane] = make_ulonglong2(pack2(p.x, p.x), pack2(p.y, p.y));
+            } else {
+                const double2 d = a.xd[q];
+                sqd[F64 ? w : 0][lane] = d;
+                if (MODE == kF64Filter) {
+                    const float qx = (float)__dsub_rn(d.x, o.x), qy = (float)__dsub_rn(d.y, o.y);
+                    sq[w][lane] = make_ulonglong2(pack2(qx, qx), pack2(qy, qy));
+                }
+            }
+        }
+        uint32_t my = 0;
+        uint2* gmask = masks ? masks + (__ldg(&moff[gi]) >> 1) : nullptr;
+        uint32_t k = 0;
+        __syncwarp();
+#pragma unroll 1
+        for (int r = 0; r < 3; ++r) {
+            const uint2 sp = __ldg(&a.cspan[3 * c + r]);
+            const uint32_t lo = sp.x, hi = sp.y;
+            if (lo >= hi) continue;
+#pragma unroll 1
+            for (uint32_t c0 = lo & ~1u; c0 < hi; c0 += 64, ++k) {
+                const uint32_t kk = k % kWin;
+                const uint32_t s0 = c0 + 2 * lane, s1 = s0 + 1;
+                const bool v0 = s0 >= lo && s0 < hi, v1 = s1 >= lo && s1 < hi;
+                u64x X, Y;
+                double2 d0 = make_double2(kFarD, kFarD), d1 = make_double2(kFarD, kFarD);
+                if (MODE == kF32) {
+                    ulonglong2 P = make_ulonglong2(0, 0);
+                    if (v0 || v1) P = xp[s0 >> 1];
+                    const float2 px = unpack2(P.x), py = unpack2(P.y);
+                    X = pack2(v0 ? px.x : kFarF, v1 ? px.y : kFarF);
+                    Y = pack2(v0 ? py.x : kFarF, v1 ? py.y : kFarF);
+                } else {
+                    if (v0) d0 = a.xd[s0];
+                    if (v1) d1 = a.xd[s1];
+                    if (MODE == kF64Filter) {
+                        X = pack2(v0 ? (float)__dsub_rn(d0.x, o.x) : kFarF, v1 ? (float)__dsub_rn(d1.x, o.x) : kFarF);
+                        Y = pack2(v0 ? (float)__dsub_rn(d0.y, o.y) : kFarF, v1 ? (float)__dsub_rn(d1.y, o.y) : kFarF);
+                    }
+                }
+                tests += (unsigned long long)nq * (min(c0 + 64, hi) - max(c0, lo));
+                uint32_t acc = 0;   // f64 filter: sign bit set <=> some |t| <= band in this lane
+#pragma unroll 4
+                for (uint32_t i = 0; i < nq; ++i) {
+                    unsigned m0, m1;
+                    if (MODE == kF64Exact) {
+                        const double2 qd = sqd[F64 ? w : 0][i];
+                        m0 = __ballot_sync(FULL, pred_f64(qd.x, qd.y, d0.x, d0.y, a.e2d));
+                        m1 = __ballot_sync(FULL, pred_f64(qd.x, qd.y, d1.x, d1.y, a.e2d));
+                    } else {
+                        const ulonglong2 Q = sq[w][i];
+                        const u64x dx = sub2(Q.x, X);
+                        const u64x dy = sub2(Q.y, Y);
+                        if (MODE == kF64Filter) {
+                            const u64x tt = fma2(dy, dy, fma2(dx, dx, NE2));   // (dx^2 - e2) + dy^2
+                            const float2 t = unpack2(tt);
+                            m0 = __ballot_sync(FULL, t.x < 0.f);
+                            m1 = __ballot_sync(FULL, t.y < 0.f);
+                            const float2 u = unpack2(fma2(tt, tt, NB2));         // t^2 - B^2 < 0  <=>  |t| < B
+                            acc |= __float_as_uint(u.x) | __float_as_uint(u.y);
+                        } else {
+                            // exact f32: fl(fl(dx^2) + fl(dy^2)) with scalar add.rn (ptxas would fuse
+                            // mul.rn.f32x2 + add.rn.f32x2 into FFMA2 -- reading R2)
+                            const float2 px = unpack2(mul2(dx, dx));
+                            const float2 py = unpack2(mul2(dy, dy));
+                            m0 = __ballot_sync(FULL, __fadd_rn(px.x, py.x) <= a.e2f);
+                            m1 = __ballot_sync(FULL, __fadd_rn(px.y, py.y) <= a.e2f);
+                        }
+                    }
+                    if (lane == 0) swin[w][i][kk] = make_uint2(m0, m1);
+                }
+                if (MODE == kF64Filter && __any_sync(FULL, (int)acc < 0)) {
+                    // replay the chunk: tests in the band are decided in exact f64
+#pragma unroll 1
+                    for (uint32_t i = 0; i < nq; ++i) {
+                        const ulonglong2 Q = sq[w][i];
+                        const u64x dx = sub2(Q.x, X);
+                        const u64x dy = sub2(Q.y, Y);
+                        const u64x tt = fma2(dy, dy, fma2(dx, dx, NE2));
+                        const float2 t = unpack2(tt);
+                        const float2 u = unpack2(fma2(tt, tt, NB2));
+                        const bool b0 = u.x < 0.f || __float_as_uint(u.x) == 0x80000000u;
+                        const bool b1 = u.y < 0.f || __float_as_uint(u.y) == 0x80000000u;
+                        if (!__any_sync(FULL, b0 | b1)) continue;
+                        const double2 qd = sqd[F64 ? w : 0][i];
+                        const bool e0 = b0 && pred_f64(qd.x, qd.y, d0.x, d0.y, a.e2d);
+                        const bool e1 = b1 && pred_f64(qd.x, qd.y, d1.x, d1.y, a.e2d);
+                        const unsigned m0 = (__ballot_sync(FULL, t.x < 0.f) & ~__ballot_sync(FULL, b0)) |
+                                            __ballot_sync(FULL, e0);
+                        const unsigned m1 = (__ballot_sync(FULL, t.y < 0.f) & ~__ballot_sync(FULL, b1)) |
+                                            __ballot_sync(FULL, e1);
+                        if (lane == 0) swin[w][i][kk] = make_uint2(m0, m1);
+                    }
+                }
+                __syncwarp();
+                if ((uint32_t)lane < nq) {
+                    const uint2 mk = swin[w][lane][kk];
+                    my += __popc(mk.x) + __popc(mk.y);
+                }
+                if (gmask && kk == kWin - 1) flush_window(swin[w], gmask, k / kWin, nq, lane);
+            }
+        }
+        if (gmask && (k % kWin) != 0) flush_window(swin[w], gmask, k / kWin, nq, lane);
+        if ((uint32_t)lane < nq) cnt[qs + lane] = my;
+        if (++gi >= gend) {
+            gi = g0 + grab(ctr, chunk, lane);
+            gend = min(gi + chunk, g1);
+        }
+    }
+    if (tests_out && lane == 0 && tests) atomicAdd(tests_out, tests);
+}
+
+// a8 (recompute variant) / legacy count: warp per query group; lane j holds the candidate PAIR (2k, 2k+1)
 // of the chunk (one 16-B load of the paired-SoA layout {x0, x1, y0, y1} gives
 // the packed operands X = {x0, x1}, Y = {y0, y1} directly); each query is
 // tested against 64 candidates with FADD2/FFMA2 and two ballots.
@@ -156,7 +317,7 @@ __global__ void __launch_bounds__(kSearchThreads) k_search(SArgs a, uint32_t g0,
                                                            uint32_t* __restrict__ out, uint2* __restrict__ masks,
                                                            const uint64_t* __restrict__ moff) {
     constexpr bool F64 = MODE != kF32;
-    __shared__ uint2 swin[WRITE ? 1 : kWarps][32][kWin];   // count pass: masks of the current window
+    __shared__ uint2 swin[WRITE ? 1 : kWarps][32][kWinPad];   // count pass: masks of the current window
     __shared__ ulonglong2 sq[kWarps][32];          // {{qx, qx}, {qy, qy}} packed f32 pairs
     __shared__ double2 sqd[F64 ? kWarps : 1][32];  // exact query coordinates (f64 modes)
     const int lane = threadIdx.x & 31;
@@ -204,7 +365,7 @@ __global__ void __launch_bounds__(kSearchThreads) k_search(SArgs a, uint32_t g0,
             if (lo >= hi) continue;   // empty span: no chunk (the mask layout counts none)
 #pragma unroll 1
             for (uint32_t c0 = lo & ~1u; c0 < hi; c0 += 64, ++k) {
-                uint2 mk = make_uint2(0, 0);   // count pass: lane i keeps query i's masks
+                const uint32_t kk = k % kWin;   // count pass: chunk slot in the window buffer
                 const uint32_t s0 = c0 + 2 * lane, s1 = s0 + 1;
                 const bool v0 = s0 >= lo && s0 < hi, v1 = s1 >= lo && s1 < hi;
                 ulonglong2 P = make_ulonglong2(0, 0);
@@ -235,9 +396,10 @@ __global__ void __launch_bounds__(kSearchThreads) k_search(SArgs a, uint32_t g0,
                             const float2 t = unpack2(fma2(dy, dy, fma2(dx, dx, NE2)));   // (dx^2 - e2) + dy^2
                             m0 = __ballot_sync(FULL, v0 && t.x < 0.f);
                             m1 = __ballot_sync(FULL, v1 && t.y < 0.f);
-                            const bool b0 = v0 & (fabsf(t.x) <= band);
-                            const bool b1 = v1 & (fabsf(t.y) <= band);
-                            if (__any_sync(FULL, b0 | b1)) {   // rare: decide these tests in exact f64
+                            const float tm = fminf(v0 ? fabsf(t.x) : INFINITY, v1 ? fabsf(t.y) : INFINITY);
+                            if (__any_sync(FULL, tm <= band)) {   // rare: decide these tests in exact f64
+                                const bool b0 = v0 & (fabsf(t.x) <= band);
+                                const bool b1 = v1 & (fabsf(t.y) <= band);
                                 const double2 qd = sqd[F64 ? w : 0][i];
                                 bool e0 = false, e1 = false;
                                 if (b0) {
@@ -271,16 +433,17 @@ __global__ void __launch_bounds__(kSearchThreads) k_search(SArgs a, uint32_t g0,
                         stg_if(p1, id.y, (m1 >> lane) & 1u);
                         const uint32_t nn = n0 + __popc(m1);
                         my += ((uint32_t)lane == i) ? nn : 0u;
-                    } else if ((uint32_t)lane == i) {
-                        mk = make_uint2(m0, m1);
+                    } else if (lane == 0) {
+                        swin[WRITE ? 0 : w][i][kk] = make_uint2(m0, m1);   // one STS instead of per-lane selects
                     }
                 }
                 if (!WRITE) {
-                    my += __popc(mk.x) + __popc(mk.y);
-                    if (gmask) {
-                        if ((uint32_t)lane < nq) swin[WRITE ? 0 : w][lane][k % kWin] = mk;
-                        if (k % kWin == kWin - 1) flush_window(swin[WRITE ? 0 : w], gmask, k / kWin, nq, lane);
+                    __syncwarp();
+                    if ((uint32_t)lane < nq) {
+                        const uint2 mk = swin[WRITE ? 0 : w][lane][kk];
+                        my += __popc(mk.x) + __popc(mk.y);
                     }
+                    if (gmask && kk == kWin - 1) flush_window(swin[WRITE ? 0 : w], gmask, k / kWin, nq, lane);
                 }
             }
         }
@@ -546,6 +709,8 @@ SArgs args_of(const DevGrid& g) {
     a.gcell = g.gcell;
     a.e2f = g.e2_f;
     a.band = g.band;
+    a.band_l = g.band_l;
+    a.nb2_l = g.nb2_l;
     a.e2d = g.e2_d;
     return a;
 }
@@ -617,9 +782,30 @@ void launch_sample_count(const DevGrid& g, uint64_t stride, uint64_t n_sample, u
 }
 
 // variant (hdb_opts.search_kernel): 0 = default, 1 = force the exact-f64-only kernel
+template <int MODE>
+void launch_count_mode(const SArgs& a, uint64_t g0, uint64_t g1, unsigned int* ctr, uint32_t* cnt,
+                       unsigned long long* tests, uint2* masks, const uint64_t* moff, cudaStream_t s) {
+    static int bps = 0;
+    uint32_t chunk;
+    unsigned ctas;
+    launch_groups(k_count<MODE>, bps, g1 - g0, chunk, ctas);
+    k_count<MODE><<<ctas, kSearchThreads, 0, s>>>(a, (uint32_t)g0, (uint32_t)g1, chunk, ctr, cnt, tests, masks, moff);
+}
+
 void launch_count(const DevGrid& g, uint64_t g0, uint64_t g1, uint32_t* cnt, unsigned long long* tests,
                   int variant, int slot, uint2* masks, cudaStream_t s) {
-    launch_search<false>(g, g0, g1, cnt, tests, nullptr, 0, nullptr, variant == 1, slot, masks, s);
+    if (g1 <= g0) return;
+    const SArgs a = args_of(g);
+    unsigned int* ctr = g.counters + (slot % kCounterSlots);
+    cudaMemsetAsync(ctr, 0, sizeof(unsigned int), s);
+    const int mode = g.dtype == HDB_F32 ? kF32 : (g.filter_l && variant != 1 ? kF64Filter : kF64Exact);
+    if (mode == kF64Filter)
+        launch_count_mode<kF64Filter>(a, g0, g1, ctr, cnt, tests, masks, g.moff, s);
+    else if (mode == kF64Exact)
+        launch_count_mode<kF64Exact>(a, g0, g1, ctr, cnt, tests, masks, g.moff, s);
+    else
+        launch_count_mode<kF32>(a, g0, g1, ctr, cnt, tests, masks, g.moff, s);
+    ++g_kernel_launches;
 }
 
 // masks != null: emission from the count pass's hit masks (k_emit); else the

@@ -29,7 +29,8 @@ def sass():
 
 
 def _mode_kernels(sass, mode):
-    return {k: v for k, v in sass.items() if re.search(rf"k_searchILi{mode}ELb[01]E", k)}
+    """count kernel k_count<MODE> + recompute-write kernel k_search<MODE, true>"""
+    return {k: v for k, v in sass.items() if re.search(rf"(k_countILi{mode}E|k_searchILi{mode}ELb1E)", k)}
 
 
 def test_sm100a_code_present(sass):
