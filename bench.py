@@ -163,6 +163,7 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--kernel", type=int, default=0, help="search kernel variant (hdb_opts.search_kernel)")
+    ap.add_argument("--cell-split", type=int, default=0, help="hdb_opts.cell_split (0 = library default)")
     args = ap.parse_args()
     wl = WORKLOADS[args.workload]
     ws, rank, local = dist_env()
@@ -186,7 +187,7 @@ def main():
     xy_dev = torch.from_numpy(xy_np).to(dev)
     stream = torch.cuda.current_stream(dev)
     opts = dict(shard_rank=rank, shard_count=ws) if ws > 1 else {}
-    ctx = hdb.hdb_ctx_create(search_kernel=args.kernel, **opts)
+    ctx = hdb.hdb_ctx_create(search_kernel=args.kernel, cell_split=args.cell_split, **opts)
     hdb.hdb_ctx_set_stream(ctx, stream.cuda_stream)
 
     def step():
@@ -242,7 +243,7 @@ def main():
     tp = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tp):
         with open(tp) as f:
-            traffic = json.load(f).get(f"{args.workload}-{args.dtype}-k{args.kernel}")
+            traffic = json.load(f).get(f"{args.workload}-{args.dtype}-k{args.kernel}-s{args.cell_split}")
     # whole-step view: SURVEY 8(d) B_alg = 4P + 64n + 8C (f64) over the step time
     esz = 16 if args.dtype == "f64" else 8
     b_step = 4 * P + (4 * esz + 32) * n + 8 * st["n_nonempty"]

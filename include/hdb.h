@@ -83,6 +83,8 @@ typedef struct {
     int shard_count;            /*   computes shard shard_rank of shard_count; 0 => unsharded          */
     int search_kernel;          /* 0 = default; other values select kernel variants        */
     int host_threads;           /* threads for host-side work (T assembly, DBSCAN); 0 = all cores      */
+    int cell_split;             /* k >= 1: grid cells of width eps/k, (2k+1)^2-cell stencil (fewer
+                                   candidate tests on dense data); 0 = default (1, the paper's eps)    */
 } hdb_opts;
 
 /* Borrowed view of a table T (T_i^min/T_i^max ranges into B).

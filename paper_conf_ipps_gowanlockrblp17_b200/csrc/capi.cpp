@@ -66,6 +66,7 @@ hdb_status hdb_ctx_create(const hdb_opts* opts, hdb_ctx** out) {
     if (o.n_devices < 0 || (o.n_devices > 0 && !o.devices)) fail(HDB_EINVAL, "bad device list");
     if (o.shard_count < 0 || (o.shard_count > 0 && (o.shard_rank < 0 || o.shard_rank >= o.shard_count)))
         fail(HDB_EINVAL, "bad shard_rank/shard_count");
+    if (o.cell_split < 0 || o.cell_split > 8) fail(HDB_EINVAL, "cell_split must be in [0, 8]");
     c = new hdb_ctx;
     int ndev_avail = 0;
     cudaError_t e = cudaGetDeviceCount(&ndev_avail);

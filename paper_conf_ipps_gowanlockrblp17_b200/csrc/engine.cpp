@@ -260,7 +260,8 @@ void set_filter_bound(DevGrid& g) {
     g.oy = 0.5 * g.ymin + 0.5 * g.ymax;
     const double R = std::max(std::max(std::fabs(g.xmax - g.ox), std::fabs(g.xmin - g.ox)),
                               std::max(std::fabs(g.ymax - g.oy), std::fabs(g.ymin - g.oy)));
-    const double Dmax = 2.0 * g.w * (1.0 + 0x1p-18);   // cell rounding: <= 2^-21 cell widths
+    // stencil of +-k cells: |x_p - x_q| < (k+1) w; cell rounding adds <= 2^-21 cell widths
+    const double Dmax = (double)(g.split + 1) * g.w * (1.0 + 0x1p-18);
     const double e2 = g.e2_d;
     g.e2_f = (float)e2;
     if (!(Dmax < 1e15) || !(e2 > 1e-30)) return;
@@ -277,6 +278,28 @@ void set_filter_bound(DevGrid& g) {
         g.nb2_l = -round_up_f(B * B);
         g.filter_l = true;
     }
+}
+
+// Default cell split (hdb_opts.cell_split == 0; split_from_occ): cells of width eps/k with
+// k = floor(sqrt(occ / 25)) clamped to [1, 6], where occ = sum n_c (n_c - 1) / n is
+// the point-weighted occupancy of the eps-wide cells, estimated from a strided
+// sample of <= 8192 points.  Finer cells shrink each group's candidate region
+// ((2 + 1/k)^2 eps^2 instead of 9 eps^2) but make groups smaller; ~25 points
+// per split cell was the measured break-even on the C2/C3 stand-ins.
+constexpr uint32_t kOccTable = 1u << 15;
+constexpr uint64_t kOccSample = 8192;
+
+uint32_t split_from_occ(const unsigned long long* h, uint64_t n, const DevGrid& g, double eps_used) {
+    if (h[1] == 0) return 1;
+    const uint64_t m = std::min<uint64_t>(n, kOccSample);
+    const double f = (double)m / (double)n;
+    const double occ = (double)h[0] / (f * (double)h[1]);
+    uint32_t k = (uint32_t)std::floor(std::sqrt(occ / 25.0));
+    k = std::max<uint32_t>(1, std::min<uint32_t>(k, 6));
+    const double inv1 = 1.0 / (eps_used * (1.0 + 0x1p-19));
+    const double ex = (g.xmax - g.xmin) * inv1, ey = (g.ymax - g.ymin) * inv1;
+    while (k > 1 && (ex * k > 0x1p30 || ey * k > 0x1p30)) --k;
+    return k;
 }
 
 void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t n, hdb_dtype dt, double eps,
@@ -314,9 +337,27 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
     HDB_CUDA(cudaMemsetAsync(bb + 4, 0, 8, s));
     launch_bbox(xin, n, dt, bb, bad, s);
     HDB_LAUNCH_CHECK();
+    // default cell split: occupancy estimate launched with the bbox, read in the same sync
+    const bool auto_k = ctx->opts.cell_split == 0 && n >= 4096;
+    DBuf hk, hc, occ;
+    unsigned long long hocc[2] = {0, 0};
+    if (auto_k) {
+        const double eps_pre = dt == HDB_F32 ? (double)(float)eps : eps;
+        hk = DBuf(8ull * kOccTable, s);
+        hc = DBuf(4ull * kOccTable, s);
+        occ = DBuf(16, s);
+        const uint64_t m = std::min<uint64_t>(n, kOccSample);
+        launch_occ_estimate(xin, n, dt, n / m, m, 1.0 / (eps_pre * (1.0 + 0x1p-19)), hk.as<unsigned long long>(),
+                            hc.as<unsigned int>(), kOccTable, occ.as<unsigned long long>(), s);
+        HDB_LAUNCH_CHECK();
+        HDB_CUDA(cudaMemcpyAsync(hocc, occ.p, sizeof hocc, cudaMemcpyDeviceToHost, s));
+    }
     unsigned long long hb[6];
     HDB_CUDA(cudaMemcpyAsync(hb, bb, sizeof hb, cudaMemcpyDeviceToHost, s));
     HDB_CUDA(cudaStreamSynchronize(s));
+    hk.reset();
+    hc.reset();
+    occ.reset();
     if ((unsigned int)hb[5] != 0) fail(HDB_EINVAL, "%u non-finite coordinate(s)", (unsigned)hb[5]);
 
     double eps_used = eps;
@@ -328,14 +369,18 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
     }
     g.e2_d = eps_used * eps_used;       // fl64(eps * eps)
     g.eps = eps_used;
-    g.w = eps_used * (1.0 + 0x1p-19);   // reading R9
-    g.inv_w = 1.0 / g.w;
     if (n > 0) {
         g.xmin = bbox_decode(hb[0], false);
         g.ymin = bbox_decode(hb[1], false);
         g.xmax = bbox_decode(hb[2], true);
         g.ymax = bbox_decode(hb[3], true);
     }
+    // reading R9: w = eps_F (1 + 2^-19) / k; a neighbour is at most k cells away
+    g.split = (uint32_t)(ctx->opts.cell_split > 0 ? ctx->opts.cell_split : 1);
+    if (auto_k) g.split = split_from_occ(hocc, n, g, eps_used);
+    g.nspan = 2 * g.split + 1;
+    g.w = eps_used * (1.0 + 0x1p-19) / (double)g.split;
+    g.inv_w = 1.0 / g.w;
     const double ex = (g.xmax - g.xmin) * g.inv_w;   // same rounded ops as the key kernel
     const double ey = (g.ymax - g.ymin) * g.inv_w;
     if (!(ex <= 0x1p30) || !(ey <= 0x1p30))
@@ -396,8 +441,8 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
     keys.reset();
     tr.mark("cells+sync");
     // ---- stencil row spans per non-empty cell + query groups
-    DBuf cspan(24 * nne, s), gcount(4 * (nne + 1), s), gofs(4 * (nne + 1), s);
-    launch_cell_spans(ckey.as<uint64_t>(), cstart.as<uint32_t>(), nne, g.nx, g.ny, cspan.as<uint2>(),
+    DBuf cspan(8 * g.nspan * nne, s), gcount(4 * (nne + 1), s), gofs(4 * (nne + 1), s);
+    launch_cell_spans(ckey.as<uint64_t>(), cstart.as<uint32_t>(), nne, g.nx, g.ny, g.split, cspan.as<uint2>(),
                       gcount.as<uint32_t>(), s);
     scan_u32_to_u32(gcount.as<uint32_t>(), gofs.as<uint32_t>(), nne, temp.p, s);
     HDB_LAUNCH_CHECK();

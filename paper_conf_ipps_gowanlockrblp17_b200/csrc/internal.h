@@ -58,6 +58,8 @@ struct DevGrid {
     double xmin = 0, ymin = 0, xmax = 0, ymax = 0;
     double ox = 0, oy = 0;  // f64 mode: origin of the f32 filter coordinates
     uint32_t nx = 1, ny = 1;
+    uint32_t split = 1;            // k: cell width eps/k, stencil (2k+1) x (2k+1) cells
+    uint32_t nspan = 3;            // 2k+1 row spans per non-empty cell
     uint64_t n_cells = 0, n_nonempty = 0, n_groups = 0;
     void* xy_s = nullptr;          // [n] double2 / float2, cell order (exact coordinates)
     float4* xp = nullptr;          // [n/2+1] paired-SoA f32 coords {x_2k, x_2k+1, y_2k, y_2k+1}: the
@@ -66,7 +68,7 @@ struct DevGrid {
     uint32_t* ids = nullptr;       // [n] sorted pos -> original id  (A)
     uint64_t* ckey = nullptr;      // [n_nonempty] cell key of each non-empty cell (ascending)
     uint32_t* cstart = nullptr;    // [n_nonempty+1] first sorted pos of each non-empty cell (G)
-    uint2* cspan = nullptr;        // [3*n_nonempty] stencil row spans [lo,hi) per non-empty cell
+    uint2* cspan = nullptr;        // [nspan*n_nonempty] stencil row spans [lo,hi) per non-empty cell
     uint32_t* gstart = nullptr;    // [n_groups+1] first sorted pos of each query group
     uint32_t* gcell = nullptr;     // [n_groups] non-empty cell index of each query group
     uint64_t* moff = nullptr;      // [n_groups+1] first 32-bit word of each group's hit masks
@@ -95,7 +97,12 @@ void launch_cell_flags(const uint64_t* keys_sorted, uint64_t n, uint32_t* flags,
 void launch_cell_scatter(const uint64_t* keys_sorted, const uint32_t* flags, const uint32_t* pos, uint64_t n,
                          uint64_t* ckey, uint32_t* cstart, cudaStream_t s);
 void launch_cell_spans(const uint64_t* ckey, const uint32_t* cstart, uint64_t nne, uint32_t nx, uint32_t ny,
-                       uint2* cspan, uint32_t* gcount, cudaStream_t s);
+                       uint32_t k, uint2* cspan, uint32_t* gcount, cudaStream_t s);
+// auto cell split: sample-based point-weighted occupancy at cell width 1/inv_w;
+// out[0] = sum s_c (s_c - 1), out[1] = sum s_c over the sampled cells
+void launch_occ_estimate(const void* xy, uint64_t n, hdb_dtype dt, uint64_t stride, uint64_t m, double inv_w,
+                         unsigned long long* hkey, unsigned int* hcnt, uint32_t tsize, unsigned long long* out,
+                         cudaStream_t s);
 void launch_group_build(const uint32_t* cstart, const uint32_t* gofs, uint64_t nne, uint64_t n, uint32_t* gstart,
                         uint32_t* gcell, cudaStream_t s);
 

@@ -13,10 +13,10 @@
 //   a4  offsets   -- run boundaries of the sorted keys + a warp-shuffle exclusive
 //                    scan -> G restricted to the NON-EMPTY cells: (key, start) pairs,
 //                    half-open (reading R11); sparse extents cost nothing
-//   +   spans     -- for every non-empty cell, its three stencil row spans: with
-//                    row-major keys the cells (cx-1..cx+1, y') are consecutive in
-//                    key order, so each stencil row is one contiguous range of
-//                    sorted positions (found by binary search over the keys)
+//   +   spans     -- for every non-empty cell, its 2k+1 stencil row spans (cells of
+//                    width eps/k): with row-major keys the cells (cx-k..cx+k, y')
+//                    are consecutive in key order, so each stencil row is one
+//                    contiguous range of sorted positions (binary search)
 //   +   groups    -- query groups: <= 32 consecutive sorted queries of one cell,
 //                    the unit of work of the search kernels.
 #include <cuda_runtime.h>
@@ -260,42 +260,38 @@ __device__ __forceinline__ uint64_t lower_bound_u64(const uint64_t* __restrict__
     return lo;
 }
 
-// Stencil row spans of every non-empty cell c (cx, cy): for y' in cy-1..cy+1,
-// the sorted positions of cells (max(cx-1,0) .. min(cx+1,nx-1), y').  The own
-// row uses the neighbouring entries directly; the rows above/below are binary
-// searches over the keys (the cells of row cy-1 precede c, of row cy+1 follow).
-// Also gcount[c] = number of 32-query groups of the cell.
+// Stencil row spans of every non-empty cell c (cx, cy): with cells of width
+// w = eps_F (1 + 2^-19) / k, a neighbour lies at most k cells away, so for each
+// of the 2k+1 rows y' in cy-k..cy+k the span covers the sorted positions of
+// cells (max(cx-k,0) .. min(cx+k,nx-1), y') -- consecutive keys, one
+// contiguous range, found by two binary searches over the non-empty keys
+// (rows below cy precede c, rows above follow it).  Also gcount[c] = number of
+// 32-query groups of the cell.
 __global__ void __launch_bounds__(256) k_cell_spans(const uint64_t* __restrict__ ckey,
                                                     const uint32_t* __restrict__ cstart, uint64_t nne,
-                                                    uint32_t nx, uint32_t ny, uint2* __restrict__ cspan,
+                                                    uint32_t nx, uint32_t ny, uint32_t k, uint2* __restrict__ cspan,
                                                     uint32_t* __restrict__ gcount) {
+    const uint32_t nspan = 2 * k + 1;
     for (uint64_t c = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; c < nne;
          c += (uint64_t)gridDim.x * blockDim.x) {
         const uint64_t key = ckey[c];
         const uint64_t cy = key / nx, cx = key - cy * nx;
-        const uint64_t xl = cx > 0 ? cx - 1 : 0;
-        const uint64_t xh = cx + 1 < nx ? cx + 1 : nx - 1;
-        // own row
-        uint64_t a = c, b = c + 1;
-        if (cx > 0 && c > 0 && ckey[c - 1] == key - 1) a = c - 1;
-        if (cx + 1 < nx && c + 1 < nne && ckey[c + 1] == key + 1) b = c + 2;
-        uint2 own = make_uint2(cstart[a], cstart[b]);
-        uint2 lo_row = make_uint2(0, 0), hi_row = make_uint2(0, 0);
-        if (cy > 0) {
-            const uint64_t rb = (cy - 1) * nx;
-            uint64_t i0 = lower_bound_u64(ckey, 0, c, rb + xl);
-            uint64_t i1 = lower_bound_u64(ckey, i0, c, rb + xh + 1);
-            lo_row = make_uint2(cstart[i0], cstart[i1]);
+        const uint64_t xl = cx >= k ? cx - k : 0;
+        const uint64_t xh = cx + k < nx ? cx + k : nx - 1;
+        for (uint32_t r = 0; r < nspan; ++r) {
+            const int64_t yy = (int64_t)cy + (int64_t)r - (int64_t)k;
+            uint2 sp = make_uint2(0, 0);
+            if (yy >= 0 && yy < (int64_t)ny) {
+                const uint64_t rb = (uint64_t)yy * nx;
+                uint64_t lo = 0, hi = nne;
+                if (yy < (int64_t)cy) hi = c;
+                else if (yy > (int64_t)cy) lo = c + 1;
+                const uint64_t i0 = lower_bound_u64(ckey, lo, hi, rb + xl);
+                const uint64_t i1 = lower_bound_u64(ckey, i0, hi, rb + xh + 1);
+                sp = make_uint2(cstart[i0], cstart[i1]);
+            }
+            cspan[nspan * c + r] = sp;
         }
-        if (cy + 1 < ny) {
-            const uint64_t rb = (cy + 1) * nx;
-            uint64_t i0 = lower_bound_u64(ckey, c + 1, nne, rb + xl);
-            uint64_t i1 = lower_bound_u64(ckey, i0, nne, rb + xh + 1);
-            hi_row = make_uint2(cstart[i0], cstart[i1]);
-        }
-        cspan[3 * c + 0] = lo_row;
-        cspan[3 * c + 1] = own;
-        cspan[3 * c + 2] = hi_row;
         gcount[c] = (cstart[c + 1] - cstart[c] + (uint32_t)kGroup - 1) / (uint32_t)kGroup;
     }
 }
@@ -313,6 +309,66 @@ __global__ void __launch_bounds__(256) k_group_build(const uint32_t* __restrict_
         }
     }
     if (blockIdx.x == 0 && threadIdx.x == 0) gstart[gofs[nne]] = (uint32_t)n;
+}
+
+// ---------------------------------------------------------------- auto cell split
+// Point-weighted cell occupancy at width eps, estimated from a strided sample of
+// m points: sample counts s_c per cell go into an open-addressing hash table;
+// sum s_c (s_c - 1) / (f sum s_c) (f = m / n) estimates sum n_c (n_c - 1) / n.
+__device__ __forceinline__ uint64_t mix_key(uint64_t x) {
+    x ^= x >> 33;
+    x *= 0xff51afd7ed558ccdull;
+    x ^= x >> 33;
+    return x;
+}
+
+template <typename T>
+__global__ void __launch_bounds__(256) k_occ_sample(const typename V2<T>::type* __restrict__ xy, uint64_t n,
+                                                    uint64_t stride, uint64_t m, double inv_w,
+                                                    unsigned long long* __restrict__ hkey,
+                                                    unsigned int* __restrict__ hcnt, uint32_t tmask) {
+    // cells of width eps anchored at the origin (no bbox needed: launched with the bbox
+    // reduction, before its host sync); the occupancy statistic does not depend on the anchor
+    for (uint64_t j = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; j < m; j += (uint64_t)gridDim.x * blockDim.x) {
+        auto p = xy[j * stride];
+        const double tx = fmin(fmax(floor((double)p.x * inv_w), -0x1p40), 0x1p40);
+        const double ty = fmin(fmax(floor((double)p.y * inv_w), -0x1p40), 0x1p40);
+        const unsigned long long key =
+            ((unsigned long long)(long long)tx << 22) ^ (unsigned long long)(long long)ty * 0x9E3779B97F4A7C15ull;
+        // warp-aggregate equal keys (dense cells would serialise the atomics)
+        const unsigned act = __activemask();
+        const unsigned peers = __match_any_sync(act, key);
+        const int lane = threadIdx.x & 31;
+        if (lane != __ffs(peers) - 1) continue;
+        uint32_t slot = (uint32_t)mix_key(key) & tmask;
+        while (true) {
+            unsigned long long prev = atomicCAS(&hkey[slot], ~0ull, key);
+            if (prev == ~0ull || prev == key) {
+                atomicAdd(&hcnt[slot], (unsigned)__popc(peers));
+                break;
+            }
+            slot = (slot + 1) & tmask;
+        }
+    }
+}
+
+__global__ void __launch_bounds__(256) k_occ_reduce(const unsigned int* __restrict__ hcnt, uint32_t tsize,
+                                                    unsigned long long* __restrict__ out) {
+    unsigned long long a = 0, b = 0;
+    for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < tsize; i += gridDim.x * blockDim.x) {
+        const unsigned long long c = hcnt[i];
+        a += c * (c > 0 ? c - 1 : 0);
+        b += c;
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        a += __shfl_xor_sync(FULL, a, o);
+        b += __shfl_xor_sync(FULL, b, o);
+    }
+    if ((threadIdx.x & 31) == 0) {
+        atomicAdd(&out[0], a);
+        atomicAdd(&out[1], b);
+    }
 }
 
 inline unsigned grid_for(uint64_t n, int threads = 256, unsigned cap = 148u * 16u) {
@@ -408,15 +464,34 @@ void launch_cell_scatter(const uint64_t* keys_sorted, const uint32_t* flags, con
 }
 
 void launch_cell_spans(const uint64_t* ckey, const uint32_t* cstart, uint64_t nne, uint32_t nx, uint32_t ny,
-                       uint2* cspan, uint32_t* gcount, cudaStream_t s) {
+                       uint32_t k, uint2* cspan, uint32_t* gcount, cudaStream_t s) {
     if (nne == 0) return;
-    k_cell_spans<<<grid_for(nne), 256, 0, s>>>(ckey, cstart, nne, nx, ny, cspan, gcount);
+    k_cell_spans<<<grid_for(nne), 256, 0, s>>>(ckey, cstart, nne, nx, ny, k, cspan, gcount);
     ++g_kernel_launches;
 }
 
 void launch_group_build(const uint32_t* cstart, const uint32_t* gofs, uint64_t nne, uint64_t n, uint32_t* gstart,
                         uint32_t* gcell, cudaStream_t s) {
     k_group_build<<<grid_for(nne), 256, 0, s>>>(cstart, gofs, nne, n, gstart, gcell);
+    ++g_kernel_launches;
+}
+
+void launch_occ_estimate(const void* xy, uint64_t n, hdb_dtype dt, uint64_t stride, uint64_t m, double inv_w,
+                         unsigned long long* hkey, unsigned int* hcnt, uint32_t tsize, unsigned long long* out,
+                         cudaStream_t s) {
+    cudaMemsetAsync(hkey, 0xff, sizeof(unsigned long long) * tsize, s);
+    cudaMemsetAsync(hcnt, 0, sizeof(unsigned int) * tsize, s);
+    cudaMemsetAsync(out, 0, 2 * sizeof(unsigned long long), s);
+    if (m) {
+        if (dt == HDB_F64)
+            k_occ_sample<double><<<grid_for(m), 256, 0, s>>>((const double2*)xy, n, stride, m, inv_w, hkey, hcnt,
+                                                             tsize - 1);
+        else
+            k_occ_sample<float><<<grid_for(m), 256, 0, s>>>((const float2*)xy, n, stride, m, inv_w, hkey, hcnt,
+                                                            tsize - 1);
+        ++g_kernel_launches;
+    }
+    k_occ_reduce<<<grid_for(tsize, 256, 148 * 2), 256, 0, s>>>(hcnt, tsize, out);
     ++g_kernel_launches;
 }
 

@@ -46,7 +46,8 @@ struct SArgs {
     const double2* xd;     // exact f64 coordinates (f64 mode)
     const uint32_t* ids;
     const uint32_t* cstart;
-    const uint2* cspan;
+    const uint2* cspan;    // [nspan * non-empty cells]
+    uint32_t nspan;        // 2k+1 stencil rows
     const uint32_t* gstart;
     const uint32_t* gcell;
     float e2f;             // f32 mode: fl32(eps^2); f64 mode: fl32(e2_d)
@@ -207,8 +208,8 @@ __global__ void __launch_bounds__(kSearchThreads) k_count(SArgs a, uint32_t g0, 
         uint32_t k = 0;
         __syncwarp();
 #pragma unroll 1
-        for (int r = 0; r < 3; ++r) {
-            const uint2 sp = __ldg(&a.cspan[3 * c + r]);
+        for (uint32_t r = 0; r < a.nspan; ++r) {
+            const uint2 sp = __ldg(&a.cspan[a.nspan * c + r]);
             const uint32_t lo = sp.x, hi = sp.y;
             if (lo >= hi) continue;
 #pragma unroll 1
@@ -359,8 +360,8 @@ __global__ void __launch_bounds__(kSearchThreads) k_search(SArgs a, uint32_t g0,
         uint32_t k = 0;
         __syncwarp();
 #pragma unroll 1
-        for (int r = 0; r < 3; ++r) {
-            const uint2 sp = __ldg(&a.cspan[3 * c + r]);
+        for (uint32_t r = 0; r < a.nspan; ++r) {
+            const uint2 sp = __ldg(&a.cspan[a.nspan * c + r]);
             const uint32_t lo = sp.x, hi = sp.y;
             if (lo >= hi) continue;   // empty span: no chunk (the mask layout counts none)
 #pragma unroll 1
@@ -499,10 +500,12 @@ __global__ void __launch_bounds__(kSearchThreads) k_emit(SArgs a, uint32_t g0, u
         asm volatile("mov.b64 %0, %0;" : "+l"(gout));
         uint32_t my = 0;   // lane i: output cursor of query i within the group
         if ((uint32_t)lane < nq) my = (uint32_t)(off[qs + lane] - gb);
-        const uint2 S0 = __ldg(&a.cspan[3 * c]), S1 = __ldg(&a.cspan[3 * c + 1]), S2 = __ldg(&a.cspan[3 * c + 2]);
-        // chunk iterator (same order as the count pass)
-        int r = S0.x < S0.y ? 0 : (S1.x < S1.y ? 1 : 2);   // the own-row span is never empty
-        uint2 sp = r == 0 ? S0 : (r == 1 ? S1 : S2);
+        // chunk iterator over the non-empty spans (same order as the count pass)
+        const uint2* cs = a.cspan + (size_t)a.nspan * c;
+        const uint32_t nspan = a.nspan;
+        uint32_t r = 0;
+        uint2 sp = __ldg(&cs[0]);
+        while (sp.x >= sp.y) sp = __ldg(&cs[++r]);   // the own-row span is never empty
         uint32_t c0 = sp.x & ~1u, hi = sp.y;
         __syncwarp();   // the previous group's buffers are no longer read
         if ((uint32_t)lane < nq) {   // prefetch window 0: lane i copies its 64-B mask row
@@ -518,17 +521,15 @@ __global__ void __launch_bounds__(kSearchThreads) k_emit(SArgs a, uint32_t g0, u
 #pragma unroll
             for (int kk = 0; kk < kWin; ++kk) {
                 ids[kk] = make_uint2(0, 0);
-                if (r < 3) {
+                if (r < nspan) {
                     if (c0 + 2 * lane < hi) ids[kk] = __ldg((const uint2*)(a.ids + c0 + 2 * lane));
                     c0 += 64;
                     if (c0 >= hi) {
-                        ++r;
-                        while (r < 3) {
-                            sp = r == 1 ? S1 : S2;
+                        while (++r < nspan) {
+                            sp = __ldg(&cs[r]);
                             if (sp.x < sp.y) break;
-                            ++r;
                         }
-                        if (r < 3) {
+                        if (r < nspan) {
                             c0 = sp.x & ~1u;
                             hi = sp.y;
                         }
@@ -582,8 +583,8 @@ __global__ void __launch_bounds__(256) k_mask_words(SArgs a, uint64_t ng, uint32
         const uint32_t qs = a.gstart[g], c = a.gcell[g];
         const uint32_t nq = min((uint32_t)kGroup, a.cstart[c + 1] - qs);
         uint32_t ch = 0;
-        for (int r = 0; r < 3; ++r) {
-            const uint2 sp = a.cspan[3 * c + r];
+        for (uint32_t r = 0; r < a.nspan; ++r) {
+            const uint2 sp = a.cspan[a.nspan * c + r];
             if (sp.y > sp.x) ch += (sp.y - (sp.x & ~1u) + 63) / 64;
         }
         words[g] = 2 * nq * kWin * ((ch + kWin - 1) / kWin);
@@ -615,8 +616,8 @@ __global__ void __launch_bounds__(256) k_sample_count(SArgs a, uint64_t nne, uin
         uint32_t cntv = 0;
         if (F64) {
             const double2 q = a.xd[s];
-            for (int r = 0; r < 3; ++r) {
-                const uint2 sp = a.cspan[3 * c + r];
+            for (uint32_t r = 0; r < a.nspan; ++r) {
+                const uint2 sp = a.cspan[a.nspan * c + r];
                 for (uint32_t k = sp.x + lane; k < sp.y; k += 32) {
                     const double2 p = a.xd[k];
                     cntv += pred_f64(q.x, q.y, p.x, p.y, a.e2d) ? 1u : 0u;
@@ -624,8 +625,8 @@ __global__ void __launch_bounds__(256) k_sample_count(SArgs a, uint64_t nne, uin
             }
         } else {
             const float2 q = a.xs[s];
-            for (int r = 0; r < 3; ++r) {
-                const uint2 sp = a.cspan[3 * c + r];
+            for (uint32_t r = 0; r < a.nspan; ++r) {
+                const uint2 sp = a.cspan[a.nspan * c + r];
                 for (uint32_t k = sp.x + lane; k < sp.y; k += 32) {
                     const float2 p = a.xs[k];
                     cntv += pred_f32(q.x, q.y, p.x, p.y, a.e2f) ? 1u : 0u;
@@ -705,6 +706,7 @@ SArgs args_of(const DevGrid& g) {
     a.ids = g.ids;
     a.cstart = g.cstart;
     a.cspan = g.cspan;
+    a.nspan = g.nspan;
     a.gstart = g.gstart;
     a.gcell = g.gcell;
     a.e2f = g.e2_f;

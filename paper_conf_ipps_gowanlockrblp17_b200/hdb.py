@@ -34,7 +34,7 @@ class hdb_opts(ctypes.Structure):
     _fields_ = [("devices", ctypes.POINTER(_int)), ("n_devices", _int), ("sample_fraction", _dbl),
                 ("alpha", _dbl), ("n_streams", _int), ("batch_pairs", _u64), ("sort_lists", _int),
                 ("host_budget_bytes", _u64), ("shard_rank", _int), ("shard_count", _int),
-                ("search_kernel", _int), ("host_threads", _int)]
+                ("search_kernel", _int), ("host_threads", _int), ("cell_split", _int)]
 
 
 class hdb_table_view(ctypes.Structure):

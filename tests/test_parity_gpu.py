@@ -428,3 +428,20 @@ def test_filter_disabled_for_huge_extent(torch_cuda):
     xy = np.concatenate([base, base + rng.normal(0, 0.02, base.shape)])
     b, c, v, _, _ = lib_table(xy, 0.05)
     assert_table_equal(xy, 0.05, b, c, v)
+
+
+@pytest.mark.parametrize("k", [2, 3])
+def test_cell_split_parity(torch_cuda, k):
+    """cell_split = k: cells of width eps/k and a (2k+1)^2 stencil; same table."""
+    cases = [(datagen.subsample(datagen.tec_like(), 40_000, seed=1), (0.15, 0.45, 1.40)),
+             (datagen.subsample(datagen.sdss_like(), 40_000, seed=2), (0.07, 0.6)),
+             (datagen.near_ties(3000, 0.45, seed=3), (0.45,)),
+             (datagen.lattice(30, origin=(-3.0, 7.0)), (1.0, math.sqrt(2.0)))]
+    for xy, eps_list in cases:
+        for eps in eps_list:
+            for device in (True, False):
+                b, c, v, view, st = lib_table(xy, eps, device=device, cell_split=k)
+                assert_table_equal(xy, eps, b, c, v)
+    xy = datagen.c1().astype(np.float32)
+    b, c, v, _, _ = lib_table(xy, 0.5, cell_split=k)
+    assert_table_equal(xy, 0.5, b, c, v, "f32")
