@@ -397,17 +397,18 @@ hdb_status hdb_dbscan_ex(const hdb_table* t, uint32_t minpts, int n_threads, int
         set_error("labels is NULL");
         return HDB_EINVAL;
     }
-    if (t->on_device) {
-        set_error("hdb_dbscan: table is device-resident (use hdb_neighbor_table)");
-        return HDB_EINVAL;
-    }
     if (t->first_query != 0 || t->end_query != t->n) {
         set_error("hdb_dbscan: table holds only a shard of the queries");
         return HDB_EINVAL;
     }
     HDB_GUARD_BEGIN
-    int T = n_threads > 0 ? n_threads : resolve_threads(t->host_threads);
-    uint32_t k = dbscan_host(t, minpts, T, labels, is_core);
+    uint32_t k = 0;
+    if (t->on_device) {
+        k = dbscan_device(t, minpts, labels, is_core);   // labels / is_core: host or device memory
+    } else {
+        int T = n_threads > 0 ? n_threads : resolve_threads(t->host_threads);
+        k = dbscan_host(t, minpts, T, labels, is_core);
+    }
     if (n_clusters) *n_clusters = k;
     HDB_GUARD_END
 }

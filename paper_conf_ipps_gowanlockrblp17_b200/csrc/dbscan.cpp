@@ -126,9 +126,14 @@ uint32_t dbscan_par(const hdb_table* t, uint32_t minpts, int T, int32_t* labels,
                 for (uint64_t u = a; u < b; ++u) {
                     if (!core[u]) continue;
                     const uint32_t* L = V + B[u];
+                    uint32_t ru = uf_find(parent.get(), (uint32_t)u);   // kept current across the list
                     for (uint32_t i = 0, m = C[u]; i < m; ++i) {
-                        uint32_t v = L[i];
-                        if (v < u && core[v]) uf_union(parent.get(), (uint32_t)u, v);
+                        const uint32_t v = L[i];
+                        if (v >= u || !core[v]) continue;
+                        const uint32_t rv = uf_find(parent.get(), v);
+                        if (rv == ru) continue;                        // already joined: no link needed
+                        uf_union(parent.get(), ru, rv);
+                        ru = uf_find(parent.get(), ru);
                     }
                 }
             }

@@ -756,6 +756,35 @@ T* pool_get(hdb_table* t, size_t count, size_t* cap) {
 
 }  // namespace
 
+// DBSCAN on a device-resident table (NEXT-4): labels / core may be host or
+// device pointers (core may be null); returns the number of clusters.
+uint32_t dbscan_device(const hdb_table* t, uint32_t minpts, int32_t* labels, uint8_t* core) {
+    DeviceGuard dg(t->device);
+    cudaStream_t s = t->dstream;
+    const uint64_t n = t->n;
+    if (n == 0) return 0;
+    const PtrInfo li = classify(labels), ci = classify(core);
+    const bool lab_dev = li.loc == Loc::Device && li.device == t->device;
+    const bool core_dev = core && ci.loc == Loc::Device && ci.device == t->device;
+    DBuf dlab, dcore(n, s), parent(4 * n, s), root(4 * n, s), is_root(4 * n, s), rank(4 * (n + 1), s),
+        temp(scan_temp_bytes(n + 1), s);
+    int32_t* L = labels;
+    if (!lab_dev) {
+        dlab = DBuf(4 * n, s);
+        L = dlab.as<int32_t>();
+    }
+    uint8_t* C = core_dev ? core : dcore.as<uint8_t>();
+    launch_dbscan_device(t->begin, t->count, t->nbrs, n, minpts, C, parent.as<uint32_t>(), root.as<uint32_t>(),
+                         is_root.as<uint32_t>(), rank.as<uint32_t>(), temp.p, L, s);
+    HDB_LAUNCH_CHECK();
+    uint32_t k = 0;
+    HDB_CUDA(cudaMemcpyAsync(&k, rank.as<uint32_t>() + n, 4, cudaMemcpyDeviceToHost, s));
+    if (!lab_dev) HDB_CUDA(cudaMemcpyAsync(labels, L, 4 * n, cudaMemcpyDeviceToHost, s));
+    if (core && !core_dev) HDB_CUDA(cudaMemcpyAsync(core, C, n, cudaMemcpyDeviceToHost, s));
+    HDB_CUDA(cudaStreamSynchronize(s));
+    return k;
+}
+
 void table_free(hdb_table* t) {
     if (!t) return;
     if (t->on_device) {

@@ -132,6 +132,10 @@ void launch_batch_cuts(const uint32_t* gstart, const uint64_t* off, uint64_t g0,
 // map sorted positions -> the first group starting at or after them (binary search in gstart)
 void launch_pos_to_group(const uint32_t* gstart, uint64_t n_groups, const uint64_t* pos, uint32_t m,
                          uint64_t* grp, cudaStream_t s);
+// DBSCAN on a device-resident table (kernels_dbscan.cu); rank[n] = number of clusters
+void launch_dbscan_device(const uint64_t* begin, const uint32_t* count, const uint32_t* nbrs, uint64_t n,
+                          uint32_t minpts, uint8_t* core, uint32_t* parent, uint32_t* root, uint32_t* is_root,
+                          uint32_t* rank, void* scan_temp, int32_t* labels, cudaStream_t s);
 // T assembly by original id: begin[ids[q]] = off[q] - off[q0] + base, count[ids[q]] = cnt[q], q in [q0,q1)
 void launch_scatter_rows(const uint32_t* ids, const uint64_t* off, const uint32_t* cnt, uint64_t q0,
                          uint64_t q1, uint64_t base, uint64_t* begin, uint32_t* count, cudaStream_t s);
@@ -203,5 +207,6 @@ void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hd
 void table_free(hdb_table* t);
 // dbscan.cpp
 uint32_t dbscan_host(const hdb_table* t, uint32_t minpts, int n_threads, int32_t* labels, uint8_t* core);
+uint32_t dbscan_device(const hdb_table* t, uint32_t minpts, int32_t* labels, uint8_t* core);
 void canonicalize(hdb_table* t);
 }  // namespace hdb

@@ -259,6 +259,8 @@ def hdb_table_free(table):
 
 
 def hdb_dbscan(table, minpts: int, n_threads: int = 0, labels=None, is_core=None):
+    """DBSCAN on a host table (host threads) or a device table (GPU, NEXT-4).
+    labels / is_core: numpy (host) or torch CUDA tensors; allocated on the host if None."""
     v = hdb_table_view_get(table)
     if labels is None:
         labels = np.empty(v.n, np.int32)

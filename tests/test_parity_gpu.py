@@ -445,3 +445,53 @@ def test_cell_split_parity(torch_cuda, k):
     xy = datagen.c1().astype(np.float32)
     b, c, v, _, _ = lib_table(xy, 0.5, cell_split=k)
     assert_table_equal(xy, 0.5, b, c, v, "f32")
+
+
+@pytest.mark.parametrize("split", [0, 1])
+def test_device_dbscan_matches_oracle(torch_cuda, split):
+    """NEXT-4: DBSCAN on the device-resident table gives the canonical labels."""
+    torch = torch_cuda
+    cases = [(datagen.c1(), 0.5, 4), (datagen.c1(), 2.0, 1),
+             (datagen.subsample(datagen.tec_like(), 40_000, seed=1), 0.45, 4),
+             (datagen.subsample(datagen.tec_like(), 40_000, seed=1), 0.15, 8),
+             (datagen.subsample(datagen.sdss_like(), 40_000, seed=2), 0.3, 4),
+             (datagen.lattice(12), 1.0, 5)]
+    for xy, eps, minpts in cases:
+        want = oracle.dbscan(*oracle.eps_join(xy, eps), minpts)
+        ctx = _ctx(cell_split=split)
+        try:
+            g = hdb.hdb_grid_build(ctx, xy, eps)
+            t = hdb.hdb_neighbor_table_device(ctx, g)
+            hdb.hdb_grid_free(g)
+            lab, core, k = hdb.hdb_dbscan(t, minpts)                 # host output buffers
+            dlab = torch.empty(xy.shape[0], dtype=torch.int32, device="cuda")
+            _, _, k2 = hdb.hdb_dbscan(t, minpts, labels=dlab)        # device output buffer
+            for _ in range(4):                                        # lock-free union-find: repeatable
+                again, _, k3 = hdb.hdb_dbscan(t, minpts)
+                assert k3 == k and np.array_equal(again, lab)
+            hdb.hdb_table_free(t)
+        finally:
+            hdb.hdb_ctx_destroy(ctx)
+        assert k == want[2] == k2
+        assert np.array_equal(core, want[1])
+        assert np.array_equal(lab, want[0])
+        assert np.array_equal(dlab.cpu().numpy(), want[0])
+
+
+def test_device_dbscan_shared_border_orders(torch_cuda):
+    import json
+    import os
+    with open(os.path.join(os.path.dirname(__file__), "golden", "border_orders.json")) as f:
+        g = json.load(f)
+    for o in g["orders"]:
+        xy = np.stack([np.array(o["x"], float), np.zeros(len(o["x"]))], axis=1)
+        ctx = _ctx()
+        try:
+            gr = hdb.hdb_grid_build(ctx, xy, g["eps"])
+            t = hdb.hdb_neighbor_table_device(ctx, gr)
+            hdb.hdb_grid_free(gr)
+            lab, core, k = hdb.hdb_dbscan(t, g["minpts"])
+            hdb.hdb_table_free(t)
+        finally:
+            hdb.hdb_ctx_destroy(ctx)
+        assert lab.tolist() == o["labels"] and core.tolist() == o["core"] and k == o["n_clusters"]

@@ -3,7 +3,7 @@
 # Usage (via gpurun): bash tools/gpu_cycle.sh [bench args...]
 cd "$(dirname "$0")/.."
 mkdir -p gpurun_out
-if [ "${FULL:-0}" = "1" ]; then SEL=""; else SEL="-k c1_full or workload or near_ties or lattice or batching or shards or exact_f64 or dbscan_end or grid_structure or sparse or cell_split"; fi
+if [ "${FULL:-0}" = "1" ]; then SEL=""; else SEL="-k c1_full or workload or near_ties or lattice or batching or shards or exact_f64 or dbscan_end or grid_structure or sparse or cell_split or device_dbscan"; fi
 timeout 900 python -m pytest tests -m gpu -q -x --timeout 300 ${SEL:+-k "${SEL#-k }"} > gpurun_out/cycle_pytest.txt 2>&1
 echo "PYTEST: $(tail -1 gpurun_out/cycle_pytest.txt)"
 grep -E "FAILED|Error" gpurun_out/cycle_pytest.txt | head -5
