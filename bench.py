@@ -175,10 +175,18 @@ def main():
     from paper_conf_ipps_gowanlockrblp17_b200 import hdb
 
     assert torch.cuda.is_available(), "bench.py needs a GPU"
-    torch.cuda.set_device(local)
+    ndev = torch.cuda.device_count()
+    local_dev = local % ndev
+    torch.cuda.set_device(local_dev)
     if ws > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    dev = torch.device("cuda", local)
+        # one process per GPU over NCCL; ranks sharing a GPU (testing on fewer GPUs than ranks)
+        # fall back to gloo for the one collective (the gather of per-shard pair counts)
+        if ndev >= ws:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local_dev))
+        else:
+            dist.init_process_group("gloo")
+    dev = torch.device("cuda", local_dev)
+    coll_dev = dev if (ws == 1 or ndev >= ws) else torch.device("cpu")
     xy_np = wl["gen"]()
     if args.dtype == "f32":
         xy_np = xy_np.astype(np.float32)
@@ -208,7 +216,7 @@ def main():
     write_ms, count_ms, pairs_local, launches = [], [], 0, 0
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     l0 = hdb.hdb_kernel_launches()
-    with ClockSampler(local) as clk:
+    with ClockSampler(local_dev) as clk:
         ev0.record(stream)
         for _ in range(args.steps):
             st, v = step()
@@ -221,11 +229,11 @@ def main():
     ms = ev0.elapsed_time(ev1)
     if ws > 1:
         from paper_conf_ipps_gowanlockrblp17_b200 import dist as hdist
-        t = torch.tensor([ms], device=dev)
+        t = torch.tensor([ms], device=coll_dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         ms = float(t.item())
         # the path's one exchange: the gather of per-shard pair counts
-        _, pairs_total = hdist.gather_pair_counts(pairs_local, device=dev)
+        _, pairs_total = hdist.gather_pair_counts(pairs_local, device=coll_dev)
     else:
         pairs_total = pairs_local
     P = pairs_total // max(args.steps, 1)
