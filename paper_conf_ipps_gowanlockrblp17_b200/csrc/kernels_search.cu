@@ -79,11 +79,6 @@ __device__ __forceinline__ u64x mul2(u64x a, u64x b) {
     asm("mul.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(a), "l"(b));
     return r;
 }
-__device__ __forceinline__ u64x add2(u64x a, u64x b) {
-    u64x r;
-    asm("add.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(a), "l"(b));
-    return r;
-}
 // predicated global store (keeps the st.global space after the pointer is laundered).
 // No "memory" clobber: nothing in the kernels reads the output, and a clobber
 // would pin every later shared/global load behind the store (serialising the
@@ -467,6 +462,9 @@ __global__ void __launch_bounds__(kSearchThreads) k_search(SArgs a, uint32_t g0,
 // segment, written by ballot-free popc prefixes with all 32 lanes (lane j owns
 // candidate pair (2j, 2j+1) of each chunk).  Long per-warp store streams keep
 // L2 lines whole -- interleaving 32 query lists per chunk halved the store rate.
+constexpr int kEmitThreads = 128;   // 4 warps per CTA (the padded window buffers are 28 KB per CTA)
+constexpr int kEmitWarps = kEmitThreads / 32;
+
 __device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
     const uint32_t sa = (uint32_t)__cvta_generic_to_shared(smem);
     asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(sa), "l"(gmem));
@@ -477,13 +475,14 @@ __device__ __forceinline__ void cp_async_wait() {
     asm volatile("cp.async.wait_group %0;" ::"n"(N));
 }
 
-__global__ void __launch_bounds__(kSearchThreads) k_emit(SArgs a, uint32_t g0, uint32_t g1, uint32_t chunk,
+__global__ void __launch_bounds__(kEmitThreads) k_emit(SArgs a, uint32_t g0, uint32_t g1, uint32_t chunk,
                                                          unsigned int* __restrict__ ctr,
                                                          const uint64_t* __restrict__ off, uint64_t out_base,
                                                          uint32_t* __restrict__ out, const uint2* __restrict__ masks,
                                                          const uint64_t* __restrict__ moff) {
-    __shared__ uint2 raw[kWarps][32][kWin];   // cp.async landing buffer (next window's masks)
-    __shared__ uint4 wq[kWarps][32][kWin];    // current window: {m0, m1, pos0, pos1} per (query, chunk)
+    // rows padded (80-B / 144-B strides) so the per-lane row accesses are bank-conflict free
+    __shared__ __align__(16) uint2 raw[kEmitWarps][32][kWin + 2];   // cp.async landing buffer (next window's masks)
+    __shared__ uint4 wq[kEmitWarps][32][kWin + 1];    // current window: {m0, m1, pos0, pos1} per (query, chunk)
     const int lane = threadIdx.x & 31;
     const int w = threadIdx.x >> 5;
     const unsigned lt = (1u << lane) - 1u;
@@ -720,16 +719,18 @@ SArgs args_of(const DevGrid& g) {
 // One wave of resident CTAs; warps grab `chunk` groups at a time (~32 grabs
 // per resident warp keeps the tail short while bounding counter atomics).
 template <typename K>
-void launch_groups(K kern, int& blocks_per_sm, uint64_t ng, uint32_t& chunk, unsigned& ctas) {
+void launch_groups(K kern, int& blocks_per_sm, uint64_t ng, uint32_t& chunk, unsigned& ctas,
+                   int threads = kSearchThreads) {
     if (!blocks_per_sm) {
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks_per_sm, kern, kSearchThreads, 0);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks_per_sm, kern, threads, 0);
         if (blocks_per_sm < 1) blocks_per_sm = 1;
     }
     int dev = 0, nsm = 148;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
-    const uint64_t wave_warps = (uint64_t)nsm * blocks_per_sm * kWarps;
-    ctas = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>((ng + kWarps - 1) / kWarps, (uint64_t)nsm * blocks_per_sm));
+    const uint64_t wpb = (uint64_t)threads / 32;
+    const uint64_t wave_warps = (uint64_t)nsm * blocks_per_sm * wpb;
+    ctas = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>((ng + wpb - 1) / wpb, (uint64_t)nsm * blocks_per_sm));
     chunk = (uint32_t)std::max<uint64_t>(1, ng / (wave_warps * 32));
 }
 
@@ -824,8 +825,8 @@ void launch_write(const DevGrid& g, uint64_t g0, uint64_t g1, const uint64_t* of
     static int bps = 0;
     uint32_t chunk;
     unsigned ctas;
-    launch_groups(k_emit, bps, g1 - g0, chunk, ctas);
-    k_emit<<<ctas, kSearchThreads, 0, s>>>(args_of(g), (uint32_t)g0, (uint32_t)g1, chunk, ctr, off, out_base, out,
+    launch_groups(k_emit, bps, g1 - g0, chunk, ctas, kEmitThreads);
+    k_emit<<<ctas, kEmitThreads, 0, s>>>(args_of(g), (uint32_t)g0, (uint32_t)g1, chunk, ctr, off, out_base, out,
                                            masks, g.moff);
     ++g_kernel_launches;
 }
