@@ -145,6 +145,58 @@ __device__ __forceinline__ void flush_window(uint2 (*swin)[kWinPad], uint2* gmas
     __syncwarp();
 }
 
+// ---------------------------------------------------------------- virtual chunks
+// A group's candidates are its 2k+1 row spans.  They are visited as ONE
+// sequence of candidate pairs (2p, 2p+1) -- span r contributes the pairs
+// lo_r/2 .. (hi_r-1)/2 -- cut into chunks of 32 pairs (one per lane), so only
+// the group's last chunk is ragged (per-span chunks left ~17% of the lanes idle
+// at k = 3).  VSpan r: [lo, hi) of the span, its first pair index and the
+// position of that pair in the virtual sequence; entry nspan holds the total.
+constexpr int kMaxSpans = 13;   // 2k + 1 for cell_split k <= 6
+struct VSpan {
+    uint32_t lo, hi, pbase, vstart;
+};
+
+// lanes r < nspan load span r; warp prefix over the pair counts; returns the
+// number of virtual pairs
+__device__ __forceinline__ uint32_t load_vspans(const SArgs& a, uint32_t c, VSpan* vs, int lane) {
+    uint32_t lo = 0, hi = 0, np = 0;
+    if ((uint32_t)lane < a.nspan) {
+        const uint2 sp = __ldg(&a.cspan[a.nspan * c + lane]);
+        lo = sp.x;
+        hi = sp.y;
+        np = hi > lo ? ((hi + 1) >> 1) - (lo >> 1) : 0;
+    }
+    uint32_t incl = np;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(FULL, incl, o);
+        if (lane >= o) incl += y;
+    }
+    const uint32_t total = __shfl_sync(FULL, incl, a.nspan - 1);
+    __syncwarp();
+    if ((uint32_t)lane < a.nspan) vs[lane] = VSpan{lo, hi, lo >> 1, incl - np};
+    if ((uint32_t)lane == a.nspan) vs[lane] = VSpan{0, 0, 0, total};
+    __syncwarp();
+    return total;
+}
+
+// candidate pair of virtual pair vp for this lane; r advances monotonically
+// across a group's chunks.  Returns s0 (= 2p) and the two validity flags.
+__device__ __forceinline__ uint32_t vpair(const VSpan* vs, uint32_t nspan, uint32_t vp, uint32_t& r, bool& v0,
+                                          bool& v1) {
+    while (r < nspan && vp >= vs[r + 1].vstart) ++r;
+    if (r >= nspan) {
+        v0 = v1 = false;
+        return 0;
+    }
+    const VSpan e = vs[r];
+    const uint32_t s0 = 2 * (e.pbase + (vp - e.vstart));
+    v0 = s0 >= e.lo && s0 < e.hi;
+    v1 = s0 + 1 >= e.lo && s0 + 1 < e.hi;
+    return s0;
+}
+
 // a6: the count pass.  Warp per query group; lane j holds the candidate PAIR
 // (2k, 2k+1) of a 64-candidate chunk of the group's row spans (packed f32x2
 // operands X = {x0, x1}, Y = {y0, y1}); every query of the group (broadcast
@@ -166,6 +218,7 @@ __global__ void __launch_bounds__(kSearchThreads) k_count(SArgs a, uint32_t g0, 
                                                           uint2* __restrict__ masks, const uint64_t* __restrict__ moff) {
     constexpr bool F64 = MODE != kF32;
     __shared__ uint2 swin[kWarps][32][kWinPad];   // masks of the current window [query][chunk]
+    __shared__ VSpan vsp[kWarps][kMaxSpans + 1];     // the group's spans as one pair sequence
     __shared__ ulonglong2 sq[kWarps][32];           // {{qx, qx}, {qy, qy}} packed f32 pairs
     __shared__ double2 sqd[F64 ? kWarps : 1][32];   // exact query coordinates (f64 modes)
     const int lane = threadIdx.x & 31;
@@ -200,18 +253,16 @@ __global__ void __launch_bounds__(kSearchThreads) k_count(SArgs a, uint32_t g0, 
         }
         uint32_t my = 0;
         uint2* gmask = masks ? masks + (__ldg(&moff[gi]) >> 1) : nullptr;
+        const uint32_t npairs = load_vspans(a, c, vsp[w], lane);
+        const uint32_t nch = (npairs + 31) / 32;
+        uint32_t rs = 0;   // this lane's current span
         uint32_t k = 0;
-        __syncwarp();
 #pragma unroll 1
-        for (uint32_t r = 0; r < a.nspan; ++r) {
-            const uint2 sp = __ldg(&a.cspan[a.nspan * c + r]);
-            const uint32_t lo = sp.x, hi = sp.y;
-            if (lo >= hi) continue;
-#pragma unroll 1
-            for (uint32_t c0 = lo & ~1u; c0 < hi; c0 += 64, ++k) {
+        for (; k < nch; ++k) {
+            {
                 const uint32_t kk = k % kWin;
-                const uint32_t s0 = c0 + 2 * lane, s1 = s0 + 1;
-                const bool v0 = s0 >= lo && s0 < hi, v1 = s1 >= lo && s1 < hi;
+                bool v0, v1;
+                const uint32_t s0 = vpair(vsp[w], a.nspan, 32 * k + lane, rs, v0, v1), s1 = s0 + 1;
                 u64x X, Y;
                 double2 d0 = make_double2(kFarD, kFarD), d1 = make_double2(kFarD, kFarD);
                 if (MODE == kF32) {
@@ -228,7 +279,7 @@ __global__ void __launch_bounds__(kSearchThreads) k_count(SArgs a, uint32_t g0, 
                         Y = pack2(v0 ? (float)__dsub_rn(d0.y, o.y) : kFarF, v1 ? (float)__dsub_rn(d1.y, o.y) : kFarF);
                     }
                 }
-                tests += (unsigned long long)nq * (min(c0 + 64, hi) - max(c0, lo));
+                tests += (unsigned long long)nq * ((v0 ? 1u : 0u) + (v1 ? 1u : 0u));   // per lane; reduced at exit
                 uint32_t acc = 0;   // f64 filter: sign bit set <=> some |t| <= band in this lane
 #pragma unroll 4
                 for (uint32_t i = 0; i < nq; ++i) {
@@ -297,6 +348,8 @@ __global__ void __launch_bounds__(kSearchThreads) k_count(SArgs a, uint32_t g0, 
             gend = min(gi + chunk, g1);
         }
     }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) tests += __shfl_xor_sync(FULL, tests, o);
     if (tests_out && lane == 0 && tests) atomicAdd(tests_out, tests);
 }
 
@@ -483,6 +536,7 @@ __global__ void __launch_bounds__(kEmitThreads) k_emit(SArgs a, uint32_t g0, uin
     // rows padded (80-B / 144-B strides) so the per-lane row accesses are bank-conflict free
     __shared__ __align__(16) uint2 raw[kEmitWarps][32][kWin + 2];   // cp.async landing buffer (next window's masks)
     __shared__ uint4 wq[kEmitWarps][32][kWin + 1];    // current window: {m0, m1, pos0, pos1} per (query, chunk)
+    __shared__ VSpan vsp[kEmitWarps][kMaxSpans + 1];  // the group's spans as one pair sequence
     const int lane = threadIdx.x & 31;
     const int w = threadIdx.x >> 5;
     const unsigned lt = (1u << lane) - 1u;
@@ -499,13 +553,9 @@ __global__ void __launch_bounds__(kEmitThreads) k_emit(SArgs a, uint32_t g0, uin
         asm volatile("mov.b64 %0, %0;" : "+l"(gout));
         uint32_t my = 0;   // lane i: output cursor of query i within the group
         if ((uint32_t)lane < nq) my = (uint32_t)(off[qs + lane] - gb);
-        // chunk iterator over the non-empty spans (same order as the count pass)
-        const uint2* cs = a.cspan + (size_t)a.nspan * c;
-        const uint32_t nspan = a.nspan;
-        uint32_t r = 0;
-        uint2 sp = __ldg(&cs[0]);
-        while (sp.x >= sp.y) sp = __ldg(&cs[++r]);   // the own-row span is never empty
-        uint32_t c0 = sp.x & ~1u, hi = sp.y;
+        // the group's spans as one sequence of candidate pairs (same chunks as the count pass)
+        load_vspans(a, c, vsp[w], lane);
+        uint32_t rs = 0;   // this lane's current span
         __syncwarp();   // the previous group's buffers are no longer read
         if ((uint32_t)lane < nq) {   // prefetch window 0: lane i copies its 64-B mask row
             const uint4* src = (const uint4*)(gmask + (size_t)lane * kWin);
@@ -516,24 +566,13 @@ __global__ void __launch_bounds__(kEmitThreads) k_emit(SArgs a, uint32_t g0, uin
 #pragma unroll 1
         for (uint32_t v = 0; v < nwin; ++v) {
             // this window's candidate ids: lane j holds pair (2j, 2j+1) of each chunk
-            uint2 ids[kWin];
+            uint2 ids[kWin];   // lane j: ids of candidate pair (2j, 2j+1) of each chunk of the window
 #pragma unroll
             for (int kk = 0; kk < kWin; ++kk) {
+                bool v0, v1;
+                const uint32_t s0 = vpair(vsp[w], a.nspan, 32 * (v * kWin + kk) + lane, rs, v0, v1);
                 ids[kk] = make_uint2(0, 0);
-                if (r < nspan) {
-                    if (c0 + 2 * lane < hi) ids[kk] = __ldg((const uint2*)(a.ids + c0 + 2 * lane));
-                    c0 += 64;
-                    if (c0 >= hi) {
-                        while (++r < nspan) {
-                            sp = __ldg(&cs[r]);
-                            if (sp.x < sp.y) break;
-                        }
-                        if (r < nspan) {
-                            c0 = sp.x & ~1u;
-                            hi = sp.y;
-                        }
-                    }
-                }
+                if (v0 | v1) ids[kk] = __ldg((const uint2*)(a.ids + s0));
             }
             cp_async_wait<0>();
             __syncwarp();
@@ -575,17 +614,18 @@ __global__ void __launch_bounds__(kEmitThreads) k_emit(SArgs a, uint32_t g0, uin
     }
 }
 
-// Mask-table layout: words of group g = 2 * nq * (number of 64-candidate chunks of its 3 spans)
+// Mask-table layout: words of group g = 2 * nq * kWin * (windows of kWin chunks of 32 virtual pairs)
 __global__ void __launch_bounds__(256) k_mask_words(SArgs a, uint64_t ng, uint32_t* __restrict__ words) {
     for (uint64_t g = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; g < ng;
          g += (uint64_t)gridDim.x * blockDim.x) {
         const uint32_t qs = a.gstart[g], c = a.gcell[g];
         const uint32_t nq = min((uint32_t)kGroup, a.cstart[c + 1] - qs);
-        uint32_t ch = 0;
+        uint32_t npairs = 0;
         for (uint32_t r = 0; r < a.nspan; ++r) {
             const uint2 sp = a.cspan[a.nspan * c + r];
-            if (sp.y > sp.x) ch += (sp.y - (sp.x & ~1u) + 63) / 64;
+            if (sp.y > sp.x) npairs += ((sp.y + 1) >> 1) - (sp.x >> 1);
         }
+        const uint32_t ch = (npairs + 31) / 32;
         words[g] = 2 * nq * kWin * ((ch + kWin - 1) / kWin);
     }
 }
