@@ -99,6 +99,7 @@ hdb_status hdb_ctx_create(const hdb_opts* opts, hdb_ctx** out) {
             HDB_CUDA(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
             dc.streams.push_back(s);
         }
+        HDB_CUDA(cudaHostAlloc((void**)&dc.pin, 256, cudaHostAllocPortable));
         cudaMemPool_t pool;
         HDB_CUDA(cudaDeviceGetDefaultMemPool(&pool, d));
         uint64_t thr = UINT64_MAX;
@@ -133,6 +134,7 @@ void hdb_ctx_destroy(hdb_ctx* c) {
             if (b) cudaFree(b);
         for (auto s : dc.streams) cudaStreamDestroy(s);
         if (dc.main && dc.own_main) cudaStreamDestroy(dc.main);
+        if (dc.pin) cudaFreeHost(dc.pin);
     }
     cudaSetDevice(prev);
     delete c;

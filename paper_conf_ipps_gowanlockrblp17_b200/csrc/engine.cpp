@@ -440,28 +440,17 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
     pos.reset();
     keys.reset();
     tr.mark("cells+sync");
-    // ---- stencil row spans per non-empty cell + query groups
+    // ---- stencil row spans per non-empty cell + query groups + hit-mask layout,
+    // sized by upper bounds (groups <= n) so that one sync reads both counts
     DBuf cspan(8 * g.nspan * nne, s), gcount(4 * (nne + 1), s), gofs(4 * (nne + 1), s);
     launch_cell_spans(ckey.as<uint64_t>(), cstart.as<uint32_t>(), nne, g.nx, g.ny, g.split, cspan.as<uint2>(),
                       gcount.as<uint32_t>(), s);
     scan_u32_to_u32(gcount.as<uint32_t>(), gofs.as<uint32_t>(), nne, temp.p, s);
     HDB_LAUNCH_CHECK();
-    uint32_t hng = 0;
-    HDB_CUDA(cudaMemcpyAsync(&hng, gofs.as<uint32_t>() + nne, 4, cudaMemcpyDeviceToHost, s));
-    HDB_CUDA(cudaStreamSynchronize(s));
-    g.n_groups = hng;
-    DBuf gstart(4 * (g.n_groups + 1), s), gcell(4 * (g.n_groups + 1), s);
+    DBuf gstart(4 * (n + 1), s), gcell(4 * (n + 1), s);
     launch_group_build(cstart.as<uint32_t>(), gofs.as<uint32_t>(), nne, n, gstart.as<uint32_t>(),
                        gcell.as<uint32_t>(), s);
     HDB_LAUNCH_CHECK();
-    gcount.reset();
-    gofs.reset();
-    temp.reset();
-    misc.reset();
-    HDB_CUDA(cudaEventRecord(ev1.e, s));
-    HDB_CUDA(cudaEventSynchronize(ev1.e));
-    g.ms_build = elapsed(ev0, ev1);
-    tr.mark("groups+sync");
     g.xy_s = xy_s.release();
     g.xp = (float4*)xp.release();
     g.counters = (unsigned int*)counters.release();
@@ -471,17 +460,25 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
     g.cspan = (uint2*)cspan.release();
     g.gstart = (uint32_t*)gstart.release();
     g.gcell = (uint32_t*)gcell.release();
-    // hit-mask table layout of the two-pass search (count stores, write replays)
     {
-        DBuf words(4 * (g.n_groups + 1), s), mtemp(scan_temp_bytes(g.n_groups + 1), s), moff(8 * (g.n_groups + 1), s);
-        launch_mask_words(g, words.as<uint32_t>(), s);
-        scan_u32_to_u64(words.as<uint32_t>(), moff.as<uint64_t>(), g.n_groups, mtemp.p, s);
+        DBuf words(4 * (n + 1), s), mtemp(scan_temp_bytes(n + 1), s), moff(8 * (n + 1), s);
+        launch_mask_words(g, gofs.as<uint32_t>() + nne, n, words.as<uint32_t>(), s);
+        scan_u32_to_u64(words.as<uint32_t>(), moff.as<uint64_t>(), n, mtemp.p, s);
         HDB_LAUNCH_CHECK();
-        HDB_CUDA(cudaMemcpyAsync(&g.mask_words, moff.as<uint64_t>() + g.n_groups, 8, cudaMemcpyDeviceToHost, s));
-        HDB_CUDA(cudaStreamSynchronize(s));
+        uint32_t hng = 0;
+        HDB_CUDA(cudaMemcpyAsync(&hng, gofs.as<uint32_t>() + nne, 4, cudaMemcpyDeviceToHost, s));
+        HDB_CUDA(cudaMemcpyAsync(&g.mask_words, moff.as<uint64_t>() + n, 8, cudaMemcpyDeviceToHost, s));
+        HDB_CUDA(cudaEventRecord(ev1.e, s));
+        HDB_CUDA(cudaEventSynchronize(ev1.e));
+        g.n_groups = hng;
         g.moff = (uint64_t*)moff.release();
     }
-    tr.mark("mask-layout+sync");
+    g.ms_build = elapsed(ev0, ev1);
+    gcount.reset();
+    gofs.reset();
+    temp.reset();
+    misc.reset();
+    tr.mark("groups+mask-layout+sync");
 }
 
 void free_dev_grid(DevGrid& g) {
@@ -836,24 +833,41 @@ void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hd
         const double f = ctx->opts.sample_fraction;
         const uint64_t stride = std::max<uint64_t>(1, (uint64_t)std::floor(1.0 / f));
         const uint64_t ns = n ? (n + stride - 1) / stride : 0;
-        std::vector<uint32_t> samp(ns);
+        std::vector<uint32_t> samp;
+        const uint32_t parts = R_proc * (uint32_t)ndev;
+        cudaStream_t s0 = dc0.main;
+        DBuf dsamp(4 * (ns ? ns : 1), s0), dsum(8, s0);
+        Event es0, es1;
+        HDB_CUDA(cudaMemsetAsync(dsum.p, 0, 8, s0));
+        HDB_CUDA(cudaEventRecord(es0.e, s0));
+        launch_sample_count(G0, stride, ns, dsamp.as<uint32_t>(), dsum.as<unsigned long long>(), s0);
+        HDB_LAUNCH_CHECK();
+        HDB_CUDA(cudaEventRecord(es1.e, s0));
+        // e_b lands in pinned scratch; unsharded calls read it after the count pass's sync
+        HDB_CUDA(cudaMemcpyAsync(dc0.pin, dsum.p, 8, cudaMemcpyDeviceToHost, s0));
+        if (parts > 1 && ns) {   // shard cuts need the per-sample counts now
+            samp.resize(ns);
+            HDB_CUDA(cudaMemcpyAsync(samp.data(), dsamp.p, 4 * ns, cudaMemcpyDeviceToHost, s0));
+            HDB_CUDA(cudaStreamSynchronize(s0));
+        }
+        // ---- query shards: processes x devices, balanced by sampled counts
+        std::vector<uint64_t> cuts = shard_cuts(G0, dc0, samp, stride, parts);
+        for (size_t d = 0; d < ndev; ++d) {
+            const uint32_t k = rank * (uint32_t)ndev + (uint32_t)d;
+            sh[d].r.g0 = cuts[k];
+            sh[d].r.g1 = cuts[k + 1];
+        }
+        tr.mark("sample+cuts");
+        // ---- a6/a7 on every device
+        run_parallel(ndev, [&](size_t d) { count_phase(ctx, ctx->dev[d], grid->dev[d], sh[d]); });
+        tr.mark("count_phase");
+        HDB_CUDA(cudaStreamSynchronize(s0));   // no-op when device 0 ran the count pass (same stream)
         {
-            cudaStream_t s = dc0.main;
-            DBuf dsamp(4 * (ns ? ns : 1), s), dsum(8, s);
-            HDB_CUDA(cudaMemsetAsync(dsum.p, 0, 8, s));
-            Event e0, e1;
-            HDB_CUDA(cudaEventRecord(e0.e, s));
-            launch_sample_count(G0, stride, ns, dsamp.as<uint32_t>(), dsum.as<unsigned long long>(), s);
-            HDB_LAUNCH_CHECK();
-            HDB_CUDA(cudaEventRecord(e1.e, s));
-            uint64_t eb = 0;
-            HDB_CUDA(cudaMemcpyAsync(&eb, dsum.p, 8, cudaMemcpyDeviceToHost, s));
-            if (ns) HDB_CUDA(cudaMemcpyAsync(samp.data(), dsamp.p, 4 * ns, cudaMemcpyDeviceToHost, s));
-            HDB_CUDA(cudaStreamSynchronize(s));
+            const uint64_t eb = dc0.pin[0];
             S.sample_size = ns;
             S.sample_pairs = eb;
             S.est_pairs = eb * stride;   // a_b = e_b / f  (reading R15)
-            S.ms_sample = elapsed(e0, e1);
+            S.ms_sample = elapsed(es0, es1);
         }
         double bb_plan = 0;
         uint64_t nb_plan = 0;
@@ -864,19 +878,6 @@ void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hd
         S.planned_batches = ctx->opts.batch_pairs
                                 ? (uint64_t)std::ceil((1.0 + ctx->opts.alpha) * (double)S.est_pairs / (double)batch_pairs)
                                 : nb_plan;
-
-        tr.mark("sample+sync");
-        // ---- query shards: processes x devices, balanced by sampled counts
-        const uint32_t parts = R_proc * (uint32_t)ndev;
-        std::vector<uint64_t> cuts = shard_cuts(G0, dc0, samp, stride, parts);
-        for (size_t d = 0; d < ndev; ++d) {
-            const uint32_t k = rank * (uint32_t)ndev + (uint32_t)d;
-            sh[d].r.g0 = cuts[k];
-            sh[d].r.g1 = cuts[k + 1];
-        }
-        // ---- a6/a7 on every device
-        run_parallel(ndev, [&](size_t d) { count_phase(ctx, ctx->dev[d], grid->dev[d], sh[d]); });
-        tr.mark("count_phase");
         // ---- the final gather of counts: shard bases
         uint64_t P = 0;
         for (size_t d = 0; d < ndev; ++d) {

@@ -123,8 +123,8 @@ void launch_count(const DevGrid& g, uint64_t g0, uint64_t g1, uint32_t* cnt, uns
 // masks != null: emit from the stored hit masks; null: recompute the tests.
 void launch_write(const DevGrid& g, uint64_t g0, uint64_t g1, const uint64_t* off, uint64_t out_base,
                   uint32_t* out, int variant, int slot, const uint2* masks, cudaStream_t s);
-// words[g] = 32-bit words of group g's hit masks (scan -> g.moff)
-void launch_mask_words(const DevGrid& g, uint32_t* words, cudaStream_t s);
+// words[g] = 32-bit words of group g's hit masks for g < *ng_dev, 0 for g in [*ng_dev, n) (scan -> g.moff)
+void launch_mask_words(const DevGrid& g, const uint32_t* ng_dev, uint64_t n, uint32_t* words, cudaStream_t s);
 // cuts: for b in 0..nb, gcut[b] = first group g in [g0,g1] with off[gstart[g]] >= target_b,
 // target_b = off[gstart[g0]] + b * span / nb (gcut[0] = g0, gcut[nb] = g1); pcut[b] = off[gstart[gcut[b]]]
 void launch_batch_cuts(const uint32_t* gstart, const uint64_t* off, uint64_t g0, uint64_t g1, uint32_t nb,
@@ -157,6 +157,7 @@ struct DevCtx {
     bool own_main = true;
     std::vector<cudaStream_t> streams;     // write + D2H streams
     std::vector<cudaEvent_t> ev_pool;
+    uint64_t* pin = nullptr;                // small pinned scratch for async readbacks
     // cached per-stream device batch buffers (reused across calls)
     std::vector<uint32_t*> batch_buf;
     std::vector<size_t> batch_cap;

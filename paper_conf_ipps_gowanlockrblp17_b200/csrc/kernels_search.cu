@@ -615,9 +615,15 @@ __global__ void __launch_bounds__(kEmitThreads) k_emit(SArgs a, uint32_t g0, uin
 }
 
 // Mask-table layout: words of group g = 2 * nq * kWin * (windows of kWin chunks of 32 virtual pairs)
-__global__ void __launch_bounds__(256) k_mask_words(SArgs a, uint64_t ng, uint32_t* __restrict__ words) {
-    for (uint64_t g = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; g < ng;
+__global__ void __launch_bounds__(256) k_mask_words(SArgs a, const uint32_t* __restrict__ ng_dev, uint64_t n,
+                                                    uint32_t* __restrict__ words) {
+    const uint64_t ng = *ng_dev;
+    for (uint64_t g = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; g < n;
          g += (uint64_t)gridDim.x * blockDim.x) {
+        if (g >= ng) {
+            words[g] = 0;
+            continue;
+        }
         const uint32_t qs = a.gstart[g], c = a.gcell[g];
         const uint32_t nq = min((uint32_t)kGroup, a.cstart[c + 1] - qs);
         uint32_t npairs = 0;
@@ -871,10 +877,9 @@ void launch_write(const DevGrid& g, uint64_t g0, uint64_t g1, const uint64_t* of
     ++g_kernel_launches;
 }
 
-void launch_mask_words(const DevGrid& g, uint32_t* words, cudaStream_t s) {
-    if (g.n_groups == 0) return;
-    unsigned blocks = (unsigned)std::min<uint64_t>((g.n_groups + 255) / 256, 148 * 16);
-    k_mask_words<<<blocks, 256, 0, s>>>(args_of(g), g.n_groups, words);
+void launch_mask_words(const DevGrid& g, const uint32_t* ng_dev, uint64_t n, uint32_t* words, cudaStream_t s) {
+    unsigned blocks = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>((n + 255) / 256, 148 * 16));
+    k_mask_words<<<blocks, 256, 0, s>>>(args_of(g), ng_dev, n, words);
     ++g_kernel_launches;
 }
 
