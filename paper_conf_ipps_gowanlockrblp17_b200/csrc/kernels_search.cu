@@ -87,6 +87,11 @@ __device__ __forceinline__ void stg_if(uint32_t* p, uint32_t v, bool f) {
     asm volatile("{ .reg .pred q; setp.ne.b32 q, %2, 0; @q st.global.u32 [%0], %1; }" ::"l"(p), "r"(v),
                  "r"((uint32_t)f));
 }
+// store v at p iff (m & bit) != 0 -- the mask test inside the asm keeps it one LOP3.P
+__device__ __forceinline__ void stg_if_bit(uint32_t* p, uint32_t v, uint32_t m, uint32_t bit) {
+    asm volatile("{ .reg .pred q; .reg .b32 t; and.b32 t, %2, %3; setp.ne.b32 q, t, 0; @q st.global.u32 [%0], %1; }" ::"l"(p),
+                 "r"(v), "r"(m), "r"(bit));
+}
 __device__ __forceinline__ u64x fma2(u64x a, u64x b, u64x c) {
     u64x r;
     asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(r) : "l"(a), "l"(b), "l"(c));
@@ -539,7 +544,7 @@ __global__ void __launch_bounds__(kEmitThreads) k_emit(SArgs a, uint32_t g0, uin
     __shared__ VSpan vsp[kEmitWarps][kMaxSpans + 1];  // the group's spans as one pair sequence
     const int lane = threadIdx.x & 31;
     const int w = threadIdx.x >> 5;
-    const unsigned lt = (1u << lane) - 1u;
+    const unsigned lt = (1u << lane) - 1u, lbit = 1u << lane;
     uint32_t gi = g0 + grab(ctr, chunk, lane), gend = min(gi + chunk, g1);
     while (gi < g1) {
         const uint32_t qs = __ldg(&a.gstart[gi]);
@@ -600,8 +605,8 @@ __global__ void __launch_bounds__(kEmitThreads) k_emit(SArgs a, uint32_t g0, uin
 #pragma unroll
                 for (int kk = 0; kk < kWin; ++kk) {
                     const uint4 e = wq[w][i][kk];   // broadcast
-                    stg_if(gout + (e.z + __popc(e.x & lt)), ids[kk].x, (e.x >> lane) & 1u);
-                    stg_if(gout + (e.w + __popc(e.y & lt)), ids[kk].y, (e.y >> lane) & 1u);
+                    stg_if_bit(gout + (e.z + __popc(e.x & lt)), ids[kk].x, e.x, lbit);
+                    stg_if_bit(gout + (e.w + __popc(e.y & lt)), ids[kk].y, e.y, lbit);
                 }
             }
             __syncwarp();   // wq is rewritten for the next window
