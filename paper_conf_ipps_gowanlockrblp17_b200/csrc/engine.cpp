@@ -394,16 +394,16 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
     // ---- a2: keys
     // ids and points are padded by 2 entries: the search kernels load candidate
     // pairs (2k, 2k+1) with one vector load and mask the invalid half
-    DBuf k0(8 * n, s), v0(4 * (n + 2), s), k1(8 * n, s), v1(4 * (n + 2), s);
-    launch_keys(xin, n, dt, g.xmin, g.ymin, g.inv_w, g.nx, g.ny, k0.as<uint64_t>(), v0.as<uint32_t>(), s);
+    const int kb = g.n_cells <= (1ull << 32) ? 4 : 8;   // 32-bit keys whenever they fit
+    DBuf k0(kb * n, s), v0(4 * (n + 2), s), k1(kb * n, s), v1(4 * (n + 2), s);
+    launch_keys(xin, n, dt, g.xmin, g.ymin, g.inv_w, g.nx, g.ny, k0.p, kb, v0.as<uint32_t>(), s);
     HDB_LAUNCH_CHECK();
     // ---- a3: stable radix sort by key (only the bits the key range needs)
     int bits = 1;
     while (bits < 64 && (1ull << bits) < g.n_cells) ++bits;
     size_t tb = std::max(radix_sort_temp_bytes(n), scan_temp_bytes(n + 1));
     DBuf temp(tb, s);
-    int which = radix_sort_pairs(k0.as<uint64_t>(), v0.as<uint32_t>(), k1.as<uint64_t>(), v1.as<uint32_t>(), n,
-                                 bits, temp.p, s);
+    int which = radix_sort_pairs(k0.p, v0.as<uint32_t>(), k1.p, v1.as<uint32_t>(), kb, n, bits, temp.p, s);
     HDB_LAUNCH_CHECK();
     DBuf keys = which ? std::move(k1) : std::move(k0);
     DBuf ids = which ? std::move(v1) : std::move(v0);
@@ -424,7 +424,7 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
     tr.mark("keys+sort+gather(enqueue)");
     // ---- a4: run boundaries -> scan -> (key, start) of the non-empty cells
     DBuf flags(4 * n, s), pos(4 * (n + 1), s);
-    launch_cell_flags(keys.as<uint64_t>(), n, flags.as<uint32_t>(), s);
+    launch_cell_flags(keys.p, kb, n, flags.as<uint32_t>(), s);
     scan_u32_to_u32(flags.as<uint32_t>(), pos.as<uint32_t>(), n, temp.p, s);
     HDB_LAUNCH_CHECK();
     uint32_t hne = 0;
@@ -433,7 +433,7 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
     g.n_nonempty = hne;
     const uint64_t nne = hne;
     DBuf ckey(8 * nne, s), cstart(4 * (nne + 1), s);
-    launch_cell_scatter(keys.as<uint64_t>(), flags.as<uint32_t>(), pos.as<uint32_t>(), n, ckey.as<uint64_t>(),
+    launch_cell_scatter(keys.p, kb, flags.as<uint32_t>(), pos.as<uint32_t>(), n, ckey.as<uint64_t>(),
                         cstart.as<uint32_t>(), s);
     HDB_LAUNCH_CHECK();
     flags.reset();

@@ -83,19 +83,20 @@ void launch_bbox_init(unsigned long long* bb, unsigned int* bad, cudaStream_t s)
 void launch_bbox(const void* xy, uint64_t n, hdb_dtype dt, unsigned long long* bb, unsigned int* bad,
                  cudaStream_t s);
 double bbox_decode(unsigned long long v, bool is_max);
+// keys: key_bytes = 4 (grids of <= 2^32 cells) or 8
 void launch_keys(const void* xy, uint64_t n, hdb_dtype dt, double xmin, double ymin, double inv_w,
-                 uint32_t nx, uint32_t ny, uint64_t* keys, uint32_t* vals, cudaStream_t s);
+                 uint32_t nx, uint32_t ny, void* keys, int key_bytes, uint32_t* vals, cudaStream_t s);
 size_t radix_sort_temp_bytes(uint64_t n);
 // Stable LSD radix sort of (keys, vals) on the low `bits` bits.  Ping-pongs
 // between (k0,v0) and (k1,v1); returns 0 if the result is in (k0,v0), 1 else.
-int radix_sort_pairs(uint64_t* k0, uint32_t* v0, uint64_t* k1, uint32_t* v1, uint64_t n, int bits,
+int radix_sort_pairs(void* k0, uint32_t* v0, void* k1, uint32_t* v1, int key_bytes, uint64_t n, int bits,
                      void* temp, cudaStream_t s);
 // gather sorted points; f64 mode also writes the f32 filter coordinates (x-ox, y-oy)
 void launch_gather_points(const void* xy_in, const uint32_t* ids, uint64_t n, hdb_dtype dt, void* xy_s,
                           float4* xp, double ox, double oy, cudaStream_t s);
-void launch_cell_flags(const uint64_t* keys_sorted, uint64_t n, uint32_t* flags, cudaStream_t s);
-void launch_cell_scatter(const uint64_t* keys_sorted, const uint32_t* flags, const uint32_t* pos, uint64_t n,
-                         uint64_t* ckey, uint32_t* cstart, cudaStream_t s);
+void launch_cell_flags(const void* keys_sorted, int key_bytes, uint64_t n, uint32_t* flags, cudaStream_t s);
+void launch_cell_scatter(const void* keys_sorted, int key_bytes, const uint32_t* flags, const uint32_t* pos,
+                         uint64_t n, uint64_t* ckey, uint32_t* cstart, cudaStream_t s);
 void launch_cell_spans(const uint64_t* ckey, const uint32_t* cstart, uint64_t nne, uint32_t nx, uint32_t ny,
                        uint32_t k, uint2* cspan, uint32_t* gcount, cudaStream_t s);
 // auto cell split: sample-based point-weighted occupancy at cell width 1/inv_w;

@@ -96,10 +96,11 @@ __global__ void __launch_bounds__(256) k_bbox(const typename V2<T>::type* __rest
 }
 
 // a2: cell keys.  FP64 cell arithmetic with explicitly rounded ops (no FMA).
-template <typename T>
+// Keys are 32-bit when the grid has <= 2^32 cells (halves the sort traffic).
+template <typename T, typename K>
 __global__ void __launch_bounds__(256) k_keys(const typename V2<T>::type* __restrict__ xy, uint64_t n,
                                               double xmin, double ymin, double inv_w, uint32_t nx,
-                                              uint32_t ny, uint64_t* __restrict__ keys,
+                                              uint32_t ny, K* __restrict__ keys,
                                               uint32_t* __restrict__ vals) {
     for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n;
          i += (uint64_t)gridDim.x * blockDim.x) {
@@ -108,30 +109,39 @@ __global__ void __launch_bounds__(256) k_keys(const typename V2<T>::type* __rest
         double ty = floor(__dmul_rn(__dsub_rn((double)p.y, ymin), inv_w));
         uint64_t cx = (uint64_t)fmin(fmax(tx, 0.0), (double)(nx - 1));
         uint64_t cy = (uint64_t)fmin(fmax(ty, 0.0), (double)(ny - 1));
-        keys[i] = cy * nx + cx;
+        keys[i] = (K)(cy * nx + cx);
         vals[i] = (uint32_t)i;
     }
 }
 
 // ---------------------------------------------------------------- radix sort
+// Stable LSD radix sort of (key, id), 8-bit digits.  Per pass: a per-tile digit
+// histogram, a scan of the (digit, tile) counts, and a scatter that ranks each
+// tile's keys stably (warp match_any ranks + warp-ordered prefixes), stages them
+// in shared memory in digit order, and writes every digit's run of the tile
+// contiguously (coalesced) to its global position.
 constexpr int RS_THREADS = 256;
 constexpr int RS_WARPS = RS_THREADS / 32;
-constexpr int RS_ITEMS = 16;                         // per thread
-constexpr int RS_TILE = RS_THREADS * RS_ITEMS;       // 4096 keys per CTA
 constexpr int RS_BITS = 8;
 constexpr int RS_BINS = 1 << RS_BITS;
+template <typename K>
+struct RsCfg {
+    static constexpr int ITEMS = sizeof(K) == 4 ? 16 : 8;       // per thread
+    static constexpr int TILE = RS_THREADS * ITEMS;             // 4096 (u32) / 2048 (u64) keys per CTA
+};
 
-__global__ void __launch_bounds__(RS_THREADS) k_radix_hist(const uint64_t* __restrict__ keys, uint64_t n,
-                                                           int shift, uint32_t* __restrict__ hist,
-                                                           uint32_t nblocks) {
+template <typename K>
+__global__ void __launch_bounds__(RS_THREADS) k_radix_hist(const K* __restrict__ keys, uint64_t n, int shift,
+                                                           uint32_t* __restrict__ hist, uint32_t nblocks) {
+    constexpr int ITEMS = RsCfg<K>::ITEMS, TILE = RsCfg<K>::TILE;
     __shared__ uint32_t h[RS_BINS];
     const int tid = threadIdx.x;
     const int lane = tid & 31;
     h[tid] = 0;
     __syncthreads();
-    const uint64_t base = (uint64_t)blockIdx.x * RS_TILE;
+    const uint64_t base = (uint64_t)blockIdx.x * TILE;
 #pragma unroll 4
-    for (int r = 0; r < RS_ITEMS; ++r) {
+    for (int r = 0; r < ITEMS; ++r) {
         uint64_t idx = base + (uint64_t)r * RS_THREADS + tid;
         bool valid = idx < n;
         uint32_t d = valid ? (uint32_t)((keys[idx] >> shift) & (RS_BINS - 1)) : (0x100u + lane);
@@ -142,32 +152,33 @@ __global__ void __launch_bounds__(RS_THREADS) k_radix_hist(const uint64_t* __res
     hist[(uint64_t)tid * nblocks + blockIdx.x] = h[tid];
 }
 
-// Stable scatter: warp w owns keys [w*512, (w+1)*512) of the tile, processed in
-// 16 rounds of 32 consecutive keys; the rank of a key is the number of earlier
-// keys of the same digit in (earlier warps of the tile, earlier rounds of this
-// warp, lower lanes of this round) plus the digit's global base for the tile.
-__global__ void __launch_bounds__(RS_THREADS) k_radix_scatter(const uint64_t* __restrict__ kin,
+template <typename K>
+__global__ void __launch_bounds__(RS_THREADS) k_radix_scatter(const K* __restrict__ kin,
                                                               const uint32_t* __restrict__ vin,
-                                                              uint64_t* __restrict__ kout,
-                                                              uint32_t* __restrict__ vout, uint64_t n,
-                                                              int shift, const uint32_t* __restrict__ hscan,
-                                                              uint32_t nblocks) {
+                                                              K* __restrict__ kout, uint32_t* __restrict__ vout,
+                                                              uint64_t n, int shift,
+                                                              const uint32_t* __restrict__ hscan, uint32_t nblocks) {
+    constexpr int ITEMS = RsCfg<K>::ITEMS, TILE = RsCfg<K>::TILE;
     __shared__ uint32_t wcnt[RS_WARPS][RS_BINS];
-    __shared__ uint32_t gbase[RS_BINS];
+    __shared__ uint32_t gbase[RS_BINS];     // global start of each digit's run of this tile
+    __shared__ uint32_t dstart[RS_BINS];    // tile-local start of each digit
+    __shared__ K skey[TILE];
+    __shared__ uint32_t sval[TILE];
     const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
 #pragma unroll
     for (int i = 0; i < RS_WARPS; ++i) wcnt[i][tid] = 0;
     gbase[tid] = hscan[(uint64_t)tid * nblocks + blockIdx.x];
     __syncthreads();
-    const uint64_t base = (uint64_t)blockIdx.x * RS_TILE + (uint64_t)w * (RS_ITEMS * 32);
+    const uint64_t tbase = (uint64_t)blockIdx.x * TILE;
+    const uint64_t base = tbase + (uint64_t)w * (ITEMS * 32);
     const unsigned lt = (1u << lane) - 1u;
-    uint64_t key[RS_ITEMS];
-    uint32_t val[RS_ITEMS], rank[RS_ITEMS];
+    K key[ITEMS];
+    uint32_t val[ITEMS], rank[ITEMS];
 #pragma unroll
-    for (int r = 0; r < RS_ITEMS; ++r) {
+    for (int r = 0; r < ITEMS; ++r) {
         uint64_t idx = base + (uint64_t)r * 32 + lane;
         bool valid = idx < n;
-        key[r] = valid ? kin[idx] : 0ull;
+        key[r] = valid ? kin[idx] : (K)0;
         val[r] = valid ? vin[idx] : 0u;
         uint32_t d = valid ? (uint32_t)((key[r] >> shift) & (RS_BINS - 1)) : (0x100u + lane);
         unsigned peers = __match_any_sync(FULL, d);
@@ -178,25 +189,49 @@ __global__ void __launch_bounds__(RS_THREADS) k_radix_scatter(const uint64_t* __
         __syncwarp();
     }
     __syncthreads();
-    {
-        uint32_t s = 0;
+    // per digit: exclusive prefix over the warps, and the digit's tile total
+    uint32_t tot = 0;
 #pragma unroll
-        for (int i = 0; i < RS_WARPS; ++i) {
-            uint32_t t = wcnt[i][tid];
-            wcnt[i][tid] = s;
-            s += t;
-        }
+    for (int i = 0; i < RS_WARPS; ++i) {
+        uint32_t t = wcnt[i][tid];
+        wcnt[i][tid] = tot;
+        tot += t;
     }
-    __syncthreads();
+    // exclusive scan of the 256 digit totals (warp shuffles + the 8 warp sums)
+    __shared__ uint32_t wsum[RS_WARPS];
+    uint32_t incl = tot;
 #pragma unroll
-    for (int r = 0; r < RS_ITEMS; ++r) {
+    for (int o = 1; o < 32; o <<= 1) {
+        uint32_t y = __shfl_up_sync(FULL, incl, o);
+        if (lane >= o) incl += y;
+    }
+    if (lane == 31) wsum[w] = incl;
+    __syncthreads();
+    uint32_t wpre = 0;
+#pragma unroll
+    for (int i = 0; i < RS_WARPS; ++i) wpre += i < w ? wsum[i] : 0u;
+    dstart[tid] = wpre + incl - tot;
+    __syncthreads();
+    // stage in digit order
+#pragma unroll
+    for (int r = 0; r < ITEMS; ++r) {
         uint64_t idx = base + (uint64_t)r * 32 + lane;
         if (idx < n) {
             uint32_t d = (uint32_t)((key[r] >> shift) & (RS_BINS - 1));
-            uint32_t pos = gbase[d] + wcnt[w][d] + rank[r];
-            kout[pos] = key[r];
-            vout[pos] = val[r];
+            uint32_t lp = dstart[d] + wcnt[w][d] + rank[r];
+            skey[lp] = key[r];
+            sval[lp] = val[r];
         }
+    }
+    __syncthreads();
+    // write each digit's run contiguously
+    const uint32_t cnt = (uint32_t)min((uint64_t)TILE, n - tbase);
+    for (uint32_t i = tid; i < cnt; i += RS_THREADS) {
+        const K k = skey[i];
+        const uint32_t d = (uint32_t)((k >> shift) & (RS_BINS - 1));
+        const uint32_t pos = gbase[d] + (i - dstart[d]);
+        kout[pos] = k;
+        vout[pos] = sval[i];
     }
 }
 
@@ -227,21 +262,23 @@ __global__ void __launch_bounds__(256) k_gather(const typename V2<T>::type* __re
 }
 
 // a4: run boundaries of the sorted keys
-__global__ void __launch_bounds__(256) k_cell_flags(const uint64_t* __restrict__ keys, uint64_t n,
+template <typename K>
+__global__ void __launch_bounds__(256) k_cell_flags(const K* __restrict__ keys, uint64_t n,
                                                     uint32_t* __restrict__ flags) {
     for (uint64_t s = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; s < n;
          s += (uint64_t)gridDim.x * blockDim.x)
         flags[s] = (s == 0 || keys[s] != keys[s - 1]) ? 1u : 0u;
 }
 
-__global__ void __launch_bounds__(256) k_cell_scatter(const uint64_t* __restrict__ keys,
+template <typename K>
+__global__ void __launch_bounds__(256) k_cell_scatter(const K* __restrict__ keys,
                                                       const uint32_t* __restrict__ flags,
                                                       const uint32_t* __restrict__ pos, uint64_t n,
                                                       uint64_t* __restrict__ ckey, uint32_t* __restrict__ cstart) {
     for (uint64_t s = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; s < n;
          s += (uint64_t)gridDim.x * blockDim.x)
         if (flags[s]) {
-            ckey[pos[s]] = keys[s];
+            ckey[pos[s]] = (uint64_t)keys[s];
             cstart[pos[s]] = (uint32_t)s;
         }
     if (blockIdx.x == 0 && threadIdx.x == 0) cstart[pos[n]] = (uint32_t)n;
@@ -402,43 +439,57 @@ void launch_bbox(const void* xy, uint64_t n, hdb_dtype dt, unsigned long long* b
 }
 
 void launch_keys(const void* xy, uint64_t n, hdb_dtype dt, double xmin, double ymin, double inv_w,
-                 uint32_t nx, uint32_t ny, uint64_t* keys, uint32_t* vals, cudaStream_t s) {
+                 uint32_t nx, uint32_t ny, void* keys, int key_bytes, uint32_t* vals, cudaStream_t s) {
     if (n == 0) return;
-    if (dt == HDB_F64)
-        k_keys<double><<<grid_for(n), 256, 0, s>>>((const double2*)xy, n, xmin, ymin, inv_w, nx, ny, keys, vals);
-    else
-        k_keys<float><<<grid_for(n), 256, 0, s>>>((const float2*)xy, n, xmin, ymin, inv_w, nx, ny, keys, vals);
+#define HDB_KEYS(T, K) \
+    k_keys<T, K><<<grid_for(n), 256, 0, s>>>((const V2<T>::type*)xy, n, xmin, ymin, inv_w, nx, ny, (K*)keys, vals)
+    if (dt == HDB_F64) {
+        if (key_bytes == 4) HDB_KEYS(double, uint32_t);
+        else HDB_KEYS(double, uint64_t);
+    } else {
+        if (key_bytes == 4) HDB_KEYS(float, uint32_t);
+        else HDB_KEYS(float, uint64_t);
+    }
+#undef HDB_KEYS
     ++g_kernel_launches;
 }
 
 size_t radix_sort_temp_bytes(uint64_t n) {
-    uint64_t nblocks = (n + RS_TILE - 1) / RS_TILE;
+    uint64_t nblocks = (n + RsCfg<uint64_t>::TILE - 1) / RsCfg<uint64_t>::TILE;   // the smaller tile: upper bound
     uint64_t m = nblocks * RS_BINS;
     return (m + 1) * sizeof(uint32_t) * 2 + scan_temp_bytes(m) + 256;
 }
 
-int radix_sort_pairs(uint64_t* k0, uint32_t* v0, uint64_t* k1, uint32_t* v1, uint64_t n, int bits, void* temp,
-                     cudaStream_t s) {
+template <typename K>
+int radix_sort_impl(K* k0, uint32_t* v0, K* k1, uint32_t* v1, uint64_t n, int bits, void* temp, cudaStream_t s) {
     if (n <= 1 || bits <= 0) return 0;
-    uint32_t nblocks = (uint32_t)((n + RS_TILE - 1) / RS_TILE);
+    constexpr int TILE = RsCfg<K>::TILE;
+    uint32_t nblocks = (uint32_t)((n + TILE - 1) / TILE);
     uint64_t m = (uint64_t)nblocks * RS_BINS;
     uint32_t* hist = (uint32_t*)temp;
     uint32_t* hscan = hist + (m + 1);
     void* stemp = (void*)(((uintptr_t)(hscan + m + 1) + 255) & ~(uintptr_t)255);
     int cur = 0;
     for (int shift = 0; shift < bits; shift += RS_BITS) {
-        uint64_t* ki = cur ? k1 : k0;
+        K* ki = cur ? k1 : k0;
         uint32_t* vi = cur ? v1 : v0;
-        uint64_t* ko = cur ? k0 : k1;
+        K* ko = cur ? k0 : k1;
         uint32_t* vo = cur ? v0 : v1;
-        k_radix_hist<<<nblocks, RS_THREADS, 0, s>>>(ki, n, shift, hist, nblocks);
+        k_radix_hist<K><<<nblocks, RS_THREADS, 0, s>>>(ki, n, shift, hist, nblocks);
         ++g_kernel_launches;
         scan_u32_to_u32(hist, hscan, m, stemp, s);
-        k_radix_scatter<<<nblocks, RS_THREADS, 0, s>>>(ki, vi, ko, vo, n, shift, hscan, nblocks);
+        k_radix_scatter<K><<<nblocks, RS_THREADS, 0, s>>>(ki, vi, ko, vo, n, shift, hscan, nblocks);
         ++g_kernel_launches;
         cur ^= 1;
     }
     return cur;
+}
+
+int radix_sort_pairs(void* k0, uint32_t* v0, void* k1, uint32_t* v1, int key_bytes, uint64_t n, int bits, void* temp,
+                     cudaStream_t s) {
+    if (key_bytes == 4)
+        return radix_sort_impl<uint32_t>((uint32_t*)k0, v0, (uint32_t*)k1, v1, n, bits, temp, s);
+    return radix_sort_impl<uint64_t>((uint64_t*)k0, v0, (uint64_t*)k1, v1, n, bits, temp, s);
 }
 
 void launch_gather_points(const void* xy_in, const uint32_t* ids, uint64_t n, hdb_dtype dt, void* xy_s, float4* xp,
@@ -451,15 +502,21 @@ void launch_gather_points(const void* xy_in, const uint32_t* ids, uint64_t n, hd
     ++g_kernel_launches;
 }
 
-void launch_cell_flags(const uint64_t* keys_sorted, uint64_t n, uint32_t* flags, cudaStream_t s) {
+void launch_cell_flags(const void* keys_sorted, int key_bytes, uint64_t n, uint32_t* flags, cudaStream_t s) {
     if (n == 0) return;
-    k_cell_flags<<<grid_for(n), 256, 0, s>>>(keys_sorted, n, flags);
+    if (key_bytes == 4)
+        k_cell_flags<uint32_t><<<grid_for(n), 256, 0, s>>>((const uint32_t*)keys_sorted, n, flags);
+    else
+        k_cell_flags<uint64_t><<<grid_for(n), 256, 0, s>>>((const uint64_t*)keys_sorted, n, flags);
     ++g_kernel_launches;
 }
 
-void launch_cell_scatter(const uint64_t* keys_sorted, const uint32_t* flags, const uint32_t* pos, uint64_t n,
-                         uint64_t* ckey, uint32_t* cstart, cudaStream_t s) {
-    k_cell_scatter<<<grid_for(n), 256, 0, s>>>(keys_sorted, flags, pos, n, ckey, cstart);
+void launch_cell_scatter(const void* keys_sorted, int key_bytes, const uint32_t* flags, const uint32_t* pos,
+                         uint64_t n, uint64_t* ckey, uint32_t* cstart, cudaStream_t s) {
+    if (key_bytes == 4)
+        k_cell_scatter<uint32_t><<<grid_for(n), 256, 0, s>>>((const uint32_t*)keys_sorted, flags, pos, n, ckey, cstart);
+    else
+        k_cell_scatter<uint64_t><<<grid_for(n), 256, 0, s>>>((const uint64_t*)keys_sorted, flags, pos, n, ckey, cstart);
     ++g_kernel_launches;
 }
 
