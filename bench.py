@@ -128,6 +128,31 @@ def cpu_baseline_run(xy, eps, budget_s=12.0, rows=None, dtype="f64"):
                        f"({pairs} pairs, {rows.size * n:.3g} tests, {dt:.2f} s)"), rows
 
 
+def cpu_gridjoin_run(xy, eps, dtype="f64", budget_s=4.0):
+    """CPU grid-join comparator (cpu_baseline/, SURVEY 8(d) baselines 2 and 3):
+    one core, then all cores, on an evenly spaced sample of query rows against
+    the full grid; the grid build over all n points is timed separately."""
+    import cpu_baseline
+    n = xy.shape[0]
+    probe = np.linspace(0, n - 1, min(n, 2000)).astype(np.int64)
+    t = {}
+    cpu_baseline.gridjoin_rows(xy, eps, probe, dtype=dtype, threads=1, timings=t)
+    m = int(min(n, max(2000, 2000 * budget_s / max(t["join_s"], 1e-4))))
+    rows = np.linspace(0, n - 1, m).astype(np.int64)
+    out = {}
+    cores = os.cpu_count() or 1
+    for key, th in (("single_thread", 1), ("all_cores", cores)):
+        t = {}
+        off, _ = cpu_baseline.gridjoin_rows(xy, eps, rows, dtype=dtype, threads=th, timings=t)
+        pairs = int(off[-1])
+        out[key] = dict(value=pairs / t["join_s"], unit="pairs/s", cores=th, kind="cpu_grid_join",
+                        grid_build_s=t["build_s"],
+                        sample=f"{m} evenly spaced query rows vs the eps-grid of all {n} points "
+                               f"({pairs} pairs, join {t['join_s']:.2f} s; grid build over all n "
+                               f"{t['build_s']:.2f} s, 1 thread, qsort)")
+    return out
+
+
 def run_reference(args, wl, ws, rank):
     if rank != 0:
         return
@@ -340,6 +365,7 @@ def main():
         line["e2e"] = None
     if rank == 0 and not args.no_cpu_baseline:
         line["cpu_baseline"], _ = cpu_baseline_run(xy_np, eps, dtype=args.dtype)
+        line["cpu_baseline"]["grid_join"] = cpu_gridjoin_run(xy_np, eps, dtype=args.dtype)
     hdb.hdb_ctx_destroy(ctx)
     if rank == 0:
         print(json.dumps(line), flush=True)

@@ -7,6 +7,7 @@ Plain CPU implementation of what the HYBRID-DBSCAN hot path computes
 * ``eps_join``        -- O2, the neighbour table T by brute force.
 * ``eps_join_rows``   -- O2 restricted to sampled query rows (each vs all n).
 * ``eps_join_rowhash``-- O2 streamed as per-row (count, order-free hash).
+* ``sweep_rowhash``   -- O2 by an x-sorted plane sweep (the R-tree-free scan).
 * ``dbscan``          -- O3, Algorithm 1 on T.
 * ``hybrid_dbscan``   -- Algorithm 4 with the GPU steps replaced by O2.
 
@@ -64,6 +65,8 @@ def _load():
             getattr(lib, f"oracle_join_count_{t}").argtypes = [P, i64, et, P, i64, P]
             getattr(lib, f"oracle_join_fill_{t}").argtypes = [P, i64, et, P, i64, P, P]
             getattr(lib, f"oracle_join_rowhash_{t}").argtypes = [P, i64, et, P, i64, P, P]
+            getattr(lib, f"oracle_sweep_rowhash_{t}").argtypes = [P, i64, et, P, P]
+            getattr(lib, f"oracle_sweep_rowhash_{t}").restype = ctypes.c_int
         lib.oracle_dbscan.argtypes = [P, P, i64, u64, P, P]
         lib.oracle_dbscan.restype = i64
         _lib = lib
@@ -137,6 +140,19 @@ def eps_join_rowhash(xy, eps, rows=None, dtype="f64"):
     h = np.zeros(nrows, dtype=np.uint64)
     getattr(lib, f"oracle_join_rowhash_{dtype}")(_ptr(xy), n, float(npdt(eps)), _ptr(rptr), nrows,
                                                  _ptr(cnt), _ptr(h))
+    return cnt, h
+
+
+def sweep_rowhash(xy, eps, dtype="f64"):
+    """O2 by the x-sorted plane sweep (no cells): per-row (count, hash) for all
+    rows, equal to ``eps_join_rowhash`` by construction (see oracle.c)."""
+    lib = _load()
+    xy, npdt = _prep(xy, dtype)
+    n = xy.shape[0]
+    cnt = np.zeros(n, dtype=np.uint64)
+    h = np.zeros(n, dtype=np.uint64)
+    if getattr(lib, f"oracle_sweep_rowhash_{dtype}")(_ptr(xy), n, float(npdt(eps)), _ptr(cnt), _ptr(h)) != 0:
+        raise MemoryError("oracle_sweep_rowhash: allocation failed")
     return cnt, h
 
 

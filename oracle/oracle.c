@@ -216,6 +216,112 @@ void oracle_join_rowhash_f32(const float* xy, int64_t n, float eps,
 }
 
 /* ------------------------------------------------------------------------ */
+/* O2, second construction: an x-sorted plane sweep (no cells, no tree).    */
+/* The north star asks for the oracle to be checked against "a naive        */
+/* R-tree-free scan"; this is that scan ("O2 at scale" (i)).   */
+/* Points are ordered by (x, id); for each p the scan walks outwards from p */
+/* in both directions and stops at the first q with fl(dx*dx) > fl(eps^2),  */
+/* dx = fl(x_q - x_p).  The stop is exact under O1: fl(x_q - x_p) is         */
+/* monotone in x_q, so dx*dx only grows along each direction, and           */
+/* d2 = fl(dx2 + dy2) >= dx2 because dy2 >= 0 and rounding is monotone.     */
+/* Output: per-row (count, sum of mix64(q)) like oracle_join_rowhash_*.     */
+/* ------------------------------------------------------------------------ */
+typedef struct { double x; int64_t id; } sweep_key;
+
+static int sweep_cmp(const void* a, const void* b)
+{
+    const sweep_key* u = (const sweep_key*)a;
+    const sweep_key* v = (const sweep_key*)b;
+    if (u->x < v->x) return -1;
+    if (u->x > v->x) return 1;
+    return (u->id > v->id) - (u->id < v->id);
+}
+
+static sweep_key* sweep_order(const double* xs, int64_t n)
+{
+    sweep_key* k = (sweep_key*)malloc(sizeof(sweep_key) * (size_t)(n ? n : 1));
+    if (!k) return NULL;
+    for (int64_t i = 0; i < n; ++i) {
+        k[i].x = xs[i];
+        k[i].id = i;
+    }
+    qsort(k, (size_t)n, sizeof(sweep_key), sweep_cmp);
+    return k;
+}
+
+int oracle_sweep_rowhash_f64(const double* xy, int64_t n, double eps, uint64_t* cnt, uint64_t* hash)
+{
+    double eps2 = eps * eps;
+    double* xs = (double*)malloc(sizeof(double) * (size_t)(n ? n : 1));
+    if (!xs) return -1;
+    for (int64_t i = 0; i < n; ++i) xs[i] = xy[2 * i];
+    sweep_key* ord = sweep_order(xs, n);
+    free(xs);
+    if (!ord) return -1;
+    int64_t i;
+#pragma omp parallel for schedule(dynamic, 256)
+    for (i = 0; i < n; ++i) {
+        int64_t p = ord[i].id;
+        double xp = xy[2 * p], yp = xy[2 * p + 1];
+        uint64_t c = 0, h = 0;
+        for (int64_t j = i; j < n; ++j) {          /* rightwards, including p itself */
+            int64_t q = ord[j].id;
+            double dx = xy[2 * q] - xp;
+            double dx2 = dx * dx;
+            if (dx2 > eps2) break;
+            if (is_neighbor_f64(xp, yp, xy[2 * q], xy[2 * q + 1], eps2)) { ++c; h += mix64((uint64_t)q); }
+        }
+        for (int64_t j = i - 1; j >= 0; --j) {     /* leftwards */
+            int64_t q = ord[j].id;
+            double dx = xy[2 * q] - xp;
+            double dx2 = dx * dx;
+            if (dx2 > eps2) break;
+            if (is_neighbor_f64(xp, yp, xy[2 * q], xy[2 * q + 1], eps2)) { ++c; h += mix64((uint64_t)q); }
+        }
+        cnt[p] = c;
+        hash[p] = h;
+    }
+    free(ord);
+    return 0;
+}
+
+int oracle_sweep_rowhash_f32(const float* xy, int64_t n, float eps, uint64_t* cnt, uint64_t* hash)
+{
+    float eps2 = eps * eps;
+    double* xs = (double*)malloc(sizeof(double) * (size_t)(n ? n : 1));
+    if (!xs) return -1;
+    for (int64_t i = 0; i < n; ++i) xs[i] = (double)xy[2 * i];   /* exact widening: same order */
+    sweep_key* ord = sweep_order(xs, n);
+    free(xs);
+    if (!ord) return -1;
+    int64_t i;
+#pragma omp parallel for schedule(dynamic, 256)
+    for (i = 0; i < n; ++i) {
+        int64_t p = ord[i].id;
+        float xp = xy[2 * p], yp = xy[2 * p + 1];
+        uint64_t c = 0, h = 0;
+        for (int64_t j = i; j < n; ++j) {
+            int64_t q = ord[j].id;
+            float dx = xy[2 * q] - xp;
+            float dx2 = dx * dx;
+            if (dx2 > eps2) break;
+            if (is_neighbor_f32(xp, yp, xy[2 * q], xy[2 * q + 1], eps2)) { ++c; h += mix64((uint64_t)q); }
+        }
+        for (int64_t j = i - 1; j >= 0; --j) {
+            int64_t q = ord[j].id;
+            float dx = xy[2 * q] - xp;
+            float dx2 = dx * dx;
+            if (dx2 > eps2) break;
+            if (is_neighbor_f32(xp, yp, xy[2 * q], xy[2 * q + 1], eps2)) { ++c; h += mix64((uint64_t)q); }
+        }
+        cnt[p] = c;
+        hash[p] = h;
+    }
+    free(ord);
+    return 0;
+}
+
+/* ------------------------------------------------------------------------ */
 /* O3: Algorithm 1 on the neighbour table T.         */
 /*                                                                          */
 /* T is CSR: N_eps(p) = nbr[off[p] .. off[p+1]).                             */

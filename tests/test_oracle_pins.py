@@ -237,6 +237,36 @@ def test_rows_and_rowhash_agree_with_full_table():
             assert h[i] == np.sum(mix(lst), dtype=np.uint64)
 
 
+@pytest.mark.parametrize("dtype", ["f64", "f32"])
+def test_plane_sweep_equals_brute_force(dtype):
+    """The R-tree-free scan the north star names: an x-sorted plane sweep (a
+    different search order and pruning rule) must reproduce the brute-force
+    rows exactly, including near-ties, duplicates and the lattice ties."""
+    sets = [
+        (datagen.uniform(3000, (0, 0), (30, 30), seed=21), 0.7),
+        (datagen.subsample(datagen.tec_like(200_000, seed=2), 6000, seed=3), 0.45),
+        (datagen.near_ties(2500, 0.45, seed=12, extent=40.0), 0.45),
+        (datagen.lattice(9), 1.0),
+        (datagen.lattice(9), math.sqrt(2.0)),
+        (np.repeat(datagen.uniform(200, (0, 0), (5, 5), seed=4), 3, axis=0), 0.3),
+    ]
+    for xy, eps in sets:
+        c0, h0 = oracle.eps_join_rowhash(xy, eps, dtype=dtype)
+        c1, h1 = oracle.sweep_rowhash(xy, eps, dtype=dtype)
+        np.testing.assert_array_equal(c0, c1)
+        np.testing.assert_array_equal(h0, h1)
+
+
+def test_plane_sweep_lattice_golden():
+    g = _gold("lattice5.json")
+    xy = datagen.lattice(g["k"])
+    c, _ = oracle.sweep_rowhash(xy, g["eps_sqrt2"]["eps"])
+    assert sorted(set(c.tolist())) == sorted({g["eps_sqrt2"]["count_corner"], g["eps_sqrt2"]["count_edge"],
+                                              g["eps_sqrt2"]["count_interior"]})
+    assert int(c.sum()) == 4 * g["eps_sqrt2"]["count_corner"] + 12 * g["eps_sqrt2"]["count_edge"] \
+        + 9 * g["eps_sqrt2"]["count_interior"]
+
+
 def test_identical_points_give_n_squared():
     xy = np.tile([[1.25, -3.5]], (37, 1))
     off, nbr = oracle.eps_join(xy, 1e-9)
