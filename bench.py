@@ -42,6 +42,11 @@ WORKLOADS = {
     "C5-eps0.5": dict(gen=datagen.dense_skew, eps=0.5, desc="dense-skew n=50,000,000 eps=0.5 minpts=4"),
 }
 MINPTS = 4
+SWEEP_WORKLOADS = {
+    "C4-sweep": dict(gen=datagen.tec_like, eps=datagen.C4_EPS, minpts=datagen.C4_MINPTS,
+                     desc="TEC-like n=1,864,620, eps {0.15,0.20,0.30,0.45,0.60,0.80,1.00,1.40} x minpts "
+                          "{4,8,16}: 8 tables, each reused for 3 minpts"),
+}
 
 
 def load_peaks():
@@ -123,7 +128,7 @@ def cpu_baseline_run(xy, eps, budget_s=12.0, rows=None, dtype="f64"):
     cnt, _ = oracle.eps_join_rowhash(xy, eps, rows, dtype=dtype)
     dt = time.perf_counter() - t0
     pairs = int(cnt.sum())
-    return dict(value=pairs / dt, unit="pairs/s", cores=oracle.threads(), kind="oracle",
+    return dict(value=pairs / dt, unit="pairs/s", cores=oracle.threads(), kind="oracle", seconds=dt,
                 sample=f"{rows.size} evenly spaced query rows x all {n} points, brute force "
                        f"({pairs} pairs, {rows.size * n:.3g} tests, {dt:.2f} s)"), rows
 
@@ -177,21 +182,161 @@ def run_reference(args, wl, ws, rank):
     print(json.dumps(line), flush=True)
 
 
+def run_sweep(args, wl, ws, rank, local):
+    """C4 (BASELINE.json configs[3]): the multi-clustering sweep.  One step = one
+    hdb_sweep over all (eps, minpts) variants; metric = points clustered/s =
+    n * |variants| / step time.  value: points and labels in HBM, tables in HBM,
+    GPU DBSCAN (sweep_on_device=1).  e2e: the same call from pinned HOST points
+    into HOST labels.  "hybrid": the paper's pipeline (tables D2H into host
+    memory, host DBSCAN on T(eps_i) while the GPU builds T(eps_i+1)).
+    N > 1: the eps values (independent tables) are dealt round-robin to ranks."""
+    eps_all, mp = list(wl["eps"]), list(wl["minpts"])
+    xy_np = wl["gen"]()
+    if args.dtype == "f32":
+        xy_np = xy_np.astype(np.float32)
+    n = xy_np.shape[0]
+    variants = len(eps_all) * len(mp)
+    if args.impl == "reference":
+        if rank != 0:
+            return
+        # the oracle as it stands: brute-force rows (sampled) + Alg. 1 would need
+        # the full table; time the brute-force join on a bounded row sample per eps
+        K, W = args.steps, args.warmup
+        res, t_full = [], 0.0
+        for e in eps_all:
+            r, rows = cpu_baseline_run(xy_np, e, budget_s=max(1.0, 40.0 / len(eps_all) / max(K + W, 1)))
+            res.append(r)
+            t_full += r["seconds"] * n / rows.size
+        v = n * variants / t_full   # extrapolated: full brute-force tables; DBSCAN on T is negligible beside it
+        line = {"impl": "reference", "metric": "points_clustered_per_sec", "value": v, "unit": "points/s",
+                "n_gpus": ws, "steps": K, "warmup": W, "ms_per_step": 1e3 * t_full,
+                "higher_is_better": True, "scaling": "strong",
+                "vs_baseline": None, "dtype": args.dtype, "data": "synthetic",
+                "config": {"workload": args.workload, "desc": wl["desc"]},
+                "cpu_baseline": {"value": v, "unit": "points/s", "cores": res[0]["cores"], "kind": "oracle",
+                                 "sample": "per eps, brute-force rows (extrapolated to all n rows): "
+                                           + "; ".join(r["sample"] for r in res)},
+                "e2e": {"value": v, "unit": "points/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+        print(json.dumps(line), flush=True)
+        return
+
+    import torch
+    import torch.distributed as dist
+    from paper_conf_ipps_gowanlockrblp17_b200 import hdb
+
+    assert torch.cuda.is_available(), "bench.py needs a GPU"
+    ndev = torch.cuda.device_count()
+    local_dev = local % ndev
+    torch.cuda.set_device(local_dev)
+    if ws > 1:
+        if ndev >= ws:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local_dev))
+        else:
+            dist.init_process_group("gloo")
+    dev = torch.device("cuda", local_dev)
+    coll_dev = dev if (ws == 1 or ndev >= ws) else torch.device("cpu")
+    my_eps = eps_all[rank::ws]
+    xy_dev = torch.from_numpy(xy_np).to(dev)
+    ctx = hdb.hdb_ctx_create(sweep_on_device=1, cell_split=args.cell_split, search_kernel=args.kernel)
+    lab_dev = torch.empty((max(len(my_eps), 1), len(mp), n), dtype=torch.int32, device=dev)
+
+    def step():
+        if my_eps:
+            return hdb.hdb_sweep(ctx, xy_dev, my_eps, mp, labels=lab_dev)[1]
+        return None
+
+    for _ in range(max(args.warmup, 0)):
+        step()
+    torch.cuda.synchronize()
+    if ws > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    stream = torch.cuda.current_stream(dev)
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    l0 = hdb.hdb_kernel_launches()
+    with ClockSampler(local_dev) as clk:
+        ev0.record(stream)
+        for _ in range(args.steps):
+            k_dev = step()
+        ev1.record(stream)
+        torch.cuda.synchronize()
+    launches = hdb.hdb_kernel_launches() - l0
+    ms = ev0.elapsed_time(ev1)
+    if ws > 1:
+        t = torch.tensor([ms], device=coll_dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+    value = n * variants * args.steps / (ms / 1e3)
+    line = {"metric": "points_clustered_per_sec", "value": value, "unit": "points/s", "n_gpus": ws,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms / args.steps,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": args.dtype,
+            "data": "synthetic",
+            "config": {"workload": args.workload, "desc": wl["desc"], "n": n, "variants": variants,
+                       "parallelism": f"eps-shard{ws}",
+                       "l2": "not flushed: every step writes 8 tables totalling ~88 GB (>> 126 MB L2)",
+                       "step": "hdb_sweep, sweep_on_device=1: per eps grid + device table; per minpts GPU "
+                               "DBSCAN into device labels"},
+            "gpu_launches": launches, "clocks": clk.summary()}
+    if rank == 0 and ws == 1:
+        # e2e: same call from pinned host points into host labels
+        xy_pin = torch.from_numpy(xy_np).pin_memory()
+        lab_host = np.empty((len(eps_all), len(mp), n), np.int32)
+        hdb.hdb_sweep(ctx, xy_pin, eps_all, mp, labels=lab_host)
+        ts = []
+        for _ in range(max(1, min(args.steps, 3))):
+            t0 = time.perf_counter()
+            _, k_host = hdb.hdb_sweep(ctx, xy_pin, eps_all, mp, labels=lab_host)
+            ts.append(time.perf_counter() - t0)
+        te = float(np.median(ts))
+        esz = xy_np.itemsize * 2
+        line["e2e"] = {"value": n * variants / te, "unit": "points/s", "h2d_bytes_per_step": esz * n * len(eps_all),
+                       "d2h_bytes_per_step": 4 * n * variants, "s_per_step": te,
+                       "includes": "pinned host points -> per eps: H2D, grid, device table, GPU DBSCAN x3 "
+                                   "minpts, labels D2H"}
+        same = bool(np.array_equal(lab_dev.cpu().numpy(), lab_host)) if len(my_eps) == len(eps_all) else None
+        line["e2e"]["labels_equal_device_run"] = same
+        line["n_clusters"] = k_host.tolist()
+        if args.hybrid_steps > 0:
+            ctx_h = hdb.hdb_ctx_create(sweep_on_device=0, cell_split=args.cell_split, search_kernel=args.kernel)
+            lab_h = np.empty_like(lab_host)
+            ts = []
+            for _ in range(args.hybrid_steps):
+                t0 = time.perf_counter()
+                _, k_h = hdb.hdb_sweep(ctx_h, xy_pin, eps_all, mp, labels=lab_h)
+                ts.append(time.perf_counter() - t0)
+            hdb.hdb_ctx_destroy(ctx_h)
+            th = float(np.median(ts))
+            line["hybrid"] = {"value": n * variants / th, "unit": "points/s", "s_per_step": th,
+                              "labels_equal": bool(np.array_equal(lab_h, lab_host)),
+                              "desc": "the paper's S2/S3 pipeline: tables D2H into pinned host memory, host "
+                                      "DBSCAN (3 minpts threads) on T(eps_i) while the GPU builds T(eps_i+1)"}
+        del k_dev
+    hdb.hdb_ctx_destroy(ctx)
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if ws > 1:
+        dist.destroy_process_group()
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="hdb", choices=["hdb", "reference"])
-    ap.add_argument("--workload", default="C2-eps0.45", choices=sorted(WORKLOADS))
+    ap.add_argument("--workload", default="C2-eps0.45", choices=sorted(WORKLOADS) + sorted(SWEEP_WORKLOADS))
+    ap.add_argument("--hybrid-steps", type=int, default=1,
+                    help="C4-sweep: timed runs of the paper's hybrid sweep (host tables + host DBSCAN)")
     ap.add_argument("--dtype", default="f64", choices=["f64", "f32"])
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--kernel", type=int, default=0, help="search kernel variant (hdb_opts.search_kernel)")
     ap.add_argument("--cell-split", type=int, default=0, help="hdb_opts.cell_split (0 = library default)")
     args = ap.parse_args()
-    wl = WORKLOADS[args.workload]
     ws, rank, local = dist_env()
+    if args.workload in SWEEP_WORKLOADS:
+        return run_sweep(args, SWEEP_WORKLOADS[args.workload], ws, rank, local)
+    wl = WORKLOADS[args.workload]
     if args.impl == "reference":
         return run_reference(args, wl, ws, rank)
 

@@ -84,7 +84,12 @@ typedef struct {
     int search_kernel;          /* 0 = default; other values select kernel variants        */
     int host_threads;           /* threads for host-side work (T assembly, DBSCAN); 0 = all cores      */
     int cell_split;             /* k >= 1: grid cells of width eps/k, (2k+1)^2-cell stencil (fewer
-                                   candidate tests on dense data); 0 = default (1, the paper's eps)    */
+                                   candidate tests on dense data); 0 = auto (k from a sampled cell
+                                   occupancy); 1 = the paper's eps cells      */
+    int sweep_on_device;        /* hdb_sweep only: 0 = the paper's hybrid split (tables D2H, host
+                                   DBSCAN pipelined with the next table's build);
+                                   1 = tables stay in HBM and DBSCAN runs on the GPU (NEXT-4);
+                                   labels are identical either way                                    */
 } hdb_opts;
 
 /* Borrowed view of a table T (T_i^min/T_i^max ranges into B).
@@ -207,7 +212,12 @@ hdb_status  hdb_dbscan_ex(const hdb_table* table, uint32_t minpts, int n_threads
 /* ---- (4) sweep ----------------------------------------------------------- */
 /* For each eps[i] (one grid + one table, built while the host clusters the
  * previous table) and each minpts[j] (concurrent):
- * labels[(i * n_minpts + j) * n + p], n_clusters[i * n_minpts + j]. */
+ * labels[(i * n_minpts + j) * n + p], n_clusters[i * n_minpts + j].
+ * xy: host or device memory (as hdb_grid_build).  labels: caller-allocated,
+ * host memory, or -- with opts.sweep_on_device = 1 -- host or device memory
+ * (HDB_EINVAL otherwise); n_clusters: host memory or NULL.  With
+ * sweep_on_device = 1 each table stays in HBM and DBSCAN runs on the GPU
+ * (NEXT-4); the labels are identical to the hybrid path's. */
 hdb_status  hdb_sweep(hdb_ctx* ctx, const void* xy, uint64_t n, hdb_dtype dtype,
                       const double* eps, uint32_t n_eps, const uint32_t* minpts, uint32_t n_minpts,
                       int32_t* labels, uint32_t* n_clusters);

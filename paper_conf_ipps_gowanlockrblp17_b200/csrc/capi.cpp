@@ -67,6 +67,7 @@ hdb_status hdb_ctx_create(const hdb_opts* opts, hdb_ctx** out) {
     if (o.shard_count < 0 || (o.shard_count > 0 && (o.shard_rank < 0 || o.shard_rank >= o.shard_count)))
         fail(HDB_EINVAL, "bad shard_rank/shard_count");
     if (o.cell_split < 0 || o.cell_split > 8) fail(HDB_EINVAL, "cell_split must be in [0, 8]");
+    if (o.sweep_on_device != 0 && o.sweep_on_device != 1) fail(HDB_EINVAL, "sweep_on_device must be 0 or 1");
     c = new hdb_ctx;
     int ndev_avail = 0;
     cudaError_t e = cudaGetDeviceCount(&ndev_avail);
@@ -443,6 +444,33 @@ hdb_status hdb_sweep(hdb_ctx* c, const void* xy, uint64_t n, hdb_dtype dt, const
         }
     std::lock_guard<std::recursive_mutex> lk(c->mu);
     HDB_GUARD_BEGIN
+    if (c->opts.sweep_on_device) {
+        if (c->opts.shard_count > 1) fail(HDB_EINVAL, "sweep_on_device needs an unsharded context");
+        // NEXT-4 variant: T(eps_i) stays in HBM; every minpts variant runs the
+        // device DBSCAN on it and only labels cross PCIe.
+        for (uint32_t i = 0; i < n_eps; ++i) {
+            hdb_grid* g = nullptr;
+            hdb_table* t = nullptr;
+            try {
+                grid_build(c, xy, n, dt, eps[i], &g);
+                neighbor_table(c, g, true, &t);
+                grid_free(g);
+                g = nullptr;
+                for (uint32_t j = 0; j < n_minpts; ++j) {
+                    const uint32_t k = dbscan_device(t, minpts[j], labels + ((uint64_t)i * n_minpts + j) * n, nullptr);
+                    if (n_clusters) n_clusters[(uint64_t)i * n_minpts + j] = k;
+                }
+                table_free(t);
+            } catch (...) {
+                if (g) grid_free(g);
+                if (t) table_free(t);
+                throw;
+            }
+        }
+        return HDB_OK;
+    }
+    if (n && n_eps && n_minpts && is_device_ptr(labels))
+        fail(HDB_EINVAL, "hdb_sweep: labels must be host memory unless opts.sweep_on_device = 1");
     std::mutex m;
     std::condition_variable cv;
     std::deque<std::pair<uint32_t, hdb_table*>> q;

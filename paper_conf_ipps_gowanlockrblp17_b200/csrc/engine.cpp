@@ -220,6 +220,12 @@ PtrInfo classify(const void* p) {
     return r;
 }
 
+}  // namespace
+
+bool is_device_ptr(const void* p) { return classify(p).loc == Loc::Device; }
+
+namespace {
+
 // f64 mode: bound on |t_f32 - (d2_f64 - e2_f64)| for the search kernels' f32
 // filter.  Filter coordinates are X = fl32(fl64(x - o))
 // for an origin o with |x - o| <= R; every candidate lies in the 3x3 stencil,
@@ -771,8 +777,8 @@ uint32_t dbscan_device(const hdb_table* t, uint32_t minpts, int32_t* labels, uin
         L = dlab.as<int32_t>();
     }
     uint8_t* C = core_dev ? core : dcore.as<uint8_t>();
-    launch_dbscan_device(t->begin, t->count, t->nbrs, n, minpts, C, parent.as<uint32_t>(), root.as<uint32_t>(),
-                         is_root.as<uint32_t>(), rank.as<uint32_t>(), temp.p, L, s);
+    launch_dbscan_device(t->begin, t->count, t->nbrs, t->rows, n, t->npairs, minpts, C, parent.as<uint32_t>(),
+                         root.as<uint32_t>(), is_root.as<uint32_t>(), rank.as<uint32_t>(), temp.p, L, s);
     HDB_LAUNCH_CHECK();
     uint32_t k = 0;
     HDB_CUDA(cudaMemcpyAsync(&k, rank.as<uint32_t>() + n, 4, cudaMemcpyDeviceToHost, s));
@@ -786,7 +792,7 @@ void table_free(hdb_table* t) {
     if (!t) return;
     if (t->on_device) {
         DeviceGuard dg(t->device);
-        for (void* p : {(void*)t->begin, (void*)t->count, (void*)t->nbrs})
+        for (void* p : {(void*)t->begin, (void*)t->count, (void*)t->nbrs, (void*)t->rows})
             if (p) cudaFreeAsync(p, t->dstream);   // stream-ordered: no host sync needed
     } else if (t->pool) {
         t->pool->release(t->begin, t->cap_begin);
@@ -929,6 +935,13 @@ void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hd
             st.write_launches = 1;
             st.n_batches = 1;
             st.max_batch = P;
+            if (whole && n) {
+                // production order of the rows: DBSCAN walks them in this (cell-sorted) order so
+                // that consecutive rows share neighbours (cache locality of the union-find)
+                DBuf rw(4 * n, s);
+                HDB_CUDA(cudaMemcpyAsync(rw.p, g.ids, 4 * n, cudaMemcpyDeviceToDevice, s));
+                t->rows = (uint32_t*)rw.release();
+            }
             t->nbrs = (uint32_t*)nb.release();
             t->begin = (uint64_t*)beg.release();
             t->count = (uint32_t*)cnt.release();

@@ -134,9 +134,11 @@ void launch_batch_cuts(const uint32_t* gstart, const uint64_t* off, uint64_t g0,
 void launch_pos_to_group(const uint32_t* gstart, uint64_t n_groups, const uint64_t* pos, uint32_t m,
                          uint64_t* grp, cudaStream_t s);
 // DBSCAN on a device-resident table (kernels_dbscan.cu); rank[n] = number of clusters
-void launch_dbscan_device(const uint64_t* begin, const uint32_t* count, const uint32_t* nbrs, uint64_t n,
-                          uint32_t minpts, uint8_t* core, uint32_t* parent, uint32_t* root, uint32_t* is_root,
-                          uint32_t* rank, void* scan_temp, int32_t* labels, cudaStream_t s);
+// rows: the table's production order (begin[rows[r]] non-decreasing), or null
+void launch_dbscan_device(const uint64_t* begin, const uint32_t* count, const uint32_t* nbrs, const uint32_t* rows,
+                          uint64_t n, uint64_t npairs, uint32_t minpts, uint8_t* core, uint32_t* parent,
+                          uint32_t* root, uint32_t* is_root, uint32_t* rank, void* scan_temp, int32_t* labels,
+                          cudaStream_t s);
 // T assembly by original id: begin[ids[q]] = off[q] - off[q0] + base, count[ids[q]] = cnt[q], q in [q0,q1)
 void launch_scatter_rows(const uint32_t* ids, const uint64_t* off, const uint32_t* cnt, uint64_t q0,
                          uint64_t q1, uint64_t base, uint64_t* begin, uint32_t* count, cudaStream_t s);
@@ -191,6 +193,7 @@ struct hdb_table {
     uint64_t* begin = nullptr;
     uint32_t* count = nullptr;
     uint32_t* nbrs = nullptr;
+    uint32_t* rows = nullptr;   // device tables only: query ids in production (cell-sorted) order
     // ownership
     std::shared_ptr<hdb::PinnedPool> pool;   // non-null: begin/count/nbrs are pinned pool blocks
     size_t cap_begin = 0, cap_count = 0, cap_nbrs = 0;
@@ -210,5 +213,6 @@ void table_free(hdb_table* t);
 // dbscan.cpp
 uint32_t dbscan_host(const hdb_table* t, uint32_t minpts, int n_threads, int32_t* labels, uint8_t* core);
 uint32_t dbscan_device(const hdb_table* t, uint32_t minpts, int32_t* labels, uint8_t* core);
+bool is_device_ptr(const void* p);   // CUDA device / managed memory
 void canonicalize(hdb_table* t);
 }  // namespace hdb

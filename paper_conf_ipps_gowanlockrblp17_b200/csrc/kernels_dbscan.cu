@@ -7,7 +7,8 @@
 // the lowest-numbered cluster among its core neighbours; noise = -1.
 //
 //   k_core_init   core flags, parent[p] = p
-//   k_union       warp per core u: for every core neighbour v < u, union(u, v) by
+//   k_union       warp per core u (rows taken in the table's cell-sorted production
+//                 order): for every core neighbour v < u, union(u, v) by
 //                 hooking the larger root under the smaller (atomicCAS), so every
 //                 root stays the minimum id of its tree (ECL-CC style, path halving)
 //   k_flatten     root[p] = root(p) for cores (read-only find); root flags
@@ -66,33 +67,99 @@ __device__ __forceinline__ void unite(uint32_t* __restrict__ parent, uint32_t a,
     }
 }
 
+// parent[p] of a non-core point is kNonCore for the whole union phase: one
+// load of parent[v] then answers both "is v core" and "where is v's root".
+constexpr uint32_t kNonCore = 0xffffffffu;
+
 __global__ void __launch_bounds__(256) k_core_init(const uint32_t* __restrict__ count, uint64_t n, uint32_t minpts,
                                                    uint8_t* __restrict__ core, uint32_t* __restrict__ parent) {
     for (uint64_t p = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; p < n; p += (uint64_t)gridDim.x * blockDim.x) {
-        core[p] = count[p] >= minpts ? 1 : 0;
-        parent[p] = (uint32_t)p;
+        const bool c = count[p] >= minpts;
+        core[p] = c ? 1 : 0;
+        parent[p] = c ? (uint32_t)p : kNonCore;
     }
 }
 
-// warp per core vertex u (grid-stride over ids); lanes stride over u's list
-__global__ void __launch_bounds__(256) k_union(const uint64_t* __restrict__ begin, const uint32_t* __restrict__ count,
-                                               const uint32_t* __restrict__ nbrs, const uint8_t* __restrict__ core,
-                                               uint64_t n, uint32_t* __restrict__ parent) {
+// True if x's root is `r` (read-only, possibly stale L1 reads): stops as soon
+// as the chain reaches r, so the common case -- x hangs directly under the
+// root already found for u -- costs one load.
+__device__ __forceinline__ bool reaches(const uint32_t* __restrict__ parent, uint32_t x, uint32_t r) {
+    uint32_t p = __ldca(&parent[x]);
+    while (p != x) {
+        if (p == r) return true;
+        x = p;
+        p = __ldca(&parent[x]);
+    }
+    return x == r;
+}
+
+constexpr uint32_t kRowsPerGrab = 4;      // consecutive (cell-sorted) rows per warp grab
+constexpr int kUnionThreads = 1024;       // one CTA per SM
+
+// first row r in [0, n) with begin[rows[r]] >= x (begin is non-decreasing
+// along the production order of a whole table)
+__device__ uint32_t row_of_pair(const uint64_t* __restrict__ begin, const uint32_t* __restrict__ rows, uint32_t n,
+                                uint64_t x) {
+    uint32_t lo = 0, hi = n;
+    while (lo < hi) {
+        const uint32_t mid = lo + (hi - lo) / 2;
+        if (begin[rows[mid]] < x) lo = mid + 1;
+        else hi = mid;
+    }
+    return lo;
+}
+
+// One CTA per SM owns a contiguous range of the production (cell-sorted) order
+// holding ~1/G of the pairs; its warps take kRowsPerGrab consecutive rows at a
+// time from a shared counter.  All warps of an SM therefore work in one small
+// region of space at any moment and their random parent[v] reads share L1.
+// For core u, lanes stride over u's list (4 independent edges per lane per
+// pass); every core neighbour v < u whose root differs is united with u.
+__global__ void __launch_bounds__(kUnionThreads, 1)
+    k_union(const uint64_t* __restrict__ begin, const uint32_t* __restrict__ count, const uint32_t* __restrict__ nbrs,
+            const uint32_t* __restrict__ rows, uint32_t n, uint64_t npairs, uint32_t* __restrict__ parent) {
+    __shared__ uint32_t s_next, s_end;
     const int lane = threadIdx.x & 31;
-    const uint64_t wid = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
-    const uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
-    for (uint64_t u = wid; u < n; u += nw) {
-        if (!core[u]) continue;   // uniform
-        const uint32_t* L = nbrs + begin[u];
-        const uint32_t m = count[u];
-        uint32_t ru = find_fast(parent, (uint32_t)u);
-        for (uint32_t j = lane; j < m; j += 32) {
-            const uint32_t v = __ldg(&L[j]);
-            if (v < u && core[v]) {
-                const uint32_t rv = find_fast(parent, v);
-                if (rv != ru) {
-                    unite(parent, (uint32_t)u, v);
-                    ru = find_fast(parent, (uint32_t)u);
+    if (threadIdx.x == 0) {
+        const uint64_t G = gridDim.x, c = blockIdx.x;
+        if (rows) {
+            s_next = row_of_pair(begin, rows, n, npairs * c / G);
+            s_end = c + 1 == G ? n : row_of_pair(begin, rows, n, npairs * (c + 1) / G);
+        } else {
+            s_next = (uint32_t)((uint64_t)n * c / G);
+            s_end = (uint32_t)((uint64_t)n * (c + 1) / G);
+        }
+    }
+    __syncthreads();
+    const uint32_t end = s_end;
+    while (true) {
+        uint32_t r0 = 0;
+        if (lane == 0) r0 = atomicAdd(&s_next, kRowsPerGrab);
+        r0 = __shfl_sync(FULL, r0, 0);
+        if (r0 >= end) return;
+        const uint32_t r1 = min(end, r0 + kRowsPerGrab);
+        for (uint32_t r = r0; r < r1; ++r) {
+            const uint32_t u = rows ? __ldg(&rows[r]) : r;
+            if (__ldca(&parent[u]) == kNonCore) continue;   // uniform: non-core rows add no edge
+            const uint32_t* L = nbrs + begin[u];
+            const uint32_t m = count[u];
+            uint32_t ru = find_fast(parent, u);
+            for (uint32_t j0 = 0; j0 < m; j0 += 128) {
+                uint32_t v[4], p[4];
+#pragma unroll
+                for (int k = 0; k < 4; ++k) {
+                    const uint32_t j = j0 + lane + 32 * k;
+                    v[k] = j < m ? __ldg(&L[j]) : 0xffffffffu;
+                }
+#pragma unroll
+                for (int k = 0; k < 4; ++k) p[k] = v[k] < u ? __ldca(&parent[v[k]]) : kNonCore;
+#pragma unroll
+                for (int k = 0; k < 4; ++k) {
+                    // skip non-cores and v hanging directly under u's root; else follow the chain
+                    if (p[k] != kNonCore && p[k] != ru && !(p[k] != v[k] && reaches(parent, p[k], ru))) {
+                        unite(parent, u, v[k]);
+                        ru = find_fast(parent, u);
+                    }
                 }
             }
         }
@@ -117,10 +184,12 @@ __global__ void __launch_bounds__(256) k_flatten(const uint8_t* __restrict__ cor
 
 // thread per point: cores read their root's rank; non-cores scan their (short) list
 __global__ void __launch_bounds__(256) k_labels(const uint64_t* __restrict__ begin, const uint32_t* __restrict__ count,
-                                                const uint32_t* __restrict__ nbrs, const uint8_t* __restrict__ core,
+                                                const uint32_t* __restrict__ nbrs, const uint32_t* __restrict__ rows,
+                                                const uint8_t* __restrict__ core,
                                                 const uint32_t* __restrict__ parent, const uint32_t* __restrict__ rank,
                                                 uint64_t n, int32_t* __restrict__ labels) {
-    for (uint64_t p = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; p < n; p += (uint64_t)gridDim.x * blockDim.x) {
+    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+        const uint64_t p = rows ? rows[i] : i;
         int32_t lab = -1;
         if (core[p]) {
             lab = (int32_t)rank[parent[p]];
@@ -146,15 +215,23 @@ inline unsigned blocks_for(uint64_t n, unsigned cap = 148u * 16u) {
 
 }  // namespace
 
-void launch_dbscan_device(const uint64_t* begin, const uint32_t* count, const uint32_t* nbrs, uint64_t n,
-                          uint32_t minpts, uint8_t* core, uint32_t* parent, uint32_t* root, uint32_t* is_root,
-                          uint32_t* rank, void* scan_temp, int32_t* labels, cudaStream_t s) {
+void launch_dbscan_device(const uint64_t* begin, const uint32_t* count, const uint32_t* nbrs, const uint32_t* rows,
+                          uint64_t n, uint64_t npairs, uint32_t minpts, uint8_t* core, uint32_t* parent, uint32_t* root,
+                          uint32_t* is_root, uint32_t* rank, void* scan_temp, int32_t* labels, cudaStream_t s) {
     if (n == 0) return;
     k_core_init<<<blocks_for(n), 256, 0, s>>>(count, n, minpts, core, parent);
-    k_union<<<148 * 8, 256, 0, s>>>(begin, count, nbrs, core, n, parent);
+    static int sms = 0;
+    if (!sms) {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        cudaFuncSetAttribute(k_union, cudaFuncAttributePreferredSharedMemoryCarveout, 0);   // all of it as L1
+        if (sms <= 0) sms = 148;
+    }
+    k_union<<<sms, kUnionThreads, 0, s>>>(begin, count, nbrs, rows, (uint32_t)n, npairs, parent);
     k_flatten<<<blocks_for(n), 256, 0, s>>>(core, n, parent, root, is_root);
     scan_u32_to_u32(is_root, rank, n, scan_temp, s);
-    k_labels<<<blocks_for(n), 256, 0, s>>>(begin, count, nbrs, core, root, rank, n, labels);
+    k_labels<<<blocks_for(n), 256, 0, s>>>(begin, count, nbrs, rows, core, root, rank, n, labels);
     g_kernel_launches += 4;
 }
 

@@ -34,7 +34,8 @@ class hdb_opts(ctypes.Structure):
     _fields_ = [("devices", ctypes.POINTER(_int)), ("n_devices", _int), ("sample_fraction", _dbl),
                 ("alpha", _dbl), ("n_streams", _int), ("batch_pairs", _u64), ("sort_lists", _int),
                 ("host_budget_bytes", _u64), ("shard_rank", _int), ("shard_count", _int),
-                ("search_kernel", _int), ("host_threads", _int), ("cell_split", _int)]
+                ("search_kernel", _int), ("host_threads", _int), ("cell_split", _int),
+                ("sweep_on_device", _int)]
 
 
 class hdb_table_view(ctypes.Structure):
@@ -272,12 +273,15 @@ def hdb_dbscan(table, minpts: int, n_threads: int = 0, labels=None, is_core=None
     return labels, is_core, int(k.value)
 
 
-def hdb_sweep(ctx, xy, eps_list, minpts_list, dtype: int | None = None):
+def hdb_sweep(ctx, xy, eps_list, minpts_list, dtype: int | None = None, labels=None):
+    """labels: optional preallocated int32 [n_eps, n_minpts, n] (numpy, or a CUDA
+    tensor when the context was created with sweep_on_device=1)."""
     n = _nrows(xy)
     dt = _dtype_of(xy) if dtype is None else dtype
     eps = np.ascontiguousarray(eps_list, np.float64)
     mp = np.ascontiguousarray(minpts_list, np.uint32)
-    labels = np.empty((eps.size, mp.size, n), np.int32)
+    if labels is None:
+        labels = np.empty((eps.size, mp.size, n), np.int32)
     k = np.empty((eps.size, mp.size), np.uint32)
     _check(lib.hdb_sweep(ctx, _ptr(xy), n, dt, _ptr(eps), eps.size, _ptr(mp), mp.size, _ptr(labels), _ptr(k)),
            "hdb_sweep")

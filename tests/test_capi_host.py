@@ -166,3 +166,12 @@ def test_ctx_create_without_gpu_fails_loudly():
     with pytest.raises(hdb.HdbError) as e:
         hdb.hdb_ctx_create()
     assert e.value.status == hdb.HDB_ECUDA
+
+
+@pytest.mark.parametrize("bad", [dict(sweep_on_device=2), dict(cell_split=9), dict(n_streams=0),
+                                 dict(sample_fraction=0.0), dict(alpha=-1.0), dict(shard_count=2, shard_rank=2)])
+def test_opts_validation_before_device(bad):
+    """Option errors are reported as HDB_EINVAL before any device is touched."""
+    with pytest.raises(hdb.HdbError) as e:
+        hdb.hdb_ctx_create(**bad)
+    assert e.value.status == hdb.HDB_EINVAL

@@ -359,11 +359,12 @@ def test_dbscan_end_to_end(torch_cuda, threads):
         assert np.array_equal(lab, want[0])
 
 
-def test_sweep_matches_oracle(torch_cuda):
+@pytest.mark.parametrize("on_device", [0, 1])
+def test_sweep_matches_oracle(torch_cuda, on_device):
     xy = datagen.subsample(datagen.tec_like(), 20_000, seed=11)
     eps_list = (0.15, 0.3, 0.45, 1.0)
     mp = (4, 8, 16)
-    ctx = _ctx()
+    ctx = _ctx(sweep_on_device=on_device)
     try:
         labels, k = hdb.hdb_sweep(ctx, xy, eps_list, mp)
     finally:
