@@ -7,10 +7,15 @@
 // the lowest-numbered cluster among its core neighbours; noise = -1.
 //
 //   k_core_init   core flags, parent[p] = p
-//   k_union       warp per core u (rows taken in the table's cell-sorted production
-//                 order): for every core neighbour v < u, union(u, v) by
-//                 hooking the larger root under the smaller (atomicCAS), so every
-//                 root stays the minimum id of its tree (ECL-CC style, path halving)
+//   k_sample_link every core u unites with 2 sampled core neighbours (Afforest-style
+//                 pre-pass: assembles most of every dense cluster cheaply)
+//   k_giant       the two most frequent roots among 1024 sampled points = the giant
+//                 components A, B; k_giant_bits: their membership bitmaps
+//   k_union       warp per core row (rows taken in the table's cell-sorted production
+//                 order); each core-core edge not inside A or B is taken once
+//                 (rule at k_union): union(u, v) by hooking the larger root under the smaller
+//                 (atomicCAS), so every root stays the minimum id of its tree
+//                 (ECL-CC style, path halving)
 //   k_flatten     root[p] = root(p) for cores (read-only find); root flags
 //   scan          cluster number of each root = rank of its id among the roots
 //   k_labels      cores: number of their root; non-cores (lists < minpts long):
@@ -95,6 +100,7 @@ __device__ __forceinline__ bool reaches(const uint32_t* __restrict__ parent, uin
 
 constexpr uint32_t kRowsPerGrab = 4;      // consecutive (cell-sorted) rows per warp grab
 constexpr int kUnionThreads = 1024;       // one CTA per SM
+constexpr uint32_t kRangesPerCta = 32;    // pair-balanced ranges, taken dynamically
 
 // first row r in [0, n) with begin[rows[r]] >= x (begin is non-decreasing
 // along the production order of a whole table)
@@ -109,60 +115,181 @@ __device__ uint32_t row_of_pair(const uint64_t* __restrict__ begin, const uint32
     return lo;
 }
 
-// One CTA per SM owns a contiguous range of the production (cell-sorted) order
-// holding ~1/G of the pairs; its warps take kRowsPerGrab consecutive rows at a
-// time from a shared counter.  All warps of an SM therefore work in one small
-// region of space at any moment and their random parent[v] reads share L1.
-// For core u, lanes stride over u's list (4 independent edges per lane per
-// pass); every core neighbour v < u whose root differs is united with u.
-__global__ void __launch_bounds__(kUnionThreads, 1)
-    k_union(const uint64_t* __restrict__ begin, const uint32_t* __restrict__ count, const uint32_t* __restrict__ nbrs,
-            const uint32_t* __restrict__ rows, uint32_t n, uint64_t npairs, uint32_t* __restrict__ parent) {
-    __shared__ uint32_t s_next, s_end;
-    const int lane = threadIdx.x & 31;
-    if (threadIdx.x == 0) {
-        const uint64_t G = gridDim.x, c = blockIdx.x;
-        if (rows) {
-            s_next = row_of_pair(begin, rows, n, npairs * c / G);
-            s_end = c + 1 == G ? n : row_of_pair(begin, rows, n, npairs * (c + 1) / G);
-        } else {
-            s_next = (uint32_t)((uint64_t)n * c / G);
-            s_end = (uint32_t)((uint64_t)n * (c + 1) / G);
+constexpr uint32_t kSampleLinks = 2;   // edges per core linked before the full pass
+
+// Afforest-style pre-pass (Sutton et al., IPDPS 2018): every core u unites with
+// kSampleLinks of its core neighbours, taken at evenly spaced list positions.
+// On an eps-graph this already assembles most of every dense cluster.  The
+// read-only root test first keeps the CAS traffic off the giant roots.
+__global__ void __launch_bounds__(256) k_sample_link(const uint64_t* __restrict__ begin,
+                                                     const uint32_t* __restrict__ count,
+                                                     const uint32_t* __restrict__ nbrs,
+                                                     const uint32_t* __restrict__ rows, uint64_t n,
+                                                     uint32_t* __restrict__ parent) {
+    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+        const uint32_t u = rows ? rows[i] : (uint32_t)i;
+        if (__ldcg(&parent[u]) == kNonCore) continue;
+        const uint32_t* L = nbrs + begin[u];
+        const uint32_t m = count[u];
+        for (uint32_t k = 1; k <= kSampleLinks; ++k) {
+            const uint32_t v = L[(uint64_t)m * k / (kSampleLinks + 1)];
+            if (v != u && __ldcg(&parent[v]) != kNonCore && find_fast(parent, u) != find_fast(parent, v))
+                unite(parent, u, v);
         }
     }
+}
+
+// One CTA: the two most frequent roots among 1024 sampled points after the
+// pre-pass (the "giant" components A = giant[0], B = giant[1]; kNonCore if a
+// root holds fewer than kGiantMin samples).  Also resets k_union's counter.
+constexpr int kGiantSamples = 1024;
+constexpr unsigned long long kGiantMin = kGiantSamples / 8;
+__global__ void __launch_bounds__(kGiantSamples) k_giant(const uint32_t* __restrict__ rows, uint64_t n,
+                                                         uint32_t* __restrict__ parent, uint32_t* __restrict__ giant) {
+    __shared__ uint32_t sv[kGiantSamples];
+    __shared__ unsigned long long best, second;
+    const uint32_t t = threadIdx.x;
+    const uint64_t i = (uint64_t)t * n / kGiantSamples;
+    uint32_t r = kNonCore;
+    if (i < n) {
+        const uint32_t p = rows ? rows[i] : (uint32_t)i;
+        if (__ldcg(&parent[p]) != kNonCore) r = find_root(parent, p);
+    }
+    sv[t] = r;
+    if (t == 0) best = second = 0;
     __syncthreads();
-    const uint32_t end = s_end;
-    while (true) {
-        uint32_t r0 = 0;
-        if (lane == 0) r0 = atomicAdd(&s_next, kRowsPerGrab);
-        r0 = __shfl_sync(FULL, r0, 0);
-        if (r0 >= end) return;
-        const uint32_t r1 = min(end, r0 + kRowsPerGrab);
-        for (uint32_t r = r0; r < r1; ++r) {
-            const uint32_t u = rows ? __ldg(&rows[r]) : r;
-            if (__ldca(&parent[u]) == kNonCore) continue;   // uniform: non-core rows add no edge
-            const uint32_t* L = nbrs + begin[u];
-            const uint32_t m = count[u];
-            uint32_t ru = find_fast(parent, u);
-            for (uint32_t j0 = 0; j0 < m; j0 += 128) {
-                uint32_t v[4], p[4];
-#pragma unroll
-                for (int k = 0; k < 4; ++k) {
-                    const uint32_t j = j0 + lane + 32 * k;
-                    v[k] = j < m ? __ldg(&L[j]) : 0xffffffffu;
+    for (int k = 2; k <= kGiantSamples; k <<= 1)   // bitonic sort
+        for (int j = k >> 1; j > 0; j >>= 1) {
+            const uint32_t o = t ^ j;
+            if (o > t) {
+                const uint32_t x = sv[t], y = sv[o];
+                if (((t & k) == 0) == (x > y)) {
+                    sv[t] = y;
+                    sv[o] = x;
                 }
+            }
+            __syncthreads();
+        }
+    unsigned long long run = 0;
+    if (sv[t] != kNonCore && (t == 0 || sv[t - 1] != sv[t])) {
+        uint32_t e = t + 1;
+        while (e < kGiantSamples && sv[e] == sv[t]) ++e;
+        run = ((unsigned long long)(e - t) << 32) | sv[t];
+        atomicMax(&best, run);
+    }
+    __syncthreads();
+    if (run && run != best) atomicMax(&second, run);
+    __syncthreads();
+    if (t == 0) {
+        giant[0] = (best >> 32) >= kGiantMin ? (uint32_t)best : kNonCore;
+        giant[1] = (second >> 32) >= kGiantMin ? (uint32_t)second : kNonCore;
+        giant[2] = 0;   // k_union's range counter
+    }
+}
+
+// Membership bitmaps of A and B after the pre-pass (bit p of word p/32).
+__global__ void __launch_bounds__(256) k_giant_bits(uint64_t n, const uint32_t* __restrict__ parent,
+                                                    const uint32_t* __restrict__ giant, uint32_t* __restrict__ bits_a,
+                                                    uint32_t* __restrict__ bits_b) {
+    const uint32_t A = giant[0], B = giant[1];
+    const uint64_t nw = (n + 31) / 32;
+    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < 32 * nw;
+         i += (uint64_t)gridDim.x * blockDim.x) {
+        uint32_t r = kNonCore;
+        if (i < n && A != kNonCore && __ldcg(&parent[i]) != kNonCore) r = find_fast(parent, (uint32_t)i);
+        const unsigned ma = __ballot_sync(FULL, r == A && r != kNonCore);
+        const unsigned mb = __ballot_sync(FULL, r == B && r != kNonCore);
+        if ((threadIdx.x & 31) == 0) {
+            bits_a[i / 32] = ma;
+            bits_b[i / 32] = mb;
+        }
+    }
+}
+
+__device__ __forceinline__ bool bit_of(const uint32_t* __restrict__ bits, uint32_t v) {
+    return (__ldg(&bits[v >> 5]) >> (v & 31)) & 1u;
+}
+
+// Main pass.  One CTA per SM takes pair-balanced ranges of the production
+// (cell-sorted) order from a global counter; its warps take kRowsPerGrab
+// consecutive rows at a time from a shared counter, so an SM works in one small
+// region of space and its random parent[v] reads share L1.
+//
+// Which core-core edges (u, v) a row u processes, with A, B the giant
+// components of the pre-pass (each edge of the graph ends up processed once,
+// or is already inside one component):
+//   u in A:        none           (A-A: one component; A-x: done by x's side)
+//   u in B:        v in A         (B-B: one component; B-other: done by other's side)
+//   u elsewhere:   v in A or B, or v < u (other-other edges from the larger end)
+// Processing = one load of parent[v] (kNonCore: v not core); skip if v hangs
+// under u's root; else follow the chain and unite if the roots differ.
+__global__ void __launch_bounds__(kUnionThreads, 1)
+    k_union(const uint64_t* __restrict__ begin, const uint32_t* __restrict__ count, const uint32_t* __restrict__ nbrs,
+            const uint32_t* __restrict__ rows, uint32_t n, uint64_t npairs, uint32_t* __restrict__ parent,
+            uint32_t* __restrict__ giant, const uint32_t* __restrict__ bits_a, const uint32_t* __restrict__ bits_b) {
+    __shared__ uint32_t s_next, s_end, s_range;
+    const bool have_a = giant[0] != kNonCore, have_b = giant[1] != kNonCore;
+    const uint32_t R = gridDim.x * kRangesPerCta;
+    const int lane = threadIdx.x & 31;
+    while (true) {
+        if (threadIdx.x == 0) {
+            const uint32_t c = atomicAdd(&giant[2], 1u);   // next range (persistent CTAs)
+            s_range = c;
+            if (c < R) {
+                if (rows) {
+                    s_next = row_of_pair(begin, rows, n, npairs * c / R);
+                    s_end = c + 1 == R ? n : row_of_pair(begin, rows, n, npairs * (c + 1) / R);
+                } else {
+                    s_next = (uint32_t)((uint64_t)n * c / R);
+                    s_end = (uint32_t)((uint64_t)n * (c + 1) / R);
+                }
+            }
+        }
+        __syncthreads();
+        if (s_range >= R) return;
+        const uint32_t end = s_end;
+        while (true) {
+            uint32_t r0 = 0;
+            if (lane == 0) r0 = atomicAdd(&s_next, kRowsPerGrab);
+            r0 = __shfl_sync(FULL, r0, 0);
+            if (r0 >= end) break;
+            const uint32_t r1 = min(end, r0 + kRowsPerGrab);
+            for (uint32_t r = r0; r < r1; ++r) {
+                const uint32_t u = rows ? __ldg(&rows[r]) : r;
+                if (have_a && bit_of(bits_a, u)) continue;                 // uniform
+                if (__ldca(&parent[u]) == kNonCore) continue;              // uniform: non-core rows add no edge
+                const bool in_b = have_b && bit_of(bits_b, u);
+                const uint32_t* L = nbrs + begin[u];
+                const uint32_t m = count[u];
+                uint32_t ru = find_fast(parent, u);
+                for (uint32_t j0 = 0; j0 < m; j0 += 128) {
+                    uint32_t v[4], p[4];
 #pragma unroll
-                for (int k = 0; k < 4; ++k) p[k] = v[k] < u ? __ldca(&parent[v[k]]) : kNonCore;
+                    for (int k = 0; k < 4; ++k) {
+                        const uint32_t j = j0 + lane + 32 * k;
+                        v[k] = j < m ? __ldg(&L[j]) : 0xffffffffu;
+                    }
 #pragma unroll
-                for (int k = 0; k < 4; ++k) {
-                    // skip non-cores and v hanging directly under u's root; else follow the chain
-                    if (p[k] != kNonCore && p[k] != ru && !(p[k] != v[k] && reaches(parent, p[k], ru))) {
-                        unite(parent, u, v[k]);
-                        ru = find_fast(parent, u);
+                    for (int k = 0; k < 4; ++k) {
+                        bool take = false;
+                        if (v[k] != 0xffffffffu) {
+                            const bool va = have_a && bit_of(bits_a, v[k]);
+                            take = in_b ? va : (va || v[k] < u || (have_b && bit_of(bits_b, v[k])));
+                        }
+                        p[k] = take ? __ldca(&parent[v[k]]) : kNonCore;
+                    }
+#pragma unroll
+                    for (int k = 0; k < 4; ++k) {
+                        // skip non-cores and v hanging directly under u's root; else follow the chain
+                        if (p[k] != kNonCore && p[k] != ru && !(p[k] != v[k] && reaches(parent, p[k], ru))) {
+                            unite(parent, u, v[k]);
+                            ru = find_fast(parent, u);
+                        }
                     }
                 }
             }
         }
+        __syncthreads();   // every warp is done with this range
     }
 }
 
@@ -217,9 +344,13 @@ inline unsigned blocks_for(uint64_t n, unsigned cap = 148u * 16u) {
 
 void launch_dbscan_device(const uint64_t* begin, const uint32_t* count, const uint32_t* nbrs, const uint32_t* rows,
                           uint64_t n, uint64_t npairs, uint32_t minpts, uint8_t* core, uint32_t* parent, uint32_t* root,
-                          uint32_t* is_root, uint32_t* rank, void* scan_temp, int32_t* labels, cudaStream_t s) {
+                          uint32_t* is_root, uint32_t* rank, uint32_t* giant, uint32_t* bits, void* scan_temp,
+                          int32_t* labels, cudaStream_t s) {
     if (n == 0) return;
     k_core_init<<<blocks_for(n), 256, 0, s>>>(count, n, minpts, core, parent);
+    k_sample_link<<<blocks_for(n), 256, 0, s>>>(begin, count, nbrs, rows, n, parent);
+    k_giant<<<1, kGiantSamples, 0, s>>>(rows, n, parent, giant);
+    k_giant_bits<<<blocks_for(n), 256, 0, s>>>(n, parent, giant, bits, bits + (n + 31) / 32);
     static int sms = 0;
     if (!sms) {
         int dev = 0;
@@ -228,11 +359,12 @@ void launch_dbscan_device(const uint64_t* begin, const uint32_t* count, const ui
         cudaFuncSetAttribute(k_union, cudaFuncAttributePreferredSharedMemoryCarveout, 0);   // all of it as L1
         if (sms <= 0) sms = 148;
     }
-    k_union<<<sms, kUnionThreads, 0, s>>>(begin, count, nbrs, rows, (uint32_t)n, npairs, parent);
+    k_union<<<sms, kUnionThreads, 0, s>>>(begin, count, nbrs, rows, (uint32_t)n, npairs, parent, giant, bits,
+                                          bits + (n + 31) / 32);
     k_flatten<<<blocks_for(n), 256, 0, s>>>(core, n, parent, root, is_root);
     scan_u32_to_u32(is_root, rank, n, scan_temp, s);
     k_labels<<<blocks_for(n), 256, 0, s>>>(begin, count, nbrs, rows, core, root, rank, n, labels);
-    g_kernel_launches += 4;
+    g_kernel_launches += 7;
 }
 
 }  // namespace hdb

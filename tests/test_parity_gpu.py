@@ -479,6 +479,43 @@ def test_device_dbscan_matches_oracle(torch_cuda, split):
         assert np.array_equal(dlab.cpu().numpy(), want[0])
 
 
+def _giants(seed, bridge):
+    """Two dense squares (giant components A, B of the union pre-pass) + sparse
+    background + optionally a thin chain of points joining the squares."""
+    rng = np.random.default_rng(seed)
+    a = rng.uniform((0, 0), (10, 10), size=(12_000, 2))
+    b = rng.uniform((20, 0), (30, 10), size=(9_000, 2))
+    c = rng.uniform((-5, -5), (35, 15), size=(2_000, 2))
+    parts = [a, b, c]
+    if bridge:
+        x = np.arange(10.0, 20.0001, 0.2)
+        parts.append(np.stack([x, np.full_like(x, 5.0)], axis=1))
+    xy = np.concatenate(parts)
+    return xy[rng.permutation(xy.shape[0])]
+
+
+@pytest.mark.parametrize("bridge", [False, True])
+def test_device_dbscan_giant_components(torch_cuda, bridge):
+    """Exercises the giant-component skip rule of k_union: rows in A skip, rows in
+    B take only edges into A, other rows take edges into A/B and v < u."""
+    xy = _giants(5, bridge)
+    for eps, minpts in ((0.25, 4), (0.25, 12), (0.5, 30)):
+        want = oracle.dbscan(*oracle.eps_join(xy, eps), minpts)
+        ctx = _ctx()
+        try:
+            g = hdb.hdb_grid_build(ctx, xy, eps)
+            t = hdb.hdb_neighbor_table_device(ctx, g)
+            hdb.hdb_grid_free(g)
+            for _ in range(3):
+                lab, core, k = hdb.hdb_dbscan(t, minpts)
+                assert k == want[2]
+                assert np.array_equal(core, want[1])
+                assert np.array_equal(lab, want[0])
+            hdb.hdb_table_free(t)
+        finally:
+            hdb.hdb_ctx_destroy(ctx)
+
+
 def test_device_dbscan_shared_border_orders(torch_cuda):
     import json
     import os

@@ -26,6 +26,16 @@ for _ in range(5):
 torch.cuda.synchronize()
 print("device dbscan ms", (time.perf_counter() - t0) / 5 * 1e3, "clusters", k)
 th = hdb.hdb_neighbor_table(ctx, g)
+if os.environ.get("GIANT"):
+    import ctypes
+    L = lab.cpu().numpy()
+    v = hdb.hdb_table_view_get(th)
+    cnt_np = np.ctypeslib.as_array(ctypes.cast(v.count, ctypes.POINTER(ctypes.c_uint32)), shape=(n,))
+    sizes = np.bincount(L[L >= 0])
+    top = np.argsort(sizes)[::-1][:5]
+    pairs = np.bincount(L[L >= 0], weights=cnt_np[L >= 0].astype(np.float64))
+    print("top clusters: point share", [round(sizes[c] / n, 3) for c in top],
+          "pair share", [round(pairs[c] / v.npairs, 3) for c in top], flush=True)
 labh = np.empty(n, np.int32)
 for threads in (1, 16, 0):
     t0 = time.perf_counter()
