@@ -770,7 +770,7 @@ uint32_t dbscan_device(const hdb_table* t, uint32_t minpts, int32_t* labels, uin
     const bool lab_dev = li.loc == Loc::Device && li.device == t->device;
     const bool core_dev = core && ci.loc == Loc::Device && ci.device == t->device;
     DBuf dlab, dcore(n, s), parent(4 * n, s), root(4 * n, s), is_root(4 * n, s), rank(4 * (n + 1), s),
-        temp(scan_temp_bytes(n + 1), s), giant(16, s), bits(8 * ((n + 31) / 32), s);
+        temp(scan_temp_bytes(n + 1), s), giant(16, s), bits(8 * ((n + 31) / 32), s), sched(8 * 1024, s);
     int32_t* L = labels;
     if (!lab_dev) {
         dlab = DBuf(4 * n, s);
@@ -779,7 +779,7 @@ uint32_t dbscan_device(const hdb_table* t, uint32_t minpts, int32_t* labels, uin
     uint8_t* C = core_dev ? core : dcore.as<uint8_t>();
     launch_dbscan_device(t->begin, t->count, t->nbrs, t->rows, n, t->npairs, minpts, C, parent.as<uint32_t>(),
                          root.as<uint32_t>(), is_root.as<uint32_t>(), rank.as<uint32_t>(), giant.as<uint32_t>(),
-                         bits.as<uint32_t>(), temp.p, L, s);
+                         bits.as<uint32_t>(), sched.as<uint32_t>(), temp.p, L, s);
     HDB_LAUNCH_CHECK();
     uint32_t k = 0;
     HDB_CUDA(cudaMemcpyAsync(&k, rank.as<uint32_t>() + n, 4, cudaMemcpyDeviceToHost, s));

@@ -138,7 +138,7 @@ void launch_pos_to_group(const uint32_t* gstart, uint64_t n_groups, const uint64
 void launch_dbscan_device(const uint64_t* begin, const uint32_t* count, const uint32_t* nbrs, const uint32_t* rows,
                           uint64_t n, uint64_t npairs, uint32_t minpts, uint8_t* core, uint32_t* parent,
                           uint32_t* root, uint32_t* is_root, uint32_t* rank, uint32_t* giant, uint32_t* bits,
-                          void* scan_temp, int32_t* labels, cudaStream_t s);
+                          uint32_t* sched /* 2 x SM count */, void* scan_temp, int32_t* labels, cudaStream_t s);
 // T assembly by original id: begin[ids[q]] = off[q] - off[q0] + base, count[ids[q]] = cnt[q], q in [q0,q1)
 void launch_scatter_rows(const uint32_t* ids, const uint64_t* off, const uint32_t* cnt, uint64_t q0,
                          uint64_t q1, uint64_t base, uint64_t* begin, uint32_t* count, cudaStream_t s);

@@ -100,7 +100,6 @@ __device__ __forceinline__ bool reaches(const uint32_t* __restrict__ parent, uin
 
 constexpr uint32_t kRowsPerGrab = 4;      // consecutive (cell-sorted) rows per warp grab
 constexpr int kUnionThreads = 1024;       // one CTA per SM
-constexpr uint32_t kRangesPerCta = 32;    // pair-balanced ranges, taken dynamically
 
 // first row r in [0, n) with begin[rows[r]] >= x (begin is non-decreasing
 // along the production order of a whole table)
@@ -121,27 +120,39 @@ constexpr uint32_t kSampleLinks = 2;   // edges per core linked before the full 
 // kSampleLinks of its core neighbours, taken at evenly spaced list positions.
 // On an eps-graph this already assembles most of every dense cluster.  The
 // read-only root test first keeps the CAS traffic off the giant roots.
+// Round k links every core u with its list entry at position m*k/(kSampleLinks+1);
+// k_compress between rounds points every core straight at its root.
 __global__ void __launch_bounds__(256) k_sample_link(const uint64_t* __restrict__ begin,
                                                      const uint32_t* __restrict__ count,
                                                      const uint32_t* __restrict__ nbrs,
-                                                     const uint32_t* __restrict__ rows, uint64_t n,
+                                                     const uint32_t* __restrict__ rows, uint64_t n, uint32_t k,
                                                      uint32_t* __restrict__ parent) {
     for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
         const uint32_t u = rows ? rows[i] : (uint32_t)i;
-        if (__ldcg(&parent[u]) == kNonCore) continue;
-        const uint32_t* L = nbrs + begin[u];
-        const uint32_t m = count[u];
-        for (uint32_t k = 1; k <= kSampleLinks; ++k) {
-            const uint32_t v = L[(uint64_t)m * k / (kSampleLinks + 1)];
-            if (v != u && __ldcg(&parent[v]) != kNonCore && find_fast(parent, u) != find_fast(parent, v))
-                unite(parent, u, v);
+        const uint32_t pu = __ldcg(&parent[u]);
+        if (pu == kNonCore) continue;
+        const uint32_t v = nbrs[begin[u] + (uint64_t)count[u] * k / (kSampleLinks + 1)];
+        const uint32_t pv = __ldcg(&parent[v]);
+        if (v != u && pv != kNonCore && pv != pu) unite(parent, u, v);
+    }
+}
+
+__global__ void __launch_bounds__(256) k_compress(uint64_t n, uint32_t* __restrict__ parent) {
+    for (uint64_t p = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; p < n; p += (uint64_t)gridDim.x * blockDim.x) {
+        const uint32_t q = __ldcg(&parent[p]);
+        if (q == kNonCore || q == (uint32_t)p) continue;
+        uint32_t r = q, x = __ldcg(&parent[r]);
+        while (x != r) {
+            r = x;
+            x = __ldcg(&parent[r]);
         }
+        if (r != q) __stcg(&parent[p], r);
     }
 }
 
 // One CTA: the two most frequent roots among 1024 sampled points after the
 // pre-pass (the "giant" components A = giant[0], B = giant[1]; kNonCore if a
-// root holds fewer than kGiantMin samples).  Also resets k_union's counter.
+// root holds fewer than kGiantMin samples).
 constexpr int kGiantSamples = 1024;
 constexpr unsigned long long kGiantMin = kGiantSamples / 8;
 __global__ void __launch_bounds__(kGiantSamples) k_giant(const uint32_t* __restrict__ rows, uint64_t n,
@@ -183,7 +194,6 @@ __global__ void __launch_bounds__(kGiantSamples) k_giant(const uint32_t* __restr
     if (t == 0) {
         giant[0] = (best >> 32) >= kGiantMin ? (uint32_t)best : kNonCore;
         giant[1] = (second >> 32) >= kGiantMin ? (uint32_t)second : kNonCore;
-        giant[2] = 0;   // k_union's range counter
     }
 }
 
@@ -210,10 +220,27 @@ __device__ __forceinline__ bool bit_of(const uint32_t* __restrict__ bits, uint32
     return (__ldg(&bits[v >> 5]) >> (v & 31)) & 1u;
 }
 
-// Main pass.  One CTA per SM takes pair-balanced ranges of the production
-// (cell-sorted) order from a global counter; its warps take kRowsPerGrab
-// consecutive rows at a time from a shared counter, so an SM works in one small
-// region of space and its random parent[v] reads share L1.
+// Work regions of k_union: region c = rows [sched[c], sched[G + c]) of the
+// production order holding ~1/G of the pairs; sched[c] doubles as the region's
+// grab counter.
+__global__ void k_sched_init(const uint64_t* __restrict__ begin, const uint32_t* __restrict__ rows, uint32_t n,
+                             uint64_t npairs, uint32_t G, uint32_t* __restrict__ sched) {
+    for (uint32_t c = threadIdx.x; c < G; c += blockDim.x) {
+        if (rows) {
+            sched[c] = row_of_pair(begin, rows, n, npairs * c / G);
+            sched[G + c] = c + 1 == G ? n : row_of_pair(begin, rows, n, npairs * (c + 1) / G);
+        } else {
+            sched[c] = (uint32_t)((uint64_t)n * c / G);
+            sched[G + c] = (uint32_t)((uint64_t)n * (c + 1) / G);
+        }
+    }
+}
+
+// Main pass.  CTA c (one per SM) starts in region c; its warps take
+// kRowsPerGrab consecutive rows at a time from the region's counter, so an SM
+// works in one small region of space and its random parent[v] reads share L1.
+// A warp whose region is exhausted moves on to region c+1, c+2, ... (work
+// stealing without barriers).
 //
 // Which core-core edges (u, v) a row u processes, with A, B the giant
 // components of the pre-pass (each edge of the graph ends up processed once,
@@ -225,34 +252,23 @@ __device__ __forceinline__ bool bit_of(const uint32_t* __restrict__ bits, uint32
 // under u's root; else follow the chain and unite if the roots differ.
 __global__ void __launch_bounds__(kUnionThreads, 1)
     k_union(const uint64_t* __restrict__ begin, const uint32_t* __restrict__ count, const uint32_t* __restrict__ nbrs,
-            const uint32_t* __restrict__ rows, uint32_t n, uint64_t npairs, uint32_t* __restrict__ parent,
-            uint32_t* __restrict__ giant, const uint32_t* __restrict__ bits_a, const uint32_t* __restrict__ bits_b) {
-    __shared__ uint32_t s_next, s_end, s_range;
+            const uint32_t* __restrict__ rows, uint32_t* __restrict__ parent, const uint32_t* __restrict__ giant,
+            const uint32_t* __restrict__ bits_a, const uint32_t* __restrict__ bits_b, uint32_t* __restrict__ sched) {
     const bool have_a = giant[0] != kNonCore, have_b = giant[1] != kNonCore;
-    const uint32_t R = gridDim.x * kRangesPerCta;
+    const uint32_t G = gridDim.x;
     const int lane = threadIdx.x & 31;
-    while (true) {
-        if (threadIdx.x == 0) {
-            const uint32_t c = atomicAdd(&giant[2], 1u);   // next range (persistent CTAs)
-            s_range = c;
-            if (c < R) {
-                if (rows) {
-                    s_next = row_of_pair(begin, rows, n, npairs * c / R);
-                    s_end = c + 1 == R ? n : row_of_pair(begin, rows, n, npairs * (c + 1) / R);
-                } else {
-                    s_next = (uint32_t)((uint64_t)n * c / R);
-                    s_end = (uint32_t)((uint64_t)n * (c + 1) / R);
-                }
-            }
-        }
-        __syncthreads();
-        if (s_range >= R) return;
-        const uint32_t end = s_end;
-        while (true) {
+    uint32_t region = blockIdx.x, visited = 0;
+    while (visited < G) {
+        {
             uint32_t r0 = 0;
-            if (lane == 0) r0 = atomicAdd(&s_next, kRowsPerGrab);
+            if (lane == 0) r0 = atomicAdd(&sched[region], kRowsPerGrab);
             r0 = __shfl_sync(FULL, r0, 0);
-            if (r0 >= end) break;
+            const uint32_t end = __ldg(&sched[G + region]);
+            if (r0 >= end) {
+                region = region + 1 == G ? 0 : region + 1;
+                ++visited;
+                continue;
+            }
             const uint32_t r1 = min(end, r0 + kRowsPerGrab);
             for (uint32_t r = r0; r < r1; ++r) {
                 const uint32_t u = rows ? __ldg(&rows[r]) : r;
@@ -289,7 +305,6 @@ __global__ void __launch_bounds__(kUnionThreads, 1)
                 }
             }
         }
-        __syncthreads();   // every warp is done with this range
     }
 }
 
@@ -344,11 +359,14 @@ inline unsigned blocks_for(uint64_t n, unsigned cap = 148u * 16u) {
 
 void launch_dbscan_device(const uint64_t* begin, const uint32_t* count, const uint32_t* nbrs, const uint32_t* rows,
                           uint64_t n, uint64_t npairs, uint32_t minpts, uint8_t* core, uint32_t* parent, uint32_t* root,
-                          uint32_t* is_root, uint32_t* rank, uint32_t* giant, uint32_t* bits, void* scan_temp,
-                          int32_t* labels, cudaStream_t s) {
+                          uint32_t* is_root, uint32_t* rank, uint32_t* giant, uint32_t* bits, uint32_t* sched,
+                          void* scan_temp, int32_t* labels, cudaStream_t s) {
     if (n == 0) return;
     k_core_init<<<blocks_for(n), 256, 0, s>>>(count, n, minpts, core, parent);
-    k_sample_link<<<blocks_for(n), 256, 0, s>>>(begin, count, nbrs, rows, n, parent);
+    for (uint32_t k = 1; k <= kSampleLinks; ++k) {
+        k_sample_link<<<blocks_for(n), 256, 0, s>>>(begin, count, nbrs, rows, n, k, parent);
+        k_compress<<<blocks_for(n), 256, 0, s>>>(n, parent);
+    }
     k_giant<<<1, kGiantSamples, 0, s>>>(rows, n, parent, giant);
     k_giant_bits<<<blocks_for(n), 256, 0, s>>>(n, parent, giant, bits, bits + (n + 31) / 32);
     static int sms = 0;
@@ -359,12 +377,12 @@ void launch_dbscan_device(const uint64_t* begin, const uint32_t* count, const ui
         cudaFuncSetAttribute(k_union, cudaFuncAttributePreferredSharedMemoryCarveout, 0);   // all of it as L1
         if (sms <= 0) sms = 148;
     }
-    k_union<<<sms, kUnionThreads, 0, s>>>(begin, count, nbrs, rows, (uint32_t)n, npairs, parent, giant, bits,
-                                          bits + (n + 31) / 32);
+    k_sched_init<<<1, 256, 0, s>>>(begin, rows, (uint32_t)n, npairs, (uint32_t)sms, sched);
+    k_union<<<sms, kUnionThreads, 0, s>>>(begin, count, nbrs, rows, parent, giant, bits, bits + (n + 31) / 32, sched);
     k_flatten<<<blocks_for(n), 256, 0, s>>>(core, n, parent, root, is_root);
     scan_u32_to_u32(is_root, rank, n, scan_temp, s);
     k_labels<<<blocks_for(n), 256, 0, s>>>(begin, count, nbrs, rows, core, root, rank, n, labels);
-    g_kernel_launches += 7;
+    g_kernel_launches += 7 + 2 * kSampleLinks;
 }
 
 }  // namespace hdb
