@@ -150,6 +150,22 @@ def lattice(k: int, spacing: float = 1.0, origin=(0.0, 0.0)) -> np.ndarray:
                                 dtype=np.float64)
 
 
+def giants(seed: int = 5, bridge: bool = False) -> np.ndarray:
+    """Two dense squares (12,000 and 9,000 points; the giant components of the
+    union-find pre-pass) + 2,000 background points, optionally joined by a
+    thin chain of points (spacing 0.2) -- test input for the DBSCAN skip rules."""
+    rng = _rng(seed)
+    a = rng.uniform((0, 0), (10, 10), size=(12_000, 2))
+    b = rng.uniform((20, 0), (30, 10), size=(9_000, 2))
+    c = rng.uniform((-5, -5), (35, 15), size=(2_000, 2))
+    parts = [a, b, c]
+    if bridge:
+        x = np.arange(10.0, 20.0001, 0.2)
+        parts.append(np.stack([x, np.full_like(x, 5.0)], axis=1))
+    xy = np.concatenate(parts)
+    return xy[rng.permutation(xy.shape[0])]
+
+
 def near_ties(m: int, eps: float, seed: int = 11, extent: float = 400.0) -> np.ndarray:
     """Adversarial near-tie set: pairs of points whose distance is eps up to
     a few ulps, at random offsets inside a large extent so that cell

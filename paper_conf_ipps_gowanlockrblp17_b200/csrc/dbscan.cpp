@@ -13,9 +13,11 @@
 //   noise     = everything else, label -1.
 // Two implementations with identical output:
 //   * sequential: cluster-at-a-time BFS over cores in id order (n_threads == 1);
-//   * parallel:   lock-free union-find over core-core edges with min-id roots,
-//                 root ranks by a prefix count, borders by a min over core
-//                 neighbours (NEXT-2; the paper runs variants, not one
+//   * parallel:   lock-free union-find over core-core edges with min-id roots
+//                 (Afforest-style sampled links, then the lists of the two
+//                 giant components skipped by the rule in dbscan_par, as the
+//                 device code), root ranks by a prefix count, borders by a min
+//                 over core neighbours (NEXT-2; the paper runs variants, not one
 //                 variant, in parallel).
 #include <algorithm>
 #include <atomic>
@@ -114,7 +116,64 @@ uint32_t dbscan_par(const hdb_table* t, uint32_t minpts, int T, int32_t* labels,
             parent[p].store((uint32_t)p, std::memory_order_relaxed);
         }
     });
-    // union over core-core edges (each unordered edge once: v < u)
+    // Afforest-style pre-pass (as the device code): two rounds of one sampled
+    // link per core, each followed by a compression of every core to its root.
+    for (uint32_t k = 1; k <= 2; ++k) {
+        parallel_for(T, n, [&](uint64_t a, uint64_t b, int) {
+            for (uint64_t u = a; u < b; ++u) {
+                if (!core[u] || C[u] == 0) continue;
+                const uint32_t v = V[B[u] + (uint64_t)C[u] * k / 3];
+                if (v != u && core[v]) uf_union(parent.get(), (uint32_t)u, v);
+            }
+        });
+        parallel_for(T, n, [&](uint64_t a, uint64_t b, int) {
+            for (uint64_t p = a; p < b; ++p)
+                if (core[p]) parent[p].store(uf_find(parent.get(), (uint32_t)p), std::memory_order_relaxed);
+        });
+    }
+    // the two most frequent roots among 1024 sampled points (>= 1/8 of them):
+    // giant components A and B, with membership bitmaps
+    const uint32_t kNone = 0xffffffffu;
+    uint32_t gA = kNone, gB = kNone;
+    if (n >= 4096) {
+        std::vector<uint32_t> smp;
+        for (uint64_t i = 0; i < 1024; ++i) {
+            const uint64_t p = i * n / 1024;
+            if (core[p]) smp.push_back(uf_find(parent.get(), (uint32_t)p));
+        }
+        std::sort(smp.begin(), smp.end());
+        std::vector<std::pair<uint32_t, uint32_t>> runs;   // (count, root)
+        for (size_t i = 0; i < smp.size();) {
+            size_t j = i;
+            while (j < smp.size() && smp[j] == smp[i]) ++j;
+            runs.emplace_back((uint32_t)(j - i), smp[i]);
+            i = j;
+        }
+        std::sort(runs.begin(), runs.end(), std::greater<>());
+        if (runs.size() > 0 && runs[0].first >= 128) gA = runs[0].second;
+        if (runs.size() > 1 && runs[1].first >= 128) gB = runs[1].second;
+    }
+    const uint64_t nw = (n + 63) / 64;
+    std::vector<uint64_t> bitA(gA != kNone ? nw : 0), bitB(gB != kNone ? nw : 0);
+    if (gA != kNone) {
+        parallel_for(T, nw, [&](uint64_t a, uint64_t b, int) {
+            for (uint64_t w = a; w < b; ++w) {
+                uint64_t ma = 0, mb = 0;
+                for (uint64_t p = 64 * w; p < std::min(n, 64 * w + 64); ++p) {
+                    if (!core[p]) continue;
+                    const uint32_t r = uf_find(parent.get(), (uint32_t)p);
+                    if (r == gA) ma |= 1ull << (p & 63);
+                    if (r == gB) mb |= 1ull << (p & 63);
+                }
+                bitA[w] = ma;
+                if (gB != kNone) bitB[w] = mb;
+            }
+        });
+    }
+    auto inA = [&](uint32_t v) { return gA != kNone && ((bitA[v >> 6] >> (v & 63)) & 1); };
+    auto inB = [&](uint32_t v) { return gB != kNone && ((bitB[v >> 6] >> (v & 63)) & 1); };
+    // Main pass.  Each core-core edge not inside A or B is taken once:
+    //   u in A: none; u in B: v in A; otherwise: v in A or B, or v < u.
     {
         std::atomic<uint64_t> next{0};
         const uint64_t blk = 2048;
@@ -124,12 +183,14 @@ uint32_t dbscan_par(const hdb_table* t, uint32_t minpts, int T, int32_t* labels,
                 if (a >= n) break;
                 uint64_t b = std::min(n, a + blk);
                 for (uint64_t u = a; u < b; ++u) {
-                    if (!core[u]) continue;
+                    if (!core[u] || inA((uint32_t)u)) continue;
+                    const bool ub = inB((uint32_t)u);
                     const uint32_t* L = V + B[u];
                     uint32_t ru = uf_find(parent.get(), (uint32_t)u);   // kept current across the list
                     for (uint32_t i = 0, m = C[u]; i < m; ++i) {
                         const uint32_t v = L[i];
-                        if (v >= u || !core[v]) continue;
+                        const bool va = inA(v);
+                        if (!(ub ? va : (va || v < u || inB(v))) || !core[v]) continue;
                         const uint32_t rv = uf_find(parent.get(), v);
                         if (rv == ru) continue;                        // already joined: no link needed
                         uf_union(parent.get(), ru, rv);

@@ -957,10 +957,12 @@ void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hd
                 memset(t->begin, 0, 8 * (n ? n : 1));
                 memset(t->count, 0, 4 * (n ? n : 1));
             }
+            tr.mark("pinned-pool");
             std::vector<uint64_t> dev_grows(ndev, 0);
             run_parallel(ndev, [&](size_t d) {
                 write_phase_host(ctx, ctx->dev[d], grid->dev[d], sh[d], t->nbrs, batch_pairs, &dev_grows[d]);
             });
+            tr.mark("write+d2h");
             // begin/count by original id
             if (whole) {
                 DevCtx& dc = ctx->dev[0];

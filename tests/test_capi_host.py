@@ -103,6 +103,25 @@ def test_host_dbscan_matches_oracle(threads):
         assert np.array_equal(lab, want_lab)
 
 
+@pytest.mark.parametrize("bridge", [False, True])
+def test_host_dbscan_giant_components(bridge):
+    """Exercises the parallel host DBSCAN's giant-component skip rule (two dense
+    squares -> giants A and B; optional bridge -> A-B edges through other rows)."""
+    xy = datagen.giants(5, bridge)
+    for eps, minpts in ((0.25, 4), (0.25, 12), (0.5, 30)):
+        off, nbr = oracle.eps_join(xy, eps)
+        want = oracle.dbscan(off, nbr, minpts)
+        t = _lib_table(off, nbr)
+        try:
+            for threads in (4, 16):
+                lab, core, k = hdb.hdb_dbscan(t, minpts, n_threads=threads)
+                assert k == want[2]
+                assert np.array_equal(core, want[1])
+                assert np.array_equal(lab, want[0])
+        finally:
+            hdb.hdb_table_free(t)
+
+
 def test_host_dbscan_shared_border_golden():
     g = _gold("border_orders.json")
     for o in g["orders"]:

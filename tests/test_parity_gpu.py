@@ -479,26 +479,11 @@ def test_device_dbscan_matches_oracle(torch_cuda, split):
         assert np.array_equal(dlab.cpu().numpy(), want[0])
 
 
-def _giants(seed, bridge):
-    """Two dense squares (giant components A, B of the union pre-pass) + sparse
-    background + optionally a thin chain of points joining the squares."""
-    rng = np.random.default_rng(seed)
-    a = rng.uniform((0, 0), (10, 10), size=(12_000, 2))
-    b = rng.uniform((20, 0), (30, 10), size=(9_000, 2))
-    c = rng.uniform((-5, -5), (35, 15), size=(2_000, 2))
-    parts = [a, b, c]
-    if bridge:
-        x = np.arange(10.0, 20.0001, 0.2)
-        parts.append(np.stack([x, np.full_like(x, 5.0)], axis=1))
-    xy = np.concatenate(parts)
-    return xy[rng.permutation(xy.shape[0])]
-
-
 @pytest.mark.parametrize("bridge", [False, True])
 def test_device_dbscan_giant_components(torch_cuda, bridge):
     """Exercises the giant-component skip rule of k_union: rows in A skip, rows in
     B take only edges into A, other rows take edges into A/B and v < u."""
-    xy = _giants(5, bridge)
+    xy = datagen.giants(5, bridge)
     for eps, minpts in ((0.25, 4), (0.25, 12), (0.5, 30)):
         want = oracle.dbscan(*oracle.eps_join(xy, eps), minpts)
         ctx = _ctx()
