@@ -415,12 +415,16 @@ def main():
     P = pairs_total // max(args.steps, 1)
     value = pairs_total / (ms / 1000.0)
 
-    # roofline of the dominant kernel: the neighbour write kernel (a8, k_emit),
-    # HBM-write bound.  Algorithmic bytes per launch:
-    # 4 B per pair written + 12 B per query (uint64 offset + uint32 id map).
+    # roofline of the dominant kernel, HBM-write bound:
+    #  * single pass (k_fused, device-resident tables): 4 B per pair written + per query
+    #    12 B (begin/count by id) + 4 B (sorted count) + the query/candidate reads of the
+    #    sorted coordinates and ids (16 B f64 / 8 B f32 + 4 B) = 4P + 36n (f64) / 4P + 28n (f32);
+    #  * two-pass write kernel (k_emit): 4 B per pair + 12 B per query (offset + id map).
     hbm, peak_kind = load_peaks()
     n_shard = (v.end_query - v.first_query) if ws > 1 else n
-    alg_bytes = 4 * v.npairs + 12 * n_shard
+    single = bool(st.get("single_pass", 0))
+    esz = 16 if args.dtype == "f64" else 8
+    alg_bytes = 4 * v.npairs + ((esz + 20) * n_shard if single else 12 * n_shard)
     wms = float(np.mean(write_ms))
     achieved = alg_bytes / (wms / 1000.0) / 1e9
     traffic = None
@@ -429,7 +433,6 @@ def main():
         with open(tp) as f:
             traffic = json.load(f).get(f"{args.workload}-{args.dtype}-k{args.kernel}-s{args.cell_split}")
     # whole-step view: SURVEY 8(d) B_alg = 4P + 64n + 8C (f64) over the step time
-    esz = 16 if args.dtype == "f64" else 8
     b_step = 4 * P + (4 * esz + 32) * n + 8 * st["n_nonempty"]
     cms = float(np.mean(count_ms))
 
@@ -444,15 +447,22 @@ def main():
             "gpu_launches": launches,
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
                          "frac": achieved / hbm, "traffic": traffic, "peak_kind": peak_kind,
-                         "kernel": "k_emit (neighbour write, a8)", "kernel_ms": wms, "alg_bytes": alg_bytes},
-            "count_kernel": {"bound": "alu", "kernel": "k_search (count + hit masks, a6)", "ms": cms,
-                             "tests": st["candidate_tests"],
-                             "tests_per_s": st["candidate_tests"] / (cms / 1e3) if cms > 0 else None},
+                         "kernel": ("k_fused (single pass: count + reserve + emit, a6-a8)" if single
+                                    else "k_emit (neighbour write, a8)"),
+                         "kernel_ms": wms, "alg_bytes": alg_bytes},
+            "count_kernel": ({"bound": "alu", "kernel": "k_fused (count part, a6)", "ms": wms,
+                              "tests": st["candidate_tests"],
+                              "tests_per_s": st["candidate_tests"] / (wms / 1e3) if wms > 0 else None,
+                              "note": "single pass: the count and write share one kernel"} if single else
+                             {"bound": "alu", "kernel": "k_count (count + hit masks, a6)", "ms": cms,
+                              "tests": st["candidate_tests"],
+                              "tests_per_s": st["candidate_tests"] / (cms / 1e3) if cms > 0 else None}),
             "step_roofline": {"alg_bytes": b_step, "achieved_gbs": b_step / (ms / args.steps / 1e3) / 1e9,
                               "frac": b_step / (ms / args.steps / 1e3) / 1e9 / hbm},
             "clocks": clk.summary(),
             "stats": {k: st[k] for k in ("n_nonempty", "n_groups", "candidate_tests", "ms_grid", "ms_sample",
-                                         "ms_count", "ms_scan", "ms_write_kernel", "kernel_launches")}}
+                                         "ms_count", "ms_scan", "ms_write_kernel", "kernel_launches",
+                                         "single_pass", "est_pairs")}}
 
     # ---- e2e through the C-ABI from pinned HOST points (H2D inside the timed region):
     #   value: the same metric (pairs/s) with the table delivered to a HOST table (D2H inside);

@@ -152,6 +152,9 @@ typedef struct {
     double ms_sample, ms_count, ms_scan;
     double ms_write_kernel;      /* summed device time of the write-kernel launches (CUDA events)  */
     double ms_table_wall;        /* host wall time of the whole table call                         */
+    int single_pass;             /* 1: the last device-resident table was built in one pass (count +
+                                    reserve + emit per query group, rows in reservation order);
+                                    ms_write_kernel is that kernel's time, ms_count = ms_scan = 0    */
 } hdb_stats;
 
 /* ---- context ------------------------------------------------------------- */

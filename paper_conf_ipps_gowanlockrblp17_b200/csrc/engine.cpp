@@ -650,6 +650,61 @@ void count_phase(hdb_ctx* ctx, DevCtx& dc, const DevGrid& g, ShardState& st) {
     st.ms_scan = elapsed(e1, e2);
 }
 
+// Single-pass device-resident table (k_fused: count + reserve + emit per
+// group; search_kernel = 4 -- measured slower than the two passes on B200,
+// see DESIGN.md).  The table is sized from the sampled estimate a_b (cap = 1.25
+// max(a_b, n) + 2^20 pairs).  Returns false -- nothing published, the caller
+// then runs the exact two-pass path (a6-a8) -- if the mask table or the table
+// cannot be allocated or a reservation passed the capacity.
+bool single_pass_table(hdb_ctx* ctx, const DevGrid& g, hdb_table* t, hdb_stats& S, uint64_t est) {
+    DevCtx& dc = ctx->dev[0];
+    cudaStream_t s = dc.main;
+    const uint64_t n = g.n;
+    const uint64_t cap = (uint64_t)((double)std::max<uint64_t>(est, n) * 1.25) + (1ull << 20);
+    DBuf masks, nb;
+    if (cudaMallocAsync(&masks.p, 4 * std::max<uint64_t>(g.mask_words, 4), s) != cudaSuccess ||
+        cudaMallocAsync(&nb.p, 4 * cap, s) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
+    masks.s = nb.s = s;
+    DBuf beg(8 * n, s), cnt_id(4 * n, s), cnt(4 * n, s), scratch(32, s);
+    HDB_CUDA(cudaMemsetAsync(scratch.p, 0, 32, s));
+    unsigned long long* sc = scratch.as<unsigned long long>();
+    Event e0, e1;
+    HDB_CUDA(cudaEventRecord(e0.e, s));
+    launch_fused(g, cnt.as<uint32_t>(), sc, masks.as<uint2>(), sc + 1, cap, nb.as<uint32_t>(), beg.as<uint64_t>(),
+                 cnt_id.as<uint32_t>(), (unsigned int*)(sc + 2), s);
+    HDB_LAUNCH_CHECK();
+    HDB_CUDA(cudaEventRecord(e1.e, s));
+    HDB_CUDA(cudaMemcpyAsync(dc.pin + 4, sc, 24, cudaMemcpyDeviceToHost, s));
+    masks.reset();
+    HDB_CUDA(cudaStreamSynchronize(s));
+    const uint64_t tests = dc.pin[4], P = dc.pin[5];
+    if ((uint32_t)dc.pin[6] != 0) return false;   // estimate exceeded: exact two-pass path
+    t->on_device = true;
+    t->device = dc.device;
+    t->dstream = s;
+    t->npairs = P;
+    t->first_query = 0;
+    t->end_query = n;
+    DBuf rw(4 * n, s);
+    HDB_CUDA(cudaMemcpyAsync(rw.p, g.ids, 4 * n, cudaMemcpyDeviceToDevice, s));
+    t->rows = (uint32_t*)rw.release();
+    t->nbrs = (uint32_t*)nb.release();
+    t->begin = (uint64_t*)beg.release();
+    t->count = (uint32_t*)cnt_id.release();
+    S.npairs = P;
+    S.candidate_tests = tests;
+    S.ms_count = S.ms_scan = 0;
+    S.ms_write_kernel = elapsed(e0, e1);
+    S.write_launches = 1;
+    S.n_batches = 1;
+    S.max_batch_pairs = P;
+    S.single_pass = 1;
+    return true;
+}
+
 void ensure_batch_buf(DevCtx& dc, size_t si, size_t pairs, uint64_t* grows) {
     if (dc.batch_buf.size() <= si) {
         dc.batch_buf.resize(si + 1, nullptr);
@@ -770,7 +825,7 @@ uint32_t dbscan_device(const hdb_table* t, uint32_t minpts, int32_t* labels, uin
     const bool lab_dev = li.loc == Loc::Device && li.device == t->device;
     const bool core_dev = core && ci.loc == Loc::Device && ci.device == t->device;
     DBuf dlab, dcore(n, s), parent(4 * n, s), root(4 * n, s), is_root(4 * n, s), rank(4 * (n + 1), s),
-        temp(scan_temp_bytes(n + 1), s), giant(16, s), bits(8 * ((n + 31) / 32), s), sched(8 * 1024, s);
+        temp(scan_temp_bytes(n + 1), s), giant(16, s), bits(8 * ((n + 31) / 32), s), sched(8 * 1024, s), pre(8 * (n + 1), s);
     int32_t* L = labels;
     if (!lab_dev) {
         dlab = DBuf(4 * n, s);
@@ -779,7 +834,7 @@ uint32_t dbscan_device(const hdb_table* t, uint32_t minpts, int32_t* labels, uin
     uint8_t* C = core_dev ? core : dcore.as<uint8_t>();
     launch_dbscan_device(t->begin, t->count, t->nbrs, t->rows, n, t->npairs, minpts, C, parent.as<uint32_t>(),
                          root.as<uint32_t>(), is_root.as<uint32_t>(), rank.as<uint32_t>(), giant.as<uint32_t>(),
-                         bits.as<uint32_t>(), sched.as<uint32_t>(), temp.p, L, s);
+                         bits.as<uint32_t>(), sched.as<uint32_t>(), pre.as<uint64_t>(), temp.p, L, s);
     HDB_LAUNCH_CHECK();
     uint32_t k = 0;
     HDB_CUDA(cudaMemcpyAsync(&k, rank.as<uint32_t>() + n, 4, cudaMemcpyDeviceToHost, s));
@@ -865,160 +920,181 @@ void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hd
             sh[d].r.g1 = cuts[k + 1];
         }
         tr.mark("sample+cuts");
-        // ---- a6/a7 on every device
-        run_parallel(ndev, [&](size_t d) { count_phase(ctx, ctx->dev[d], grid->dev[d], sh[d]); });
-        tr.mark("count_phase");
-        HDB_CUDA(cudaStreamSynchronize(s0));   // no-op when device 0 ran the count pass (same stream)
-        {
+        S.single_pass = 0;
+        bool single = false;
+        if (device_resident && parts == 1 && ctx->opts.search_kernel == 4 && n > 0) {
+            HDB_CUDA(cudaStreamSynchronize(s0));   // e_b is in dc0.pin[0]
             const uint64_t eb = dc0.pin[0];
             S.sample_size = ns;
             S.sample_pairs = eb;
-            S.est_pairs = eb * stride;   // a_b = e_b / f  (reading R15)
+            S.est_pairs = eb * stride;
             S.ms_sample = elapsed(es0, es1);
+            single = single_pass_table(ctx, G0, t, S, eb * stride);
+            if (single) {
+                double bb = 0;
+                uint64_t nbp = 0;
+                hdb_plan_batches((double)S.est_pairs, ctx->opts.alpha, ctx->opts.n_streams, &bb, &nbp);
+                S.planned_batch_pairs = (uint64_t)std::ceil(bb);
+                S.planned_batches = nbp;
+            }
+            tr.mark("single-pass");
         }
-        double bb_plan = 0;
-        uint64_t nb_plan = 0;
-        hdb_plan_batches((double)S.est_pairs, ctx->opts.alpha, ctx->opts.n_streams, &bb_plan, &nb_plan);
-        uint64_t batch_pairs = ctx->opts.batch_pairs ? ctx->opts.batch_pairs : (uint64_t)std::ceil(bb_plan);
-        batch_pairs = std::max<uint64_t>(batch_pairs, 1);
-        S.planned_batch_pairs = batch_pairs;
-        S.planned_batches = ctx->opts.batch_pairs
-                                ? (uint64_t)std::ceil((1.0 + ctx->opts.alpha) * (double)S.est_pairs / (double)batch_pairs)
-                                : nb_plan;
-        // ---- the final gather of counts: shard bases
-        uint64_t P = 0;
-        for (size_t d = 0; d < ndev; ++d) {
-            sh[d].base = P;
-            P += sh[d].pairs;
-        }
-        S.npairs = P;
-        S.candidate_tests = 0;
-        S.ms_count = S.ms_scan = 0;
-        for (auto& st : sh) {
-            S.candidate_tests += st.tests;
-            S.ms_count = std::max(S.ms_count, (double)st.ms_count);
-            S.ms_scan = std::max(S.ms_scan, (double)st.ms_scan);
-        }
-        if (ctx->opts.host_budget_bytes && 4 * P > ctx->opts.host_budget_bytes && !device_resident)
-            fail(HDB_ENOMEM, "table needs %llu bytes (P=%llu) > host budget %llu", (unsigned long long)(4 * P),
-                 (unsigned long long)P, (unsigned long long)ctx->opts.host_budget_bytes);
-        t->npairs = P;
-        const bool whole = (parts == 1);
-        t->first_query = whole ? 0 : sh[0].r.q0;
-        t->end_query = whole ? n : sh[ndev - 1].r.q1;
+        if (!single) {
+            // ---- a6/a7 on every device
+            run_parallel(ndev, [&](size_t d) { count_phase(ctx, ctx->dev[d], grid->dev[d], sh[d]); });
+            tr.mark("count_phase");
+            HDB_CUDA(cudaStreamSynchronize(s0));   // no-op when device 0 ran the count pass (same stream)
+            {
+                const uint64_t eb = dc0.pin[0];
+                S.sample_size = ns;
+                S.sample_pairs = eb;
+                S.est_pairs = eb * stride;   // a_b = e_b / f  (reading R15)
+                S.ms_sample = elapsed(es0, es1);
+            }
+            double bb_plan = 0;
+            uint64_t nb_plan = 0;
+            hdb_plan_batches((double)S.est_pairs, ctx->opts.alpha, ctx->opts.n_streams, &bb_plan, &nb_plan);
+            uint64_t batch_pairs = ctx->opts.batch_pairs ? ctx->opts.batch_pairs : (uint64_t)std::ceil(bb_plan);
+            batch_pairs = std::max<uint64_t>(batch_pairs, 1);
+            S.planned_batch_pairs = batch_pairs;
+            S.planned_batches = ctx->opts.batch_pairs
+                                    ? (uint64_t)std::ceil((1.0 + ctx->opts.alpha) * (double)S.est_pairs / (double)batch_pairs)
+                                    : nb_plan;
+            // ---- the final gather of counts: shard bases
+            uint64_t P = 0;
+            for (size_t d = 0; d < ndev; ++d) {
+                sh[d].base = P;
+                P += sh[d].pairs;
+            }
+            S.npairs = P;
+            S.candidate_tests = 0;
+            S.ms_count = S.ms_scan = 0;
+            for (auto& st : sh) {
+                S.candidate_tests += st.tests;
+                S.ms_count = std::max(S.ms_count, (double)st.ms_count);
+                S.ms_scan = std::max(S.ms_scan, (double)st.ms_scan);
+            }
+            if (ctx->opts.host_budget_bytes && 4 * P > ctx->opts.host_budget_bytes && !device_resident)
+                fail(HDB_ENOMEM, "table needs %llu bytes (P=%llu) > host budget %llu", (unsigned long long)(4 * P),
+                     (unsigned long long)P, (unsigned long long)ctx->opts.host_budget_bytes);
+            t->npairs = P;
+            const bool whole = (parts == 1);
+            t->first_query = whole ? 0 : sh[0].r.q0;
+            t->end_query = whole ? n : sh[ndev - 1].r.q1;
 
-        if (device_resident) {
-            // ---- a8 into a device-resident table
-            DevCtx& dc = ctx->dev[0];
-            const DevGrid& g = grid->dev[0];
-            ShardState& st = sh[0];
-            cudaStream_t s = dc.main;
-            t->on_device = true;
-            t->device = dc.device;
-            t->dstream = s;
-            DBuf nb(4 * (P ? P : 1), s), beg(8 * (n ? n : 1), s), cnt(4 * (n ? n : 1), s);
-            if (!whole) {
-                HDB_CUDA(cudaMemsetAsync(beg.p, 0, 8 * (n ? n : 1), s));
-                HDB_CUDA(cudaMemsetAsync(cnt.p, 0, 4 * (n ? n : 1), s));
-            }
-            Event e0, e1;
-            HDB_CUDA(cudaEventRecord(e0.e, s));
-            launch_write(g, st.r.g0, st.r.g1, st.off.as<uint64_t>(), 0, nb.as<uint32_t>(), ctx->opts.search_kernel, 1,
-                         st.mask_base, s);
-            HDB_LAUNCH_CHECK();
-            HDB_CUDA(cudaEventRecord(e1.e, s));
-            launch_scatter_rows(g.ids, st.off.as<uint64_t>(), st.cnt.as<uint32_t>(), st.r.q0, st.r.q1, 0,
-                                beg.as<uint64_t>(), cnt.as<uint32_t>(), s);
-            HDB_LAUNCH_CHECK();
-            HDB_CUDA(cudaStreamSynchronize(s));
-            st.ms_write = elapsed(e0, e1);
-            tr.mark("alloc+write+scatter+sync");
-            st.write_launches = 1;
-            st.n_batches = 1;
-            st.max_batch = P;
-            if (whole && n) {
-                // production order of the rows: DBSCAN walks them in this (cell-sorted) order so
-                // that consecutive rows share neighbours (cache locality of the union-find)
-                DBuf rw(4 * n, s);
-                HDB_CUDA(cudaMemcpyAsync(rw.p, g.ids, 4 * n, cudaMemcpyDeviceToDevice, s));
-                t->rows = (uint32_t*)rw.release();
-            }
-            t->nbrs = (uint32_t*)nb.release();
-            t->begin = (uint64_t*)beg.release();
-            t->count = (uint32_t*)cnt.release();
-        } else {
-            // ---- a8/a9/a10 into the host table
-            t->pool = ctx->pinned;
-            uint64_t grows0 = ctx->pinned->grows;
-            t->nbrs = pool_get<uint32_t>(t, P ? P : 1, &t->cap_nbrs);
-            t->begin = pool_get<uint64_t>(t, n ? n : 1, &t->cap_begin);
-            t->count = pool_get<uint32_t>(t, n ? n : 1, &t->cap_count);
-            if (!whole) {
-                memset(t->begin, 0, 8 * (n ? n : 1));
-                memset(t->count, 0, 4 * (n ? n : 1));
-            }
-            tr.mark("pinned-pool");
-            std::vector<uint64_t> dev_grows(ndev, 0);
-            run_parallel(ndev, [&](size_t d) {
-                write_phase_host(ctx, ctx->dev[d], grid->dev[d], sh[d], t->nbrs, batch_pairs, &dev_grows[d]);
-            });
-            tr.mark("write+d2h");
-            // begin/count by original id
-            if (whole) {
+            if (device_resident) {
+                // ---- a8 into a device-resident table
                 DevCtx& dc = ctx->dev[0];
-                DeviceGuard dg(dc.device);
+                const DevGrid& g = grid->dev[0];
+                ShardState& st = sh[0];
                 cudaStream_t s = dc.main;
-                DBuf beg(8 * (n ? n : 1), s), cnt(4 * (n ? n : 1), s);
-                launch_scatter_rows(grid->dev[0].ids, sh[0].off.as<uint64_t>(), sh[0].cnt.as<uint32_t>(), 0, n, 0,
+                t->on_device = true;
+                t->device = dc.device;
+                t->dstream = s;
+                DBuf nb(4 * (P ? P : 1), s), beg(8 * (n ? n : 1), s), cnt(4 * (n ? n : 1), s);
+                if (!whole) {
+                    HDB_CUDA(cudaMemsetAsync(beg.p, 0, 8 * (n ? n : 1), s));
+                    HDB_CUDA(cudaMemsetAsync(cnt.p, 0, 4 * (n ? n : 1), s));
+                }
+                Event e0, e1;
+                HDB_CUDA(cudaEventRecord(e0.e, s));
+                launch_write(g, st.r.g0, st.r.g1, st.off.as<uint64_t>(), 0, nb.as<uint32_t>(), ctx->opts.search_kernel, 1,
+                             st.mask_base, s);
+                HDB_LAUNCH_CHECK();
+                HDB_CUDA(cudaEventRecord(e1.e, s));
+                launch_scatter_rows(g.ids, st.off.as<uint64_t>(), st.cnt.as<uint32_t>(), st.r.q0, st.r.q1, 0,
                                     beg.as<uint64_t>(), cnt.as<uint32_t>(), s);
                 HDB_LAUNCH_CHECK();
-                if (n) {
-                    HDB_CUDA(cudaMemcpyAsync(t->begin, beg.p, 8 * n, cudaMemcpyDeviceToHost, s));
-                    HDB_CUDA(cudaMemcpyAsync(t->count, cnt.p, 4 * n, cudaMemcpyDeviceToHost, s));
-                }
                 HDB_CUDA(cudaStreamSynchronize(s));
-                S.bytes_d2h += 12 * n;
+                st.ms_write = elapsed(e0, e1);
+                tr.mark("alloc+write+scatter+sync");
+                st.write_launches = 1;
+                st.n_batches = 1;
+                st.max_batch = P;
+                if (whole && n) {
+                    // production order of the rows: DBSCAN walks them in this (cell-sorted) order so
+                    // that consecutive rows share neighbours (cache locality of the union-find)
+                    DBuf rw(4 * n, s);
+                    HDB_CUDA(cudaMemcpyAsync(rw.p, g.ids, 4 * n, cudaMemcpyDeviceToDevice, s));
+                    t->rows = (uint32_t*)rw.release();
+                }
+                t->nbrs = (uint32_t*)nb.release();
+                t->begin = (uint64_t*)beg.release();
+                t->count = (uint32_t*)cnt.release();
             } else {
+                // ---- a8/a9/a10 into the host table
+                t->pool = ctx->pinned;
+                uint64_t grows0 = ctx->pinned->grows;
+                t->nbrs = pool_get<uint32_t>(t, P ? P : 1, &t->cap_nbrs);
+                t->begin = pool_get<uint64_t>(t, n ? n : 1, &t->cap_begin);
+                t->count = pool_get<uint32_t>(t, n ? n : 1, &t->cap_count);
+                if (!whole) {
+                    memset(t->begin, 0, 8 * (n ? n : 1));
+                    memset(t->count, 0, 4 * (n ? n : 1));
+                }
+                tr.mark("pinned-pool");
+                std::vector<uint64_t> dev_grows(ndev, 0);
                 run_parallel(ndev, [&](size_t d) {
-                    ShardState& st = sh[d];
-                    const uint64_t len = st.r.q1 - st.r.q0;
-                    if (!len) return;
-                    DeviceGuard dg(ctx->dev[d].device);
-                    cudaStream_t s = ctx->dev[d].main;
-                    std::vector<uint32_t> ids(len), cnt(len);
-                    std::vector<uint64_t> off(len);
-                    HDB_CUDA(cudaMemcpyAsync(ids.data(), grid->dev[d].ids + st.r.q0, 4 * len, cudaMemcpyDeviceToHost, s));
-                    HDB_CUDA(cudaMemcpyAsync(cnt.data(), st.cnt.as<uint32_t>() + st.r.q0, 4 * len,
-                                             cudaMemcpyDeviceToHost, s));
-                    HDB_CUDA(cudaMemcpyAsync(off.data(), st.off.as<uint64_t>() + st.r.q0, 8 * len,
-                                             cudaMemcpyDeviceToHost, s));
-                    HDB_CUDA(cudaStreamSynchronize(s));
-                    for (uint64_t i = 0; i < len; ++i) {
-                        t->begin[ids[i]] = off[i] + st.base;
-                        t->count[ids[i]] = cnt[i];
+                    write_phase_host(ctx, ctx->dev[d], grid->dev[d], sh[d], t->nbrs, batch_pairs, &dev_grows[d]);
+                });
+                tr.mark("write+d2h");
+                // begin/count by original id
+                if (whole) {
+                    DevCtx& dc = ctx->dev[0];
+                    DeviceGuard dg(dc.device);
+                    cudaStream_t s = dc.main;
+                    DBuf beg(8 * (n ? n : 1), s), cnt(4 * (n ? n : 1), s);
+                    launch_scatter_rows(grid->dev[0].ids, sh[0].off.as<uint64_t>(), sh[0].cnt.as<uint32_t>(), 0, n, 0,
+                                        beg.as<uint64_t>(), cnt.as<uint32_t>(), s);
+                    HDB_LAUNCH_CHECK();
+                    if (n) {
+                        HDB_CUDA(cudaMemcpyAsync(t->begin, beg.p, 8 * n, cudaMemcpyDeviceToHost, s));
+                        HDB_CUDA(cudaMemcpyAsync(t->count, cnt.p, 4 * n, cudaMemcpyDeviceToHost, s));
                     }
-                    st.d2h += 16 * len;
-                });
+                    HDB_CUDA(cudaStreamSynchronize(s));
+                    S.bytes_d2h += 12 * n;
+                } else {
+                    run_parallel(ndev, [&](size_t d) {
+                        ShardState& st = sh[d];
+                        const uint64_t len = st.r.q1 - st.r.q0;
+                        if (!len) return;
+                        DeviceGuard dg(ctx->dev[d].device);
+                        cudaStream_t s = ctx->dev[d].main;
+                        std::vector<uint32_t> ids(len), cnt(len);
+                        std::vector<uint64_t> off(len);
+                        HDB_CUDA(cudaMemcpyAsync(ids.data(), grid->dev[d].ids + st.r.q0, 4 * len, cudaMemcpyDeviceToHost, s));
+                        HDB_CUDA(cudaMemcpyAsync(cnt.data(), st.cnt.as<uint32_t>() + st.r.q0, 4 * len,
+                                                 cudaMemcpyDeviceToHost, s));
+                        HDB_CUDA(cudaMemcpyAsync(off.data(), st.off.as<uint64_t>() + st.r.q0, 8 * len,
+                                                 cudaMemcpyDeviceToHost, s));
+                        HDB_CUDA(cudaStreamSynchronize(s));
+                        for (uint64_t i = 0; i < len; ++i) {
+                            t->begin[ids[i]] = off[i] + st.base;
+                            t->count[ids[i]] = cnt[i];
+                        }
+                        st.d2h += 16 * len;
+                    });
+                }
+                for (size_t d = 0; d < ndev; ++d) S.pool_grows += dev_grows[d];
+                S.pool_grows += ctx->pinned->grows - grows0;
+                if (ctx->opts.sort_lists) {
+                    const int T = resolve_threads(ctx->opts.host_threads);
+                    run_parallel((size_t)T, [&](size_t k) {
+                        for (uint64_t p = k; p < n; p += (uint64_t)T)
+                            std::sort(t->nbrs + t->begin[p], t->nbrs + t->begin[p] + t->count[p]);
+                    });
+                }
             }
-            for (size_t d = 0; d < ndev; ++d) S.pool_grows += dev_grows[d];
-            S.pool_grows += ctx->pinned->grows - grows0;
-            if (ctx->opts.sort_lists) {
-                const int T = resolve_threads(ctx->opts.host_threads);
-                run_parallel((size_t)T, [&](size_t k) {
-                    for (uint64_t p = k; p < n; p += (uint64_t)T)
-                        std::sort(t->nbrs + t->begin[p], t->nbrs + t->begin[p] + t->count[p]);
-                });
+            S.n_batches = S.max_batch_pairs = 0;
+            S.ms_write_kernel = 0;
+            S.write_launches = 0;
+            for (auto& st : sh) {
+                S.n_batches += st.n_batches;
+                S.max_batch_pairs = std::max(S.max_batch_pairs, st.max_batch);
+                S.ms_write_kernel += st.ms_write;
+                S.write_launches += st.write_launches;
+                S.bytes_d2h += st.d2h;
             }
-        }
-        S.n_batches = S.max_batch_pairs = 0;
-        S.ms_write_kernel = 0;
-        S.write_launches = 0;
-        for (auto& st : sh) {
-            S.n_batches += st.n_batches;
-            S.max_batch_pairs = std::max(S.max_batch_pairs, st.max_batch);
-            S.ms_write_kernel += st.ms_write;
-            S.write_launches += st.write_launches;
-            S.bytes_d2h += st.d2h;
         }
     } catch (...) {
         for (auto& st : sh) {

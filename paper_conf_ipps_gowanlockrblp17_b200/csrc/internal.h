@@ -122,6 +122,12 @@ void launch_count(const DevGrid& g, uint64_t g0, uint64_t g1, uint32_t* cnt, uns
                   int variant, int slot, uint2* masks, cudaStream_t s);
 // Write (a8) over groups [g0, g1): out[off[q] - out_base + k] = k-th neighbour id of q.
 // masks != null: emit from the stored hit masks; null: recompute the tests.
+// single-pass device table (k_fused): count + reserve + emit per group; mask
+// table `masks` laid out by g.moff; rows reserved on *pair_ctr (zeroed by the
+// caller); *overflow set if a reservation passed cap
+void launch_fused(const DevGrid& g, uint32_t* cnt, unsigned long long* tests, uint2* masks,
+                  unsigned long long* pair_ctr, uint64_t cap, uint32_t* out, uint64_t* begin, uint32_t* count,
+                  unsigned int* overflow, cudaStream_t s);
 void launch_write(const DevGrid& g, uint64_t g0, uint64_t g1, const uint64_t* off, uint64_t out_base,
                   uint32_t* out, int variant, int slot, const uint2* masks, cudaStream_t s);
 // words[g] = 32-bit words of group g's hit masks for g < *ng_dev, 0 for g in [*ng_dev, n) (scan -> g.moff)
@@ -134,11 +140,12 @@ void launch_batch_cuts(const uint32_t* gstart, const uint64_t* off, uint64_t g0,
 void launch_pos_to_group(const uint32_t* gstart, uint64_t n_groups, const uint64_t* pos, uint32_t m,
                          uint64_t* grp, cudaStream_t s);
 // DBSCAN on a device-resident table (kernels_dbscan.cu); rank[n] = number of clusters
-// rows: the table's production order (begin[rows[r]] non-decreasing), or null
+// rows: the table's production order (cell-sorted queries), or null
 void launch_dbscan_device(const uint64_t* begin, const uint32_t* count, const uint32_t* nbrs, const uint32_t* rows,
                           uint64_t n, uint64_t npairs, uint32_t minpts, uint8_t* core, uint32_t* parent,
                           uint32_t* root, uint32_t* is_root, uint32_t* rank, uint32_t* giant, uint32_t* bits,
-                          uint32_t* sched /* 2 x SM count */, void* scan_temp, int32_t* labels, cudaStream_t s);
+                          uint32_t* sched /* 2 x SM count */, uint64_t* pre /* n + 1 */, void* scan_temp,
+                          int32_t* labels, cudaStream_t s);
 // T assembly by original id: begin[ids[q]] = off[q] - off[q0] + base, count[ids[q]] = cnt[q], q in [q0,q1)
 void launch_scatter_rows(const uint32_t* ids, const uint64_t* off, const uint32_t* cnt, uint64_t q0,
                          uint64_t q1, uint64_t base, uint64_t* begin, uint32_t* count, cudaStream_t s);

@@ -101,17 +101,24 @@ __device__ __forceinline__ bool reaches(const uint32_t* __restrict__ parent, uin
 constexpr uint32_t kRowsPerGrab = 4;      // consecutive (cell-sorted) rows per warp grab
 constexpr int kUnionThreads = 1024;       // one CTA per SM
 
-// first row r in [0, n) with begin[rows[r]] >= x (begin is non-decreasing
-// along the production order of a whole table)
-__device__ uint32_t row_of_pair(const uint64_t* __restrict__ begin, const uint32_t* __restrict__ rows, uint32_t n,
-                                uint64_t x) {
+// first row r in [0, n) with pre[r] >= x (pre = exclusive prefix of the list
+// lengths along the walk order)
+__device__ uint32_t row_of_pair(const uint64_t* __restrict__ pre, uint32_t n, uint64_t x) {
     uint32_t lo = 0, hi = n;
     while (lo < hi) {
         const uint32_t mid = lo + (hi - lo) / 2;
-        if (begin[rows[mid]] < x) lo = mid + 1;
+        if (pre[mid] < x) lo = mid + 1;
         else hi = mid;
     }
     return lo;
+}
+
+// list lengths along the walk order (rows[], identity if null)
+__global__ void __launch_bounds__(256) k_row_counts(const uint32_t* __restrict__ count,
+                                                    const uint32_t* __restrict__ rows, uint64_t n,
+                                                    uint32_t* __restrict__ out) {
+    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
+        out[i] = count[rows ? rows[i] : i];
 }
 
 constexpr uint32_t kSampleLinks = 2;   // edges per core linked before the full pass
@@ -223,16 +230,11 @@ __device__ __forceinline__ bool bit_of(const uint32_t* __restrict__ bits, uint32
 // Work regions of k_union: region c = rows [sched[c], sched[G + c]) of the
 // production order holding ~1/G of the pairs; sched[c] doubles as the region's
 // grab counter.
-__global__ void k_sched_init(const uint64_t* __restrict__ begin, const uint32_t* __restrict__ rows, uint32_t n,
-                             uint64_t npairs, uint32_t G, uint32_t* __restrict__ sched) {
+__global__ void k_sched_init(const uint64_t* __restrict__ pre, uint32_t n, uint64_t npairs, uint32_t G,
+                             uint32_t* __restrict__ sched) {
     for (uint32_t c = threadIdx.x; c < G; c += blockDim.x) {
-        if (rows) {
-            sched[c] = row_of_pair(begin, rows, n, npairs * c / G);
-            sched[G + c] = c + 1 == G ? n : row_of_pair(begin, rows, n, npairs * (c + 1) / G);
-        } else {
-            sched[c] = (uint32_t)((uint64_t)n * c / G);
-            sched[G + c] = (uint32_t)((uint64_t)n * (c + 1) / G);
-        }
+        sched[c] = row_of_pair(pre, n, npairs * c / G);
+        sched[G + c] = c + 1 == G ? n : row_of_pair(pre, n, npairs * (c + 1) / G);
     }
 }
 
@@ -360,7 +362,7 @@ inline unsigned blocks_for(uint64_t n, unsigned cap = 148u * 16u) {
 void launch_dbscan_device(const uint64_t* begin, const uint32_t* count, const uint32_t* nbrs, const uint32_t* rows,
                           uint64_t n, uint64_t npairs, uint32_t minpts, uint8_t* core, uint32_t* parent, uint32_t* root,
                           uint32_t* is_root, uint32_t* rank, uint32_t* giant, uint32_t* bits, uint32_t* sched,
-                          void* scan_temp, int32_t* labels, cudaStream_t s) {
+                          uint64_t* pre, void* scan_temp, int32_t* labels, cudaStream_t s) {
     if (n == 0) return;
     k_core_init<<<blocks_for(n), 256, 0, s>>>(count, n, minpts, core, parent);
     for (uint32_t k = 1; k <= kSampleLinks; ++k) {
@@ -377,12 +379,15 @@ void launch_dbscan_device(const uint64_t* begin, const uint32_t* count, const ui
         cudaFuncSetAttribute(k_union, cudaFuncAttributePreferredSharedMemoryCarveout, 0);   // all of it as L1
         if (sms <= 0) sms = 148;
     }
-    k_sched_init<<<1, 256, 0, s>>>(begin, rows, (uint32_t)n, npairs, (uint32_t)sms, sched);
+    // pair-balanced regions: prefix of the list lengths along the walk order
+    k_row_counts<<<blocks_for(n), 256, 0, s>>>(count, rows, n, (uint32_t*)root);   // root[] is free until k_flatten
+    scan_u32_to_u64((const uint32_t*)root, pre, n, scan_temp, s);
+    k_sched_init<<<1, 256, 0, s>>>(pre, (uint32_t)n, npairs, (uint32_t)sms, sched);
     k_union<<<sms, kUnionThreads, 0, s>>>(begin, count, nbrs, rows, parent, giant, bits, bits + (n + 31) / 32, sched);
     k_flatten<<<blocks_for(n), 256, 0, s>>>(core, n, parent, root, is_root);
     scan_u32_to_u32(is_root, rank, n, scan_temp, s);
     k_labels<<<blocks_for(n), 256, 0, s>>>(begin, count, nbrs, rows, core, root, rank, n, labels);
-    g_kernel_launches += 7 + 2 * kSampleLinks;
+    g_kernel_launches += 8 + 2 * kSampleLinks;
 }
 
 }  // namespace hdb

@@ -216,6 +216,125 @@ __device__ __forceinline__ uint32_t vpair(const VSpan* vs, uint32_t nspan, uint3
 constexpr float kFarF = 1e30f;
 constexpr double kFarD = 1e300;
 
+// Count one query group (queries qs .. qs+nq-1 of non-empty cell c): hit masks
+// to gmask (windowed layout; null = do not store), tests accumulated per lane;
+// returns lane i's |N_eps(query i)| (0 for lanes >= nq).  With masks, swin
+// must be all zero on entry and is left all zero (flush_window clears it).
+template <int MODE>
+__device__ __forceinline__ uint32_t count_group(const SArgs& a, uint32_t qs, uint32_t c, uint32_t nq,
+                                                uint2 (*swin)[kWinPad], VSpan* vsp, ulonglong2* sq, double2* sqd,
+                                                uint2* gmask, unsigned long long& tests, int lane) {
+    const ulonglong2* __restrict__ xp = (const ulonglong2*)a.xp;
+    const u64x NE2 = pack2(-a.e2f, -a.e2f);
+    const u64x NB2 = pack2(a.nb2_l, a.nb2_l);
+    double2 o = make_double2(0, 0);
+    if (MODE == kF64Filter) o = a.xd[qs];
+    __syncwarp();
+    if ((uint32_t)lane < nq) {
+        const uint32_t q = qs + lane;
+        if (MODE == kF32) {
+            const float2 p = a.xs[q];
+            sq[lane] = make_ulonglong2(pack2(p.x, p.x), pack2(p.y, p.y));
+        } else {
+            const double2 d = a.xd[q];
+            sqd[lane] = d;
+            if (MODE == kF64Filter) {
+                const float qx = (float)__dsub_rn(d.x, o.x), qy = (float)__dsub_rn(d.y, o.y);
+                sq[lane] = make_ulonglong2(pack2(qx, qx), pack2(qy, qy));
+            }
+        }
+    }
+    uint32_t my = 0;
+    const uint32_t npairs = load_vspans(a, c, vsp, lane);
+    const uint32_t nch = (npairs + 31) / 32;
+    uint32_t rs = 0;   // this lane's current span
+    uint32_t k = 0;
+#pragma unroll 1
+    for (; k < nch; ++k) {
+        const uint32_t kk = k % kWin;
+        bool v0, v1;
+        const uint32_t s0 = vpair(vsp, a.nspan, 32 * k + lane, rs, v0, v1), s1 = s0 + 1;
+        u64x X, Y;
+        double2 d0 = make_double2(kFarD, kFarD), d1 = make_double2(kFarD, kFarD);
+        if (MODE == kF32) {
+            ulonglong2 P = make_ulonglong2(0, 0);
+            if (v0 || v1) P = xp[s0 >> 1];
+            const float2 px = unpack2(P.x), py = unpack2(P.y);
+            X = pack2(v0 ? px.x : kFarF, v1 ? px.y : kFarF);
+            Y = pack2(v0 ? py.x : kFarF, v1 ? py.y : kFarF);
+        } else {
+            if (v0) d0 = a.xd[s0];
+            if (v1) d1 = a.xd[s1];
+            if (MODE == kF64Filter) {
+                X = pack2(v0 ? (float)__dsub_rn(d0.x, o.x) : kFarF, v1 ? (float)__dsub_rn(d1.x, o.x) : kFarF);
+                Y = pack2(v0 ? (float)__dsub_rn(d0.y, o.y) : kFarF, v1 ? (float)__dsub_rn(d1.y, o.y) : kFarF);
+            }
+        }
+        tests += (unsigned long long)nq * ((v0 ? 1u : 0u) + (v1 ? 1u : 0u));   // per lane; reduced at exit
+        uint32_t acc = 0;   // f64 filter: sign bit set <=> some |t| <= band in this lane
+#pragma unroll 4
+        for (uint32_t i = 0; i < nq; ++i) {
+            unsigned m0, m1;
+            if (MODE == kF64Exact) {
+                const double2 qd = sqd[i];
+                m0 = __ballot_sync(FULL, pred_f64(qd.x, qd.y, d0.x, d0.y, a.e2d));
+                m1 = __ballot_sync(FULL, pred_f64(qd.x, qd.y, d1.x, d1.y, a.e2d));
+            } else {
+                const ulonglong2 Q = sq[i];
+                const u64x dx = sub2(Q.x, X);
+                const u64x dy = sub2(Q.y, Y);
+                if (MODE == kF64Filter) {
+                    const u64x tt = fma2(dy, dy, fma2(dx, dx, NE2));   // (dx^2 - e2) + dy^2
+                    const float2 t = unpack2(tt);
+                    m0 = __ballot_sync(FULL, t.x < 0.f);
+                    m1 = __ballot_sync(FULL, t.y < 0.f);
+                    const float2 u = unpack2(fma2(tt, tt, NB2));         // t^2 - B^2 < 0  <=>  |t| < B
+                    acc |= __float_as_uint(u.x) | __float_as_uint(u.y);
+                } else {
+                    // exact f32: fl(fl(dx^2) + fl(dy^2)) with scalar add.rn (ptxas would fuse
+                    // mul.rn.f32x2 + add.rn.f32x2 into FFMA2 -- reading R2)
+                    const float2 px = unpack2(mul2(dx, dx));
+                    const float2 py = unpack2(mul2(dy, dy));
+                    m0 = __ballot_sync(FULL, __fadd_rn(px.x, py.x) <= a.e2f);
+                    m1 = __ballot_sync(FULL, __fadd_rn(px.y, py.y) <= a.e2f);
+                }
+            }
+            if (lane == 0) swin[i][kk] = make_uint2(m0, m1);
+        }
+        if (MODE == kF64Filter && __any_sync(FULL, (int)acc < 0)) {
+            // replay the chunk: tests in the band are decided in exact f64
+#pragma unroll 1
+            for (uint32_t i = 0; i < nq; ++i) {
+                const ulonglong2 Q = sq[i];
+                const u64x dx = sub2(Q.x, X);
+                const u64x dy = sub2(Q.y, Y);
+                const u64x tt = fma2(dy, dy, fma2(dx, dx, NE2));
+                const float2 t = unpack2(tt);
+                const float2 u = unpack2(fma2(tt, tt, NB2));
+                const bool b0 = u.x < 0.f || __float_as_uint(u.x) == 0x80000000u;
+                const bool b1 = u.y < 0.f || __float_as_uint(u.y) == 0x80000000u;
+                if (!__any_sync(FULL, b0 | b1)) continue;
+                const double2 qd = sqd[i];
+                const bool e0 = b0 && pred_f64(qd.x, qd.y, d0.x, d0.y, a.e2d);
+                const bool e1 = b1 && pred_f64(qd.x, qd.y, d1.x, d1.y, a.e2d);
+                const unsigned m0 = (__ballot_sync(FULL, t.x < 0.f) & ~__ballot_sync(FULL, b0)) |
+                                    __ballot_sync(FULL, e0);
+                const unsigned m1 = (__ballot_sync(FULL, t.y < 0.f) & ~__ballot_sync(FULL, b1)) |
+                                    __ballot_sync(FULL, e1);
+                if (lane == 0) swin[i][kk] = make_uint2(m0, m1);
+            }
+        }
+        __syncwarp();
+        if ((uint32_t)lane < nq) {
+            const uint2 mk = swin[lane][kk];
+            my += __popc(mk.x) + __popc(mk.y);
+        }
+        if (gmask && kk == kWin - 1) flush_window(swin, gmask, k / kWin, nq, lane);
+    }
+    if (gmask && (k % kWin) != 0) flush_window(swin, gmask, k / kWin, nq, lane);
+    return my;
+}
+
 template <int MODE>
 __global__ void __launch_bounds__(kSearchThreads) k_count(SArgs a, uint32_t g0, uint32_t g1, uint32_t chunk,
                                                           unsigned int* __restrict__ ctr, uint32_t* __restrict__ cnt,
@@ -228,125 +347,17 @@ __global__ void __launch_bounds__(kSearchThreads) k_count(SArgs a, uint32_t g0, 
     __shared__ double2 sqd[F64 ? kWarps : 1][32];   // exact query coordinates (f64 modes)
     const int lane = threadIdx.x & 31;
     const int w = threadIdx.x >> 5;
-    const ulonglong2* __restrict__ xp = (const ulonglong2*)a.xp;
 #pragma unroll
     for (int kk = 0; kk < kWin; ++kk) swin[w][lane][kk] = make_uint2(0, 0);
-    const u64x NE2 = pack2(-a.e2f, -a.e2f);
-    const u64x NB2 = pack2(a.nb2_l, a.nb2_l);
     unsigned long long tests = 0;
     uint32_t gi = g0 + grab(ctr, chunk, lane), gend = min(gi + chunk, g1);
     while (gi < g1) {
         const uint32_t qs = __ldg(&a.gstart[gi]);
         const uint32_t c = __ldg(&a.gcell[gi]);
         const uint32_t nq = min((uint32_t)kGroup, __ldg(&a.cstart[c + 1]) - qs);
-        double2 o = make_double2(0, 0);
-        if (MODE == kF64Filter) o = a.xd[qs];
-        __syncwarp();
-        if ((uint32_t)lane < nq) {
-            const uint32_t q = qs + lane;
-            if (MODE == kF32) {
-                const float2 p = a.xs[q];
-                sq[w][lane] = make_ulonglong2(pack2(p.x, p.x), pack2(p.y, p.y));
-            } else {
-                const double2 d = a.xd[q];
-                sqd[F64 ? w : 0][lane] = d;
-                if (MODE == kF64Filter) {
-                    const float qx = (float)__dsub_rn(d.x, o.x), qy = (float)__dsub_rn(d.y, o.y);
-                    sq[w][lane] = make_ulonglong2(pack2(qx, qx), pack2(qy, qy));
-                }
-            }
-        }
-        uint32_t my = 0;
         uint2* gmask = masks ? masks + (__ldg(&moff[gi]) >> 1) : nullptr;
-        const uint32_t npairs = load_vspans(a, c, vsp[w], lane);
-        const uint32_t nch = (npairs + 31) / 32;
-        uint32_t rs = 0;   // this lane's current span
-        uint32_t k = 0;
-#pragma unroll 1
-        for (; k < nch; ++k) {
-            {
-                const uint32_t kk = k % kWin;
-                bool v0, v1;
-                const uint32_t s0 = vpair(vsp[w], a.nspan, 32 * k + lane, rs, v0, v1), s1 = s0 + 1;
-                u64x X, Y;
-                double2 d0 = make_double2(kFarD, kFarD), d1 = make_double2(kFarD, kFarD);
-                if (MODE == kF32) {
-                    ulonglong2 P = make_ulonglong2(0, 0);
-                    if (v0 || v1) P = xp[s0 >> 1];
-                    const float2 px = unpack2(P.x), py = unpack2(P.y);
-                    X = pack2(v0 ? px.x : kFarF, v1 ? px.y : kFarF);
-                    Y = pack2(v0 ? py.x : kFarF, v1 ? py.y : kFarF);
-                } else {
-                    if (v0) d0 = a.xd[s0];
-                    if (v1) d1 = a.xd[s1];
-                    if (MODE == kF64Filter) {
-                        X = pack2(v0 ? (float)__dsub_rn(d0.x, o.x) : kFarF, v1 ? (float)__dsub_rn(d1.x, o.x) : kFarF);
-                        Y = pack2(v0 ? (float)__dsub_rn(d0.y, o.y) : kFarF, v1 ? (float)__dsub_rn(d1.y, o.y) : kFarF);
-                    }
-                }
-                tests += (unsigned long long)nq * ((v0 ? 1u : 0u) + (v1 ? 1u : 0u));   // per lane; reduced at exit
-                uint32_t acc = 0;   // f64 filter: sign bit set <=> some |t| <= band in this lane
-#pragma unroll 4
-                for (uint32_t i = 0; i < nq; ++i) {
-                    unsigned m0, m1;
-                    if (MODE == kF64Exact) {
-                        const double2 qd = sqd[F64 ? w : 0][i];
-                        m0 = __ballot_sync(FULL, pred_f64(qd.x, qd.y, d0.x, d0.y, a.e2d));
-                        m1 = __ballot_sync(FULL, pred_f64(qd.x, qd.y, d1.x, d1.y, a.e2d));
-                    } else {
-                        const ulonglong2 Q = sq[w][i];
-                        const u64x dx = sub2(Q.x, X);
-                        const u64x dy = sub2(Q.y, Y);
-                        if (MODE == kF64Filter) {
-                            const u64x tt = fma2(dy, dy, fma2(dx, dx, NE2));   // (dx^2 - e2) + dy^2
-                            const float2 t = unpack2(tt);
-                            m0 = __ballot_sync(FULL, t.x < 0.f);
-                            m1 = __ballot_sync(FULL, t.y < 0.f);
-                            const float2 u = unpack2(fma2(tt, tt, NB2));         // t^2 - B^2 < 0  <=>  |t| < B
-                            acc |= __float_as_uint(u.x) | __float_as_uint(u.y);
-                        } else {
-                            // exact f32: fl(fl(dx^2) + fl(dy^2)) with scalar add.rn (ptxas would fuse
-                            // mul.rn.f32x2 + add.rn.f32x2 into FFMA2 -- reading R2)
-                            const float2 px = unpack2(mul2(dx, dx));
-                            const float2 py = unpack2(mul2(dy, dy));
-                            m0 = __ballot_sync(FULL, __fadd_rn(px.x, py.x) <= a.e2f);
-                            m1 = __ballot_sync(FULL, __fadd_rn(px.y, py.y) <= a.e2f);
-                        }
-                    }
-                    if (lane == 0) swin[w][i][kk] = make_uint2(m0, m1);
-                }
-                if (MODE == kF64Filter && __any_sync(FULL, (int)acc < 0)) {
-                    // replay the chunk: tests in the band are decided in exact f64
-#pragma unroll 1
-                    for (uint32_t i = 0; i < nq; ++i) {
-                        const ulonglong2 Q = sq[w][i];
-                        const u64x dx = sub2(Q.x, X);
-                        const u64x dy = sub2(Q.y, Y);
-                        const u64x tt = fma2(dy, dy, fma2(dx, dx, NE2));
-                        const float2 t = unpack2(tt);
-                        const float2 u = unpack2(fma2(tt, tt, NB2));
-                        const bool b0 = u.x < 0.f || __float_as_uint(u.x) == 0x80000000u;
-                        const bool b1 = u.y < 0.f || __float_as_uint(u.y) == 0x80000000u;
-                        if (!__any_sync(FULL, b0 | b1)) continue;
-                        const double2 qd = sqd[F64 ? w : 0][i];
-                        const bool e0 = b0 && pred_f64(qd.x, qd.y, d0.x, d0.y, a.e2d);
-                        const bool e1 = b1 && pred_f64(qd.x, qd.y, d1.x, d1.y, a.e2d);
-                        const unsigned m0 = (__ballot_sync(FULL, t.x < 0.f) & ~__ballot_sync(FULL, b0)) |
-                                            __ballot_sync(FULL, e0);
-                        const unsigned m1 = (__ballot_sync(FULL, t.y < 0.f) & ~__ballot_sync(FULL, b1)) |
-                                            __ballot_sync(FULL, e1);
-                        if (lane == 0) swin[w][i][kk] = make_uint2(m0, m1);
-                    }
-                }
-                __syncwarp();
-                if ((uint32_t)lane < nq) {
-                    const uint2 mk = swin[w][lane][kk];
-                    my += __popc(mk.x) + __popc(mk.y);
-                }
-                if (gmask && kk == kWin - 1) flush_window(swin[w], gmask, k / kWin, nq, lane);
-            }
-        }
-        if (gmask && (k % kWin) != 0) flush_window(swin[w], gmask, k / kWin, nq, lane);
+        const uint32_t my =
+            count_group<MODE>(a, qs, c, nq, swin[w], vsp[w], sq[w], sqd[F64 ? w : 0], gmask, tests, lane);
         if ((uint32_t)lane < nq) cnt[qs + lane] = my;
         if (++gi >= gend) {
             gi = g0 + grab(ctr, chunk, lane);
@@ -533,6 +544,68 @@ __device__ __forceinline__ void cp_async_wait() {
     asm volatile("cp.async.wait_group %0;" ::"n"(N));
 }
 
+// Emit one query group from its hit masks: lane i starts query i's list at
+// gout + my; raw / wq / vsp are the warp's buffers (see k_emit).
+__device__ __forceinline__ void emit_group(const SArgs& a, uint32_t c, uint32_t nq, uint32_t nwin,
+                                           const uint2* gmask, uint32_t* gout, uint32_t my,
+                                           uint2 (*raw)[kWin + 2], uint4 (*wq)[kWin + 1], VSpan* vsp, int lane) {
+    const unsigned lt = (1u << lane) - 1u, lbit = 1u << lane;
+    // the group's spans as one sequence of candidate pairs (same chunks as the count pass)
+    load_vspans(a, c, vsp, lane);
+    uint32_t rs = 0;   // this lane's current span
+    __syncwarp();   // the previous group's buffers are no longer read
+    if ((uint32_t)lane < nq) {   // prefetch window 0: lane i copies its 64-B mask row
+        const uint4* src = (const uint4*)(gmask + (size_t)lane * kWin);
+#pragma unroll
+        for (int u = 0; u < kWin / 2; ++u) cp_async16(&raw[lane][2 * u], src + u);
+    }
+    cp_async_commit();
+#pragma unroll 1
+    for (uint32_t v = 0; v < nwin; ++v) {
+        // this window's candidate ids: lane j holds pair (2j, 2j+1) of each chunk
+        uint2 ids[kWin];
+#pragma unroll
+        for (int kk = 0; kk < kWin; ++kk) {
+            bool v0, v1;
+            const uint32_t s0 = vpair(vsp, a.nspan, 32 * (v * kWin + kk) + lane, rs, v0, v1);
+            ids[kk] = make_uint2(0, 0);
+            if (v0 | v1) ids[kk] = __ldg((const uint2*)(a.ids + s0));
+        }
+        cp_async_wait<0>();
+        __syncwarp();
+        // lane i turns its row of masks into output positions (all queries in parallel)
+        if ((uint32_t)lane < nq) {
+#pragma unroll
+            for (int kk = 0; kk < kWin; ++kk) {
+                const uint2 m = raw[lane][kk];
+                const uint32_t p0 = my;
+                my += __popc(m.x);
+                wq[lane][kk] = make_uint4(m.x, m.y, p0, my);
+                my += __popc(m.y);
+            }
+        }
+        __syncwarp();
+        // prefetch the next window's masks into the landing buffer (overlaps the stores)
+        if (v + 1 < nwin && (uint32_t)lane < nq) {
+            const uint4* src = (const uint4*)(gmask + ((size_t)(v + 1) * nq + lane) * kWin);
+#pragma unroll
+            for (int u = 0; u < kWin / 2; ++u) cp_async16(&raw[lane][2 * u], src + u);
+        }
+        cp_async_commit();
+#pragma unroll 1
+        for (uint32_t i = 0; i < nq; ++i) {
+#pragma unroll
+            for (int kk = 0; kk < kWin; ++kk) {
+                const uint4 e = wq[i][kk];   // broadcast
+                stg_if_bit(gout + (e.z + __popc(e.x & lt)), ids[kk].x, e.x, lbit);
+                stg_if_bit(gout + (e.w + __popc(e.y & lt)), ids[kk].y, e.y, lbit);
+            }
+        }
+        __syncwarp();   // wq is rewritten for the next window
+    }
+    cp_async_wait<0>();
+}
+
 __global__ void __launch_bounds__(kEmitThreads) k_emit(SArgs a, uint32_t g0, uint32_t g1, uint32_t chunk,
                                                          unsigned int* __restrict__ ctr,
                                                          const uint64_t* __restrict__ off, uint64_t out_base,
@@ -544,7 +617,6 @@ __global__ void __launch_bounds__(kEmitThreads) k_emit(SArgs a, uint32_t g0, uin
     __shared__ VSpan vsp[kEmitWarps][kMaxSpans + 1];  // the group's spans as one pair sequence
     const int lane = threadIdx.x & 31;
     const int w = threadIdx.x >> 5;
-    const unsigned lt = (1u << lane) - 1u, lbit = 1u << lane;
     uint32_t gi = g0 + grab(ctr, chunk, lane), gend = min(gi + chunk, g1);
     while (gi < g1) {
         const uint32_t qs = __ldg(&a.gstart[gi]);
@@ -552,71 +624,96 @@ __global__ void __launch_bounds__(kEmitThreads) k_emit(SArgs a, uint32_t g0, uin
         const uint32_t nq = min((uint32_t)kGroup, __ldg(&a.cstart[c + 1]) - qs);
         const uint64_t m_a = __ldg(&moff[gi]), m_b = __ldg(&moff[gi + 1]);
         const uint32_t nwin = (uint32_t)((m_b - m_a) / (2ull * nq * kWin));
-        const uint2* gmask = masks + (m_a >> 1);
         const uint64_t gb = off[qs];
         uint32_t* gout = out + (gb - out_base);
         asm volatile("mov.b64 %0, %0;" : "+l"(gout));
         uint32_t my = 0;   // lane i: output cursor of query i within the group
         if ((uint32_t)lane < nq) my = (uint32_t)(off[qs + lane] - gb);
-        // the group's spans as one sequence of candidate pairs (same chunks as the count pass)
-        load_vspans(a, c, vsp[w], lane);
-        uint32_t rs = 0;   // this lane's current span
-        __syncwarp();   // the previous group's buffers are no longer read
-        if ((uint32_t)lane < nq) {   // prefetch window 0: lane i copies its 64-B mask row
-            const uint4* src = (const uint4*)(gmask + (size_t)lane * kWin);
-#pragma unroll
-            for (int u = 0; u < kWin / 2; ++u) cp_async16(&raw[w][lane][2 * u], src + u);
-        }
-        cp_async_commit();
-#pragma unroll 1
-        for (uint32_t v = 0; v < nwin; ++v) {
-            // this window's candidate ids: lane j holds pair (2j, 2j+1) of each chunk
-            uint2 ids[kWin];   // lane j: ids of candidate pair (2j, 2j+1) of each chunk of the window
-#pragma unroll
-            for (int kk = 0; kk < kWin; ++kk) {
-                bool v0, v1;
-                const uint32_t s0 = vpair(vsp[w], a.nspan, 32 * (v * kWin + kk) + lane, rs, v0, v1);
-                ids[kk] = make_uint2(0, 0);
-                if (v0 | v1) ids[kk] = __ldg((const uint2*)(a.ids + s0));
-            }
-            cp_async_wait<0>();
-            __syncwarp();
-            // lane i turns its row of masks into output positions (all queries in parallel)
-            if ((uint32_t)lane < nq) {
-#pragma unroll
-                for (int kk = 0; kk < kWin; ++kk) {
-                    const uint2 m = raw[w][lane][kk];
-                    const uint32_t p0 = my;
-                    my += __popc(m.x);
-                    wq[w][lane][kk] = make_uint4(m.x, m.y, p0, my);
-                    my += __popc(m.y);
-                }
-            }
-            __syncwarp();
-            // prefetch the next window's masks into the landing buffer (overlaps the stores)
-            if (v + 1 < nwin && (uint32_t)lane < nq) {
-                const uint4* src = (const uint4*)(gmask + ((size_t)(v + 1) * nq + lane) * kWin);
-#pragma unroll
-                for (int u = 0; u < kWin / 2; ++u) cp_async16(&raw[w][lane][2 * u], src + u);
-            }
-            cp_async_commit();
-#pragma unroll 1
-            for (uint32_t i = 0; i < nq; ++i) {
-#pragma unroll
-                for (int kk = 0; kk < kWin; ++kk) {
-                    const uint4 e = wq[w][i][kk];   // broadcast
-                    stg_if_bit(gout + (e.z + __popc(e.x & lt)), ids[kk].x, e.x, lbit);
-                    stg_if_bit(gout + (e.w + __popc(e.y & lt)), ids[kk].y, e.y, lbit);
-                }
-            }
-            __syncwarp();   // wq is rewritten for the next window
-        }
-        cp_async_wait<0>();
+        emit_group(a, c, nq, nwin, masks + (m_a >> 1), gout, my, raw[w], wq[w], vsp[w], lane);
         if (++gi >= gend) {
             gi = g0 + grab(ctr, chunk, lane);
             gend = min(gi + chunk, g1);
         }
     }
+}
+
+// Single pass for a device-resident table (search_kernel 4, whole table):
+// per group, count (hit masks to the group's slot of the mask table, which the
+// same warp reads back right away -- it is still in L2), reserve the group's
+// output with one atomicAdd on the pair counter, write begin/count by original
+// id, then emit.  Rows land in reservation order (each list is still in
+// candidate order).  If the reservation passes `cap` (the table was sized from
+// the sampled estimate) the group is not emitted and *overflow is set; the
+// host then rebuilds the table with the exact two-pass path.  Count work (FP32/
+// ALU) of some warps overlaps the store streams of others.
+constexpr int kFusedThreads = 128;
+constexpr int kFusedWarps = kFusedThreads / 32;
+template <int MODE>
+__global__ void __launch_bounds__(kFusedThreads) k_fused(SArgs a, uint32_t g0, uint32_t g1, uint32_t chunk,
+                                                          unsigned int* __restrict__ ctr, uint32_t* __restrict__ cnt,
+                                                          unsigned long long* __restrict__ tests_out,
+                                                          uint2* __restrict__ masks, const uint64_t* __restrict__ moff,
+                                                          unsigned long long* __restrict__ pair_ctr, uint64_t cap,
+                                                          uint32_t* __restrict__ out, uint64_t* __restrict__ begin,
+                                                          uint32_t* __restrict__ count,
+                                                          unsigned int* __restrict__ overflow) {
+    constexpr bool F64 = MODE != kF32;
+    __shared__ uint2 swin[kFusedWarps][32][kWinPad];
+    __shared__ VSpan vsp[kFusedWarps][kMaxSpans + 1];
+    __shared__ ulonglong2 sq[kFusedWarps][32];
+    __shared__ double2 sqd[F64 ? kFusedWarps : 1][32];
+    __shared__ __align__(16) uint2 raw[kFusedWarps][32][kWin + 2];
+    __shared__ uint4 wq[kFusedWarps][32][kWin + 1];
+    const int lane = threadIdx.x & 31;
+    const int w = threadIdx.x >> 5;
+#pragma unroll
+    for (int kk = 0; kk < kWin; ++kk) swin[w][lane][kk] = make_uint2(0, 0);
+    unsigned long long tests = 0;
+    uint32_t gi = g0 + grab(ctr, chunk, lane), gend = min(gi + chunk, g1);
+    while (gi < g1) {
+        const uint32_t qs = __ldg(&a.gstart[gi]);
+        const uint32_t c = __ldg(&a.gcell[gi]);
+        const uint32_t nq = min((uint32_t)kGroup, __ldg(&a.cstart[c + 1]) - qs);
+        const uint64_t m_a = __ldg(&moff[gi]), m_b = __ldg(&moff[gi + 1]);
+        uint2* gmask = masks + (m_a >> 1);
+        const uint32_t my =
+            count_group<MODE>(a, qs, c, nq, swin[w], vsp[w], sq[w], sqd[F64 ? w : 0], gmask, tests, lane);
+        // reserve the group's output
+        uint32_t incl = my;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t y = __shfl_up_sync(FULL, incl, o);
+            if (lane >= o) incl += y;
+        }
+        const uint32_t total = __shfl_sync(FULL, incl, 31);
+        unsigned long long base = 0;
+        if (lane == 0) base = atomicAdd(pair_ctr, (unsigned long long)total);
+        base = __shfl_sync(FULL, base, 0);
+        const uint32_t excl = incl - my;
+        if ((uint32_t)lane < nq) {
+            const uint32_t id = __ldg(&a.ids[qs + lane]);
+            cnt[qs + lane] = my;
+            begin[id] = base + excl;
+            count[id] = my;
+        }
+        if (base + total <= cap) {
+            __threadfence_block();   // the masks this warp just stored are read back by cp.async
+            __syncwarp();
+            uint32_t* gout = out + base;
+            asm volatile("mov.b64 %0, %0;" : "+l"(gout));
+            const uint32_t nwin = (uint32_t)((m_b - m_a) / (2ull * nq * kWin));
+            emit_group(a, c, nq, nwin, gmask, gout, excl, raw[w], wq[w], vsp[w], lane);
+        } else if (lane == 0) {
+            atomicOr(overflow, 1u);
+        }
+        if (++gi >= gend) {
+            gi = g0 + grab(ctr, chunk, lane);
+            gend = min(gi + chunk, g1);
+        }
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) tests += __shfl_xor_sync(FULL, tests, o);
+    if (tests_out && lane == 0 && tests) atomicAdd(tests_out, tests);
 }
 
 // Mask-table layout: words of group g = 2 * nq * kWin * (windows of kWin chunks of 32 virtual pairs)
@@ -879,6 +976,39 @@ void launch_write(const DevGrid& g, uint64_t g0, uint64_t g1, const uint64_t* of
     launch_groups(k_emit, bps, g1 - g0, chunk, ctas, kEmitThreads);
     k_emit<<<ctas, kEmitThreads, 0, s>>>(args_of(g), (uint32_t)g0, (uint32_t)g1, chunk, ctr, off, out_base, out,
                                            masks, g.moff);
+    ++g_kernel_launches;
+}
+
+template <int MODE>
+void launch_fused_mode(const SArgs& a, uint64_t g0, uint64_t g1, unsigned int* ctr, uint32_t* cnt,
+                       unsigned long long* tests, uint2* masks, const uint64_t* moff, unsigned long long* pair_ctr,
+                       uint64_t cap, uint32_t* out, uint64_t* begin, uint32_t* count, unsigned int* overflow,
+                       cudaStream_t s) {
+    static int bps = 0;
+    uint32_t chunk;
+    unsigned ctas;
+    launch_groups(k_fused<MODE>, bps, g1 - g0, chunk, ctas, kFusedThreads);
+    k_fused<MODE><<<ctas, kFusedThreads, 0, s>>>(a, (uint32_t)g0, (uint32_t)g1, chunk, ctr, cnt, tests, masks, moff,
+                                                 pair_ctr, cap, out, begin, count, overflow);
+}
+
+void launch_fused(const DevGrid& g, uint32_t* cnt, unsigned long long* tests, uint2* masks,
+                  unsigned long long* pair_ctr, uint64_t cap, uint32_t* out, uint64_t* begin, uint32_t* count,
+                  unsigned int* overflow, cudaStream_t s) {
+    if (g.n_groups == 0) return;
+    const SArgs a = args_of(g);
+    unsigned int* ctr = g.counters;
+    cudaMemsetAsync(ctr, 0, sizeof(unsigned int), s);
+    const int mode = g.dtype == HDB_F32 ? kF32 : (g.filter_l ? kF64Filter : kF64Exact);
+    if (mode == kF64Filter)
+        launch_fused_mode<kF64Filter>(a, 0, g.n_groups, ctr, cnt, tests, masks, g.moff, pair_ctr, cap, out, begin,
+                                      count, overflow, s);
+    else if (mode == kF64Exact)
+        launch_fused_mode<kF64Exact>(a, 0, g.n_groups, ctr, cnt, tests, masks, g.moff, pair_ctr, cap, out, begin,
+                                     count, overflow, s);
+    else
+        launch_fused_mode<kF32>(a, 0, g.n_groups, ctr, cnt, tests, masks, g.moff, pair_ctr, cap, out, begin, count,
+                                overflow, s);
     ++g_kernel_launches;
 }
 

@@ -321,6 +321,28 @@ def test_process_shards_partition_the_table(torch_cuda, R):
     assert np.array_equal(count, full[1].astype(np.int64))
 
 
+def test_single_pass_device_table_and_fallback(torch_cuda):
+    """search_kernel=4 builds device-resident tables in one pass (count + reserve
+    + emit per group) into a table sized from the sampled estimate; an estimate
+    that is far too low must fall back to the exact two-pass path, with the
+    same table."""
+    xy = datagen.subsample(datagen.tec_like(), 30_000, seed=4)
+    for eps in (0.15, 0.45, 1.0):
+        b, c, v, view, st = lib_table(xy, eps, device=True, search_kernel=4)
+        assert st["single_pass"] == 1
+        assert view.npairs == int(c.astype(np.int64).sum())
+        assert_table_equal(xy, eps, b, c, v)
+    # one sample (stride > n) on a sparse point: a_b ~ 1e6 << P ~ 9e6
+    rng = np.random.default_rng(3)
+    sparse = rng.uniform(0, 100, size=(17_000, 2))
+    sparse[0] = (-50.0, -50.0)           # sorted position 0: an isolated point
+    xy2 = np.concatenate([sparse, np.full((3_000, 2), 50.0)])
+    b, c, v, view, st = lib_table(xy2, 0.5, device=True, sample_fraction=1e-6, search_kernel=4)
+    assert st["single_pass"] == 0
+    assert st["est_pairs"] < view.npairs
+    assert_table_equal(xy2, 0.5, b, c, v)
+
+
 def test_deterministic(torch_cuda):
     xy = datagen.subsample(datagen.tec_like(), 30_000, seed=9)
     a = lib_table(xy, 0.45)
