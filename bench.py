@@ -423,8 +423,11 @@ def main():
     hbm, peak_kind = load_peaks()
     n_shard = (v.end_query - v.first_query) if ws > 1 else n
     single = bool(st.get("single_pass", 0))
+    paper = args.kernel in (7, 8)   # the paper's GPUCalcGlobal / GPUCalcShared (Table II baseline)
     esz = 16 if args.dtype == "f64" else 8
-    alg_bytes = 4 * v.npairs + ((esz + 20) * n_shard if single else 12 * n_shard)
+    #  * paper kernels: the key/value result set R, 8 B per pair, + the query's coordinates and id
+    alg_bytes = (8 * v.npairs + (esz + 4) * n_shard if paper else
+                 4 * v.npairs + ((esz + 20) * n_shard if single else 12 * n_shard))
     wms = float(np.mean(write_ms))
     achieved = alg_bytes / (wms / 1000.0) / 1e9
     traffic = None
@@ -447,7 +450,9 @@ def main():
             "gpu_launches": launches,
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
                          "frac": achieved / hbm, "traffic": traffic, "peak_kind": peak_kind,
-                         "kernel": ("k_fused (single pass: count + reserve + emit, a6-a8)" if single
+                         "kernel": ({7: "k_paper_global (GPUCalcGlobal, Alg. 2)",
+                                     8: "k_paper_shared (GPUCalcShared, Alg. 3)"}[args.kernel] if paper else
+                                    "k_fused (single pass: count + reserve + emit, a6-a8)" if single
                                     else "k_emit (neighbour write, a8)"),
                          "kernel_ms": wms, "alg_bytes": alg_bytes},
             "count_kernel": ({"bound": "alu", "kernel": "k_fused (count part, a6)", "ms": wms,
@@ -462,13 +467,13 @@ def main():
             "clocks": clk.summary(),
             "stats": {k: st[k] for k in ("n_nonempty", "n_groups", "candidate_tests", "ms_grid", "ms_sample",
                                          "ms_count", "ms_scan", "ms_write_kernel", "kernel_launches",
-                                         "single_pass", "est_pairs")}}
+                                         "single_pass", "est_pairs", "ms_sort")}}
 
     # ---- e2e through the C-ABI from pinned HOST points (H2D inside the timed region):
     #   value: the same metric (pairs/s) with the table delivered to a HOST table (D2H inside);
     #   plus points clustered/s for the paper's hybrid (host table + host DBSCAN) and for the
     #   device path (device table + GPU DBSCAN, labels D2H).
-    if rank == 0 and ws == 1 and args.e2e_steps > 0:
+    if rank == 0 and ws == 1 and args.e2e_steps > 0 and not paper:
         hdb.hdb_ctx_set_stream(ctx, None)
         xy_pin = torch.from_numpy(xy_np).pin_memory()
         labels = np.empty(n, np.int32)

@@ -81,7 +81,12 @@ typedef struct {
     uint64_t host_budget_bytes; /* 0 = unlimited; else HDB_ENOMEM when 4*P exceeds it                  */
     int shard_rank;             /* process-level query sharding (torchrun mode): this process          */
     int shard_count;            /*   computes shard shard_rank of shard_count; 0 => unsharded          */
-    int search_kernel;          /* 0 = default; other values select kernel variants        */
+    int search_kernel;          /* 0 = default; other values select kernel variants:
+                                   1 = exact-f64-only tests, 2 = write pass recomputes the tests,
+                                   4 = single-pass device table, 7 / 8 = the paper's GPUCalcGlobal
+                                   (Alg. 2) / GPUCalcShared (Alg. 3) with an atomic key/value result
+                                   set sorted by key (device-resident whole tables; the Table II
+                                   baseline)                                               */
     int host_threads;           /* threads for host-side work (T assembly, DBSCAN); 0 = all cores      */
     int cell_split;             /* k >= 1: grid cells of width eps/k, (2k+1)^2-cell stencil (fewer
                                    candidate tests on dense data); 0 = auto (k from a sampled cell
@@ -155,6 +160,9 @@ typedef struct {
     int single_pass;             /* 1: the last device-resident table was built in one pass (count +
                                     reserve + emit per query group, rows in reservation order);
                                     ms_write_kernel is that kernel's time, ms_count = ms_scan = 0    */
+    double ms_sort;              /* search_kernel 7 / 8 (the paper's kernels): device time of the sort
+                                    of the key/value result set by key + the T ranges (Alg. 4 line 7-8);
+                                    ms_write_kernel is then the search kernel's time                   */
 } hdb_stats;
 
 /* ---- context ------------------------------------------------------------- */

@@ -705,6 +705,76 @@ bool single_pass_table(hdb_ctx* ctx, const DevGrid& g, hdb_table* t, hdb_stats& 
     return true;
 }
 
+// The paper's kernels (search_kernel 7 / 8; NEXT-3): GPUCalcGlobal (Alg. 2) or
+// GPUCalcShared (Alg. 3) append the key/value result set R with atomics into a
+// buffer sized from the sampled estimate ((1 + 2 alpha) a_b + n, P:736-741,
+// P:812-823); the append counter keeps counting past the capacity, so an
+// overflow reruns the kernel once at the exact |R| (reading R14).  R is then
+// sorted by key (Alg. 4 line 7, the paper's sort_by_key; here the library's
+// LSD radix sort) and T's ranges are read off the sorted keys
+// (ConstructNeighborTable).  Device-resident whole tables only.
+void paper_table(hdb_ctx* ctx, const DevGrid& g, hdb_table* t, hdb_stats& S, uint64_t est, int which) {
+    DevCtx& dc = ctx->dev[0];
+    cudaStream_t s = dc.main;
+    const uint64_t n = g.n;
+    uint64_t cap = (uint64_t)((1.0 + 2.0 * ctx->opts.alpha) * (double)est) + n + 1024;
+    DBuf ctr(8, s);
+    float ms_search = 0;
+    uint64_t P = 0;
+    DBuf rkey, rval;
+    for (int attempt = 0; attempt < 2; ++attempt) {
+        if (cap >= (1ull << 32)) cap = (1ull << 32) - 1;
+        rkey = DBuf(4 * cap, s);
+        rval = DBuf(4 * cap, s);
+        HDB_CUDA(cudaMemsetAsync(ctr.p, 0, 8, s));
+        Event e0, e1;
+        HDB_CUDA(cudaEventRecord(e0.e, s));
+        launch_paper_search(g, which, ctr.as<unsigned long long>(), cap, rkey.as<uint32_t>(), rval.as<uint32_t>(), s);
+        HDB_LAUNCH_CHECK();
+        HDB_CUDA(cudaEventRecord(e1.e, s));
+        HDB_CUDA(cudaMemcpyAsync(dc.pin + 4, ctr.p, 8, cudaMemcpyDeviceToHost, s));
+        HDB_CUDA(cudaStreamSynchronize(s));
+        ms_search += elapsed(e0, e1);
+        P = dc.pin[4];
+        if (P <= cap) break;
+        ++S.pool_grows;
+        cap = P;   // exact |R| now known
+        if (P >= (1ull << 32) - 1)
+            fail(HDB_ERANGE, "the paper kernels' result set (%llu pairs) needs 32-bit positions",
+                 (unsigned long long)P);
+    }
+    // Alg. 4 line 7: sort R by key (stable LSD radix sort on the key's bits)
+    int bits = 1;
+    while (bits < 32 && (1ull << bits) < n) ++bits;
+    DBuf k1(4 * (P ? P : 1), s), v1(4 * (P ? P : 1), s), tmp(radix_sort_temp_bytes(P ? P : 1), s);
+    DBuf beg(8 * (n ? n : 1), s), cnt(4 * (n ? n : 1), s);
+    Event e2, e3;
+    HDB_CUDA(cudaEventRecord(e2.e, s));
+    const int where = radix_sort_pairs(rkey.p, rval.as<uint32_t>(), k1.p, v1.as<uint32_t>(), 4, P, bits, tmp.p, s);
+    const uint32_t* ks = where ? k1.as<uint32_t>() : rkey.as<uint32_t>();
+    launch_rows_from_keys(ks, P, n, beg.as<uint64_t>(), cnt.as<uint32_t>(), s);
+    HDB_LAUNCH_CHECK();
+    HDB_CUDA(cudaEventRecord(e3.e, s));
+    HDB_CUDA(cudaStreamSynchronize(s));
+    t->on_device = true;
+    t->device = dc.device;
+    t->dstream = s;
+    t->npairs = P;
+    t->first_query = 0;
+    t->end_query = n;
+    t->nbrs = (uint32_t*)(where ? v1.release() : rval.release());
+    t->begin = (uint64_t*)beg.release();
+    t->count = (uint32_t*)cnt.release();
+    S.npairs = P;
+    S.candidate_tests = 0;
+    S.ms_count = S.ms_scan = 0;
+    S.ms_write_kernel = ms_search;
+    S.ms_sort = elapsed(e2, e3);
+    S.write_launches = 1;
+    S.n_batches = 1;
+    S.max_batch_pairs = P;
+}
+
 void ensure_batch_buf(DevCtx& dc, size_t si, size_t pairs, uint64_t* grows) {
     if (dc.batch_buf.size() <= si) {
         dc.batch_buf.resize(si + 1, nullptr);
@@ -921,8 +991,23 @@ void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hd
         }
         tr.mark("sample+cuts");
         S.single_pass = 0;
+        S.ms_sort = 0;
         bool single = false;
-        if (device_resident && parts == 1 && ctx->opts.search_kernel == 4 && n > 0) {
+        const int sk = ctx->opts.search_kernel;
+        if ((sk == kPaperGlobal || sk == kPaperShared) && !(device_resident && parts == 1))
+            fail(HDB_EINVAL, "search_kernel %d (the paper's kernels) builds device-resident, unsharded tables only", sk);
+        if ((sk == kPaperGlobal || sk == kPaperShared) && n > 0) {
+            HDB_CUDA(cudaStreamSynchronize(s0));   // e_b is in dc0.pin[0]
+            const uint64_t eb = dc0.pin[0];
+            S.sample_size = ns;
+            S.sample_pairs = eb;
+            S.est_pairs = eb * stride;
+            S.ms_sample = elapsed(es0, es1);
+            paper_table(ctx, G0, t, S, eb * stride, sk);
+            single = true;
+            tr.mark("paper-kernel");
+        }
+        if (!single && device_resident && parts == 1 && sk == 4 && n > 0) {
             HDB_CUDA(cudaStreamSynchronize(s0));   // e_b is in dc0.pin[0]
             const uint64_t eb = dc0.pin[0];
             S.sample_size = ns;

@@ -150,6 +150,16 @@ void launch_dbscan_device(const uint64_t* begin, const uint32_t* count, const ui
 void launch_scatter_rows(const uint32_t* ids, const uint64_t* off, const uint32_t* cnt, uint64_t q0,
                          uint64_t q1, uint64_t base, uint64_t* begin, uint32_t* count, cudaStream_t s);
 
+// the paper's kernels (kernels_paper.cu; search_kernel 7 / 8):
+// the key/value result set R of GPUCalcGlobal (Alg. 2) or GPUCalcShared (Alg. 3),
+// appended at *ctr (zeroed by the caller; counts past cap, writes only below it)
+constexpr int kPaperGlobal = 7, kPaperShared = 8;
+void launch_paper_search(const DevGrid& g, int which, unsigned long long* ctr, uint64_t cap, uint32_t* rkey,
+                         uint32_t* rval, cudaStream_t s);
+// T ranges from R sorted by key: begin[k] = first position of key k, count[k] = its run length
+void launch_rows_from_keys(const uint32_t* key_sorted, uint64_t m, uint64_t n, uint64_t* begin, uint32_t* count,
+                           cudaStream_t s);
+
 // ---------------------------------------------------------------- pools
 struct PinnedPool {
     std::mutex m;

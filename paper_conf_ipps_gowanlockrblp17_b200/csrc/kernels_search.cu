@@ -31,6 +31,7 @@
 #include <algorithm>
 
 #include "internal.h"
+#include "predicate.cuh"
 
 namespace hdb {
 
@@ -96,18 +97,6 @@ __device__ __forceinline__ u64x fma2(u64x a, u64x b, u64x c) {
     u64x r;
     asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(r) : "l"(a), "l"(b), "l"(c));
     return r;
-}
-
-// O1 predicate in exact f64: no FMA contraction possible with explicit _rn ops.
-__device__ __forceinline__ bool pred_f64(double xp, double yp, double xq, double yq, double e2) {
-    double dx = __dsub_rn(xp, xq);
-    double dy = __dsub_rn(yp, yq);
-    return __dadd_rn(__dmul_rn(dx, dx), __dmul_rn(dy, dy)) <= e2;
-}
-__device__ __forceinline__ bool pred_f32(float xp, float yp, float xq, float yq, float e2) {
-    float dx = __fsub_rn(xp, xq);
-    float dy = __fsub_rn(yp, yq);
-    return __fadd_rn(__fmul_rn(dx, dx), __fmul_rn(dy, dy)) <= e2;
 }
 
 // Kernel modes: f32 input (exact f32 predicate), f64 input with the f32

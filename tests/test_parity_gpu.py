@@ -540,3 +540,48 @@ def test_device_dbscan_shared_border_orders(torch_cuda):
         finally:
             hdb.hdb_ctx_destroy(ctx)
         assert lab.tolist() == o["labels"] and core.tolist() == o["core"] and k == o["n_clusters"]
+
+
+# ------------------------------------------------- the paper's kernels (NEXT-3)
+@pytest.mark.parametrize("kernel", [7, 8])
+@pytest.mark.parametrize("dtype", ["f64", "f32"])
+def test_paper_kernels_match_oracle(torch_cuda, kernel, dtype):
+    """search_kernel 7 / 8 = GPUCalcGlobal (Alg. 2) / GPUCalcShared (Alg. 3):
+    atomic key/value result set, sorted by key, T read off the keys -- the same
+    table as the oracle on the paper's eps cells (cell_split 1) and on split
+    grids, for uniform, banded and clustered data."""
+    cases = [(datagen.c1(), (datagen.C1_EPS,)),
+             (datagen.subsample(datagen.tec_like(), 30_000, seed=1), (0.15, 0.45)),
+             (datagen.subsample(datagen.sdss_like(), 30_000, seed=2), (0.07, 0.6))]
+    for xy, eps_list in cases:
+        if dtype == "f32":
+            xy = xy.astype(np.float32)
+        for eps in eps_list:
+            for split in (1, 2):
+                b, c, v, view, st = lib_table(xy, eps, device=True, search_kernel=kernel, cell_split=split)
+                assert view.npairs == int(c.astype(np.int64).sum()) == st["npairs"]
+                assert st["ms_sort"] > 0
+                assert_table_equal(xy, eps, b, c, v, dtype)
+
+
+@pytest.mark.parametrize("kernel", [7, 8])
+def test_paper_kernels_dense_cell_and_overflow(torch_cuda, kernel):
+    """A cell of 5,000 points (> blockDim = 256: Alg. 3's "additional loop",
+    P:518-521) and an estimate far below |R| (one sample on an isolated point):
+    the append counter reports the exact |R| and the kernel reruns once."""
+    rng = np.random.default_rng(5)
+    xy = np.concatenate([rng.normal(0, 0.05, (5000, 2)), rng.uniform(-5, 5, (3000, 2))])
+    b, c, v, _, st = lib_table(xy, 0.3, device=True, search_kernel=kernel, cell_split=1)
+    assert_table_equal(xy, 0.3, b, c, v)
+    sparse = rng.uniform(0, 100, size=(17_000, 2))
+    sparse[0] = (-50.0, -50.0)
+    xy2 = np.concatenate([sparse, np.full((3_000, 2), 50.0)])
+    b, c, v, view, st = lib_table(xy2, 0.5, device=True, sample_fraction=1e-6, search_kernel=kernel)
+    assert st["est_pairs"] < view.npairs and st["pool_grows"] >= 1
+    assert_table_equal(xy2, 0.5, b, c, v)
+
+
+def test_paper_kernels_need_device_tables(torch_cuda):
+    xy = datagen.c1()
+    with pytest.raises(hdb.HdbError):
+        lib_table(xy, datagen.C1_EPS, device=False, search_kernel=7)
