@@ -36,9 +36,10 @@ WORKLOADS = {
     "C2-eps0.45": dict(gen=datagen.tec_like, eps=0.45, desc="TEC-like n=1,864,620 eps=0.45 minpts=4"),
     "C2-eps0.15": dict(gen=datagen.tec_like, eps=0.15, desc="TEC-like n=1,864,620 eps=0.15 minpts=4"),
     "C2-eps1.40": dict(gen=datagen.tec_like, eps=1.40, desc="TEC-like n=1,864,620 eps=1.40 minpts=4"),
-    "C3-eps0.20": dict(gen=datagen.sdss_like, eps=0.20, desc="SDSS-like n=2,000,000 eps=0.20 minpts=4"),
-    "C3L-eps0.20": dict(gen=lambda: datagen.sdss_like(datagen.C3_N_LARGE, seed=4), eps=0.20,
-                        desc="SDSS-like n=5,000,000 eps=0.20 minpts=4"),
+    **{f"C3-eps{e:.2f}": dict(gen=datagen.sdss_like, eps=e, desc=f"SDSS-like n=2,000,000 eps={e:.2f} minpts=4")
+       for e in datagen.C3_EPS},
+    **{f"C3L-eps{e:.2f}": dict(gen=lambda: datagen.sdss_like(datagen.C3_N_LARGE, seed=4), eps=e,
+                               desc=f"SDSS-like n=5,000,000 eps={e:.2f} minpts=4") for e in datagen.C3_EPS},
     "C5-eps0.5": dict(gen=datagen.dense_skew, eps=0.5, desc="dense-skew n=50,000,000 eps=0.5 minpts=4"),
 }
 MINPTS = 4
@@ -467,7 +468,7 @@ def main():
             "clocks": clk.summary(),
             "stats": {k: st[k] for k in ("n_nonempty", "n_groups", "candidate_tests", "ms_grid", "ms_sample",
                                          "ms_count", "ms_scan", "ms_write_kernel", "kernel_launches",
-                                         "single_pass", "est_pairs", "ms_sort")}}
+                                         "single_pass", "est_pairs", "ms_sort", "n_sparse_queries")}}
 
     # ---- e2e through the C-ABI from pinned HOST points (H2D inside the timed region):
     #   value: the same metric (pairs/s) with the table delivered to a HOST table (D2H inside);

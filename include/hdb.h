@@ -163,6 +163,8 @@ typedef struct {
     double ms_sort;              /* search_kernel 7 / 8 (the paper's kernels): device time of the sort
                                     of the key/value result set by key + the T ranges (Alg. 4 line 7-8);
                                     ms_write_kernel is then the search kernel's time                   */
+    uint64_t n_sparse_queries;   /* queries of the grid's sparse groups, handled thread-per-query (the
+                                    dense/sparse hybrid); 0 = none       */
 } hdb_stats;
 
 /* ---- context ------------------------------------------------------------- */

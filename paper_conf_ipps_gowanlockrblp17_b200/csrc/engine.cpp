@@ -197,6 +197,18 @@ float elapsed(const Event& a, const Event& b) {
 
 constexpr uint64_t kMaxCellsAbs = 1ull << 30;
 
+// Dense/sparse split (NEXT-1): a query group goes to the thread-per-query kernel
+// when (queries x candidates) <= this many tests (
+// HDB_SPARSE_TESTS overrides it for tuning, 0 disables the split).
+constexpr double kSparseMinShare = 0.25;   // split only when >= this share of the queries is sparse
+uint32_t sparse_max_tests() {
+    static const uint32_t v = [] {
+        const char* e = std::getenv("HDB_SPARSE_TESTS");
+        return e ? (uint32_t)std::strtoul(e, nullptr, 10) : 256u;
+    }();
+    return v;
+}
+
 enum class Loc { Host, Device };
 
 struct PtrInfo {
@@ -449,8 +461,22 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
     // ---- stencil row spans per non-empty cell + query groups + hit-mask layout,
     // sized by upper bounds (groups <= n) so that one sync reads both counts
     DBuf cspan(8 * g.nspan * nne, s), gcount(4 * (nne + 1), s), gofs(4 * (nne + 1), s);
+    // the paper's dense G (Fig. 1) as a lookup, when the full grid is not much larger than the
+    // data: cnext[h] = first non-empty cell with key >= h (a scan of the occupancy marks)
+    DBuf cmark, cnext;
+    if (nne > 0 && g.n_cells <= std::max<uint64_t>(8 * n, 1ull << 22) && g.n_cells < (1ull << 32) - 1) {
+        cmark = DBuf(4 * (g.n_cells + 1), s);
+        cnext = DBuf(4 * (g.n_cells + 1), s);
+        DBuf ctemp(scan_temp_bytes(g.n_cells + 1), s);
+        HDB_CUDA(cudaMemsetAsync(cmark.p, 0, 4 * (g.n_cells + 1), s));
+        launch_cell_mark(ckey.as<uint64_t>(), nne, cmark.as<uint32_t>(), s);
+        scan_u32_to_u32(cmark.as<uint32_t>(), cnext.as<uint32_t>(), g.n_cells, ctemp.p, s);
+        HDB_LAUNCH_CHECK();
+    }
     launch_cell_spans(ckey.as<uint64_t>(), cstart.as<uint32_t>(), nne, g.nx, g.ny, g.split, cspan.as<uint2>(),
-                      gcount.as<uint32_t>(), s);
+                      gcount.as<uint32_t>(), cnext.as<uint32_t>(), s);
+    cmark.reset();
+    cnext.reset();
     scan_u32_to_u32(gcount.as<uint32_t>(), gofs.as<uint32_t>(), nne, temp.p, s);
     HDB_LAUNCH_CHECK();
     DBuf gstart(4 * (n + 1), s), gcell(4 * (n + 1), s);
@@ -466,6 +492,35 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
     g.cspan = (uint2*)cspan.release();
     g.gstart = (uint32_t*)gstart.release();
     g.gcell = (uint32_t*)gcell.release();
+    // dense/sparse hybrid (NEXT-1): groups with few tests take the thread-per-query
+    // kernel; search_kernel 3 / 4 (and the paper's kernels) keep one path for all groups
+    const int sk = ctx->opts.search_kernel;
+    const uint32_t max_tests = sparse_max_tests();
+    if ((sk == 0 || sk == 1 || sk == 2) && max_tests > 0 && n > 0) {
+        DBuf dflag(4 * (n + 1), s), sqn(4 * (n + 1), s);
+        DBuf dpre(4 * (n + 1), s), spre(4 * (n + 1), s), dl(4 * (n + 1), s), sql(8 * (n + 1), s);
+        const uint32_t* ngd = gofs.as<uint32_t>() + nne;
+        unsigned long long* nsp = bb + 8;
+        HDB_CUDA(cudaMemsetAsync(nsp, 0, 8, s));
+        launch_group_class(g.cstart, g.cspan, g.nspan, g.gstart, g.gcell, ngd, n, max_tests, dflag.as<uint32_t>(),
+                           sqn.as<uint32_t>(), nsp, s);
+        HDB_LAUNCH_CHECK();
+        HDB_CUDA(cudaMemcpyAsync(dc.pin + 6, nsp, 8, cudaMemcpyDeviceToHost, s));
+        HDB_CUDA(cudaStreamSynchronize(s));
+        // the split pays only when a good share of the queries is sparse: the thread-per-query
+        // kernels run after the dense ones and a few sparse groups only add their latency
+        if ((double)dc.pin[6] >= kSparseMinShare * (double)n) {
+            scan_u32_to_u32(dflag.as<uint32_t>(), dpre.as<uint32_t>(), n, temp.p, s);
+            scan_u32_to_u32(sqn.as<uint32_t>(), spre.as<uint32_t>(), n, temp.p, s);
+            launch_group_lists(g.gstart, g.gcell, ngd, n, dpre.as<uint32_t>(), spre.as<uint32_t>(),
+                               dl.as<uint32_t>(), sql.as<uint2>(), s);
+            HDB_LAUNCH_CHECK();
+            g.dpre = (uint32_t*)dpre.release();
+            g.spre = (uint32_t*)spre.release();
+            g.dl = (uint32_t*)dl.release();
+            g.sql = (uint2*)sql.release();
+        }
+    }
     {
         DBuf words(4 * (n + 1), s), mtemp(scan_temp_bytes(n + 1), s), moff(8 * (n + 1), s);
         launch_mask_words(g, gofs.as<uint32_t>() + nne, n, words.as<uint32_t>(), s);
@@ -474,10 +529,17 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
         uint32_t hng = 0;
         HDB_CUDA(cudaMemcpyAsync(&hng, gofs.as<uint32_t>() + nne, 4, cudaMemcpyDeviceToHost, s));
         HDB_CUDA(cudaMemcpyAsync(&g.mask_words, moff.as<uint64_t>() + n, 8, cudaMemcpyDeviceToHost, s));
+        uint32_t hds[2] = {0, 0};
+        if (g.dl) {
+            HDB_CUDA(cudaMemcpyAsync(&hds[0], g.dpre + n, 4, cudaMemcpyDeviceToHost, s));
+            HDB_CUDA(cudaMemcpyAsync(&hds[1], g.spre + n, 4, cudaMemcpyDeviceToHost, s));
+        }
         HDB_CUDA(cudaEventRecord(ev1.e, s));
         HDB_CUDA(cudaEventSynchronize(ev1.e));
         g.n_groups = hng;
         g.moff = (uint64_t*)moff.release();
+        g.n_dense_groups = g.dl ? hds[0] : hng;
+        g.n_sparse_q = hds[1];
     }
     g.ms_build = elapsed(ev0, ev1);
     gcount.reset();
@@ -491,13 +553,16 @@ void free_dev_grid(DevGrid& g) {
     if (!g.stream) return;
     DeviceGuard dg(g.device);
     for (void* p : {(void*)g.xy_s, (void*)g.xp, (void*)g.counters, (void*)g.ids, (void*)g.ckey, (void*)g.cstart,
-                    (void*)g.cspan, (void*)g.gstart, (void*)g.gcell, (void*)g.moff})
+                    (void*)g.cspan, (void*)g.gstart, (void*)g.gcell, (void*)g.moff, (void*)g.dpre, (void*)g.spre,
+                    (void*)g.dl, (void*)g.sql})
         if (p) cudaFreeAsync(p, g.stream);   // stream-ordered: no host sync needed
     g.xy_s = nullptr;
     g.xp = nullptr;
     g.counters = nullptr;
     g.ids = g.cstart = g.gstart = g.gcell = nullptr;
     g.moff = nullptr;
+    g.dpre = g.spre = g.dl = nullptr;
+    g.sql = nullptr;
     g.ckey = nullptr;
     g.cspan = nullptr;
     cudaStreamSynchronize(g.stream);
@@ -528,6 +593,7 @@ void grid_build(hdb_ctx* ctx, const void* xy, uint64_t n, hdb_dtype dt, double e
     ctx->stats.n_cells = g0.n_cells;
     ctx->stats.n_nonempty = g0.n_nonempty;
     ctx->stats.n_groups = g0.n_groups;
+    ctx->stats.n_sparse_queries = g0.n_sparse_q;
     ctx->stats.ms_grid = g0.ms_build;
     ctx->stats.kernel_launches = (uint32_t)(g_kernel_launches.load() - launches0);
     ctx->live_objects++;
@@ -943,6 +1009,7 @@ void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hd
     S.n_cells = G0.n_cells;
     S.n_nonempty = G0.n_nonempty;
     S.n_groups = G0.n_groups;
+    S.n_sparse_queries = G0.n_sparse_q;
     S.bytes_d2h = 0;
     S.pool_grows = 0;
     S.n_streams = ctx->opts.n_streams;

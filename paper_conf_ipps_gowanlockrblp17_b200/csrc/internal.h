@@ -73,6 +73,12 @@ struct DevGrid {
     uint32_t* gcell = nullptr;     // [n_groups] non-empty cell index of each query group
     uint64_t* moff = nullptr;      // [n_groups+1] first 32-bit word of each group's hit masks
     uint64_t mask_words = 0;       // moff[n_groups]
+    // dense/sparse hybrid (NEXT-1): null when every group takes the warp-per-group path
+    uint32_t* dpre = nullptr;      // [n_groups+1] dense groups before g
+    uint32_t* dl = nullptr;        // [#dense] the dense groups, ascending
+    uint32_t* spre = nullptr;      // [n_groups+1] sparse queries before group g
+    uint2* sql = nullptr;          // [n_sparse_q] {sorted position, non-empty cell} of each sparse query
+    uint64_t n_sparse_q = 0, n_dense_groups = 0;
     cudaStream_t stream = nullptr; // stream the buffers were allocated on
     float ms_build = 0;
 };
@@ -97,8 +103,11 @@ void launch_gather_points(const void* xy_in, const uint32_t* ids, uint64_t n, hd
 void launch_cell_flags(const void* keys_sorted, int key_bytes, uint64_t n, uint32_t* flags, cudaStream_t s);
 void launch_cell_scatter(const void* keys_sorted, int key_bytes, const uint32_t* flags, const uint32_t* pos,
                          uint64_t n, uint64_t* ckey, uint32_t* cstart, cudaStream_t s);
+// cnext: optional dense lookup (first non-empty cell with key >= h, h in [0, nx*ny]); null = binary search
 void launch_cell_spans(const uint64_t* ckey, const uint32_t* cstart, uint64_t nne, uint32_t nx, uint32_t ny,
-                       uint32_t k, uint2* cspan, uint32_t* gcount, cudaStream_t s);
+                       uint32_t k, uint2* cspan, uint32_t* gcount, const uint32_t* cnext, cudaStream_t s);
+// mark[ckey[c]] = 1 for every non-empty cell (mark zeroed by the caller)
+void launch_cell_mark(const uint64_t* ckey, uint64_t nne, uint32_t* mark, cudaStream_t s);
 // auto cell split: sample-based point-weighted occupancy at cell width 1/inv_w;
 // out[0] = sum s_c (s_c - 1), out[1] = sum s_c over the sampled cells
 void launch_occ_estimate(const void* xy, uint64_t n, hdb_dtype dt, uint64_t stride, uint64_t m, double inv_w,
@@ -106,6 +115,15 @@ void launch_occ_estimate(const void* xy, uint64_t n, hdb_dtype dt, uint64_t stri
                          cudaStream_t s);
 void launch_group_build(const uint32_t* cstart, const uint32_t* gofs, uint64_t nne, uint64_t n, uint32_t* gstart,
                         uint32_t* gcell, cudaStream_t s);
+// dense/sparse classification of the groups g < *ng_dev (entries up to n): dflag[g] = 1 for a
+// dense group, sqn[g] = its query count for a sparse one (sparse <=> queries x candidates <=
+// max_tests), *n_sparse += the sparse queries; then the lists dl[dpre[g]] = g (dense) and
+// sql[spre[g] + i] = {gstart[g] + i, gcell[g]}
+void launch_group_class(const uint32_t* cstart, const uint2* cspan, uint32_t nspan, const uint32_t* gstart,
+                        const uint32_t* gcell, const uint32_t* ng_dev, uint64_t n, uint32_t max_tests,
+                        uint32_t* dflag, uint32_t* sqn, unsigned long long* n_sparse, cudaStream_t s);
+void launch_group_lists(const uint32_t* gstart, const uint32_t* gcell, const uint32_t* ng_dev, uint64_t n,
+                        const uint32_t* dpre, const uint32_t* spre, uint32_t* dl, uint2* sql, cudaStream_t s);
 
 // scans (kernels_scan.cu): exclusive scan of in[0..n) into out[0..n], out[n] = total
 size_t scan_temp_bytes(uint64_t n);

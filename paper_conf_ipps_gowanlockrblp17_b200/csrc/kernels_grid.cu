@@ -304,10 +304,14 @@ __device__ __forceinline__ uint64_t lower_bound_u64(const uint64_t* __restrict__
 // contiguous range, found by two binary searches over the non-empty keys
 // (rows below cy precede c, rows above follow it).  Also gcount[c] = number of
 // 32-query groups of the cell.
+// cnext (optional): the paper's dense G over all cells (Fig. 1) in lookup form,
+// cnext[h] = index of the first non-empty cell with key >= h, h <= nx*ny --
+// then every span is two lookups instead of two binary searches.
 __global__ void __launch_bounds__(256) k_cell_spans(const uint64_t* __restrict__ ckey,
                                                     const uint32_t* __restrict__ cstart, uint64_t nne,
                                                     uint32_t nx, uint32_t ny, uint32_t k, uint2* __restrict__ cspan,
-                                                    uint32_t* __restrict__ gcount) {
+                                                    uint32_t* __restrict__ gcount,
+                                                    const uint32_t* __restrict__ cnext) {
     const uint32_t nspan = 2 * k + 1;
     for (uint64_t c = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; c < nne;
          c += (uint64_t)gridDim.x * blockDim.x) {
@@ -320,17 +324,29 @@ __global__ void __launch_bounds__(256) k_cell_spans(const uint64_t* __restrict__
             uint2 sp = make_uint2(0, 0);
             if (yy >= 0 && yy < (int64_t)ny) {
                 const uint64_t rb = (uint64_t)yy * nx;
-                uint64_t lo = 0, hi = nne;
-                if (yy < (int64_t)cy) hi = c;
-                else if (yy > (int64_t)cy) lo = c + 1;
-                const uint64_t i0 = lower_bound_u64(ckey, lo, hi, rb + xl);
-                const uint64_t i1 = lower_bound_u64(ckey, i0, hi, rb + xh + 1);
+                uint64_t i0, i1;
+                if (cnext) {
+                    i0 = __ldg(&cnext[rb + xl]);
+                    i1 = __ldg(&cnext[rb + xh + 1]);
+                } else {
+                    uint64_t lo = 0, hi = nne;
+                    if (yy < (int64_t)cy) hi = c;
+                    else if (yy > (int64_t)cy) lo = c + 1;
+                    i0 = lower_bound_u64(ckey, lo, hi, rb + xl);
+                    i1 = lower_bound_u64(ckey, i0, hi, rb + xh + 1);
+                }
                 sp = make_uint2(cstart[i0], cstart[i1]);
             }
             cspan[nspan * c + r] = sp;
         }
         gcount[c] = (cstart[c + 1] - cstart[c] + (uint32_t)kGroup - 1) / (uint32_t)kGroup;
     }
+}
+
+__global__ void __launch_bounds__(256) k_cell_mark(const uint64_t* __restrict__ ckey, uint64_t nne,
+                                                   uint32_t* __restrict__ mark) {
+    for (uint64_t c = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; c < nne; c += (uint64_t)gridDim.x * blockDim.x)
+        mark[ckey[c]] = 1;
 }
 
 __global__ void __launch_bounds__(256) k_group_build(const uint32_t* __restrict__ cstart,
@@ -346,6 +362,55 @@ __global__ void __launch_bounds__(256) k_group_build(const uint32_t* __restrict_
         }
     }
     if (blockIdx.x == 0 && threadIdx.x == 0) gstart[gofs[nne]] = (uint32_t)n;
+}
+
+// ---------------------------------------------------------------- dense / sparse groups (NEXT-1)
+__global__ void __launch_bounds__(256) k_group_class(const uint32_t* __restrict__ cstart,
+                                                     const uint2* __restrict__ cspan, uint32_t nspan,
+                                                     const uint32_t* __restrict__ gstart,
+                                                     const uint32_t* __restrict__ gcell,
+                                                     const uint32_t* __restrict__ ng_dev, uint64_t n,
+                                                     uint32_t max_tests, uint32_t* __restrict__ dflag,
+                                                     uint32_t* __restrict__ sqn,
+                                                     unsigned long long* __restrict__ n_sparse) {
+    const uint64_t ng = *ng_dev;
+    uint32_t tot = 0;
+    for (uint64_t g = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; g < n; g += (uint64_t)gridDim.x * blockDim.x) {
+        uint32_t d = 0, sq = 0;
+        if (g < ng) {
+            const uint32_t qs = gstart[g], c = gcell[g];
+            const uint32_t nq = min((uint32_t)kGroup, cstart[c + 1] - qs);
+            uint64_t cand = 0;
+            for (uint32_t r = 0; r < nspan; ++r) {
+                const uint2 sp = cspan[(uint64_t)nspan * c + r];
+                cand += sp.y - sp.x;
+            }
+            if ((uint64_t)nq * cand <= max_tests) sq = nq;
+            else d = 1;
+        }
+        dflag[g] = d;
+        sqn[g] = sq;
+        tot += sq;
+    }
+    for (int o = 16; o > 0; o >>= 1) tot += __shfl_xor_sync(0xffffffffu, tot, o);
+    if ((threadIdx.x & 31) == 0 && tot) atomicAdd(n_sparse, (unsigned long long)tot);
+}
+
+__global__ void __launch_bounds__(256) k_group_lists(const uint32_t* __restrict__ gstart,
+                                                     const uint32_t* __restrict__ gcell,
+                                                     const uint32_t* __restrict__ ng_dev, uint64_t n,
+                                                     const uint32_t* __restrict__ dpre,
+                                                     const uint32_t* __restrict__ spre, uint32_t* __restrict__ dl,
+                                                     uint2* __restrict__ sql) {
+    const uint64_t ng = *ng_dev;
+    for (uint64_t g = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; g < ng; g += (uint64_t)gridDim.x * blockDim.x) {
+        if (dpre[g + 1] != dpre[g]) {
+            dl[dpre[g]] = (uint32_t)g;
+        } else {
+            const uint32_t j = spre[g], m = spre[g + 1] - j, qs = gstart[g], c = gcell[g];
+            for (uint32_t i = 0; i < m; ++i) sql[j + i] = make_uint2(qs + i, c);
+        }
+    }
 }
 
 // ---------------------------------------------------------------- auto cell split
@@ -521,15 +586,37 @@ void launch_cell_scatter(const void* keys_sorted, int key_bytes, const uint32_t*
 }
 
 void launch_cell_spans(const uint64_t* ckey, const uint32_t* cstart, uint64_t nne, uint32_t nx, uint32_t ny,
-                       uint32_t k, uint2* cspan, uint32_t* gcount, cudaStream_t s) {
+                       uint32_t k, uint2* cspan, uint32_t* gcount, const uint32_t* cnext, cudaStream_t s) {
     if (nne == 0) return;
-    k_cell_spans<<<grid_for(nne), 256, 0, s>>>(ckey, cstart, nne, nx, ny, k, cspan, gcount);
+    k_cell_spans<<<grid_for(nne), 256, 0, s>>>(ckey, cstart, nne, nx, ny, k, cspan, gcount, cnext);
+    ++g_kernel_launches;
+}
+
+void launch_cell_mark(const uint64_t* ckey, uint64_t nne, uint32_t* mark, cudaStream_t s) {
+    if (nne == 0) return;
+    k_cell_mark<<<grid_for(nne), 256, 0, s>>>(ckey, nne, mark);
     ++g_kernel_launches;
 }
 
 void launch_group_build(const uint32_t* cstart, const uint32_t* gofs, uint64_t nne, uint64_t n, uint32_t* gstart,
                         uint32_t* gcell, cudaStream_t s) {
     k_group_build<<<grid_for(nne), 256, 0, s>>>(cstart, gofs, nne, n, gstart, gcell);
+    ++g_kernel_launches;
+}
+
+void launch_group_class(const uint32_t* cstart, const uint2* cspan, uint32_t nspan, const uint32_t* gstart,
+                        const uint32_t* gcell, const uint32_t* ng_dev, uint64_t n, uint32_t max_tests,
+                        uint32_t* dflag, uint32_t* sqn, unsigned long long* n_sparse, cudaStream_t s) {
+    if (n == 0) return;
+    k_group_class<<<grid_for(n), 256, 0, s>>>(cstart, cspan, nspan, gstart, gcell, ng_dev, n, max_tests, dflag, sqn,
+                                              n_sparse);
+    ++g_kernel_launches;
+}
+
+void launch_group_lists(const uint32_t* gstart, const uint32_t* gcell, const uint32_t* ng_dev, uint64_t n,
+                        const uint32_t* dpre, const uint32_t* spre, uint32_t* dl, uint2* sql, cudaStream_t s) {
+    if (n == 0) return;
+    k_group_lists<<<grid_for(n), 256, 0, s>>>(gstart, gcell, ng_dev, n, dpre, spre, dl, sql);
     ++g_kernel_launches;
 }
 

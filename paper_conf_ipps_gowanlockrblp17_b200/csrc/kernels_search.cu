@@ -56,7 +56,22 @@ struct SArgs {
     float band_l;          // f64 mode, group-local filter (count pass)
     float nb2_l;           //   -(band_l (1 + 2^-20))^2
     double e2d;            // fl64(eps^2)
+    // dense/sparse hybrid (NEXT-1): the warp-per-group
+    // kernels visit only the dense groups dl[dpre[g0] .. dpre[g1]) of a group range
+    // (dl == null: every group); the sparse groups' queries sql[spre[g0] .. spre[g1])
+    // = {sorted position, cell} go to the thread-per-query kernel k_sparse
+    const uint32_t* dl;
+    const uint32_t* dpre;
+    const uint2* sql;
+    const uint32_t* spre;
 };
+
+__device__ __forceinline__ void dense_range(const SArgs& a, uint32_t& i0, uint32_t& i1) {
+    if (a.dl) {
+        i0 = __ldg(&a.dpre[i0]);
+        i1 = __ldg(&a.dpre[i1]);
+    }
+}
 
 typedef unsigned long long u64x;
 
@@ -339,8 +354,11 @@ __global__ void __launch_bounds__(kSearchThreads) k_count(SArgs a, uint32_t g0, 
 #pragma unroll
     for (int kk = 0; kk < kWin; ++kk) swin[w][lane][kk] = make_uint2(0, 0);
     unsigned long long tests = 0;
-    uint32_t gi = g0 + grab(ctr, chunk, lane), gend = min(gi + chunk, g1);
-    while (gi < g1) {
+    uint32_t i0 = g0, i1 = g1;
+    dense_range(a, i0, i1);
+    uint32_t ii = i0 + grab(ctr, chunk, lane), iend = min(ii + chunk, i1);
+    while (ii < i1) {
+        const uint32_t gi = a.dl ? __ldg(&a.dl[ii]) : ii;
         const uint32_t qs = __ldg(&a.gstart[gi]);
         const uint32_t c = __ldg(&a.gcell[gi]);
         const uint32_t nq = min((uint32_t)kGroup, __ldg(&a.cstart[c + 1]) - qs);
@@ -348,9 +366,9 @@ __global__ void __launch_bounds__(kSearchThreads) k_count(SArgs a, uint32_t g0, 
         const uint32_t my =
             count_group<MODE>(a, qs, c, nq, swin[w], vsp[w], sq[w], sqd[F64 ? w : 0], gmask, tests, lane);
         if ((uint32_t)lane < nq) cnt[qs + lane] = my;
-        if (++gi >= gend) {
-            gi = g0 + grab(ctr, chunk, lane);
-            gend = min(gi + chunk, g1);
+        if (++ii >= iend) {
+            ii = i0 + grab(ctr, chunk, lane);
+            iend = min(ii + chunk, i1);
         }
     }
 #pragma unroll
@@ -385,8 +403,11 @@ __global__ void __launch_bounds__(kSearchThreads) k_search(SArgs a, uint32_t g0,
     const u64x NE2 = pack2(-a.e2f, -a.e2f);
     const float band = a.band;
     unsigned long long tests = 0;
-    uint32_t gi = g0 + grab(ctr, chunk, lane), gend = min(gi + chunk, g1);
-    while (gi < g1) {
+    uint32_t i0 = g0, i1 = g1;
+    dense_range(a, i0, i1);
+    uint32_t ii = i0 + grab(ctr, chunk, lane), iend = min(ii + chunk, i1);
+    while (ii < i1) {
+        const uint32_t gi = a.dl ? __ldg(&a.dl[ii]) : ii;
         const uint32_t qs = __ldg(&a.gstart[gi]);
         const uint32_t c = __ldg(&a.gcell[gi]);
         const uint32_t nq = min((uint32_t)kGroup, __ldg(&a.cstart[c + 1]) - qs);
@@ -503,9 +524,9 @@ __global__ void __launch_bounds__(kSearchThreads) k_search(SArgs a, uint32_t g0,
         }
         if (!WRITE && gmask && (k % kWin) != 0) flush_window(swin[WRITE ? 0 : w], gmask, k / kWin, nq, lane);
         if (!WRITE && (uint32_t)lane < nq) cnt[qs + lane] = my;
-        if (++gi >= gend) {
-            gi = g0 + grab(ctr, chunk, lane);
-            gend = min(gi + chunk, g1);
+        if (++ii >= iend) {
+            ii = i0 + grab(ctr, chunk, lane);
+            iend = min(ii + chunk, i1);
         }
     }
     if (!WRITE && tests_out && lane == 0 && tests) atomicAdd(tests_out, tests);
@@ -606,8 +627,11 @@ __global__ void __launch_bounds__(kEmitThreads) k_emit(SArgs a, uint32_t g0, uin
     __shared__ VSpan vsp[kEmitWarps][kMaxSpans + 1];  // the group's spans as one pair sequence
     const int lane = threadIdx.x & 31;
     const int w = threadIdx.x >> 5;
-    uint32_t gi = g0 + grab(ctr, chunk, lane), gend = min(gi + chunk, g1);
-    while (gi < g1) {
+    uint32_t i0 = g0, i1 = g1;
+    dense_range(a, i0, i1);
+    uint32_t ii = i0 + grab(ctr, chunk, lane), iend = min(ii + chunk, i1);
+    while (ii < i1) {
+        const uint32_t gi = a.dl ? __ldg(&a.dl[ii]) : ii;
         const uint32_t qs = __ldg(&a.gstart[gi]);
         const uint32_t c = __ldg(&a.gcell[gi]);
         const uint32_t nq = min((uint32_t)kGroup, __ldg(&a.cstart[c + 1]) - qs);
@@ -619,9 +643,9 @@ __global__ void __launch_bounds__(kEmitThreads) k_emit(SArgs a, uint32_t g0, uin
         uint32_t my = 0;   // lane i: output cursor of query i within the group
         if ((uint32_t)lane < nq) my = (uint32_t)(off[qs + lane] - gb);
         emit_group(a, c, nq, nwin, masks + (m_a >> 1), gout, my, raw[w], wq[w], vsp[w], lane);
-        if (++gi >= gend) {
-            gi = g0 + grab(ctr, chunk, lane);
-            gend = min(gi + chunk, g1);
+        if (++ii >= iend) {
+            ii = i0 + grab(ctr, chunk, lane);
+            iend = min(ii + chunk, i1);
         }
     }
 }
@@ -658,8 +682,11 @@ __global__ void __launch_bounds__(kFusedThreads) k_fused(SArgs a, uint32_t g0, u
 #pragma unroll
     for (int kk = 0; kk < kWin; ++kk) swin[w][lane][kk] = make_uint2(0, 0);
     unsigned long long tests = 0;
-    uint32_t gi = g0 + grab(ctr, chunk, lane), gend = min(gi + chunk, g1);
-    while (gi < g1) {
+    uint32_t i0 = g0, i1 = g1;
+    dense_range(a, i0, i1);
+    uint32_t ii = i0 + grab(ctr, chunk, lane), iend = min(ii + chunk, i1);
+    while (ii < i1) {
+        const uint32_t gi = a.dl ? __ldg(&a.dl[ii]) : ii;
         const uint32_t qs = __ldg(&a.gstart[gi]);
         const uint32_t c = __ldg(&a.gcell[gi]);
         const uint32_t nq = min((uint32_t)kGroup, __ldg(&a.cstart[c + 1]) - qs);
@@ -695,9 +722,9 @@ __global__ void __launch_bounds__(kFusedThreads) k_fused(SArgs a, uint32_t g0, u
         } else if (lane == 0) {
             atomicOr(overflow, 1u);
         }
-        if (++gi >= gend) {
-            gi = g0 + grab(ctr, chunk, lane);
-            gend = min(gi + chunk, g1);
+        if (++ii >= iend) {
+            ii = i0 + grab(ctr, chunk, lane);
+            iend = min(ii + chunk, i1);
         }
     }
 #pragma unroll
@@ -715,6 +742,10 @@ __global__ void __launch_bounds__(256) k_mask_words(SArgs a, const uint32_t* __r
             words[g] = 0;
             continue;
         }
+        if (a.dl && a.dpre[g + 1] == a.dpre[g]) {   // sparse group: thread-per-query path, no masks
+            words[g] = 0;
+            continue;
+        }
         const uint32_t qs = a.gstart[g], c = a.gcell[g];
         const uint32_t nq = min((uint32_t)kGroup, a.cstart[c + 1] - qs);
         uint32_t npairs = 0;
@@ -724,6 +755,73 @@ __global__ void __launch_bounds__(256) k_mask_words(SArgs a, const uint32_t* __r
         }
         const uint32_t ch = (npairs + 31) / 32;
         words[g] = 2 * nq * kWin * ((ch + kWin - 1) / kWin);
+    }
+}
+
+// Sparse queries (NEXT-1, the dense/sparse hybrid):
+// one thread per query of a sparse group -- GPUCalcGlobal's mapping (Alg. 2,
+// P:443-450), which the paper found best where cells hold few points
+// (Table II) -- scanning its cell's row spans with the exact
+// predicate in the input precision.  Count pass: cnt[q]; write pass (same
+// candidate order): out[off[q] - out_base ...].  A warp-per-group iteration
+// costs ~300 instructions of set-up plus ~100 per 64-candidate chunk; a group
+// of 2 queries with ~20 candidates (SDSS-like at eps 0.07) would use a whole
+// warp for 40 tests.
+template <bool F64, bool WRITE>
+__global__ void __launch_bounds__(256) k_sparse(SArgs a, uint32_t g0, uint32_t g1, uint32_t* __restrict__ cnt,
+                                                unsigned long long* __restrict__ tests_out,
+                                                const uint64_t* __restrict__ off, uint64_t out_base,
+                                                uint32_t* __restrict__ out) {
+    const uint32_t j0 = __ldg(&a.spre[g0]), j1 = __ldg(&a.spre[g1]);
+    unsigned long long tests = 0;
+    for (uint32_t j = j0 + blockIdx.x * blockDim.x + threadIdx.x; j < j1; j += gridDim.x * blockDim.x) {
+        const uint2 e = __ldg(&a.sql[j]);
+        const uint32_t q = e.x, c = e.y;
+        double2 pd = make_double2(0, 0);
+        float2 pf = make_float2(0, 0);
+        if (F64) pd = a.xd[q];
+        else pf = a.xs[q];
+        uint32_t m = 0;
+        uint32_t* o = nullptr;
+        if (WRITE) o = out + (off[q] - out_base);
+        auto test = [&](uint32_t k) -> bool {
+            if (F64) {
+                const double2 v = __ldg(&a.xd[k]);
+                return pred_f64(pd.x, pd.y, v.x, v.y, a.e2d);
+            }
+            const float2 v = __ldg(&a.xs[k]);
+            return pred_f32(pf.x, pf.y, v.x, v.y, a.e2f);
+        };
+        for (uint32_t r = 0; r < a.nspan; ++r) {
+            const uint2 sp = __ldg(&a.cspan[a.nspan * c + r]);
+            if (!WRITE) tests += sp.y - sp.x;
+            uint32_t k = sp.x;
+            // four candidates per step: the loads are issued together (memory-level parallelism;
+            // a thread's candidates are a few short spans, so latency, not bandwidth, bounds it)
+            for (; k + 4 <= sp.y; k += 4) {
+                const bool h0 = test(k), h1 = test(k + 1), h2 = test(k + 2), h3 = test(k + 3);
+                if (WRITE) {
+                    if (h0) o[m++] = __ldg(&a.ids[k]);
+                    if (h1) o[m++] = __ldg(&a.ids[k + 1]);
+                    if (h2) o[m++] = __ldg(&a.ids[k + 2]);
+                    if (h3) o[m++] = __ldg(&a.ids[k + 3]);
+                } else {
+                    m += (uint32_t)h0 + (uint32_t)h1 + (uint32_t)h2 + (uint32_t)h3;
+                }
+            }
+            for (; k < sp.y; ++k) {
+                if (test(k)) {
+                    if (WRITE) o[m] = __ldg(&a.ids[k]);
+                    ++m;
+                }
+            }
+        }
+        if (!WRITE) cnt[q] = m;
+    }
+    if (!WRITE && tests_out) {
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) tests += __shfl_xor_sync(FULL, tests, o);
+        if ((threadIdx.x & 31) == 0 && tests) atomicAdd(tests_out, tests);
     }
 }
 
@@ -850,7 +948,19 @@ SArgs args_of(const DevGrid& g) {
     a.band_l = g.band_l;
     a.nb2_l = g.nb2_l;
     a.e2d = g.e2_d;
+    a.dl = g.dl;
+    a.dpre = g.dpre;
+    a.sql = g.sql;
+    a.spre = g.spre;
     return a;
+}
+
+// Groups the warp kernels visit in [g0, g1): all, or (dense/sparse split) the
+// range's share of the dense groups -- sizes the grab chunk, so that a few
+// heavy dense groups among many sparse ones still spread over every warp.
+uint64_t dense_groups(const DevGrid& g, uint64_t g0, uint64_t g1) {
+    if (!g.dl || g.n_groups == 0) return g1 - g0;
+    return std::max<uint64_t>(1, (uint64_t)((double)(g1 - g0) * (double)g.n_dense_groups / (double)g.n_groups));
 }
 
 // One wave of resident CTAs; warps grab `chunk` groups at a time (~32 grabs
@@ -872,13 +982,13 @@ void launch_groups(K kern, int& blocks_per_sm, uint64_t ng, uint32_t& chunk, uns
 }
 
 template <int MODE, bool WRITE>
-void launch_mode(const SArgs& a, uint64_t g0, uint64_t g1, unsigned int* ctr, uint32_t* cnt,
+void launch_mode(const SArgs& a, uint64_t g0, uint64_t g1, uint64_t ngd, unsigned int* ctr, uint32_t* cnt,
                  unsigned long long* tests, const uint64_t* off, uint64_t out_base, uint32_t* out, uint2* masks,
                  const uint64_t* moff, cudaStream_t s) {
     static int bps = 0;
     uint32_t chunk;
     unsigned ctas;
-    launch_groups(k_search<MODE, WRITE>, bps, g1 - g0, chunk, ctas);
+    launch_groups(k_search<MODE, WRITE>, bps, ngd, chunk, ctas);
     k_search<MODE, WRITE><<<ctas, kSearchThreads, 0, s>>>(a, (uint32_t)g0, (uint32_t)g1, chunk, ctr, cnt, tests, off,
                                                           out_base, out, masks, moff);
 }
@@ -897,11 +1007,11 @@ void launch_search(const DevGrid& g, uint64_t g0, uint64_t g1, uint32_t* cnt, un
     cudaMemsetAsync(ctr, 0, sizeof(unsigned int), s);
     const int mode = mode_of(g, force_exact);
     if (mode == kF64Filter)
-        launch_mode<kF64Filter, WRITE>(a, g0, g1, ctr, cnt, tests, off, out_base, out, masks, g.moff, s);
+        launch_mode<kF64Filter, WRITE>(a, g0, g1, dense_groups(g, g0, g1), ctr, cnt, tests, off, out_base, out, masks, g.moff, s);
     else if (mode == kF64Exact)
-        launch_mode<kF64Exact, WRITE>(a, g0, g1, ctr, cnt, tests, off, out_base, out, masks, g.moff, s);
+        launch_mode<kF64Exact, WRITE>(a, g0, g1, dense_groups(g, g0, g1), ctr, cnt, tests, off, out_base, out, masks, g.moff, s);
     else
-        launch_mode<kF32, WRITE>(a, g0, g1, ctr, cnt, tests, off, out_base, out, masks, g.moff, s);
+        launch_mode<kF32, WRITE>(a, g0, g1, dense_groups(g, g0, g1), ctr, cnt, tests, off, out_base, out, masks, g.moff, s);
     ++g_kernel_launches;
 }
 
@@ -921,14 +1031,28 @@ void launch_sample_count(const DevGrid& g, uint64_t stride, uint64_t n_sample, u
     ++g_kernel_launches;
 }
 
+template <bool WRITE>
+void launch_sparse(const DevGrid& g, uint64_t g0, uint64_t g1, uint32_t* cnt, unsigned long long* tests,
+                   const uint64_t* off, uint64_t out_base, uint32_t* out, cudaStream_t s) {
+    if (!g.sql || g.n_sparse_q == 0 || g1 <= g0) return;
+    const unsigned blocks = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>((g.n_sparse_q + 255) / 256, 148 * 16));
+    if (g.dtype == HDB_F64)
+        k_sparse<true, WRITE><<<blocks, 256, 0, s>>>(args_of(g), (uint32_t)g0, (uint32_t)g1, cnt, tests, off, out_base,
+                                                     out);
+    else
+        k_sparse<false, WRITE><<<blocks, 256, 0, s>>>(args_of(g), (uint32_t)g0, (uint32_t)g1, cnt, tests, off,
+                                                      out_base, out);
+    ++g_kernel_launches;
+}
+
 // variant (hdb_opts.search_kernel): 0 = default, 1 = force the exact-f64-only kernel
 template <int MODE>
-void launch_count_mode(const SArgs& a, uint64_t g0, uint64_t g1, unsigned int* ctr, uint32_t* cnt,
+void launch_count_mode(const SArgs& a, uint64_t g0, uint64_t g1, uint64_t ngd, unsigned int* ctr, uint32_t* cnt,
                        unsigned long long* tests, uint2* masks, const uint64_t* moff, cudaStream_t s) {
     static int bps = 0;
     uint32_t chunk;
     unsigned ctas;
-    launch_groups(k_count<MODE>, bps, g1 - g0, chunk, ctas);
+    launch_groups(k_count<MODE>, bps, ngd, chunk, ctas);
     k_count<MODE><<<ctas, kSearchThreads, 0, s>>>(a, (uint32_t)g0, (uint32_t)g1, chunk, ctr, cnt, tests, masks, moff);
 }
 
@@ -936,15 +1060,16 @@ void launch_count(const DevGrid& g, uint64_t g0, uint64_t g1, uint32_t* cnt, uns
                   int variant, int slot, uint2* masks, cudaStream_t s) {
     if (g1 <= g0) return;
     const SArgs a = args_of(g);
+    launch_sparse<false>(g, g0, g1, cnt, tests, nullptr, 0, nullptr, s);
     unsigned int* ctr = g.counters + (slot % kCounterSlots);
     cudaMemsetAsync(ctr, 0, sizeof(unsigned int), s);
     const int mode = g.dtype == HDB_F32 ? kF32 : (g.filter_l && variant != 1 ? kF64Filter : kF64Exact);
     if (mode == kF64Filter)
-        launch_count_mode<kF64Filter>(a, g0, g1, ctr, cnt, tests, masks, g.moff, s);
+        launch_count_mode<kF64Filter>(a, g0, g1, dense_groups(g, g0, g1), ctr, cnt, tests, masks, g.moff, s);
     else if (mode == kF64Exact)
-        launch_count_mode<kF64Exact>(a, g0, g1, ctr, cnt, tests, masks, g.moff, s);
+        launch_count_mode<kF64Exact>(a, g0, g1, dense_groups(g, g0, g1), ctr, cnt, tests, masks, g.moff, s);
     else
-        launch_count_mode<kF32>(a, g0, g1, ctr, cnt, tests, masks, g.moff, s);
+        launch_count_mode<kF32>(a, g0, g1, dense_groups(g, g0, g1), ctr, cnt, tests, masks, g.moff, s);
     ++g_kernel_launches;
 }
 
@@ -952,6 +1077,7 @@ void launch_count(const DevGrid& g, uint64_t g0, uint64_t g1, uint32_t* cnt, uns
 // write pass recomputes the distance tests (k_search<WRITE>).
 void launch_write(const DevGrid& g, uint64_t g0, uint64_t g1, const uint64_t* off, uint64_t out_base,
                   uint32_t* out, int variant, int slot, const uint2* masks, cudaStream_t s) {
+    launch_sparse<true>(g, g0, g1, nullptr, nullptr, off, out_base, out, s);
     if (!masks) {
         launch_search<true>(g, g0, g1, nullptr, nullptr, off, out_base, out, variant == 1, slot, nullptr, s);
         return;
@@ -962,7 +1088,7 @@ void launch_write(const DevGrid& g, uint64_t g0, uint64_t g1, const uint64_t* of
     static int bps = 0;
     uint32_t chunk;
     unsigned ctas;
-    launch_groups(k_emit, bps, g1 - g0, chunk, ctas, kEmitThreads);
+    launch_groups(k_emit, bps, dense_groups(g, g0, g1), chunk, ctas, kEmitThreads);
     k_emit<<<ctas, kEmitThreads, 0, s>>>(args_of(g), (uint32_t)g0, (uint32_t)g1, chunk, ctr, off, out_base, out,
                                            masks, g.moff);
     ++g_kernel_launches;

@@ -585,3 +585,44 @@ def test_paper_kernels_need_device_tables(torch_cuda):
     xy = datagen.c1()
     with pytest.raises(hdb.HdbError):
         lib_table(xy, datagen.C1_EPS, device=False, search_kernel=7)
+
+
+# ------------------------------------------- dense/sparse hybrid (NEXT-1)
+def test_sparse_dense_hybrid(torch_cuda):
+    """Groups with few tests go to the thread-per-query kernel, the rest to the
+    warp-per-group kernels, in one call: sparse-dominated (SDSS-like at small
+    eps), mixed (dense square in sparse background) and dense-dominated data
+    give the oracle's table, host- and device-resident, f64 and f32, the same
+    as with the split disabled (search_kernel 3)."""
+    cases = [(datagen.subsample(datagen.sdss_like(datagen.C3_N_LARGE, seed=4), 60_000, seed=3), 0.07 * 4),
+             (datagen.dense_skew(40_000, seed=9), 2.0),
+             (datagen.subsample(datagen.tec_like(), 40_000, seed=5), 0.45)]
+    saw_mixed = False
+    for xy, eps in cases:
+        for dtype in ("f64", "f32"):
+            x = xy.astype(np.float32) if dtype == "f32" else xy
+            for device in (False, True):
+                b, c, v, view, st = lib_table(x, eps, device=device)
+                assert_table_equal(x, eps, b, c, v, dtype)
+                saw_mixed |= 0 < st["n_sparse_queries"] < x.shape[0]
+            b3, c3, v3, _, st3 = lib_table(x, eps, device=True, search_kernel=3)
+            assert st3["n_sparse_queries"] == 0
+            assert np.array_equal(c3, c)
+    assert saw_mixed
+
+
+def test_sparse_batches_and_shards(torch_cuda):
+    """The sparse queries of a group range follow the range: many small batches
+    (host table) and process shards give the oracle's table."""
+    xy = datagen.dense_skew(40_000, seed=9)
+    P = int(oracle.eps_join(xy, 2.0)[0][-1])
+    b, c, v, view, st = lib_table(xy, 2.0, batch_pairs=P // 40 + 1, n_streams=3)
+    assert st["n_batches"] > 10 and st["n_sparse_queries"] > 0
+    assert_table_equal(xy, 2.0, b, c, v)
+    off, nbr = oracle.eps_join(xy, 2.0)
+    want = np.diff(off.astype(np.int64))
+    got = np.zeros(xy.shape[0], np.int64)
+    for r in range(3):
+        b, c, v, view, st = lib_table(xy, 2.0, device=True, shard_rank=r, shard_count=3)
+        got += c.astype(np.int64)
+    assert np.array_equal(got, want)
