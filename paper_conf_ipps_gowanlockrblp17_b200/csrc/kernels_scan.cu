@@ -1,8 +1,8 @@
 // kernels_scan.cu -- device exclusive scans (SURVEY 8(a) a4 cell offsets, a7
-// neighbour-list offsets).  Reduce-then-scan over 2048-element tiles; inside a
-// tile every thread scans 8 consecutive items serially, the warp combines its
-// lanes with __shfl_up_sync and the CTA combines its 8 warp totals.  Block
-// sums are scanned recursively, in place.  out[n] receives the total.
+// neighbour-list offsets).  One pass over 2048-element tiles; inside a tile
+// every thread scans 8 consecutive items serially, the warp combines its lanes
+// with __shfl_up_sync and the CTA combines its 8 warp totals; tiles chain their
+// prefixes by decoupled look-back.  out[n] receives the total.
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -19,38 +19,33 @@ constexpr int SC_THREADS = 256;
 constexpr int SC_ITEMS = 8;
 constexpr int SC_TILE = SC_THREADS * SC_ITEMS;
 
-template <typename Tin, typename Tacc>
-__global__ void __launch_bounds__(SC_THREADS) k_tile_reduce(const Tin* __restrict__ in, uint64_t n,
-                                                            Tacc* __restrict__ sums) {
-    __shared__ Tacc ws[SC_THREADS / 32];
-    const uint64_t base = (uint64_t)blockIdx.x * SC_TILE;
-    Tacc acc = 0;
-#pragma unroll
-    for (int i = 0; i < SC_ITEMS; ++i) {
-        uint64_t idx = base + (uint64_t)i * SC_THREADS + threadIdx.x;
-        if (idx < n) acc += (Tacc)in[idx];
-    }
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(FULL, acc, o);
-    if ((threadIdx.x & 31) == 0) ws[threadIdx.x >> 5] = acc;
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        Tacc t = 0;
-#pragma unroll
-        for (int w = 0; w < SC_THREADS / 32; ++w) t += ws[w];
-        sums[blockIdx.x] = t;
-    }
+// Single-pass scan with decoupled look-back (Merrill & Garland 2016): tile t
+// publishes its aggregate, then its inclusive prefix once known, as one packed
+// 64-bit word {status:2, value:62}; a tile finds its exclusive prefix by walking
+// back over its predecessors' words, 32 at a time (one per lane of warp 0),
+// summing aggregates until it meets an inclusive prefix.  Tiles are blockIdx
+// ordered and only wait on lower tiles, which the hardware dispatched first.
+// One kernel per scan (plus a memset of the tile words).
+constexpr uint64_t kStAgg = 1ull << 62, kStPre = 2ull << 62, kValMask = (1ull << 62) - 1;
+
+__device__ __forceinline__ void publish(unsigned long long* w, uint64_t v) {
+    asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(w), "l"(v) : "memory");
+}
+__device__ __forceinline__ uint64_t peek(const unsigned long long* w) {
+    uint64_t v;
+    asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(w) : "memory");
+    return v;
 }
 
-// Exclusive scan of one tile; thread t owns items [t*ITEMS, (t+1)*ITEMS) of the
-// tile (blocked arrangement, loaded through shared memory for coalescing).
 template <typename Tin, typename Tout>
-__global__ void __launch_bounds__(SC_THREADS) k_tile_scan(const Tin* __restrict__ in, Tout* __restrict__ out,
-                                                          uint64_t n, const Tout* __restrict__ offs) {
+__global__ void __launch_bounds__(SC_THREADS) k_scan_lookback(const Tin* __restrict__ in, Tout* __restrict__ out,
+                                                              uint64_t n, unsigned long long* __restrict__ tiles) {
     __shared__ Tout buf[SC_TILE];
     __shared__ Tout wsum[SC_THREADS / 32];
+    __shared__ Tout s_excl;
     const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
-    const uint64_t base = (uint64_t)blockIdx.x * SC_TILE;
+    const uint64_t t = blockIdx.x;
+    const uint64_t base = t * SC_TILE;
 #pragma unroll
     for (int i = 0; i < SC_ITEMS; ++i) {
         uint64_t idx = base + (uint64_t)i * SC_THREADS + tid;
@@ -64,7 +59,6 @@ __global__ void __launch_bounds__(SC_THREADS) k_tile_scan(const Tin* __restrict_
         v[i] = run;
         run += buf[tid * SC_ITEMS + i];
     }
-    // warp inclusive scan of per-thread totals
     Tout incl = run;
 #pragma unroll
     for (int o = 1; o < 32; o <<= 1) {
@@ -73,16 +67,41 @@ __global__ void __launch_bounds__(SC_THREADS) k_tile_scan(const Tin* __restrict_
     }
     if (lane == 31) wsum[w] = incl;
     __syncthreads();
-    Tout wpre = 0;
-    Tout tot = 0;
+    Tout wpre = 0, tot = 0;
 #pragma unroll
     for (int i = 0; i < SC_THREADS / 32; ++i) {
-        Tout t = wsum[i];
-        wpre += (i < w) ? t : (Tout)0;
-        tot += t;
+        Tout x = wsum[i];
+        wpre += (i < w) ? x : (Tout)0;
+        tot += x;
     }
-    const Tout boff = offs ? offs[blockIdx.x] : (Tout)0;
-    const Tout pre = boff + wpre + (incl - run);
+    if (w == 0) {
+        Tout excl = 0;
+        if (t == 0) {
+            if (lane == 0 && tiles) publish(&tiles[0], kStPre | (uint64_t)tot);
+        } else {
+            if (lane == 0) publish(&tiles[t], kStAgg | (uint64_t)tot);
+            int64_t pred = (int64_t)t - 1;
+            while (true) {
+                const int64_t j = pred - lane;
+                uint64_t word = j >= 0 ? peek(&tiles[j]) : kStPre;   // before tile 0: prefix 0
+                while (__any_sync(FULL, (word >> 62) == 0)) {          // wait for every predecessor in view
+                    if ((word >> 62) == 0) word = peek(&tiles[j]);
+                }
+                const unsigned pre = __ballot_sync(FULL, (word >> 62) == 2);
+                const int first = pre ? __ffs(pre) - 1 : 32;           // nearest inclusive prefix
+                Tout val = lane <= first ? (Tout)(word & kValMask) : (Tout)0;
+#pragma unroll
+                for (int o = 16; o > 0; o >>= 1) val += __shfl_xor_sync(FULL, val, o);
+                excl += val;
+                if (pre) break;
+                pred -= 32;
+            }
+            if (lane == 0) publish(&tiles[t], kStPre | (uint64_t)(excl + tot));
+        }
+        if (lane == 0) s_excl = excl;
+    }
+    __syncthreads();
+    const Tout pre = s_excl + wpre + (incl - run);
 #pragma unroll
     for (int i = 0; i < SC_ITEMS; ++i) buf[tid * SC_ITEMS + i] = pre + v[i];
     __syncthreads();
@@ -91,48 +110,37 @@ __global__ void __launch_bounds__(SC_THREADS) k_tile_scan(const Tin* __restrict_
         uint64_t idx = base + (uint64_t)i * SC_THREADS + tid;
         if (idx < n) out[idx] = buf[i * SC_THREADS + tid];
     }
-    if (tid == 0 && base + SC_TILE >= n) out[n] = boff + tot;   // last tile writes the total
+    if (tid == 0 && base + SC_TILE >= n) out[n] = s_excl + tot;   // last tile writes the total
 }
 
 template <typename Tin, typename Tout>
-void scan_rec(const Tin* in, Tout* out, uint64_t n, Tout* temp, cudaStream_t s) {
+void scan_impl(const Tin* in, Tout* out, uint64_t n, void* temp, cudaStream_t s) {
     if (n == 0) {
         cudaMemsetAsync(out, 0, sizeof(Tout), s);
         return;
     }
-    uint64_t nb = (n + SC_TILE - 1) / SC_TILE;
-    if (nb == 1) {
-        k_tile_scan<Tin, Tout><<<1, SC_THREADS, 0, s>>>(in, out, n, nullptr);
-        ++g_kernel_launches;
-        return;
+    const uint64_t nb = (n + SC_TILE - 1) / SC_TILE;
+    unsigned long long* tiles = nullptr;
+    if (nb > 1) {
+        tiles = (unsigned long long*)temp;
+        cudaMemsetAsync(tiles, 0, nb * sizeof(unsigned long long), s);
     }
-    Tout* sums = temp;                 // nb + 1 entries
-    Tout* next = temp + (nb + 1);
-    k_tile_reduce<Tin, Tout><<<(unsigned)nb, SC_THREADS, 0, s>>>(in, n, sums);
-    ++g_kernel_launches;
-    scan_rec<Tout, Tout>(sums, sums, nb, next, s);   // in place
-    k_tile_scan<Tin, Tout><<<(unsigned)nb, SC_THREADS, 0, s>>>(in, out, n, sums);
+    k_scan_lookback<Tin, Tout><<<(unsigned)nb, SC_THREADS, 0, s>>>(in, out, n, tiles);
     ++g_kernel_launches;
 }
 
 }  // namespace
 
 size_t scan_temp_bytes(uint64_t n) {
-    size_t total = 0;
-    while (n > (uint64_t)SC_TILE) {
-        uint64_t nb = (n + SC_TILE - 1) / SC_TILE;
-        total += (nb + 1) * sizeof(uint64_t);
-        n = nb;
-    }
-    return total + 64;
+    return ((n + SC_TILE - 1) / SC_TILE + 1) * sizeof(unsigned long long) + 64;
 }
 
 void scan_u32_to_u32(const uint32_t* in, uint32_t* out, uint64_t n, void* temp, cudaStream_t s) {
-    scan_rec<uint32_t, uint32_t>(in, out, n, (uint32_t*)temp, s);
+    scan_impl<uint32_t, uint32_t>(in, out, n, temp, s);
 }
 
 void scan_u32_to_u64(const uint32_t* in, uint64_t* out, uint64_t n, void* temp, cudaStream_t s) {
-    scan_rec<uint32_t, uint64_t>(in, out, n, (uint64_t*)temp, s);
+    scan_impl<uint32_t, uint64_t>(in, out, n, temp, s);
 }
 
 }  // namespace hdb

@@ -837,14 +837,17 @@ __global__ void __launch_bounds__(256) k_sample_count(SArgs a, uint64_t nne, uin
     unsigned long long tot = 0;
     for (uint64_t j = wid; j < ns; j += nw) {
         const uint64_t s = j * stride;
-        // cell of sorted position s: last c with cstart[c] <= s
+        // cell of sorted position s: last c with cstart[c] <= s, by a 32-way warp search
+        // (invariant cstart[lo] <= s < cstart[hi]; ~log32 steps of one load per lane)
         uint64_t lo = 0, hi = nne;
         while (hi - lo > 1) {
-            uint64_t mid = (lo + hi) >> 1;
-            if (__ldg(&a.cstart[mid]) <= s)
-                lo = mid;
-            else
-                hi = mid;
+            const uint64_t step = (hi - lo + 31) / 32;
+            const uint64_t idx = lo + (uint64_t)lane * step;
+            const bool le = idx < hi && __ldg(&a.cstart[idx]) <= s;
+            const uint32_t m = __popc(__ballot_sync(FULL, le));   // >= 1: lane 0 reads cstart[lo]
+            const uint64_t nlo = lo + (uint64_t)(m - 1) * step;
+            hi = min(hi, nlo + step);
+            lo = nlo;
         }
         const uint64_t c = lo;
         uint32_t cntv = 0;
