@@ -561,7 +561,7 @@ __device__ __forceinline__ void emit_group(const SArgs& a, uint32_t c, uint32_t 
                                            uint2 (*raw)[kWin + 2], uint4 (*wq)[kWin + 1], VSpan* vsp, int lane) {
     const unsigned lt = (1u << lane) - 1u, lbit = 1u << lane;
     // the group's spans as one sequence of candidate pairs (same chunks as the count pass)
-    load_vspans(a, c, vsp, lane);
+    const uint32_t nch = (load_vspans(a, c, vsp, lane) + 31) / 32;
     uint32_t rs = 0;   // this lane's current span
     __syncwarp();   // the previous group's buffers are no longer read
     if ((uint32_t)lane < nq) {   // prefetch window 0: lane i copies its 64-B mask row
@@ -602,13 +602,31 @@ __device__ __forceinline__ void emit_group(const SArgs& a, uint32_t c, uint32_t 
             for (int u = 0; u < kWin / 2; ++u) cp_async16(&raw[lane][2 * u], src + u);
         }
         cp_async_commit();
+        // chunks of this window (the last window of a group is usually partial: short
+        // groups, e.g. ~100-400 candidates on C5, have 2-7 of the 8 chunks -- emitting the
+        // empty ones cost ~6 instructions per half-chunk and query)
+        const uint32_t nck = min((uint32_t)kWin, nch - v * kWin);
+        if (nck == kWin) {
 #pragma unroll 1
-        for (uint32_t i = 0; i < nq; ++i) {
+            for (uint32_t i = 0; i < nq; ++i) {
 #pragma unroll
-            for (int kk = 0; kk < kWin; ++kk) {
-                const uint4 e = wq[i][kk];   // broadcast
-                stg_if_bit(gout + (e.z + __popc(e.x & lt)), ids[kk].x, e.x, lbit);
-                stg_if_bit(gout + (e.w + __popc(e.y & lt)), ids[kk].y, e.y, lbit);
+                for (int kk = 0; kk < kWin; ++kk) {
+                    const uint4 e = wq[i][kk];   // broadcast
+                    stg_if_bit(gout + (e.z + __popc(e.x & lt)), ids[kk].x, e.x, lbit);
+                    stg_if_bit(gout + (e.w + __popc(e.y & lt)), ids[kk].y, e.y, lbit);
+                }
+            }
+        } else {
+#pragma unroll 1
+            for (uint32_t i = 0; i < nq; ++i) {
+#pragma unroll
+                for (int kk = 0; kk < kWin; ++kk) {
+                    if ((uint32_t)kk < nck) {
+                        const uint4 e = wq[i][kk];
+                        stg_if_bit(gout + (e.z + __popc(e.x & lt)), ids[kk].x, e.x, lbit);
+                        stg_if_bit(gout + (e.w + __popc(e.y & lt)), ids[kk].y, e.y, lbit);
+                    }
+                }
             }
         }
         __syncwarp();   // wq is rewritten for the next window
