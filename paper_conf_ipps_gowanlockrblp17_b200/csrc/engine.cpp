@@ -694,6 +694,7 @@ void count_phase(hdb_ctx* ctx, DevCtx& dc, const DevGrid& g, ShardState& st) {
             cudaGetLastError();
         }
     }
+    tr.mark("alloc");
     Event e0, e1, e2;
     HDB_CUDA(cudaEventRecord(e0.e, s));
     launch_count(g, st.r.g0, st.r.g1, st.cnt.as<uint32_t>(), tests.as<unsigned long long>(), ctx->opts.search_kernel,
@@ -701,6 +702,7 @@ void count_phase(hdb_ctx* ctx, DevCtx& dc, const DevGrid& g, ShardState& st) {
     HDB_LAUNCH_CHECK();
     HDB_CUDA(cudaEventRecord(e1.e, s));
     const uint64_t len = st.r.q1 - st.r.q0;
+    tr.mark("count-enqueue");
     DBuf temp(scan_temp_bytes(len + 1), s);
     scan_u32_to_u64(st.cnt.as<uint32_t>() + st.r.q0, st.off.as<uint64_t>() + st.r.q0, len, temp.p, s);
     HDB_LAUNCH_CHECK();
@@ -1154,7 +1156,7 @@ void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hd
                              st.mask_base, s);
                 HDB_LAUNCH_CHECK();
                 HDB_CUDA(cudaEventRecord(e1.e, s));
-                launch_scatter_rows(g.ids, st.off.as<uint64_t>(), st.cnt.as<uint32_t>(), st.r.q0, st.r.q1, 0,
+                launch_scatter_rows(g.ids, g.n, st.off.as<uint64_t>(), st.cnt.as<uint32_t>(), st.r.q0, st.r.q1, 0,
                                     beg.as<uint64_t>(), cnt.as<uint32_t>(), s);
                 HDB_LAUNCH_CHECK();
                 HDB_CUDA(cudaStreamSynchronize(s));
@@ -1196,7 +1198,7 @@ void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hd
                     DeviceGuard dg(dc.device);
                     cudaStream_t s = dc.main;
                     DBuf beg(8 * (n ? n : 1), s), cnt(4 * (n ? n : 1), s);
-                    launch_scatter_rows(grid->dev[0].ids, sh[0].off.as<uint64_t>(), sh[0].cnt.as<uint32_t>(), 0, n, 0,
+                    launch_scatter_rows(grid->dev[0].ids, n, sh[0].off.as<uint64_t>(), sh[0].cnt.as<uint32_t>(), 0, n, 0,
                                         beg.as<uint64_t>(), cnt.as<uint32_t>(), s);
                     HDB_LAUNCH_CHECK();
                     if (n) {

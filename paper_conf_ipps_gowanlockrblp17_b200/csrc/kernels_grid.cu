@@ -526,8 +526,9 @@ size_t radix_sort_temp_bytes(uint64_t n) {
 }
 
 template <typename K>
-int radix_sort_impl(K* k0, uint32_t* v0, K* k1, uint32_t* v1, uint64_t n, int bits, void* temp, cudaStream_t s) {
-    if (n <= 1 || bits <= 0) return 0;
+int radix_sort_impl(K* k0, uint32_t* v0, K* k1, uint32_t* v1, uint64_t n, int bits, void* temp, cudaStream_t s,
+                    int shift0 = 0) {
+    if (n <= 1 || bits <= shift0) return 0;
     constexpr int TILE = RsCfg<K>::TILE;
     uint32_t nblocks = (uint32_t)((n + TILE - 1) / TILE);
     uint64_t m = (uint64_t)nblocks * RS_BINS;
@@ -535,7 +536,7 @@ int radix_sort_impl(K* k0, uint32_t* v0, K* k1, uint32_t* v1, uint64_t n, int bi
     uint32_t* hscan = hist + (m + 1);
     void* stemp = (void*)(((uintptr_t)(hscan + m + 1) + 255) & ~(uintptr_t)255);
     int cur = 0;
-    for (int shift = 0; shift < bits; shift += RS_BITS) {
+    for (int shift = shift0; shift < bits; shift += RS_BITS) {
         K* ki = cur ? k1 : k0;
         uint32_t* vi = cur ? v1 : v0;
         K* ko = cur ? k0 : k1;
@@ -548,6 +549,11 @@ int radix_sort_impl(K* k0, uint32_t* v0, K* k1, uint32_t* v1, uint64_t n, int bi
         cur ^= 1;
     }
     return cur;
+}
+
+int radix_sort_u32_digits(uint32_t* k0, uint32_t* v0, uint32_t* k1, uint32_t* v1, uint64_t n, int shift0, int bits,
+                          void* temp, cudaStream_t s) {
+    return radix_sort_impl<uint32_t>(k0, v0, k1, v1, n, bits, temp, s, shift0);
 }
 
 int radix_sort_pairs(void* k0, uint32_t* v0, void* k1, uint32_t* v1, int key_bytes, uint64_t n, int bits, void* temp,

@@ -626,3 +626,20 @@ def test_sparse_batches_and_shards(torch_cuda):
         b, c, v, view, st = lib_table(xy, 2.0, device=True, shard_rank=r, shard_count=3)
         got += c.astype(np.int64)
     assert np.array_equal(got, want)
+
+
+def test_c3_large_bucketed_row_scatter(torch_cuda):
+    """5,000,000 points (C3L, SDSS2-size): the by-id row scatter takes the
+    bucketed path (>= 2^22 rows) -- rows must tile the value array exactly and
+    sampled rows equal the oracle's, device- and host-resident."""
+    xy = datagen.sdss_like(datagen.C3_N_LARGE, seed=4)
+    for device in (True, False):
+        b, c, v, view, st = lib_table(xy, 0.07, device=device)
+        order = np.argsort(b)
+        bs, cs = b[order].astype(np.int64), c[order].astype(np.int64)
+        assert bs[0] == 0 and np.array_equal(bs[1:], bs[:-1] + cs[:-1]) and bs[-1] + cs[-1] == view.npairs
+        rng = np.random.default_rng(17)
+        rows = np.unique(np.concatenate([rng.choice(xy.shape[0], 1000, replace=False), np.argsort(c)[-20:]]))
+        roff, rnbr = oracle.eps_join_rows(xy, 0.07, rows)
+        for i, p in enumerate(rows):
+            assert np.array_equal(np.sort(v[b[p]:b[p] + c[p]]), rnbr[roff[i]:roff[i + 1]]), p
