@@ -276,8 +276,37 @@ __device__ __forceinline__ uint32_t count_group(const SArgs& a, uint32_t qs, uin
         }
         tests += (unsigned long long)nq * ((v0 ? 1u : 0u) + (v1 ? 1u : 0u));   // per lane; reduced at exit
         uint32_t acc = 0;   // f64 filter: sign bit set <=> some |t| <= band in this lane
+        uint32_t i0 = 0;
+        if (MODE == kF64Filter) {
+            // four queries per step with their arithmetic issued before any ballot: the
+            // ballots are warp-synchronous points the compiler does not schedule across, so
+            // one query at a time left each FADD2 -> FFMA2 -> FFMA2 -> FSETP chain exposed
+#pragma unroll 1
+            for (; i0 + 4 <= nq; i0 += 4) {
+                u64x tt[4];
+#pragma unroll
+                for (int j = 0; j < 4; ++j) {
+                    const ulonglong2 Q = sq[i0 + j];
+                    const u64x dx = sub2(Q.x, X);
+                    const u64x dy = sub2(Q.y, Y);
+                    tt[j] = fma2(dy, dy, fma2(dx, dx, NE2));   // (dx^2 - e2) + dy^2
+                }
+#pragma unroll
+                for (int j = 0; j < 4; ++j) {
+                    const float2 u = unpack2(fma2(tt[j], tt[j], NB2));   // t^2 - B^2 < 0  <=>  |t| < B
+                    acc |= __float_as_uint(u.x) | __float_as_uint(u.y);
+                }
+#pragma unroll
+                for (int j = 0; j < 4; ++j) {
+                    const float2 t = unpack2(tt[j]);
+                    const unsigned m0 = __ballot_sync(FULL, t.x < 0.f);
+                    const unsigned m1 = __ballot_sync(FULL, t.y < 0.f);
+                    if (lane == 0) swin[i0 + j][kk] = make_uint2(m0, m1);
+                }
+            }
+        }
 #pragma unroll 4
-        for (uint32_t i = 0; i < nq; ++i) {
+        for (uint32_t i = i0; i < nq; ++i) {
             unsigned m0, m1;
             if (MODE == kF64Exact) {
                 const double2 qd = sqd[i];
