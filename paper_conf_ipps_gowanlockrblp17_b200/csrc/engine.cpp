@@ -493,33 +493,30 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
     g.gstart = (uint32_t*)gstart.release();
     g.gcell = (uint32_t*)gcell.release();
     // dense/sparse hybrid (NEXT-1): groups with few tests take the thread-per-query
-    // kernel; search_kernel 3 / 4 (and the paper's kernels) keep one path for all groups
+    // kernel; search_kernel 3 / 4 (and the paper's kernels) keep one path for all groups.
+    // The lists are built unconditionally and adopted after the final sync only if a
+    // good share of the queries is sparse (no extra host sync); the mask layout keeps
+    // words for every group either way.
     const int sk = ctx->opts.search_kernel;
     const uint32_t max_tests = sparse_max_tests();
-    if ((sk == 0 || sk == 1 || sk == 2) && max_tests > 0 && n > 0) {
+    const bool classify = (sk == 0 || sk == 1 || sk == 2) && max_tests > 0 && n > 0;
+    DBuf dpre, spre, dl, sql;
+    unsigned long long* nsp = bb + 8;
+    if (classify) {
         DBuf dflag(4 * (n + 1), s), sqn(4 * (n + 1), s);
-        DBuf dpre(4 * (n + 1), s), spre(4 * (n + 1), s), dl(4 * (n + 1), s), sql(8 * (n + 1), s);
+        dpre = DBuf(4 * (n + 1), s);
+        spre = DBuf(4 * (n + 1), s);
+        dl = DBuf(4 * (n + 1), s);
+        sql = DBuf(8 * (n + 1), s);
         const uint32_t* ngd = gofs.as<uint32_t>() + nne;
-        unsigned long long* nsp = bb + 8;
         HDB_CUDA(cudaMemsetAsync(nsp, 0, 8, s));
         launch_group_class(g.cstart, g.cspan, g.nspan, g.gstart, g.gcell, ngd, n, max_tests, dflag.as<uint32_t>(),
                            sqn.as<uint32_t>(), nsp, s);
+        scan_u32_to_u32(dflag.as<uint32_t>(), dpre.as<uint32_t>(), n, temp.p, s);
+        scan_u32_to_u32(sqn.as<uint32_t>(), spre.as<uint32_t>(), n, temp.p, s);
+        launch_group_lists(g.gstart, g.gcell, ngd, n, dpre.as<uint32_t>(), spre.as<uint32_t>(), dl.as<uint32_t>(),
+                           sql.as<uint2>(), s);
         HDB_LAUNCH_CHECK();
-        HDB_CUDA(cudaMemcpyAsync(dc.pin + 6, nsp, 8, cudaMemcpyDeviceToHost, s));
-        HDB_CUDA(cudaStreamSynchronize(s));
-        // the split pays only when a good share of the queries is sparse: the thread-per-query
-        // kernels run after the dense ones and a few sparse groups only add their latency
-        if ((double)dc.pin[6] >= kSparseMinShare * (double)n) {
-            scan_u32_to_u32(dflag.as<uint32_t>(), dpre.as<uint32_t>(), n, temp.p, s);
-            scan_u32_to_u32(sqn.as<uint32_t>(), spre.as<uint32_t>(), n, temp.p, s);
-            launch_group_lists(g.gstart, g.gcell, ngd, n, dpre.as<uint32_t>(), spre.as<uint32_t>(),
-                               dl.as<uint32_t>(), sql.as<uint2>(), s);
-            HDB_LAUNCH_CHECK();
-            g.dpre = (uint32_t*)dpre.release();
-            g.spre = (uint32_t*)spre.release();
-            g.dl = (uint32_t*)dl.release();
-            g.sql = (uint2*)sql.release();
-        }
     }
     {
         DBuf words(4 * (n + 1), s), mtemp(scan_temp_bytes(n + 1), s), moff(8 * (n + 1), s);
@@ -527,19 +524,31 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
         scan_u32_to_u64(words.as<uint32_t>(), moff.as<uint64_t>(), n, mtemp.p, s);
         HDB_LAUNCH_CHECK();
         uint32_t hng = 0;
+        uint32_t hds[2] = {0, 0};
+        uint64_t hsp = 0;
         HDB_CUDA(cudaMemcpyAsync(&hng, gofs.as<uint32_t>() + nne, 4, cudaMemcpyDeviceToHost, s));
         HDB_CUDA(cudaMemcpyAsync(&g.mask_words, moff.as<uint64_t>() + n, 8, cudaMemcpyDeviceToHost, s));
-        uint32_t hds[2] = {0, 0};
-        if (g.dl) {
-            HDB_CUDA(cudaMemcpyAsync(&hds[0], g.dpre + n, 4, cudaMemcpyDeviceToHost, s));
-            HDB_CUDA(cudaMemcpyAsync(&hds[1], g.spre + n, 4, cudaMemcpyDeviceToHost, s));
+        if (classify) {
+            HDB_CUDA(cudaMemcpyAsync(&hds[0], dpre.as<uint32_t>() + n, 4, cudaMemcpyDeviceToHost, s));
+            HDB_CUDA(cudaMemcpyAsync(&hds[1], spre.as<uint32_t>() + n, 4, cudaMemcpyDeviceToHost, s));
+            HDB_CUDA(cudaMemcpyAsync(&hsp, nsp, 8, cudaMemcpyDeviceToHost, s));
         }
         HDB_CUDA(cudaEventRecord(ev1.e, s));
         HDB_CUDA(cudaEventSynchronize(ev1.e));
         g.n_groups = hng;
         g.moff = (uint64_t*)moff.release();
-        g.n_dense_groups = g.dl ? hds[0] : hng;
-        g.n_sparse_q = hds[1];
+        g.n_dense_groups = hng;
+        g.n_sparse_q = 0;
+        // the split pays only when a good share of the queries is sparse: the thread-per-query
+        // kernels run after the dense ones and a few sparse groups only add their latency
+        if (classify && (double)hsp >= kSparseMinShare * (double)n) {
+            g.dpre = (uint32_t*)dpre.release();
+            g.spre = (uint32_t*)spre.release();
+            g.dl = (uint32_t*)dl.release();
+            g.sql = (uint2*)sql.release();
+            g.n_dense_groups = hds[0];
+            g.n_sparse_q = hds[1];
+        }
     }
     g.ms_build = elapsed(ev0, ev1);
     gcount.reset();

@@ -304,6 +304,28 @@ __device__ __forceinline__ uint32_t count_group(const SArgs& a, uint32_t qs, uin
                     if (lane == 0) swin[i0 + j][kk] = make_uint2(m0, m1);
                 }
             }
+        } else if (MODE == kF32) {
+#pragma unroll 1
+            for (; i0 + 4 <= nq; i0 += 4) {
+                bool h0[4], h1[4];
+#pragma unroll
+                for (int j = 0; j < 4; ++j) {
+                    const ulonglong2 Q = sq[i0 + j];
+                    const u64x dx = sub2(Q.x, X);
+                    const u64x dy = sub2(Q.y, Y);
+                    // exact f32: fl(fl(dx^2) + fl(dy^2)), scalar add.rn (reading R2)
+                    const float2 px = unpack2(mul2(dx, dx));
+                    const float2 py = unpack2(mul2(dy, dy));
+                    h0[j] = __fadd_rn(px.x, py.x) <= a.e2f;
+                    h1[j] = __fadd_rn(px.y, py.y) <= a.e2f;
+                }
+#pragma unroll
+                for (int j = 0; j < 4; ++j) {
+                    const unsigned m0 = __ballot_sync(FULL, h0[j]);
+                    const unsigned m1 = __ballot_sync(FULL, h1[j]);
+                    if (lane == 0) swin[i0 + j][kk] = make_uint2(m0, m1);
+                }
+            }
         }
 #pragma unroll 4
         for (uint32_t i = i0; i < nq; ++i) {
