@@ -119,11 +119,12 @@ def cpu_baseline_run(xy, eps, budget_s=12.0, rows=None, dtype="f64"):
     n = xy.shape[0]
     if rows is None:
         # calibrate on a small sample, then size the sample to ~budget_s
-        probe = np.arange(0, n, max(1, n // 64))[:64]
+        probe = np.linspace(0, n - 1, min(n, 512)).astype(np.int64)
+        oracle.eps_join_rowhash(xy, eps, probe[:8], dtype=dtype)   # warm (thread pool, pages)
         t0 = time.perf_counter()
         oracle.eps_join_rowhash(xy, eps, probe, dtype=dtype)
         dt = max(time.perf_counter() - t0, 1e-3)
-        m = int(min(n, max(64, 64 * budget_s / dt)))
+        m = int(min(n, max(probe.size, probe.size * budget_s / dt)))
         rows = np.linspace(0, n - 1, m).astype(np.int64)
     t0 = time.perf_counter()
     cnt, _ = oracle.eps_join_rowhash(xy, eps, rows, dtype=dtype)
@@ -159,9 +160,20 @@ def cpu_gridjoin_run(xy, eps, dtype="f64", budget_s=4.0):
     return out
 
 
+def all_host_cores():
+    """The reference arm runs on rank 0 alone: give the oracle's OpenMP every host
+    core (torchrun exports OMP_NUM_THREADS=1 to each rank); set before liboracle loads."""
+    try:
+        cores = len(os.sched_getaffinity(0))
+    except Exception:
+        cores = os.cpu_count() or 1
+    os.environ["OMP_NUM_THREADS"] = str(cores)
+
+
 def run_reference(args, wl, ws, rank):
     if rank != 0:
         return
+    all_host_cores()
     xy = wl["gen"]()
     K, W = args.steps, args.warmup
     res, rows = cpu_baseline_run(xy, wl["eps"], budget_s=max(2.0, 60.0 / max(K + W, 1)))
@@ -200,6 +212,7 @@ def run_sweep(args, wl, ws, rank, local):
     if args.impl == "reference":
         if rank != 0:
             return
+        all_host_cores()
         # the oracle as it stands: brute-force rows (sampled) + Alg. 1 would need
         # the full table; time the brute-force join on a bounded row sample per eps
         K, W = args.steps, args.warmup
