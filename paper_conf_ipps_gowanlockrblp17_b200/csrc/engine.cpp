@@ -500,10 +500,11 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
     const int sk = ctx->opts.search_kernel;
     const uint32_t max_tests = sparse_max_tests();
     const bool classify = (sk == 0 || sk == 1 || sk == 2) && max_tests > 0 && n > 0;
-    DBuf dpre, spre, dl, sql;
+    DBuf dpre, spre, dl, sql, ord;
     unsigned long long* nsp = bb + 8;
     if (classify) {
-        DBuf dflag(4 * (n + 1), s), sqn(4 * (n + 1), s);
+        DBuf dflag(4 * (n + 1), s), sqn(4 * (n + 1), s), gbin(n + 1, s), ohist(8 * kOrderBins, s);
+        ord = DBuf(4 * (n + 1), s);
         dpre = DBuf(4 * (n + 1), s);
         spre = DBuf(4 * (n + 1), s);
         dl = DBuf(4 * (n + 1), s);
@@ -511,7 +512,8 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
         const uint32_t* ngd = gofs.as<uint32_t>() + nne;
         HDB_CUDA(cudaMemsetAsync(nsp, 0, 8, s));
         launch_group_class(g.cstart, g.cspan, g.nspan, g.gstart, g.gcell, ngd, n, max_tests, dflag.as<uint32_t>(),
-                           sqn.as<uint32_t>(), nsp, s);
+                           sqn.as<uint32_t>(), nsp, (uint8_t*)gbin.p, ohist.as<uint32_t>(), s);
+        launch_order_scatter((const uint8_t*)gbin.p, ngd, n, ohist.as<uint32_t>(), ord.as<uint32_t>(), s);
         scan_u32_to_u32(dflag.as<uint32_t>(), dpre.as<uint32_t>(), n, temp.p, s);
         scan_u32_to_u32(sqn.as<uint32_t>(), spre.as<uint32_t>(), n, temp.p, s);
         launch_group_lists(g.gstart, g.gcell, ngd, n, dpre.as<uint32_t>(), spre.as<uint32_t>(), dl.as<uint32_t>(),
@@ -539,6 +541,7 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
         g.moff = (uint64_t*)moff.release();
         g.n_dense_groups = hng;
         g.n_sparse_q = 0;
+        if (classify) g.ord = (uint32_t*)ord.release();
         // the split pays only when a good share of the queries is sparse: the thread-per-query
         // kernels run after the dense ones and a few sparse groups only add their latency
         if (classify && (double)hsp >= kSparseMinShare * (double)n) {
@@ -563,14 +566,14 @@ void free_dev_grid(DevGrid& g) {
     DeviceGuard dg(g.device);
     for (void* p : {(void*)g.xy_s, (void*)g.xp, (void*)g.counters, (void*)g.ids, (void*)g.ckey, (void*)g.cstart,
                     (void*)g.cspan, (void*)g.gstart, (void*)g.gcell, (void*)g.moff, (void*)g.dpre, (void*)g.spre,
-                    (void*)g.dl, (void*)g.sql})
+                    (void*)g.dl, (void*)g.sql, (void*)g.ord})
         if (p) cudaFreeAsync(p, g.stream);   // stream-ordered: no host sync needed
     g.xy_s = nullptr;
     g.xp = nullptr;
     g.counters = nullptr;
     g.ids = g.cstart = g.gstart = g.gcell = nullptr;
     g.moff = nullptr;
-    g.dpre = g.spre = g.dl = nullptr;
+    g.dpre = g.spre = g.dl = g.ord = nullptr;
     g.sql = nullptr;
     g.ckey = nullptr;
     g.cspan = nullptr;

@@ -76,6 +76,8 @@ struct DevGrid {
     // dense/sparse hybrid (NEXT-1): null when every group takes the warp-per-group path
     uint32_t* dpre = nullptr;      // [n_groups+1] dense groups before g
     uint32_t* dl = nullptr;        // [#dense] the dense groups, ascending
+    uint32_t* ord = nullptr;       // [n_groups] cost order: dense groups heaviest first, then the sparse
+                                   // ones (whole-range count / write launches visit groups in this order)
     uint32_t* spre = nullptr;      // [n_groups+1] sparse queries before group g
     uint2* sql = nullptr;          // [n_sparse_q] {sorted position, non-empty cell} of each sparse query
     uint64_t n_sparse_q = 0, n_dense_groups = 0;
@@ -124,7 +126,13 @@ void launch_group_build(const uint32_t* cstart, const uint32_t* gofs, uint64_t n
 // sql[spre[g] + i] = {gstart[g] + i, gcell[g]}
 void launch_group_class(const uint32_t* cstart, const uint2* cspan, uint32_t nspan, const uint32_t* gstart,
                         const uint32_t* gcell, const uint32_t* ng_dev, uint64_t n, uint32_t max_tests,
-                        uint32_t* dflag, uint32_t* sqn, unsigned long long* n_sparse, cudaStream_t s);
+                        uint32_t* dflag, uint32_t* sqn, unsigned long long* n_sparse, uint8_t* gbin,
+                        uint32_t* ohist, cudaStream_t s);
+// cost order: ord = the groups by gbin (dense groups first, heaviest first); ohist holds
+// 2 * kOrderBins words (bin sizes from launch_group_class, then cursors)
+constexpr int kOrderBins = 64;
+void launch_order_scatter(const uint8_t* gbin, const uint32_t* ng_dev, uint64_t n, uint32_t* ohist, uint32_t* ord,
+                          cudaStream_t s);
 void launch_group_lists(const uint32_t* gstart, const uint32_t* gcell, const uint32_t* ng_dev, uint64_t n,
                         const uint32_t* dpre, const uint32_t* spre, uint32_t* dl, uint2* sql, cudaStream_t s);
 

@@ -372,7 +372,11 @@ __global__ void __launch_bounds__(256) k_group_class(const uint32_t* __restrict_
                                                      const uint32_t* __restrict__ ng_dev, uint64_t n,
                                                      uint32_t max_tests, uint32_t* __restrict__ dflag,
                                                      uint32_t* __restrict__ sqn,
-                                                     unsigned long long* __restrict__ n_sparse) {
+                                                     unsigned long long* __restrict__ n_sparse,
+                                                     uint8_t* __restrict__ gbin, uint32_t* __restrict__ ohist) {
+    __shared__ uint32_t sh[kOrderBins];
+    for (int b = threadIdx.x; b < kOrderBins; b += blockDim.x) sh[b] = 0;
+    __syncthreads();
     const uint64_t ng = *ng_dev;
     uint32_t tot = 0;
     for (uint64_t g = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; g < n; g += (uint64_t)gridDim.x * blockDim.x) {
@@ -385,8 +389,14 @@ __global__ void __launch_bounds__(256) k_group_class(const uint32_t* __restrict_
                 const uint2 sp = cspan[(uint64_t)nspan * c + r];
                 cand += sp.y - sp.x;
             }
-            if ((uint64_t)nq * cand <= max_tests) sq = nq;
+            const uint64_t tests = (uint64_t)nq * cand;
+            if (tests <= max_tests) sq = nq;
             else d = 1;
+            // cost bin: dense groups first, each class by decreasing log2(tests)
+            const uint32_t lg = 63 - __clzll(tests | 1);
+            const uint32_t b = (d ? 0u : kOrderBins / 2) + (kOrderBins / 2 - 1 - min(lg, (uint32_t)kOrderBins / 2 - 1));
+            gbin[g] = (uint8_t)b;
+            atomicAdd(&sh[b], 1u);
         }
         dflag[g] = d;
         sqn[g] = sq;
@@ -394,6 +404,45 @@ __global__ void __launch_bounds__(256) k_group_class(const uint32_t* __restrict_
     }
     for (int o = 16; o > 0; o >>= 1) tot += __shfl_xor_sync(0xffffffffu, tot, o);
     if ((threadIdx.x & 31) == 0 && tot) atomicAdd(n_sparse, (unsigned long long)tot);
+    __syncthreads();
+    for (int b = threadIdx.x; b < kOrderBins; b += blockDim.x)
+        if (sh[b]) atomicAdd(&ohist[b], sh[b]);
+}
+
+// Cost order: ord = the groups sorted by gbin (a counting
+// sort; order inside a bin is arbitrary -- results do not depend on the visiting
+// order, only the tail of the dynamic schedule does).  ohist[0..kOrderBins) are
+// the bin sizes, ocur[kOrderBins] zeroed cursors.  Tiles of 256 groups per block
+// step: block-local ranks by shared atomics, one global atomic per bin and tile.
+__global__ void __launch_bounds__(256) k_order_scatter(const uint8_t* __restrict__ gbin,
+                                                       const uint32_t* __restrict__ ng_dev, uint64_t n,
+                                                       const uint32_t* __restrict__ ohist,
+                                                       uint32_t* __restrict__ ocur, uint32_t* __restrict__ ord) {
+    __shared__ uint32_t base[kOrderBins], cnt[kOrderBins], at[kOrderBins];
+    const uint64_t ng = *ng_dev;
+    if (threadIdx.x == 0) {
+        uint32_t acc = 0;
+        for (int b = 0; b < kOrderBins; ++b) {
+            base[b] = acc;
+            acc += ohist[b];
+        }
+    }
+    for (uint64_t t0 = (uint64_t)blockIdx.x * blockDim.x; t0 < ng; t0 += (uint64_t)gridDim.x * blockDim.x) {
+        for (int b = threadIdx.x; b < kOrderBins; b += blockDim.x) cnt[b] = 0;
+        __syncthreads();
+        const uint64_t g = t0 + threadIdx.x;
+        uint32_t b = 0, r = 0;
+        if (g < ng) {
+            b = gbin[g];
+            r = atomicAdd(&cnt[b], 1u);
+        }
+        __syncthreads();
+        for (int k = threadIdx.x; k < kOrderBins; k += blockDim.x)
+            at[k] = cnt[k] ? atomicAdd(&ocur[k], cnt[k]) : 0;
+        __syncthreads();
+        if (g < ng) ord[base[b] + at[b] + r] = (uint32_t)g;
+        __syncthreads();
+    }
 }
 
 __global__ void __launch_bounds__(256) k_group_lists(const uint32_t* __restrict__ gstart,
@@ -612,10 +661,19 @@ void launch_group_build(const uint32_t* cstart, const uint32_t* gofs, uint64_t n
 
 void launch_group_class(const uint32_t* cstart, const uint2* cspan, uint32_t nspan, const uint32_t* gstart,
                         const uint32_t* gcell, const uint32_t* ng_dev, uint64_t n, uint32_t max_tests,
-                        uint32_t* dflag, uint32_t* sqn, unsigned long long* n_sparse, cudaStream_t s) {
+                        uint32_t* dflag, uint32_t* sqn, unsigned long long* n_sparse, uint8_t* gbin,
+                        uint32_t* ohist, cudaStream_t s) {
     if (n == 0) return;
+    cudaMemsetAsync(ohist, 0, 2 * kOrderBins * sizeof(uint32_t), s);
     k_group_class<<<grid_for(n), 256, 0, s>>>(cstart, cspan, nspan, gstart, gcell, ng_dev, n, max_tests, dflag, sqn,
-                                              n_sparse);
+                                              n_sparse, gbin, ohist);
+    ++g_kernel_launches;
+}
+
+void launch_order_scatter(const uint8_t* gbin, const uint32_t* ng_dev, uint64_t n, uint32_t* ohist, uint32_t* ord,
+                          cudaStream_t s) {
+    if (n == 0) return;
+    k_order_scatter<<<grid_for(n), 256, 0, s>>>(gbin, ng_dev, n, ohist, ohist + kOrderBins, ord);
     ++g_kernel_launches;
 }
 

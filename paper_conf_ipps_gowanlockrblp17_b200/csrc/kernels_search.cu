@@ -62,6 +62,9 @@ struct SArgs {
     // = {sorted position, cell} go to the thread-per-query kernel k_sparse
     const uint32_t* dl;
     const uint32_t* dpre;
+    // cost order (whole-range launches of the count / write pass): the dense groups, heaviest
+    // first (group ids; the first dpre[ng] entries when dl is set) -- DESIGN.md "cost order"
+    const uint32_t* ord;
     const uint2* sql;
     const uint32_t* spre;
 };
@@ -126,6 +129,73 @@ __device__ __forceinline__ uint32_t grab(unsigned int* ctr, uint32_t chunk, int 
     uint32_t v = 0;
     if (lane == 0) v = atomicAdd(ctr, chunk);
     return __shfl_sync(FULL, v, 0);
+}
+
+// Group feed with look-ahead (warp-per-group kernels).  Per group the warp
+// used to wait on a chain of dependent loads before its first useful
+// instruction -- the grab's atomic, then gstart / gcell / moff, then the spans
+// and offsets; ncu put ~20% of the write pass's stall samples there.  Here the
+// index stream runs two groups ahead (the next range's grab is issued one range
+// early, the group id behind an index -- through the cost order or the dense
+// list -- is loaded one group before its metadata) and the next group's level-1
+// metadata (qs, nq, c, mask-table offsets) is loaded while the current group
+// runs.  Holding reserved groups lengthens the tail only if the last groups are
+// heavy; a.ord (heavy groups first, built with the grid) makes them light.
+struct GMeta {
+    uint32_t qs, nq, c;
+    uint64_t ma, mb;   // mask-table words [ma, mb) (0 when moff is null)
+};
+__device__ __forceinline__ GMeta load_meta(const SArgs& a, const uint64_t* __restrict__ moff, uint32_t gi) {
+    GMeta m;
+    m.qs = __ldg(&a.gstart[gi]);
+    m.nq = __ldg(&a.gstart[gi + 1]) - m.qs;   // groups tile the sorted order: gstart[ng] = n
+    m.c = __ldg(&a.gcell[gi]);
+    m.ma = moff ? __ldg(&moff[gi]) : 0;
+    m.mb = moff ? __ldg(&moff[gi + 1]) : 0;
+    return m;
+}
+template <class F>
+__device__ __forceinline__ void for_each_group(const SArgs& a, const uint64_t* __restrict__ moff, uint32_t g0,
+                                               uint32_t g1, uint32_t chunk, unsigned int* ctr, int lane, F&& body) {
+    uint32_t i0 = g0, i1 = g1;
+    dense_range(a, i0, i1);
+    if (i1 <= i0) return;
+    uint32_t tk = 0;   // lane 0: the pending grab (start of the range after the newest one)
+    // the next index of the warp's stream after i (range end e); consumes the pending grab
+    auto advance = [&](uint32_t& i, uint32_t& e) {
+        uint32_t j = i + 1;
+        if (j >= e) {
+            j = i0 + __shfl_sync(FULL, tk, 0);
+            e = min(j + chunk, i1);
+            if (lane == 0 && j < i1) tk = atomicAdd(ctr, chunk);
+        }
+        i = j;
+    };
+    // group id of stream index i (clamped: look-ahead loads past the end stay in bounds)
+    auto gid = [&](uint32_t i) -> uint32_t {
+        i = min(i, i1 - 1);
+        return a.ord ? __ldg(&a.ord[i]) : a.dl ? __ldg(&a.dl[i]) : i;
+    };
+    uint32_t ci = i0 + grab(ctr, chunk, lane), cend = min(ci + chunk, i1);
+    if (lane == 0) tk = atomicAdd(ctr, chunk);
+    uint32_t ni = ci, nend = cend;
+    advance(ni, nend);
+    GMeta m = load_meta(a, moff, gid(ci));
+    uint32_t gn = gid(ni);
+    while (ci < i1) {
+        // unconditional (clamped) loads straight into the look-ahead registers: a
+        // conditional load merged with a copy would wait for the data right here
+        const GMeta mn = load_meta(a, moff, gn);   // gn arrived during the previous group
+        uint32_t nni = ni, nnend = nend;
+        advance(nni, nnend);                       // its grab was issued a range earlier
+        const uint32_t gnn = gid(nni);
+        body(m);
+        ci = ni;
+        m = mn;
+        ni = nni;
+        nend = nnend;
+        gn = gnn;
+    }
 }
 
 // Hit-mask table (count pass -> write pass).  Per group, chunks are grouped in
@@ -260,15 +330,18 @@ __device__ __forceinline__ uint32_t count_group(const SArgs& a, uint32_t qs, uin
         const uint32_t s0 = vpair(vsp, a.nspan, 32 * k + lane, rs, v0, v1), s1 = s0 + 1;
         u64x X, Y;
         double2 d0 = make_double2(kFarD, kFarD), d1 = make_double2(kFarD, kFarD);
+        ulonglong2 P = make_ulonglong2(0, 0);
         if (MODE == kF32) {
-            ulonglong2 P = make_ulonglong2(0, 0);
             if (v0 || v1) P = xp[s0 >> 1];
+        } else {
+            if (v0) d0 = a.xd[s0];
+            if (v1) d1 = a.xd[s1];
+        }
+        if (MODE == kF32) {
             const float2 px = unpack2(P.x), py = unpack2(P.y);
             X = pack2(v0 ? px.x : kFarF, v1 ? px.y : kFarF);
             Y = pack2(v0 ? py.x : kFarF, v1 ? py.y : kFarF);
         } else {
-            if (v0) d0 = a.xd[s0];
-            if (v1) d1 = a.xd[s1];
             if (MODE == kF64Filter) {
                 X = pack2(v0 ? (float)__dsub_rn(d0.x, o.x) : kFarF, v1 ? (float)__dsub_rn(d1.x, o.x) : kFarF);
                 Y = pack2(v0 ? (float)__dsub_rn(d0.y, o.y) : kFarF, v1 ? (float)__dsub_rn(d1.y, o.y) : kFarF);
@@ -405,23 +478,12 @@ __global__ void __launch_bounds__(kSearchThreads) k_count(SArgs a, uint32_t g0, 
 #pragma unroll
     for (int kk = 0; kk < kWin; ++kk) swin[w][lane][kk] = make_uint2(0, 0);
     unsigned long long tests = 0;
-    uint32_t i0 = g0, i1 = g1;
-    dense_range(a, i0, i1);
-    uint32_t ii = i0 + grab(ctr, chunk, lane), iend = min(ii + chunk, i1);
-    while (ii < i1) {
-        const uint32_t gi = a.dl ? __ldg(&a.dl[ii]) : ii;
-        const uint32_t qs = __ldg(&a.gstart[gi]);
-        const uint32_t c = __ldg(&a.gcell[gi]);
-        const uint32_t nq = min((uint32_t)kGroup, __ldg(&a.cstart[c + 1]) - qs);
-        uint2* gmask = masks ? masks + (__ldg(&moff[gi]) >> 1) : nullptr;
+    for_each_group(a, masks ? moff : nullptr, g0, g1, chunk, ctr, lane, [&](const GMeta& m) {
+        uint2* gmask = masks ? masks + (m.ma >> 1) : nullptr;
         const uint32_t my =
-            count_group<MODE>(a, qs, c, nq, swin[w], vsp[w], sq[w], sqd[F64 ? w : 0], gmask, tests, lane);
-        if ((uint32_t)lane < nq) cnt[qs + lane] = my;
-        if (++ii >= iend) {
-            ii = i0 + grab(ctr, chunk, lane);
-            iend = min(ii + chunk, i1);
-        }
-    }
+            count_group<MODE>(a, m.qs, m.c, m.nq, swin[w], vsp[w], sq[w], sqd[F64 ? w : 0], gmask, tests, lane);
+        if ((uint32_t)lane < m.nq) cnt[m.qs + lane] = my;
+    });
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) tests += __shfl_xor_sync(FULL, tests, o);
     if (tests_out && lane == 0 && tests) atomicAdd(tests_out, tests);
@@ -696,22 +758,20 @@ __global__ void __launch_bounds__(kEmitThreads) k_emit(SArgs a, uint32_t g0, uin
     __shared__ VSpan vsp[kEmitWarps][kMaxSpans + 1];  // the group's spans as one pair sequence
     const int lane = threadIdx.x & 31;
     const int w = threadIdx.x >> 5;
+    auto body = [&](const GMeta& m) {
+        const uint32_t nwin = (uint32_t)((m.mb - m.ma) / (2ull * m.nq * kWin));
+        const uint64_t gb = off[m.qs];
+        uint32_t* gout = out + (gb - out_base);
+        asm volatile("mov.b64 %0, %0;" : "+l"(gout));
+        uint32_t my = 0;   // lane i: output cursor of query i within the group
+        if ((uint32_t)lane < m.nq) my = (uint32_t)(off[m.qs + lane] - gb);
+        emit_group(a, m.c, m.nq, nwin, masks + (m.ma >> 1), gout, my, raw[w], wq[w], vsp[w], lane);
+    };
     uint32_t i0 = g0, i1 = g1;
     dense_range(a, i0, i1);
     uint32_t ii = i0 + grab(ctr, chunk, lane), iend = min(ii + chunk, i1);
     while (ii < i1) {
-        const uint32_t gi = a.dl ? __ldg(&a.dl[ii]) : ii;
-        const uint32_t qs = __ldg(&a.gstart[gi]);
-        const uint32_t c = __ldg(&a.gcell[gi]);
-        const uint32_t nq = min((uint32_t)kGroup, __ldg(&a.cstart[c + 1]) - qs);
-        const uint64_t m_a = __ldg(&moff[gi]), m_b = __ldg(&moff[gi + 1]);
-        const uint32_t nwin = (uint32_t)((m_b - m_a) / (2ull * nq * kWin));
-        const uint64_t gb = off[qs];
-        uint32_t* gout = out + (gb - out_base);
-        asm volatile("mov.b64 %0, %0;" : "+l"(gout));
-        uint32_t my = 0;   // lane i: output cursor of query i within the group
-        if ((uint32_t)lane < nq) my = (uint32_t)(off[qs + lane] - gb);
-        emit_group(a, c, nq, nwin, masks + (m_a >> 1), gout, my, raw[w], wq[w], vsp[w], lane);
+        body(load_meta(a, moff, a.dl ? __ldg(&a.dl[ii]) : ii));
         if (++ii >= iend) {
             ii = i0 + grab(ctr, chunk, lane);
             iend = min(ii + chunk, i1);
@@ -1046,6 +1106,7 @@ SArgs args_of(const DevGrid& g) {
     a.e2d = g.e2_d;
     a.dl = g.dl;
     a.dpre = g.dpre;
+    a.ord = nullptr;   // set by the whole-range count / write launches
     a.sql = g.sql;
     a.spre = g.spre;
     return a;
@@ -1155,7 +1216,8 @@ void launch_count_mode(const SArgs& a, uint64_t g0, uint64_t g1, uint64_t ngd, u
 void launch_count(const DevGrid& g, uint64_t g0, uint64_t g1, uint32_t* cnt, unsigned long long* tests,
                   int variant, int slot, uint2* masks, cudaStream_t s) {
     if (g1 <= g0) return;
-    const SArgs a = args_of(g);
+    SArgs a = args_of(g);
+    if (g0 == 0 && g1 == g.n_groups) a.ord = g.ord;
     launch_sparse<false>(g, g0, g1, cnt, tests, nullptr, 0, nullptr, s);
     unsigned int* ctr = g.counters + (slot % kCounterSlots);
     cudaMemsetAsync(ctr, 0, sizeof(unsigned int), s);
@@ -1181,12 +1243,16 @@ void launch_write(const DevGrid& g, uint64_t g0, uint64_t g1, const uint64_t* of
     if (g1 <= g0) return;
     unsigned int* ctr = g.counters + (slot % kCounterSlots);
     cudaMemsetAsync(ctr, 0, sizeof(unsigned int), s);
+    // the write pass keeps the natural (cell-sorted) group order without look-ahead:
+    // measured on B200 (tools/ab.sh), both cost order and look-ahead slowed the
+    // store streams (C2 eps 0.45: 1.48 ms plain vs 1.55 ordered vs 1.56 look-ahead)
+    const SArgs a = args_of(g);
     static int bps = 0;
     uint32_t chunk;
     unsigned ctas;
     launch_groups(k_emit, bps, dense_groups(g, g0, g1), chunk, ctas, kEmitThreads);
-    k_emit<<<ctas, kEmitThreads, 0, s>>>(args_of(g), (uint32_t)g0, (uint32_t)g1, chunk, ctr, off, out_base, out,
-                                           masks, g.moff);
+    k_emit<<<ctas, kEmitThreads, 0, s>>>(a, (uint32_t)g0, (uint32_t)g1, chunk, ctr, off, out_base, out, masks,
+                                         g.moff);
     ++g_kernel_launches;
 }
 

@@ -14,7 +14,7 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libhdb.so")
+LIB_PATH = os.environ.get("HDB_LIB") or os.path.join(_HERE, "libhdb.so")   # HDB_LIB: A/B builds (tools/ab.sh)
 
 if not os.path.exists(LIB_PATH):
     raise ImportError(f"{LIB_PATH} not built: run `python -c 'import __graft_entry__ as g; g.build()'`")
