@@ -201,6 +201,14 @@ constexpr uint64_t kMaxCellsAbs = 1ull << 30;
 // when (queries x candidates) <= this many tests (
 // HDB_SPARSE_TESTS overrides it for tuning, 0 disables the split).
 constexpr double kSparseMinShare = 0.25;   // split only when >= this share of the queries is sparse
+// Device-resident whole tables take the single-pass kernel (k_fused: count,
+// reserve, emit per group; heavy groups first) unless the dense/sparse split is
+// on or the sampled estimate says < this many pairs per query.  Measured on one
+// B200 (ms of table kernels, two passes vs single pass): C2 eps 0.15 (97 pairs
+// per query) 0.72 vs 0.65, eps 0.45 (700) 2.39 vs 2.10, eps 1.40 (4,600) 13.1 vs
+// 9.8 -- the count pass's ALU work hides under the emission's store stream; C5
+// (80 pairs per query) 13.6 vs 14.4.
+constexpr double kFusedMinPairsPerQuery = 90.0;
 uint32_t sparse_max_tests() {
     static const uint32_t v = [] {
         const char* e = std::getenv("HDB_SPARSE_TESTS");
@@ -499,7 +507,7 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
     // words for every group either way.
     const int sk = ctx->opts.search_kernel;
     const uint32_t max_tests = sparse_max_tests();
-    const bool classify = (sk == 0 || sk == 1 || sk == 2) && max_tests > 0 && n > 0;
+    const bool classify = (sk == 0 || sk == 1 || sk == 2 || sk == 4) && max_tests > 0 && n > 0;
     DBuf dpre, spre, dl, sql, ord;
     unsigned long long* nsp = bb + 8;
     if (classify) {
@@ -544,7 +552,7 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
         if (classify) g.ord = (uint32_t*)ord.release();
         // the split pays only when a good share of the queries is sparse: the thread-per-query
         // kernels run after the dense ones and a few sparse groups only add their latency
-        if (classify && (double)hsp >= kSparseMinShare * (double)n) {
+        if (classify && sk != 4 && (double)hsp >= kSparseMinShare * (double)n) {
             g.dpre = (uint32_t*)dpre.release();
             g.spre = (uint32_t*)spre.release();
             g.dl = (uint32_t*)dl.release();
@@ -1088,14 +1096,20 @@ void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hd
             single = true;
             tr.mark("paper-kernel");
         }
-        if (!single && device_resident && parts == 1 && sk == 4 && n > 0) {
+        // single pass (k_fused): asked for (search_kernel 4) or chosen for dense tables;
+        // the dense/sparse split keeps the two passes (the sparse queries' kernels
+        // write at scanned offsets)
+        if (!single && device_resident && parts == 1 && (sk == 4 || sk == 0) && n > 0 && !G0.dl) {
             HDB_CUDA(cudaStreamSynchronize(s0));   // e_b is in dc0.pin[0]
             const uint64_t eb = dc0.pin[0];
-            S.sample_size = ns;
-            S.sample_pairs = eb;
-            S.est_pairs = eb * stride;
-            S.ms_sample = elapsed(es0, es1);
-            single = single_pass_table(ctx, G0, t, S, eb * stride);
+            const bool fused = sk == 4 || (double)(eb * stride) >= kFusedMinPairsPerQuery * (double)n;
+            if (fused) {
+                S.sample_size = ns;
+                S.sample_pairs = eb;
+                S.est_pairs = eb * stride;
+                S.ms_sample = elapsed(es0, es1);
+                single = single_pass_table(ctx, G0, t, S, eb * stride);
+            }
             if (single) {
                 double bb = 0;
                 uint64_t nbp = 0;
