@@ -13,6 +13,9 @@ done
 python bench.py --workload C4-sweep --steps 3 --warmup 1 > gpurun_out/${T}_bench_C4.json 2>> gpurun_out/${T}_bench.err
 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/${T}_launches_c2_eps045.csv \
     python bench.py --steps 2 --warmup 1 --e2e-steps 0 --no-cpu-baseline > /dev/null 2>&1
-ncu --set full --clock-control none --import-source on -k regex:"k_count|k_emit" -c 2 -o gpurun_out/${T}_prof_c2 \
+ncu --set full --clock-control none --import-source on -k regex:"k_fused|k_count|k_emit" -c 2 -o gpurun_out/${T}_prof_c2 \
     python bench.py --steps 1 --warmup 0 --e2e-steps 0 --no-cpu-baseline > /dev/null 2>&1
+# the two-pass kernels (count + write) on the workload that takes them by default (C5, 80 pairs/query)
+ncu --set full --clock-control none --import-source on -k regex:"k_count|k_emit" -c 2 -o gpurun_out/${T}_prof_c5 \
+    python bench.py --workload C5-eps0.5 --steps 1 --warmup 0 --e2e-steps 0 --no-cpu-baseline > /dev/null 2>&1
 ls -la gpurun_out | grep $T
