@@ -105,6 +105,12 @@ hdb_status hdb_ctx_create(const hdb_opts* opts, hdb_ctx** out) {
         HDB_CUDA(cudaDeviceGetDefaultMemPool(&pool, d));
         uint64_t thr = UINT64_MAX;
         HDB_CUDA(cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr));
+        cudaMemPoolProps props{};
+        props.allocType = cudaMemAllocationTypePinned;
+        props.location.type = cudaMemLocationTypeDevice;
+        props.location.id = d;
+        HDB_CUDA(cudaMemPoolCreate(&dc.big_pool, &props));
+        HDB_CUDA(cudaMemPoolSetAttribute(dc.big_pool, cudaMemPoolAttrReleaseThreshold, &thr));
         c->dev.push_back(dc);
     }
     cudaSetDevice(prev);
@@ -136,6 +142,8 @@ void hdb_ctx_destroy(hdb_ctx* c) {
         for (auto s : dc.streams) cudaStreamDestroy(s);
         if (dc.main && dc.own_main) cudaStreamDestroy(dc.main);
         if (dc.pin) cudaFreeHost(dc.pin);
+        // tables still alive keep their blocks: the pool is then left to process exit
+        if (dc.big_pool && c->live_objects == 0) cudaMemPoolDestroy(dc.big_pool);
     }
     cudaSetDevice(prev);
     delete c;

@@ -144,9 +144,10 @@ struct DBuf {
     void* p = nullptr;
     cudaStream_t s = nullptr;
     DBuf() = default;
-    DBuf(size_t bytes, cudaStream_t st) : s(st) {
+    // pool: the device's big_pool for table-sized buffers (null = the default pool)
+    DBuf(size_t bytes, cudaStream_t st, cudaMemPool_t pool = nullptr) : s(st) {
         if (bytes == 0) bytes = 16;
-        cudaError_t e = cudaMallocAsync(&p, bytes, st);
+        cudaError_t e = pool ? cudaMallocFromPoolAsync(&p, bytes, pool, st) : cudaMallocAsync(&p, bytes, st);
         if (e != cudaSuccess) {
             cudaGetLastError();
             p = nullptr;
@@ -706,7 +707,7 @@ void count_phase(hdb_ctx* ctx, DevCtx& dc, const DevGrid& g, ShardState& st) {
         }
         const size_t bytes = 4 * (mo[1] - mo[0]);
         void* p = nullptr;
-        if (cudaMallocAsync(&p, bytes ? bytes : 16, s) == cudaSuccess) {
+        if (cudaMallocFromPoolAsync(&p, bytes ? bytes : 16, dc.big_pool, s) == cudaSuccess) {
             st.masks.p = p;
             st.masks.s = s;
             st.mask_base = (uint2*)p - (mo[0] >> 1);
@@ -750,13 +751,13 @@ bool single_pass_table(hdb_ctx* ctx, const DevGrid& g, hdb_table* t, hdb_stats& 
     const uint64_t n = g.n;
     const uint64_t cap = (uint64_t)((double)std::max<uint64_t>(est, n) * 1.25) + (1ull << 20);
     DBuf masks, nb;
-    if (cudaMallocAsync(&masks.p, 4 * std::max<uint64_t>(g.mask_words, 4), s) != cudaSuccess ||
-        cudaMallocAsync(&nb.p, 4 * cap, s) != cudaSuccess) {
+    if (cudaMallocFromPoolAsync(&masks.p, 4 * std::max<uint64_t>(g.mask_words, 4), dc.big_pool, s) != cudaSuccess ||
+        cudaMallocFromPoolAsync(&nb.p, 4 * cap, dc.big_pool, s) != cudaSuccess) {
         cudaGetLastError();
         return false;
     }
     masks.s = nb.s = s;
-    DBuf beg(8 * n, s), cnt_id(4 * n, s), cnt(4 * n, s), scratch(32, s);
+    DBuf beg(8 * n, s, dc.big_pool), cnt_id(4 * n, s, dc.big_pool), cnt(4 * n, s), scratch(32, s);
     HDB_CUDA(cudaMemsetAsync(scratch.p, 0, 32, s));
     unsigned long long* sc = scratch.as<unsigned long long>();
     Event e0, e1;
@@ -776,7 +777,7 @@ bool single_pass_table(hdb_ctx* ctx, const DevGrid& g, hdb_table* t, hdb_stats& 
     t->npairs = P;
     t->first_query = 0;
     t->end_query = n;
-    DBuf rw(4 * n, s);
+    DBuf rw(4 * n, s, dc.big_pool);
     HDB_CUDA(cudaMemcpyAsync(rw.p, g.ids, 4 * n, cudaMemcpyDeviceToDevice, s));
     t->rows = (uint32_t*)rw.release();
     t->nbrs = (uint32_t*)nb.release();
@@ -1171,7 +1172,8 @@ void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hd
                 t->on_device = true;
                 t->device = dc.device;
                 t->dstream = s;
-                DBuf nb(4 * (P ? P : 1), s), beg(8 * (n ? n : 1), s), cnt(4 * (n ? n : 1), s);
+                DBuf nb(4 * (P ? P : 1), s, dc.big_pool), beg(8 * (n ? n : 1), s, dc.big_pool),
+                    cnt(4 * (n ? n : 1), s, dc.big_pool);
                 if (!whole) {
                     HDB_CUDA(cudaMemsetAsync(beg.p, 0, 8 * (n ? n : 1), s));
                     HDB_CUDA(cudaMemsetAsync(cnt.p, 0, 4 * (n ? n : 1), s));

@@ -209,6 +209,11 @@ struct DevCtx {
     std::vector<cudaStream_t> streams;     // write + D2H streams
     std::vector<cudaEvent_t> ev_pool;
     uint64_t* pin = nullptr;                // small pinned scratch for async readbacks
+    // Stream-ordered pool of its own for the table-sized buffers (neighbour lists,
+    // hit masks, T by id): step-sized blocks then reuse each other instead of
+    // being carved up by the grid's smaller buffers in the default pool (which
+    // made C5 steps map fresh memory: 27 -> 60..120 ms outliers)
+    cudaMemPool_t big_pool = nullptr;
     // cached per-stream device batch buffers (reused across calls)
     std::vector<uint32_t*> batch_buf;
     std::vector<size_t> batch_cap;
