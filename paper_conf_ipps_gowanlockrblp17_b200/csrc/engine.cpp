@@ -441,11 +441,12 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
     DBuf xy_s((n + 2) * esz, s);
     DBuf xp(16 * (n / 2 + 2), s);
     DBuf counters(4 * kCounterSlots, s);
+    DBuf inv(4 * (n + 1), s);
     HDB_CUDA(cudaMemsetAsync(xy_s.as<char>() + n * esz, 0, 2 * esz, s));
     HDB_CUDA(cudaMemsetAsync(ids.as<uint32_t>() + n, 0, 8, s));
     HDB_CUDA(cudaMemsetAsync(xp.p, 0, 16 * (n / 2 + 2), s));
     HDB_CUDA(cudaMemsetAsync(counters.p, 0, 4 * kCounterSlots, s));
-    launch_gather_points(xin, ids.as<uint32_t>(), n, dt, xy_s.p, xp.as<float4>(), g.ox, g.oy, s);
+    launch_gather_points(xin, ids.as<uint32_t>(), n, dt, xy_s.p, xp.as<float4>(), g.ox, g.oy, inv.as<uint32_t>(), s);
     HDB_LAUNCH_CHECK();
     xin_owned.reset();
     tr.mark("keys+sort+gather(enqueue)");
@@ -496,6 +497,7 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
     g.xp = (float4*)xp.release();
     g.counters = (unsigned int*)counters.release();
     g.ids = (uint32_t*)ids.release();
+    g.inv = (uint32_t*)inv.release();
     g.ckey = (uint64_t*)ckey.release();
     g.cstart = (uint32_t*)cstart.release();
     g.cspan = (uint2*)cspan.release();
@@ -573,14 +575,14 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
 void free_dev_grid(DevGrid& g) {
     if (!g.stream) return;
     DeviceGuard dg(g.device);
-    for (void* p : {(void*)g.xy_s, (void*)g.xp, (void*)g.counters, (void*)g.ids, (void*)g.ckey, (void*)g.cstart,
+    for (void* p : {(void*)g.xy_s, (void*)g.xp, (void*)g.counters, (void*)g.ids, (void*)g.inv, (void*)g.ckey, (void*)g.cstart,
                     (void*)g.cspan, (void*)g.gstart, (void*)g.gcell, (void*)g.moff, (void*)g.dpre, (void*)g.spre,
                     (void*)g.dl, (void*)g.sql, (void*)g.ord})
         if (p) cudaFreeAsync(p, g.stream);   // stream-ordered: no host sync needed
     g.xy_s = nullptr;
     g.xp = nullptr;
     g.counters = nullptr;
-    g.ids = g.cstart = g.gstart = g.gcell = nullptr;
+    g.ids = g.inv = g.cstart = g.gstart = g.gcell = nullptr;
     g.moff = nullptr;
     g.dpre = g.spre = g.dl = g.ord = nullptr;
     g.sql = nullptr;
@@ -1184,8 +1186,8 @@ void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hd
                              st.mask_base, s);
                 HDB_LAUNCH_CHECK();
                 HDB_CUDA(cudaEventRecord(e1.e, s));
-                launch_scatter_rows(g.ids, g.n, st.off.as<uint64_t>(), st.cnt.as<uint32_t>(), st.r.q0, st.r.q1, 0,
-                                    beg.as<uint64_t>(), cnt.as<uint32_t>(), s);
+                launch_rows_by_id(g.inv, g.n, st.off.as<uint64_t>(), st.cnt.as<uint32_t>(), st.r.q0, st.r.q1, 0,
+                                  beg.as<uint64_t>(), cnt.as<uint32_t>(), s);
                 HDB_LAUNCH_CHECK();
                 HDB_CUDA(cudaStreamSynchronize(s));
                 st.ms_write = elapsed(e0, e1);
@@ -1226,8 +1228,8 @@ void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hd
                     DeviceGuard dg(dc.device);
                     cudaStream_t s = dc.main;
                     DBuf beg(8 * (n ? n : 1), s), cnt(4 * (n ? n : 1), s);
-                    launch_scatter_rows(grid->dev[0].ids, n, sh[0].off.as<uint64_t>(), sh[0].cnt.as<uint32_t>(), 0, n, 0,
-                                        beg.as<uint64_t>(), cnt.as<uint32_t>(), s);
+                    launch_rows_by_id(grid->dev[0].inv, n, sh[0].off.as<uint64_t>(), sh[0].cnt.as<uint32_t>(), 0, n, 0,
+                                      beg.as<uint64_t>(), cnt.as<uint32_t>(), s);
                     HDB_LAUNCH_CHECK();
                     if (n) {
                         HDB_CUDA(cudaMemcpyAsync(t->begin, beg.p, 8 * n, cudaMemcpyDeviceToHost, s));

@@ -66,6 +66,7 @@ struct DevGrid {
                                    // filter coords x-ox, y-oy (f64 mode) / the exact coords (f32 mode)
     unsigned int* counters = nullptr;  // [kCounterSlots] work counters of the search kernels
     uint32_t* ids = nullptr;       // [n] sorted pos -> original id  (A)
+    uint32_t* inv = nullptr;       // [n] original id -> sorted pos  (A^-1, written by the gather)
     uint64_t* ckey = nullptr;      // [n_nonempty] cell key of each non-empty cell (ascending)
     uint32_t* cstart = nullptr;    // [n_nonempty+1] first sorted pos of each non-empty cell (G)
     uint2* cspan = nullptr;        // [nspan*n_nonempty] stencil row spans [lo,hi) per non-empty cell
@@ -99,12 +100,9 @@ size_t radix_sort_temp_bytes(uint64_t n);
 // between (k0,v0) and (k1,v1); returns 0 if the result is in (k0,v0), 1 else.
 int radix_sort_pairs(void* k0, uint32_t* v0, void* k1, uint32_t* v1, int key_bytes, uint64_t n, int bits,
                      void* temp, cudaStream_t s);
-// the same on 32-bit keys, digits of bits [shift0, bits) only (a partial, most-significant sort)
-int radix_sort_u32_digits(uint32_t* k0, uint32_t* v0, uint32_t* k1, uint32_t* v1, uint64_t n, int shift0, int bits,
-                          void* temp, cudaStream_t s);
 // gather sorted points; f64 mode also writes the f32 filter coordinates (x-ox, y-oy)
 void launch_gather_points(const void* xy_in, const uint32_t* ids, uint64_t n, hdb_dtype dt, void* xy_s,
-                          float4* xp, double ox, double oy, cudaStream_t s);
+                          float4* xp, double ox, double oy, uint32_t* inv, cudaStream_t s);
 void launch_cell_flags(const void* keys_sorted, int key_bytes, uint64_t n, uint32_t* flags, cudaStream_t s);
 void launch_cell_scatter(const void* keys_sorted, int key_bytes, const uint32_t* flags, const uint32_t* pos,
                          uint64_t n, uint64_t* ckey, uint32_t* cstart, cudaStream_t s);
@@ -175,11 +173,10 @@ void launch_dbscan_device(const uint64_t* begin, const uint32_t* count, const ui
                           uint32_t* root, uint32_t* is_root, uint32_t* rank, uint32_t* giant, uint32_t* bits,
                           uint32_t* sched /* 2 x SM count */, uint64_t* pre /* n + 1 */, void* scan_temp,
                           int32_t* labels, cudaStream_t s);
-// T assembly by original id: begin[ids[q]] = off[q] - off[q0] + base, count[ids[q]] = cnt[q], q in [q0,q1);
-// ids < n_ids.  Large ranges first partition (id, q) by the id's top digit (one stable radix
-// pass) so that the scattered writes of each bucket stay inside an L2-resident window.
-void launch_scatter_rows(const uint32_t* ids, uint64_t n_ids, const uint64_t* off, const uint32_t* cnt, uint64_t q0,
-                         uint64_t q1, uint64_t base, uint64_t* begin, uint32_t* count, cudaStream_t s);
+// T by original id through A^-1 (sequential writes, gathered reads): for every id
+// whose sorted position q lies in [q0, q1): begin[id] = off[q] - off[q0] + base, count[id] = cnt[q]
+void launch_rows_by_id(const uint32_t* inv, uint64_t n_ids, const uint64_t* off, const uint32_t* cnt, uint64_t q0,
+                       uint64_t q1, uint64_t base, uint64_t* begin, uint32_t* count, cudaStream_t s);
 
 // the paper's kernels (kernels_paper.cu; search_kernel 7 / 8):
 // the key/value result set R of GPUCalcGlobal (Alg. 2) or GPUCalcShared (Alg. 3),

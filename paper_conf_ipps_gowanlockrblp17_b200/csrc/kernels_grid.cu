@@ -239,14 +239,16 @@ template <typename T>
 __global__ void __launch_bounds__(256) k_gather(const typename V2<T>::type* __restrict__ in,
                                                 const uint32_t* __restrict__ ids, uint64_t n,
                                                 typename V2<T>::type* __restrict__ out, float4* __restrict__ xp,
-                                                double ox, double oy) {
+                                                double ox, double oy, uint32_t* __restrict__ inv) {
     // xp: paired-SoA f32 copy {x_2k, x_2k+1, y_2k, y_2k+1} -- f64 input: filter
     // coordinates fl32(fl64(x - ox)); f32 input: the exact coordinates
     float* xpf = (float*)xp;
     for (uint64_t s = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; s < n;
          s += (uint64_t)gridDim.x * blockDim.x) {
-        auto p = in[ids[s]];
+        const uint32_t id = ids[s];
+        auto p = in[id];
         out[s] = p;
+        inv[id] = (uint32_t)s;   // A^-1: T by original id gathers through it (launch_rows_by_id)
         float fx, fy;
         if (sizeof(p.x) == 8) {
             fx = (float)__dsub_rn((double)p.x, ox);
@@ -600,10 +602,6 @@ int radix_sort_impl(K* k0, uint32_t* v0, K* k1, uint32_t* v1, uint64_t n, int bi
     return cur;
 }
 
-int radix_sort_u32_digits(uint32_t* k0, uint32_t* v0, uint32_t* k1, uint32_t* v1, uint64_t n, int shift0, int bits,
-                          void* temp, cudaStream_t s) {
-    return radix_sort_impl<uint32_t>(k0, v0, k1, v1, n, bits, temp, s, shift0);
-}
 
 int radix_sort_pairs(void* k0, uint32_t* v0, void* k1, uint32_t* v1, int key_bytes, uint64_t n, int bits, void* temp,
                      cudaStream_t s) {
@@ -613,12 +611,12 @@ int radix_sort_pairs(void* k0, uint32_t* v0, void* k1, uint32_t* v1, int key_byt
 }
 
 void launch_gather_points(const void* xy_in, const uint32_t* ids, uint64_t n, hdb_dtype dt, void* xy_s, float4* xp,
-                          double ox, double oy, cudaStream_t s) {
+                          double ox, double oy, uint32_t* inv, cudaStream_t s) {
     if (n == 0) return;
     if (dt == HDB_F64)
-        k_gather<double><<<grid_for(n), 256, 0, s>>>((const double2*)xy_in, ids, n, (double2*)xy_s, xp, ox, oy);
+        k_gather<double><<<grid_for(n), 256, 0, s>>>((const double2*)xy_in, ids, n, (double2*)xy_s, xp, ox, oy, inv);
     else
-        k_gather<float><<<grid_for(n), 256, 0, s>>>((const float2*)xy_in, ids, n, (float2*)xy_s, xp, 0, 0);
+        k_gather<float><<<grid_for(n), 256, 0, s>>>((const float2*)xy_in, ids, n, (float2*)xy_s, xp, 0, 0, inv);
     ++g_kernel_launches;
 }
 

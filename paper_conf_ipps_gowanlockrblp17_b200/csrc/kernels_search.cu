@@ -1051,43 +1051,7 @@ __global__ void k_pos_to_group(const uint32_t* __restrict__ gstart, uint64_t ng,
     grp[i] = lo;
 }
 
-__global__ void __launch_bounds__(256) k_scatter_rows(const uint32_t* __restrict__ ids,
-                                                      const uint64_t* __restrict__ off,
-                                                      const uint32_t* __restrict__ cnt, uint64_t q0, uint64_t q1,
-                                                      uint64_t base, uint64_t* __restrict__ begin,
-                                                      uint32_t* __restrict__ count) {
-    const uint64_t o0 = off[q0];
-    for (uint64_t q = q0 + blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; q < q1;
-         q += (uint64_t)gridDim.x * blockDim.x) {
-        uint32_t id = ids[q];
-        begin[id] = off[q] - o0 + base;
-        count[id] = cnt[q];
-    }
-}
 
-__global__ void __launch_bounds__(256) k_bucket_prep(const uint32_t* __restrict__ ids, uint64_t q0, uint64_t m,
-                                                     uint32_t* __restrict__ key, uint32_t* __restrict__ val) {
-    for (uint64_t j = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; j < m; j += (uint64_t)gridDim.x * blockDim.x) {
-        key[j] = ids[q0 + j];
-        val[j] = (uint32_t)(q0 + j);
-    }
-}
-
-// (id, q) pairs in bucket order: consecutive threads write into one bucket's id window
-__global__ void __launch_bounds__(256) k_scatter_sorted(const uint32_t* __restrict__ key,
-                                                        const uint32_t* __restrict__ val, uint64_t m, uint64_t q0,
-                                                        const uint64_t* __restrict__ off,
-                                                        const uint32_t* __restrict__ cnt, uint64_t base,
-                                                        uint64_t* __restrict__ begin, uint32_t* __restrict__ count) {
-    const uint64_t o0 = off[q0];
-    for (uint64_t j = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; j < m; j += (uint64_t)gridDim.x * blockDim.x) {
-        const uint32_t id = key[j], q = val[j];
-        begin[id] = off[q] - o0 + base;
-        count[id] = cnt[q];
-    }
-}
-
-constexpr uint64_t kBucketScatterMin = 1ull << 22;   // rows from which the bucketed scatter pays
 
 SArgs args_of(const DevGrid& g) {
     SArgs a;
@@ -1310,36 +1274,27 @@ void launch_pos_to_group(const uint32_t* gstart, uint64_t n_groups, const uint64
     ++g_kernel_launches;
 }
 
-void launch_scatter_rows(const uint32_t* ids, uint64_t n_ids, const uint64_t* off, const uint32_t* cnt, uint64_t q0,
-                         uint64_t q1, uint64_t base, uint64_t* begin, uint32_t* count, cudaStream_t s) {
-    if (q1 <= q0) return;
-    uint64_t n = q1 - q0;
-    if (n >= kBucketScatterMin) {
-        int bits = 1;
-        while (bits < 32 && (1ull << bits) < n_ids) ++bits;
-        const int shift0 = bits > 8 ? bits - 8 : 0;   // one pass: 256 buckets of the id range
-        void *k0 = nullptr, *v0 = nullptr, *k1 = nullptr, *v1 = nullptr, *tmp = nullptr;
-        const size_t tb = radix_sort_temp_bytes(n);
-        if (cudaMallocAsync(&k0, 4 * n, s) == cudaSuccess && cudaMallocAsync(&v0, 4 * n, s) == cudaSuccess &&
-            cudaMallocAsync(&k1, 4 * n, s) == cudaSuccess && cudaMallocAsync(&v1, 4 * n, s) == cudaSuccess &&
-            cudaMallocAsync(&tmp, tb, s) == cudaSuccess) {
-            const unsigned nb = (unsigned)std::min<uint64_t>((n + 255) / 256, 148 * 16);
-            k_bucket_prep<<<nb, 256, 0, s>>>(ids, q0, n, (uint32_t*)k0, (uint32_t*)v0);
-            const int w = radix_sort_u32_digits((uint32_t*)k0, (uint32_t*)v0, (uint32_t*)k1, (uint32_t*)v1, n, shift0,
-                                                bits, tmp, s);
-            k_scatter_sorted<<<nb, 256, 0, s>>>((const uint32_t*)(w ? k1 : k0), (const uint32_t*)(w ? v1 : v0), n, q0,
-                                                off, cnt, base, begin, count);
-            g_kernel_launches += 2;
-            for (void* p : {k0, v0, k1, v1, tmp}) cudaFreeAsync(p, s);
-            return;
+__global__ void __launch_bounds__(256) k_rows_by_id(const uint32_t* __restrict__ inv, uint64_t n_ids,
+                                                    const uint64_t* __restrict__ off,
+                                                    const uint32_t* __restrict__ cnt, uint64_t q0, uint64_t q1,
+                                                    uint64_t base, uint64_t* __restrict__ begin,
+                                                    uint32_t* __restrict__ count) {
+    const uint64_t o0 = off[q0];
+    for (uint64_t id = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; id < n_ids;
+         id += (uint64_t)gridDim.x * blockDim.x) {
+        const uint32_t q = inv[id];
+        if (q >= q0 && q < q1) {
+            begin[id] = off[q] - o0 + base;
+            count[id] = cnt[q];
         }
-        cudaGetLastError();   // no scratch memory: the direct scatter below
-        for (void* p : {k0, v0, k1, v1, tmp})
-            if (p) cudaFreeAsync(p, s);
     }
-    unsigned blocks = (unsigned)((n + 255) / 256);
-    if (blocks > 148 * 16) blocks = 148 * 16;
-    k_scatter_rows<<<blocks, 256, 0, s>>>(ids, off, cnt, q0, q1, base, begin, count);
+}
+
+void launch_rows_by_id(const uint32_t* inv, uint64_t n_ids, const uint64_t* off, const uint32_t* cnt, uint64_t q0,
+                       uint64_t q1, uint64_t base, uint64_t* begin, uint32_t* count, cudaStream_t s) {
+    if (q1 <= q0 || n_ids == 0) return;
+    const unsigned blocks = (unsigned)std::min<uint64_t>((n_ids + 255) / 256, 148 * 16);
+    k_rows_by_id<<<blocks, 256, 0, s>>>(inv, n_ids, off, cnt, q0, q1, base, begin, count);
     ++g_kernel_launches;
 }
 
