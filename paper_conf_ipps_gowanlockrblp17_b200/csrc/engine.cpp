@@ -364,10 +364,14 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
     HDB_CUDA(cudaMemsetAsync(bb + 4, 0, 8, s));
     launch_bbox(xin, n, dt, bb, bad, s);
     HDB_LAUNCH_CHECK();
+    tr.mark("bbox-enqueue");
     // default cell split: occupancy estimate launched with the bbox, read in the same sync
     const bool auto_k = ctx->opts.cell_split == 0 && n >= 4096;
     DBuf hk, hc, occ;
-    unsigned long long hocc[2] = {0, 0};
+    // small readbacks go through the context's pinned scratch (pin[8..21]): a D2H copy
+    // into pageable memory is synchronous and cost ~30 us each here
+    unsigned long long* hocc = (unsigned long long*)dc.pin + 8;
+    hocc[0] = hocc[1] = 0;
     if (auto_k) {
         const double eps_pre = dt == HDB_F32 ? (double)(float)eps : eps;
         hk = DBuf(8ull * kOccTable, s);
@@ -377,10 +381,11 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
         launch_occ_estimate(xin, n, dt, n / m, m, 1.0 / (eps_pre * (1.0 + 0x1p-19)), hk.as<unsigned long long>(),
                             hc.as<unsigned int>(), kOccTable, occ.as<unsigned long long>(), s);
         HDB_LAUNCH_CHECK();
-        HDB_CUDA(cudaMemcpyAsync(hocc, occ.p, sizeof hocc, cudaMemcpyDeviceToHost, s));
+        HDB_CUDA(cudaMemcpyAsync(hocc, occ.p, 16, cudaMemcpyDeviceToHost, s));
     }
-    unsigned long long hb[6];
-    HDB_CUDA(cudaMemcpyAsync(hb, bb, sizeof hb, cudaMemcpyDeviceToHost, s));
+    unsigned long long* hb = (unsigned long long*)dc.pin + 10;   // [10..15]
+    HDB_CUDA(cudaMemcpyAsync(hb, bb, 48, cudaMemcpyDeviceToHost, s));
+    tr.mark("occ-enqueue");
     HDB_CUDA(cudaStreamSynchronize(s));
     hk.reset();
     hc.reset();
@@ -455,9 +460,11 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
     launch_cell_flags(keys.p, kb, n, flags.as<uint32_t>(), s);
     scan_u32_to_u32(flags.as<uint32_t>(), pos.as<uint32_t>(), n, temp.p, s);
     HDB_LAUNCH_CHECK();
-    uint32_t hne = 0;
-    HDB_CUDA(cudaMemcpyAsync(&hne, pos.as<uint32_t>() + n, 4, cudaMemcpyDeviceToHost, s));
+    uint32_t* hne_p = (uint32_t*)(dc.pin + 16);
+    *hne_p = 0;
+    HDB_CUDA(cudaMemcpyAsync(hne_p, pos.as<uint32_t>() + n, 4, cudaMemcpyDeviceToHost, s));
     HDB_CUDA(cudaStreamSynchronize(s));
+    const uint32_t hne = *hne_p;
     g.n_nonempty = hne;
     const uint64_t nne = hne;
     DBuf ckey(8 * nne, s), cstart(4 * (nne + 1), s);
@@ -493,6 +500,7 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
     launch_group_build(cstart.as<uint32_t>(), gofs.as<uint32_t>(), nne, n, gstart.as<uint32_t>(),
                        gcell.as<uint32_t>(), s);
     HDB_LAUNCH_CHECK();
+    tr.mark("spans+groups-enqueue");
     g.xy_s = xy_s.release();
     g.xp = (float4*)xp.release();
     g.counters = (unsigned int*)counters.release();
@@ -536,18 +544,22 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
         launch_mask_words(g, gofs.as<uint32_t>() + nne, n, words.as<uint32_t>(), s);
         scan_u32_to_u64(words.as<uint32_t>(), moff.as<uint64_t>(), n, mtemp.p, s);
         HDB_LAUNCH_CHECK();
-        uint32_t hng = 0;
-        uint32_t hds[2] = {0, 0};
-        uint64_t hsp = 0;
-        HDB_CUDA(cudaMemcpyAsync(&hng, gofs.as<uint32_t>() + nne, 4, cudaMemcpyDeviceToHost, s));
-        HDB_CUDA(cudaMemcpyAsync(&g.mask_words, moff.as<uint64_t>() + n, 8, cudaMemcpyDeviceToHost, s));
+        uint64_t* pr = dc.pin + 17;   // [17] groups, [18] mask words, [19] dense groups, [20] sparse queries
+        pr[0] = pr[1] = pr[2] = pr[3] = pr[4] = 0;   //   (pinned: asynchronous readbacks), [21] sparse count
+        HDB_CUDA(cudaMemcpyAsync(&pr[0], gofs.as<uint32_t>() + nne, 4, cudaMemcpyDeviceToHost, s));
+        HDB_CUDA(cudaMemcpyAsync(&pr[1], moff.as<uint64_t>() + n, 8, cudaMemcpyDeviceToHost, s));
         if (classify) {
-            HDB_CUDA(cudaMemcpyAsync(&hds[0], dpre.as<uint32_t>() + n, 4, cudaMemcpyDeviceToHost, s));
-            HDB_CUDA(cudaMemcpyAsync(&hds[1], spre.as<uint32_t>() + n, 4, cudaMemcpyDeviceToHost, s));
-            HDB_CUDA(cudaMemcpyAsync(&hsp, nsp, 8, cudaMemcpyDeviceToHost, s));
+            HDB_CUDA(cudaMemcpyAsync(&pr[2], dpre.as<uint32_t>() + n, 4, cudaMemcpyDeviceToHost, s));
+            HDB_CUDA(cudaMemcpyAsync(&pr[3], spre.as<uint32_t>() + n, 4, cudaMemcpyDeviceToHost, s));
+            HDB_CUDA(cudaMemcpyAsync(&pr[4], nsp, 8, cudaMemcpyDeviceToHost, s));
         }
         HDB_CUDA(cudaEventRecord(ev1.e, s));
+        tr.mark("class+order+masklayout-enqueue");
         HDB_CUDA(cudaEventSynchronize(ev1.e));
+        const uint32_t hng = (uint32_t)pr[0];
+        g.mask_words = pr[1];
+        const uint32_t hds[2] = {(uint32_t)pr[2], (uint32_t)pr[3]};
+        const uint64_t hsp = pr[4];
         g.n_groups = hng;
         g.moff = (uint64_t*)moff.release();
         g.n_dense_groups = hng;
@@ -730,7 +742,7 @@ void count_phase(hdb_ctx* ctx, DevCtx& dc, const DevGrid& g, ShardState& st) {
     scan_u32_to_u64(st.cnt.as<uint32_t>() + st.r.q0, st.off.as<uint64_t>() + st.r.q0, len, temp.p, s);
     HDB_LAUNCH_CHECK();
     HDB_CUDA(cudaEventRecord(e2.e, s));
-    uint64_t h[2] = {0, 0};
+    uint64_t* h = dc.pin + 22;   // pinned: asynchronous readbacks
     HDB_CUDA(cudaMemcpyAsync(&h[0], st.off.as<uint64_t>() + st.r.q1, 8, cudaMemcpyDeviceToHost, s));
     HDB_CUDA(cudaMemcpyAsync(&h[1], tests.p, 8, cudaMemcpyDeviceToHost, s));
     HDB_CUDA(cudaStreamSynchronize(s));
