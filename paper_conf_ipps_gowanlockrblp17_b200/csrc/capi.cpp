@@ -110,6 +110,8 @@ hdb_status hdb_ctx_create(const hdb_opts* opts, hdb_ctx** out) {
         props.location.type = cudaMemLocationTypeDevice;
         props.location.id = d;
         HDB_CUDA(cudaMemPoolCreate(&dc.big_pool, &props));
+        size_t free_b = 0;
+        HDB_CUDA(cudaMemGetInfo(&free_b, &dc.total_mem));
         HDB_CUDA(cudaMemPoolSetAttribute(dc.big_pool, cudaMemPoolAttrReleaseThreshold, &thr));
         c->dev.push_back(dc);
     }

@@ -210,6 +210,11 @@ constexpr double kSparseMinShare = 0.25;   // split only when >= this share of t
 // 9.8 -- the count pass's ALU work hides under the emission's store stream; C5
 // (80 pairs per query) 13.6 vs 14.4.
 constexpr double kFusedMinPairsPerQuery = 90.0;
+// ... and without any sample when the grid's candidate tests per query are clearly in the
+// single pass's regime (C2 eps 0.45: 1,128, eps 1.40: 6,280; C5: 224, C2 eps 0.15: 245) and
+// 4 B per test fits in this share of the device memory
+constexpr double kFusedDirectTestsPerQuery = 400.0;
+constexpr double kFusedDirectMemShare = 0.3;
 uint32_t sparse_max_tests() {
     static const uint32_t v = [] {
         const char* e = std::getenv("HDB_SPARSE_TESTS");
@@ -529,7 +534,7 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
         dl = DBuf(4 * (n + 1), s);
         sql = DBuf(8 * (n + 1), s);
         const uint32_t* ngd = gofs.as<uint32_t>() + nne;
-        HDB_CUDA(cudaMemsetAsync(nsp, 0, 8, s));
+        HDB_CUDA(cudaMemsetAsync(nsp, 0, 16, s));   // [0] sparse queries, [1] candidate tests
         launch_group_class(g.cstart, g.cspan, g.nspan, g.gstart, g.gcell, ngd, n, max_tests, dflag.as<uint32_t>(),
                            sqn.as<uint32_t>(), nsp, (uint8_t*)gbin.p, ohist.as<uint32_t>(), s);
         launch_order_scatter((const uint8_t*)gbin.p, ngd, n, ohist.as<uint32_t>(), ord.as<uint32_t>(), s);
@@ -545,13 +550,13 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
         scan_u32_to_u64(words.as<uint32_t>(), moff.as<uint64_t>(), n, mtemp.p, s);
         HDB_LAUNCH_CHECK();
         uint64_t* pr = dc.pin + 17;   // [17] groups, [18] mask words, [19] dense groups, [20] sparse queries
-        pr[0] = pr[1] = pr[2] = pr[3] = pr[4] = 0;   //   (pinned: asynchronous readbacks), [21] sparse count
+        pr[0] = pr[1] = pr[2] = pr[3] = pr[4] = pr[5] = 0;   // (pinned), [21] sparse count, [22] tests
         HDB_CUDA(cudaMemcpyAsync(&pr[0], gofs.as<uint32_t>() + nne, 4, cudaMemcpyDeviceToHost, s));
         HDB_CUDA(cudaMemcpyAsync(&pr[1], moff.as<uint64_t>() + n, 8, cudaMemcpyDeviceToHost, s));
         if (classify) {
             HDB_CUDA(cudaMemcpyAsync(&pr[2], dpre.as<uint32_t>() + n, 4, cudaMemcpyDeviceToHost, s));
             HDB_CUDA(cudaMemcpyAsync(&pr[3], spre.as<uint32_t>() + n, 4, cudaMemcpyDeviceToHost, s));
-            HDB_CUDA(cudaMemcpyAsync(&pr[4], nsp, 8, cudaMemcpyDeviceToHost, s));
+            HDB_CUDA(cudaMemcpyAsync(&pr[4], nsp, 16, cudaMemcpyDeviceToHost, s));   // -> pr[4], pr[5]
         }
         HDB_CUDA(cudaEventRecord(ev1.e, s));
         tr.mark("class+order+masklayout-enqueue");
@@ -560,6 +565,7 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
         g.mask_words = pr[1];
         const uint32_t hds[2] = {(uint32_t)pr[2], (uint32_t)pr[3]};
         const uint64_t hsp = pr[4];
+        g.tests_total = pr[5];
         g.n_groups = hng;
         g.moff = (uint64_t*)moff.release();
         g.n_dense_groups = hng;
@@ -742,7 +748,7 @@ void count_phase(hdb_ctx* ctx, DevCtx& dc, const DevGrid& g, ShardState& st) {
     scan_u32_to_u64(st.cnt.as<uint32_t>() + st.r.q0, st.off.as<uint64_t>() + st.r.q0, len, temp.p, s);
     HDB_LAUNCH_CHECK();
     HDB_CUDA(cudaEventRecord(e2.e, s));
-    uint64_t* h = dc.pin + 22;   // pinned: asynchronous readbacks
+    uint64_t* h = dc.pin + 24;   // pinned: asynchronous readbacks
     HDB_CUDA(cudaMemcpyAsync(&h[0], st.off.as<uint64_t>() + st.r.q1, 8, cudaMemcpyDeviceToHost, s));
     HDB_CUDA(cudaMemcpyAsync(&h[1], tests.p, 8, cudaMemcpyDeviceToHost, s));
     HDB_CUDA(cudaStreamSynchronize(s));
@@ -759,11 +765,15 @@ void count_phase(hdb_ctx* ctx, DevCtx& dc, const DevGrid& g, ShardState& st) {
 // max(a_b, n) + 2^20 pairs).  Returns false -- nothing published, the caller
 // then runs the exact two-pass path (a6-a8) -- if the mask table or the table
 // cannot be allocated or a reservation passed the capacity.
-bool single_pass_table(hdb_ctx* ctx, const DevGrid& g, hdb_table* t, hdb_stats& S, uint64_t est) {
+bool single_pass_table(hdb_ctx* ctx, const DevGrid& g, hdb_table* t, hdb_stats& S, uint64_t est,
+                       bool exact_bound = false) {
     DevCtx& dc = ctx->dev[0];
     cudaStream_t s = dc.main;
     const uint64_t n = g.n;
-    const uint64_t cap = (uint64_t)((double)std::max<uint64_t>(est, n) * 1.25) + (1ull << 20);
+    // est: the sampled estimate a_b (cap with headroom; a reservation past it falls back to
+    // the two passes) or, exact_bound, an upper bound on P (the grid's candidate tests)
+    const uint64_t cap = exact_bound ? std::max<uint64_t>(est, 1)
+                                     : (uint64_t)((double)std::max<uint64_t>(est, n) * 1.25) + (1ull << 20);
     DBuf masks, nb;
     if (cudaMallocFromPoolAsync(&masks.p, 4 * std::max<uint64_t>(g.mask_words, 4), dc.big_pool, s) != cudaSuccess ||
         cudaMallocFromPoolAsync(&nb.p, 4 * cap, dc.big_pool, s) != cudaSuccess) {
@@ -1063,14 +1073,37 @@ void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hd
     std::vector<ShardState> sh(ndev);
     try {
         Trace tr("neighbor_table");
-        // ---- a5: sampled count + plan (device 0)
         DevCtx& dc0 = ctx->dev[0];
         DeviceGuard dg0(dc0.device);
+        const uint32_t parts = R_proc * (uint32_t)ndev;
+        // ---- dense device-resident whole table: the single pass sized by the exact upper
+        // bound P <= candidate tests (known from the grid), no sampled estimate needed (the
+        // sample kernel and its readback sync were ~3% of a C2 step)
+        if (device_resident && parts == 1 && ctx->opts.search_kernel == 0 && n > 0 && !G0.dl &&
+            G0.tests_total >= (uint64_t)(kFusedDirectTestsPerQuery * (double)n) &&
+            4.0 * (double)G0.tests_total <= kFusedDirectMemShare * (double)dc0.total_mem) {
+            S.sample_size = 0;
+            S.sample_pairs = 0;
+            S.est_pairs = 0;
+            S.ms_sample = 0;
+            S.ms_sort = 0;
+            S.planned_batch_pairs = S.planned_batches = 0;
+            if (single_pass_table(ctx, G0, t, S, G0.tests_total, true)) {   // (cannot overflow)
+                tr.mark("single-pass (exact bound)");
+                S.kernel_launches = (uint32_t)(g_kernel_launches.load() - launches0);
+                S.ms_table_wall =
+                    std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_wall0).count();
+                t->ctx = ctx;
+                ctx->live_objects++;
+                *out = t;
+                return;
+            }
+        }
+        // ---- a5: sampled count + plan (device 0)
         const double f = ctx->opts.sample_fraction;
         const uint64_t stride = std::max<uint64_t>(1, (uint64_t)std::floor(1.0 / f));
         const uint64_t ns = n ? (n + stride - 1) / stride : 0;
         std::vector<uint32_t> samp;
-        const uint32_t parts = R_proc * (uint32_t)ndev;
         cudaStream_t s0 = dc0.main;
         DBuf dsamp(4 * (ns ? ns : 1), s0), dsum(8, s0);
         Event es0, es1;

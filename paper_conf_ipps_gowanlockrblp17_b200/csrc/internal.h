@@ -82,6 +82,7 @@ struct DevGrid {
     uint32_t* spre = nullptr;      // [n_groups+1] sparse queries before group g
     uint2* sql = nullptr;          // [n_sparse_q] {sorted position, non-empty cell} of each sparse query
     uint64_t n_sparse_q = 0, n_dense_groups = 0;
+    uint64_t tests_total = 0;      // sum over groups of queries x candidates (0: not computed); >= P
     cudaStream_t stream = nullptr; // stream the buffers were allocated on
     float ms_build = 0;
 };
@@ -120,7 +121,7 @@ void launch_group_build(const uint32_t* cstart, const uint32_t* gofs, uint64_t n
                         uint32_t* gcell, cudaStream_t s);
 // dense/sparse classification of the groups g < *ng_dev (entries up to n): dflag[g] = 1 for a
 // dense group, sqn[g] = its query count for a sparse one (sparse <=> queries x candidates <=
-// max_tests), *n_sparse += the sparse queries; then the lists dl[dpre[g]] = g (dense) and
+// max_tests), n_sparse[0] += the sparse queries, n_sparse[1] += every group's candidate tests; then the lists dl[dpre[g]] = g (dense) and
 // sql[spre[g] + i] = {gstart[g] + i, gcell[g]}
 void launch_group_class(const uint32_t* cstart, const uint2* cspan, uint32_t nspan, const uint32_t* gstart,
                         const uint32_t* gcell, const uint32_t* ng_dev, uint64_t n, uint32_t max_tests,
@@ -211,6 +212,7 @@ struct DevCtx {
     // being carved up by the grid's smaller buffers in the default pool (which
     // made C5 steps map fresh memory: 27 -> 60..120 ms outliers)
     cudaMemPool_t big_pool = nullptr;
+    size_t total_mem = 0;                   // device memory (bytes), for sizing decisions
     // cached per-stream device batch buffers (reused across calls)
     std::vector<uint32_t*> batch_buf;
     std::vector<size_t> batch_cap;

@@ -381,6 +381,7 @@ __global__ void __launch_bounds__(256) k_group_class(const uint32_t* __restrict_
     __syncthreads();
     const uint64_t ng = *ng_dev;
     uint32_t tot = 0;
+    unsigned long long ttot = 0;   // candidate tests of the thread's groups
     for (uint64_t g = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; g < n; g += (uint64_t)gridDim.x * blockDim.x) {
         uint32_t d = 0, sq = 0;
         if (g < ng) {
@@ -392,6 +393,7 @@ __global__ void __launch_bounds__(256) k_group_class(const uint32_t* __restrict_
                 cand += sp.y - sp.x;
             }
             const uint64_t tests = (uint64_t)nq * cand;
+            ttot += tests;
             if (tests <= max_tests) sq = nq;
             else d = 1;
             // cost bin: dense groups first, each class by decreasing log2(tests)
@@ -404,8 +406,12 @@ __global__ void __launch_bounds__(256) k_group_class(const uint32_t* __restrict_
         sqn[g] = sq;
         tot += sq;
     }
-    for (int o = 16; o > 0; o >>= 1) tot += __shfl_xor_sync(0xffffffffu, tot, o);
+    for (int o = 16; o > 0; o >>= 1) {
+        tot += __shfl_xor_sync(0xffffffffu, tot, o);
+        ttot += __shfl_xor_sync(0xffffffffu, ttot, o);
+    }
     if ((threadIdx.x & 31) == 0 && tot) atomicAdd(n_sparse, (unsigned long long)tot);
+    if ((threadIdx.x & 31) == 0 && ttot) atomicAdd(n_sparse + 1, ttot);
     __syncthreads();
     for (int b = threadIdx.x; b < kOrderBins; b += blockDim.x)
         if (sh[b]) atomicAdd(&ohist[b], sh[b]);
