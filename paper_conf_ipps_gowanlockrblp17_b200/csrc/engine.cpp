@@ -365,23 +365,25 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
     DBuf misc(256, s);
     unsigned long long* bb = misc.as<unsigned long long>();          // [0..3] bbox, [4] nonempty
     unsigned int* bad = (unsigned int*)(bb + 5);
-    launch_bbox_init(bb, bad, s);
-    HDB_CUDA(cudaMemsetAsync(bb + 4, 0, 8, s));
-    launch_bbox(xin, n, dt, bb, bad, s);
-    HDB_LAUNCH_CHECK();
-    tr.mark("bbox-enqueue");
     // default cell split: occupancy estimate launched with the bbox, read in the same sync
     const bool auto_k = ctx->opts.cell_split == 0 && n >= 4096;
     DBuf hk, hc, occ;
+    if (auto_k) {
+        hk = DBuf(8ull * kOccTable, s);
+        hc = DBuf(4ull * kOccTable, s);
+        occ = DBuf(16, s);
+    }
+    launch_bbox_init(bb, bad, hk.as<unsigned long long>(), hc.as<unsigned int>(), auto_k ? kOccTable : 0,
+                     occ.as<unsigned long long>(), s);
+    launch_bbox(xin, n, dt, bb, bad, s);
+    HDB_LAUNCH_CHECK();
+    tr.mark("bbox-enqueue");
     // small readbacks go through the context's pinned scratch (pin[8..21]): a D2H copy
     // into pageable memory is synchronous and cost ~30 us each here
     unsigned long long* hocc = (unsigned long long*)dc.pin + 8;
     hocc[0] = hocc[1] = 0;
     if (auto_k) {
         const double eps_pre = dt == HDB_F32 ? (double)(float)eps : eps;
-        hk = DBuf(8ull * kOccTable, s);
-        hc = DBuf(4ull * kOccTable, s);
-        occ = DBuf(16, s);
         const uint64_t m = std::min<uint64_t>(n, kOccSample);
         launch_occ_estimate(xin, n, dt, n / m, m, 1.0 / (eps_pre * (1.0 + 0x1p-19)), hk.as<unsigned long long>(),
                             hc.as<unsigned int>(), kOccTable, occ.as<unsigned long long>(), s);
@@ -452,11 +454,9 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
     DBuf xp(16 * (n / 2 + 2), s);
     DBuf counters(4 * kCounterSlots, s);
     DBuf inv(4 * (n + 1), s);
-    HDB_CUDA(cudaMemsetAsync(xy_s.as<char>() + n * esz, 0, 2 * esz, s));
-    HDB_CUDA(cudaMemsetAsync(ids.as<uint32_t>() + n, 0, 8, s));
-    HDB_CUDA(cudaMemsetAsync(xp.p, 0, 16 * (n / 2 + 2), s));
-    HDB_CUDA(cudaMemsetAsync(counters.p, 0, 4 * kCounterSlots, s));
-    launch_gather_points(xin, ids.as<uint32_t>(), n, dt, xy_s.p, xp.as<float4>(), g.ox, g.oy, inv.as<uint32_t>(), s);
+    // (the gather also zeroes the padding of xy_s / ids / xp and the work counters)
+    launch_gather_points(xin, ids.as<uint32_t>(), n, dt, xy_s.p, xp.as<float4>(), g.ox, g.oy, inv.as<uint32_t>(),
+                         counters.as<unsigned int>(), kCounterSlots, s);
     HDB_LAUNCH_CHECK();
     xin_owned.reset();
     tr.mark("keys+sort+gather(enqueue)");

@@ -89,7 +89,9 @@ struct DevGrid {
 
 // ---------------------------------------------------------------- kernels
 // grid build (kernels_grid.cu)
-void launch_bbox_init(unsigned long long* bb, unsigned int* bad, cudaStream_t s);
+// bbox sentinels + bad counter + bb[4]; with hkey: the occupancy hash table (tsize entries) and occ[0..1]
+void launch_bbox_init(unsigned long long* bb, unsigned int* bad, unsigned long long* hkey, unsigned int* hcnt,
+                      uint32_t tsize, unsigned long long* occ, cudaStream_t s);
 void launch_bbox(const void* xy, uint64_t n, hdb_dtype dt, unsigned long long* bb, unsigned int* bad,
                  cudaStream_t s);
 double bbox_decode(unsigned long long v, bool is_max);
@@ -102,8 +104,9 @@ size_t radix_sort_temp_bytes(uint64_t n);
 int radix_sort_pairs(void* k0, uint32_t* v0, void* k1, uint32_t* v1, int key_bytes, uint64_t n, int bits,
                      void* temp, cudaStream_t s);
 // gather sorted points; f64 mode also writes the f32 filter coordinates (x-ox, y-oy)
-void launch_gather_points(const void* xy_in, const uint32_t* ids, uint64_t n, hdb_dtype dt, void* xy_s,
-                          float4* xp, double ox, double oy, uint32_t* inv, cudaStream_t s);
+void launch_gather_points(const void* xy_in, uint32_t* ids, uint64_t n, hdb_dtype dt, void* xy_s, float4* xp,
+                          double ox, double oy, uint32_t* inv, unsigned int* counters, uint32_t n_counters,
+                          cudaStream_t s);
 void launch_cell_flags(const void* keys_sorted, int key_bytes, uint64_t n, uint32_t* flags, cudaStream_t s);
 void launch_cell_scatter(const void* keys_sorted, int key_bytes, const uint32_t* flags, const uint32_t* pos,
                          uint64_t n, uint64_t* ckey, uint32_t* cstart, cudaStream_t s);

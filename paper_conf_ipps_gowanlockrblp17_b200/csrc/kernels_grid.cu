@@ -50,12 +50,24 @@ struct V2<float> {
     using type = float2;
 };
 
-__global__ void k_bbox_init(unsigned long long* bb, unsigned int* bad) {
-    bb[0] = ~0ull;  // xmin (ordered min)
-    bb[1] = ~0ull;  // ymin
-    bb[2] = 0ull;   // xmax (ordered max)
-    bb[3] = 0ull;   // ymax
-    *bad = 0;
+// One launch initialises the bbox reduction and the occupancy-estimate hash table
+// (it replaced a kernel + four memsets: each stream op costs ~2-5 us at C2 sizes)
+__global__ void k_bbox_init(unsigned long long* bb, unsigned int* bad, unsigned long long* hkey,
+                            unsigned int* hcnt, uint32_t tsize, unsigned long long* occ) {
+    const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i == 0) {
+        bb[0] = ~0ull;  // xmin (ordered min)
+        bb[1] = ~0ull;  // ymin
+        bb[2] = 0ull;   // xmax (ordered max)
+        bb[3] = 0ull;   // ymax
+        bb[4] = 0ull;
+        *bad = 0;
+        if (occ) occ[0] = occ[1] = 0;
+    }
+    for (uint32_t j = i; j < tsize; j += gridDim.x * blockDim.x) {
+        hkey[j] = ~0ull;
+        hcnt[j] = 0;
+    }
 }
 
 template <typename T>
@@ -239,10 +251,24 @@ template <typename T>
 __global__ void __launch_bounds__(256) k_gather(const typename V2<T>::type* __restrict__ in,
                                                 const uint32_t* __restrict__ ids, uint64_t n,
                                                 typename V2<T>::type* __restrict__ out, float4* __restrict__ xp,
-                                                double ox, double oy, uint32_t* __restrict__ inv) {
+                                                double ox, double oy, uint32_t* __restrict__ inv,
+                                                uint32_t* __restrict__ ids_pad, unsigned int* __restrict__ counters,
+                                                uint32_t n_counters) {
     // xp: paired-SoA f32 copy {x_2k, x_2k+1, y_2k, y_2k+1} -- f64 input: filter
     // coordinates fl32(fl64(x - ox)); f32 input: the exact coordinates
     float* xpf = (float*)xp;
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        // padding read by the candidate-pair loads (2 entries past n) and the work
+        // counters -- zeroed here instead of by four memsets
+        out[n] = out[n + 1] = typename V2<T>::type{0, 0};
+        ids_pad[0] = ids_pad[1] = 0;
+        for (uint64_t s = n; s < 2 * (n / 2 + 2); ++s) {
+            const uint64_t k = s >> 1, o = s & 1;
+            xpf[4 * k + o] = 0.f;
+            xpf[4 * k + 2 + o] = 0.f;
+        }
+        for (uint32_t c = 0; c < n_counters; ++c) counters[c] = 0;
+    }
     for (uint64_t s = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; s < n;
          s += (uint64_t)gridDim.x * blockDim.x) {
         const uint32_t id = ids[s];
@@ -545,8 +571,9 @@ double bbox_decode(unsigned long long v, bool) {
     return d;
 }
 
-void launch_bbox_init(unsigned long long* bb, unsigned int* bad, cudaStream_t s) {
-    k_bbox_init<<<1, 1, 0, s>>>(bb, bad);
+void launch_bbox_init(unsigned long long* bb, unsigned int* bad, unsigned long long* hkey, unsigned int* hcnt,
+                      uint32_t tsize, unsigned long long* occ, cudaStream_t s) {
+    k_bbox_init<<<tsize ? (tsize + 255) / 256 : 1, 256, 0, s>>>(bb, bad, hkey, hcnt, tsize, occ);
     ++g_kernel_launches;
 }
 
@@ -616,13 +643,16 @@ int radix_sort_pairs(void* k0, uint32_t* v0, void* k1, uint32_t* v1, int key_byt
     return radix_sort_impl<uint64_t>((uint64_t*)k0, v0, (uint64_t*)k1, v1, n, bits, temp, s);
 }
 
-void launch_gather_points(const void* xy_in, const uint32_t* ids, uint64_t n, hdb_dtype dt, void* xy_s, float4* xp,
-                          double ox, double oy, uint32_t* inv, cudaStream_t s) {
-    if (n == 0) return;
+void launch_gather_points(const void* xy_in, uint32_t* ids, uint64_t n, hdb_dtype dt, void* xy_s, float4* xp,
+                          double ox, double oy, uint32_t* inv, unsigned int* counters, uint32_t n_counters,
+                          cudaStream_t s) {
+    const unsigned blocks = n ? grid_for(n) : 1;
     if (dt == HDB_F64)
-        k_gather<double><<<grid_for(n), 256, 0, s>>>((const double2*)xy_in, ids, n, (double2*)xy_s, xp, ox, oy, inv);
+        k_gather<double><<<blocks, 256, 0, s>>>((const double2*)xy_in, ids, n, (double2*)xy_s, xp, ox, oy, inv,
+                                                ids + n, counters, n_counters);
     else
-        k_gather<float><<<grid_for(n), 256, 0, s>>>((const float2*)xy_in, ids, n, (float2*)xy_s, xp, 0, 0, inv);
+        k_gather<float><<<blocks, 256, 0, s>>>((const float2*)xy_in, ids, n, (float2*)xy_s, xp, 0, 0, inv, ids + n,
+                                               counters, n_counters);
     ++g_kernel_launches;
 }
 
@@ -691,9 +721,7 @@ void launch_group_lists(const uint32_t* gstart, const uint32_t* gcell, const uin
 void launch_occ_estimate(const void* xy, uint64_t n, hdb_dtype dt, uint64_t stride, uint64_t m, double inv_w,
                          unsigned long long* hkey, unsigned int* hcnt, uint32_t tsize, unsigned long long* out,
                          cudaStream_t s) {
-    cudaMemsetAsync(hkey, 0xff, sizeof(unsigned long long) * tsize, s);
-    cudaMemsetAsync(hcnt, 0, sizeof(unsigned int) * tsize, s);
-    cudaMemsetAsync(out, 0, 2 * sizeof(unsigned long long), s);
+    // hkey / hcnt / out were initialised by launch_bbox_init
     if (m) {
         if (dt == HDB_F64)
             k_occ_sample<double><<<grid_for(m), 256, 0, s>>>((const double2*)xy, n, stride, m, inv_w, hkey, hcnt,
