@@ -112,6 +112,9 @@ hdb_status hdb_ctx_create(const hdb_opts* opts, hdb_ctx** out) {
         HDB_CUDA(cudaMemPoolCreate(&dc.big_pool, &props));
         size_t free_b = 0;
         HDB_CUDA(cudaMemGetInfo(&free_b, &dc.total_mem));
+        dc.scan_ep.cap = 1u << 20;   // tiles of 2,048 elements: scans of up to 2^31 elements
+        HDB_CUDA(cudaMalloc((void**)&dc.scan_ep.tiles, dc.scan_ep.cap * sizeof(unsigned long long)));
+        HDB_CUDA(cudaMemset(dc.scan_ep.tiles, 0, dc.scan_ep.cap * sizeof(unsigned long long)));
         HDB_CUDA(cudaMemPoolSetAttribute(dc.big_pool, cudaMemPoolAttrReleaseThreshold, &thr));
         c->dev.push_back(dc);
     }
@@ -144,6 +147,7 @@ void hdb_ctx_destroy(hdb_ctx* c) {
         for (auto s : dc.streams) cudaStreamDestroy(s);
         if (dc.main && dc.own_main) cudaStreamDestroy(dc.main);
         if (dc.pin) cudaFreeHost(dc.pin);
+        if (dc.scan_ep.tiles) cudaFree(dc.scan_ep.tiles);
         // tables still alive keep their blocks: the pool is then left to process exit
         if (dc.big_pool && c->live_objects == 0) cudaMemPoolDestroy(dc.big_pool);
     }

@@ -347,6 +347,7 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
     HDB_CUDA(cudaEventRecord(ev0.e, s));
 
     Trace tr("grid_build");
+    ScanEpochScope scan_scope(&dc.scan_ep);   // the build's scans: no status memsets
     // ---- a1: ingest + bbox + validation
     DBuf xin_owned;
     const void* xin = xy;
@@ -694,6 +695,7 @@ std::vector<uint64_t> shard_cuts(const DevGrid& g, DevCtx& dc, const std::vector
 
 // a6 + a7 on one device for one shard
 void count_phase(hdb_ctx* ctx, DevCtx& dc, const DevGrid& g, ShardState& st) {
+    ScanEpochScope scan_scope(&dc.scan_ep);
     DeviceGuard dg(dc.device);
     Trace tr("count_phase");
     cudaStream_t s = dc.main;

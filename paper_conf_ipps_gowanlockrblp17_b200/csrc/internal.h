@@ -140,6 +140,20 @@ void launch_group_lists(const uint32_t* gstart, const uint32_t* gcell, const uin
 
 // scans (kernels_scan.cu): exclusive scan of in[0..n) into out[0..n], out[n] = total
 size_t scan_temp_bytes(uint64_t n);
+// Per-device tile-status buffer for memset-free scans (zeroed once, one epoch per scan).
+// Scans issued by a thread while a ScanEpochScope is alive use it (all on one stream: the
+// scans of one scope must not run concurrently); others zero their status tiles in temp.
+struct ScanEpochs {
+    unsigned long long* tiles = nullptr;
+    uint64_t cap = 0;      // tiles
+    uint32_t epoch = 0;    // last epoch used
+};
+extern thread_local ScanEpochs* t_scan_epochs;
+struct ScanEpochScope {
+    ScanEpochs* prev;
+    explicit ScanEpochScope(ScanEpochs* e) : prev(t_scan_epochs) { t_scan_epochs = e; }
+    ~ScanEpochScope() { t_scan_epochs = prev; }
+};
 void scan_u32_to_u32(const uint32_t* in, uint32_t* out, uint64_t n, void* temp, cudaStream_t s);
 void scan_u32_to_u64(const uint32_t* in, uint64_t* out, uint64_t n, void* temp, cudaStream_t s);
 
@@ -216,6 +230,7 @@ struct DevCtx {
     // made C5 steps map fresh memory: 27 -> 60..120 ms outliers)
     cudaMemPool_t big_pool = nullptr;
     size_t total_mem = 0;                   // device memory (bytes), for sizing decisions
+    ScanEpochs scan_ep;                     // memset-free scans of the grid build / count phase
     // cached per-stream device batch buffers (reused across calls)
     std::vector<uint32_t*> batch_buf;
     std::vector<size_t> batch_cap;

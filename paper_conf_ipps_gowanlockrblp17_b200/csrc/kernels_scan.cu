@@ -26,7 +26,14 @@ constexpr int SC_TILE = SC_THREADS * SC_ITEMS;
 // summing aggregates until it meets an inclusive prefix.  Tiles are blockIdx
 // ordered and only wait on lower tiles, which the hardware dispatched first.
 // One kernel per scan (plus a memset of the tile words).
-constexpr uint64_t kStAgg = 1ull << 62, kStPre = 2ull << 62, kValMask = (1ull << 62) - 1;
+// Tile status word: flag (2 bits: aggregate / inclusive prefix) | epoch (20 bits) | value (42 bits).
+// A word is ready only with a flag and the scan's own epoch: memset-path scans use epoch 0 on a
+// zeroed buffer; epoch scans (ScanEpochScope) reuse one zeroed per-device buffer with a new
+// epoch per call and need no memset.  Values stay < 2^42 (counts of points / pairs / mask words
+// bounded by device memory).
+constexpr uint64_t kStAgg = 1ull << 62, kStPre = 2ull << 62, kValMask = (1ull << 42) - 1;
+constexpr int kEpShift = 42;
+constexpr uint64_t kEpMask = (1ull << 20) - 1;
 
 __device__ __forceinline__ void publish(unsigned long long* w, uint64_t v) {
     asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(w), "l"(v) : "memory");
@@ -39,7 +46,8 @@ __device__ __forceinline__ uint64_t peek(const unsigned long long* w) {
 
 template <typename Tin, typename Tout>
 __global__ void __launch_bounds__(SC_THREADS) k_scan_lookback(const Tin* __restrict__ in, Tout* __restrict__ out,
-                                                              uint64_t n, unsigned long long* __restrict__ tiles) {
+                                                              uint64_t n, unsigned long long* __restrict__ tiles,
+                                                              uint64_t ep) {
     __shared__ Tout buf[SC_TILE];
     __shared__ Tout wsum[SC_THREADS / 32];
     __shared__ Tout s_excl;
@@ -77,15 +85,17 @@ __global__ void __launch_bounds__(SC_THREADS) k_scan_lookback(const Tin* __restr
     if (w == 0) {
         Tout excl = 0;
         if (t == 0) {
-            if (lane == 0 && tiles) publish(&tiles[0], kStPre | (uint64_t)tot);
+            if (lane == 0 && tiles) publish(&tiles[0], kStPre | ep | (uint64_t)tot);
         } else {
-            if (lane == 0) publish(&tiles[t], kStAgg | (uint64_t)tot);
+            if (lane == 0) publish(&tiles[t], kStAgg | ep | (uint64_t)tot);
             int64_t pred = (int64_t)t - 1;
             while (true) {
                 const int64_t j = pred - lane;
-                uint64_t word = j >= 0 ? peek(&tiles[j]) : kStPre;   // before tile 0: prefix 0
-                while (__any_sync(FULL, (word >> 62) == 0)) {          // wait for every predecessor in view
-                    if ((word >> 62) == 0) word = peek(&tiles[j]);
+                // before tile 0: prefix 0; a word of another epoch counts as not yet published
+                auto ready = [&](uint64_t wd) { return (wd >> 62) != 0 && (wd & (kEpMask << kEpShift)) == ep; };
+                uint64_t word = j >= 0 ? peek(&tiles[j]) : (kStPre | ep);
+                while (__any_sync(FULL, !ready(word))) {               // wait for every predecessor in view
+                    if (!ready(word)) word = peek(&tiles[j]);
                 }
                 const unsigned pre = __ballot_sync(FULL, (word >> 62) == 2);
                 const int first = pre ? __ffs(pre) - 1 : 32;           // nearest inclusive prefix
@@ -96,7 +106,7 @@ __global__ void __launch_bounds__(SC_THREADS) k_scan_lookback(const Tin* __restr
                 if (pre) break;
                 pred -= 32;
             }
-            if (lane == 0) publish(&tiles[t], kStPre | (uint64_t)(excl + tot));
+            if (lane == 0) publish(&tiles[t], kStPre | ep | (uint64_t)(excl + tot));
         }
         if (lane == 0) s_excl = excl;
     }
@@ -121,15 +131,28 @@ void scan_impl(const Tin* in, Tout* out, uint64_t n, void* temp, cudaStream_t s)
     }
     const uint64_t nb = (n + SC_TILE - 1) / SC_TILE;
     unsigned long long* tiles = nullptr;
+    uint64_t ep = 0;
     if (nb > 1) {
-        tiles = (unsigned long long*)temp;
-        cudaMemsetAsync(tiles, 0, nb * sizeof(unsigned long long), s);
+        ScanEpochs* se = t_scan_epochs;
+        if (se && nb <= se->cap) {
+            if (++se->epoch > kEpMask) {   // epochs wrap: start again on a zeroed buffer
+                cudaMemsetAsync(se->tiles, 0, se->cap * sizeof(unsigned long long), s);
+                se->epoch = 1;
+            }
+            tiles = se->tiles;
+            ep = (uint64_t)se->epoch << kEpShift;
+        } else {
+            tiles = (unsigned long long*)temp;
+            cudaMemsetAsync(tiles, 0, nb * sizeof(unsigned long long), s);
+        }
     }
-    k_scan_lookback<Tin, Tout><<<(unsigned)nb, SC_THREADS, 0, s>>>(in, out, n, tiles);
+    k_scan_lookback<Tin, Tout><<<(unsigned)nb, SC_THREADS, 0, s>>>(in, out, n, tiles, ep);
     ++g_kernel_launches;
 }
 
 }  // namespace
+
+thread_local ScanEpochs* t_scan_epochs = nullptr;
 
 size_t scan_temp_bytes(uint64_t n) {
     return ((n + SC_TILE - 1) / SC_TILE + 1) * sizeof(unsigned long long) + 64;
