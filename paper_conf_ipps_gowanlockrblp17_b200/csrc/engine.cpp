@@ -363,41 +363,40 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
             xin = xin_owned.p;
         }
     }
-    DBuf misc(256, s);
-    unsigned long long* bb = misc.as<unsigned long long>();          // [0..3] bbox, [4] nonempty
+    // misc (1 KB, zeroed by the bbox init except the bbox sentinels): [0..3] bbox, [4] nonempty,
+    // [5] bad count, [6..7] occupancy sums, [8..9] sparse queries / candidate tests,
+    // [16..21] readbacks of the group phase, [32..95] cost-order histogram + cursors
+    constexpr uint32_t kMiscWords = 128;
+    DBuf misc(8 * kMiscWords, s);
+    unsigned long long* bb = misc.as<unsigned long long>();
     unsigned int* bad = (unsigned int*)(bb + 5);
     // default cell split: occupancy estimate launched with the bbox, read in the same sync
     const bool auto_k = ctx->opts.cell_split == 0 && n >= 4096;
-    DBuf hk, hc, occ;
+    DBuf hk, hc;
     if (auto_k) {
         hk = DBuf(8ull * kOccTable, s);
         hc = DBuf(4ull * kOccTable, s);
-        occ = DBuf(16, s);
     }
-    launch_bbox_init(bb, bad, hk.as<unsigned long long>(), hc.as<unsigned int>(), auto_k ? kOccTable : 0,
-                     occ.as<unsigned long long>(), s);
+    launch_bbox_init(bb, kMiscWords, hk.as<unsigned long long>(), hc.as<unsigned int>(), auto_k ? kOccTable : 0, s);
     launch_bbox(xin, n, dt, bb, bad, s);
     HDB_LAUNCH_CHECK();
     tr.mark("bbox-enqueue");
-    // small readbacks go through the context's pinned scratch (pin[8..21]): a D2H copy
+    // small readbacks go through the context's pinned scratch (pin[10..23]): a D2H copy
     // into pageable memory is synchronous and cost ~30 us each here
-    unsigned long long* hocc = (unsigned long long*)dc.pin + 8;
-    hocc[0] = hocc[1] = 0;
+    unsigned long long* hb = (unsigned long long*)dc.pin + 10;   // bb[0..7] -> pin[10..17]
+    const unsigned long long* hocc = hb + 6;
     if (auto_k) {
         const double eps_pre = dt == HDB_F32 ? (double)(float)eps : eps;
         const uint64_t m = std::min<uint64_t>(n, kOccSample);
         launch_occ_estimate(xin, n, dt, n / m, m, 1.0 / (eps_pre * (1.0 + 0x1p-19)), hk.as<unsigned long long>(),
-                            hc.as<unsigned int>(), kOccTable, occ.as<unsigned long long>(), s);
+                            hc.as<unsigned int>(), kOccTable, bb + 6, s);
         HDB_LAUNCH_CHECK();
-        HDB_CUDA(cudaMemcpyAsync(hocc, occ.p, 16, cudaMemcpyDeviceToHost, s));
     }
-    unsigned long long* hb = (unsigned long long*)dc.pin + 10;   // [10..15]
-    HDB_CUDA(cudaMemcpyAsync(hb, bb, 48, cudaMemcpyDeviceToHost, s));
+    HDB_CUDA(cudaMemcpyAsync(hb, bb, 64, cudaMemcpyDeviceToHost, s));
     tr.mark("occ-enqueue");
     HDB_CUDA(cudaStreamSynchronize(s));
     hk.reset();
     hc.reset();
-    occ.reset();
     if ((unsigned int)hb[5] != 0) fail(HDB_EINVAL, "%u non-finite coordinate(s)", (unsigned)hb[5]);
 
     double eps_used = eps;
@@ -466,7 +465,7 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
     launch_cell_flags(keys.p, kb, n, flags.as<uint32_t>(), s);
     scan_u32_to_u32(flags.as<uint32_t>(), pos.as<uint32_t>(), n, temp.p, s);
     HDB_LAUNCH_CHECK();
-    uint32_t* hne_p = (uint32_t*)(dc.pin + 16);
+    uint32_t* hne_p = (uint32_t*)(dc.pin + 26);
     *hne_p = 0;
     HDB_CUDA(cudaMemcpyAsync(hne_p, pos.as<uint32_t>() + n, 4, cudaMemcpyDeviceToHost, s));
     HDB_CUDA(cudaStreamSynchronize(s));
@@ -526,19 +525,21 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
     const uint32_t max_tests = sparse_max_tests();
     const bool classify = (sk == 0 || sk == 1 || sk == 2 || sk == 4) && max_tests > 0 && n > 0;
     DBuf dpre, spre, dl, sql, ord;
+    DBuf words(4 * (n + 1), s);   // hit-mask words per group (written with the classification)
     unsigned long long* nsp = bb + 8;
     if (classify) {
-        DBuf dflag(4 * (n + 1), s), sqn(4 * (n + 1), s), gbin(n + 1, s), ohist(8 * kOrderBins, s);
+        DBuf dflag(4 * (n + 1), s), sqn(4 * (n + 1), s), gbin(n + 1, s);
+        uint32_t* ohist = (uint32_t*)(bb + 32);   // 2 x kOrderBins words, zeroed by the bbox init
         ord = DBuf(4 * (n + 1), s);
         dpre = DBuf(4 * (n + 1), s);
         spre = DBuf(4 * (n + 1), s);
         dl = DBuf(4 * (n + 1), s);
         sql = DBuf(8 * (n + 1), s);
         const uint32_t* ngd = gofs.as<uint32_t>() + nne;
-        HDB_CUDA(cudaMemsetAsync(nsp, 0, 16, s));   // [0] sparse queries, [1] candidate tests
+        // nsp: [0] sparse queries, [1] candidate tests (zeroed by the bbox init)
         launch_group_class(g.cstart, g.cspan, g.nspan, g.gstart, g.gcell, ngd, n, max_tests, dflag.as<uint32_t>(),
-                           sqn.as<uint32_t>(), nsp, (uint8_t*)gbin.p, ohist.as<uint32_t>(), s);
-        launch_order_scatter((const uint8_t*)gbin.p, ngd, n, ohist.as<uint32_t>(), ord.as<uint32_t>(), s);
+                           sqn.as<uint32_t>(), nsp, (uint8_t*)gbin.p, ohist, words.as<uint32_t>(), kMaskWin, s);
+        launch_order_scatter((const uint8_t*)gbin.p, ngd, n, ohist, ord.as<uint32_t>(), s);
         scan_u32_to_u32(dflag.as<uint32_t>(), dpre.as<uint32_t>(), n, temp.p, s);
         scan_u32_to_u32(sqn.as<uint32_t>(), spre.as<uint32_t>(), n, temp.p, s);
         launch_group_lists(g.gstart, g.gcell, ngd, n, dpre.as<uint32_t>(), spre.as<uint32_t>(), dl.as<uint32_t>(),
@@ -546,19 +547,17 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
         HDB_LAUNCH_CHECK();
     }
     {
-        DBuf words(4 * (n + 1), s), mtemp(scan_temp_bytes(n + 1), s), moff(8 * (n + 1), s);
-        launch_mask_words(g, gofs.as<uint32_t>() + nne, n, words.as<uint32_t>(), s);
+        DBuf mtemp(scan_temp_bytes(n + 1), s), moff(8 * (n + 1), s);
+        if (!classify) launch_mask_words(g, gofs.as<uint32_t>() + nne, n, words.as<uint32_t>(), s);
         scan_u32_to_u64(words.as<uint32_t>(), moff.as<uint64_t>(), n, mtemp.p, s);
         HDB_LAUNCH_CHECK();
-        uint64_t* pr = dc.pin + 17;   // [17] groups, [18] mask words, [19] dense groups, [20] sparse queries
-        pr[0] = pr[1] = pr[2] = pr[3] = pr[4] = pr[5] = 0;   // (pinned), [21] sparse count, [22] tests
-        HDB_CUDA(cudaMemcpyAsync(&pr[0], gofs.as<uint32_t>() + nne, 4, cudaMemcpyDeviceToHost, s));
-        HDB_CUDA(cudaMemcpyAsync(&pr[1], moff.as<uint64_t>() + n, 8, cudaMemcpyDeviceToHost, s));
-        if (classify) {
-            HDB_CUDA(cudaMemcpyAsync(&pr[2], dpre.as<uint32_t>() + n, 4, cudaMemcpyDeviceToHost, s));
-            HDB_CUDA(cudaMemcpyAsync(&pr[3], spre.as<uint32_t>() + n, 4, cudaMemcpyDeviceToHost, s));
-            HDB_CUDA(cudaMemcpyAsync(&pr[4], nsp, 16, cudaMemcpyDeviceToHost, s));   // -> pr[4], pr[5]
-        }
+        // [18] groups, [19] mask words, [20] dense groups, [21] sparse queries, [22] sparse count,
+        // [23] candidate tests: gathered on the device, one pinned readback
+        launch_readback(bb + 16, gofs.as<uint32_t>() + nne, moff.as<uint64_t>() + n,
+                        classify ? dpre.as<uint32_t>() + n : nullptr, classify ? spre.as<uint32_t>() + n : nullptr,
+                        classify ? nsp : nullptr, s);
+        uint64_t* pr = dc.pin + 18;
+        HDB_CUDA(cudaMemcpyAsync(pr, bb + 16, 48, cudaMemcpyDeviceToHost, s));
         HDB_CUDA(cudaEventRecord(ev1.e, s));
         tr.mark("class+order+masklayout-enqueue");
         HDB_CUDA(cudaEventSynchronize(ev1.e));

@@ -89,9 +89,12 @@ struct DevGrid {
 
 // ---------------------------------------------------------------- kernels
 // grid build (kernels_grid.cu)
-// bbox sentinels + bad counter + bb[4]; with hkey: the occupancy hash table (tsize entries) and occ[0..1]
-void launch_bbox_init(unsigned long long* bb, unsigned int* bad, unsigned long long* hkey, unsigned int* hcnt,
-                      uint32_t tsize, unsigned long long* occ, cudaStream_t s);
+// bbox sentinels bb[0..3], zeroes bb[4..nz); with hkey: the occupancy hash table (tsize entries)
+void launch_bbox_init(unsigned long long* bb, uint32_t nz, unsigned long long* hkey, unsigned int* hcnt,
+                      uint32_t tsize, cudaStream_t s);
+// the grid build's readbacks in one place: out[0..5] = *ng, *mw, *dn, *sn, sp[0], sp[1] (null -> 0)
+void launch_readback(unsigned long long* out, const uint32_t* ng, const uint64_t* mw, const uint32_t* dn,
+                     const uint32_t* sn, const unsigned long long* sp, cudaStream_t s);
 void launch_bbox(const void* xy, uint64_t n, hdb_dtype dt, unsigned long long* bb, unsigned int* bad,
                  cudaStream_t s);
 double bbox_decode(unsigned long long v, bool is_max);
@@ -129,10 +132,12 @@ void launch_group_build(const uint32_t* cstart, const uint32_t* gofs, uint64_t n
 void launch_group_class(const uint32_t* cstart, const uint2* cspan, uint32_t nspan, const uint32_t* gstart,
                         const uint32_t* gcell, const uint32_t* ng_dev, uint64_t n, uint32_t max_tests,
                         uint32_t* dflag, uint32_t* sqn, unsigned long long* n_sparse, uint8_t* gbin,
-                        uint32_t* ohist, cudaStream_t s);
+                        uint32_t* ohist, uint32_t* words, uint32_t win, cudaStream_t s);
 // cost order: ord = the groups by gbin (dense groups first, heaviest first); ohist holds
-// 2 * kOrderBins words (bin sizes from launch_group_class, then cursors)
+// 2 * kOrderBins words (bin sizes from launch_group_class, then cursors; zeroed by the caller);
+// launch_group_class also writes the hit-mask words per group (windows of win chunks)
 constexpr int kOrderBins = 64;
+constexpr int kMaskWin = 8;   // chunks per window of the hit-mask layout (kernels_search.cu kWin)
 void launch_order_scatter(const uint8_t* gbin, const uint32_t* ng_dev, uint64_t n, uint32_t* ohist, uint32_t* ord,
                           cudaStream_t s);
 void launch_group_lists(const uint32_t* gstart, const uint32_t* gcell, const uint32_t* ng_dev, uint64_t n,

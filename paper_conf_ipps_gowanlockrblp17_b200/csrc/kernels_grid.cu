@@ -24,6 +24,8 @@
 #include <string.h>
 #include <stdint.h>
 
+#include <algorithm>
+
 #include "internal.h"
 
 namespace hdb {
@@ -50,20 +52,20 @@ struct V2<float> {
     using type = float2;
 };
 
-// One launch initialises the bbox reduction and the occupancy-estimate hash table
-// (it replaced a kernel + four memsets: each stream op costs ~2-5 us at C2 sizes)
-__global__ void k_bbox_init(unsigned long long* bb, unsigned int* bad, unsigned long long* hkey,
-                            unsigned int* hcnt, uint32_t tsize, unsigned long long* occ) {
+// One launch initialises the bbox reduction, the zeroed words of the build's misc
+// buffer (bb[4..nz): counters, occupancy sums, cost histogram) and the
+// occupancy-estimate hash table (it replaced a kernel + six memsets: each stream
+// op costs several us at C2 sizes)
+__global__ void k_bbox_init(unsigned long long* bb, uint32_t nz, unsigned long long* hkey, unsigned int* hcnt,
+                            uint32_t tsize) {
     const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
     if (i == 0) {
         bb[0] = ~0ull;  // xmin (ordered min)
         bb[1] = ~0ull;  // ymin
         bb[2] = 0ull;   // xmax (ordered max)
         bb[3] = 0ull;   // ymax
-        bb[4] = 0ull;
-        *bad = 0;
-        if (occ) occ[0] = occ[1] = 0;
     }
+    if (i >= 4 && i < nz) bb[i] = 0ull;
     for (uint32_t j = i; j < tsize; j += gridDim.x * blockDim.x) {
         hkey[j] = ~0ull;
         hcnt[j] = 0;
@@ -401,7 +403,8 @@ __global__ void __launch_bounds__(256) k_group_class(const uint32_t* __restrict_
                                                      uint32_t max_tests, uint32_t* __restrict__ dflag,
                                                      uint32_t* __restrict__ sqn,
                                                      unsigned long long* __restrict__ n_sparse,
-                                                     uint8_t* __restrict__ gbin, uint32_t* __restrict__ ohist) {
+                                                     uint8_t* __restrict__ gbin, uint32_t* __restrict__ ohist,
+                                                     uint32_t* __restrict__ words, uint32_t win) {
     __shared__ uint32_t sh[kOrderBins];
     for (int b = threadIdx.x; b < kOrderBins; b += blockDim.x) sh[b] = 0;
     __syncthreads();
@@ -414,10 +417,14 @@ __global__ void __launch_bounds__(256) k_group_class(const uint32_t* __restrict_
             const uint32_t qs = gstart[g], c = gcell[g];
             const uint32_t nq = min((uint32_t)kGroup, cstart[c + 1] - qs);
             uint64_t cand = 0;
+            uint32_t npairs = 0;   // candidate pairs of the virtual chunk sequence (mask layout)
             for (uint32_t r = 0; r < nspan; ++r) {
                 const uint2 sp = cspan[(uint64_t)nspan * c + r];
                 cand += sp.y - sp.x;
+                if (sp.y > sp.x) npairs += ((sp.y + 1) >> 1) - (sp.x >> 1);
             }
+            const uint32_t ch = (npairs + 31) / 32;
+            words[g] = 2 * nq * win * ((ch + win - 1) / win);
             const uint64_t tests = (uint64_t)nq * cand;
             ttot += tests;
             if (tests <= max_tests) sq = nq;
@@ -428,6 +435,7 @@ __global__ void __launch_bounds__(256) k_group_class(const uint32_t* __restrict_
             gbin[g] = (uint8_t)b;
             atomicAdd(&sh[b], 1u);
         }
+        if (g >= ng) words[g] = 0;
         dflag[g] = d;
         sqn[g] = sq;
         tot += sq;
@@ -571,9 +579,25 @@ double bbox_decode(unsigned long long v, bool) {
     return d;
 }
 
-void launch_bbox_init(unsigned long long* bb, unsigned int* bad, unsigned long long* hkey, unsigned int* hcnt,
-                      uint32_t tsize, unsigned long long* occ, cudaStream_t s) {
-    k_bbox_init<<<tsize ? (tsize + 255) / 256 : 1, 256, 0, s>>>(bb, bad, hkey, hcnt, tsize, occ);
+void launch_bbox_init(unsigned long long* bb, uint32_t nz, unsigned long long* hkey, unsigned int* hcnt,
+                      uint32_t tsize, cudaStream_t s) {
+    const uint32_t m = std::max(tsize, nz);
+    k_bbox_init<<<(m + 255) / 256, 256, 0, s>>>(bb, nz, hkey, hcnt, tsize);
+    ++g_kernel_launches;
+}
+
+__global__ void k_readback(unsigned long long* out, const uint32_t* ng, const uint64_t* mw, const uint32_t* dn,
+                           const uint32_t* sn, const unsigned long long* sp) {
+    out[0] = *ng;
+    out[1] = *mw;
+    out[2] = dn ? *dn : 0;
+    out[3] = sn ? *sn : 0;
+    out[4] = sp ? sp[0] : 0;
+    out[5] = sp ? sp[1] : 0;
+}
+void launch_readback(unsigned long long* out, const uint32_t* ng, const uint64_t* mw, const uint32_t* dn,
+                     const uint32_t* sn, const unsigned long long* sp, cudaStream_t s) {
+    k_readback<<<1, 1, 0, s>>>(out, ng, mw, dn, sn, sp);
     ++g_kernel_launches;
 }
 
@@ -696,11 +720,10 @@ void launch_group_build(const uint32_t* cstart, const uint32_t* gofs, uint64_t n
 void launch_group_class(const uint32_t* cstart, const uint2* cspan, uint32_t nspan, const uint32_t* gstart,
                         const uint32_t* gcell, const uint32_t* ng_dev, uint64_t n, uint32_t max_tests,
                         uint32_t* dflag, uint32_t* sqn, unsigned long long* n_sparse, uint8_t* gbin,
-                        uint32_t* ohist, cudaStream_t s) {
+                        uint32_t* ohist, uint32_t* words, uint32_t win, cudaStream_t s) {
     if (n == 0) return;
-    cudaMemsetAsync(ohist, 0, 2 * kOrderBins * sizeof(uint32_t), s);
     k_group_class<<<grid_for(n), 256, 0, s>>>(cstart, cspan, nspan, gstart, gcell, ng_dev, n, max_tests, dflag, sqn,
-                                              n_sparse, gbin, ohist);
+                                              n_sparse, gbin, ohist, words, win);
     ++g_kernel_launches;
 }
 

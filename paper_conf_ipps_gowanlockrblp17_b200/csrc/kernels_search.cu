@@ -203,7 +203,7 @@ __device__ __forceinline__ void for_each_group(const SArgs& a, const uint64_t* _
 // contiguously: masks[v][i][kk] (uint2 = even / odd candidate halves).  The
 // write pass then emits query by query inside a window, i.e. in runs of
 // ~kWin * 27 consecutive ids per query (long sequential store streams).
-constexpr int kWin = 8;
+constexpr int kWin = kMaskWin;
 
 constexpr int kWinPad = kWin + 1;   // padded smem rows: 72-B stride, conflict-free per-lane access
 
