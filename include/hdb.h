@@ -81,9 +81,14 @@ typedef struct {
     uint64_t host_budget_bytes; /* 0 = unlimited; else HDB_ENOMEM when 4*P exceeds it                  */
     int shard_rank;             /* process-level query sharding (torchrun mode): this process          */
     int shard_count;            /*   computes shard shard_rank of shard_count; 0 => unsharded          */
-    int search_kernel;          /* 0 = default; other values select kernel variants:
+    int search_kernel;          /* 0 = default: dense device-resident whole tables take the single
+                                   pass (count + reserve + write in one kernel) when the grid's
+                                   candidate tests per query or the sampled pairs per query say
+                                   dense, everything else the count -> scan -> write passes;
+                                   other values select kernel variants:
                                    1 = exact-f64-only tests, 2 = write pass recomputes the tests,
-                                   4 = single-pass device table, 7 / 8 = the paper's GPUCalcGlobal
+                                   3 = no dense/sparse split, 4 = single-pass device table
+                                   (sampled-estimate capacity), 7 / 8 = the paper's GPUCalcGlobal
                                    (Alg. 2) / GPUCalcShared (Alg. 3) with an atomic key/value result
                                    set sorted by key (device-resident whole tables; the Table II
                                    baseline)                                               */
