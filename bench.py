@@ -491,7 +491,10 @@ def main():
     tp = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tp):
         with open(tp) as f:
-            traffic = json.load(f).get(f"{args.workload}-{args.dtype}-k{args.kernel}-s{args.cell_split}")
+            # keyed by the kernel that ran (single pass / two passes); per-launch bytes of an
+            # unsharded run only
+            key = f"{args.workload}-{args.dtype}-k{args.kernel}-s{args.cell_split}" + ("" if single else "-2p")
+            traffic = json.load(f).get(key) if ws == 1 else None
     # whole-step view: SURVEY 8(d) B_alg = 4P + 64n + 8C (f64) over the step time
     b_step = 4 * P + (4 * esz + 32) * n + 8 * st["n_nonempty"]
     cms = float(np.mean(count_ms))
@@ -586,6 +589,39 @@ def main():
                        "points_clustered_per_sec_device": n / td, "s_per_step_device": td,
                        "device": "pinned host points -> device table -> GPU DBSCAN -> labels D2H (NEXT-4)",
                        "n_clusters": kh, "n_clusters_device": kd}
+    elif ws > 1 and args.e2e_steps > 0 and not paper:
+        # N ranks: every rank takes the pinned host points to a HOST table of its query shard
+        # (H2D of all points, its shard's D2H); time = max over ranks (barriers around each
+        # step), value = the pairs of all shards / that time.  Clustering needs the whole table
+        # in one process and is reported at N = 1 only.
+        hdb.hdb_ctx_set_stream(ctx, None)
+        xy_pin = torch.from_numpy(xy_np).pin_memory()
+
+        def shard_to_host():
+            g = hdb.hdb_grid_build(ctx, xy_pin, eps)
+            t = hdb.hdb_neighbor_table(ctx, g)
+            hdb.hdb_grid_free(g)
+            P_ = hdb.hdb_table_view_get(t).npairs
+            hdb.hdb_table_free(t)
+            return P_
+
+        shard_to_host()   # warm the pinned pool / device pools
+        ts, Ps = [], 0
+        for _ in range(args.e2e_steps):
+            dist.barrier()
+            t0 = time.perf_counter()
+            Ps = shard_to_host()
+            tt = torch.tensor([time.perf_counter() - t0], device=coll_dev)
+            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+            ts.append(float(tt.item()))
+        pt = torch.tensor([float(Ps)], device=coll_dev, dtype=torch.float64)
+        dist.all_reduce(pt)
+        te = float(np.median(ts))
+        line["e2e"] = {"value": float(pt.item()) / te, "unit": "pairs/s", "h2d_bytes_per_step": esz * n * ws,
+                       "d2h_bytes_per_step": 4 * int(pt.item()) + 12 * n, "s_per_step": te,
+                       "includes": "per rank: pinned host points -> H2D -> grid -> count -> batched write + D2H of "
+                                   "its query shard into a host table (a1-a10); max over ranks",
+                       "points_clustered_per_sec_hybrid": None, "points_clustered_per_sec_device": None}
     else:
         line["e2e"] = None
     if rank == 0 and not args.no_cpu_baseline:
