@@ -343,6 +343,35 @@ def test_single_pass_device_table_and_fallback(torch_cuda):
     assert_table_equal(xy2, 0.5, b, c, v)
 
 
+def test_single_pass_selection_and_exact_bound(torch_cuda):
+    """search_kernel 0 on device-resident tables: dense data (>= 400 candidate tests
+    per query) takes the single pass sized by the exact bound P <= tests without a
+    sampled estimate (est_pairs 0); moderately dense data the single pass sized from
+    the sample; sparse data the two passes.  Every table equals the oracle, including
+    the degenerate all-in-one-cell case (P = n^2) and f32 input."""
+    rng = np.random.default_rng(22)
+    dense = rng.uniform(0, 10, size=(40_000, 2))   # ~310 pairs, >= 400 candidate tests per query
+    b, c, v, view, st = lib_table(dense, 0.5, device=True)
+    assert st["single_pass"] == 1 and st["est_pairs"] == 0
+    assert_table_equal(dense, 0.5, b, c, v)
+    xf = dense.astype(np.float32)
+    b, c, v, view, st = lib_table(xf, 0.5, device=True)
+    assert st["single_pass"] == 1
+    assert_table_equal(xf, 0.5, b, c, v, dtype="f32")
+    tec = datagen.subsample(datagen.tec_like(), 40_000, seed=21)   # sampled estimate decides
+    b, c, v, view, st = lib_table(tec, 1.4, device=True)
+    assert st["single_pass"] == 1 and st["est_pairs"] > 0
+    assert_table_equal(tec, 1.4, b, c, v)
+    same = np.repeat(rng.uniform(0, 1, size=(1, 2)), 3_000, axis=0)   # one cell, every pair a neighbour
+    b, c, v, view, st = lib_table(same, 0.5, device=True)
+    assert st["single_pass"] == 1 and view.npairs == 3_000 ** 2
+    assert_table_equal(same, 0.5, b, c, v)
+    uni = rng.uniform(0, 100, size=(20_000, 2))   # ~3 pairs per query: two passes
+    b, c, v, view, st = lib_table(uni, 0.5, device=True)
+    assert st["single_pass"] == 0
+    assert_table_equal(uni, 0.5, b, c, v)
+
+
 def test_deterministic(torch_cuda):
     xy = datagen.subsample(datagen.tec_like(), 30_000, seed=9)
     a = lib_table(xy, 0.45)
