@@ -207,15 +207,25 @@ constexpr int kWin = kMaskWin;
 
 constexpr int kWinPad = kWin + 1;   // padded smem rows: 72-B stride, conflict-free per-lane access
 
+// End of a window of the count pass: lane i (< nq) adds the popcounts of query
+// i's kWin chunk masks to my (per window instead of per chunk: one warp
+// barrier and shared load per window), stores them to the mask table (gmask
+// non-null) and the window buffer is cleared for the next window.
 __device__ __forceinline__ void flush_window(uint2 (*swin)[kWinPad], uint2* gmask, uint32_t v, uint32_t nq,
-                                             int lane) {
+                                             uint32_t& my, int lane) {
     __syncwarp();
     if ((uint32_t)lane < nq) {
-        uint4* dst = (uint4*)(gmask + ((size_t)v * nq + lane) * kWin);
+        uint2 r[kWin];
 #pragma unroll
-        for (int u = 0; u < kWin / 2; ++u) {
-            const uint2 a = swin[lane][2 * u], b = swin[lane][2 * u + 1];
-            dst[u] = make_uint4(a.x, a.y, b.x, b.y);
+        for (int kk = 0; kk < kWin; ++kk) {
+            r[kk] = swin[lane][kk];
+            my += __popc(r[kk].x) + __popc(r[kk].y);
+        }
+        if (gmask) {
+            uint4* dst = (uint4*)(gmask + ((size_t)v * nq + lane) * kWin);
+#pragma unroll
+            for (int u = 0; u < kWin / 2; ++u)
+                dst[u] = make_uint4(r[2 * u].x, r[2 * u].y, r[2 * u + 1].x, r[2 * u + 1].y);
         }
     }
     __syncwarp();
@@ -321,6 +331,11 @@ __device__ __forceinline__ uint32_t count_group(const SArgs& a, uint32_t qs, uin
     uint32_t my = 0;
     const uint32_t npairs = load_vspans(a, c, vsp, lane);
     const uint32_t nch = (npairs + 31) / 32;
+    if (lane == 0) {   // candidate tests of the group: nq x (candidates of its spans)
+        uint32_t ncand = 0;
+        for (uint32_t r = 0; r < a.nspan; ++r) ncand += vsp[r].hi - vsp[r].lo;
+        tests += (unsigned long long)nq * ncand;
+    }
     uint32_t rs = 0;   // this lane's current span
     uint32_t k = 0;
 #pragma unroll 1
@@ -347,7 +362,6 @@ __device__ __forceinline__ uint32_t count_group(const SArgs& a, uint32_t qs, uin
                 Y = pack2(v0 ? (float)__dsub_rn(d0.y, o.y) : kFarF, v1 ? (float)__dsub_rn(d1.y, o.y) : kFarF);
             }
         }
-        tests += (unsigned long long)nq * ((v0 ? 1u : 0u) + (v1 ? 1u : 0u));   // per lane; reduced at exit
         uint32_t acc = 0;   // f64 filter: sign bit set <=> some |t| <= band in this lane
         uint32_t i0 = 0;
         if (MODE == kF64Filter) {
@@ -452,14 +466,9 @@ __device__ __forceinline__ uint32_t count_group(const SArgs& a, uint32_t qs, uin
                 if (lane == 0) swin[i][kk] = make_uint2(m0, m1);
             }
         }
-        __syncwarp();
-        if ((uint32_t)lane < nq) {
-            const uint2 mk = swin[lane][kk];
-            my += __popc(mk.x) + __popc(mk.y);
-        }
-        if (gmask && kk == kWin - 1) flush_window(swin, gmask, k / kWin, nq, lane);
+        if (kk == kWin - 1) flush_window(swin, gmask, k / kWin, nq, my, lane);
     }
-    if (gmask && (k % kWin) != 0) flush_window(swin, gmask, k / kWin, nq, lane);
+    if ((k % kWin) != 0) flush_window(swin, gmask, k / kWin, nq, my, lane);
     return my;
 }
 
@@ -631,11 +640,13 @@ __global__ void __launch_bounds__(kSearchThreads) k_search(SArgs a, uint32_t g0,
                         const uint2 mk = swin[WRITE ? 0 : w][lane][kk];
                         my += __popc(mk.x) + __popc(mk.y);
                     }
-                    if (gmask && kk == kWin - 1) flush_window(swin[WRITE ? 0 : w], gmask, k / kWin, nq, lane);
+                    uint32_t junk = 0;   // (counted above, per chunk)
+                    if (gmask && kk == kWin - 1) flush_window(swin[WRITE ? 0 : w], gmask, k / kWin, nq, junk, lane);
                 }
             }
         }
-        if (!WRITE && gmask && (k % kWin) != 0) flush_window(swin[WRITE ? 0 : w], gmask, k / kWin, nq, lane);
+        uint32_t junk = 0;
+        if (!WRITE && gmask && (k % kWin) != 0) flush_window(swin[WRITE ? 0 : w], gmask, k / kWin, nq, junk, lane);
         if (!WRITE && (uint32_t)lane < nq) cnt[qs + lane] = my;
         if (++ii >= iend) {
             ii = i0 + grab(ctr, chunk, lane);

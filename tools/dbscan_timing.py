@@ -12,7 +12,7 @@ from paper_conf_ipps_gowanlockrblp17_b200 import hdb
 
 eps = float(sys.argv[1]) if len(sys.argv) > 1 else 0.45
 xy = torch.from_numpy(datagen.tec_like()).cuda()
-ctx = hdb.hdb_ctx_create()
+ctx = hdb.hdb_ctx_create(search_kernel=int(os.environ.get("SK", "0")))   # SK=3: two passes
 g = hdb.hdb_grid_build(ctx, xy, eps)
 t = hdb.hdb_neighbor_table_device(ctx, g)
 n = xy.shape[0]
@@ -37,7 +37,7 @@ if os.environ.get("GIANT"):
     print("top clusters: point share", [round(sizes[c] / n, 3) for c in top],
           "pair share", [round(pairs[c] / v.npairs, 3) for c in top], flush=True)
 labh = np.empty(n, np.int32)
-for threads in (1, 16, 0):
+for threads in ((1, 16, 0) if not os.environ.get("NOHOST") else ()):
     t0 = time.perf_counter()
     _, _, kh = hdb.hdb_dbscan(th, 4, n_threads=threads, labels=labh)
     print("host dbscan threads", threads, "ms", (time.perf_counter() - t0) * 1e3, "clusters", kh)
