@@ -347,9 +347,22 @@ __global__ void __launch_bounds__(256) k_cell_spans(const uint64_t* __restrict__
          c += (uint64_t)gridDim.x * blockDim.x) {
         const uint64_t key = ckey[c];
         const uint64_t cy = key / nx, cx = key - cy * nx;
-        const uint64_t xl = cx >= k ? cx - k : 0;
-        const uint64_t xh = cx + k < nx ? cx + k : nx - 1;
         for (uint32_t r = 0; r < nspan; ++r) {
+            // Row dy = r - k of the stencil reaches kx(dy) columns either side: a neighbour in
+            // cell (dx, dy) is >= (|dx|-1) w, (|dy|-1) w away in x, y, and (eps / w)^2 =
+            // k^2 / (1 + 2^-19)^2 < k^2, so (|dx|-1)^2 + (|dy|-1)^2 <= k^2 holds for every
+            // neighbour (the 2^-19 margin covers the rounding of the cell indices).  Trims
+            // the outer rows' corner cells for k >= 4 (k = 6: 169 -> 157 cells).
+            const uint32_t a = r > k ? r - k : k - r;
+            uint32_t kx = k;
+            if (a >= 2) {
+                const uint32_t rem = k * k - (a - 1) * (a - 1);
+                uint32_t m = 0;
+                while ((m + 1) * (m + 1) <= rem) ++m;   // isqrt (k <= 6)
+                kx = min(k, 1 + m);
+            }
+            const uint64_t xl = cx >= kx ? cx - kx : 0;
+            const uint64_t xh = cx + kx < nx ? cx + kx : nx - 1;
             const int64_t yy = (int64_t)cy + (int64_t)r - (int64_t)k;
             uint2 sp = make_uint2(0, 0);
             if (yy >= 0 && yy < (int64_t)ny) {
