@@ -482,9 +482,10 @@ def test_filter_disabled_for_huge_extent(torch_cuda):
     assert_table_equal(xy, 0.05, b, c, v)
 
 
-@pytest.mark.parametrize("k", [2, 3])
+@pytest.mark.parametrize("k", [2, 3, 4, 6])
 def test_cell_split_parity(torch_cuda, k):
-    """cell_split = k: cells of width eps/k and a (2k+1)^2 stencil; same table."""
+    """cell_split = k: cells of width eps/k and a (2k+1)^2 stencil (rows trimmed to the
+    eps-disc for k >= 4; the lattice cases put exact ties on the disc); same table."""
     cases = [(datagen.subsample(datagen.tec_like(), 40_000, seed=1), (0.15, 0.45, 1.40)),
              (datagen.subsample(datagen.sdss_like(), 40_000, seed=2), (0.07, 0.6)),
              (datagen.near_ties(3000, 0.45, seed=3), (0.45,)),
