@@ -453,9 +453,8 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
     DBuf xy_s((n + 2) * esz, s);
     DBuf xp(16 * (n / 2 + 2), s);
     DBuf counters(4 * kCounterSlots, s);
-    DBuf inv(4 * (n + 1), s);
     // (the gather also zeroes the padding of xy_s / ids / xp and the work counters)
-    launch_gather_points(xin, ids.as<uint32_t>(), n, dt, xy_s.p, xp.as<float4>(), g.ox, g.oy, inv.as<uint32_t>(),
+    launch_gather_points(xin, ids.as<uint32_t>(), n, dt, xy_s.p, xp.as<float4>(), g.ox, g.oy,
                          counters.as<unsigned int>(), kCounterSlots, s);
     HDB_LAUNCH_CHECK();
     xin_owned.reset();
@@ -510,7 +509,6 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
     g.xp = (float4*)xp.release();
     g.counters = (unsigned int*)counters.release();
     g.ids = (uint32_t*)ids.release();
-    g.inv = (uint32_t*)inv.release();
     g.ckey = (uint64_t*)ckey.release();
     g.cstart = (uint32_t*)cstart.release();
     g.cspan = (uint2*)cspan.release();
@@ -593,14 +591,14 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
 void free_dev_grid(DevGrid& g) {
     if (!g.stream) return;
     DeviceGuard dg(g.device);
-    for (void* p : {(void*)g.xy_s, (void*)g.xp, (void*)g.counters, (void*)g.ids, (void*)g.inv, (void*)g.ckey, (void*)g.cstart,
+    for (void* p : {(void*)g.xy_s, (void*)g.xp, (void*)g.counters, (void*)g.ids, (void*)g.ckey, (void*)g.cstart,
                     (void*)g.cspan, (void*)g.gstart, (void*)g.gcell, (void*)g.moff, (void*)g.dpre, (void*)g.spre,
                     (void*)g.dl, (void*)g.sql, (void*)g.ord})
         if (p) cudaFreeAsync(p, g.stream);   // stream-ordered: no host sync needed
     g.xy_s = nullptr;
     g.xp = nullptr;
     g.counters = nullptr;
-    g.ids = g.inv = g.cstart = g.gstart = g.gcell = nullptr;
+    g.ids = g.cstart = g.gstart = g.gcell = nullptr;
     g.moff = nullptr;
     g.dpre = g.spre = g.dl = g.ord = nullptr;
     g.sql = nullptr;
@@ -667,6 +665,8 @@ struct ShardState {
     float ms_count = 0, ms_scan = 0, ms_write = 0;
     uint32_t write_launches = 0;
     uint64_t n_batches = 0, max_batch = 0, d2h = 0;
+    uint64_t* dbeg = nullptr;   // device T by original id, written by the write kernels (null: not wanted)
+    uint32_t* dcnt = nullptr;
 };
 
 // Sorted position -> group boundaries for `parts` shards balanced by the sampled counts.
@@ -950,7 +950,7 @@ void write_phase_host(hdb_ctx* ctx, DevCtx& dc, const DevGrid& g, ShardState& st
         if (b < S) HDB_CUDA(cudaStreamWaitEvent(ss, ready.e, 0));
         HDB_CUDA(cudaEventRecord(evs[2 * b].e, ss));
         launch_write(g, hg[b], hg[b + 1], st.off.as<uint64_t>(), hp[b], dc.batch_buf[si], ctx->opts.search_kernel,
-                     1 + (int)si, st.mask_base, ss);
+                     1 + (int)si, st.mask_base, ss, st.dbeg, st.dcnt);
         HDB_LAUNCH_CHECK();
         HDB_CUDA(cudaEventRecord(evs[2 * b + 1].e, ss));
         if (pairs_b)
@@ -1228,13 +1228,11 @@ void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hd
                 }
                 Event e0, e1;
                 HDB_CUDA(cudaEventRecord(e0.e, s));
+                // the write kernels also write T by original id (begin/count) for their rows
                 launch_write(g, st.r.g0, st.r.g1, st.off.as<uint64_t>(), 0, nb.as<uint32_t>(), ctx->opts.search_kernel, 1,
-                             st.mask_base, s);
+                             st.mask_base, s, beg.as<uint64_t>(), cnt.as<uint32_t>());
                 HDB_LAUNCH_CHECK();
                 HDB_CUDA(cudaEventRecord(e1.e, s));
-                launch_rows_by_id(g.inv, g.n, st.off.as<uint64_t>(), st.cnt.as<uint32_t>(), st.r.q0, st.r.q1, 0,
-                                  beg.as<uint64_t>(), cnt.as<uint32_t>(), s);
-                HDB_LAUNCH_CHECK();
                 HDB_CUDA(cudaStreamSynchronize(s));
                 st.ms_write = elapsed(e0, e1);
                 tr.mark("alloc+write+scatter+sync");
@@ -1263,20 +1261,26 @@ void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hd
                     memset(t->count, 0, 4 * (n ? n : 1));
                 }
                 tr.mark("pinned-pool");
+                // begin/count by original id: written on the device by the write kernels
+                // (one device, whole range), then one copy each
+                DBuf beg, cnt;
+                if (whole) {
+                    DevCtx& dc = ctx->dev[0];
+                    DeviceGuard dg(dc.device);
+                    beg = DBuf(8 * (n ? n : 1), dc.main);
+                    cnt = DBuf(4 * (n ? n : 1), dc.main);
+                    sh[0].dbeg = beg.as<uint64_t>();
+                    sh[0].dcnt = cnt.as<uint32_t>();
+                }
                 std::vector<uint64_t> dev_grows(ndev, 0);
                 run_parallel(ndev, [&](size_t d) {
                     write_phase_host(ctx, ctx->dev[d], grid->dev[d], sh[d], t->nbrs, batch_pairs, &dev_grows[d]);
                 });
                 tr.mark("write+d2h");
-                // begin/count by original id
                 if (whole) {
                     DevCtx& dc = ctx->dev[0];
                     DeviceGuard dg(dc.device);
                     cudaStream_t s = dc.main;
-                    DBuf beg(8 * (n ? n : 1), s), cnt(4 * (n ? n : 1), s);
-                    launch_rows_by_id(grid->dev[0].inv, n, sh[0].off.as<uint64_t>(), sh[0].cnt.as<uint32_t>(), 0, n, 0,
-                                      beg.as<uint64_t>(), cnt.as<uint32_t>(), s);
-                    HDB_LAUNCH_CHECK();
                     if (n) {
                         HDB_CUDA(cudaMemcpyAsync(t->begin, beg.p, 8 * n, cudaMemcpyDeviceToHost, s));
                         HDB_CUDA(cudaMemcpyAsync(t->count, cnt.p, 4 * n, cudaMemcpyDeviceToHost, s));

@@ -66,7 +66,6 @@ struct DevGrid {
                                    // filter coords x-ox, y-oy (f64 mode) / the exact coords (f32 mode)
     unsigned int* counters = nullptr;  // [kCounterSlots] work counters of the search kernels
     uint32_t* ids = nullptr;       // [n] sorted pos -> original id  (A)
-    uint32_t* inv = nullptr;       // [n] original id -> sorted pos  (A^-1, written by the gather)
     uint64_t* ckey = nullptr;      // [n_nonempty] cell key of each non-empty cell (ascending)
     uint32_t* cstart = nullptr;    // [n_nonempty+1] first sorted pos of each non-empty cell (G)
     uint2* cspan = nullptr;        // [nspan*n_nonempty] stencil row spans [lo,hi) per non-empty cell
@@ -108,8 +107,7 @@ int radix_sort_pairs(void* k0, uint32_t* v0, void* k1, uint32_t* v1, int key_byt
                      void* temp, cudaStream_t s);
 // gather sorted points; f64 mode also writes the f32 filter coordinates (x-ox, y-oy)
 void launch_gather_points(const void* xy_in, uint32_t* ids, uint64_t n, hdb_dtype dt, void* xy_s, float4* xp,
-                          double ox, double oy, uint32_t* inv, unsigned int* counters, uint32_t n_counters,
-                          cudaStream_t s);
+                          double ox, double oy, unsigned int* counters, uint32_t n_counters, cudaStream_t s);
 void launch_cell_flags(const void* keys_sorted, int key_bytes, uint64_t n, uint32_t* flags, cudaStream_t s);
 void launch_cell_scatter(const void* keys_sorted, int key_bytes, const uint32_t* flags, const uint32_t* pos,
                          uint64_t n, uint64_t* ckey, uint32_t* cstart, cudaStream_t s);
@@ -179,7 +177,8 @@ void launch_fused(const DevGrid& g, uint32_t* cnt, unsigned long long* tests, ui
                   unsigned long long* pair_ctr, uint64_t cap, uint32_t* out, uint64_t* begin, uint32_t* count,
                   unsigned int* overflow, cudaStream_t s);
 void launch_write(const DevGrid& g, uint64_t g0, uint64_t g1, const uint64_t* off, uint64_t out_base,
-                  uint32_t* out, int variant, int slot, const uint2* masks, cudaStream_t s);
+                  uint32_t* out, int variant, int slot, const uint2* masks, cudaStream_t s,
+                  uint64_t* begin = nullptr, uint32_t* count = nullptr);
 // words[g] = 32-bit words of group g's hit masks for g < *ng_dev, 0 for g in [*ng_dev, n) (scan -> g.moff)
 void launch_mask_words(const DevGrid& g, const uint32_t* ng_dev, uint64_t n, uint32_t* words, cudaStream_t s);
 // cuts: for b in 0..nb, gcut[b] = first group g in [g0,g1] with off[gstart[g]] >= target_b,
@@ -196,10 +195,6 @@ void launch_dbscan_device(const uint64_t* begin, const uint32_t* count, const ui
                           uint32_t* root, uint32_t* is_root, uint32_t* rank, uint32_t* giant, uint32_t* bits,
                           uint32_t* sched /* 2 x SM count */, uint64_t* pre /* n + 1 */, void* scan_temp,
                           int32_t* labels, cudaStream_t s);
-// T by original id through A^-1 (sequential writes, gathered reads): for every id
-// whose sorted position q lies in [q0, q1): begin[id] = off[q] - off[q0] + base, count[id] = cnt[q]
-void launch_rows_by_id(const uint32_t* inv, uint64_t n_ids, const uint64_t* off, const uint32_t* cnt, uint64_t q0,
-                       uint64_t q1, uint64_t base, uint64_t* begin, uint32_t* count, cudaStream_t s);
 
 // the paper's kernels (kernels_paper.cu; search_kernel 7 / 8):
 // the key/value result set R of GPUCalcGlobal (Alg. 2) or GPUCalcShared (Alg. 3),

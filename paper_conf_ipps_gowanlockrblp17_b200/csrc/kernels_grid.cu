@@ -253,8 +253,7 @@ template <typename T>
 __global__ void __launch_bounds__(256) k_gather(const typename V2<T>::type* __restrict__ in,
                                                 const uint32_t* __restrict__ ids, uint64_t n,
                                                 typename V2<T>::type* __restrict__ out, float4* __restrict__ xp,
-                                                double ox, double oy, uint32_t* __restrict__ inv,
-                                                uint32_t* __restrict__ ids_pad, unsigned int* __restrict__ counters,
+                                                double ox, double oy, uint32_t* __restrict__ ids_pad, unsigned int* __restrict__ counters,
                                                 uint32_t n_counters) {
     // xp: paired-SoA f32 copy {x_2k, x_2k+1, y_2k, y_2k+1} -- f64 input: filter
     // coordinates fl32(fl64(x - ox)); f32 input: the exact coordinates
@@ -273,10 +272,8 @@ __global__ void __launch_bounds__(256) k_gather(const typename V2<T>::type* __re
     }
     for (uint64_t s = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; s < n;
          s += (uint64_t)gridDim.x * blockDim.x) {
-        const uint32_t id = ids[s];
-        auto p = in[id];
+        auto p = in[ids[s]];
         out[s] = p;
-        inv[id] = (uint32_t)s;   // A^-1: T by original id gathers through it (launch_rows_by_id)
         float fx, fy;
         if (sizeof(p.x) == 8) {
             fx = (float)__dsub_rn((double)p.x, ox);
@@ -681,14 +678,13 @@ int radix_sort_pairs(void* k0, uint32_t* v0, void* k1, uint32_t* v1, int key_byt
 }
 
 void launch_gather_points(const void* xy_in, uint32_t* ids, uint64_t n, hdb_dtype dt, void* xy_s, float4* xp,
-                          double ox, double oy, uint32_t* inv, unsigned int* counters, uint32_t n_counters,
-                          cudaStream_t s) {
+                          double ox, double oy, unsigned int* counters, uint32_t n_counters, cudaStream_t s) {
     const unsigned blocks = n ? grid_for(n) : 1;
     if (dt == HDB_F64)
-        k_gather<double><<<blocks, 256, 0, s>>>((const double2*)xy_in, ids, n, (double2*)xy_s, xp, ox, oy, inv,
-                                                ids + n, counters, n_counters);
+        k_gather<double><<<blocks, 256, 0, s>>>((const double2*)xy_in, ids, n, (double2*)xy_s, xp, ox, oy, ids + n,
+                                                counters, n_counters);
     else
-        k_gather<float><<<blocks, 256, 0, s>>>((const float2*)xy_in, ids, n, (float2*)xy_s, xp, 0, 0, inv, ids + n,
+        k_gather<float><<<blocks, 256, 0, s>>>((const float2*)xy_in, ids, n, (float2*)xy_s, xp, 0, 0, ids + n,
                                                counters, n_counters);
     ++g_kernel_launches;
 }

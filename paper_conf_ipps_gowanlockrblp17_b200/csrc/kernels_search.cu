@@ -762,7 +762,8 @@ __global__ void __launch_bounds__(kEmitThreads) k_emit(SArgs a, uint32_t g0, uin
                                                          unsigned int* __restrict__ ctr,
                                                          const uint64_t* __restrict__ off, uint64_t out_base,
                                                          uint32_t* __restrict__ out, const uint2* __restrict__ masks,
-                                                         const uint64_t* __restrict__ moff) {
+                                                         const uint64_t* __restrict__ moff,
+                                                         uint64_t* __restrict__ begin, uint32_t* __restrict__ count) {
     // rows padded (80-B / 144-B strides) so the per-lane row accesses are bank-conflict free
     __shared__ __align__(16) uint2 raw[kEmitWarps][32][kWin + 2];   // cp.async landing buffer (next window's masks)
     __shared__ uint4 wq[kEmitWarps][32][kWin + 1];    // current window: {m0, m1, pos0, pos1} per (query, chunk)
@@ -775,7 +776,15 @@ __global__ void __launch_bounds__(kEmitThreads) k_emit(SArgs a, uint32_t g0, uin
         uint32_t* gout = out + (gb - out_base);
         asm volatile("mov.b64 %0, %0;" : "+l"(gout));
         uint32_t my = 0;   // lane i: output cursor of query i within the group
-        if ((uint32_t)lane < m.nq) my = (uint32_t)(off[m.qs + lane] - gb);
+        if ((uint32_t)lane < m.nq) {
+            const uint64_t b = off[m.qs + lane];
+            my = (uint32_t)(b - gb);
+            if (begin) {   // T by original id (a10): random 12-B writes overlapping the store stream
+                const uint32_t id = __ldg(&a.ids[m.qs + lane]);
+                begin[id] = b;
+                count[id] = (uint32_t)(off[m.qs + lane + 1] - b);
+            }
+        }
         emit_group(a, m.c, m.nq, nwin, masks + (m.ma >> 1), gout, my, raw[w], wq[w], vsp[w], lane);
     };
     uint32_t i0 = g0, i1 = g1;
@@ -912,7 +921,8 @@ template <bool F64, bool WRITE>
 __global__ void __launch_bounds__(256) k_sparse(SArgs a, uint32_t g0, uint32_t g1, uint32_t* __restrict__ cnt,
                                                 unsigned long long* __restrict__ tests_out,
                                                 const uint64_t* __restrict__ off, uint64_t out_base,
-                                                uint32_t* __restrict__ out) {
+                                                uint32_t* __restrict__ out, uint64_t* __restrict__ begin,
+                                                uint32_t* __restrict__ count) {
     const uint32_t j0 = __ldg(&a.spre[g0]), j1 = __ldg(&a.spre[g1]);
     unsigned long long tests = 0;
     for (uint32_t j = j0 + blockIdx.x * blockDim.x + threadIdx.x; j < j1; j += gridDim.x * blockDim.x) {
@@ -924,7 +934,15 @@ __global__ void __launch_bounds__(256) k_sparse(SArgs a, uint32_t g0, uint32_t g
         else pf = a.xs[q];
         uint32_t m = 0;
         uint32_t* o = nullptr;
-        if (WRITE) o = out + (off[q] - out_base);
+        if (WRITE) {
+            const uint64_t b = off[q];
+            o = out + (b - out_base);
+            if (begin) {   // T by original id (a10): the row's place in the table
+                const uint32_t id = __ldg(&a.ids[q]);
+                begin[id] = b;
+                count[id] = (uint32_t)(off[q + 1] - b);
+            }
+        }
         auto test = [&](uint32_t k) -> bool {
             if (F64) {
                 const double2 v = __ldg(&a.xd[k]);
@@ -1166,15 +1184,16 @@ void launch_sample_count(const DevGrid& g, uint64_t stride, uint64_t n_sample, u
 
 template <bool WRITE>
 void launch_sparse(const DevGrid& g, uint64_t g0, uint64_t g1, uint32_t* cnt, unsigned long long* tests,
-                   const uint64_t* off, uint64_t out_base, uint32_t* out, cudaStream_t s) {
+                   const uint64_t* off, uint64_t out_base, uint32_t* out, cudaStream_t s, uint64_t* begin = nullptr,
+                   uint32_t* count = nullptr) {
     if (!g.sql || g.n_sparse_q == 0 || g1 <= g0) return;
     const unsigned blocks = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>((g.n_sparse_q + 255) / 256, 148 * 16));
     if (g.dtype == HDB_F64)
         k_sparse<true, WRITE><<<blocks, 256, 0, s>>>(args_of(g), (uint32_t)g0, (uint32_t)g1, cnt, tests, off, out_base,
-                                                     out);
+                                                     out, begin, count);
     else
         k_sparse<false, WRITE><<<blocks, 256, 0, s>>>(args_of(g), (uint32_t)g0, (uint32_t)g1, cnt, tests, off,
-                                                      out_base, out);
+                                                      out_base, out, begin, count);
     ++g_kernel_launches;
 }
 
@@ -1207,13 +1226,41 @@ void launch_count(const DevGrid& g, uint64_t g0, uint64_t g1, uint32_t* cnt, uns
     ++g_kernel_launches;
 }
 
+// T by original id for the sorted positions of groups [g0, g1) (the recompute write
+// variant; the default write kernels write it themselves): begin[ids[q]] = off[q],
+// count[ids[q]] = off[q+1] - off[q], q in [gstart[g0], gstart[g1])
+__global__ void __launch_bounds__(256) k_rows_direct(const uint32_t* __restrict__ ids,
+                                                     const uint32_t* __restrict__ gstart, uint32_t g0, uint32_t g1,
+                                                     const uint64_t* __restrict__ off, uint64_t* __restrict__ begin,
+                                                     uint32_t* __restrict__ count) {
+    const uint64_t q0 = gstart[g0], q1 = gstart[g1];
+    for (uint64_t q = q0 + blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; q < q1;
+         q += (uint64_t)gridDim.x * blockDim.x) {
+        const uint32_t id = ids[q];
+        const uint64_t b = off[q];
+        begin[id] = b;
+        count[id] = (uint32_t)(off[q + 1] - b);
+    }
+}
+
+void launch_rows_direct(const DevGrid& g, uint64_t g0, uint64_t g1, const uint64_t* off, uint64_t* begin,
+                        uint32_t* count, cudaStream_t s) {
+    const unsigned blocks = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>((g.n + 255) / 256, 148 * 16));
+    k_rows_direct<<<blocks, 256, 0, s>>>(g.ids, g.gstart, (uint32_t)g0, (uint32_t)g1, off, begin, count);
+    ++g_kernel_launches;
+}
+
 // masks != null: emission from the count pass's hit masks (k_emit); else the
 // write pass recomputes the distance tests (k_search<WRITE>).
 void launch_write(const DevGrid& g, uint64_t g0, uint64_t g1, const uint64_t* off, uint64_t out_base,
-                  uint32_t* out, int variant, int slot, const uint2* masks, cudaStream_t s) {
-    launch_sparse<true>(g, g0, g1, nullptr, nullptr, off, out_base, out, s);
+                  uint32_t* out, int variant, int slot, const uint2* masks, cudaStream_t s, uint64_t* begin,
+                  uint32_t* count) {
+    launch_sparse<true>(g, g0, g1, nullptr, nullptr, off, out_base, out, s, begin, count);
     if (!masks) {
         launch_search<true>(g, g0, g1, nullptr, nullptr, off, out_base, out, variant == 1, slot, nullptr, s);
+        if (begin && g1 > g0) {   // the recompute variant leaves T by id to a direct pass
+            launch_rows_direct(g, g0, g1, off, begin, count, s);
+        }
         return;
     }
     if (g1 <= g0) return;
@@ -1228,7 +1275,7 @@ void launch_write(const DevGrid& g, uint64_t g0, uint64_t g1, const uint64_t* of
     unsigned ctas;
     launch_groups(k_emit, bps, dense_groups(g, g0, g1), chunk, ctas, kEmitThreads);
     k_emit<<<ctas, kEmitThreads, 0, s>>>(a, (uint32_t)g0, (uint32_t)g1, chunk, ctr, off, out_base, out, masks,
-                                         g.moff);
+                                         g.moff, begin, count);
     ++g_kernel_launches;
 }
 
@@ -1285,28 +1332,5 @@ void launch_pos_to_group(const uint32_t* gstart, uint64_t n_groups, const uint64
     ++g_kernel_launches;
 }
 
-__global__ void __launch_bounds__(256) k_rows_by_id(const uint32_t* __restrict__ inv, uint64_t n_ids,
-                                                    const uint64_t* __restrict__ off,
-                                                    const uint32_t* __restrict__ cnt, uint64_t q0, uint64_t q1,
-                                                    uint64_t base, uint64_t* __restrict__ begin,
-                                                    uint32_t* __restrict__ count) {
-    const uint64_t o0 = off[q0];
-    for (uint64_t id = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; id < n_ids;
-         id += (uint64_t)gridDim.x * blockDim.x) {
-        const uint32_t q = inv[id];
-        if (q >= q0 && q < q1) {
-            begin[id] = off[q] - o0 + base;
-            count[id] = cnt[q];
-        }
-    }
-}
-
-void launch_rows_by_id(const uint32_t* inv, uint64_t n_ids, const uint64_t* off, const uint32_t* cnt, uint64_t q0,
-                       uint64_t q1, uint64_t base, uint64_t* begin, uint32_t* count, cudaStream_t s) {
-    if (q1 <= q0 || n_ids == 0) return;
-    const unsigned blocks = (unsigned)std::min<uint64_t>((n_ids + 255) / 256, 148 * 16);
-    k_rows_by_id<<<blocks, 256, 0, s>>>(inv, n_ids, off, cnt, q0, q1, base, begin, count);
-    ++g_kernel_launches;
-}
 
 }  // namespace hdb
