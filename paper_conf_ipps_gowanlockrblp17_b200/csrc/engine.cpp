@@ -203,17 +203,17 @@ constexpr uint64_t kMaxCellsAbs = 1ull << 30;
 // HDB_SPARSE_TESTS overrides it for tuning, 0 disables the split).
 constexpr double kSparseMinShare = 0.25;   // split only when >= this share of the queries is sparse
 // Device-resident whole tables take the single-pass kernel (k_fused: count,
-// reserve, emit per group; heavy groups first) unless the dense/sparse split is
-// on or the sampled estimate says < this many pairs per query.  Measured on one
-// B200 (ms of table kernels, two passes vs single pass): C2 eps 0.15 (97 pairs
-// per query) 0.72 vs 0.65, eps 0.45 (700) 2.39 vs 2.10, eps 1.40 (4,600) 13.1 vs
-// 9.8 -- the count pass's ALU work hides under the emission's store stream; C5
-// (80 pairs per query) 13.6 vs 14.4.
-constexpr double kFusedMinPairsPerQuery = 90.0;
+// reserve, emit and T by id per group; heavy groups first) unless the
+// dense/sparse split is on or the sampled estimate says < this many pairs per
+// query.  Measured on one B200 (ms per step, two passes vs single pass, both
+// writing T by id): C2 eps 0.15 (97 pairs per query) 1.40 vs 1.25, eps 0.45
+// (709) 2.39 vs 2.10 (table kernels), eps 1.40 (4,600) 13.1 vs 9.8 (table
+// kernels); C5 (80) 23.1 vs 21.5.  The count work hides under the store stream.
+constexpr double kFusedMinPairsPerQuery = 20.0;
 // ... and without any sample when the grid's candidate tests per query are clearly in the
-// single pass's regime (C2 eps 0.45: 1,128, eps 1.40: 6,280; C5: 224, C2 eps 0.15: 245) and
+// single pass's regime (C2 eps 0.15: 245, eps 0.45: 1,128, eps 1.40: 6,280; C5: 224) and
 // 4 B per test fits in this share of the device memory
-constexpr double kFusedDirectTestsPerQuery = 400.0;
+constexpr double kFusedDirectTestsPerQuery = 150.0;
 constexpr double kFusedDirectMemShare = 0.3;
 uint32_t sparse_max_tests() {
     static const uint32_t v = [] {

@@ -260,8 +260,10 @@ def test_host_budget_enomem(torch_cuda):
 
 
 def test_estimate_and_plan_stats(torch_cuda):
+    """The sampled estimate a_b and the Eq. 1 plan of the batched host-table path (a5);
+    dense device tables skip the sample (test_single_pass_selection_and_exact_bound)."""
     xy = datagen.subsample(datagen.tec_like(), 200_000, seed=8)
-    b, c, v, view, st = lib_table(xy, 0.45, device=True)
+    b, c, v, view, st = lib_table(xy, 0.45)
     assert st["sample_size"] == math.ceil(xy.shape[0] / 100)
     assert st["est_pairs"] == st["sample_pairs"] * 100
     bb, nb = hdb.hdb_plan_batches(st["est_pairs"], 0.05, 3)
@@ -344,7 +346,7 @@ def test_single_pass_device_table_and_fallback(torch_cuda):
 
 
 def test_single_pass_selection_and_exact_bound(torch_cuda):
-    """search_kernel 0 on device-resident tables: dense data (>= 400 candidate tests
+    """search_kernel 0 on device-resident tables: dense data (>= 150 candidate tests
     per query) takes the single pass sized by the exact bound P <= tests without a
     sampled estimate (est_pairs 0); moderately dense data the single pass sized from
     the sample; sparse data the two passes.  Every table equals the oracle, including
@@ -358,10 +360,10 @@ def test_single_pass_selection_and_exact_bound(torch_cuda):
     b, c, v, view, st = lib_table(xf, 0.5, device=True)
     assert st["single_pass"] == 1
     assert_table_equal(xf, 0.5, b, c, v, dtype="f32")
-    tec = datagen.subsample(datagen.tec_like(), 40_000, seed=21)   # sampled estimate decides
-    b, c, v, view, st = lib_table(tec, 1.4, device=True)
+    mid = rng.uniform(0, 40, size=(40_000, 2))   # ~38 pairs, ~110 tests per query: the sample decides
+    b, c, v, view, st = lib_table(mid, 0.7, device=True)
     assert st["single_pass"] == 1 and st["est_pairs"] > 0
-    assert_table_equal(tec, 1.4, b, c, v)
+    assert_table_equal(mid, 0.7, b, c, v)
     same = np.repeat(rng.uniform(0, 1, size=(1, 2)), 3_000, axis=0)   # one cell, every pair a neighbour
     b, c, v, view, st = lib_table(same, 0.5, device=True)
     assert st["single_pass"] == 1 and view.npairs == 3_000 ** 2
