@@ -15,7 +15,9 @@ ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpuru
     python bench.py --steps 2 --warmup 1 --e2e-steps 0 --no-cpu-baseline > /dev/null 2>&1
 ncu --set full --clock-control none --import-source on -k regex:"k_fused|k_count|k_emit" -c 2 -o gpurun_out/${T}_prof_c2 \
     python bench.py --steps 1 --warmup 0 --e2e-steps 0 --no-cpu-baseline > /dev/null 2>&1
-# the two-pass kernels (count + write) on the workload that takes them by default (C5, 80 pairs/query)
-ncu --set full --clock-control none --import-source on -k regex:"k_count|k_emit" -c 2 -o gpurun_out/${T}_prof_c5 \
+# the single pass on C5 (50M points) and the two-pass kernels on C3L (the dense/sparse split keeps them)
+ncu --set full --clock-control none --import-source on -k regex:"k_fused" -c 1 -o gpurun_out/${T}_prof_c5 \
     python bench.py --workload C5-eps0.5 --steps 1 --warmup 0 --e2e-steps 0 --no-cpu-baseline > /dev/null 2>&1
+ncu --set full --clock-control none --import-source on -k regex:"k_count|k_emit|k_sparse" -c 4 -o gpurun_out/${T}_prof_c3l \
+    python bench.py --workload C3L-eps0.07 --steps 1 --warmup 0 --e2e-steps 0 --no-cpu-baseline > /dev/null 2>&1
 ls -la gpurun_out | grep $T
