@@ -506,7 +506,9 @@ def main():
             "config": {"workload": args.workload, "desc": wl["desc"], "n": n, "eps": eps,
                        "pairs_per_step": P, "parallelism": f"query-shard{ws}",
                        "l2": "not flushed: each step writes a %.1f GB table (>> 126 MB L2)" % (4 * P / 1e9),
-                       "step": ("grid build + sampled count + single-pass count/reserve/write (k_fused, "
+                       "step": (("grid build + single-pass count/reserve/write (k_fused, capacity = the grid's "
+                                 "candidate tests, no sample; device-resident table)") if single and not st["est_pairs"] else
+                                "grid build + sampled count + single-pass count/reserve/write (k_fused, "
                                 "device-resident table)" if single else
                                 "grid build + sampled count + count + scan + write (device-resident table)")},
             "gpu_launches": launches,
