@@ -199,7 +199,14 @@ hdb_status  hdb_grid_copy_to_host(const hdb_grid* grid, uint32_t* ids, uint64_t*
 /* Host-resident T: count -> scan -> batched write kernels on n_streams streams,
  * each batch DMA'd straight into the host table (pinned pool of ctx). */
 hdb_status  hdb_neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, hdb_table** out);
-/* Device-resident T (first device, or this process's shard): no D2H. */
+/* Device-resident T (first device, or this process's shard): no D2H.  begin /
+ * count are by original id as for host tables; the rows' placement in nbrs is
+ * the production order -- cell-sorted for the count -> scan -> write passes,
+ * reservation order for the single pass that dense whole tables take with
+ * search_kernel 0 -- so begin[] is not monotone in id.
+ * Dense whole tables are sized by the grid's candidate tests (an upper bound on
+ * the pairs; HDB_ENOMEM only if that bound cannot be allocated and the exact
+ * two-pass path cannot either). */
 hdb_status  hdb_neighbor_table_device(hdb_ctx* ctx, const hdb_grid* grid, hdb_table** out);
 /* Wrap a copy of a host CSR as a table (for reuse / tests): begin/count by id. */
 hdb_status  hdb_table_from_host(uint64_t n, const uint64_t* begin, const uint32_t* count,
