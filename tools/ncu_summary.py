@@ -47,6 +47,8 @@ def raw(rep):
 
 
 def launches(path):
+    if path == "-":   # no launch list for this capture
+        return []
     rows = list(csv.reader(open(path)))
     hdr_i = next(i for i, r in enumerate(rows) if "Kernel Name" in r)
     hdr = rows[hdr_i]
@@ -57,7 +59,7 @@ def launches(path):
             name = r[ki].split("(")[0].replace("void ", "")
             agg[name][0] += 1
             agg[name][1] += float(r[vi].replace(",", ""))
-    tot = sum(v[1] for v in agg.values())
+    tot = sum(v[1] for v in agg.values()) or 1.0
     return [{"kernel": k, "launches": v[0], "total_ns": v[1], "share": v[1] / tot}
             for k, v in sorted(agg.items(), key=lambda kv: -kv[1][1])]
 
