@@ -463,6 +463,27 @@ def test_c3_full_size_sampled_rows(torch_cuda):
         _sampled_rows_check(xy, eps, m_rows=800, seed=int(eps * 100))
 
 
+def test_single_pass_natural_order_large_point_set(torch_cuda):
+    """C5's recipe at 14M points (> 256 MB of coordinates + ids): the single
+    pass visits the groups in cell-sorted order instead of the cost order
+    ("C5 in the single pass") -- only point sets of C5's
+    scale take this branch, so it is checked here on sampled rows."""
+    xy = datagen.dense_skew(n=14_000_000, seed=15)
+    assert xy.shape[0] * (16 + 4) > (256 << 20)
+    view, st = _sampled_rows_check(xy, 0.7, m_rows=1000, seed=15)
+    assert st["single_pass"] == 1
+    assert 3e8 < view.npairs < 1e9
+
+
+def test_c5_full_size_sampled_rows(torch_cuda):
+    """C5 at the size and launch configuration bench.py times (50M points,
+    eps 0.5, single pass in the natural order; a 15.8 GB device table)."""
+    xy = datagen.dense_skew()
+    view, st = _sampled_rows_check(xy, datagen.C5_EPS[0], m_rows=600, seed=5)
+    assert st["single_pass"] == 1
+    assert 3.5e9 < view.npairs < 4.5e9
+
+
 def test_exact_f64_kernel_variant(torch_cuda):
     """search_kernel=1 forces the exact-f64-only kernel, 2 the write pass that
     recomputes the tests instead of replaying stored hit masks; all must equal
