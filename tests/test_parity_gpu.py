@@ -457,6 +457,26 @@ def test_c2_full_size_sampled_rows(torch_cuda):
     assert 1.0e9 < view.npairs < 2.0e9
 
 
+@pytest.mark.parametrize("eps,lo,hi", [(0.15, 1.0e8, 3.0e8), (1.40, 7.0e9, 1.0e10)])
+def test_c2_other_eps_full_size_sampled_rows(torch_cuda, eps, lo, hi):
+    """The other C2 bench workloads at full size (the auto cell split picks
+    k = 1 at eps 0.15 and k = 6 at eps 1.40; 1.40 is a 34 GB device table)."""
+    xy = datagen.tec_like()
+    view, st = _sampled_rows_check(xy, eps, m_rows=600, seed=int(eps * 100))
+    assert lo < view.npairs < hi
+
+
+def test_c3l_full_size_sampled_rows(torch_cuda):
+    """C3L (5M SDSS-like) bench workloads at full size: eps 0.07 takes the
+    dense/sparse split (two passes, thread-per-query sparse groups), eps 0.20
+    the single pass."""
+    xy = datagen.sdss_like(datagen.C3_N_LARGE, seed=4)
+    view, st = _sampled_rows_check(xy, 0.07, m_rows=800, seed=7)
+    assert st["n_sparse_queries"] > 0 and st["single_pass"] == 0
+    view, st = _sampled_rows_check(xy, 0.20, m_rows=800, seed=20)
+    assert st["single_pass"] == 1
+
+
 def test_c3_full_size_sampled_rows(torch_cuda):
     xy = datagen.sdss_like()
     for eps in datagen.C3_EPS:
