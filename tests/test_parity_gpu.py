@@ -431,7 +431,7 @@ def test_sweep_matches_oracle(torch_cuda, on_device):
 
 
 # ------------------------------------------------------------------ full-size sampled rows
-def _sampled_rows_check(xy, eps, m_rows=1500, seed=0, **opts):
+def _sampled_rows_check(xy, eps, m_rows=1500, seed=0, dtype="f64", **opts):
     b, c, v, view, st = lib_table(xy, eps, device=True, **opts)
     n = xy.shape[0]
     assert view.npairs == c.astype(np.int64).sum()
@@ -439,7 +439,7 @@ def _sampled_rows_check(xy, eps, m_rows=1500, seed=0, **opts):
     rows = rng.choice(n, size=m_rows, replace=False)
     # plus the rows with the largest lists (dense-cell stress)
     rows = np.unique(np.concatenate([rows, np.argsort(c)[-50:]]))
-    roff, rnbr = oracle.eps_join_rows(xy, eps, rows)
+    roff, rnbr = oracle.eps_join_rows(xy, eps, rows, dtype=dtype)
     for i, p in enumerate(rows):
         got = np.sort(v[b[p]:b[p] + c[p]])
         assert np.array_equal(got, rnbr[roff[i]:roff[i + 1]]), p
@@ -464,6 +464,13 @@ def test_c2_other_eps_full_size_sampled_rows(torch_cuda, eps, lo, hi):
     xy = datagen.tec_like()
     view, st = _sampled_rows_check(xy, eps, m_rows=600, seed=int(eps * 100))
     assert lo < view.npairs < hi
+
+
+def test_c2_full_size_f32_sampled_rows(torch_cuda):
+    """bench.py --dtype f32 at full size: the predicate in f32 (reading R1/R2)."""
+    xy = datagen.tec_like().astype(np.float32)
+    view, st = _sampled_rows_check(xy, 0.45, m_rows=800, seed=32, dtype="f32")
+    assert 1.0e9 < view.npairs < 2.0e9
 
 
 def test_c3l_full_size_sampled_rows(torch_cuda):
