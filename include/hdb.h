@@ -95,7 +95,8 @@ typedef struct {
     int host_threads;           /* threads for host-side work (T assembly, DBSCAN); 0 = all cores      */
     int cell_split;             /* k >= 1: grid cells of width eps/k, (2k+1)^2-cell stencil (fewer
                                    candidate tests on dense data); 0 = auto (k from a sampled cell
-                                   occupancy); 1 = the paper's eps cells      */
+                                   occupancy); 1 = the paper's eps cells;
+                                   k <= 6 (HDB_EINVAL above)                                         */
     int sweep_on_device;        /* hdb_sweep only: 0 = the paper's hybrid split (tables D2H, host
                                    DBSCAN pipelined with the next table's build);
                                    1 = tables stay in HBM and DBSCAN runs on the GPU (NEXT-4);

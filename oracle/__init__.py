@@ -8,8 +8,9 @@ Plain CPU implementation of what the HYBRID-DBSCAN hot path computes
 * ``eps_join_rows``   -- O2 restricted to sampled query rows (each vs all n).
 * ``eps_join_rowhash``-- O2 streamed as per-row (count, order-free hash).
 * ``sweep_rowhash``   -- O2 by an x-sorted plane sweep (the R-tree-free scan).
+* ``strip_rowhash``   -- the same sweep inside horizontal strips (50M points).
+* ``strip_join``      -- O2 as a full CSR table by the strip sweep.
 * ``dbscan``          -- O3, Algorithm 1 on T.
-* ``hybrid_dbscan``   -- Algorithm 4 with the GPU steps replaced by O2.
 
 Only ``tests/``, ``__graft_entry__.smoke()`` and ``bench.py``'s cpu_baseline /
 ``--impl reference`` legs may import this package.  It shares no code with the
@@ -67,6 +68,10 @@ def _load():
             getattr(lib, f"oracle_join_rowhash_{t}").argtypes = [P, i64, et, P, i64, P, P]
             getattr(lib, f"oracle_sweep_rowhash_{t}").argtypes = [P, i64, et, P, P]
             getattr(lib, f"oracle_sweep_rowhash_{t}").restype = ctypes.c_int
+            getattr(lib, f"oracle_strip_rowhash_{t}").argtypes = [P, i64, et, P, P]
+            getattr(lib, f"oracle_strip_rowhash_{t}").restype = ctypes.c_int
+            getattr(lib, f"oracle_strip_join_{t}").argtypes = [P, i64, et, P, P]
+            getattr(lib, f"oracle_strip_join_{t}").restype = ctypes.c_int
         lib.oracle_dbscan.argtypes = [P, P, i64, u64, P, P]
         lib.oracle_dbscan.restype = i64
         _lib = lib
@@ -156,6 +161,46 @@ def sweep_rowhash(xy, eps, dtype="f64"):
     return cnt, h
 
 
+def strip_rowhash(xy, eps, dtype="f64"):
+    """O2 by the plane sweep inside horizontal strips of width ~2 eps (the
+    scale-out of ``sweep_rowhash`` for 50M points): per-row (count, hash) for
+    all rows, equal to ``sweep_rowhash`` / ``eps_join_rowhash`` (see oracle.c
+    for the exactness argument; the strip widths are checked at run time)."""
+    lib = _load()
+    xy, npdt = _prep(xy, dtype)
+    n = xy.shape[0]
+    cnt = np.zeros(n, dtype=np.uint64)
+    h = np.zeros(n, dtype=np.uint64)
+    rc = getattr(lib, f"oracle_strip_rowhash_{dtype}")(_ptr(xy), n, float(npdt(eps)), _ptr(cnt), _ptr(h))
+    if rc == -1:
+        raise MemoryError("oracle_strip_rowhash: allocation failed")
+    if rc != 0:
+        raise ValueError("oracle_strip_rowhash: a strip is not wider than eps (exactness check failed)")
+    return cnt, h
+
+
+def strip_join(xy, eps, dtype="f64"):
+    """O2 as a full CSR table (off[n+1], nbr) with ascending lists, built by the
+    strip sweep -- equal to ``eps_join`` (pinned), in seconds at millions of
+    points (the full-size DBSCAN partitions of the GPU parity tests)."""
+    lib = _load()
+    xy, npdt = _prep(xy, dtype)
+    n = xy.shape[0]
+    off = np.zeros(n + 1, dtype=np.uint64)
+    fn = getattr(lib, f"oracle_strip_join_{dtype}")
+    e = float(npdt(eps))
+    for rc in (fn(_ptr(xy), n, e, _ptr(off), None),):
+        if rc == -1:
+            raise MemoryError("oracle_strip_join: allocation failed")
+        if rc != 0:
+            raise ValueError("oracle_strip_join: a strip is not wider than eps")
+    nbr = np.empty(int(off[-1]), dtype=np.uint32)
+    rc = fn(_ptr(xy), n, e, _ptr(off), _ptr(nbr) if nbr.size else _ptr(np.empty(1, np.uint32)))
+    if rc != 0:
+        raise MemoryError("oracle_strip_join: fill pass failed")
+    return off, nbr
+
+
 def dbscan(off, nbr, minpts):
     """O3: Algorithm 1 on T.  Returns (labels int32[n], is_core uint8[n], n_clusters)."""
     lib = _load()
@@ -170,10 +215,3 @@ def dbscan(off, nbr, minpts):
     if k < 0:
         raise MemoryError("oracle_dbscan: allocation failed")
     return labels, core, int(k)
-
-
-def hybrid_dbscan(xy, eps, minpts, dtype="f64"):
-    """Algorithm 4 with lines 5-8 replaced by the brute-force O2."""
-    off, nbr = eps_join(xy, eps, dtype)
-    labels, core, k = dbscan(off, nbr, minpts)
-    return labels, core, k, off, nbr

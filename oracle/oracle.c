@@ -249,39 +249,62 @@ static sweep_key* sweep_order(const double* xs, int64_t n)
     return k;
 }
 
+/* The scan reads the points through sorted copies (sx, sy, sid): the same
+ * values in the same order as ord[j].id would give, laid out for locality
+ * (the arithmetic is unchanged; only the memory layout differs). */
+#define SWEEP_BODY(T, IS_NEIGHBOR)                                                  \
+    int64_t i;                                                                      \
+    _Pragma("omp parallel for schedule(dynamic, 256)")                              \
+    for (i = 0; i < n; ++i) {                                                       \
+        T xp = sx[i], yp = sy[i];                                                   \
+        /* the scan's stop points: first j > i (rightwards) and last j < i         \
+         * (leftwards) with fl(dx*dx) > eps2 -- binary searches, exact because    \
+         * fl(dx*dx) is monotone along each direction (see above) */              \
+        int64_t lo = i + 1, hi = n;                                                 \
+        while (lo < hi) {                                                           \
+            int64_t m = lo + (hi - lo) / 2;                                         \
+            T dx = sx[m] - xp;                                                      \
+            if (dx * dx > eps2) hi = m; else lo = m + 1;                            \
+        }                                                                           \
+        int64_t jend = lo;                                                          \
+        lo = 0; hi = i;                                                             \
+        while (lo < hi) {                                                           \
+            int64_t m = lo + (hi - lo) / 2;                                         \
+            T dx = sx[m] - xp;                                                      \
+            if (dx * dx > eps2) lo = m + 1; else hi = m;                            \
+        }                                                                           \
+        int64_t jbeg = lo;                                                          \
+        uint64_t c = 0, h = 0;                                                      \
+        for (int64_t j = jbeg; j < jend; ++j) {                                     \
+            int hit = IS_NEIGHBOR(xp, yp, sx[j], sy[j], eps2);                      \
+            c += (uint64_t)hit;                                                     \
+            h += hit ? mix64((uint64_t)sid[j]) : 0;                                 \
+        }                                                                           \
+        cnt[sid[i]] = c;                                                            \
+        hash[sid[i]] = h;                                                           \
+    }
+
 int oracle_sweep_rowhash_f64(const double* xy, int64_t n, double eps, uint64_t* cnt, uint64_t* hash)
 {
     double eps2 = eps * eps;
     double* xs = (double*)malloc(sizeof(double) * (size_t)(n ? n : 1));
     if (!xs) return -1;
-    for (int64_t i = 0; i < n; ++i) xs[i] = xy[2 * i];
+    for (int64_t k = 0; k < n; ++k) xs[k] = xy[2 * k];
     sweep_key* ord = sweep_order(xs, n);
     free(xs);
     if (!ord) return -1;
-    int64_t i;
-#pragma omp parallel for schedule(dynamic, 256)
-    for (i = 0; i < n; ++i) {
-        int64_t p = ord[i].id;
-        double xp = xy[2 * p], yp = xy[2 * p + 1];
-        uint64_t c = 0, h = 0;
-        for (int64_t j = i; j < n; ++j) {          /* rightwards, including p itself */
-            int64_t q = ord[j].id;
-            double dx = xy[2 * q] - xp;
-            double dx2 = dx * dx;
-            if (dx2 > eps2) break;
-            if (is_neighbor_f64(xp, yp, xy[2 * q], xy[2 * q + 1], eps2)) { ++c; h += mix64((uint64_t)q); }
-        }
-        for (int64_t j = i - 1; j >= 0; --j) {     /* leftwards */
-            int64_t q = ord[j].id;
-            double dx = xy[2 * q] - xp;
-            double dx2 = dx * dx;
-            if (dx2 > eps2) break;
-            if (is_neighbor_f64(xp, yp, xy[2 * q], xy[2 * q + 1], eps2)) { ++c; h += mix64((uint64_t)q); }
-        }
-        cnt[p] = c;
-        hash[p] = h;
+    double* sx = (double*)malloc(sizeof(double) * (size_t)(n ? n : 1));
+    double* sy = (double*)malloc(sizeof(double) * (size_t)(n ? n : 1));
+    int64_t* sid = (int64_t*)malloc(sizeof(int64_t) * (size_t)(n ? n : 1));
+    if (!sx || !sy || !sid) { free(ord); free(sx); free(sy); free(sid); return -1; }
+    for (int64_t k = 0; k < n; ++k) {
+        sid[k] = ord[k].id;
+        sx[k] = xy[2 * ord[k].id];
+        sy[k] = xy[2 * ord[k].id + 1];
     }
     free(ord);
+    SWEEP_BODY(double, is_neighbor_f64)
+    free(sx); free(sy); free(sid);
     return 0;
 }
 
@@ -290,36 +313,221 @@ int oracle_sweep_rowhash_f32(const float* xy, int64_t n, float eps, uint64_t* cn
     float eps2 = eps * eps;
     double* xs = (double*)malloc(sizeof(double) * (size_t)(n ? n : 1));
     if (!xs) return -1;
-    for (int64_t i = 0; i < n; ++i) xs[i] = (double)xy[2 * i];   /* exact widening: same order */
+    for (int64_t k = 0; k < n; ++k) xs[k] = (double)xy[2 * k];   /* exact widening: same order */
     sweep_key* ord = sweep_order(xs, n);
     free(xs);
     if (!ord) return -1;
-    int64_t i;
-#pragma omp parallel for schedule(dynamic, 256)
-    for (i = 0; i < n; ++i) {
-        int64_t p = ord[i].id;
-        float xp = xy[2 * p], yp = xy[2 * p + 1];
-        uint64_t c = 0, h = 0;
-        for (int64_t j = i; j < n; ++j) {
-            int64_t q = ord[j].id;
-            float dx = xy[2 * q] - xp;
-            float dx2 = dx * dx;
-            if (dx2 > eps2) break;
-            if (is_neighbor_f32(xp, yp, xy[2 * q], xy[2 * q + 1], eps2)) { ++c; h += mix64((uint64_t)q); }
-        }
-        for (int64_t j = i - 1; j >= 0; --j) {
-            int64_t q = ord[j].id;
-            float dx = xy[2 * q] - xp;
-            float dx2 = dx * dx;
-            if (dx2 > eps2) break;
-            if (is_neighbor_f32(xp, yp, xy[2 * q], xy[2 * q + 1], eps2)) { ++c; h += mix64((uint64_t)q); }
-        }
-        cnt[p] = c;
-        hash[p] = h;
+    float* sx = (float*)malloc(sizeof(float) * (size_t)(n ? n : 1));
+    float* sy = (float*)malloc(sizeof(float) * (size_t)(n ? n : 1));
+    int64_t* sid = (int64_t*)malloc(sizeof(int64_t) * (size_t)(n ? n : 1));
+    if (!sx || !sy || !sid) { free(ord); free(sx); free(sy); free(sid); return -1; }
+    for (int64_t k = 0; k < n; ++k) {
+        sid[k] = ord[k].id;
+        sx[k] = xy[2 * ord[k].id];
+        sy[k] = xy[2 * ord[k].id + 1];
     }
     free(ord);
+    SWEEP_BODY(float, is_neighbor_f32)
+    free(sx); free(sy); free(sid);
     return 0;
 }
+
+/* ------------------------------------------------------------------------ */
+/* O2, third construction: the plane sweep inside horizontal strips.        */
+/* At 50M points (C5) a single x-sorted sweep tests ~5*10^4 points per row; */
+/* here the points are cut into strips b_t <= y < b_{t+1} of width about    */
+/* 2*eps, each strip sorted by (x, id), and row p scans the x-window of its */
+/* own strip and the two adjacent ones exactly as the plane sweep does.     */
+/* Exactness: for p in strip s and q in strip >= s+2 (or <= s-2), the real  */
+/* |y_q - y_p| exceeds the real width b_{t+1} - b_t of a strip between      */
+/* them, so by monotone rounding fl(|y_q - y_p|) >= fl(b_{t+1} - b_t) and   */
+/* d2 >= fl(dy*dy) >= fl(fl(b_{t+1} - b_t)^2).  The code checks that this   */
+/* last value exceeds eps2 for EVERY strip (else it returns -2), so no      */
+/* neighbour is ever outside the three strips.  Per-row output as above.    */
+/* ------------------------------------------------------------------------ */
+static int strip_cmp(const void* a, const void* b)   /* keys (strip, x, id) */
+{
+    const double* u = (const double*)a;
+    const double* v = (const double*)b;
+    if (u[0] < v[0]) return -1;
+    if (u[0] > v[0]) return 1;
+    if (u[1] < v[1]) return -1;
+    if (u[1] > v[1]) return 1;
+    return (u[2] > v[2]) - (u[2] < v[2]);
+}
+
+static int cmp_u32(const void* a, const void* b)
+{
+    uint32_t u = *(const uint32_t*)a, v = *(const uint32_t*)b;
+    return (u > v) - (u < v);
+}
+
+#define DEFINE_STRIPS(T, SUF, IS_NEIGHBOR)                                                     \
+typedef struct { int64_t n, ns; T *sx, *sy; int64_t *sid, *sst, *sbeg; } strips_##SUF;        \
+static void strips_free_##SUF(strips_##SUF* s)                                                 \
+{                                                                                              \
+    free(s->sx); free(s->sy); free(s->sid); free(s->sst); free(s->sbeg);                       \
+}                                                                                              \
+/* 0 = ok, -1 = allocation failed, -2 = a strip is not wider than eps */                      \
+static int strips_build_##SUF(const T* xy, int64_t n, T eps, T eps2, strips_##SUF* s)         \
+{                                                                                              \
+    memset(s, 0, sizeof(*s));                                                                  \
+    s->n = n;                                                                                  \
+    double ymin = 0, ymax = 0;                                                                 \
+    for (int64_t k = 0; k < n; ++k) {                                                          \
+        double y = (double)xy[2 * k + 1];                                                      \
+        if (k == 0 || y < ymin) ymin = y;                                                      \
+        if (k == 0 || y > ymax) ymax = y;                                                      \
+    }                                                                                          \
+    double H = 2.0 * (double)eps;                                                              \
+    if ((ymax - ymin) / H > (double)(1 << 22)) H = (ymax - ymin) / (double)(1 << 22);          \
+    int64_t ns = (int64_t)((ymax - ymin) / H) + 2;                                             \
+    s->ns = ns;                                                                                \
+    T* b = (T*)malloc(sizeof(T) * (size_t)(ns + 1));                                           \
+    s->sbeg = (int64_t*)calloc((size_t)(ns + 1), sizeof(int64_t));                             \
+    int64_t* sk = (int64_t*)malloc(sizeof(int64_t) * (size_t)(n ? n : 1));                     \
+    if (!b || !s->sbeg || !sk) { free(b); free(sk); strips_free_##SUF(s); return -1; }         \
+    for (int64_t t = 0; t <= ns; ++t) b[t] = (T)(ymin + (double)t * H);                       \
+    b[0] = (T)ymin;                                                                            \
+    for (int64_t t = 0; t < ns; ++t) {   /* every strip is wider than eps (header above) */    \
+        T wd = b[t + 1] - b[t];                                                                \
+        T wd2 = wd * wd;                                                                       \
+        if (!(wd2 > eps2)) { free(b); free(sk); strips_free_##SUF(s); return -2; }             \
+    }                                                                                          \
+    if (!((double)b[ns] > ymax)) { free(b); free(sk); strips_free_##SUF(s); return -2; }       \
+    for (int64_t k = 0; k < n; ++k) {   /* strip of k: last t with b[t] <= y */                \
+        T y = xy[2 * k + 1];                                                                   \
+        int64_t lo = 0, hi = ns;                                                               \
+        while (hi - lo > 1) {                                                                  \
+            int64_t m = lo + (hi - lo) / 2;                                                    \
+            if (b[m] <= y) lo = m; else hi = m;                                                \
+        }                                                                                      \
+        sk[k] = lo;                                                                            \
+        s->sbeg[lo + 1]++;                                                                     \
+    }                                                                                          \
+    free(b);                                                                                   \
+    for (int64_t t = 0; t < ns; ++t) s->sbeg[t + 1] += s->sbeg[t];                             \
+    int64_t* cur = (int64_t*)malloc(sizeof(int64_t) * (size_t)(ns + 1));                       \
+    double* key = (double*)malloc(sizeof(double) * 3 * (size_t)(n ? n : 1));                  \
+    s->sst = (int64_t*)malloc(sizeof(int64_t) * (size_t)(n ? n : 1));                          \
+    if (!cur || !key || !s->sst) { free(cur); free(key); free(sk); strips_free_##SUF(s); return -1; } \
+    memcpy(cur, s->sbeg, sizeof(int64_t) * (size_t)(ns + 1));                                  \
+    for (int64_t k = 0; k < n; ++k) {   /* counting scatter by strip */                        \
+        int64_t d = cur[sk[k]]++;                                                              \
+        key[3 * d] = (double)sk[k];                                                            \
+        key[3 * d + 1] = (double)xy[2 * k];                                                    \
+        key[3 * d + 2] = (double)k;                                                            \
+        s->sst[d] = sk[k];                                                                     \
+    }                                                                                          \
+    free(cur); free(sk);                                                                       \
+    int64_t t_;                                                                                \
+    _Pragma("omp parallel for schedule(dynamic, 16)")                                          \
+    for (t_ = 0; t_ < ns; ++t_)   /* each strip by (x, id) */                                  \
+        qsort(key + 3 * s->sbeg[t_], (size_t)(s->sbeg[t_ + 1] - s->sbeg[t_]), 3 * sizeof(double), strip_cmp); \
+    s->sx = (T*)malloc(sizeof(T) * (size_t)(n ? n : 1));                                       \
+    s->sy = (T*)malloc(sizeof(T) * (size_t)(n ? n : 1));                                       \
+    s->sid = (int64_t*)malloc(sizeof(int64_t) * (size_t)(n ? n : 1));                          \
+    if (!s->sx || !s->sy || !s->sid) { free(key); strips_free_##SUF(s); return -1; }           \
+    for (int64_t k = 0; k < n; ++k) {                                                          \
+        s->sid[k] = (int64_t)key[3 * k + 2];                                                   \
+        s->sx[k] = xy[2 * s->sid[k]];                                                          \
+        s->sy[k] = xy[2 * s->sid[k] + 1];                                                      \
+    }                                                                                          \
+    free(key);                                                                                 \
+    return 0;                                                                                  \
+}                                                                                              \
+/* x-window [*jb, *je) of strip t around xp: the plane sweep's stop points     */             \
+/* (exact: fl(x_j - xp) is monotone along the strip's x order)                 */             \
+static void strips_window_##SUF(const strips_##SUF* s, int64_t t, T xp, T eps2, int64_t* jb, int64_t* je) \
+{                                                                                              \
+    int64_t lo = s->sbeg[t], hi = s->sbeg[t + 1];                                              \
+    while (lo < hi) {   /* first j not left-outside (dx < 0, dx^2 > eps2) */                   \
+        int64_t m = lo + (hi - lo) / 2;                                                        \
+        T dx = s->sx[m] - xp;                                                                  \
+        if (dx < 0 && dx * dx > eps2) lo = m + 1; else hi = m;                                 \
+    }                                                                                          \
+    *jb = lo;                                                                                  \
+    hi = s->sbeg[t + 1];                                                                       \
+    while (lo < hi) {   /* first j right-outside (dx > 0, dx^2 > eps2) */                      \
+        int64_t m = lo + (hi - lo) / 2;                                                        \
+        T dx = s->sx[m] - xp;                                                                  \
+        if (dx > 0 && dx * dx > eps2) hi = m; else lo = m + 1;                                 \
+    }                                                                                          \
+    *je = lo;                                                                                  \
+}                                                                                              \
+int oracle_strip_rowhash_##SUF(const T* xy, int64_t n, T eps, uint64_t* cnt, uint64_t* hash)  \
+{                                                                                              \
+    T eps2 = eps * eps;                                                                        \
+    strips_##SUF s;                                                                            \
+    int rc = strips_build_##SUF(xy, n, eps, eps2, &s);                                         \
+    if (rc) return rc;                                                                         \
+    int64_t i;                                                                                 \
+    _Pragma("omp parallel for schedule(dynamic, 256)")                                         \
+    for (i = 0; i < n; ++i) {                                                                  \
+        T xp = s.sx[i], yp = s.sy[i];                                                          \
+        uint64_t c = 0, h = 0;                                                                 \
+        for (int64_t t = s.sst[i] - 1; t <= s.sst[i] + 1; ++t) {                               \
+            if (t < 0 || t >= s.ns) continue;                                                  \
+            int64_t jb, je;                                                                    \
+            strips_window_##SUF(&s, t, xp, eps2, &jb, &je);                                    \
+            for (int64_t j = jb; j < je; ++j) {                                                \
+                int hit = IS_NEIGHBOR(xp, yp, s.sx[j], s.sy[j], eps2);                         \
+                c += (uint64_t)hit;                                                            \
+                h += hit ? mix64((uint64_t)s.sid[j]) : 0;                                      \
+            }                                                                                  \
+        }                                                                                      \
+        cnt[s.sid[i]] = c;                                                                     \
+        hash[s.sid[i]] = h;                                                                    \
+    }                                                                                          \
+    strips_free_##SUF(&s);                                                                     \
+    return 0;                                                                                  \
+}                                                                                              \
+/* O2 as a full CSR table (count then fill, each list ascending): off[n+1]   */               \
+/* is filled here; nbr must hold off[n] entries (second call)                */               \
+int oracle_strip_join_##SUF(const T* xy, int64_t n, T eps, uint64_t* off, uint32_t* nbr)       \
+{                                                                                              \
+    T eps2 = eps * eps;                                                                        \
+    strips_##SUF s;                                                                            \
+    int rc = strips_build_##SUF(xy, n, eps, eps2, &s);                                         \
+    if (rc) return rc;                                                                         \
+    int64_t i;                                                                                 \
+    if (!nbr) {   /* count pass: off[p + 1] = |N_eps(p)|, then the prefix sum */               \
+        off[0] = 0;                                                                            \
+        _Pragma("omp parallel for schedule(dynamic, 256)")                                     \
+        for (i = 0; i < n; ++i) {                                                              \
+            T xp = s.sx[i], yp = s.sy[i];                                                      \
+            uint64_t c = 0;                                                                    \
+            for (int64_t t = s.sst[i] - 1; t <= s.sst[i] + 1; ++t) {                           \
+                if (t < 0 || t >= s.ns) continue;                                              \
+                int64_t jb, je;                                                                \
+                strips_window_##SUF(&s, t, xp, eps2, &jb, &je);                                \
+                for (int64_t j = jb; j < je; ++j) c += (uint64_t)IS_NEIGHBOR(xp, yp, s.sx[j], s.sy[j], eps2); \
+            }                                                                                  \
+            off[s.sid[i] + 1] = c;                                                             \
+        }                                                                                      \
+        for (int64_t p = 0; p < n; ++p) off[p + 1] += off[p];                                  \
+    } else {      /* fill pass: the lists at off[p], sorted ascending */                       \
+        _Pragma("omp parallel for schedule(dynamic, 256)")                                     \
+        for (i = 0; i < n; ++i) {                                                              \
+            T xp = s.sx[i], yp = s.sy[i];                                                      \
+            uint32_t* out = nbr + off[s.sid[i]];                                               \
+            uint64_t c = 0;                                                                    \
+            for (int64_t t = s.sst[i] - 1; t <= s.sst[i] + 1; ++t) {                           \
+                if (t < 0 || t >= s.ns) continue;                                              \
+                int64_t jb, je;                                                                \
+                strips_window_##SUF(&s, t, xp, eps2, &jb, &je);                                \
+                for (int64_t j = jb; j < je; ++j)                                              \
+                    if (IS_NEIGHBOR(xp, yp, s.sx[j], s.sy[j], eps2)) out[c++] = (uint32_t)s.sid[j]; \
+            }                                                                                  \
+            qsort(out, (size_t)c, sizeof(uint32_t), cmp_u32);                                  \
+        }                                                                                      \
+    }                                                                                          \
+    strips_free_##SUF(&s);                                                                     \
+    return 0;                                                                                  \
+}
+
+DEFINE_STRIPS(double, f64, is_neighbor_f64)
+DEFINE_STRIPS(float, f32, is_neighbor_f32)
 
 /* ------------------------------------------------------------------------ */
 /* O3: Algorithm 1 on the neighbour table T.         */

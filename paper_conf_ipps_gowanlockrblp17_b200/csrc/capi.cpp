@@ -66,7 +66,9 @@ hdb_status hdb_ctx_create(const hdb_opts* opts, hdb_ctx** out) {
     if (o.n_devices < 0 || (o.n_devices > 0 && !o.devices)) fail(HDB_EINVAL, "bad device list");
     if (o.shard_count < 0 || (o.shard_count > 0 && (o.shard_rank < 0 || o.shard_rank >= o.shard_count)))
         fail(HDB_EINVAL, "bad shard_rank/shard_count");
-    if (o.cell_split < 0 || o.cell_split > 8) fail(HDB_EINVAL, "cell_split must be in [0, 8]");
+    // the search kernels hold 2k+1 <= kMaxSpans row spans per group (kernels_search.cu)
+    if (o.cell_split < 0 || o.cell_split > kMaxCellSplit)
+        fail(HDB_EINVAL, "cell_split must be in [0, %d]", kMaxCellSplit);
     if (o.sweep_on_device != 0 && o.sweep_on_device != 1) fail(HDB_EINVAL, "sweep_on_device must be 0 or 1");
     c = new hdb_ctx;
     int ndev_avail = 0;
@@ -113,8 +115,8 @@ hdb_status hdb_ctx_create(const hdb_opts* opts, hdb_ctx** out) {
         size_t free_b = 0;
         HDB_CUDA(cudaMemGetInfo(&free_b, &dc.total_mem));
         dc.scan_ep.cap = 1u << 20;   // tiles of 2,048 elements: scans of up to 2^31 elements
-        HDB_CUDA(cudaMalloc((void**)&dc.scan_ep.tiles, dc.scan_ep.cap * sizeof(unsigned long long)));
-        HDB_CUDA(cudaMemset(dc.scan_ep.tiles, 0, dc.scan_ep.cap * sizeof(unsigned long long)));
+        HDB_CUDA(cudaMalloc((void**)&dc.scan_ep.tiles, (dc.scan_ep.cap + 1) * sizeof(unsigned long long)));
+        HDB_CUDA(cudaMemset(dc.scan_ep.tiles, 0, (dc.scan_ep.cap + 1) * sizeof(unsigned long long)));
         HDB_CUDA(cudaMemPoolSetAttribute(dc.big_pool, cudaMemPoolAttrReleaseThreshold, &thr));
         c->dev.push_back(dc);
     }
@@ -458,8 +460,9 @@ hdb_status hdb_sweep(hdb_ctx* c, const void* xy, uint64_t n, hdb_dtype dt, const
         }
     std::lock_guard<std::recursive_mutex> lk(c->mu);
     HDB_GUARD_BEGIN
+    // a process shard builds only its rows of T: clustering it would be silently wrong
+    if (c->opts.shard_count > 1) fail(HDB_EINVAL, "hdb_sweep needs an unsharded context (shard_count <= 1)");
     if (c->opts.sweep_on_device) {
-        if (c->opts.shard_count > 1) fail(HDB_EINVAL, "sweep_on_device needs an unsharded context");
         // NEXT-4 variant: T(eps_i) stays in HBM; every minpts variant runs the
         // device DBSCAN on it and only labels cross PCIe.
         for (uint32_t i = 0; i < n_eps; ++i) {
@@ -498,7 +501,8 @@ hdb_status hdb_sweep(hdb_ctx* c, const void* xy, uint64_t n, hdb_dtype dt, const
         for (uint32_t i = 0; i < n_eps; ++i) {
             {
                 std::unique_lock<std::mutex> l(m);
-                cv.wait(l, [&] { return slot_free; });
+                cv.wait(l, [&] { return slot_free || done; });
+                if (done) return;   // the consumer stopped (a DBSCAN variant failed)
                 slot_free = false;
             }
             hdb_grid* g = nullptr;
@@ -566,8 +570,14 @@ hdb_status hdb_sweep(hdb_ctx* c, const void* xy, uint64_t n, hdb_dtype dt, const
                 {
                     std::lock_guard<std::mutex> l(m);
                     done = true;
+                    cv.notify_all();
                 }
                 producer.join();
+                // tables the producer queued meanwhile are freed before reporting
+                while (!q.empty()) {
+                    table_free(q.front().second);
+                    q.pop_front();
+                }
                 fail(s, "sweep: DBSCAN variant failed");
             }
     }

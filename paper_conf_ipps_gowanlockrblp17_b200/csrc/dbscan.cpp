@@ -315,8 +315,7 @@ void canonicalize(hdb_table* t) {
     t->nbrs = nv;
     t->npairs = acc;
     t->malloced = true;
-    t->first_query = 0;
-    t->end_query = n;
+    // first_query / end_query are kept: a process shard stays a shard (hdb_dbscan rejects it)
 }
 
 }  // namespace hdb

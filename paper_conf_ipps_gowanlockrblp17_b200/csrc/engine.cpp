@@ -1208,8 +1208,22 @@ void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hd
                      (unsigned long long)P, (unsigned long long)ctx->opts.host_budget_bytes);
             t->npairs = P;
             const bool whole = (parts == 1);
-            t->first_query = whole ? 0 : sh[0].r.q0;
-            t->end_query = whole ? n : sh[ndev - 1].r.q1;
+            // this process's rows: [first_query, end_query) of the sorted order -- the whole
+            // table unless the process is one of several shards (R_proc > 1); empty shards
+            // (q0 = q1 = 0) do not count
+            if (R_proc == 1) {
+                t->first_query = 0;
+                t->end_query = n;
+            } else {
+                t->first_query = t->end_query = 0;
+                bool any = false;
+                for (size_t d = 0; d < ndev; ++d) {
+                    if (sh[d].r.q1 <= sh[d].r.q0) continue;
+                    t->first_query = any ? std::min(t->first_query, sh[d].r.q0) : sh[d].r.q0;
+                    t->end_query = any ? std::max(t->end_query, sh[d].r.q1) : sh[d].r.q1;
+                    any = true;
+                }
+            }
 
             if (device_resident) {
                 // ---- a8 into a device-resident table

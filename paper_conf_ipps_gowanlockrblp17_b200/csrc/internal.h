@@ -37,6 +37,7 @@ struct Error {
 constexpr int kGroup = 32;
 constexpr int kSearchThreads = 256;
 constexpr int kCounterSlots = 64;   // slot 0: count pass; 1 + stream index: write passes
+constexpr int kMaxCellSplit = 6;    // cell_split k <= 6: 2k+1 <= 13 stencil row spans (kMaxSpans)
 
 // ---------------------------------------------------------------- grid
 // One device's copy of the grid (Fig. 1 re-laid out):
@@ -147,9 +148,10 @@ size_t scan_temp_bytes(uint64_t n);
 // Scans issued by a thread while a ScanEpochScope is alive use it (all on one stream: the
 // scans of one scope must not run concurrently); others zero their status tiles in temp.
 struct ScanEpochs {
-    unsigned long long* tiles = nullptr;
+    unsigned long long* tiles = nullptr;   // cap tile words + the tile-id counter (tiles[cap])
     uint64_t cap = 0;      // tiles
     uint32_t epoch = 0;    // last epoch used
+    uint64_t ctr_base = 0; // tile ids handed out so far by tiles[cap] (scans in stream order)
 };
 extern thread_local ScanEpochs* t_scan_epochs;
 struct ScanEpochScope {

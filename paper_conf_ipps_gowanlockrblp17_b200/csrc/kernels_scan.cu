@@ -23,9 +23,13 @@ constexpr int SC_TILE = SC_THREADS * SC_ITEMS;
 // publishes its aggregate, then its inclusive prefix once known, as one packed
 // 64-bit word {status:2, value:62}; a tile finds its exclusive prefix by walking
 // back over its predecessors' words, 32 at a time (one per lane of warp 0),
-// summing aggregates until it meets an inclusive prefix.  Tiles are blockIdx
-// ordered and only wait on lower tiles, which the hardware dispatched first.
-// One kernel per scan (plus a memset of the tile words).
+// summing aggregates until it meets an inclusive prefix.  A CTA takes its tile
+// index from an atomic counter when it starts (not blockIdx.x: the CUDA model
+// does not promise dispatch in blockIdx order), so a tile only ever waits on
+// tiles whose CTAs are already running -- no deadlock under concurrent kernels
+// or MPS.  The counter is never reset: a scan's tiles are the counter values
+// [ctr_base, ctr_base + nb), ctr_base tracked on the host (stream order).
+// One kernel per scan (plus a memset of the tile words on the memset path).
 // Tile status word: flag (2 bits: aggregate / inclusive prefix) | epoch (20 bits) | value (42 bits).
 // A word is ready only with a flag and the scan's own epoch: memset-path scans use epoch 0 on a
 // zeroed buffer; epoch scans (ScanEpochScope) reuse one zeroed per-device buffer with a new
@@ -47,12 +51,16 @@ __device__ __forceinline__ uint64_t peek(const unsigned long long* w) {
 template <typename Tin, typename Tout>
 __global__ void __launch_bounds__(SC_THREADS) k_scan_lookback(const Tin* __restrict__ in, Tout* __restrict__ out,
                                                               uint64_t n, unsigned long long* __restrict__ tiles,
-                                                              uint64_t ep) {
+                                                              uint64_t ep, unsigned long long* __restrict__ ctr,
+                                                              uint64_t ctr_base) {
     __shared__ Tout buf[SC_TILE];
     __shared__ Tout wsum[SC_THREADS / 32];
     __shared__ Tout s_excl;
+    __shared__ uint64_t s_tile;
     const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
-    const uint64_t t = blockIdx.x;
+    if (tid == 0) s_tile = ctr ? atomicAdd(ctr, 1ull) - ctr_base : 0;
+    __syncthreads();
+    const uint64_t t = s_tile;
     const uint64_t base = t * SC_TILE;
 #pragma unroll
     for (int i = 0; i < SC_ITEMS; ++i) {
@@ -131,22 +139,28 @@ void scan_impl(const Tin* in, Tout* out, uint64_t n, void* temp, cudaStream_t s)
     }
     const uint64_t nb = (n + SC_TILE - 1) / SC_TILE;
     unsigned long long* tiles = nullptr;
-    uint64_t ep = 0;
+    unsigned long long* ctr = nullptr;   // tile-id counter (null: one tile, id 0)
+    uint64_t ep = 0, ctr_base = 0;
     if (nb > 1) {
         ScanEpochs* se = t_scan_epochs;
         if (se && nb <= se->cap) {
-            if (++se->epoch > kEpMask) {   // epochs wrap: start again on a zeroed buffer
-                cudaMemsetAsync(se->tiles, 0, se->cap * sizeof(unsigned long long), s);
+            if (++se->epoch > kEpMask) {   // epochs wrap: start again on a zeroed buffer (+ counter)
+                cudaMemsetAsync(se->tiles, 0, (se->cap + 1) * sizeof(unsigned long long), s);
                 se->epoch = 1;
+                se->ctr_base = 0;
             }
             tiles = se->tiles;
+            ctr = se->tiles + se->cap;
+            ctr_base = se->ctr_base;
+            se->ctr_base += nb;
             ep = (uint64_t)se->epoch << kEpShift;
         } else {
             tiles = (unsigned long long*)temp;
-            cudaMemsetAsync(tiles, 0, nb * sizeof(unsigned long long), s);
+            ctr = tiles + nb;
+            cudaMemsetAsync(tiles, 0, (nb + 1) * sizeof(unsigned long long), s);
         }
     }
-    k_scan_lookback<Tin, Tout><<<(unsigned)nb, SC_THREADS, 0, s>>>(in, out, n, tiles, ep);
+    k_scan_lookback<Tin, Tout><<<(unsigned)nb, SC_THREADS, 0, s>>>(in, out, n, tiles, ep, ctr, ctr_base);
     ++g_kernel_launches;
 }
 
@@ -155,7 +169,7 @@ void scan_impl(const Tin* in, Tout* out, uint64_t n, void* temp, cudaStream_t s)
 thread_local ScanEpochs* t_scan_epochs = nullptr;
 
 size_t scan_temp_bytes(uint64_t n) {
-    return ((n + SC_TILE - 1) / SC_TILE + 1) * sizeof(unsigned long long) + 64;
+    return ((n + SC_TILE - 1) / SC_TILE + 2) * sizeof(unsigned long long) + 64;   // tile words + counter
 }
 
 void scan_u32_to_u32(const uint32_t* in, uint32_t* out, uint64_t n, void* temp, cudaStream_t s) {

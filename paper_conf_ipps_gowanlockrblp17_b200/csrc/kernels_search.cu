@@ -242,6 +242,7 @@ __device__ __forceinline__ void flush_window(uint2 (*swin)[kWinPad], uint2* gmas
 // at k = 3).  VSpan r: [lo, hi) of the span, its first pair index and the
 // position of that pair in the virtual sequence; entry nspan holds the total.
 constexpr int kMaxSpans = 13;   // 2k + 1 for cell_split k <= 6
+static_assert(kMaxSpans >= 2 * kMaxCellSplit + 1, "span table too small for the largest cell split");
 struct VSpan {
     uint32_t lo, hi, pbase, vstart;
 };

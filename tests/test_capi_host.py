@@ -187,7 +187,7 @@ def test_ctx_create_without_gpu_fails_loudly():
     assert e.value.status == hdb.HDB_ECUDA
 
 
-@pytest.mark.parametrize("bad", [dict(sweep_on_device=2), dict(cell_split=9), dict(n_streams=0),
+@pytest.mark.parametrize("bad", [dict(sweep_on_device=2), dict(cell_split=9), dict(cell_split=7), dict(n_streams=0),
                                  dict(sample_fraction=0.0), dict(alpha=-1.0), dict(shard_count=2, shard_rank=2)])
 def test_opts_validation_before_device(bad):
     """Option errors are reported as HDB_EINVAL before any device is touched."""

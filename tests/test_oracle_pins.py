@@ -255,12 +255,48 @@ def test_plane_sweep_equals_brute_force(dtype):
         c1, h1 = oracle.sweep_rowhash(xy, eps, dtype=dtype)
         np.testing.assert_array_equal(c0, c1)
         np.testing.assert_array_equal(h0, h1)
+        c2, h2 = oracle.strip_rowhash(xy, eps, dtype=dtype)
+        np.testing.assert_array_equal(c0, c2)
+        np.testing.assert_array_equal(h0, h2)
+        off0, nbr0 = oracle.eps_join(xy, eps, dtype=dtype)
+        off1, nbr1 = oracle.strip_join(xy, eps, dtype=dtype)
+        np.testing.assert_array_equal(off0, off1)
+        np.testing.assert_array_equal(nbr0, nbr1)
 
 
-def test_plane_sweep_lattice_golden():
+@pytest.mark.parametrize("dtype", ["f64", "f32"])
+def test_strip_sweep_equals_brute_force_on_strip_edges(dtype):
+    """The strip sweep (the plane sweep inside horizontal strips of width ~2 eps,
+    used for the 50M-point rows of C5) against brute force where the strips
+    matter: neighbours straddling strip boundaries, points exactly on the
+    boundaries y = ymin + t * 2 eps, a single column (one strip per point
+    pair), a domain tall enough to cap the strip count, dense skew."""
+    rng = np.random.default_rng(5)
+    eps = 0.25
+    on_edges = np.stack([rng.uniform(0, 6, 2000), np.floor(rng.uniform(0, 12, 2000)) * 2 * eps], 1)
+    near_edges = on_edges + np.stack([np.zeros(2000), rng.choice([-1, 1], 2000) * rng.uniform(0, 1e-9, 2000)], 1)
+    column = np.stack([np.full(1500, 3.0), np.sort(rng.uniform(0, 40, 1500))], 1)
+    tall = np.stack([rng.uniform(0, 1, 1200), rng.uniform(-5e6, 5e6, 1200)], 1)
+    tall[:600, 1] = rng.uniform(0, 2, 600)   # plus a dense patch
+    sets = [(on_edges, eps), (near_edges, eps), (np.concatenate([on_edges, near_edges]), 2 * eps),
+            (column, eps), (tall, 0.05), (datagen.dense_skew(20_000, seed=9), 4.0),
+            (datagen.near_ties(2500, 0.45, seed=13, extent=20.0), 0.45)]
+    for xy, e in sets:
+        c0, h0 = oracle.eps_join_rowhash(xy, e, dtype=dtype)
+        c1, h1 = oracle.strip_rowhash(xy, e, dtype=dtype)
+        np.testing.assert_array_equal(c0, c1)
+        np.testing.assert_array_equal(h0, h1)
+        off0, nbr0 = oracle.eps_join(xy, e, dtype=dtype)
+        off1, nbr1 = oracle.strip_join(xy, e, dtype=dtype)
+        np.testing.assert_array_equal(off0, off1)
+        np.testing.assert_array_equal(nbr0, nbr1)
+
+
+@pytest.mark.parametrize("fn", ["sweep_rowhash", "strip_rowhash"])
+def test_plane_sweep_lattice_golden(fn):
     g = _gold("lattice5.json")
     xy = datagen.lattice(g["k"])
-    c, _ = oracle.sweep_rowhash(xy, g["eps_sqrt2"]["eps"])
+    c, _ = getattr(oracle, fn)(xy, g["eps_sqrt2"]["eps"])
     assert sorted(set(c.tolist())) == sorted({g["eps_sqrt2"]["count_corner"], g["eps_sqrt2"]["count_edge"],
                                               g["eps_sqrt2"]["count_interior"]})
     assert int(c.sum()) == 4 * g["eps_sqrt2"]["count_corner"] + 12 * g["eps_sqrt2"]["count_edge"] \

@@ -1,0 +1,169 @@
+"""GPU parity at FULL size on every config (north_star target: "bit-exact
+eps-neighbor tables and DBSCAN partitions vs the oracle on all five configs").
+
+* Tables: EVERY row of the library's table -- (count, sum of mix64(id)) per
+  row, hashed on the GPU by the test helper tests/_rowhash.py -- against the
+  oracle's strip sweep (``oracle.strip_rowhash``, pinned equal to brute force
+  and to the plane sweep in tests/test_oracle_pins.py).  Device tables in the
+  launch configuration bench.py times (library defaults), plus the batched
+  host-table path (the e2e leg).
+* Partitions: labels / core flags / cluster count of the library's DBSCAN
+  (host DBSCAN on a host table, device DBSCAN on a device table) against the
+  oracle's Alg. 1 (``oracle.dbscan``) run on the oracle's own full table
+  (``oracle.strip_join``) -- C2 at eps 0.15 and 0.45, C3 at eps 0.20.
+* The C4 sweep (eps {0.15, 0.45} x minpts {4, 8, 16}) through ``hdb_sweep``,
+  hybrid (host DBSCAN) and on-device.
+
+Not marked ``slow``: the driver's ``-m gpu`` run must collect them.
+"""
+import functools
+
+import numpy as np
+import pytest
+
+import datagen
+import oracle
+from paper_conf_ipps_gowanlockrblp17_b200 import hdb
+import _rowhash
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def torch_cuda():
+    import torch
+    assert torch.cuda.is_available(), "GPU tests need a CUDA device"
+    torch.cuda.set_device(0)
+    return torch
+
+
+@functools.lru_cache(maxsize=None)
+def _data(name):
+    if name == "C2":
+        return datagen.tec_like()
+    if name == "C2f32":
+        return datagen.tec_like().astype(np.float32)
+    if name == "C3":
+        return datagen.sdss_like()
+    if name == "C3L":
+        return datagen.sdss_like(datagen.C3_N_LARGE, seed=4)
+    if name == "C5":
+        return datagen.dense_skew()
+    raise KeyError(name)
+
+
+@functools.lru_cache(maxsize=4)
+def _oracle_table(name, eps):
+    return oracle.strip_join(_data(name), eps)
+
+
+@functools.lru_cache(maxsize=None)
+def _oracle_dbscan(name, eps, minpts):
+    off, nbr = _oracle_table(name, eps)
+    return oracle.dbscan(off, nbr, minpts)
+
+
+def _rows_equal(torch, xy, eps, dtype, view):
+    b, c, v = _rowhash.view_tensors(torch, view)
+    got_c, got_h = _rowhash.table_rowhash(torch, b, c, v)
+    del b, c, v
+    want_c, want_h = oracle.strip_rowhash(xy, eps, dtype=dtype)
+    bad = np.nonzero(got_c != want_c)[0]
+    assert bad.size == 0, f"{bad.size} rows with a wrong count, e.g. {bad[:8]}: {got_c[bad[:8]]} vs {want_c[bad[:8]]}"
+    bad = np.nonzero(got_h != want_h)[0]
+    assert bad.size == 0, f"{bad.size} rows with a wrong neighbour set, e.g. {bad[:8]}"
+    assert int(view.npairs) == int(want_c.sum())
+
+
+CASES = [("C2", 0.15, "f64"), ("C2", 0.45, "f64"), ("C2", 1.40, "f64"), ("C2f32", 0.45, "f32"),
+         ("C3", 0.07, "f64"), ("C3", 0.12, "f64"), ("C3", 0.20, "f64"),
+         ("C3L", 0.07, "f64"), ("C3L", 0.12, "f64"), ("C3L", 0.20, "f64"),
+         ("C5", 0.5, "f64")]
+
+
+@pytest.mark.parametrize("name,eps,dtype", CASES, ids=[f"{c[0]}-eps{c[1]}" for c in CASES])
+def test_full_size_device_table_every_row(torch_cuda, name, eps, dtype):
+    torch = torch_cuda
+    xy = _data(name)
+    ctx = hdb.hdb_ctx_create()
+    try:
+        g = hdb.hdb_grid_build(ctx, torch.from_numpy(xy).cuda(), eps)
+        try:
+            t = hdb.hdb_neighbor_table_device(ctx, g)
+        finally:
+            hdb.hdb_grid_free(g)
+        try:
+            view = hdb.hdb_table_view_get(t)
+            assert view.on_device and view.first_query == 0 and view.end_query == xy.shape[0]
+            _rows_equal(torch, xy, eps, dtype, view)
+        finally:
+            hdb.hdb_table_free(t)
+    finally:
+        hdb.hdb_ctx_destroy(ctx)
+    torch.cuda.empty_cache()
+
+
+def test_full_size_host_table_every_row(torch_cuda):
+    """The e2e leg: pinned host points -> batched write + D2H on 3 streams into the host table."""
+    torch = torch_cuda
+    xy = _data("C2")
+    ctx = hdb.hdb_ctx_create()
+    try:
+        g = hdb.hdb_grid_build(ctx, xy, 0.45)
+        try:
+            t = hdb.hdb_neighbor_table(ctx, g)
+        finally:
+            hdb.hdb_grid_free(g)
+        try:
+            view = hdb.hdb_table_view_get(t)
+            assert not view.on_device
+            _rows_equal(torch, xy, 0.45, "f64", view)
+        finally:
+            hdb.hdb_table_free(t)
+        st = hdb.hdb_stats_get(ctx)
+        assert st["n_batches"] >= 3
+    finally:
+        hdb.hdb_ctx_destroy(ctx)
+
+
+@pytest.mark.parametrize("name,eps", [("C2", 0.15), ("C2", 0.45), ("C3", 0.20)])
+def test_full_size_dbscan_partition(torch_cuda, name, eps):
+    torch = torch_cuda
+    xy = _data(name)
+    want_lab, want_core, want_k = _oracle_dbscan(name, eps, datagen.MINPTS)
+    ctx = hdb.hdb_ctx_create()
+    try:
+        for device in (False, True):
+            g = hdb.hdb_grid_build(ctx, xy, eps)
+            try:
+                t = (hdb.hdb_neighbor_table_device if device else hdb.hdb_neighbor_table)(ctx, g)
+            finally:
+                hdb.hdb_grid_free(g)
+            try:
+                lab, core, k = hdb.hdb_dbscan(t, datagen.MINPTS)
+            finally:
+                hdb.hdb_table_free(t)
+            where = "device DBSCAN" if device else "host DBSCAN"
+            assert k == want_k, where
+            assert np.array_equal(core, want_core), where
+            bad = np.nonzero(lab != want_lab)[0]
+            assert bad.size == 0, f"{where}: {bad.size} labels differ, e.g. {bad[:8]}"
+    finally:
+        hdb.hdb_ctx_destroy(ctx)
+
+
+@pytest.mark.parametrize("on_device", [0, 1])
+def test_full_size_c4_sweep(torch_cuda, on_device):
+    xy = _data("C2")
+    eps_list, mp = (0.15, 0.45), (4, 8, 16)
+    ctx = hdb.hdb_ctx_create(sweep_on_device=on_device)
+    try:
+        labels, k = hdb.hdb_sweep(ctx, xy, eps_list, mp)
+    finally:
+        hdb.hdb_ctx_destroy(ctx)
+    for i, eps in enumerate(eps_list):
+        for j, m in enumerate(mp):
+            want_lab, _, want_k = _oracle_dbscan("C2", eps, m)
+            assert k[i, j] == want_k, (eps, m)
+            bad = np.nonzero(labels[i, j] != want_lab)[0]
+            assert bad.size == 0, f"eps {eps} minpts {m}: {bad.size} labels differ"
