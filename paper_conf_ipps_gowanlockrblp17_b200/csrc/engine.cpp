@@ -430,57 +430,54 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
     set_filter_bound(g);
 
     tr.mark("bbox+sync");
-    // ---- a2: keys
-    // ids and points are padded by 2 entries: the search kernels load candidate
-    // pairs (2k, 2k+1) with one vector load and mask the invalid half
+    // ---- a2 + a3: the points sorted by cell key (record radix sort over only the bits the
+    // key range needs; the first pass computes the keys from the input points, the last
+    // writes A, the sorted points and the f32 filter copy -- no separate gather).  ids and
+    // points are padded by 2 entries: the search kernels load candidate pairs (2k, 2k+1)
+    // with one vector load and mask the invalid half
     const int kb = g.n_cells <= (1ull << 32) ? 4 : 8;   // 32-bit keys whenever they fit
-    DBuf k0(kb * n, s), v0(4 * (n + 2), s), k1(kb * n, s), v1(4 * (n + 2), s);
-    launch_keys(xin, n, dt, g.xmin, g.ymin, g.inv_w, g.nx, g.ny, k0.p, kb, v0.as<uint32_t>(), s);
-    HDB_LAUNCH_CHECK();
-    // ---- a3: stable radix sort by key (only the bits the key range needs)
     int bits = 1;
     while (bits < 64 && (1ull << bits) < g.n_cells) ++bits;
-    size_t tb = std::max(radix_sort_temp_bytes(n), scan_temp_bytes(n + 1));
-    DBuf temp(tb, s);
-    int which = radix_sort_pairs(k0.p, v0.as<uint32_t>(), k1.p, v1.as<uint32_t>(), kb, n, bits, temp.p, s);
-    HDB_LAUNCH_CHECK();
-    DBuf keys = which ? std::move(k1) : std::move(k0);
-    DBuf ids = which ? std::move(v1) : std::move(v0);
-    k0.reset();
-    k1.reset();
-    v0.reset();
-    v1.reset();
+    DBuf keys(kb * (n ? n : 1), s), ids(4 * (n + 2), s);
     DBuf xy_s((n + 2) * esz, s);
     DBuf xp(16 * (n / 2 + 2), s);
     DBuf counters(4 * kCounterSlots, s);
-    // (the gather also zeroes the padding of xy_s / ids / xp and the work counters)
-    launch_gather_points(xin, ids.as<uint32_t>(), n, dt, xy_s.p, xp.as<float4>(), g.ox, g.oy,
-                         counters.as<unsigned int>(), kCounterSlots, s);
-    HDB_LAUNCH_CHECK();
+    if (n > 0) {
+        DBuf stemp(point_sort_temp_bytes(n, dt, kb, bits), s);   // stream-ordered: freed after the sort
+        sort_points(xin, n, dt, g.xmin, g.ymin, g.inv_w, g.nx, g.ny, kb, bits, keys.p, ids.as<uint32_t>(), xy_s.p,
+                    xp.as<float4>(), g.ox, g.oy, counters.as<unsigned int>(), kCounterSlots, stemp.p, s);
+        HDB_LAUNCH_CHECK();
+    } else {
+        HDB_CUDA(cudaMemsetAsync(ids.p, 0, 8, s));
+        HDB_CUDA(cudaMemsetAsync(xy_s.p, 0, 2 * esz, s));
+        HDB_CUDA(cudaMemsetAsync(xp.p, 0, 32, s));
+        HDB_CUDA(cudaMemsetAsync(counters.p, 0, 4 * kCounterSlots, s));
+    }
     xin_owned.reset();
-    tr.mark("keys+sort+gather(enqueue)");
-    // ---- a4: run boundaries -> scan -> (key, start) of the non-empty cells
-    DBuf flags(4 * n, s), pos(4 * (n + 1), s);
-    launch_cell_flags(keys.p, kb, n, flags.as<uint32_t>(), s);
-    scan_u32_to_u32(flags.as<uint32_t>(), pos.as<uint32_t>(), n, temp.p, s);
-    HDB_LAUNCH_CHECK();
+    DBuf temp(scan_temp_bytes(n + 1), s);
+    tr.mark("sort(enqueue)");
+    // ---- a4: run-length encoding of the sorted keys -> (key, start) of the non-empty cells
+    // (one scan kernel; the arrays are sized by n, the cell count is read back)
+    DBuf ckey(8 * (n ? n : 1), s), cstart(4 * (n + 1), s);
     uint32_t* hne_p = (uint32_t*)(dc.pin + 26);
     *hne_p = 0;
-    HDB_CUDA(cudaMemcpyAsync(hne_p, pos.as<uint32_t>() + n, 4, cudaMemcpyDeviceToHost, s));
+    {
+        DBuf dne(8, s);
+        cell_rle(keys.p, kb, n, ckey.as<uint64_t>(), cstart.as<uint32_t>(), dne.as<uint32_t>(), temp.p, s);
+        HDB_LAUNCH_CHECK();
+        HDB_CUDA(cudaMemcpyAsync(hne_p, dne.p, 4, cudaMemcpyDeviceToHost, s));
+    }
     HDB_CUDA(cudaStreamSynchronize(s));
     const uint32_t hne = *hne_p;
     g.n_nonempty = hne;
     const uint64_t nne = hne;
-    DBuf ckey(8 * nne, s), cstart(4 * (nne + 1), s);
-    launch_cell_scatter(keys.p, kb, flags.as<uint32_t>(), pos.as<uint32_t>(), n, ckey.as<uint64_t>(),
-                        cstart.as<uint32_t>(), s);
-    HDB_LAUNCH_CHECK();
-    flags.reset();
-    pos.reset();
+    // group-level arrays are sized (and scanned) by a bound on the group count instead of n:
+    // a cell of c points has ceil(c / 32) <= c / 32 + 1 groups
+    const uint64_t NG = std::min<uint64_t>(n, nne + n / kGroup + 1);
     keys.reset();
     tr.mark("cells+sync");
     // ---- stencil row spans per non-empty cell + query groups + hit-mask layout,
-    // sized by upper bounds (groups <= n) so that one sync reads both counts
+    // sized by upper bounds (groups <= NG) so that one sync reads both counts
     DBuf cspan(8 * g.nspan * nne, s), gcount(4 * (nne + 1), s), gofs(4 * (nne + 1), s);
     // the paper's dense G (Fig. 1) as a lookup, when the full grid is not much larger than the
     // data: cnext[h] = first non-empty cell with key >= h (a scan of the occupancy marks)
@@ -500,7 +497,7 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
     cnext.reset();
     scan_u32_to_u32(gcount.as<uint32_t>(), gofs.as<uint32_t>(), nne, temp.p, s);
     HDB_LAUNCH_CHECK();
-    DBuf gstart(4 * (n + 1), s), gcell(4 * (n + 1), s);
+    DBuf gstart(4 * (NG + 1), s), gcell(4 * (NG + 1), s);
     launch_group_build(cstart.as<uint32_t>(), gofs.as<uint32_t>(), nne, n, gstart.as<uint32_t>(),
                        gcell.as<uint32_t>(), s);
     HDB_LAUNCH_CHECK();
@@ -523,36 +520,36 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
     const uint32_t max_tests = sparse_max_tests();
     const bool classify = (sk == 0 || sk == 1 || sk == 2 || sk == 4) && max_tests > 0 && n > 0;
     DBuf dpre, spre, dl, sql, ord;
-    DBuf words(4 * (n + 1), s);   // hit-mask words per group (written with the classification)
+    DBuf words(4 * (NG + 1), s);   // hit-mask words per group (written with the classification)
     unsigned long long* nsp = bb + 8;
     if (classify) {
-        DBuf dflag(4 * (n + 1), s), sqn(4 * (n + 1), s), gbin(n + 1, s);
+        DBuf dflag(4 * (NG + 1), s), sqn(4 * (NG + 1), s), gbin(NG + 1, s);
         uint32_t* ohist = (uint32_t*)(bb + 32);   // 2 x kOrderBins words, zeroed by the bbox init
-        ord = DBuf(4 * (n + 1), s);
-        dpre = DBuf(4 * (n + 1), s);
-        spre = DBuf(4 * (n + 1), s);
-        dl = DBuf(4 * (n + 1), s);
+        ord = DBuf(4 * (NG + 1), s);
+        dpre = DBuf(4 * (NG + 1), s);
+        spre = DBuf(4 * (NG + 1), s);
+        dl = DBuf(4 * (NG + 1), s);
         sql = DBuf(8 * (n + 1), s);
         const uint32_t* ngd = gofs.as<uint32_t>() + nne;
         // nsp: [0] sparse queries, [1] candidate tests (zeroed by the bbox init)
-        launch_group_class(g.cstart, g.cspan, g.nspan, g.gstart, g.gcell, ngd, n, max_tests, dflag.as<uint32_t>(),
+        launch_group_class(g.cstart, g.cspan, g.nspan, g.gstart, g.gcell, ngd, NG, max_tests, dflag.as<uint32_t>(),
                            sqn.as<uint32_t>(), nsp, (uint8_t*)gbin.p, ohist, words.as<uint32_t>(), kMaskWin, s);
-        launch_order_scatter((const uint8_t*)gbin.p, ngd, n, ohist, ord.as<uint32_t>(), s);
-        scan_u32_to_u32(dflag.as<uint32_t>(), dpre.as<uint32_t>(), n, temp.p, s);
-        scan_u32_to_u32(sqn.as<uint32_t>(), spre.as<uint32_t>(), n, temp.p, s);
-        launch_group_lists(g.gstart, g.gcell, ngd, n, dpre.as<uint32_t>(), spre.as<uint32_t>(), dl.as<uint32_t>(),
+        launch_order_scatter((const uint8_t*)gbin.p, ngd, NG, ohist, ord.as<uint32_t>(), s);
+        scan_u32_to_u32(dflag.as<uint32_t>(), dpre.as<uint32_t>(), NG, temp.p, s);
+        scan_u32_to_u32(sqn.as<uint32_t>(), spre.as<uint32_t>(), NG, temp.p, s);
+        launch_group_lists(g.gstart, g.gcell, ngd, NG, dpre.as<uint32_t>(), spre.as<uint32_t>(), dl.as<uint32_t>(),
                            sql.as<uint2>(), s);
         HDB_LAUNCH_CHECK();
     }
     {
-        DBuf mtemp(scan_temp_bytes(n + 1), s), moff(8 * (n + 1), s);
-        if (!classify) launch_mask_words(g, gofs.as<uint32_t>() + nne, n, words.as<uint32_t>(), s);
-        scan_u32_to_u64(words.as<uint32_t>(), moff.as<uint64_t>(), n, mtemp.p, s);
+        DBuf mtemp(scan_temp_bytes(NG + 1), s), moff(8 * (NG + 1), s);
+        if (!classify) launch_mask_words(g, gofs.as<uint32_t>() + nne, NG, words.as<uint32_t>(), s);
+        scan_u32_to_u64(words.as<uint32_t>(), moff.as<uint64_t>(), NG, mtemp.p, s);
         HDB_LAUNCH_CHECK();
         // [18] groups, [19] mask words, [20] dense groups, [21] sparse queries, [22] sparse count,
         // [23] candidate tests: gathered on the device, one pinned readback
-        launch_readback(bb + 16, gofs.as<uint32_t>() + nne, moff.as<uint64_t>() + n,
-                        classify ? dpre.as<uint32_t>() + n : nullptr, classify ? spre.as<uint32_t>() + n : nullptr,
+        launch_readback(bb + 16, gofs.as<uint32_t>() + nne, moff.as<uint64_t>() + NG,
+                        classify ? dpre.as<uint32_t>() + NG : nullptr, classify ? spre.as<uint32_t>() + NG : nullptr,
                         classify ? nsp : nullptr, s);
         uint64_t* pr = dc.pin + 18;
         HDB_CUDA(cudaMemcpyAsync(pr, bb + 16, 48, cudaMemcpyDeviceToHost, s));

@@ -98,20 +98,19 @@ void launch_readback(unsigned long long* out, const uint32_t* ng, const uint64_t
 void launch_bbox(const void* xy, uint64_t n, hdb_dtype dt, unsigned long long* bb, unsigned int* bad,
                  cudaStream_t s);
 double bbox_decode(unsigned long long v, bool is_max);
-// keys: key_bytes = 4 (grids of <= 2^32 cells) or 8
-void launch_keys(const void* xy, uint64_t n, hdb_dtype dt, double xmin, double ymin, double inv_w,
-                 uint32_t nx, uint32_t ny, void* keys, int key_bytes, uint32_t* vals, cudaStream_t s);
 size_t radix_sort_temp_bytes(uint64_t n);
 // Stable LSD radix sort of (keys, vals) on the low `bits` bits.  Ping-pongs
 // between (k0,v0) and (k1,v1); returns 0 if the result is in (k0,v0), 1 else.
 int radix_sort_pairs(void* k0, uint32_t* v0, void* k1, uint32_t* v1, int key_bytes, uint64_t n, int bits,
                      void* temp, cudaStream_t s);
-// gather sorted points; f64 mode also writes the f32 filter coordinates (x-ox, y-oy)
-void launch_gather_points(const void* xy_in, uint32_t* ids, uint64_t n, hdb_dtype dt, void* xy_s, float4* xp,
-                          double ox, double oy, unsigned int* counters, uint32_t n_counters, cudaStream_t s);
-void launch_cell_flags(const void* keys_sorted, int key_bytes, uint64_t n, uint32_t* flags, cudaStream_t s);
-void launch_cell_scatter(const void* keys_sorted, int key_bytes, const uint32_t* flags, const uint32_t* pos,
-                         uint64_t n, uint64_t* ckey, uint32_t* cstart, cudaStream_t s);
+// a2 + a3 + gather: the points sorted by cell key (stable LSD radix sort of (key, id, xy)
+// records, keys computed by the first pass from the input points): keys_out[n] sorted keys,
+// ids_out[n + 2] A (padded), xy_s[n + 2] sorted points (padded), xp the f32 filter copy
+// (padded), counters zeroed.  temp: point_sort_temp_bytes(n, dt, key_bytes, bits)
+size_t point_sort_temp_bytes(uint64_t n, hdb_dtype dt, int key_bytes, int bits);
+void sort_points(const void* xy_in, uint64_t n, hdb_dtype dt, double xmin, double ymin, double inv_w, uint32_t nx,
+                 uint32_t ny, int key_bytes, int bits, void* keys_out, uint32_t* ids_out, void* xy_s, float4* xp,
+                 double ox, double oy, unsigned int* counters, uint32_t n_counters, void* temp, cudaStream_t s);
 // cnext: optional dense lookup (first non-empty cell with key >= h, h in [0, nx*ny]); null = binary search
 void launch_cell_spans(const uint64_t* ckey, const uint32_t* cstart, uint64_t nne, uint32_t nx, uint32_t ny,
                        uint32_t k, uint2* cspan, uint32_t* gcount, const uint32_t* cnext, cudaStream_t s);
@@ -161,6 +160,11 @@ struct ScanEpochScope {
 };
 void scan_u32_to_u32(const uint32_t* in, uint32_t* out, uint64_t n, void* temp, cudaStream_t s);
 void scan_u32_to_u64(const uint32_t* in, uint64_t* out, uint64_t n, void* temp, cudaStream_t s);
+// a4: run-length encoding of n sorted cell keys (one look-back scan of the run-start flags):
+// ckey[c], cstart[c] for every non-empty cell c, cstart[nne] = n, *nne_out = nne.
+// ckey / cstart must hold n / n + 1 entries (nne <= n is known only after the call)
+void cell_rle(const void* keys_sorted, int key_bytes, uint64_t n, uint64_t* ckey, uint32_t* cstart, uint32_t* nne_out,
+              void* temp, cudaStream_t s);
 
 // search (kernels_search.cu)
 // Sampled count (a5): |N_eps| of sorted positions j*stride, j < n_sample -> samp_cnt, sum.

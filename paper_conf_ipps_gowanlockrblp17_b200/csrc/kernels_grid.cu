@@ -98,7 +98,26 @@ __global__ void __launch_bounds__(256) k_bbox(const typename V2<T>::type* __rest
         ymx = fmax(ymx, __shfl_xor_sync(FULL, ymx, o));
         nb += __shfl_xor_sync(FULL, nb, o);
     }
-    if ((threadIdx.x & 31) == 0) {
+    // block reduction, then one set of atomics per block (per-warp atomics on the same four
+    // words serialised at the L2: 31 us of a 1.86M-point bbox)
+    __shared__ double red[5][8];
+    const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    if (lane == 0) {
+        red[0][w] = xmn;
+        red[1][w] = ymn;
+        red[2][w] = xmx;
+        red[3][w] = ymx;
+        red[4][w] = (double)nb;
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        for (int i = 1; i < (int)(blockDim.x >> 5); ++i) {
+            xmn = fmin(xmn, red[0][i]);
+            ymn = fmin(ymn, red[1][i]);
+            xmx = fmax(xmx, red[2][i]);
+            ymx = fmax(ymx, red[3][i]);
+            nb += (unsigned)red[4][i];
+        }
         if (xmn <= xmx) {
             atomicMin(&bb[0], ord_encode(xmn));
             atomicMin(&bb[1], ord_encode(ymn));
@@ -106,25 +125,6 @@ __global__ void __launch_bounds__(256) k_bbox(const typename V2<T>::type* __rest
             atomicMax(&bb[3], ord_encode(ymx));
         }
         if (nb) atomicAdd(bad, nb);
-    }
-}
-
-// a2: cell keys.  FP64 cell arithmetic with explicitly rounded ops (no FMA).
-// Keys are 32-bit when the grid has <= 2^32 cells (halves the sort traffic).
-template <typename T, typename K>
-__global__ void __launch_bounds__(256) k_keys(const typename V2<T>::type* __restrict__ xy, uint64_t n,
-                                              double xmin, double ymin, double inv_w, uint32_t nx,
-                                              uint32_t ny, K* __restrict__ keys,
-                                              uint32_t* __restrict__ vals) {
-    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n;
-         i += (uint64_t)gridDim.x * blockDim.x) {
-        auto p = xy[i];
-        double tx = floor(__dmul_rn(__dsub_rn((double)p.x, xmin), inv_w));
-        double ty = floor(__dmul_rn(__dsub_rn((double)p.y, ymin), inv_w));
-        uint64_t cx = (uint64_t)fmin(fmax(tx, 0.0), (double)(nx - 1));
-        uint64_t cy = (uint64_t)fmin(fmax(ty, 0.0), (double)(ny - 1));
-        keys[i] = (K)(cy * nx + cx);
-        vals[i] = (uint32_t)i;
     }
 }
 
@@ -148,22 +148,22 @@ template <typename K>
 __global__ void __launch_bounds__(RS_THREADS) k_radix_hist(const K* __restrict__ keys, uint64_t n, int shift,
                                                            uint32_t* __restrict__ hist, uint32_t nblocks) {
     constexpr int ITEMS = RsCfg<K>::ITEMS, TILE = RsCfg<K>::TILE;
-    __shared__ uint32_t h[RS_BINS];
-    const int tid = threadIdx.x;
-    const int lane = tid & 31;
-    h[tid] = 0;
+    __shared__ uint32_t h[RS_WARPS][RS_BINS];   // warp-private counters (no match_any)
+    const int tid = threadIdx.x, w = tid >> 5;
+#pragma unroll
+    for (int i = 0; i < RS_WARPS; ++i) h[i][tid] = 0;
     __syncthreads();
     const uint64_t base = (uint64_t)blockIdx.x * TILE;
 #pragma unroll 4
     for (int r = 0; r < ITEMS; ++r) {
         uint64_t idx = base + (uint64_t)r * RS_THREADS + tid;
-        bool valid = idx < n;
-        uint32_t d = valid ? (uint32_t)((keys[idx] >> shift) & (RS_BINS - 1)) : (0x100u + lane);
-        unsigned peers = __match_any_sync(FULL, d);
-        if (valid && lane == __ffs(peers) - 1) atomicAdd(&h[d], __popc(peers));
+        if (idx < n) atomicAdd(&h[w][(uint32_t)((keys[idx] >> shift) & (RS_BINS - 1))], 1u);
     }
     __syncthreads();
-    hist[(uint64_t)tid * nblocks + blockIdx.x] = h[tid];
+    uint32_t t = 0;
+#pragma unroll
+    for (int i = 0; i < RS_WARPS; ++i) t += h[i][tid];
+    hist[(uint64_t)tid * nblocks + blockIdx.x] = t;
 }
 
 template <typename K>
@@ -249,66 +249,195 @@ __global__ void __launch_bounds__(RS_THREADS) k_radix_scatter(const K* __restric
     }
 }
 
-template <typename T>
-__global__ void __launch_bounds__(256) k_gather(const typename V2<T>::type* __restrict__ in,
-                                                const uint32_t* __restrict__ ids, uint64_t n,
-                                                typename V2<T>::type* __restrict__ out, float4* __restrict__ xp,
-                                                double ox, double oy, uint32_t* __restrict__ ids_pad, unsigned int* __restrict__ counters,
-                                                uint32_t n_counters) {
-    // xp: paired-SoA f32 copy {x_2k, x_2k+1, y_2k, y_2k+1} -- f64 input: filter
-    // coordinates fl32(fl64(x - ox)); f32 input: the exact coordinates
-    float* xpf = (float*)xp;
-    if (blockIdx.x == 0 && threadIdx.x == 0) {
-        // padding read by the candidate-pair loads (2 entries past n) and the work
-        // counters -- zeroed here instead of by four memsets
-        out[n] = out[n + 1] = typename V2<T>::type{0, 0};
-        ids_pad[0] = ids_pad[1] = 0;
-        for (uint64_t s = n; s < 2 * (n / 2 + 2); ++s) {
-            const uint64_t k = s >> 1, o = s & 1;
-            xpf[4 * k + o] = 0.f;
-            xpf[4 * k + 2 + o] = 0.f;
+// ---------------------------------------------------------------- point sort (a2 + a3 + gather)
+// The points sorted by cell key with a stable LSD radix sort (8-bit digits)
+// whose passes carry the whole record (key, id, xy): the first pass reads the
+// INPUT points in input order and computes their keys (a2) on the fly (id =
+// input row), the last pass writes the sorted keys, A (sorted pos -> id), the
+// sorted points and their f32 filter copy.  This replaces keys -> (key, id) sort
+// -> gather: the gather's random reads of the input points (1.4 ms at C5's 50M
+// points) are gone, every pass streams coalesced digit runs.  Per pass: a
+// per-tile digit histogram (warp-private shared counters, no match_any), a scan
+// of the (digit, tile) counts, and the scatter (stable warp match_any ranks,
+// staging in shared memory in digit order, coalesced runs).
+constexpr int PS_THREADS = 256;
+constexpr int PS_WARPS = PS_THREADS / 32;
+constexpr int PS_ITEMS = 8;
+constexpr int PS_TILE = PS_THREADS * PS_ITEMS;   // 2048 records per CTA
+
+struct KeyParams {
+    double xmin, ymin, inv_w;
+    uint32_t nx, ny;
+};
+
+// a2: cell key of p -- FP64 cell arithmetic with explicitly rounded ops (no FMA),
+// cx = floor(fl(fl(x - xmin) * fl(1/w))) clamped to [0, nx-1] (reading R9)
+template <typename T, typename K>
+__device__ __forceinline__ K cell_key(const typename V2<T>::type p, const KeyParams& kp) {
+    const double tx = floor(__dmul_rn(__dsub_rn((double)p.x, kp.xmin), kp.inv_w));
+    const double ty = floor(__dmul_rn(__dsub_rn((double)p.y, kp.ymin), kp.inv_w));
+    const uint64_t cx = (uint64_t)fmin(fmax(tx, 0.0), (double)(kp.nx - 1));
+    const uint64_t cy = (uint64_t)fmin(fmax(ty, 0.0), (double)(kp.ny - 1));
+    return (K)(cy * kp.nx + cx);
+}
+
+template <typename T, typename K, bool FROM_POINTS>
+__global__ void __launch_bounds__(PS_THREADS) k_ps_hist(const typename V2<T>::type* __restrict__ xy,
+                                                        const K* __restrict__ keys, KeyParams kp, uint64_t n,
+                                                        int shift, uint32_t* __restrict__ hist, uint32_t nblocks) {
+    __shared__ uint32_t h[PS_WARPS][RS_BINS];
+    const int tid = threadIdx.x, w = tid >> 5;
+#pragma unroll
+    for (int i = 0; i < PS_WARPS; ++i) h[i][tid] = 0;
+    __syncthreads();
+    const uint64_t base = (uint64_t)blockIdx.x * PS_TILE;
+#pragma unroll
+    for (int r = 0; r < PS_ITEMS; ++r) {
+        const uint64_t idx = base + (uint64_t)r * PS_THREADS + tid;
+        if (idx < n) {
+            const K k = FROM_POINTS ? cell_key<T, K>(xy[idx], kp) : keys[idx];
+            atomicAdd(&h[w][(uint32_t)((k >> shift) & (RS_BINS - 1))], 1u);
         }
-        for (uint32_t c = 0; c < n_counters; ++c) counters[c] = 0;
     }
-    for (uint64_t s = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; s < n;
-         s += (uint64_t)gridDim.x * blockDim.x) {
-        auto p = in[ids[s]];
-        out[s] = p;
-        float fx, fy;
-        if (sizeof(p.x) == 8) {
-            fx = (float)__dsub_rn((double)p.x, ox);
-            fy = (float)__dsub_rn((double)p.y, oy);
+    __syncthreads();
+    uint32_t t = 0;
+#pragma unroll
+    for (int i = 0; i < PS_WARPS; ++i) t += h[i][tid];
+    hist[(uint64_t)tid * nblocks + blockIdx.x] = t;
+}
+
+template <typename T, typename K>
+constexpr size_t ps_smem_bytes() {
+    return (size_t)PS_TILE * (sizeof(typename V2<T>::type) + sizeof(K) + 4) + (PS_WARPS + 2) * RS_BINS * 4;
+}
+
+template <typename T, typename K, bool FIRST, bool LAST>
+__global__ void __launch_bounds__(PS_THREADS) k_ps_scatter(const typename V2<T>::type* __restrict__ xyin,
+                                                           const K* __restrict__ kin, const uint32_t* __restrict__ vin,
+                                                           KeyParams kp, K* __restrict__ kout,
+                                                           uint32_t* __restrict__ vout,
+                                                           typename V2<T>::type* __restrict__ xyout,
+                                                           float4* __restrict__ xp, double ox, double oy, uint64_t n,
+                                                           int shift, const uint32_t* __restrict__ hscan,
+                                                           uint32_t nblocks, unsigned int* __restrict__ counters,
+                                                           uint32_t n_counters) {
+    using P2 = typename V2<T>::type;
+    extern __shared__ __align__(16) unsigned char ps_smem[];
+    P2* sxy = (P2*)ps_smem;
+    K* skey = (K*)(sxy + PS_TILE);
+    uint32_t* sval = (uint32_t*)(skey + PS_TILE);
+    uint32_t(*wcnt)[RS_BINS] = (uint32_t(*)[RS_BINS])(sval + PS_TILE);
+    uint32_t* gbase = (uint32_t*)(wcnt + PS_WARPS);   // global start of each digit's run of this tile
+    uint32_t* dstart = gbase + RS_BINS;                // tile-local start of each digit
+    __shared__ uint32_t wsum[PS_WARPS];
+    const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
+#pragma unroll
+    for (int i = 0; i < PS_WARPS; ++i) wcnt[i][tid] = 0;
+    gbase[tid] = hscan[(uint64_t)tid * nblocks + blockIdx.x];
+    if (LAST && blockIdx.x == 0) {
+        // padding read by the candidate-pair loads (2 entries past n) and the work counters
+        if (tid < 2) {
+            xyout[n + tid] = P2{0, 0};
+            vout[n + tid] = 0;
+        }
+        float* xpf = (float*)xp;
+        for (uint64_t q = n + tid; q < 2 * (n / 2 + 2); q += PS_THREADS) {
+            xpf[4 * (q >> 1) + (q & 1)] = 0.f;
+            xpf[4 * (q >> 1) + 2 + (q & 1)] = 0.f;
+        }
+        for (uint32_t c = tid; c < n_counters; c += PS_THREADS) counters[c] = 0;
+    }
+    __syncthreads();
+    const uint64_t tbase = (uint64_t)blockIdx.x * PS_TILE;
+    const uint64_t base = tbase + (uint64_t)w * (PS_ITEMS * 32);
+    const unsigned lt = (1u << lane) - 1u;
+    K key[PS_ITEMS];
+    uint32_t val[PS_ITEMS], rank[PS_ITEMS];
+    P2 pt[PS_ITEMS];
+#pragma unroll
+    for (int r = 0; r < PS_ITEMS; ++r) {
+        const uint64_t idx = base + (uint64_t)r * 32 + lane;
+        const bool valid = idx < n;
+        pt[r] = valid ? xyin[idx] : P2{0, 0};
+        if (FIRST) {
+            key[r] = valid ? cell_key<T, K>(pt[r], kp) : (K)0;
+            val[r] = (uint32_t)idx;
         } else {
-            fx = (float)p.x;
-            fy = (float)p.y;
+            key[r] = valid ? kin[idx] : (K)0;
+            val[r] = valid ? vin[idx] : 0u;
         }
-        const uint64_t k = s >> 1, o = s & 1;
-        xpf[4 * k + o] = fx;
-        xpf[4 * k + 2 + o] = fy;
     }
-}
-
-// a4: run boundaries of the sorted keys
-template <typename K>
-__global__ void __launch_bounds__(256) k_cell_flags(const K* __restrict__ keys, uint64_t n,
-                                                    uint32_t* __restrict__ flags) {
-    for (uint64_t s = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; s < n;
-         s += (uint64_t)gridDim.x * blockDim.x)
-        flags[s] = (s == 0 || keys[s] != keys[s - 1]) ? 1u : 0u;
-}
-
-template <typename K>
-__global__ void __launch_bounds__(256) k_cell_scatter(const K* __restrict__ keys,
-                                                      const uint32_t* __restrict__ flags,
-                                                      const uint32_t* __restrict__ pos, uint64_t n,
-                                                      uint64_t* __restrict__ ckey, uint32_t* __restrict__ cstart) {
-    for (uint64_t s = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; s < n;
-         s += (uint64_t)gridDim.x * blockDim.x)
-        if (flags[s]) {
-            ckey[pos[s]] = (uint64_t)keys[s];
-            cstart[pos[s]] = (uint32_t)s;
+#pragma unroll
+    for (int r = 0; r < PS_ITEMS; ++r) {
+        const bool valid = base + (uint64_t)r * 32 + lane < n;
+        const uint32_t d = valid ? (uint32_t)((key[r] >> shift) & (RS_BINS - 1)) : (0x100u + lane);
+        const unsigned peers = __match_any_sync(FULL, d);
+        const uint32_t before = valid ? wcnt[w][d] : 0u;
+        rank[r] = before + __popc(peers & lt);
+        __syncwarp();
+        if (valid && lane == __ffs(peers) - 1) wcnt[w][d] = before + __popc(peers);
+        __syncwarp();
+    }
+    __syncthreads();
+    // per digit: exclusive prefix over the warps, and the digit's tile total
+    uint32_t tot = 0;
+#pragma unroll
+    for (int i = 0; i < PS_WARPS; ++i) {
+        const uint32_t t = wcnt[i][tid];
+        wcnt[i][tid] = tot;
+        tot += t;
+    }
+    uint32_t incl = tot;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(FULL, incl, o);
+        if (lane >= o) incl += y;
+    }
+    if (lane == 31) wsum[w] = incl;
+    __syncthreads();
+    uint32_t wpre = 0;
+#pragma unroll
+    for (int i = 0; i < PS_WARPS; ++i) wpre += i < w ? wsum[i] : 0u;
+    dstart[tid] = wpre + incl - tot;
+    __syncthreads();
+    // stage in digit order
+#pragma unroll
+    for (int r = 0; r < PS_ITEMS; ++r) {
+        if (base + (uint64_t)r * 32 + lane < n) {
+            const uint32_t d = (uint32_t)((key[r] >> shift) & (RS_BINS - 1));
+            const uint32_t lp = dstart[d] + wcnt[w][d] + rank[r];
+            skey[lp] = key[r];
+            sval[lp] = val[r];
+            sxy[lp] = pt[r];
         }
-    if (blockIdx.x == 0 && threadIdx.x == 0) cstart[pos[n]] = (uint32_t)n;
+    }
+    __syncthreads();
+    // write each digit's run contiguously
+    const uint32_t cnt = (uint32_t)min((uint64_t)PS_TILE, n - tbase);
+    float* xpf = (float*)xp;
+    for (uint32_t i = tid; i < cnt; i += PS_THREADS) {
+        const K k = skey[i];
+        const uint32_t d = (uint32_t)((k >> shift) & (RS_BINS - 1));
+        const uint64_t pos = gbase[d] + (i - dstart[d]);
+        const P2 p = sxy[i];
+        kout[pos] = k;
+        vout[pos] = sval[i];
+        xyout[pos] = p;
+        if (LAST) {
+            // xp: paired-SoA f32 copy {x_2k, x_2k+1, y_2k, y_2k+1} -- f64 input: filter
+            // coordinates fl32(fl64(x - ox)); f32 input: the exact coordinates
+            float fx, fy;
+            if (sizeof(p.x) == 8) {
+                fx = (float)__dsub_rn((double)p.x, ox);
+                fy = (float)__dsub_rn((double)p.y, oy);
+            } else {
+                fx = (float)p.x;
+                fy = (float)p.y;
+            }
+            xpf[4 * (pos >> 1) + (pos & 1)] = fx;
+            xpf[4 * (pos >> 1) + 2 + (pos & 1)] = fy;
+        }
+    }
 }
 
 // first index i in [lo, hi) with ckey[i] >= k (hi if none)
@@ -615,25 +744,9 @@ void launch_bbox(const void* xy, uint64_t n, hdb_dtype dt, unsigned long long* b
                  cudaStream_t s) {
     if (n == 0) return;
     if (dt == HDB_F64)
-        k_bbox<double><<<grid_for(n, 256, 148 * 8), 256, 0, s>>>((const double2*)xy, n, bb, bad);
+        k_bbox<double><<<grid_for(n, 256, 148 * 4), 256, 0, s>>>((const double2*)xy, n, bb, bad);
     else
-        k_bbox<float><<<grid_for(n, 256, 148 * 8), 256, 0, s>>>((const float2*)xy, n, bb, bad);
-    ++g_kernel_launches;
-}
-
-void launch_keys(const void* xy, uint64_t n, hdb_dtype dt, double xmin, double ymin, double inv_w,
-                 uint32_t nx, uint32_t ny, void* keys, int key_bytes, uint32_t* vals, cudaStream_t s) {
-    if (n == 0) return;
-#define HDB_KEYS(T, K) \
-    k_keys<T, K><<<grid_for(n), 256, 0, s>>>((const V2<T>::type*)xy, n, xmin, ymin, inv_w, nx, ny, (K*)keys, vals)
-    if (dt == HDB_F64) {
-        if (key_bytes == 4) HDB_KEYS(double, uint32_t);
-        else HDB_KEYS(double, uint64_t);
-    } else {
-        if (key_bytes == 4) HDB_KEYS(float, uint32_t);
-        else HDB_KEYS(float, uint64_t);
-    }
-#undef HDB_KEYS
+        k_bbox<float><<<grid_for(n, 256, 148 * 4), 256, 0, s>>>((const float2*)xy, n, bb, bad);
     ++g_kernel_launches;
 }
 
@@ -677,34 +790,109 @@ int radix_sort_pairs(void* k0, uint32_t* v0, void* k1, uint32_t* v1, int key_byt
     return radix_sort_impl<uint64_t>((uint64_t*)k0, v0, (uint64_t*)k1, v1, n, bits, temp, s);
 }
 
-void launch_gather_points(const void* xy_in, uint32_t* ids, uint64_t n, hdb_dtype dt, void* xy_s, float4* xp,
-                          double ox, double oy, unsigned int* counters, uint32_t n_counters, cudaStream_t s) {
-    const unsigned blocks = n ? grid_for(n) : 1;
+// ---- point sort (a2 + a3 + gather in one record sort)
+template <typename T, typename K>
+struct PointSort {
+    using P2 = typename V2<T>::type;
+    static constexpr size_t rec = sizeof(P2) + sizeof(K) + 4;
+    template <bool F, bool L>
+    static void scatter(const P2* xyin, const K* kin, const uint32_t* vin, const KeyParams& kp, K* kout,
+                        uint32_t* vout, P2* xyout, float4* xp, double ox, double oy, uint64_t n, int shift,
+                        const uint32_t* hscan, uint32_t nb, unsigned int* counters, uint32_t nc, cudaStream_t s) {
+        static bool attr = [] {
+            cudaFuncSetAttribute(k_ps_scatter<T, K, F, L>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                 (int)ps_smem_bytes<T, K>());
+            return true;
+        }();
+        (void)attr;
+        k_ps_scatter<T, K, F, L><<<nb, PS_THREADS, ps_smem_bytes<T, K>(), s>>>(
+            xyin, kin, vin, kp, kout, vout, xyout, xp, ox, oy, n, shift, hscan, nb, counters, nc);
+        ++g_kernel_launches;
+    }
+    static void run(const void* xy_in, uint64_t n, const KeyParams& kp, int bits, void* keys_out, uint32_t* ids_out,
+                    void* xy_s, float4* xp, double ox, double oy, unsigned int* counters, uint32_t nc, void* temp,
+                    cudaStream_t s) {
+        const uint32_t nb = (uint32_t)((n + PS_TILE - 1) / PS_TILE);
+        const int passes = std::max(1, (bits + RS_BITS - 1) / RS_BITS);
+        const uint64_t m = (uint64_t)nb * RS_BINS;
+        unsigned char* t = (unsigned char*)temp;
+        auto carve = [&](size_t bytes) {
+            void* p = t;
+            t += (bytes + 255) & ~(size_t)255;
+            return p;
+        };
+        uint32_t* hist = (uint32_t*)carve(4 * (m + 1));
+        uint32_t* hscan = (uint32_t*)carve(4 * (m + 1));
+        void* stemp = carve(scan_temp_bytes(m));
+        K* kb[2];
+        uint32_t* vb[2];
+        P2* xb[2];
+        for (int i = 0; i < (passes > 2 ? 2 : passes - 1); ++i) {
+            kb[i] = (K*)carve(sizeof(K) * n);
+            vb[i] = (uint32_t*)carve(4 * n);
+            xb[i] = (P2*)carve(sizeof(P2) * n);
+        }
+        const P2* xin = (const P2*)xy_in;
+        for (int p = 0; p < passes; ++p) {
+            const int shift = p * RS_BITS;
+            const bool first = p == 0, last = p == passes - 1;
+            const K* ki = first ? nullptr : kb[(p - 1) & 1];
+            const uint32_t* vi = first ? nullptr : vb[(p - 1) & 1];
+            const P2* xi = first ? xin : xb[(p - 1) & 1];
+            K* ko = last ? (K*)keys_out : kb[p & 1];
+            uint32_t* vo = last ? ids_out : vb[p & 1];
+            P2* xo = last ? (P2*)xy_s : xb[p & 1];
+            if (first)
+                k_ps_hist<T, K, true><<<nb, PS_THREADS, 0, s>>>(xin, nullptr, kp, n, shift, hist, nb);
+            else
+                k_ps_hist<T, K, false><<<nb, PS_THREADS, 0, s>>>(nullptr, ki, kp, n, shift, hist, nb);
+            ++g_kernel_launches;
+            scan_u32_to_u32(hist, hscan, m, stemp, s);
+            if (first && last)
+                scatter<true, true>(xi, ki, vi, kp, ko, vo, xo, xp, ox, oy, n, shift, hscan, nb, counters, nc, s);
+            else if (first)
+                scatter<true, false>(xi, ki, vi, kp, ko, vo, xo, xp, ox, oy, n, shift, hscan, nb, counters, nc, s);
+            else if (last)
+                scatter<false, true>(xi, ki, vi, kp, ko, vo, xo, xp, ox, oy, n, shift, hscan, nb, counters, nc, s);
+            else
+                scatter<false, false>(xi, ki, vi, kp, ko, vo, xo, xp, ox, oy, n, shift, hscan, nb, counters, nc, s);
+        }
+    }
+    static size_t temp_bytes(uint64_t n, int bits) {
+        const uint64_t nb = (n + PS_TILE - 1) / PS_TILE, m = nb * RS_BINS;
+        const int passes = std::max(1, (bits + RS_BITS - 1) / RS_BITS);
+        const int bufs = passes > 2 ? 2 : passes - 1;
+        return 2 * (4 * (m + 1) + 256) + scan_temp_bytes(m) + 256 + bufs * (n * rec + 3 * 256);
+    }
+};
+
+size_t point_sort_temp_bytes(uint64_t n, hdb_dtype dt, int key_bytes, int bits) {
     if (dt == HDB_F64)
-        k_gather<double><<<blocks, 256, 0, s>>>((const double2*)xy_in, ids, n, (double2*)xy_s, xp, ox, oy, ids + n,
-                                                counters, n_counters);
-    else
-        k_gather<float><<<blocks, 256, 0, s>>>((const float2*)xy_in, ids, n, (float2*)xy_s, xp, 0, 0, ids + n,
-                                               counters, n_counters);
-    ++g_kernel_launches;
+        return key_bytes == 4 ? PointSort<double, uint32_t>::temp_bytes(n, bits)
+                              : PointSort<double, uint64_t>::temp_bytes(n, bits);
+    return key_bytes == 4 ? PointSort<float, uint32_t>::temp_bytes(n, bits) : PointSort<float, uint64_t>::temp_bytes(n, bits);
 }
 
-void launch_cell_flags(const void* keys_sorted, int key_bytes, uint64_t n, uint32_t* flags, cudaStream_t s) {
+void sort_points(const void* xy_in, uint64_t n, hdb_dtype dt, double xmin, double ymin, double inv_w, uint32_t nx,
+                 uint32_t ny, int key_bytes, int bits, void* keys_out, uint32_t* ids_out, void* xy_s, float4* xp,
+                 double ox, double oy, unsigned int* counters, uint32_t n_counters, void* temp, cudaStream_t s) {
     if (n == 0) return;
-    if (key_bytes == 4)
-        k_cell_flags<uint32_t><<<grid_for(n), 256, 0, s>>>((const uint32_t*)keys_sorted, n, flags);
-    else
-        k_cell_flags<uint64_t><<<grid_for(n), 256, 0, s>>>((const uint64_t*)keys_sorted, n, flags);
-    ++g_kernel_launches;
-}
-
-void launch_cell_scatter(const void* keys_sorted, int key_bytes, const uint32_t* flags, const uint32_t* pos,
-                         uint64_t n, uint64_t* ckey, uint32_t* cstart, cudaStream_t s) {
-    if (key_bytes == 4)
-        k_cell_scatter<uint32_t><<<grid_for(n), 256, 0, s>>>((const uint32_t*)keys_sorted, flags, pos, n, ckey, cstart);
-    else
-        k_cell_scatter<uint64_t><<<grid_for(n), 256, 0, s>>>((const uint64_t*)keys_sorted, flags, pos, n, ckey, cstart);
-    ++g_kernel_launches;
+    const KeyParams kp{xmin, ymin, inv_w, nx, ny};
+    if (dt == HDB_F64) {
+        if (key_bytes == 4)
+            PointSort<double, uint32_t>::run(xy_in, n, kp, bits, keys_out, ids_out, xy_s, xp, ox, oy, counters,
+                                             n_counters, temp, s);
+        else
+            PointSort<double, uint64_t>::run(xy_in, n, kp, bits, keys_out, ids_out, xy_s, xp, ox, oy, counters,
+                                             n_counters, temp, s);
+    } else {
+        if (key_bytes == 4)
+            PointSort<float, uint32_t>::run(xy_in, n, kp, bits, keys_out, ids_out, xy_s, xp, 0, 0, counters,
+                                            n_counters, temp, s);
+        else
+            PointSort<float, uint64_t>::run(xy_in, n, kp, bits, keys_out, ids_out, xy_s, xp, 0, 0, counters,
+                                            n_counters, temp, s);
+    }
 }
 
 void launch_cell_spans(const uint64_t* ckey, const uint32_t* cstart, uint64_t nne, uint32_t nx, uint32_t ny,

@@ -48,9 +48,19 @@ __device__ __forceinline__ uint64_t peek(const unsigned long long* w) {
     return v;
 }
 
+// Op: Tout load(idx) (idx < n) -- the item; void store(idx, excl) -- its exclusive prefix;
+// void total(t) -- the sum of all items (written by the last tile)
 template <typename Tin, typename Tout>
-__global__ void __launch_bounds__(SC_THREADS) k_scan_lookback(const Tin* __restrict__ in, Tout* __restrict__ out,
-                                                              uint64_t n, unsigned long long* __restrict__ tiles,
+struct PlainScan {
+    const Tin* __restrict__ in;
+    Tout* __restrict__ out;
+    __device__ __forceinline__ Tout load(uint64_t i) const { return (Tout)in[i]; }
+    __device__ __forceinline__ void store(uint64_t i, Tout e) const { out[i] = e; }
+    __device__ __forceinline__ void total(uint64_t n, Tout t) const { out[n] = t; }
+};
+
+template <typename Tout, typename Op>
+__global__ void __launch_bounds__(SC_THREADS) k_scan_lookback(Op op, uint64_t n, unsigned long long* __restrict__ tiles,
                                                               uint64_t ep, unsigned long long* __restrict__ ctr,
                                                               uint64_t ctr_base) {
     __shared__ Tout buf[SC_TILE];
@@ -65,7 +75,7 @@ __global__ void __launch_bounds__(SC_THREADS) k_scan_lookback(const Tin* __restr
 #pragma unroll
     for (int i = 0; i < SC_ITEMS; ++i) {
         uint64_t idx = base + (uint64_t)i * SC_THREADS + tid;
-        buf[i * SC_THREADS + tid] = idx < n ? (Tout)in[idx] : (Tout)0;
+        buf[i * SC_THREADS + tid] = idx < n ? op.load(idx) : (Tout)0;
     }
     __syncthreads();
     Tout v[SC_ITEMS];
@@ -126,17 +136,13 @@ __global__ void __launch_bounds__(SC_THREADS) k_scan_lookback(const Tin* __restr
 #pragma unroll
     for (int i = 0; i < SC_ITEMS; ++i) {
         uint64_t idx = base + (uint64_t)i * SC_THREADS + tid;
-        if (idx < n) out[idx] = buf[i * SC_THREADS + tid];
+        if (idx < n) op.store(idx, buf[i * SC_THREADS + tid]);
     }
-    if (tid == 0 && base + SC_TILE >= n) out[n] = s_excl + tot;   // last tile writes the total
+    if (tid == 0 && base + SC_TILE >= n) op.total(n, s_excl + tot);   // last tile writes the total
 }
 
-template <typename Tin, typename Tout>
-void scan_impl(const Tin* in, Tout* out, uint64_t n, void* temp, cudaStream_t s) {
-    if (n == 0) {
-        cudaMemsetAsync(out, 0, sizeof(Tout), s);
-        return;
-    }
+template <typename Tout, typename Op>
+void scan_impl(const Op& op, uint64_t n, void* temp, cudaStream_t s) {
     const uint64_t nb = (n + SC_TILE - 1) / SC_TILE;
     unsigned long long* tiles = nullptr;
     unsigned long long* ctr = nullptr;   // tile-id counter (null: one tile, id 0)
@@ -160,7 +166,7 @@ void scan_impl(const Tin* in, Tout* out, uint64_t n, void* temp, cudaStream_t s)
             cudaMemsetAsync(tiles, 0, (nb + 1) * sizeof(unsigned long long), s);
         }
     }
-    k_scan_lookback<Tin, Tout><<<(unsigned)nb, SC_THREADS, 0, s>>>(in, out, n, tiles, ep, ctr, ctr_base);
+    k_scan_lookback<Tout, Op><<<(unsigned)nb, SC_THREADS, 0, s>>>(op, n, tiles, ep, ctr, ctr_base);
     ++g_kernel_launches;
 }
 
@@ -173,11 +179,58 @@ size_t scan_temp_bytes(uint64_t n) {
 }
 
 void scan_u32_to_u32(const uint32_t* in, uint32_t* out, uint64_t n, void* temp, cudaStream_t s) {
-    scan_impl<uint32_t, uint32_t>(in, out, n, temp, s);
+    if (n == 0) {
+        cudaMemsetAsync(out, 0, sizeof(uint32_t), s);
+        return;
+    }
+    scan_impl<uint32_t>(PlainScan<uint32_t, uint32_t>{in, out}, n, temp, s);
 }
 
 void scan_u32_to_u64(const uint32_t* in, uint64_t* out, uint64_t n, void* temp, cudaStream_t s) {
-    scan_impl<uint32_t, uint64_t>(in, out, n, temp, s);
+    if (n == 0) {
+        cudaMemsetAsync(out, 0, sizeof(uint64_t), s);
+        return;
+    }
+    scan_impl<uint64_t>(PlainScan<uint32_t, uint64_t>{in, out}, n, temp, s);
+}
+
+// a4 in one pass: run-length encoding of the sorted keys -- the scan of the run-start
+// flags (key[s] != key[s-1]) gives each run its index c; run starts write ckey[c] = key,
+// cstart[c] = s; the total (the non-empty cell count) goes to cstart's terminator slot
+// *nne_out and cstart[nne] = n is written by the last tile.  Replaces flags -> scan ->
+// scatter (three passes over n-sized arrays).
+template <typename K>
+struct RleScan {
+    const K* __restrict__ keys;
+    uint64_t* __restrict__ ckey;
+    uint32_t* __restrict__ cstart;
+    uint32_t* __restrict__ nne_out;
+    __device__ __forceinline__ uint32_t load(uint64_t i) const {
+        return (i == 0 || keys[i] != keys[i - 1]) ? 1u : 0u;
+    }
+    __device__ __forceinline__ void store(uint64_t i, uint32_t e) const {
+        if (i == 0 || keys[i] != keys[i - 1]) {
+            ckey[e] = (uint64_t)keys[i];
+            cstart[e] = (uint32_t)i;
+        }
+    }
+    __device__ __forceinline__ void total(uint64_t n, uint32_t t) const {
+        cstart[t] = (uint32_t)n;
+        *nne_out = t;
+    }
+};
+
+void cell_rle(const void* keys_sorted, int key_bytes, uint64_t n, uint64_t* ckey, uint32_t* cstart, uint32_t* nne_out,
+              void* temp, cudaStream_t s) {
+    if (n == 0) {
+        cudaMemsetAsync(cstart, 0, sizeof(uint32_t), s);
+        cudaMemsetAsync(nne_out, 0, sizeof(uint32_t), s);
+        return;
+    }
+    if (key_bytes == 4)
+        scan_impl<uint32_t>(RleScan<uint32_t>{(const uint32_t*)keys_sorted, ckey, cstart, nne_out}, n, temp, s);
+    else
+        scan_impl<uint32_t>(RleScan<uint64_t>{(const uint64_t*)keys_sorted, ckey, cstart, nne_out}, n, temp, s);
 }
 
 }  // namespace hdb
