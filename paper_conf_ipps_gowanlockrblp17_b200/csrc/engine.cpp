@@ -779,12 +779,12 @@ bool single_pass_table(hdb_ctx* ctx, const DevGrid& g, hdb_table* t, hdb_stats& 
         return false;
     }
     masks.s = nb.s = s;
-    DBuf beg(8 * n, s, dc.big_pool), cnt_id(4 * n, s, dc.big_pool), cnt(4 * n, s), scratch(32, s);
+    DBuf beg(8 * n, s, dc.big_pool), cnt_id(4 * n, s, dc.big_pool), scratch(32, s);
     HDB_CUDA(cudaMemsetAsync(scratch.p, 0, 32, s));
     unsigned long long* sc = scratch.as<unsigned long long>();
     Event e0, e1;
     HDB_CUDA(cudaEventRecord(e0.e, s));
-    launch_fused(g, cnt.as<uint32_t>(), sc, masks.as<uint2>(), sc + 1, cap, nb.as<uint32_t>(), beg.as<uint64_t>(),
+    launch_fused(g, nullptr, sc, masks.as<uint2>(), sc + 1, cap, nb.as<uint32_t>(), beg.as<uint64_t>(),
                  cnt_id.as<uint32_t>(), (unsigned int*)(sc + 2), s);
     HDB_LAUNCH_CHECK();
     HDB_CUDA(cudaEventRecord(e1.e, s));

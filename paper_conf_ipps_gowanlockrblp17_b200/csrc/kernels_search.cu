@@ -212,7 +212,7 @@ constexpr int kWinPad = kWin + 1;   // padded smem rows: 72-B stride, conflict-f
 // barrier and shared load per window), stores them to the mask table (gmask
 // non-null) and the window buffer is cleared for the next window.
 __device__ __forceinline__ void flush_window(uint2 (*swin)[kWinPad], uint2* gmask, uint32_t v, uint32_t nq,
-                                             uint32_t& my, int lane) {
+                                             uint32_t& my, int lane, bool clear = true) {
     __syncwarp();
     if ((uint32_t)lane < nq) {
         uint2 r[kWin];
@@ -229,6 +229,7 @@ __device__ __forceinline__ void flush_window(uint2 (*swin)[kWinPad], uint2* gmas
         }
     }
     __syncwarp();
+    if (!clear) return;   // the caller emits straight from swin (single-window group)
 #pragma unroll
     for (int kk = 0; kk < kWin; ++kk) swin[lane][kk] = make_uint2(0, 0);   // next window starts empty
     __syncwarp();
@@ -271,19 +272,46 @@ __device__ __forceinline__ uint32_t load_vspans(const SArgs& a, uint32_t c, VSpa
     return total;
 }
 
-// candidate pair of virtual pair vp for this lane; r advances monotonically
-// across a group's chunks.  Returns s0 (= 2p) and the two validity flags.
-__device__ __forceinline__ uint32_t vpair(const VSpan* vs, uint32_t nspan, uint32_t vp, uint32_t& r, bool& v0,
-                                          bool& v1) {
-    while (r < nspan && vp >= vs[r + 1].vstart) ++r;
-    if (r >= nspan) {
-        v0 = v1 = false;
-        return 0;
+// Per-lane cursor over the virtual pair sequence: the lane's current span is
+// cached in registers and only advanced when vp passes its end (vp grows by 32
+// per chunk), so a chunk costs a compare and a few integer ops instead of a
+// search over the span table (the search was ~15% of k_fused's instructions).
+struct VCursor {
+    uint32_t r;       // current span (~0 before the first)
+    uint32_t next;    // first virtual pair after span r
+    uint32_t delta;   // pbase - vstart of span r: s0 = 2 (vp + delta)
+    uint32_t lo, hi;  // [lo, hi) of span r (lo = ~0, hi = 0 past the last span)
+};
+__device__ __forceinline__ void vc_init(VCursor& c) {
+    c.r = ~0u;
+    c.next = 0;
+    c.delta = 0;
+    c.lo = ~0u;
+    c.hi = 0;
+}
+// candidate pair (s0, s0 + 1) of virtual pair vp (non-decreasing across calls) and
+// its two validity flags.  Inside span r the pair index runs from lo/2 to (hi-1)/2,
+// so s0 < hi and s0 + 1 >= lo always hold: v0 = s0 >= lo, v1 = s0 + 1 < hi.
+__device__ __forceinline__ uint32_t vc_pair(VCursor& c, const VSpan* vs, uint32_t nspan, uint32_t vp, bool& v0,
+                                            bool& v1) {
+    while (vp >= c.next) {
+        ++c.r;
+        if (c.r >= nspan) {
+            c.next = ~0u;
+            c.delta = 0;
+            c.lo = ~0u;
+            c.hi = 0;
+            break;
+        }
+        const VSpan e = vs[c.r];
+        c.next = vs[c.r + 1].vstart;
+        c.delta = e.pbase - e.vstart;
+        c.lo = e.lo;
+        c.hi = e.hi;
     }
-    const VSpan e = vs[r];
-    const uint32_t s0 = 2 * (e.pbase + (vp - e.vstart));
-    v0 = s0 >= e.lo && s0 < e.hi;
-    v1 = s0 + 1 >= e.lo && s0 + 1 < e.hi;
+    const uint32_t s0 = 2 * (vp + c.delta);
+    v0 = s0 >= c.lo;
+    v1 = s0 + 1 < c.hi;
     return s0;
 }
 
@@ -304,11 +332,14 @@ constexpr double kFarD = 1e300;
 // Count one query group (queries qs .. qs+nq-1 of non-empty cell c): hit masks
 // to gmask (windowed layout; null = do not store), tests accumulated per lane;
 // returns lane i's |N_eps(query i)| (0 for lanes >= nq).  With masks, swin
-// must be all zero on entry and is left all zero (flush_window clears it).
+// must be all zero on entry and is left all zero (flush_window clears it) --
+// except with keep_single when the group has a single window (*nch_out <= kWin):
+// then its masks stay in swin (and are not stored to gmask) for the caller.
 template <int MODE>
 __device__ __forceinline__ uint32_t count_group(const SArgs& a, uint32_t qs, uint32_t c, uint32_t nq,
                                                 uint2 (*swin)[kWinPad], VSpan* vsp, ulonglong2* sq, double2* sqd,
-                                                uint2* gmask, unsigned long long& tests, int lane) {
+                                                uint2* gmask, unsigned long long& tests, int lane,
+                                                bool keep_single = false, uint32_t* nch_out = nullptr) {
     const ulonglong2* __restrict__ xp = (const ulonglong2*)a.xp;
     const u64x NE2 = pack2(-a.e2f, -a.e2f);
     const u64x NB2 = pack2(a.nb2_l, a.nb2_l);
@@ -332,18 +363,22 @@ __device__ __forceinline__ uint32_t count_group(const SArgs& a, uint32_t qs, uin
     uint32_t my = 0;
     const uint32_t npairs = load_vspans(a, c, vsp, lane);
     const uint32_t nch = (npairs + 31) / 32;
+    if (nch_out) *nch_out = nch;
+    const bool keep = keep_single && nch <= kWin;
+    if (keep) gmask = nullptr;
     if (lane == 0) {   // candidate tests of the group: nq x (candidates of its spans)
         uint32_t ncand = 0;
         for (uint32_t r = 0; r < a.nspan; ++r) ncand += vsp[r].hi - vsp[r].lo;
         tests += (unsigned long long)nq * ncand;
     }
-    uint32_t rs = 0;   // this lane's current span
+    VCursor cur;
+    vc_init(cur);
     uint32_t k = 0;
 #pragma unroll 1
     for (; k < nch; ++k) {
         const uint32_t kk = k % kWin;
         bool v0, v1;
-        const uint32_t s0 = vpair(vsp, a.nspan, 32 * k + lane, rs, v0, v1), s1 = s0 + 1;
+        const uint32_t s0 = vc_pair(cur, vsp, a.nspan, 32 * k + lane, v0, v1), s1 = s0 + 1;
         u64x X, Y;
         double2 d0 = make_double2(kFarD, kFarD), d1 = make_double2(kFarD, kFarD);
         ulonglong2 P = make_ulonglong2(0, 0);
@@ -467,9 +502,9 @@ __device__ __forceinline__ uint32_t count_group(const SArgs& a, uint32_t qs, uin
                 if (lane == 0) swin[i][kk] = make_uint2(m0, m1);
             }
         }
-        if (kk == kWin - 1) flush_window(swin, gmask, k / kWin, nq, my, lane);
+        if (kk == kWin - 1) flush_window(swin, gmask, k / kWin, nq, my, lane, !keep);
     }
-    if ((k % kWin) != 0) flush_window(swin, gmask, k / kWin, nq, my, lane);
+    if ((k % kWin) != 0) flush_window(swin, gmask, k / kWin, nq, my, lane, !keep);
     return my;
 }
 
@@ -679,40 +714,89 @@ __device__ __forceinline__ void cp_async_wait() {
     asm volatile("cp.async.wait_group %0;" ::"n"(N));
 }
 
+// Emission of one window for every query of the group: per query, the window's
+// hits are one contiguous run of its list; per chunk, lane j stores its pair's
+// hits at (run start + popc of the chunk's mask below j).  NCK = the window's
+// chunks (a template: no per-chunk guards in the loop; emit_window picks one).
+template <int NCK>
+__device__ __forceinline__ void emit_rows(const uint2 (&ids)[kWin], const uint4 (*wq)[kWin + 1], uint32_t nq,
+                                          uint32_t* gout, unsigned lt, unsigned lbit) {
+#pragma unroll 1
+    for (uint32_t i = 0; i < nq; ++i) {
+#pragma unroll
+        for (int kk = 0; kk < NCK; ++kk) {
+            const uint4 e = wq[i][kk];   // broadcast
+            stg_if_bit(gout + (e.z + __popc(e.x & lt)), ids[kk].x, e.x, lbit);
+            stg_if_bit(gout + (e.w + __popc(e.y & lt)), ids[kk].y, e.y, lbit);
+        }
+    }
+}
+__device__ __forceinline__ void emit_window(uint32_t nck, const uint2 (&ids)[kWin], const uint4 (*wq)[kWin + 1],
+                                            uint32_t nq, uint32_t* gout, unsigned lt, unsigned lbit) {
+    switch (nck) {
+        case 1: emit_rows<1>(ids, wq, nq, gout, lt, lbit); break;
+        case 2: emit_rows<2>(ids, wq, nq, gout, lt, lbit); break;
+        case 3: emit_rows<3>(ids, wq, nq, gout, lt, lbit); break;
+        case 4: emit_rows<4>(ids, wq, nq, gout, lt, lbit); break;
+        case 5: emit_rows<5>(ids, wq, nq, gout, lt, lbit); break;
+        case 6: emit_rows<6>(ids, wq, nq, gout, lt, lbit); break;
+        case 7: emit_rows<7>(ids, wq, nq, gout, lt, lbit); break;
+        default: emit_rows<kWin>(ids, wq, nq, gout, lt, lbit); break;
+    }
+}
+
+// this window's candidate ids: lane j holds pair (2j, 2j+1) of each of its nck chunks
+__device__ __forceinline__ void window_ids(const SArgs& a, const VSpan* vsp, VCursor& cur, uint32_t v, uint32_t nck,
+                                           uint2 (&ids)[kWin], int lane) {
+#pragma unroll
+    for (int kk = 0; kk < kWin; ++kk) {
+        ids[kk] = make_uint2(0, 0);
+        if ((uint32_t)kk < nck) {
+            bool v0, v1;
+            const uint32_t s0 = vc_pair(cur, vsp, a.nspan, 32 * (v * kWin + kk) + lane, v0, v1);
+            if (v0 | v1) ids[kk] = __ldg((const uint2*)(a.ids + s0));
+        }
+    }
+}
+
 // Emit one query group from its hit masks: lane i starts query i's list at
 // gout + my; raw / wq / vsp are the warp's buffers (see k_emit).
+// nch: the group's chunk count when vsp already holds its spans (k_fused), else 0.
+// swin (k_fused, single-window groups): the window's masks are still in the count
+// phase's window buffer (count_group with keep_single) -- no mask round trip
+// through the L2; gmask is unused then.
 __device__ __forceinline__ void emit_group(const SArgs& a, uint32_t c, uint32_t nq, uint32_t nwin,
                                            const uint2* gmask, uint32_t* gout, uint32_t my,
-                                           uint2 (*raw)[kWin + 2], uint4 (*wq)[kWin + 1], VSpan* vsp, int lane) {
+                                           uint2 (*raw)[kWin + 2], uint4 (*wq)[kWin + 1], VSpan* vsp, int lane,
+                                           uint32_t nch = 0, const uint2 (*swin)[kWinPad] = nullptr) {
     const unsigned lt = (1u << lane) - 1u, lbit = 1u << lane;
     // the group's spans as one sequence of candidate pairs (same chunks as the count pass)
-    const uint32_t nch = (load_vspans(a, c, vsp, lane) + 31) / 32;
-    uint32_t rs = 0;   // this lane's current span
-    __syncwarp();   // the previous group's buffers are no longer read
-    if ((uint32_t)lane < nq) {   // prefetch window 0: lane i copies its 64-B mask row
-        const uint4* src = (const uint4*)(gmask + (size_t)lane * kWin);
+    if (nch == 0) nch = (load_vspans(a, c, vsp, lane) + 31) / 32;
+    VCursor cur;
+    vc_init(cur);
+    if (!swin) {
+        __syncwarp();   // the previous group's buffers are no longer read
+        if ((uint32_t)lane < nq) {   // prefetch window 0: lane i copies its 64-B mask row
+            const uint4* src = (const uint4*)(gmask + (size_t)lane * kWin);
 #pragma unroll
-        for (int u = 0; u < kWin / 2; ++u) cp_async16(&raw[lane][2 * u], src + u);
+            for (int u = 0; u < kWin / 2; ++u) cp_async16(&raw[lane][2 * u], src + u);
+        }
+        cp_async_commit();
     }
-    cp_async_commit();
 #pragma unroll 1
     for (uint32_t v = 0; v < nwin; ++v) {
         // this window's candidate ids: lane j holds pair (2j, 2j+1) of each chunk
+        const uint32_t nck = min((uint32_t)kWin, nch - v * kWin);
         uint2 ids[kWin];
-#pragma unroll
-        for (int kk = 0; kk < kWin; ++kk) {
-            bool v0, v1;
-            const uint32_t s0 = vpair(vsp, a.nspan, 32 * (v * kWin + kk) + lane, rs, v0, v1);
-            ids[kk] = make_uint2(0, 0);
-            if (v0 | v1) ids[kk] = __ldg((const uint2*)(a.ids + s0));
-        }
-        cp_async_wait<0>();
+        window_ids(a, vsp, cur, v, nck, ids, lane);
+        if (!swin) cp_async_wait<0>();
         __syncwarp();
         // lane i turns its row of masks into output positions (all queries in parallel)
         if ((uint32_t)lane < nq) {
+            const uint2* mrow = swin ? swin[lane] : raw[lane];
 #pragma unroll
             for (int kk = 0; kk < kWin; ++kk) {
-                const uint2 m = raw[lane][kk];
+                const uint2 m = mrow[kk];
                 const uint32_t p0 = my;
                 my += __popc(m.x);
                 wq[lane][kk] = make_uint4(m.x, m.y, p0, my);
@@ -721,42 +805,20 @@ __device__ __forceinline__ void emit_group(const SArgs& a, uint32_t c, uint32_t 
         }
         __syncwarp();
         // prefetch the next window's masks into the landing buffer (overlaps the stores)
-        if (v + 1 < nwin && (uint32_t)lane < nq) {
-            const uint4* src = (const uint4*)(gmask + ((size_t)(v + 1) * nq + lane) * kWin);
+        if (!swin) {
+            if (v + 1 < nwin && (uint32_t)lane < nq) {
+                const uint4* src = (const uint4*)(gmask + ((size_t)(v + 1) * nq + lane) * kWin);
 #pragma unroll
-            for (int u = 0; u < kWin / 2; ++u) cp_async16(&raw[lane][2 * u], src + u);
+                for (int u = 0; u < kWin / 2; ++u) cp_async16(&raw[lane][2 * u], src + u);
+            }
+            cp_async_commit();
         }
-        cp_async_commit();
         // chunks of this window (the last window of a group is usually partial: short
-        // groups, e.g. ~100-400 candidates on C5, have 2-7 of the 8 chunks -- emitting the
-        // empty ones cost ~6 instructions per half-chunk and query)
-        const uint32_t nck = min((uint32_t)kWin, nch - v * kWin);
-        if (nck == kWin) {
-#pragma unroll 1
-            for (uint32_t i = 0; i < nq; ++i) {
-#pragma unroll
-                for (int kk = 0; kk < kWin; ++kk) {
-                    const uint4 e = wq[i][kk];   // broadcast
-                    stg_if_bit(gout + (e.z + __popc(e.x & lt)), ids[kk].x, e.x, lbit);
-                    stg_if_bit(gout + (e.w + __popc(e.y & lt)), ids[kk].y, e.y, lbit);
-                }
-            }
-        } else {
-#pragma unroll 1
-            for (uint32_t i = 0; i < nq; ++i) {
-#pragma unroll
-                for (int kk = 0; kk < kWin; ++kk) {
-                    if ((uint32_t)kk < nck) {
-                        const uint4 e = wq[i][kk];
-                        stg_if_bit(gout + (e.z + __popc(e.x & lt)), ids[kk].x, e.x, lbit);
-                        stg_if_bit(gout + (e.w + __popc(e.y & lt)), ids[kk].y, e.y, lbit);
-                    }
-                }
-            }
-        }
+        // groups, e.g. ~100-400 candidates on C5, have 2-7 of the 8 chunks)
+        emit_window(nck, ids, wq, nq, gout, lt, lbit);
         __syncwarp();   // wq is rewritten for the next window
     }
-    cp_async_wait<0>();
+    if (!swin) cp_async_wait<0>();
 }
 
 __global__ void __launch_bounds__(kEmitThreads) k_emit(SArgs a, uint32_t g0, uint32_t g1, uint32_t chunk,
@@ -847,8 +909,9 @@ __global__ void __launch_bounds__(kFusedThreads, kFusedMinBlocks)
 #pragma unroll
         for (int kk = 0; kk < kWin; ++kk) my_sm.c.swin[lane][kk] = make_uint2(0, 0);
         uint2* gmask = masks + (m.ma >> 1);
+        uint32_t nch = 0;
         const uint32_t my = count_group<MODE>(a, m.qs, m.c, m.nq, my_sm.c.swin, vsp[w], my_sm.c.sq, my_sm.c.sqd,
-                                              gmask, tests, lane);
+                                              gmask, tests, lane, true, &nch);
         // reserve the group's output
         uint32_t incl = my;
 #pragma unroll
@@ -863,17 +926,19 @@ __global__ void __launch_bounds__(kFusedThreads, kFusedMinBlocks)
         const uint32_t excl = incl - my;
         if ((uint32_t)lane < m.nq) {
             const uint32_t id = __ldg(&a.ids[m.qs + lane]);
-            cnt[m.qs + lane] = my;
+            if (cnt) cnt[m.qs + lane] = my;   // counts in sorted order (optional)
             begin[id] = base + excl;
             count[id] = my;
         }
         if (base + total <= cap) {
-            __threadfence_block();   // the masks this warp just stored are read back by cp.async
-            __syncwarp();
             uint32_t* gout = out + base;
             asm volatile("mov.b64 %0, %0;" : "+l"(gout));
-            const uint32_t nwin = (uint32_t)((m.mb - m.ma) / (2ull * m.nq * kWin));
-            emit_group(a, m.c, m.nq, nwin, gmask, gout, excl, my_sm.e.raw, my_sm.e.wq, vsp[w], lane);
+            const bool single = nch <= kWin;   // one window: its masks are still in swin
+            if (!single) __threadfence_block();   // the masks this warp just stored are read back by cp.async
+            __syncwarp();
+            const uint32_t nwin = single ? 1u : (uint32_t)((m.mb - m.ma) / (2ull * m.nq * kWin));
+            emit_group(a, m.c, m.nq, nwin, gmask, gout, excl, my_sm.e.raw, my_sm.e.wq, vsp[w], lane, nch,
+                       single ? my_sm.c.swin : nullptr);
         } else if (lane == 0) {
             atomicOr(overflow, 1u);
         }
