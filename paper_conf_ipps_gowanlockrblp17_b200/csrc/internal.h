@@ -135,7 +135,10 @@ void launch_group_class(const uint32_t* cstart, const uint2* cspan, uint32_t nsp
 // 2 * kOrderBins words (bin sizes from launch_group_class, then cursors; zeroed by the caller);
 // launch_group_class also writes the hit-mask words per group (windows of win chunks)
 constexpr int kOrderBins = 64;
-constexpr int kMaskWin = 8;   // chunks per window of the hit-mask layout (kernels_search.cu kWin)
+#ifndef HDB_KWIN
+#define HDB_KWIN 8
+#endif
+constexpr int kMaskWin = HDB_KWIN;   // chunks per window of the hit-mask layout (kernels_search.cu kWin)
 void launch_order_scatter(const uint8_t* gbin, const uint32_t* ng_dev, uint64_t n, uint32_t* ohist, uint32_t* ord,
                           cudaStream_t s);
 void launch_group_lists(const uint32_t* gstart, const uint32_t* gcell, const uint32_t* ng_dev, uint64_t n,

@@ -29,6 +29,7 @@
 #include <stdint.h>
 
 #include <algorithm>
+#include <cstdlib>
 
 #include "internal.h"
 #include "predicate.cuh"
@@ -106,15 +107,65 @@ __device__ __forceinline__ void stg_if(uint32_t* p, uint32_t v, bool f) {
     asm volatile("{ .reg .pred q; setp.ne.b32 q, %2, 0; @q st.global.u32 [%0], %1; }" ::"l"(p), "r"(v),
                  "r"((uint32_t)f));
 }
-// store v at p iff (m & bit) != 0 -- the mask test inside the asm keeps it one LOP3.P
+// store v at p iff (m & bit) != 0 -- the mask test inside the asm keeps it one LOP3.P.
+// HDB_STG_CS: the table's id stream is written with the streaming (evict-first)
+// cache operator, so the GBs of output do not push the candidates out of the L2
+#ifndef HDB_STG_CS
+#define HDB_STG_CS 1
+#endif
 __device__ __forceinline__ void stg_if_bit(uint32_t* p, uint32_t v, uint32_t m, uint32_t bit) {
+#if HDB_STG_CS
+    asm volatile("{ .reg .pred q; .reg .b32 t; and.b32 t, %2, %3; setp.ne.b32 q, t, 0; @q st.global.cs.u32 [%0], %1; }" ::"l"(p),
+                 "r"(v), "r"(m), "r"(bit));
+#else
     asm volatile("{ .reg .pred q; .reg .b32 t; and.b32 t, %2, %3; setp.ne.b32 q, t, 0; @q st.global.u32 [%0], %1; }" ::"l"(p),
                  "r"(v), "r"(m), "r"(bit));
+#endif
+}
+// HDB_LD_EL: candidate coordinates / ids read with an L2 evict-last policy (they are
+// re-read by the neighbouring groups' stencils while the output streams past)
+#ifndef HDB_LD_EL
+#define HDB_LD_EL 1
+#endif
+#ifndef HDB_PF
+#define HDB_PF 0
+#endif
+__device__ __forceinline__ double2 ld_cand(const double2* p) {
+#if HDB_LD_EL
+    uint64_t pol;
+    asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
+    double2 r;
+    asm("ld.global.nc.L2::cache_hint.v2.f64 {%0, %1}, [%2], %3;" : "=d"(r.x), "=d"(r.y) : "l"(p), "l"(pol));
+    return r;
+#else
+    return __ldg(p);
+#endif
+}
+__device__ __forceinline__ uint2 ld_ids(const uint2* p) {
+#if HDB_LD_EL
+    uint64_t pol;
+    asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
+    uint2 r;
+    asm("ld.global.nc.L2::cache_hint.v2.u32 {%0, %1}, [%2], %3;" : "=r"(r.x), "=r"(r.y) : "l"(p), "l"(pol));
+    return r;
+#else
+    return __ldg(p);
+#endif
 }
 __device__ __forceinline__ u64x fma2(u64x a, u64x b, u64x c) {
     u64x r;
     asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(r) : "l"(a), "l"(b), "l"(c));
     return r;
+}
+
+__device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
+    const uint32_t sa = (uint32_t)__cvta_generic_to_shared(smem);
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(sa), "l"(gmem));
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() {
+    asm volatile("cp.async.wait_group %0;" ::"n"(N));
 }
 
 // Kernel modes: f32 input (exact f32 predicate), f64 input with the f32
@@ -339,7 +390,8 @@ template <int MODE>
 __device__ __forceinline__ uint32_t count_group(const SArgs& a, uint32_t qs, uint32_t c, uint32_t nq,
                                                 uint2 (*swin)[kWinPad], VSpan* vsp, ulonglong2* sq, double2* sqd,
                                                 uint2* gmask, unsigned long long& tests, int lane,
-                                                bool keep_single = false, uint32_t* nch_out = nullptr) {
+                                                bool keep_single = false, uint32_t* nch_out = nullptr,
+                                                double2* cbuf = nullptr) {
     const ulonglong2* __restrict__ xp = (const ulonglong2*)a.xp;
     const u64x NE2 = pack2(-a.e2f, -a.e2f);
     const u64x NB2 = pack2(a.nb2_l, a.nb2_l);
@@ -373,20 +425,46 @@ __device__ __forceinline__ uint32_t count_group(const SArgs& a, uint32_t qs, uin
     }
     VCursor cur;
     vc_init(cur);
+    // cbuf (f64 modes, k_fused): each chunk's candidate pair is prefetched into the
+    // warp's 2-stage buffer with cp.async one chunk ahead (lane j owns its slots, so
+    // no warp barrier is needed), hiding the L2 / DRAM latency of the candidates
+    const bool pf = MODE != kF32 && cbuf != nullptr;
+    auto issue = [&](uint32_t kc) -> uint32_t {
+        bool w0, w1;
+        const uint32_t t0 = vc_pair(cur, vsp, a.nspan, 32 * kc + lane, w0, w1);
+        double2* dst = cbuf + ((kc & 1) * 32 + lane) * 2;
+        if (w0) cp_async16(dst, a.xd + t0);
+        if (w1) cp_async16(dst + 1, a.xd + t0 + 1);
+        cp_async_commit();
+        return (uint32_t)w0 | ((uint32_t)w1 << 1);
+    };
+    uint32_t vf = (pf && nch) ? issue(0) : 0u;
     uint32_t k = 0;
 #pragma unroll 1
     for (; k < nch; ++k) {
         const uint32_t kk = k % kWin;
         bool v0, v1;
-        const uint32_t s0 = vc_pair(cur, vsp, a.nspan, 32 * k + lane, v0, v1), s1 = s0 + 1;
+        uint32_t s0 = 0;
         u64x X, Y;
         double2 d0 = make_double2(kFarD, kFarD), d1 = make_double2(kFarD, kFarD);
         ulonglong2 P = make_ulonglong2(0, 0);
-        if (MODE == kF32) {
-            if (v0 || v1) P = xp[s0 >> 1];
+        if (pf) {
+            const uint32_t vfn = k + 1 < nch ? issue(k + 1) : (cp_async_commit(), 0u);
+            cp_async_wait<1>();   // this lane's copies of chunk k have landed
+            v0 = vf & 1u;
+            v1 = vf & 2u;
+            const double2* src = cbuf + ((k & 1) * 32 + lane) * 2;
+            if (v0) d0 = src[0];
+            if (v1) d1 = src[1];
+            vf = vfn;
         } else {
-            if (v0) d0 = a.xd[s0];
-            if (v1) d1 = a.xd[s1];
+            s0 = vc_pair(cur, vsp, a.nspan, 32 * k + lane, v0, v1);
+            if (MODE == kF32) {
+                if (v0 || v1) P = xp[s0 >> 1];
+            } else {
+                if (v0) d0 = ld_cand(a.xd + s0);
+                if (v1) d1 = ld_cand(a.xd + s0 + 1);
+            }
         }
         if (MODE == kF32) {
             const float2 px = unpack2(P.x), py = unpack2(P.y);
@@ -704,16 +782,6 @@ __global__ void __launch_bounds__(kSearchThreads) k_search(SArgs a, uint32_t g0,
 constexpr int kEmitThreads = 128;   // 4 warps per CTA (the padded window buffers are 28 KB per CTA)
 constexpr int kEmitWarps = kEmitThreads / 32;
 
-__device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
-    const uint32_t sa = (uint32_t)__cvta_generic_to_shared(smem);
-    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(sa), "l"(gmem));
-}
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;"); }
-template <int N>
-__device__ __forceinline__ void cp_async_wait() {
-    asm volatile("cp.async.wait_group %0;" ::"n"(N));
-}
-
 // Emission of one window for every query of the group: per query, the window's
 // hits are one contiguous run of its list; per chunk, lane j stores its pair's
 // hits at (run start + popc of the chunk's mask below j).  NCK = the window's
@@ -733,16 +801,23 @@ __device__ __forceinline__ void emit_rows(const uint2 (&ids)[kWin], const uint4 
 }
 __device__ __forceinline__ void emit_window(uint32_t nck, const uint2 (&ids)[kWin], const uint4 (*wq)[kWin + 1],
                                             uint32_t nq, uint32_t* gout, unsigned lt, unsigned lbit) {
+#define HDB_EMIT_CASE(N)                                                                   \
+    case N:                                                                                \
+        if (N < kWin) {                                                                    \
+            emit_rows<(N < kWin ? N : kWin)>(ids, wq, nq, gout, lt, lbit);                 \
+            break;                                                                         \
+        }
     switch (nck) {
-        case 1: emit_rows<1>(ids, wq, nq, gout, lt, lbit); break;
-        case 2: emit_rows<2>(ids, wq, nq, gout, lt, lbit); break;
-        case 3: emit_rows<3>(ids, wq, nq, gout, lt, lbit); break;
-        case 4: emit_rows<4>(ids, wq, nq, gout, lt, lbit); break;
-        case 5: emit_rows<5>(ids, wq, nq, gout, lt, lbit); break;
-        case 6: emit_rows<6>(ids, wq, nq, gout, lt, lbit); break;
-        case 7: emit_rows<7>(ids, wq, nq, gout, lt, lbit); break;
+        HDB_EMIT_CASE(1)
+        HDB_EMIT_CASE(2)
+        HDB_EMIT_CASE(3)
+        HDB_EMIT_CASE(4)
+        HDB_EMIT_CASE(5)
+        HDB_EMIT_CASE(6)
+        HDB_EMIT_CASE(7)
         default: emit_rows<kWin>(ids, wq, nq, gout, lt, lbit); break;
     }
+#undef HDB_EMIT_CASE
 }
 
 // this window's candidate ids: lane j holds pair (2j, 2j+1) of each of its nck chunks
@@ -754,7 +829,7 @@ __device__ __forceinline__ void window_ids(const SArgs& a, const VSpan* vsp, VCu
         if ((uint32_t)kk < nck) {
             bool v0, v1;
             const uint32_t s0 = vc_pair(cur, vsp, a.nspan, 32 * (v * kWin + kk) + lane, v0, v1);
-            if (v0 | v1) ids[kk] = __ldg((const uint2*)(a.ids + s0));
+            if (v0 | v1) ids[kk] = ld_ids((const uint2*)(a.ids + s0));
         }
     }
 }
@@ -873,7 +948,10 @@ __global__ void __launch_bounds__(kEmitThreads) k_emit(SArgs a, uint32_t g0, uin
 // ALU) of some warps overlaps the store streams of others.
 constexpr int kFusedThreads = 128;
 constexpr int kFusedWarps = kFusedThreads / 32;
-constexpr int kFusedMinBlocks = 7;
+#ifndef HDB_FUSED_MINB
+#define HDB_FUSED_MINB (kWin <= 4 ? 8 : 7)
+#endif
+constexpr int kFusedMinBlocks = HDB_FUSED_MINB;
 // per-warp shared memory: the count phase's buffers and the emit phase's share
 // one union (the phases of a warp never overlap), so a CTA needs the larger of
 // the two (~7 KB per warp) instead of their sum
@@ -881,6 +959,9 @@ struct FusedCount {
     uint2 swin[32][kWinPad];
     ulonglong2 sq[32];
     double2 sqd[32];
+#if HDB_PF
+    double2 cand[2 * 32 * 2];   // count phase: 2-stage cp.async buffer of the candidate pairs
+#endif
 };
 struct FusedEmit {
     uint2 raw[32][kWin + 2];
@@ -910,8 +991,13 @@ __global__ void __launch_bounds__(kFusedThreads, kFusedMinBlocks)
         for (int kk = 0; kk < kWin; ++kk) my_sm.c.swin[lane][kk] = make_uint2(0, 0);
         uint2* gmask = masks + (m.ma >> 1);
         uint32_t nch = 0;
+#if HDB_PF
+        double2* cbuf = my_sm.c.cand;
+#else
+        double2* cbuf = nullptr;
+#endif
         const uint32_t my = count_group<MODE>(a, m.qs, m.c, m.nq, my_sm.c.swin, vsp[w], my_sm.c.sq, my_sm.c.sqd,
-                                              gmask, tests, lane, true, &nch);
+                                              gmask, tests, lane, true, &nch, cbuf);
         // reserve the group's output
         uint32_t incl = my;
 #pragma unroll
@@ -1364,6 +1450,15 @@ void launch_fused_mode(const SArgs& a, uint64_t g0, uint64_t g1, unsigned int* c
     uint32_t chunk;
     unsigned ctas;
     launch_groups(k_fused<MODE>, bps, g1 - g0, chunk, ctas, kFusedThreads);
+    // natural (cell-sorted) order: small grabs keep the front of groups in flight spatially
+    // narrow, so the stencil rows above / below a group are still in the L2 (C5: grabs of
+    // 31 / 16 / 8 / 4 groups: 16.13 / 15.71 / 15.60 / 15.48 ms per step)
+    if (!a.ord) chunk = std::min<uint32_t>(chunk, 4);
+    static const uint32_t chunk_env = [] {
+        const char* e = std::getenv("HDB_FUSED_CHUNK");   // tuning knob (A/B runs)
+        return e ? (uint32_t)std::strtoul(e, nullptr, 10) : 0u;
+    }();
+    if (chunk_env) chunk = chunk_env;
     k_fused<MODE><<<ctas, kFusedThreads, 0, s>>>(a, (uint32_t)g0, (uint32_t)g1, chunk, ctr, cnt, tests, masks, moff,
                                                  pair_ctr, cap, out, begin, count, overflow);
 }
