@@ -334,14 +334,46 @@ uint32_t split_from_occ(const unsigned long long* h, uint64_t n, const DevGrid& 
     return k;
 }
 
-void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t n, hdb_dtype dt, double eps,
+// HDB_BANDS=0 turns the process-shard bands off (every rank then builds the full grid)
+bool bands_enabled() {
+    static const bool on = [] {
+        const char* e = std::getenv("HDB_BANDS");
+        return !(e && *e == '0');
+    }();
+    return on;
+}
+
+// rows [y0, y1) of shard `rank` of R: the cut rows split the cumulative load into R
+// equal parts (cut r = first row whose prefix load reaches r/R of the total)
+void band_rows(const std::vector<uint64_t>& load, uint32_t R, uint32_t rank, uint64_t& y0, uint64_t& y1) {
+    const uint64_t ny = load.size();
+    unsigned __int128 total = 0;
+    for (uint64_t v : load) total += v;
+    auto cut = [&](uint32_t r) -> uint64_t {
+        if (r == 0) return 0;
+        if (r >= R) return ny;
+        const unsigned __int128 target = total * r / R;
+        unsigned __int128 acc = 0;
+        for (uint64_t y = 0; y < ny; ++y) {
+            if (acc >= target) return y;
+            acc += load[y];
+        }
+        return ny;
+    };
+    y0 = cut(rank);
+    y1 = std::max(y0, cut(rank + 1));
+}
+
+void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t n_in, hdb_dtype dt, double eps,
                DevGrid& g) {
     DeviceGuard dg(dc.device);
     cudaStream_t s = dc.main;
     const size_t esz = dt == HDB_F64 ? 16 : 8;
+    uint64_t n = n_in;   // points of this grid (a process shard's band: fewer than the input's)
     g.device = dc.device;
     g.dtype = dt;
     g.n = n;
+    g.n_ids = n_in;
     g.stream = s;
     Event ev0, ev1;
     HDB_CUDA(cudaEventRecord(ev0.e, s));
@@ -355,7 +387,7 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
         if (where.loc == Loc::Host) {
             xin_owned = DBuf(n * esz, s);
             HDB_CUDA(cudaMemcpyAsync(xin_owned.p, xy, n * esz, cudaMemcpyHostToDevice, s));
-            ctx->stats.bytes_h2d += n * esz;
+            __atomic_fetch_add(&ctx->stats.bytes_h2d, (uint64_t)(n * esz), __ATOMIC_RELAXED);   // devices build in parallel
             xin = xin_owned.p;
         } else if (where.device != dc.device) {
             xin_owned = DBuf(n * esz, s);
@@ -430,6 +462,53 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
     set_filter_bound(g);
 
     tr.mark("bbox+sync");
+    // ---- process shard (torchrun rank r of R, one device): a band of cell rows as queries
+    // plus k halo rows of candidates on either side -- only those points are sorted (the
+    // grid build is not replicated across ranks)
+    DBuf band_pts, band_gid;
+    uint64_t band_y0 = 0, band_y1 = 0;
+    const uint32_t R_proc = ctx->opts.shard_count > 0 ? (uint32_t)ctx->opts.shard_count : 1;
+    if (R_proc > 1 && ctx->dev.size() == 1 && n > 0 && g.ny <= (1u << 22) && bands_enabled()) {
+        const uint32_t rank = (uint32_t)ctx->opts.shard_rank;
+        const bool dense = g.n_cells <= std::max<uint64_t>(8 * n, 1ull << 22);
+        DBuf rc(8ull * g.ny, s), rl(8ull * g.ny, s), cc;
+        HDB_CUDA(cudaMemsetAsync(rc.p, 0, 8ull * g.ny, s));
+        HDB_CUDA(cudaMemsetAsync(rl.p, 0, 8ull * g.ny, s));
+        if (dense) {
+            cc = DBuf(4 * g.n_cells, s);
+            HDB_CUDA(cudaMemsetAsync(cc.p, 0, 4 * g.n_cells, s));
+        }
+        row_loads(xin, n, dt, g.xmin, g.ymin, g.inv_w, g.nx, g.ny, cc.as<uint32_t>(), rc.as<unsigned long long>(),
+                  rl.as<unsigned long long>(), s);
+        HDB_LAUNCH_CHECK();
+        std::vector<uint64_t> hrc(g.ny), hrl(g.ny);
+        HDB_CUDA(cudaMemcpyAsync(hrc.data(), rc.p, 8ull * g.ny, cudaMemcpyDeviceToHost, s));
+        HDB_CUDA(cudaMemcpyAsync(hrl.data(), rl.p, 8ull * g.ny, cudaMemcpyDeviceToHost, s));
+        HDB_CUDA(cudaStreamSynchronize(s));
+        const std::vector<uint64_t>& load = dense ? hrl : hrc;
+        band_rows(load, R_proc, rank, band_y0, band_y1);
+        const uint64_t ylo = band_y0 >= g.split ? band_y0 - g.split : 0;
+        const uint64_t yhi = std::min<uint64_t>(g.ny, band_y1 + g.split);
+        uint64_t q0 = 0, q1 = 0, nb = 0;
+        for (uint64_t y = 0; y < g.ny; ++y) {
+            if (y < band_y0) q0 += hrc[y];
+            if (y < band_y1) q1 += hrc[y];
+            if (y >= ylo && y < yhi) nb += hrc[y];
+        }
+        band_pts = DBuf(esz * (nb ? nb : 1), s);
+        band_gid = DBuf(4 * (nb ? nb : 1), s);
+        DBuf dnb(8, s), btemp(scan_temp_bytes(n + 1), s);
+        band_select(xin, n, dt, g.xmin, g.ymin, g.inv_w, g.nx, g.ny, ylo, yhi, band_pts.p, band_gid.as<uint32_t>(),
+                    dnb.as<uint32_t>(), btemp.p, s);
+        HDB_LAUNCH_CHECK();
+        xin = band_pts.p;
+        n = nb;
+        g.n = n;
+        g.banded = true;
+        g.band_q0 = q0;
+        g.band_q1 = q1;
+        tr.mark("band");
+    }
     // ---- a2 + a3: the points sorted by cell key (record radix sort over only the bits the
     // key range needs; the first pass computes the keys from the input points, the last
     // writes A, the sorted points and the f32 filter copy -- no separate gather).  ids and
@@ -445,7 +524,8 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
     if (n > 0) {
         DBuf stemp(point_sort_temp_bytes(n, dt, kb, bits), s);   // stream-ordered: freed after the sort
         sort_points(xin, n, dt, g.xmin, g.ymin, g.inv_w, g.nx, g.ny, kb, bits, keys.p, ids.as<uint32_t>(), xy_s.p,
-                    xp.as<float4>(), g.ox, g.oy, counters.as<unsigned int>(), kCounterSlots, stemp.p, s);
+                    xp.as<float4>(), g.ox, g.oy, counters.as<unsigned int>(), kCounterSlots, stemp.p, s,
+                    g.banded ? band_gid.as<uint32_t>() : nullptr);
         HDB_LAUNCH_CHECK();
     } else {
         HDB_CUDA(cudaMemsetAsync(ids.p, 0, 8, s));
@@ -454,6 +534,8 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
         HDB_CUDA(cudaMemsetAsync(counters.p, 0, 4 * kCounterSlots, s));
     }
     xin_owned.reset();
+    band_pts.reset();
+    band_gid.reset();
     DBuf temp(scan_temp_bytes(n + 1), s);
     tr.mark("sort(enqueue)");
     // ---- a4: run-length encoding of the sorted keys -> (key, start) of the non-empty cells
@@ -551,8 +633,10 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
         launch_readback(bb + 16, gofs.as<uint32_t>() + nne, moff.as<uint64_t>() + NG,
                         classify ? dpre.as<uint32_t>() + NG : nullptr, classify ? spre.as<uint32_t>() + NG : nullptr,
                         classify ? nsp : nullptr, s);
+        if (g.banded)   // the band's query groups -> bb[22..23]
+            launch_band_groups(g.ckey, nne, gofs.as<uint32_t>(), band_y0 * g.nx, band_y1 * g.nx, bb + 22, s);
         uint64_t* pr = dc.pin + 18;
-        HDB_CUDA(cudaMemcpyAsync(pr, bb + 16, 48, cudaMemcpyDeviceToHost, s));
+        HDB_CUDA(cudaMemcpyAsync(pr, bb + 16, 64, cudaMemcpyDeviceToHost, s));
         HDB_CUDA(cudaEventRecord(ev1.e, s));
         tr.mark("class+order+masklayout-enqueue");
         HDB_CUDA(cudaEventSynchronize(ev1.e));
@@ -562,6 +646,10 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
         const uint64_t hsp = pr[4];
         g.tests_total = pr[5];
         g.n_groups = hng;
+        if (g.banded) {
+            g.band_g0 = pr[6];
+            g.band_g1 = pr[7];
+        }
         g.moff = (uint64_t*)moff.release();
         g.n_dense_groups = hng;
         g.n_sparse_q = 0;
@@ -606,6 +694,35 @@ void free_dev_grid(DevGrid& g) {
 
 }  // namespace
 
+namespace {
+template <typename F>
+void run_parallel(size_t k, F&& f) {
+    if (k == 1) {
+        f(0);
+        return;
+    }
+    std::vector<std::exception_ptr> errs(k);
+    std::vector<std::string> msgs(k);
+    std::vector<std::thread> th;
+    for (size_t i = 0; i < k; ++i)
+        th.emplace_back([&, i] {
+            try {
+                f(i);
+            } catch (...) {
+                errs[i] = std::current_exception();
+                msgs[i] = last_error();
+            }
+        });
+    for (auto& t : th) t.join();
+    for (size_t i = 0; i < k; ++i)
+        if (errs[i]) {
+            g_err = msgs[i];
+            std::rethrow_exception(errs[i]);
+        }
+}
+
+}  // namespace
+
 // ------------------------------------------------------------------ grid
 void grid_build(hdb_ctx* ctx, const void* xy, uint64_t n, hdb_dtype dt, double eps, hdb_grid** out) {
     if (dt != HDB_F64 && dt != HDB_F32) fail(HDB_EINVAL, "unknown dtype %d", (int)dt);
@@ -618,7 +735,8 @@ void grid_build(hdb_ctx* ctx, const void* xy, uint64_t n, hdb_dtype dt, double e
     g->ctx = ctx;
     g->dev.resize(ctx->dev.size());
     try {
-        for (size_t d = 0; d < ctx->dev.size(); ++d) build_dev(ctx, ctx->dev[d], xy, where, n, dt, eps, g->dev[d]);
+        // every device builds its copy of the grid at the same time (one host thread each)
+        run_parallel(ctx->dev.size(), [&](size_t d) { build_dev(ctx, ctx->dev[d], xy, where, n, dt, eps, g->dev[d]); });
     } catch (...) {
         for (auto& dg : g->dev) free_dev_grid(dg);
         delete g;
@@ -767,11 +885,11 @@ bool single_pass_table(hdb_ctx* ctx, const DevGrid& g, hdb_table* t, hdb_stats& 
                        bool exact_bound = false) {
     DevCtx& dc = ctx->dev[0];
     cudaStream_t s = dc.main;
-    const uint64_t n = g.n;
+    const uint64_t n = g.n_ids;   // rows of T (a banded grid holds fewer points)
     // est: the sampled estimate a_b (cap with headroom; a reservation past it falls back to
     // the two passes) or, exact_bound, an upper bound on P (the grid's candidate tests)
     const uint64_t cap = exact_bound ? std::max<uint64_t>(est, 1)
-                                     : (uint64_t)((double)std::max<uint64_t>(est, n) * 1.25) + (1ull << 20);
+                                     : (uint64_t)((double)std::max<uint64_t>(est, g.n) * 1.25) + (1ull << 20);
     DBuf masks, nb;
     if (cudaMallocFromPoolAsync(&masks.p, 4 * std::max<uint64_t>(g.mask_words, 4), dc.big_pool, s) != cudaSuccess ||
         cudaMallocFromPoolAsync(&nb.p, 4 * cap, dc.big_pool, s) != cudaSuccess) {
@@ -779,12 +897,17 @@ bool single_pass_table(hdb_ctx* ctx, const DevGrid& g, hdb_table* t, hdb_stats& 
         return false;
     }
     masks.s = nb.s = s;
-    DBuf beg(8 * n, s, dc.big_pool), cnt_id(4 * n, s, dc.big_pool), scratch(32, s);
+    DBuf beg(8 * (n ? n : 1), s, dc.big_pool), cnt_id(4 * (n ? n : 1), s, dc.big_pool), scratch(32, s);
     HDB_CUDA(cudaMemsetAsync(scratch.p, 0, 32, s));
+    if (g.banded) {   // a shard's table: rows outside the band stay empty
+        HDB_CUDA(cudaMemsetAsync(beg.p, 0, 8 * n, s));
+        HDB_CUDA(cudaMemsetAsync(cnt_id.p, 0, 4 * n, s));
+    }
     unsigned long long* sc = scratch.as<unsigned long long>();
     Event e0, e1;
     HDB_CUDA(cudaEventRecord(e0.e, s));
-    launch_fused(g, nullptr, sc, masks.as<uint2>(), sc + 1, cap, nb.as<uint32_t>(), beg.as<uint64_t>(),
+    const uint64_t g0 = g.banded ? g.band_g0 : 0, g1 = g.banded ? g.band_g1 : g.n_groups;
+    launch_fused(g, g0, g1, nullptr, sc, masks.as<uint2>(), sc + 1, cap, nb.as<uint32_t>(), beg.as<uint64_t>(),
                  cnt_id.as<uint32_t>(), (unsigned int*)(sc + 2), s);
     HDB_LAUNCH_CHECK();
     HDB_CUDA(cudaEventRecord(e1.e, s));
@@ -797,11 +920,14 @@ bool single_pass_table(hdb_ctx* ctx, const DevGrid& g, hdb_table* t, hdb_stats& 
     t->device = dc.device;
     t->dstream = s;
     t->npairs = P;
-    t->first_query = 0;
-    t->end_query = n;
-    DBuf rw(4 * n, s, dc.big_pool);
-    HDB_CUDA(cudaMemcpyAsync(rw.p, g.ids, 4 * n, cudaMemcpyDeviceToDevice, s));
-    t->rows = (uint32_t*)rw.release();
+    t->first_query = g.banded ? g.band_q0 : 0;
+    t->end_query = g.banded ? g.band_q1 : n;
+    if (!g.banded && n) {
+        // production order of the rows (device DBSCAN walks them in this cell-sorted order)
+        DBuf rw(4 * n, s, dc.big_pool);
+        HDB_CUDA(cudaMemcpyAsync(rw.p, g.ids, 4 * n, cudaMemcpyDeviceToDevice, s));
+        t->rows = (uint32_t*)rw.release();
+    }
     t->nbrs = (uint32_t*)nb.release();
     t->begin = (uint64_t*)beg.release();
     t->count = (uint32_t*)cnt_id.release();
@@ -962,32 +1088,6 @@ void write_phase_host(hdb_ctx* ctx, DevCtx& dc, const DevGrid& g, ShardState& st
     st.max_batch = maxb;
 }
 
-template <typename F>
-void run_parallel(size_t k, F&& f) {
-    if (k == 1) {
-        f(0);
-        return;
-    }
-    std::vector<std::exception_ptr> errs(k);
-    std::vector<std::string> msgs(k);
-    std::vector<std::thread> th;
-    for (size_t i = 0; i < k; ++i)
-        th.emplace_back([&, i] {
-            try {
-                f(i);
-            } catch (...) {
-                errs[i] = std::current_exception();
-                msgs[i] = last_error();
-            }
-        });
-    for (auto& t : th) t.join();
-    for (size_t i = 0; i < k; ++i)
-        if (errs[i]) {
-            g_err = msgs[i];
-            std::rethrow_exception(errs[i]);
-        }
-}
-
 template <typename T>
 T* pool_get(hdb_table* t, size_t count, size_t* cap) {
     return (T*)t->pool->acquire(count * sizeof(T), cap);
@@ -1049,7 +1149,9 @@ void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hd
     const uint64_t launches0 = g_kernel_launches.load();
     hdb_stats& S = ctx->stats;
     const DevGrid& G0 = grid->dev[0];
-    const uint64_t n = G0.n;
+    const uint64_t n = G0.n_ids;    // rows of T
+    const uint64_t n_pts = G0.n;    // points of the grid (a process shard's band: fewer)
+    const bool banded = G0.banded;
     S.n = n;
     S.n_cells = G0.n_cells;
     S.n_nonempty = G0.n_nonempty;
@@ -1073,12 +1175,13 @@ void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hd
         Trace tr("neighbor_table");
         DevCtx& dc0 = ctx->dev[0];
         DeviceGuard dg0(dc0.device);
-        const uint32_t parts = R_proc * (uint32_t)ndev;
+        // a banded grid (process shard) is already this rank's part: no further cuts
+        const uint32_t parts = banded ? 1u : R_proc * (uint32_t)ndev;
         // ---- dense device-resident whole table: the single pass sized by the exact upper
         // bound P <= candidate tests (known from the grid), no sampled estimate needed (the
         // sample kernel and its readback sync were ~3% of a C2 step)
-        if (device_resident && parts == 1 && ctx->opts.search_kernel == 0 && n > 0 && !G0.dl &&
-            G0.tests_total >= (uint64_t)(kFusedDirectTestsPerQuery * (double)n) &&
+        if (device_resident && parts == 1 && ctx->opts.search_kernel == 0 && n_pts > 0 && !G0.dl &&
+            G0.tests_total >= (uint64_t)(kFusedDirectTestsPerQuery * (double)n_pts) &&
             4.0 * (double)G0.tests_total <= kFusedDirectMemShare * (double)dc0.total_mem) {
             S.sample_size = 0;
             S.sample_pairs = 0;
@@ -1100,7 +1203,7 @@ void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hd
         // ---- a5: sampled count + plan (device 0)
         const double f = ctx->opts.sample_fraction;
         const uint64_t stride = std::max<uint64_t>(1, (uint64_t)std::floor(1.0 / f));
-        const uint64_t ns = n ? (n + stride - 1) / stride : 0;
+        const uint64_t ns = n_pts ? (n_pts + stride - 1) / stride : 0;
         std::vector<uint32_t> samp;
         cudaStream_t s0 = dc0.main;
         DBuf dsamp(4 * (ns ? ns : 1), s0), dsum(8, s0);
@@ -1118,18 +1221,23 @@ void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hd
             HDB_CUDA(cudaStreamSynchronize(s0));
         }
         // ---- query shards: processes x devices, balanced by sampled counts
-        std::vector<uint64_t> cuts = shard_cuts(G0, dc0, samp, stride, parts);
-        for (size_t d = 0; d < ndev; ++d) {
-            const uint32_t k = rank * (uint32_t)ndev + (uint32_t)d;
-            sh[d].r.g0 = cuts[k];
-            sh[d].r.g1 = cuts[k + 1];
+        if (banded) {
+            sh[0].r.g0 = G0.band_g0;
+            sh[0].r.g1 = G0.band_g1;
+        } else {
+            std::vector<uint64_t> cuts = shard_cuts(G0, dc0, samp, stride, parts);
+            for (size_t d = 0; d < ndev; ++d) {
+                const uint32_t k = rank * (uint32_t)ndev + (uint32_t)d;
+                sh[d].r.g0 = cuts[k];
+                sh[d].r.g1 = cuts[k + 1];
+            }
         }
         tr.mark("sample+cuts");
         S.single_pass = 0;
         S.ms_sort = 0;
         bool single = false;
         const int sk = ctx->opts.search_kernel;
-        if ((sk == kPaperGlobal || sk == kPaperShared) && !(device_resident && parts == 1))
+        if ((sk == kPaperGlobal || sk == kPaperShared) && !(device_resident && parts == 1 && !banded))
             fail(HDB_EINVAL, "search_kernel %d (the paper's kernels) builds device-resident, unsharded tables only", sk);
         if ((sk == kPaperGlobal || sk == kPaperShared) && n > 0) {
             HDB_CUDA(cudaStreamSynchronize(s0));   // e_b is in dc0.pin[0]
@@ -1145,10 +1253,10 @@ void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hd
         // single pass (k_fused): asked for (search_kernel 4) or chosen for dense tables;
         // the dense/sparse split keeps the two passes (the sparse queries' kernels
         // write at scanned offsets)
-        if (!single && device_resident && parts == 1 && (sk == 4 || sk == 0) && n > 0 && !G0.dl) {
+        if (!single && device_resident && parts == 1 && (sk == 4 || sk == 0) && n_pts > 0 && !G0.dl) {
             HDB_CUDA(cudaStreamSynchronize(s0));   // e_b is in dc0.pin[0]
             const uint64_t eb = dc0.pin[0];
-            const bool fused = sk == 4 || (double)(eb * stride) >= kFusedMinPairsPerQuery * (double)n;
+            const bool fused = sk == 4 || (double)(eb * stride) >= kFusedMinPairsPerQuery * (double)n_pts;
             if (fused) {
                 S.sample_size = ns;
                 S.sample_pairs = eb;
@@ -1204,11 +1312,14 @@ void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hd
                 fail(HDB_ENOMEM, "table needs %llu bytes (P=%llu) > host budget %llu", (unsigned long long)(4 * P),
                      (unsigned long long)P, (unsigned long long)ctx->opts.host_budget_bytes);
             t->npairs = P;
-            const bool whole = (parts == 1);
+            const bool whole = (parts == 1) && !banded;
             // this process's rows: [first_query, end_query) of the sorted order -- the whole
             // table unless the process is one of several shards (R_proc > 1); empty shards
-            // (q0 = q1 = 0) do not count
-            if (R_proc == 1) {
+            // (q0 = q1 = 0) do not count; a band knows its global range
+            if (banded) {
+                t->first_query = G0.band_q0;
+                t->end_query = G0.band_q1;
+            } else if (R_proc == 1) {
                 t->first_query = 0;
                 t->end_query = n;
             } else {

@@ -47,7 +47,13 @@ constexpr int kMaxCellSplit = 6;    // cell_split k <= 6: 2k+1 <= 13 stencil row
 struct DevGrid {
     int device = 0;
     hdb_dtype dtype = HDB_F64;
-    uint64_t n = 0;
+    uint64_t n = 0;                // points of this grid
+    uint64_t n_ids = 0;            // the id space (rows of T): the input's point count
+    // process-shard band: the grid holds the cell rows of shard r plus k halo
+    // rows; its queries are the groups [band_g0, band_g1), rows [band_q0, band_q1) of the
+    // GLOBAL cell-sorted order; ids are input rows
+    bool banded = false;
+    uint64_t band_g0 = 0, band_g1 = 0, band_q0 = 0, band_q1 = 0;
     double eps = 0, w = 0, inv_w = 0;
     double e2_d = 0;     // fl(eps*eps) in f64
     float e2_f = 0;      // fl(eps_f*eps_f) in f32 (f32 mode) / fl32(e2_d) (f64 filter)
@@ -107,10 +113,24 @@ int radix_sort_pairs(void* k0, uint32_t* v0, void* k1, uint32_t* v1, int key_byt
 // records, keys computed by the first pass from the input points): keys_out[n] sorted keys,
 // ids_out[n + 2] A (padded), xy_s[n + 2] sorted points (padded), xp the f32 filter copy
 // (padded), counters zeroed.  temp: point_sort_temp_bytes(n, dt, key_bytes, bits)
+// process-shard bands: per cell row, the point count and a load estimate
+// (sum of squared cell counts; cell_cnt = a zeroed nx*ny histogram, or null: counts only,
+// row_load untouched); the band's points (rows [ylo, yhi)) with their input rows;
+// the band's query groups (cells with keys in [key_lo, key_hi)) -> out[0..1]
+void row_loads(const void* xy, uint64_t n, hdb_dtype dt, double xmin, double ymin, double inv_w, uint32_t nx,
+               uint32_t ny, uint32_t* cell_cnt, unsigned long long* row_cnt, unsigned long long* row_load,
+               cudaStream_t s);
+void band_select(const void* xy, uint64_t n, hdb_dtype dt, double xmin, double ymin, double inv_w, uint32_t nx,
+                 uint32_t ny, uint64_t ylo, uint64_t yhi, void* out, uint32_t* gid, uint32_t* n_out, void* temp,
+                 cudaStream_t s);
+void launch_band_groups(const uint64_t* ckey, uint64_t nne, const uint32_t* gofs, uint64_t key_lo, uint64_t key_hi,
+                        unsigned long long* out, cudaStream_t s);
 size_t point_sort_temp_bytes(uint64_t n, hdb_dtype dt, int key_bytes, int bits);
+// gid (optional): the points' ids (a process shard's band of the input); else the input row
 void sort_points(const void* xy_in, uint64_t n, hdb_dtype dt, double xmin, double ymin, double inv_w, uint32_t nx,
                  uint32_t ny, int key_bytes, int bits, void* keys_out, uint32_t* ids_out, void* xy_s, float4* xp,
-                 double ox, double oy, unsigned int* counters, uint32_t n_counters, void* temp, cudaStream_t s);
+                 double ox, double oy, unsigned int* counters, uint32_t n_counters, void* temp, cudaStream_t s,
+                 const uint32_t* gid = nullptr);
 // cnext: optional dense lookup (first non-empty cell with key >= h, h in [0, nx*ny]); null = binary search
 void launch_cell_spans(const uint64_t* ckey, const uint32_t* cstart, uint64_t nne, uint32_t nx, uint32_t ny,
                        uint32_t k, uint2* cspan, uint32_t* gcount, const uint32_t* cnext, cudaStream_t s);
@@ -182,7 +202,8 @@ void launch_count(const DevGrid& g, uint64_t g0, uint64_t g1, uint32_t* cnt, uns
 // single-pass device table (k_fused): count + reserve + emit per group; mask
 // table `masks` laid out by g.moff; rows reserved on *pair_ctr (zeroed by the
 // caller); *overflow set if a reservation passed cap
-void launch_fused(const DevGrid& g, uint32_t* cnt, unsigned long long* tests, uint2* masks,
+// over the query groups [g0, g1) (a process shard's band: its range); cnt may be null
+void launch_fused(const DevGrid& g, uint64_t g0, uint64_t g1, uint32_t* cnt, unsigned long long* tests, uint2* masks,
                   unsigned long long* pair_ctr, uint64_t cap, uint32_t* out, uint64_t* begin, uint32_t* count,
                   unsigned int* overflow, cudaStream_t s);
 void launch_write(const DevGrid& g, uint64_t g0, uint64_t g1, const uint64_t* off, uint64_t out_base,

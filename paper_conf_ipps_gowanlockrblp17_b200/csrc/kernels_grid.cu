@@ -26,6 +26,7 @@
 
 #include <algorithm>
 
+#include "cellkey.cuh"
 #include "internal.h"
 
 namespace hdb {
@@ -41,16 +42,6 @@ __device__ __forceinline__ unsigned long long ord_encode(double v) {
     return (b & 0x8000000000000000ull) ? ~b : (b | 0x8000000000000000ull);
 }
 
-template <typename T>
-struct V2;
-template <>
-struct V2<double> {
-    using type = double2;
-};
-template <>
-struct V2<float> {
-    using type = float2;
-};
 
 // One launch initialises the bbox reduction, the zeroed words of the build's misc
 // buffer (bb[4..nz): counters, occupancy sums, cost histogram) and the
@@ -249,6 +240,76 @@ __global__ void __launch_bounds__(RS_THREADS) k_radix_scatter(const K* __restric
     }
 }
 
+// ---------------------------------------------------------------- process-shard bands (8(e))
+// A process shard (torchrun rank r of R) takes a band of cell ROWS [Y_r, Y_{r+1}) of the
+// global grid as its queries; it needs the points of those rows plus k halo rows on either
+// side as candidates, and sorts only those (the grid build is no longer replicated).  The
+// bands balance a load estimate per row: the sum of squared cell occupancies (the work of
+// a cell's queries grows with its population), from a dense cell histogram.
+template <typename T>
+__global__ void __launch_bounds__(256) k_cell_hist(const typename V2<T>::type* __restrict__ xy, uint64_t n,
+                                                   KeyParams kp, uint32_t* __restrict__ cell_cnt) {
+    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
+        atomicAdd(&cell_cnt[cell_key<T, uint64_t>(xy[i], kp)], 1u);
+}
+
+// one warp per row: row_cnt[y] = sum of the row's cell counts, row_load[y] = sum of squares
+__global__ void __launch_bounds__(256) k_row_load(const uint32_t* __restrict__ cell_cnt, uint32_t nx, uint32_t ny,
+                                                  unsigned long long* __restrict__ row_cnt,
+                                                  unsigned long long* __restrict__ row_load) {
+    const int lane = threadIdx.x & 31;
+    for (uint64_t y = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5; y < ny;
+         y += ((uint64_t)gridDim.x * blockDim.x) >> 5) {
+        unsigned long long c = 0, l = 0;
+        for (uint32_t x = lane; x < nx; x += 32) {
+            const unsigned long long v = cell_cnt[y * nx + x];
+            c += v;
+            l += v * v;
+        }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) {
+            c += __shfl_xor_sync(FULL, c, o);
+            l += __shfl_xor_sync(FULL, l, o);
+        }
+        if (lane == 0) {
+            row_cnt[y] = c;
+            row_load[y] = l;
+        }
+    }
+}
+
+// grids too large for a dense cell histogram: row counts only (warp-aggregated atomics)
+template <typename T>
+__global__ void __launch_bounds__(256) k_row_count(const typename V2<T>::type* __restrict__ xy, uint64_t n,
+                                                   KeyParams kp, unsigned long long* __restrict__ row_cnt) {
+    const int lane = threadIdx.x & 31;
+    for (uint64_t i0 = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) - lane; i0 < n;
+         i0 += (uint64_t)gridDim.x * blockDim.x) {
+        const uint64_t i = i0 + lane;
+        uint64_t cx = 0, cy = ~0ull;
+        if (i < n) cell_xy<T>(xy[i], kp, cx, cy);
+        const unsigned peers = __match_any_sync(FULL, cy);
+        if (i < n && lane == __ffs(peers) - 1) atomicAdd(&row_cnt[cy], (unsigned long long)__popc(peers));
+    }
+}
+
+// the shard's query groups: the cells with keys in [key_lo, key_hi) -> groups
+// [gofs[c0], gofs[c1]) (out[0], out[1])
+__global__ void k_band_groups(const uint64_t* __restrict__ ckey, uint64_t nne, const uint32_t* __restrict__ gofs,
+                              uint64_t key_lo, uint64_t key_hi, unsigned long long* __restrict__ out) {
+    auto lb = [&](uint64_t k) {
+        uint64_t lo = 0, hi = nne;
+        while (lo < hi) {
+            const uint64_t mid = (lo + hi) >> 1;
+            if (ckey[mid] < k) lo = mid + 1;
+            else hi = mid;
+        }
+        return lo;
+    };
+    out[0] = gofs[lb(key_lo)];
+    out[1] = gofs[lb(key_hi)];
+}
+
 // ---------------------------------------------------------------- point sort (a2 + a3 + gather)
 // The points sorted by cell key with a stable LSD radix sort (8-bit digits)
 // whose passes carry the whole record (key, id, xy): the first pass reads the
@@ -264,22 +325,6 @@ constexpr int PS_THREADS = 256;
 constexpr int PS_WARPS = PS_THREADS / 32;
 constexpr int PS_ITEMS = 8;
 constexpr int PS_TILE = PS_THREADS * PS_ITEMS;   // 2048 records per CTA
-
-struct KeyParams {
-    double xmin, ymin, inv_w;
-    uint32_t nx, ny;
-};
-
-// a2: cell key of p -- FP64 cell arithmetic with explicitly rounded ops (no FMA),
-// cx = floor(fl(fl(x - xmin) * fl(1/w))) clamped to [0, nx-1] (reading R9)
-template <typename T, typename K>
-__device__ __forceinline__ K cell_key(const typename V2<T>::type p, const KeyParams& kp) {
-    const double tx = floor(__dmul_rn(__dsub_rn((double)p.x, kp.xmin), kp.inv_w));
-    const double ty = floor(__dmul_rn(__dsub_rn((double)p.y, kp.ymin), kp.inv_w));
-    const uint64_t cx = (uint64_t)fmin(fmax(tx, 0.0), (double)(kp.nx - 1));
-    const uint64_t cy = (uint64_t)fmin(fmax(ty, 0.0), (double)(kp.ny - 1));
-    return (K)(cy * kp.nx + cx);
-}
 
 template <typename T, typename K, bool FROM_POINTS>
 __global__ void __launch_bounds__(PS_THREADS) k_ps_hist(const typename V2<T>::type* __restrict__ xy,
@@ -320,7 +365,7 @@ __global__ void __launch_bounds__(PS_THREADS) k_ps_scatter(const typename V2<T>:
                                                            float4* __restrict__ xp, double ox, double oy, uint64_t n,
                                                            int shift, const uint32_t* __restrict__ hscan,
                                                            uint32_t nblocks, unsigned int* __restrict__ counters,
-                                                           uint32_t n_counters) {
+                                                           uint32_t n_counters, const uint32_t* __restrict__ gid) {
     using P2 = typename V2<T>::type;
     extern __shared__ __align__(16) unsigned char ps_smem[];
     P2* sxy = (P2*)ps_smem;
@@ -361,7 +406,7 @@ __global__ void __launch_bounds__(PS_THREADS) k_ps_scatter(const typename V2<T>:
         pt[r] = valid ? xyin[idx] : P2{0, 0};
         if (FIRST) {
             key[r] = valid ? cell_key<T, K>(pt[r], kp) : (K)0;
-            val[r] = (uint32_t)idx;
+            val[r] = gid ? (valid ? gid[idx] : 0u) : (uint32_t)idx;   // id = input row (or its global id)
         } else {
             key[r] = valid ? kin[idx] : (K)0;
             val[r] = valid ? vin[idx] : 0u;
@@ -798,7 +843,8 @@ struct PointSort {
     template <bool F, bool L>
     static void scatter(const P2* xyin, const K* kin, const uint32_t* vin, const KeyParams& kp, K* kout,
                         uint32_t* vout, P2* xyout, float4* xp, double ox, double oy, uint64_t n, int shift,
-                        const uint32_t* hscan, uint32_t nb, unsigned int* counters, uint32_t nc, cudaStream_t s) {
+                        const uint32_t* hscan, uint32_t nb, unsigned int* counters, uint32_t nc, const uint32_t* gid,
+                        cudaStream_t s) {
         static bool attr = [] {
             cudaFuncSetAttribute(k_ps_scatter<T, K, F, L>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                  (int)ps_smem_bytes<T, K>());
@@ -806,12 +852,12 @@ struct PointSort {
         }();
         (void)attr;
         k_ps_scatter<T, K, F, L><<<nb, PS_THREADS, ps_smem_bytes<T, K>(), s>>>(
-            xyin, kin, vin, kp, kout, vout, xyout, xp, ox, oy, n, shift, hscan, nb, counters, nc);
+            xyin, kin, vin, kp, kout, vout, xyout, xp, ox, oy, n, shift, hscan, nb, counters, nc, gid);
         ++g_kernel_launches;
     }
     static void run(const void* xy_in, uint64_t n, const KeyParams& kp, int bits, void* keys_out, uint32_t* ids_out,
                     void* xy_s, float4* xp, double ox, double oy, unsigned int* counters, uint32_t nc, void* temp,
-                    cudaStream_t s) {
+                    const uint32_t* gid, cudaStream_t s) {
         const uint32_t nb = (uint32_t)((n + PS_TILE - 1) / PS_TILE);
         const int passes = std::max(1, (bits + RS_BITS - 1) / RS_BITS);
         const uint64_t m = (uint64_t)nb * RS_BINS;
@@ -849,13 +895,13 @@ struct PointSort {
             ++g_kernel_launches;
             scan_u32_to_u32(hist, hscan, m, stemp, s);
             if (first && last)
-                scatter<true, true>(xi, ki, vi, kp, ko, vo, xo, xp, ox, oy, n, shift, hscan, nb, counters, nc, s);
+                scatter<true, true>(xi, ki, vi, kp, ko, vo, xo, xp, ox, oy, n, shift, hscan, nb, counters, nc, gid, s);
             else if (first)
-                scatter<true, false>(xi, ki, vi, kp, ko, vo, xo, xp, ox, oy, n, shift, hscan, nb, counters, nc, s);
+                scatter<true, false>(xi, ki, vi, kp, ko, vo, xo, xp, ox, oy, n, shift, hscan, nb, counters, nc, gid, s);
             else if (last)
-                scatter<false, true>(xi, ki, vi, kp, ko, vo, xo, xp, ox, oy, n, shift, hscan, nb, counters, nc, s);
+                scatter<false, true>(xi, ki, vi, kp, ko, vo, xo, xp, ox, oy, n, shift, hscan, nb, counters, nc, gid, s);
             else
-                scatter<false, false>(xi, ki, vi, kp, ko, vo, xo, xp, ox, oy, n, shift, hscan, nb, counters, nc, s);
+                scatter<false, false>(xi, ki, vi, kp, ko, vo, xo, xp, ox, oy, n, shift, hscan, nb, counters, nc, gid, s);
         }
     }
     static size_t temp_bytes(uint64_t n, int bits) {
@@ -866,6 +912,29 @@ struct PointSort {
     }
 };
 
+void row_loads(const void* xy, uint64_t n, hdb_dtype dt, double xmin, double ymin, double inv_w, uint32_t nx,
+               uint32_t ny, uint32_t* cell_cnt, unsigned long long* row_cnt, unsigned long long* row_load,
+               cudaStream_t s) {
+    const KeyParams kp{xmin, ymin, inv_w, nx, ny};
+    if (n == 0) return;
+    if (cell_cnt) {
+        if (dt == HDB_F64) k_cell_hist<double><<<grid_for(n), 256, 0, s>>>((const double2*)xy, n, kp, cell_cnt);
+        else k_cell_hist<float><<<grid_for(n), 256, 0, s>>>((const float2*)xy, n, kp, cell_cnt);
+        k_row_load<<<grid_for(32ull * ny), 256, 0, s>>>(cell_cnt, nx, ny, row_cnt, row_load);
+        g_kernel_launches += 2;
+    } else {
+        if (dt == HDB_F64) k_row_count<double><<<grid_for(n), 256, 0, s>>>((const double2*)xy, n, kp, row_cnt);
+        else k_row_count<float><<<grid_for(n), 256, 0, s>>>((const float2*)xy, n, kp, row_cnt);
+        ++g_kernel_launches;
+    }
+}
+
+void launch_band_groups(const uint64_t* ckey, uint64_t nne, const uint32_t* gofs, uint64_t key_lo, uint64_t key_hi,
+                        unsigned long long* out, cudaStream_t s) {
+    k_band_groups<<<1, 1, 0, s>>>(ckey, nne, gofs, key_lo, key_hi, out);
+    ++g_kernel_launches;
+}
+
 size_t point_sort_temp_bytes(uint64_t n, hdb_dtype dt, int key_bytes, int bits) {
     if (dt == HDB_F64)
         return key_bytes == 4 ? PointSort<double, uint32_t>::temp_bytes(n, bits)
@@ -875,23 +944,24 @@ size_t point_sort_temp_bytes(uint64_t n, hdb_dtype dt, int key_bytes, int bits) 
 
 void sort_points(const void* xy_in, uint64_t n, hdb_dtype dt, double xmin, double ymin, double inv_w, uint32_t nx,
                  uint32_t ny, int key_bytes, int bits, void* keys_out, uint32_t* ids_out, void* xy_s, float4* xp,
-                 double ox, double oy, unsigned int* counters, uint32_t n_counters, void* temp, cudaStream_t s) {
+                 double ox, double oy, unsigned int* counters, uint32_t n_counters, void* temp, cudaStream_t s,
+                 const uint32_t* gid) {
     if (n == 0) return;
     const KeyParams kp{xmin, ymin, inv_w, nx, ny};
     if (dt == HDB_F64) {
         if (key_bytes == 4)
             PointSort<double, uint32_t>::run(xy_in, n, kp, bits, keys_out, ids_out, xy_s, xp, ox, oy, counters,
-                                             n_counters, temp, s);
+                                             n_counters, temp, gid, s);
         else
             PointSort<double, uint64_t>::run(xy_in, n, kp, bits, keys_out, ids_out, xy_s, xp, ox, oy, counters,
-                                             n_counters, temp, s);
+                                             n_counters, temp, gid, s);
     } else {
         if (key_bytes == 4)
             PointSort<float, uint32_t>::run(xy_in, n, kp, bits, keys_out, ids_out, xy_s, xp, 0, 0, counters,
-                                            n_counters, temp, s);
+                                            n_counters, temp, gid, s);
         else
             PointSort<float, uint64_t>::run(xy_in, n, kp, bits, keys_out, ids_out, xy_s, xp, 0, 0, counters,
-                                            n_counters, temp, s);
+                                            n_counters, temp, gid, s);
     }
 }
 

@@ -6,6 +6,7 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include "cellkey.cuh"
 #include "internal.h"
 
 namespace hdb {
@@ -219,6 +220,46 @@ struct RleScan {
         *nne_out = t;
     }
 };
+
+// process-shard band: the points whose cell row is in [ylo, yhi), in input
+// order, with their input rows (stream compaction as a scan of the membership flags)
+template <typename T>
+struct BandSelect {
+    using P2 = typename V2<T>::type;
+    const P2* __restrict__ xy;
+    KeyParams kp;
+    uint64_t ylo, yhi;
+    P2* __restrict__ out;
+    uint32_t* __restrict__ gid;
+    uint32_t* __restrict__ n_out;
+    __device__ __forceinline__ bool in(uint64_t i) const {
+        uint64_t cx, cy;
+        cell_xy<T>(xy[i], kp, cx, cy);
+        return cy >= ylo && cy < yhi;
+    }
+    __device__ __forceinline__ uint32_t load(uint64_t i) const { return in(i) ? 1u : 0u; }
+    __device__ __forceinline__ void store(uint64_t i, uint32_t e) const {
+        if (in(i)) {
+            out[e] = xy[i];
+            gid[e] = (uint32_t)i;
+        }
+    }
+    __device__ __forceinline__ void total(uint64_t, uint32_t t) const { *n_out = t; }
+};
+
+void band_select(const void* xy, uint64_t n, hdb_dtype dt, double xmin, double ymin, double inv_w, uint32_t nx,
+                 uint32_t ny, uint64_t ylo, uint64_t yhi, void* out, uint32_t* gid, uint32_t* n_out, void* temp,
+                 cudaStream_t s) {
+    if (n == 0) {
+        cudaMemsetAsync(n_out, 0, sizeof(uint32_t), s);
+        return;
+    }
+    const KeyParams kp{xmin, ymin, inv_w, nx, ny};
+    if (dt == HDB_F64)
+        scan_impl<uint32_t>(BandSelect<double>{(const double2*)xy, kp, ylo, yhi, (double2*)out, gid, n_out}, n, temp, s);
+    else
+        scan_impl<uint32_t>(BandSelect<float>{(const float2*)xy, kp, ylo, yhi, (float2*)out, gid, n_out}, n, temp, s);
+}
 
 void cell_rle(const void* keys_sorted, int key_bytes, uint64_t n, uint64_t* ckey, uint32_t* cstart, uint32_t* nne_out,
               void* temp, cudaStream_t s) {

@@ -1463,24 +1463,25 @@ void launch_fused_mode(const SArgs& a, uint64_t g0, uint64_t g1, unsigned int* c
                                                  pair_ctr, cap, out, begin, count, overflow);
 }
 
-void launch_fused(const DevGrid& g, uint32_t* cnt, unsigned long long* tests, uint2* masks,
+void launch_fused(const DevGrid& g, uint64_t g0, uint64_t g1, uint32_t* cnt, unsigned long long* tests, uint2* masks,
                   unsigned long long* pair_ctr, uint64_t cap, uint32_t* out, uint64_t* begin, uint32_t* count,
                   unsigned int* overflow, cudaStream_t s) {
-    if (g.n_groups == 0) return;
+    if (g1 <= g0) return;
     SArgs a = args_of(g);
-    if (use_cost_order(g)) a.ord = g.ord;   // heavy groups first: C2 eps 0.45 2.50 -> 2.10 ms (the schedule's tail)
+    // heavy groups first (whole ranges only: ord lists every group): C2 eps 0.45 2.50 -> 2.10 ms
+    if (g0 == 0 && g1 == g.n_groups && use_cost_order(g)) a.ord = g.ord;
     unsigned int* ctr = g.counters;
     cudaMemsetAsync(ctr, 0, sizeof(unsigned int), s);
     const int mode = g.dtype == HDB_F32 ? kF32 : (g.filter_l ? kF64Filter : kF64Exact);
     if (mode == kF64Filter)
-        launch_fused_mode<kF64Filter>(a, 0, g.n_groups, ctr, cnt, tests, masks, g.moff, pair_ctr, cap, out, begin,
-                                      count, overflow, s);
+        launch_fused_mode<kF64Filter>(a, g0, g1, ctr, cnt, tests, masks, g.moff, pair_ctr, cap, out, begin, count,
+                                      overflow, s);
     else if (mode == kF64Exact)
-        launch_fused_mode<kF64Exact>(a, 0, g.n_groups, ctr, cnt, tests, masks, g.moff, pair_ctr, cap, out, begin,
-                                     count, overflow, s);
+        launch_fused_mode<kF64Exact>(a, g0, g1, ctr, cnt, tests, masks, g.moff, pair_ctr, cap, out, begin, count,
+                                     overflow, s);
     else
-        launch_fused_mode<kF32>(a, 0, g.n_groups, ctr, cnt, tests, masks, g.moff, pair_ctr, cap, out, begin, count,
-                                overflow, s);
+        launch_fused_mode<kF32>(a, g0, g1, ctr, cnt, tests, masks, g.moff, pair_ctr, cap, out, begin, count, overflow,
+                                s);
     ++g_kernel_launches;
 }
 

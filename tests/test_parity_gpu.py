@@ -691,6 +691,40 @@ def test_sparse_dense_hybrid(torch_cuda):
     assert saw_mixed
 
 
+@pytest.mark.parametrize("R", [2, 4, 7])
+def test_process_shard_bands_assemble_to_the_oracle_table(torch_cuda, R):
+    """Process shards build only their band of cell rows plus the k halo rows
+    (DESIGN.md sec. 7): each shard's grid holds fewer points than
+    the input, the bands are consecutive ranges of the global cell-sorted
+    order, and the shards' tables (single pass on device, two passes into host
+    memory) assemble into exactly the oracle's table -- also with a skewed
+    load (C5's dense square) and a cell split."""
+    from paper_conf_ipps_gowanlockrblp17_b200 import dist as hdist
+    xy = datagen.dense_skew(40_000, seed=21)
+    n = xy.shape[0]
+    for eps, split in ((3.0, 0), (5.0, 3)):
+        for device in (True, False):
+            parts, ranges = [], []
+            for r in range(R):
+                ctx = _ctx(shard_rank=r, shard_count=R, cell_split=split)
+                try:
+                    g = hdb.hdb_grid_build(ctx, xy, eps)
+                    gv = hdb.hdb_grid_view_get(g)
+                    assert gv.n < n
+                    t = (hdb.hdb_neighbor_table_device if device else hdb.hdb_neighbor_table)(ctx, g)
+                    hdb.hdb_grid_free(g)
+                    v = hdb.hdb_table_view_get(t)
+                    ranges.append((v.first_query, v.end_query))
+                    parts.append(hdb.hdb_table_copy_to_host(t))
+                    hdb.hdb_table_free(t)
+                finally:
+                    hdb.hdb_ctx_destroy(ctx)
+            assert ranges[0][0] == 0 and ranges[-1][1] == n
+            assert all(ranges[i][1] == ranges[i + 1][0] for i in range(R - 1))
+            b, c, v = hdist.assemble(parts, n)
+            assert_table_equal(xy, eps, b, c, v)
+
+
 def test_sparse_batches_and_shards(torch_cuda):
     """The sparse queries of a group range follow the range: many small batches
     (host table) and process shards give the oracle's table."""
