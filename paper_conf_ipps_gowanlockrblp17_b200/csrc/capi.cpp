@@ -7,6 +7,7 @@
 #include <condition_variable>
 #include <cstring>
 #include <deque>
+#include <chrono>
 #include <thread>
 
 #include "internal.h"
@@ -496,6 +497,15 @@ hdb_status hdb_sweep(hdb_ctx* c, const void* xy, uint64_t n, hdb_dtype dt, const
     hdb_status prod_st = HDB_OK;
     std::string prod_msg;
     int dev0 = c->dev[0].device;
+    // HDB_TIMELINE=1: host timeline of the pipeline (ms from the call's start) as one JSON
+    // line on stderr -- the overlap of T(eps_{i+1})'s build with T(eps_i)'s clustering
+    const char* tle = getenv("HDB_TIMELINE");
+    const bool tl = tle && *tle == '1';
+    const auto t_start = std::chrono::steady_clock::now();
+    auto now_ms = [&] {
+        return std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_start).count();
+    };
+    std::vector<double> tb0(n_eps, 0), tb1(n_eps, 0), tc0(n_eps, 0), tc1(n_eps, 0);
     std::thread producer([&] {
         cudaSetDevice(dev0);
         for (uint32_t i = 0; i < n_eps; ++i) {
@@ -508,9 +518,11 @@ hdb_status hdb_sweep(hdb_ctx* c, const void* xy, uint64_t n, hdb_dtype dt, const
             hdb_grid* g = nullptr;
             hdb_table* t = nullptr;
             try {
+                tb0[i] = now_ms();
                 grid_build(c, xy, n, dt, eps[i], &g);
                 neighbor_table(c, g, false, &t);
                 grid_free(g);
+                tb1[i] = now_ms();
             } catch (const hdb::Error& e) {
                 if (g) grid_free(g);
                 std::lock_guard<std::mutex> l(m);
@@ -551,6 +563,7 @@ hdb_status hdb_sweep(hdb_ctx* c, const void* xy, uint64_t n, hdb_dtype dt, const
         }
         const uint32_t i = item.first;
         hdb_table* t = item.second;
+        tc0[i] = now_ms();
         std::vector<std::thread> th;
         std::vector<hdb_status> st(n_minpts, HDB_OK);
         for (uint32_t j = 0; j < n_minpts; ++j)
@@ -564,6 +577,7 @@ hdb_status hdb_sweep(hdb_ctx* c, const void* xy, uint64_t n, hdb_dtype dt, const
                 if (n_clusters) n_clusters[(uint64_t)i * n_minpts + j] = k;
             });
         for (auto& x : th) x.join();
+        tc1[i] = now_ms();
         table_free(t);
         for (auto s : st)
             if (s != HDB_OK) {
@@ -588,6 +602,17 @@ hdb_status hdb_sweep(hdb_ctx* c, const void* xy, uint64_t n, hdb_dtype dt, const
             table_free(q.front().second);
             q.pop_front();
         }
+    }
+    if (tl) {
+        std::string js = "{\"timeline\": \"hdb_sweep\", \"total_ms\": " + std::to_string(now_ms()) + ", \"eps\": [";
+        for (uint32_t i = 0; i < n_eps; ++i) {
+            char b[256];
+            snprintf(b, sizeof b, "%s{\"eps\": %g, \"build\": [%.3f, %.3f], \"dbscan\": [%.3f, %.3f]}", i ? ", " : "",
+                     eps[i], tb0[i], tb1[i], tc0[i], tc1[i]);
+            js += b;
+        }
+        js += "]}";
+        fprintf(stderr, "%s\n", js.c_str());
     }
     if (prod_st != HDB_OK) {
         set_error("%s", prod_msg.c_str());

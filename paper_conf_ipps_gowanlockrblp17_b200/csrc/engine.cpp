@@ -128,6 +128,17 @@ struct Trace {
     }
 };
 
+// HDB_TIMELINE=1: the batched host-table write (a8 + a9) prints its GPU timeline as
+// one JSON line to stderr -- per batch, the write kernel's and the D2H copy's start / end
+// (CUDA events, ms from the first batch) and stream -- the overlap evidence of P:796-812
+bool timeline_on() {
+    static const bool on = [] {
+        const char* e = getenv("HDB_TIMELINE");
+        return e && *e == '1';
+    }();
+    return on;
+}
+
 struct DeviceGuard {
     int prev = -1;
     explicit DeviceGuard(int d) {
@@ -334,6 +345,8 @@ uint32_t split_from_occ(const unsigned long long* h, uint64_t n, const DevGrid& 
     return k;
 }
 
+constexpr double kPointPairs = 117.0;   // a query's fixed work in pair-equivalents (band weights)
+
 // HDB_BANDS=0 turns the process-shard bands off (every rank then builds the full grid)
 bool bands_enabled() {
     static const bool on = [] {
@@ -471,21 +484,31 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
     if (R_proc > 1 && ctx->dev.size() == 1 && n > 0 && g.ny <= (1u << 22) && bands_enabled()) {
         const uint32_t rank = (uint32_t)ctx->opts.shard_rank;
         const bool dense = g.n_cells <= std::max<uint64_t>(8 * n, 1ull << 22);
-        DBuf rc(8ull * g.ny, s), rl(8ull * g.ny, s), cc;
+        DBuf rc(8ull * g.ny, s), rl(8ull * g.ny, s), cc, rowid(4 * n, s);
         HDB_CUDA(cudaMemsetAsync(rc.p, 0, 8ull * g.ny, s));
         HDB_CUDA(cudaMemsetAsync(rl.p, 0, 8ull * g.ny, s));
         if (dense) {
             cc = DBuf(4 * g.n_cells, s);
             HDB_CUDA(cudaMemsetAsync(cc.p, 0, 4 * g.n_cells, s));
         }
-        row_loads(xin, n, dt, g.xmin, g.ymin, g.inv_w, g.nx, g.ny, cc.as<uint32_t>(), rc.as<unsigned long long>(),
-                  rl.as<unsigned long long>(), s);
+        band_rows_hist(xin, n, dt, g.xmin, g.ymin, g.inv_w, g.nx, g.ny, rowid.as<uint32_t>(), cc.as<uint32_t>(),
+                       rc.as<unsigned long long>(), rl.as<unsigned long long>(), s);
         HDB_LAUNCH_CHECK();
+        cc.reset();
         std::vector<uint64_t> hrc(g.ny), hrl(g.ny);
         HDB_CUDA(cudaMemcpyAsync(hrc.data(), rc.p, 8ull * g.ny, cudaMemcpyDeviceToHost, s));
         HDB_CUDA(cudaMemcpyAsync(hrl.data(), rl.p, 8ull * g.ny, cudaMemcpyDeviceToHost, s));
         HDB_CUDA(cudaStreamSynchronize(s));
-        const std::vector<uint64_t>& load = dense ? hrl : hrc;
+        // row weight = estimated pairs + a per-point cost in pair-equivalents.  A cell of m
+        // points (width eps/k, locally uniform density) has queries with ~pi k^2 m neighbours
+        // each, so a row's pairs ~ pi k^2 sum m^2; and a query costs ~117 pairs' worth of time
+        // beside its pairs (least squares over the per-rank steps of C5 at R = 4 and 8:
+        // 1.49 ms per rank + 0.187 ms per M points + 0.0016 ms per M pairs -- the grid build
+        // and the per-group set-up are per point)
+        std::vector<uint64_t> load(g.ny);
+        const double kk = 3.14159265358979 * (double)g.split * (double)g.split / 256.0;
+        for (uint64_t y = 0; y < g.ny; ++y)
+            load[y] = (uint64_t)((dense ? kk * (double)hrl[y] : 0.0) + kPointPairs * (double)hrc[y]);
         band_rows(load, R_proc, rank, band_y0, band_y1);
         const uint64_t ylo = band_y0 >= g.split ? band_y0 - g.split : 0;
         const uint64_t yhi = std::min<uint64_t>(g.ny, band_y1 + g.split);
@@ -498,7 +521,7 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
         band_pts = DBuf(esz * (nb ? nb : 1), s);
         band_gid = DBuf(4 * (nb ? nb : 1), s);
         DBuf dnb(8, s), btemp(scan_temp_bytes(n + 1), s);
-        band_select(xin, n, dt, g.xmin, g.ymin, g.inv_w, g.nx, g.ny, ylo, yhi, band_pts.p, band_gid.as<uint32_t>(),
+        band_select(xin, rowid.as<uint32_t>(), n, dt, ylo, yhi, band_pts.p, band_gid.as<uint32_t>(),
                     dnb.as<uint32_t>(), btemp.p, s);
         HDB_LAUNCH_CHECK();
         xin = band_pts.p;
@@ -1066,6 +1089,8 @@ void write_phase_host(hdb_ctx* ctx, DevCtx& dc, const DevGrid& g, ShardState& st
     Event ready;
     HDB_CUDA(cudaEventRecord(ready.e, s));
     std::vector<Event> evs(2 * nb);
+    const bool tl = timeline_on();
+    std::vector<Event> cev(tl ? nb : 0);   // end of each batch's D2H copy (timeline only)
     for (uint64_t b = 0; b < nb; ++b) {
         const uint32_t si = (uint32_t)(b % S);
         cudaStream_t ss = dc.streams[si];
@@ -1079,10 +1104,26 @@ void write_phase_host(hdb_ctx* ctx, DevCtx& dc, const DevGrid& g, ShardState& st
         if (pairs_b)
             HDB_CUDA(cudaMemcpyAsync(h_nbrs + st.base + hp[b], dc.batch_buf[si], 4 * pairs_b, cudaMemcpyDeviceToHost,
                                      ss));
+        if (tl) HDB_CUDA(cudaEventRecord(cev[b].e, ss));
         st.d2h += 4 * pairs_b;
     }
     for (uint32_t i = 0; i < S; ++i) HDB_CUDA(cudaStreamSynchronize(dc.streams[i]));
     for (uint64_t b = 0; b < nb; ++b) st.ms_write += elapsed(evs[2 * b], evs[2 * b + 1]);
+    if (tl) {
+        std::string js = "{\"timeline\": \"host_table_write\", \"device\": " + std::to_string(dc.device) +
+                         ", \"batches\": [";
+        for (uint64_t b = 0; b < nb; ++b) {
+            char buf[256];
+            snprintf(buf, sizeof buf,
+                     "%s{\"b\": %llu, \"stream\": %u, \"pairs\": %llu, \"write\": [%.4f, %.4f], \"d2h\": [%.4f, %.4f]}",
+                     b ? ", " : "", (unsigned long long)b, (unsigned)(b % S), (unsigned long long)(hp[b + 1] - hp[b]),
+                     elapsed(evs[0], evs[2 * b]), elapsed(evs[0], evs[2 * b + 1]), elapsed(evs[0], evs[2 * b + 1]),
+                     elapsed(evs[0], cev[b]));
+            js += buf;
+        }
+        js += "]}";
+        fprintf(stderr, "%s\n", js.c_str());
+    }
     st.write_launches += (uint32_t)nb;
     st.n_batches = nb;
     st.max_batch = maxb;

@@ -113,16 +113,16 @@ int radix_sort_pairs(void* k0, uint32_t* v0, void* k1, uint32_t* v1, int key_byt
 // records, keys computed by the first pass from the input points): keys_out[n] sorted keys,
 // ids_out[n + 2] A (padded), xy_s[n + 2] sorted points (padded), xp the f32 filter copy
 // (padded), counters zeroed.  temp: point_sort_temp_bytes(n, dt, key_bytes, bits)
-// process-shard bands: per cell row, the point count and a load estimate
-// (sum of squared cell counts; cell_cnt = a zeroed nx*ny histogram, or null: counts only,
-// row_load untouched); the band's points (rows [ylo, yhi)) with their input rows;
-// the band's query groups (cells with keys in [key_lo, key_hi)) -> out[0..1]
-void row_loads(const void* xy, uint64_t n, hdb_dtype dt, double xmin, double ymin, double inv_w, uint32_t nx,
-               uint32_t ny, uint32_t* cell_cnt, unsigned long long* row_cnt, unsigned long long* row_load,
-               cudaStream_t s);
-void band_select(const void* xy, uint64_t n, hdb_dtype dt, double xmin, double ymin, double inv_w, uint32_t nx,
-                 uint32_t ny, uint64_t ylo, uint64_t yhi, void* out, uint32_t* gid, uint32_t* n_out, void* temp,
-                 cudaStream_t s);
+// process-shard bands: one pass over the input -> every point's cell row
+// (rowid[n]), exact row counts row_cnt[ny] (zeroed by the caller) and, with cell_cnt (a
+// zeroed nx*ny histogram of a 1/16 sample), row_load[ny] = the estimated sum of squared cell
+// counts x 256; the band's points (rowid in [ylo, yhi)) with their input rows; the band's
+// query groups (cells with keys in [key_lo, key_hi)) -> out[0..1]
+void band_rows_hist(const void* xy, uint64_t n, hdb_dtype dt, double xmin, double ymin, double inv_w, uint32_t nx,
+                    uint32_t ny, uint32_t* rowid, uint32_t* cell_cnt, unsigned long long* row_cnt,
+                    unsigned long long* row_load, cudaStream_t s);
+void band_select(const void* xy, const uint32_t* rowid, uint64_t n, hdb_dtype dt, uint64_t ylo, uint64_t yhi, void* out,
+                 uint32_t* gid, uint32_t* n_out, void* temp, cudaStream_t s);
 void launch_band_groups(const uint64_t* ckey, uint64_t nne, const uint32_t* gofs, uint64_t key_lo, uint64_t key_hi,
                         unsigned long long* out, cudaStream_t s);
 size_t point_sort_temp_bytes(uint64_t n, hdb_dtype dt, int key_bytes, int bits);

@@ -68,19 +68,28 @@ __global__ void __launch_bounds__(256) k_bbox(const typename V2<T>::type* __rest
                                               unsigned long long* bb, unsigned int* bad) {
     double xmn = INFINITY, ymn = INFINITY, xmx = -INFINITY, ymx = -INFINITY;
     unsigned nb = 0;
-    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n;
-         i += (uint64_t)gridDim.x * blockDim.x) {
-        auto p = xy[i];
-        double x = (double)p.x, y = (double)p.y;
+    auto take = [&](typename V2<T>::type p) {
+        const double x = (double)p.x, y = (double)p.y;
         if (!isfinite(x) || !isfinite(y)) {
             ++nb;
-            continue;
+            return;
         }
         xmn = fmin(xmn, x);
         ymn = fmin(ymn, y);
         xmx = fmax(xmx, x);
         ymx = fmax(ymx, y);
+    };
+    // four independent loads in flight per thread (the reduction streams the whole input)
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+    for (; i + 3 * stride < n; i += 4 * stride) {
+        const auto p0 = xy[i], p1 = xy[i + stride], p2 = xy[i + 2 * stride], p3 = xy[i + 3 * stride];
+        take(p0);
+        take(p1);
+        take(p2);
+        take(p3);
     }
+    for (; i < n; i += stride) take(xy[i]);
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) {
         xmn = fmin(xmn, __shfl_xor_sync(FULL, xmn, o));
@@ -246,50 +255,55 @@ __global__ void __launch_bounds__(RS_THREADS) k_radix_scatter(const K* __restric
 // side as candidates, and sorts only those (the grid build is no longer replicated).  The
 // bands balance a load estimate per row: the sum of squared cell occupancies (the work of
 // a cell's queries grows with its population), from a dense cell histogram.
+// One pass over the input: every point's cell row -> rowid[i] (read again by the band
+// selection instead of the coordinates), exact row counts (per-block shared histogram
+// when the rows fit, else global atomics), and, for every kRowSample-th point, its cell
+// in the sampled cell histogram (the load estimate needs only a sample; one atomic per
+// point into tens of MB of counters cost 0.36 ms at C5)
+constexpr uint32_t kRowSample = 16;
+constexpr uint32_t kRowSmem = 8192;   // rows counted in shared memory (32 KB)
 template <typename T>
-__global__ void __launch_bounds__(256) k_cell_hist(const typename V2<T>::type* __restrict__ xy, uint64_t n,
-                                                   KeyParams kp, uint32_t* __restrict__ cell_cnt) {
-    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
-        atomicAdd(&cell_cnt[cell_key<T, uint64_t>(xy[i], kp)], 1u);
-}
-
-// one warp per row: row_cnt[y] = sum of the row's cell counts, row_load[y] = sum of squares
-__global__ void __launch_bounds__(256) k_row_load(const uint32_t* __restrict__ cell_cnt, uint32_t nx, uint32_t ny,
-                                                  unsigned long long* __restrict__ row_cnt,
-                                                  unsigned long long* __restrict__ row_load) {
-    const int lane = threadIdx.x & 31;
-    for (uint64_t y = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5; y < ny;
-         y += ((uint64_t)gridDim.x * blockDim.x) >> 5) {
-        unsigned long long c = 0, l = 0;
-        for (uint32_t x = lane; x < nx; x += 32) {
-            const unsigned long long v = cell_cnt[y * nx + x];
-            c += v;
-            l += v * v;
-        }
-#pragma unroll
-        for (int o = 16; o > 0; o >>= 1) {
-            c += __shfl_xor_sync(FULL, c, o);
-            l += __shfl_xor_sync(FULL, l, o);
-        }
-        if (lane == 0) {
-            row_cnt[y] = c;
-            row_load[y] = l;
-        }
+__global__ void __launch_bounds__(256) k_band_hist(const typename V2<T>::type* __restrict__ xy, uint64_t n,
+                                                   KeyParams kp, uint32_t* __restrict__ rowid,
+                                                   unsigned long long* __restrict__ row_cnt,
+                                                   uint32_t* __restrict__ cell_cnt) {
+    __shared__ uint32_t rh[kRowSmem];
+    const bool smem = kp.ny <= kRowSmem;
+    if (smem)
+        for (uint32_t y = threadIdx.x; y < kp.ny; y += blockDim.x) rh[y] = 0;
+    __syncthreads();
+    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+        uint64_t cx, cy;
+        cell_xy<T>(xy[i], kp, cx, cy);
+        rowid[i] = (uint32_t)cy;
+        if (smem) atomicAdd(&rh[cy], 1u);
+        else atomicAdd(&row_cnt[cy], 1ull);
+        if (cell_cnt && i % kRowSample == 0) atomicAdd(&cell_cnt[cy * kp.nx + cx], 1u);
+    }
+    if (smem) {
+        __syncthreads();
+        for (uint32_t y = threadIdx.x; y < kp.ny; y += blockDim.x)
+            if (rh[y]) atomicAdd(&row_cnt[y], (unsigned long long)rh[y]);
     }
 }
 
-// grids too large for a dense cell histogram: row counts only (warp-aggregated atomics)
-template <typename T>
-__global__ void __launch_bounds__(256) k_row_count(const typename V2<T>::type* __restrict__ xy, uint64_t n,
-                                                   KeyParams kp, unsigned long long* __restrict__ row_cnt) {
+// one warp per row: row_load[y] = sum of the sampled cell counts' squares, with the
+// sampling bias removed: E[s^2] = f^2 m^2 + f (1 - f) m for a cell of m points, so
+// (s^2 - (1 - f) s) / f^2 estimates m^2 (scaled by 2^8 to keep fractions in integers)
+__global__ void __launch_bounds__(256) k_row_load(const uint32_t* __restrict__ cell_cnt, uint32_t nx, uint32_t ny,
+                                                  unsigned long long* __restrict__ row_load) {
     const int lane = threadIdx.x & 31;
-    for (uint64_t i0 = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) - lane; i0 < n;
-         i0 += (uint64_t)gridDim.x * blockDim.x) {
-        const uint64_t i = i0 + lane;
-        uint64_t cx = 0, cy = ~0ull;
-        if (i < n) cell_xy<T>(xy[i], kp, cx, cy);
-        const unsigned peers = __match_any_sync(FULL, cy);
-        if (i < n && lane == __ffs(peers) - 1) atomicAdd(&row_cnt[cy], (unsigned long long)__popc(peers));
+    const double f = 1.0 / kRowSample;
+    for (uint64_t y = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5; y < ny;
+         y += ((uint64_t)gridDim.x * blockDim.x) >> 5) {
+        double l = 0;
+        for (uint32_t x = lane; x < nx; x += 32) {
+            const double v = cell_cnt[y * nx + x];
+            l += fmax(v * v - (1.0 - f) * v, 0.0) / (f * f);
+        }
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) l += __shfl_xor_sync(FULL, l, o);
+        if (lane == 0) row_load[y] = (unsigned long long)(l * 256.0);
     }
 }
 
@@ -912,19 +926,18 @@ struct PointSort {
     }
 };
 
-void row_loads(const void* xy, uint64_t n, hdb_dtype dt, double xmin, double ymin, double inv_w, uint32_t nx,
-               uint32_t ny, uint32_t* cell_cnt, unsigned long long* row_cnt, unsigned long long* row_load,
-               cudaStream_t s) {
+void band_rows_hist(const void* xy, uint64_t n, hdb_dtype dt, double xmin, double ymin, double inv_w, uint32_t nx,
+                    uint32_t ny, uint32_t* rowid, uint32_t* cell_cnt, unsigned long long* row_cnt,
+                    unsigned long long* row_load, cudaStream_t s) {
     const KeyParams kp{xmin, ymin, inv_w, nx, ny};
     if (n == 0) return;
+    if (dt == HDB_F64)
+        k_band_hist<double><<<grid_for(n, 256, 148 * 4), 256, 0, s>>>((const double2*)xy, n, kp, rowid, row_cnt, cell_cnt);
+    else
+        k_band_hist<float><<<grid_for(n, 256, 148 * 4), 256, 0, s>>>((const float2*)xy, n, kp, rowid, row_cnt, cell_cnt);
+    ++g_kernel_launches;
     if (cell_cnt) {
-        if (dt == HDB_F64) k_cell_hist<double><<<grid_for(n), 256, 0, s>>>((const double2*)xy, n, kp, cell_cnt);
-        else k_cell_hist<float><<<grid_for(n), 256, 0, s>>>((const float2*)xy, n, kp, cell_cnt);
-        k_row_load<<<grid_for(32ull * ny), 256, 0, s>>>(cell_cnt, nx, ny, row_cnt, row_load);
-        g_kernel_launches += 2;
-    } else {
-        if (dt == HDB_F64) k_row_count<double><<<grid_for(n), 256, 0, s>>>((const double2*)xy, n, kp, row_cnt);
-        else k_row_count<float><<<grid_for(n), 256, 0, s>>>((const float2*)xy, n, kp, row_cnt);
+        k_row_load<<<grid_for(32ull * ny), 256, 0, s>>>(cell_cnt, nx, ny, row_load);
         ++g_kernel_launches;
     }
 }

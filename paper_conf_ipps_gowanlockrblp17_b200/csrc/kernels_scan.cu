@@ -6,7 +6,6 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
-#include "cellkey.cuh"
 #include "internal.h"
 
 namespace hdb {
@@ -49,14 +48,15 @@ __device__ __forceinline__ uint64_t peek(const unsigned long long* w) {
     return v;
 }
 
-// Op: Tout load(idx) (idx < n) -- the item; void store(idx, excl) -- its exclusive prefix;
+// Op: Tout load(idx) (idx < n) -- the item; void store(idx, excl, item) -- its exclusive prefix
+// (and the item again, recovered from the prefixes -- the load is not repeated);
 // void total(t) -- the sum of all items (written by the last tile)
 template <typename Tin, typename Tout>
 struct PlainScan {
     const Tin* __restrict__ in;
     Tout* __restrict__ out;
     __device__ __forceinline__ Tout load(uint64_t i) const { return (Tout)in[i]; }
-    __device__ __forceinline__ void store(uint64_t i, Tout e) const { out[i] = e; }
+    __device__ __forceinline__ void store(uint64_t i, Tout e, Tout) const { out[i] = e; }
     __device__ __forceinline__ void total(uint64_t n, Tout t) const { out[n] = t; }
 };
 
@@ -101,43 +101,59 @@ __global__ void __launch_bounds__(SC_THREADS) k_scan_lookback(Op op, uint64_t n,
         wpre += (i < w) ? x : (Tout)0;
         tot += x;
     }
-    if (w == 0) {
-        Tout excl = 0;
-        if (t == 0) {
-            if (lane == 0 && tiles) publish(&tiles[0], kStPre | ep | (uint64_t)tot);
-        } else {
-            if (lane == 0) publish(&tiles[t], kStAgg | ep | (uint64_t)tot);
-            int64_t pred = (int64_t)t - 1;
-            while (true) {
-                const int64_t j = pred - lane;
-                // before tile 0: prefix 0; a word of another epoch counts as not yet published
-                auto ready = [&](uint64_t wd) { return (wd >> 62) != 0 && (wd & (kEpMask << kEpShift)) == ep; };
-                uint64_t word = j >= 0 ? peek(&tiles[j]) : (kStPre | ep);
-                while (__any_sync(FULL, !ready(word))) {               // wait for every predecessor in view
-                    if (!ready(word)) word = peek(&tiles[j]);
-                }
-                const unsigned pre = __ballot_sync(FULL, (word >> 62) == 2);
-                const int first = pre ? __ffs(pre) - 1 : 32;           // nearest inclusive prefix
-                Tout val = lane <= first ? (Tout)(word & kValMask) : (Tout)0;
-#pragma unroll
-                for (int o = 16; o > 0; o >>= 1) val += __shfl_xor_sync(FULL, val, o);
-                excl += val;
-                if (pre) break;
-                pred -= 32;
+    // Look-back by the whole CTA: 256 predecessors per step (a warp looking at 32 per step
+    // walked back through a whole wave of concurrently started tiles -- ~900 aggregates,
+    // ~28 dependent L2 round trips -- while the other warps waited at the barrier)
+    __shared__ int s_first;
+    __shared__ Tout s_lb[SC_THREADS / 32];
+    Tout excl = 0;
+    if (t == 0) {
+        if (tid == 0 && tiles) publish(&tiles[0], kStPre | ep | (uint64_t)tot);
+    } else {
+        if (tid == 0) publish(&tiles[t], kStAgg | ep | (uint64_t)tot);
+        // before tile 0: prefix 0; a word of another epoch counts as not yet published
+        auto ready = [&](uint64_t wd) { return (wd >> 62) != 0 && (wd & (kEpMask << kEpShift)) == ep; };
+        int64_t pred = (int64_t)t - 1;
+        while (true) {
+            const int64_t j = pred - tid;
+            uint64_t word = j >= 0 ? peek(&tiles[j]) : (kStPre | ep);
+            while (__syncthreads_or(!ready(word))) {   // wait for every predecessor in view
+                if (!ready(word)) word = peek(&tiles[j]);
             }
-            if (lane == 0) publish(&tiles[t], kStPre | ep | (uint64_t)(excl + tot));
+            if (tid == 0) s_first = SC_THREADS;
+            __syncthreads();
+            if ((word >> 62) == 2) atomicMin(&s_first, tid);   // nearest inclusive prefix
+            __syncthreads();
+            const int first = s_first;
+            Tout val = tid <= first ? (Tout)(word & kValMask) : (Tout)0;
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) val += __shfl_xor_sync(FULL, val, o);
+            if (lane == 0) s_lb[w] = val;
+            __syncthreads();
+#pragma unroll
+            for (int i = 0; i < SC_THREADS / 32; ++i) excl += s_lb[i];
+            if (first < SC_THREADS) break;
+            pred -= SC_THREADS;
+            __syncthreads();   // s_first / s_lb are rewritten by the next step
         }
-        if (lane == 0) s_excl = excl;
+        if (tid == 0) publish(&tiles[t], kStPre | ep | (uint64_t)(excl + tot));
     }
+    if (tid == 0) s_excl = excl;
     __syncthreads();
     const Tout pre = s_excl + wpre + (incl - run);
 #pragma unroll
     for (int i = 0; i < SC_ITEMS; ++i) buf[tid * SC_ITEMS + i] = pre + v[i];
     __syncthreads();
+    const Tout tile_end = s_excl + tot;   // inclusive prefix of the tile's last item
 #pragma unroll
     for (int i = 0; i < SC_ITEMS; ++i) {
-        uint64_t idx = base + (uint64_t)i * SC_THREADS + tid;
-        if (idx < n) op.store(idx, buf[i * SC_THREADS + tid]);
+        const int j = i * SC_THREADS + tid;
+        uint64_t idx = base + (uint64_t)j;
+        if (idx < n) {
+            // the item itself = the next position's exclusive prefix - this one's
+            const Tout e = buf[j];
+            op.store(idx, e, (j + 1 < SC_TILE ? buf[j + 1] : tile_end) - e);
+        }
     }
     if (tid == 0 && base + SC_TILE >= n) op.total(n, s_excl + tot);   // last tile writes the total
 }
@@ -209,8 +225,8 @@ struct RleScan {
     __device__ __forceinline__ uint32_t load(uint64_t i) const {
         return (i == 0 || keys[i] != keys[i - 1]) ? 1u : 0u;
     }
-    __device__ __forceinline__ void store(uint64_t i, uint32_t e) const {
-        if (i == 0 || keys[i] != keys[i - 1]) {
+    __device__ __forceinline__ void store(uint64_t i, uint32_t e, uint32_t run_start) const {
+        if (run_start) {
             ckey[e] = (uint64_t)keys[i];
             cstart[e] = (uint32_t)i;
         }
@@ -221,25 +237,23 @@ struct RleScan {
     }
 };
 
-// process-shard band: the points whose cell row is in [ylo, yhi), in input
-// order, with their input rows (stream compaction as a scan of the membership flags)
-template <typename T>
+// process-shard band: the points whose cell row (rowid, from the band
+// histogram pass) is in [ylo, yhi), in input order, with their input rows (stream
+// compaction as a scan of the membership flags; only members' coordinates are read)
+template <typename P2>
 struct BandSelect {
-    using P2 = typename V2<T>::type;
     const P2* __restrict__ xy;
-    KeyParams kp;
+    const uint32_t* __restrict__ rowid;
     uint64_t ylo, yhi;
     P2* __restrict__ out;
     uint32_t* __restrict__ gid;
     uint32_t* __restrict__ n_out;
-    __device__ __forceinline__ bool in(uint64_t i) const {
-        uint64_t cx, cy;
-        cell_xy<T>(xy[i], kp, cx, cy);
-        return cy >= ylo && cy < yhi;
+    __device__ __forceinline__ uint32_t load(uint64_t i) const {
+        const uint32_t y = rowid[i];
+        return y >= ylo && y < yhi ? 1u : 0u;
     }
-    __device__ __forceinline__ uint32_t load(uint64_t i) const { return in(i) ? 1u : 0u; }
-    __device__ __forceinline__ void store(uint64_t i, uint32_t e) const {
-        if (in(i)) {
+    __device__ __forceinline__ void store(uint64_t i, uint32_t e, uint32_t member) const {
+        if (member) {
             out[e] = xy[i];
             gid[e] = (uint32_t)i;
         }
@@ -247,18 +261,18 @@ struct BandSelect {
     __device__ __forceinline__ void total(uint64_t, uint32_t t) const { *n_out = t; }
 };
 
-void band_select(const void* xy, uint64_t n, hdb_dtype dt, double xmin, double ymin, double inv_w, uint32_t nx,
-                 uint32_t ny, uint64_t ylo, uint64_t yhi, void* out, uint32_t* gid, uint32_t* n_out, void* temp,
-                 cudaStream_t s) {
+void band_select(const void* xy, const uint32_t* rowid, uint64_t n, hdb_dtype dt, uint64_t ylo, uint64_t yhi, void* out,
+                 uint32_t* gid, uint32_t* n_out, void* temp, cudaStream_t s) {
     if (n == 0) {
         cudaMemsetAsync(n_out, 0, sizeof(uint32_t), s);
         return;
     }
-    const KeyParams kp{xmin, ymin, inv_w, nx, ny};
     if (dt == HDB_F64)
-        scan_impl<uint32_t>(BandSelect<double>{(const double2*)xy, kp, ylo, yhi, (double2*)out, gid, n_out}, n, temp, s);
+        scan_impl<uint32_t>(BandSelect<double2>{(const double2*)xy, rowid, ylo, yhi, (double2*)out, gid, n_out}, n,
+                            temp, s);
     else
-        scan_impl<uint32_t>(BandSelect<float>{(const float2*)xy, kp, ylo, yhi, (float2*)out, gid, n_out}, n, temp, s);
+        scan_impl<uint32_t>(BandSelect<float2>{(const float2*)xy, rowid, ylo, yhi, (float2*)out, gid, n_out}, n, temp,
+                            s);
 }
 
 void cell_rle(const void* keys_sorted, int key_bytes, uint64_t n, uint64_t* ckey, uint32_t* cstart, uint32_t* nne_out,
