@@ -8,12 +8,15 @@ count, scan, neighbour write into a device-resident table.
 through the C-ABI from pinned HOST points to a HOST table plus the host DBSCAN
 (a1-a11), with the H2D/D2H copies inside the timed region.
 
-Workload (default): C2, the TEC-like set of SW1's size (1,864,620 points,
-P:828-829), eps = 0.45, minpts = 4 (BASELINE.json configs[1]).
+Workload (default): C5, the dense-skew batching stress set (BASELINE.json
+configs[4]): 50,000,000 points in [0,1000)^2, 10% of them in 1% of the area,
+eps = 0.5, minpts = 4 -- the config BASELINE names for 1/2/4/8 GPUs.  The C2
+(TEC-like, configs[1]) and C3 lines are kept under profiles/.
 
-Multi-GPU (torchrun): every rank holds the full point set and its grid and
-computes the table for its shard of the cell-sorted queries (SURVEY 8(e));
-the only collective is an all_gather of the per-shard pair counts.
+Multi-GPU (torchrun): every rank holds the full point set, builds the grid of
+its band of cell rows (plus the halo rows its stencils reach) and computes the
+table of the band's queries; the only
+collective is an all_gather of the per-shard pair counts.
 """
 from __future__ import annotations
 
@@ -48,6 +51,34 @@ SWEEP_WORKLOADS = {
                      desc="TEC-like n=1,864,620, eps {0.15,0.20,0.30,0.45,0.60,0.80,1.00,1.40} x minpts "
                           "{4,8,16}: 8 tables, each reused for 3 minpts"),
 }
+
+
+def pcie_d2h_peak(torch, dev, nbytes=1 << 30, reps=5):
+    """Measured D2H rate into pinned host memory (the e2e table's bound)."""
+    h = torch.empty(nbytes, dtype=torch.uint8).pin_memory()
+    d = torch.empty(nbytes, dtype=torch.uint8, device=dev)
+    best = 0.0
+    for _ in range(reps):
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        h.copy_(d, non_blocking=True)
+        torch.cuda.synchronize()
+        best = max(best, nbytes / (time.perf_counter() - t0) / 1e9)
+    del h, d
+    return best
+
+
+def run_config(args, wl, ws):
+    """The config dict both arms print (same keys and values for the same run)."""
+    return {"workload": args.workload, "desc": wl["desc"], "eps": wl["eps"], "dtype": args.dtype,
+            "parallelism": f"query-shard{ws}",
+            "l2": "not flushed: every step writes the whole neighbour table (GBs, >> 126 MB L2)"}
+
+
+def sweep_config(args, wl, ws):
+    return {"workload": args.workload, "desc": wl["desc"], "dtype": args.dtype,
+            "variants": len(wl["eps"]) * len(wl["minpts"]), "parallelism": f"eps-shard{ws}",
+            "l2": "not flushed: every step writes 8 tables totalling ~88 GB (>> 126 MB L2)"}
 
 
 def load_peaks():
@@ -232,7 +263,7 @@ def run_reference(args, wl, ws, rank):
     line = {"impl": "reference", "metric": "eps_neighbor_pairs_per_sec", "value": v, "unit": "pairs/s",
             "n_gpus": ws, "steps": K, "warmup": W, "ms_per_step": 1000 * t_all / max(K, 1),
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
-            "data": "synthetic", "config": {"workload": args.workload, "desc": wl["desc"]},
+            "data": "synthetic", "config": run_config(args, wl, ws),
             "cpu_baseline": dict(res, value=v),
             "e2e": {"value": v, "unit": "pairs/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
@@ -269,7 +300,7 @@ def run_sweep(args, wl, ws, rank, local):
                 "n_gpus": ws, "steps": K, "warmup": W, "ms_per_step": 1e3 * t_full,
                 "higher_is_better": True, "scaling": "strong",
                 "vs_baseline": None, "dtype": args.dtype, "data": "synthetic",
-                "config": {"workload": args.workload, "desc": wl["desc"]},
+                "config": sweep_config(args, wl, ws),
                 "cpu_baseline": {"value": v, "unit": "points/s", "cores": res[0]["cores"], "kind": "oracle",
                                  "sample": "per eps, brute-force rows (extrapolated to all n rows): "
                                            + "; ".join(r["sample"] for r in res)},
@@ -328,11 +359,9 @@ def run_sweep(args, wl, ws, rank, local):
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms / args.steps,
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": args.dtype,
             "data": "synthetic",
-            "config": {"workload": args.workload, "desc": wl["desc"], "n": n, "variants": variants,
-                       "parallelism": f"eps-shard{ws}",
-                       "l2": "not flushed: every step writes 8 tables totalling ~88 GB (>> 126 MB L2)",
-                       "step": "hdb_sweep, sweep_on_device=1: per eps grid + device table; per minpts GPU "
-                               "DBSCAN into device labels"},
+            "config": sweep_config(args, wl, ws), "n": n,
+            "step": "hdb_sweep, sweep_on_device=1: per eps grid + device table; per minpts GPU "
+                    "DBSCAN into device labels",
             "gpu_launches": launches, "clocks": clk.summary()}
     if rank == 0 and ws == 1:
         # e2e: same call from pinned host points into host labels
@@ -387,7 +416,7 @@ def main():
     ap.add_argument("--steps", type=int, default=10)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="hdb", choices=["hdb", "reference"])
-    ap.add_argument("--workload", default="C2-eps0.45", choices=sorted(WORKLOADS) + sorted(SWEEP_WORKLOADS))
+    ap.add_argument("--workload", default="C5-eps0.5", choices=sorted(WORKLOADS) + sorted(SWEEP_WORKLOADS))
     ap.add_argument("--hybrid-steps", type=int, default=1,
                     help="C4-sweep: timed runs of the paper's hybrid sweep (host tables + host DBSCAN)")
     ap.add_argument("--dtype", default="f64", choices=["f64", "f32"])
@@ -472,10 +501,10 @@ def main():
     P = pairs_total // max(args.steps, 1)
     value = pairs_total / (ms / 1000.0)
 
-    # roofline of the dominant kernel, HBM-write bound (DESIGN.md sec. 5):
+    # roofline of the dominant kernel, HBM-write bound (DESIGN.md sec. 5; SURVEY 8(d)):
     #  * single pass (k_fused, device-resident tables): 4 B per pair written + per query
-    #    12 B (begin/count by id) + 4 B (sorted count) + the query/candidate reads of the
-    #    sorted coordinates and ids (16 B f64 / 8 B f32 + 4 B) = 4P + 36n (f64) / 4P + 28n (f32);
+    #    12 B (begin/count by id) + the reads of the sorted coordinates and ids (16 B f64 /
+    #    8 B f32 + 4 B) + 4 B per non-empty cell (its spans' starts) = 4P + 32n + 4C (f64);
     #  * two-pass write kernel (k_emit): 4 B per pair + 12 B per query (offset + id map).
     hbm, peak_kind = load_peaks()
     n_shard = (v.end_query - v.first_query) if ws > 1 else n
@@ -484,7 +513,7 @@ def main():
     esz = 16 if args.dtype == "f64" else 8
     #  * paper kernels: the key/value result set R, 8 B per pair, + the query's coordinates and id
     alg_bytes = (8 * v.npairs + (esz + 4) * n_shard if paper else
-                 4 * v.npairs + ((esz + 20) * n_shard if single else 12 * n_shard))
+                 4 * v.npairs + ((esz + 16) * n_shard + 4 * st["n_nonempty"] if single else 12 * n_shard))
     wms = float(np.mean(write_ms))
     achieved = alg_bytes / (wms / 1000.0) / 1e9
     traffic = None
@@ -503,14 +532,14 @@ def main():
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms / args.steps,
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": args.dtype,
             "data": "synthetic",
-            "config": {"workload": args.workload, "desc": wl["desc"], "n": n, "eps": eps,
-                       "pairs_per_step": P, "parallelism": f"query-shard{ws}",
-                       "l2": "not flushed: each step writes a %.1f GB table (>> 126 MB L2)" % (4 * P / 1e9),
-                       "step": (("grid build + single-pass count/reserve/write (k_fused, capacity = the grid's "
-                                 "candidate tests, no sample; device-resident table)") if single and not st["est_pairs"] else
-                                "grid build + sampled count + single-pass count/reserve/write (k_fused, "
-                                "device-resident table)" if single else
-                                "grid build + sampled count + count + scan + write (device-resident table)")},
+            "config": run_config(args, wl, ws),
+            "n": n, "pairs_per_step": P, "table_gb": 4 * P / 1e9,
+            "step": (("grid build + single-pass count/reserve/write (k_fused, capacity = the grid's "
+                      "candidate tests, no sample; device-resident table)") if single and not st["est_pairs"] else
+                     "grid build + sampled count + single-pass count/reserve/write (k_fused, "
+                     "device-resident table)" if single else
+                     "grid build + sampled count + count + scan + write (device-resident table)")
+            + (" -- per rank: the grid of its band of cell rows (+ halo), its queries' table" if ws > 1 else ""),
             "gpu_launches": launches,
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
                          "frac": achieved / hbm, "traffic": traffic, "peak_kind": peak_kind,
@@ -580,6 +609,7 @@ def main():
             return k
 
         te, Pe = timed(e2e_table, args.e2e_steps)
+        d2h_peak = pcie_d2h_peak(torch, dev)
         th, kh = timed(e2e_hybrid, max(1, args.e2e_steps - 1))
         td, kd = timed(e2e_device, args.e2e_steps)
         line["e2e"] = {"value": Pe / te, "unit": "pairs/s", "h2d_bytes_per_step": esz * n,
@@ -590,7 +620,10 @@ def main():
                        "hybrid": "e2e + host DBSCAN on T (minpts=4, all host cores) -- the paper's split",
                        "points_clustered_per_sec_device": n / td, "s_per_step_device": td,
                        "device": "pinned host points -> device table -> GPU DBSCAN -> labels D2H (NEXT-4)",
-                       "n_clusters": kh, "n_clusters_device": kd}
+                       "n_clusters": kh, "n_clusters_device": kd,
+                       "pcie": {"d2h_peak_gbs": d2h_peak, "e2e_d2h_gbs": (4 * Pe + 12 * n) / te / 1e9,
+                                "frac": (4 * Pe + 12 * n) / te / 1e9 / d2h_peak,
+                                "peak_how": "pinned host <- device copy of 1 GiB, best of 5, measured in this run"}}
     elif ws > 1 and args.e2e_steps > 0 and not paper:
         # N ranks: every rank takes the pinned host points to a HOST table of its query shard
         # (H2D of all points, its shard's D2H); time = max over ranks (barriers around each
