@@ -64,7 +64,9 @@ template <typename Tout, typename Op>
 __global__ void __launch_bounds__(SC_THREADS) k_scan_lookback(Op op, uint64_t n, unsigned long long* __restrict__ tiles,
                                                               uint64_t ep, unsigned long long* __restrict__ ctr,
                                                               uint64_t ctr_base) {
-    __shared__ Tout buf[SC_TILE];
+    // one pad word per 32: the per-thread runs (stride SC_ITEMS) are bank-conflict free
+    __shared__ Tout buf[SC_TILE + SC_TILE / 32];
+    auto bi = [](int j) { return j + (j >> 5); };
     __shared__ Tout wsum[SC_THREADS / 32];
     __shared__ Tout s_excl;
     __shared__ uint64_t s_tile;
@@ -76,7 +78,7 @@ __global__ void __launch_bounds__(SC_THREADS) k_scan_lookback(Op op, uint64_t n,
 #pragma unroll
     for (int i = 0; i < SC_ITEMS; ++i) {
         uint64_t idx = base + (uint64_t)i * SC_THREADS + tid;
-        buf[i * SC_THREADS + tid] = idx < n ? op.load(idx) : (Tout)0;
+        buf[bi(i * SC_THREADS + tid)] = idx < n ? op.load(idx) : (Tout)0;
     }
     __syncthreads();
     Tout v[SC_ITEMS];
@@ -84,7 +86,7 @@ __global__ void __launch_bounds__(SC_THREADS) k_scan_lookback(Op op, uint64_t n,
 #pragma unroll
     for (int i = 0; i < SC_ITEMS; ++i) {
         v[i] = run;
-        run += buf[tid * SC_ITEMS + i];
+        run += buf[bi(tid * SC_ITEMS + i)];
     }
     Tout incl = run;
 #pragma unroll
@@ -142,7 +144,7 @@ __global__ void __launch_bounds__(SC_THREADS) k_scan_lookback(Op op, uint64_t n,
     __syncthreads();
     const Tout pre = s_excl + wpre + (incl - run);
 #pragma unroll
-    for (int i = 0; i < SC_ITEMS; ++i) buf[tid * SC_ITEMS + i] = pre + v[i];
+    for (int i = 0; i < SC_ITEMS; ++i) buf[bi(tid * SC_ITEMS + i)] = pre + v[i];
     __syncthreads();
     const Tout tile_end = s_excl + tot;   // inclusive prefix of the tile's last item
 #pragma unroll
@@ -151,8 +153,8 @@ __global__ void __launch_bounds__(SC_THREADS) k_scan_lookback(Op op, uint64_t n,
         uint64_t idx = base + (uint64_t)j;
         if (idx < n) {
             // the item itself = the next position's exclusive prefix - this one's
-            const Tout e = buf[j];
-            op.store(idx, e, (j + 1 < SC_TILE ? buf[j + 1] : tile_end) - e);
+            const Tout e = buf[bi(j)];
+            op.store(idx, e, (j + 1 < SC_TILE ? buf[bi(j + 1)] : tile_end) - e);
         }
     }
     if (tid == 0 && base + SC_TILE >= n) op.total(n, s_excl + tot);   // last tile writes the total

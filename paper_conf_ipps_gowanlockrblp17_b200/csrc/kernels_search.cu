@@ -262,15 +262,19 @@ constexpr int kWinPad = kWin + 1;   // padded smem rows: 72-B stride, conflict-f
 // i's kWin chunk masks to my (per window instead of per chunk: one warp
 // barrier and shared load per window), stores them to the mask table (gmask
 // non-null) and the window buffer is cleared for the next window.
+// nck: the window's chunks (the rest of the row is zero)
 __device__ __forceinline__ void flush_window(uint2 (*swin)[kWinPad], uint2* gmask, uint32_t v, uint32_t nq,
-                                             uint32_t& my, int lane, bool clear = true) {
+                                             uint32_t& my, int lane, bool clear = true, uint32_t nck = kWin) {
     __syncwarp();
     if ((uint32_t)lane < nq) {
         uint2 r[kWin];
 #pragma unroll
         for (int kk = 0; kk < kWin; ++kk) {
-            r[kk] = swin[lane][kk];
-            my += __popc(r[kk].x) + __popc(r[kk].y);
+            r[kk] = make_uint2(0, 0);
+            if ((uint32_t)kk < nck) {
+                r[kk] = swin[lane][kk];
+                my += __popc(r[kk].x) + __popc(r[kk].y);
+            }
         }
         if (gmask) {
             uint4* dst = (uint4*)(gmask + ((size_t)v * nq + lane) * kWin);
@@ -301,7 +305,9 @@ struct VSpan {
 
 // lanes r < nspan load span r; warp prefix over the pair counts; returns the
 // number of virtual pairs
-__device__ __forceinline__ uint32_t load_vspans(const SArgs& a, uint32_t c, VSpan* vs, int lane) {
+// (ncand, optional: the group's candidate count, summed over the spans by one REDUX)
+__device__ __forceinline__ uint32_t load_vspans(const SArgs& a, uint32_t c, VSpan* vs, int lane,
+                                                uint32_t* ncand = nullptr) {
     uint32_t lo = 0, hi = 0, np = 0;
     if ((uint32_t)lane < a.nspan) {
         const uint2 sp = __ldg(&a.cspan[a.nspan * c + lane]);
@@ -309,9 +315,11 @@ __device__ __forceinline__ uint32_t load_vspans(const SArgs& a, uint32_t c, VSpa
         hi = sp.y;
         np = hi > lo ? ((hi + 1) >> 1) - (lo >> 1) : 0;
     }
+    if (ncand) *ncand = __reduce_add_sync(FULL, hi - lo);   // empty spans have lo == hi
+    static_assert(kMaxSpans + 1 <= 16, "the span prefix below covers 16 lanes");
     uint32_t incl = np;
 #pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
+    for (int o = 1; o < 16; o <<= 1) {
         const uint32_t y = __shfl_up_sync(FULL, incl, o);
         if (lane >= o) incl += y;
     }
@@ -413,16 +421,13 @@ __device__ __forceinline__ uint32_t count_group(const SArgs& a, uint32_t qs, uin
         }
     }
     uint32_t my = 0;
-    const uint32_t npairs = load_vspans(a, c, vsp, lane);
+    uint32_t ncand;
+    const uint32_t npairs = load_vspans(a, c, vsp, lane, &ncand);
     const uint32_t nch = (npairs + 31) / 32;
     if (nch_out) *nch_out = nch;
     const bool keep = keep_single && nch <= kWin;
     if (keep) gmask = nullptr;
-    if (lane == 0) {   // candidate tests of the group: nq x (candidates of its spans)
-        uint32_t ncand = 0;
-        for (uint32_t r = 0; r < a.nspan; ++r) ncand += vsp[r].hi - vsp[r].lo;
-        tests += (unsigned long long)nq * ncand;
-    }
+    if (lane == 0) tests += (unsigned long long)nq * ncand;   // candidate tests of the group
     VCursor cur;
     vc_init(cur);
     // cbuf (f64 modes, k_fused): each chunk's candidate pair is prefetched into the
@@ -582,7 +587,7 @@ __device__ __forceinline__ uint32_t count_group(const SArgs& a, uint32_t qs, uin
         }
         if (kk == kWin - 1) flush_window(swin, gmask, k / kWin, nq, my, lane, !keep);
     }
-    if ((k % kWin) != 0) flush_window(swin, gmask, k / kWin, nq, my, lane, !keep);
+    if ((k % kWin) != 0) flush_window(swin, gmask, k / kWin, nq, my, lane, !keep, k % kWin);
     return my;
 }
 
@@ -871,11 +876,13 @@ __device__ __forceinline__ void emit_group(const SArgs& a, uint32_t c, uint32_t 
             const uint2* mrow = swin ? swin[lane] : raw[lane];
 #pragma unroll
             for (int kk = 0; kk < kWin; ++kk) {
-                const uint2 m = mrow[kk];
-                const uint32_t p0 = my;
-                my += __popc(m.x);
-                wq[lane][kk] = make_uint4(m.x, m.y, p0, my);
-                my += __popc(m.y);
+                if ((uint32_t)kk < nck) {
+                    const uint2 m = mrow[kk];
+                    const uint32_t p0 = my;
+                    my += __popc(m.x);
+                    wq[lane][kk] = make_uint4(m.x, m.y, p0, my);
+                    my += __popc(m.y);
+                }
             }
         }
         __syncwarp();
