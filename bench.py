@@ -36,6 +36,8 @@ import numpy as np  # noqa: E402
 import datagen  # noqa: E402
 
 WORKLOADS = {
+    # C1 (BASELINE configs[0]): the oracle's small case; its bench line is a latency figure
+    "C1-eps0.5": dict(gen=datagen.c1, eps=datagen.C1_EPS, desc="uniform n=10,000 in [0,100)^2 eps=0.5 minpts=4"),
     "C2-eps0.45": dict(gen=datagen.tec_like, eps=0.45, desc="TEC-like n=1,864,620 eps=0.45 minpts=4"),
     "C2-eps0.15": dict(gen=datagen.tec_like, eps=0.15, desc="TEC-like n=1,864,620 eps=0.15 minpts=4"),
     "C2-eps1.40": dict(gen=datagen.tec_like, eps=1.40, desc="TEC-like n=1,864,620 eps=1.40 minpts=4"),
@@ -558,6 +560,8 @@ def main():
             "step_roofline": {"alg_bytes": b_step, "achieved_gbs": b_step / (ms / args.steps / 1e3) / 1e9,
                               "frac": b_step / (ms / args.steps / 1e3) / 1e9 / hbm},
             "clocks": clk.summary(),
+            "latency": {"ms_per_step": ms / args.steps, "grid_build_ms": st["ms_grid"],
+                        "table_kernels_ms": wms, "table_wall_ms": st["ms_table_wall"]},
             "stats": {k: st[k] for k in ("n_nonempty", "n_groups", "candidate_tests", "ms_grid", "ms_sample",
                                          "ms_count", "ms_scan", "ms_write_kernel", "kernel_launches",
                                          "single_pass", "est_pairs", "ms_sort", "n_sparse_queries")}}
