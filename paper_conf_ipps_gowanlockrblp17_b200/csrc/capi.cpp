@@ -115,7 +115,7 @@ hdb_status hdb_ctx_create(const hdb_opts* opts, hdb_ctx** out) {
         HDB_CUDA(cudaMemPoolCreate(&dc.big_pool, &props));
         size_t free_b = 0;
         HDB_CUDA(cudaMemGetInfo(&free_b, &dc.total_mem));
-        dc.scan_ep.cap = 1u << 20;   // tiles of 2,048 elements: scans of up to 2^31 elements
+        dc.scan_ep.cap = 1u << 20;   // tiles of 4,096 elements: scans of up to 2^32 elements
         HDB_CUDA(cudaMalloc((void**)&dc.scan_ep.tiles, (dc.scan_ep.cap + 1) * sizeof(unsigned long long)));
         HDB_CUDA(cudaMemset(dc.scan_ep.tiles, 0, (dc.scan_ep.cap + 1) * sizeof(unsigned long long)));
         HDB_CUDA(cudaMemPoolSetAttribute(dc.big_pool, cudaMemPoolAttrReleaseThreshold, &thr));
