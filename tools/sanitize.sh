@@ -5,7 +5,7 @@
 cd "$(dirname "$0")/.."
 T=${1:-r1}
 mkdir -p gpurun_out
-SEL="c1_full_table or edge_cases or lattice or single_pass or cell_split or sparse_dense_hybrid or device_dbscan_matches or paper_kernels_match or batching_fault or dbscan_end_to_end"
+SEL="c1_full_table or edge_cases or lattice or single_pass or cell_split or sparse_dense_hybrid or device_dbscan_matches or paper_kernels_match or batching_fault or dbscan_end_to_end or shard_bands or virtual_devices"
 for tool in memcheck racecheck synccheck initcheck; do
   extra=""
   [ $tool = racecheck ] && extra="--racecheck-report hazard"
