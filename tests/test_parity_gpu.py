@@ -725,6 +725,39 @@ def test_process_shard_bands_assemble_to_the_oracle_table(torch_cuda, R):
             assert_table_equal(xy, eps, b, c, v)
 
 
+def test_process_shard_bands_empty_and_tiny(torch_cuda):
+    """More shards than populated cell rows: some bands hold no queries (their
+    tables are empty, P = 0) and the rest still assemble into the oracle's
+    table; a single point and an all-identical set behave the same way."""
+    from paper_conf_ipps_gowanlockrblp17_b200 import dist as hdist
+    rng = np.random.default_rng(3)
+    sets = [(np.stack([rng.uniform(0, 50, 300), rng.choice([0.1, 0.2, 3.9], 300)], 1), 0.5),
+            (np.array([[1.5, -2.0]]), 1.0),
+            (np.tile([[0.25, 0.75]], (70, 1)), 0.1)]
+    for xy, eps in sets:
+        n = xy.shape[0]
+        for device in (True, False):
+            parts, ranges, empty = [], [], 0
+            for r in range(8):
+                ctx = _ctx(shard_rank=r, shard_count=8)
+                try:
+                    g = hdb.hdb_grid_build(ctx, xy, eps)
+                    t = (hdb.hdb_neighbor_table_device if device else hdb.hdb_neighbor_table)(ctx, g)
+                    hdb.hdb_grid_free(g)
+                    v = hdb.hdb_table_view_get(t)
+                    ranges.append((v.first_query, v.end_query))
+                    empty += v.npairs == 0
+                    parts.append(hdb.hdb_table_copy_to_host(t))
+                    hdb.hdb_table_free(t)
+                finally:
+                    hdb.hdb_ctx_destroy(ctx)
+            assert empty >= 1
+            assert ranges[0][0] == 0 and ranges[-1][1] == n
+            assert all(ranges[i][1] == ranges[i + 1][0] for i in range(7))
+            b, c, v = hdist.assemble(parts, n)
+            assert_table_equal(xy, eps, b, c, v)
+
+
 def test_sparse_batches_and_shards(torch_cuda):
     """The sparse queries of a group range follow the range: many small batches
     (host table) and process shards give the oracle's table."""
