@@ -284,10 +284,10 @@ __device__ __forceinline__ void flush_window(uint2 (*swin)[kWinPad], uint2* gmas
         }
     }
     __syncwarp();
-    if (!clear) return;   // the caller emits straight from swin (single-window group)
-#pragma unroll
-    for (int kk = 0; kk < kWin; ++kk) swin[lane][kk] = make_uint2(0, 0);   // next window starts empty
-    __syncwarp();
+    // no clearing: every (query < nq, chunk < nck) entry is rewritten by the next window's
+    // count loop before any reader looks at it, and readers stop at nck (a single-window
+    // group of k_fused emits straight from swin: `clear` = false keeps that explicit)
+    (void)clear;
 }
 
 // ---------------------------------------------------------------- virtual chunks
@@ -390,10 +390,10 @@ constexpr double kFarD = 1e300;
 
 // Count one query group (queries qs .. qs+nq-1 of non-empty cell c): hit masks
 // to gmask (windowed layout; null = do not store), tests accumulated per lane;
-// returns lane i's |N_eps(query i)| (0 for lanes >= nq).  With masks, swin
-// must be all zero on entry and is left all zero (flush_window clears it) --
-// except with keep_single when the group has a single window (*nch_out <= kWin):
-// then its masks stay in swin (and are not stored to gmask) for the caller.
+// returns lane i's |N_eps(query i)| (0 for lanes >= nq).  swin needs no
+// initialisation (every entry a reader looks at is written first); with
+// keep_single and a single window (*nch_out <= kWin) the masks stay in swin
+// (and are not stored to gmask) for the caller.
 template <int MODE>
 __device__ __forceinline__ uint32_t count_group(const SArgs& a, uint32_t qs, uint32_t c, uint32_t nq,
                                                 uint2 (*swin)[kWinPad], VSpan* vsp, ulonglong2* sq, double2* sqd,
@@ -765,7 +765,8 @@ __global__ void __launch_bounds__(kSearchThreads) k_search(SArgs a, uint32_t g0,
             }
         }
         uint32_t junk = 0;
-        if (!WRITE && gmask && (k % kWin) != 0) flush_window(swin[WRITE ? 0 : w], gmask, k / kWin, nq, junk, lane);
+        if (!WRITE && gmask && (k % kWin) != 0)
+            flush_window(swin[WRITE ? 0 : w], gmask, k / kWin, nq, junk, lane, true, k % kWin);
         if (!WRITE && (uint32_t)lane < nq) cnt[qs + lane] = my;
         if (++ii >= iend) {
             ii = i0 + grab(ctr, chunk, lane);
@@ -993,9 +994,7 @@ __global__ void __launch_bounds__(kFusedThreads, kFusedMinBlocks)
     unsigned long long tests = 0;
     for_each_group(a, moff, g0, g1, chunk, ctr, lane, [&](const GMeta& m) {
         // count (hit masks to the group's slot of the mask table)
-        __syncwarp();
-#pragma unroll
-        for (int kk = 0; kk < kWin; ++kk) my_sm.c.swin[lane][kk] = make_uint2(0, 0);
+        __syncwarp();   // the previous group's readers of the warp's buffers are done
         uint2* gmask = masks + (m.ma >> 1);
         uint32_t nch = 0;
 #if HDB_PF
