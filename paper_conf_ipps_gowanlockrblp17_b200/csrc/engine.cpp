@@ -932,6 +932,9 @@ bool single_pass_table(hdb_ctx* ctx, const DevGrid& g, hdb_table* t, hdb_stats& 
     const uint64_t g0 = g.banded ? g.band_g0 : 0, g1 = g.banded ? g.band_g1 : g.n_groups;
     launch_fused(g, g0, g1, nullptr, sc, masks.as<uint2>(), sc + 1, cap, nb.as<uint32_t>(), beg.as<uint64_t>(),
                  cnt_id.as<uint32_t>(), (unsigned int*)(sc + 2), s);
+    if (g.dl)   // dense/sparse split: the range's sparse queries reserve on the same counter
+        launch_sparse_fused(g, g0, g1, sc, sc + 1, cap, nb.as<uint32_t>(), beg.as<uint64_t>(), cnt_id.as<uint32_t>(),
+                            (unsigned int*)(sc + 2), s);
     HDB_LAUNCH_CHECK();
     HDB_CUDA(cudaEventRecord(e1.e, s));
     HDB_CUDA(cudaMemcpyAsync(dc.pin + 4, sc, 24, cudaMemcpyDeviceToHost, s));
@@ -1221,8 +1224,10 @@ void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hd
         // ---- dense device-resident whole table: the single pass sized by the exact upper
         // bound P <= candidate tests (known from the grid), no sampled estimate needed (the
         // sample kernel and its readback sync were ~3% of a C2 step)
-        if (device_resident && parts == 1 && ctx->opts.search_kernel == 0 && n_pts > 0 && !G0.dl &&
-            G0.tests_total >= (uint64_t)(kFusedDirectTestsPerQuery * (double)n_pts) &&
+        // (with the dense/sparse split: k_fused on the dense groups + the thread-per-query
+        // single pass on the sparse queries, whatever the pairs per query)
+        if (device_resident && parts == 1 && ctx->opts.search_kernel == 0 && n_pts > 0 &&
+            (G0.dl || G0.tests_total >= (uint64_t)(kFusedDirectTestsPerQuery * (double)n_pts)) &&
             4.0 * (double)G0.tests_total <= kFusedDirectMemShare * (double)dc0.total_mem) {
             S.sample_size = 0;
             S.sample_pairs = 0;
@@ -1294,7 +1299,7 @@ void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hd
         // single pass (k_fused): asked for (search_kernel 4) or chosen for dense tables;
         // the dense/sparse split keeps the two passes (the sparse queries' kernels
         // write at scanned offsets)
-        if (!single && device_resident && parts == 1 && (sk == 4 || sk == 0) && n_pts > 0 && !G0.dl) {
+        if (!single && device_resident && parts == 1 && (sk == 4 || sk == 0) && n_pts > 0) {
             HDB_CUDA(cudaStreamSynchronize(s0));   // e_b is in dc0.pin[0]
             const uint64_t eb = dc0.pin[0];
             const bool fused = sk == 4 || (double)(eb * stride) >= kFusedMinPairsPerQuery * (double)n_pts;

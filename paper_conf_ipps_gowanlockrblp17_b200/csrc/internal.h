@@ -206,6 +206,11 @@ void launch_count(const DevGrid& g, uint64_t g0, uint64_t g1, uint32_t* cnt, uns
 void launch_fused(const DevGrid& g, uint64_t g0, uint64_t g1, uint32_t* cnt, unsigned long long* tests, uint2* masks,
                   unsigned long long* pair_ctr, uint64_t cap, uint32_t* out, uint64_t* begin, uint32_t* count,
                   unsigned int* overflow, cudaStream_t s);
+// single pass for the sparse queries (dense/sparse split): thread per query, rows reserved
+// on the same pair counter as launch_fused (run both on one stream)
+void launch_sparse_fused(const DevGrid& g, uint64_t g0, uint64_t g1, unsigned long long* tests,
+                         unsigned long long* pair_ctr, uint64_t cap, uint32_t* out, uint64_t* begin, uint32_t* count,
+                         unsigned int* overflow, cudaStream_t s);
 void launch_write(const DevGrid& g, uint64_t g0, uint64_t g1, const uint64_t* off, uint64_t out_base,
                   uint32_t* out, int variant, int slot, const uint2* masks, cudaStream_t s,
                   uint64_t* begin = nullptr, uint32_t* count = nullptr);

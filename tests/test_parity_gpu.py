@@ -368,9 +368,12 @@ def test_single_pass_selection_and_exact_bound(torch_cuda):
     b, c, v, view, st = lib_table(same, 0.5, device=True)
     assert st["single_pass"] == 1 and view.npairs == 3_000 ** 2
     assert_table_equal(same, 0.5, b, c, v)
-    uni = rng.uniform(0, 100, size=(20_000, 2))   # ~3 pairs per query: two passes
-    b, c, v, view, st = lib_table(uni, 0.5, device=True)
-    assert st["single_pass"] == 0
+    uni = rng.uniform(0, 100, size=(20_000, 2))   # ~3 pairs per query: the dense/sparse split,
+    b, c, v, view, st = lib_table(uni, 0.5, device=True)   # single pass on both kinds of group
+    assert st["single_pass"] == 1 and st["n_sparse_queries"] > 0 and st["est_pairs"] == 0
+    assert_table_equal(uni, 0.5, b, c, v)
+    b, c, v, view, st = lib_table(uni, 0.5, device=True, search_kernel=3)   # no split: two passes
+    assert st["single_pass"] == 0 and st["n_sparse_queries"] == 0
     assert_table_equal(uni, 0.5, b, c, v)
 
 
@@ -475,11 +478,12 @@ def test_c2_full_size_f32_sampled_rows(torch_cuda):
 
 def test_c3l_full_size_sampled_rows(torch_cuda):
     """C3L (5M SDSS-like) bench workloads at full size: eps 0.07 takes the
-    dense/sparse split (two passes, thread-per-query sparse groups), eps 0.20
-    the single pass."""
+    dense/sparse split (single pass: warp-per-group k_fused on the dense groups,
+    thread-per-query k_sparse_fused on the sparse queries), eps 0.20 the single
+    pass without the split."""
     xy = datagen.sdss_like(datagen.C3_N_LARGE, seed=4)
     view, st = _sampled_rows_check(xy, 0.07, m_rows=800, seed=7)
-    assert st["n_sparse_queries"] > 0 and st["single_pass"] == 0
+    assert st["n_sparse_queries"] > 0 and st["single_pass"] == 1
     view, st = _sampled_rows_check(xy, 0.20, m_rows=800, seed=20)
     assert st["single_pass"] == 1
 
@@ -689,6 +693,24 @@ def test_sparse_dense_hybrid(torch_cuda):
             assert st3["n_sparse_queries"] == 0
             assert np.array_equal(c3, c)
     assert saw_mixed
+
+
+def test_sparse_single_pass_many_hits(torch_cuda):
+    """A sparse query (one query x <= 256 candidates) with more hits than the
+    single-pass sparse kernel buffers (32): it re-scans its candidates to write
+    them; the table still equals the oracle, f64 and f32, next to dense groups
+    and isolated points."""
+    rng = np.random.default_rng(8)
+    lone = np.array([[0.99, 0.5]])                                        # alone in its cell
+    clump = np.stack([rng.uniform(1.0, 1.3, 100), rng.uniform(0.4, 0.6, 100)], 1)   # all within eps of it
+    far = rng.uniform(10, 400, size=(400, 2))                             # isolated: sparse groups
+    xy = np.concatenate([lone, clump, far])
+    for dtype in ("f64", "f32"):
+        x = xy.astype(np.float32) if dtype == "f32" else xy
+        b, c, v, view, st = lib_table(x, 1.0, device=True)
+        assert st["single_pass"] == 1 and st["n_sparse_queries"] > 0
+        assert c[0] == 101
+        assert_table_equal(x, 1.0, b, c, v, dtype)
 
 
 @pytest.mark.parametrize("R", [2, 4, 7])
