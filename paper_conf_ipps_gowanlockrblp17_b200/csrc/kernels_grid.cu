@@ -272,13 +272,26 @@ __global__ void __launch_bounds__(256) k_band_hist(const typename V2<T>::type* _
     if (smem)
         for (uint32_t y = threadIdx.x; y < kp.ny; y += blockDim.x) rh[y] = 0;
     __syncthreads();
-    for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
-        uint64_t cx, cy;
-        cell_xy<T>(xy[i], kp, cx, cy);
-        rowid[i] = (uint32_t)cy;
-        if (smem) atomicAdd(&rh[cy], 1u);
-        else atomicAdd(&row_cnt[cy], 1ull);
-        if (cell_cnt && i % kRowSample == 0) atomicAdd(&cell_cnt[cy * kp.nx + cx], 1u);
+    // four points per thread and step, loaded before any atomic (latency hiding)
+    const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+    for (uint64_t i0 = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i0 < n; i0 += 4 * stride) {
+        typename V2<T>::type p[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+            const uint64_t i = i0 + u * stride;
+            if (i < n) p[u] = xy[i];
+        }
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+            const uint64_t i = i0 + u * stride;
+            if (i >= n) break;
+            uint64_t cx, cy;
+            cell_xy<T>(p[u], kp, cx, cy);
+            rowid[i] = (uint32_t)cy;
+            if (smem) atomicAdd(&rh[cy], 1u);
+            else atomicAdd(&row_cnt[cy], 1ull);
+            if (cell_cnt && i % kRowSample == 0) atomicAdd(&cell_cnt[cy * kp.nx + cx], 1u);
+        }
     }
     if (smem) {
         __syncthreads();
@@ -350,14 +363,23 @@ __global__ void __launch_bounds__(PS_THREADS) k_ps_hist(const typename V2<T>::ty
     for (int i = 0; i < PS_WARPS; ++i) h[i][tid] = 0;
     __syncthreads();
     const uint64_t base = (uint64_t)blockIdx.x * PS_TILE;
+    // all loads first, then the shared atomics (an atomic between two loads would keep
+    // the next load from being issued early: one DRAM latency per item)
+    K kr[PS_ITEMS];
 #pragma unroll
     for (int r = 0; r < PS_ITEMS; ++r) {
         const uint64_t idx = base + (uint64_t)r * PS_THREADS + tid;
-        if (idx < n) {
-            const K k = FROM_POINTS ? cell_key<T, K>(xy[idx], kp) : keys[idx];
-            atomicAdd(&h[w][(uint32_t)((k >> shift) & (RS_BINS - 1))], 1u);
+        if (FROM_POINTS) {
+            typename V2<T>::type p{0, 0};
+            if (idx < n) p = xy[idx];
+            kr[r] = cell_key<T, K>(p, kp);
+        } else {
+            kr[r] = idx < n ? keys[idx] : (K)0;
         }
     }
+#pragma unroll
+    for (int r = 0; r < PS_ITEMS; ++r)
+        if (base + (uint64_t)r * PS_THREADS + tid < n) atomicAdd(&h[w][(uint32_t)((kr[r] >> shift) & (RS_BINS - 1))], 1u);
     __syncthreads();
     uint32_t t = 0;
 #pragma unroll
