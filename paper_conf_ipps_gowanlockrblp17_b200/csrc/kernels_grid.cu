@@ -350,7 +350,10 @@ __global__ void k_band_groups(const uint64_t* __restrict__ ckey, uint64_t nne, c
 // staging in shared memory in digit order, coalesced runs).
 constexpr int PS_THREADS = 256;
 constexpr int PS_WARPS = PS_THREADS / 32;
-constexpr int PS_ITEMS = 8;
+#ifndef HDB_PS_ITEMS
+#define HDB_PS_ITEMS 8
+#endif
+constexpr int PS_ITEMS = HDB_PS_ITEMS;
 constexpr int PS_TILE = PS_THREADS * PS_ITEMS;   // 2048 records per CTA
 
 template <typename T, typename K, bool FROM_POINTS>
