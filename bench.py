@@ -547,7 +547,9 @@ def main():
                          "frac": achieved / hbm, "traffic": traffic, "peak_kind": peak_kind,
                          "kernel": ({7: "k_paper_global (GPUCalcGlobal, Alg. 2)",
                                      8: "k_paper_shared (GPUCalcShared, Alg. 3)"}[args.kernel] if paper else
-                                    "k_fused (single pass: count + reserve + emit, a6-a8)" if single
+                                    ("k_fused (single pass: count + reserve + emit, a6-a8)"
+                                     + (" + k_sparse_fused (the sparse queries)" if st["n_sparse_queries"] else ""))
+                                    if single
                                     else "k_emit (neighbour write, a8)"),
                          "kernel_ms": wms, "alg_bytes": alg_bytes},
             "count_kernel": ({"bound": "alu", "kernel": "k_fused (count part, a6)", "ms": wms,

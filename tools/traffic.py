@@ -42,7 +42,8 @@ def capture(wl, dtype="f64", kernel=0, split=0):
         d = per.setdefault(r[iid], {"kernel": r[ik]})
         d[r[im]] = float(r[iv].replace(",", "")) * scale
     launches = list(per.values())
-    fused = [d for d in launches if "k_fused" in d["kernel"]]
+    # single pass: k_fused (+ k_sparse_fused for the sparse queries of the dense/sparse split)
+    fused = [d for d in launches if "k_fused" in d["kernel"] or "k_sparse_fused" in d["kernel"]]
     if fused:
         pick, single = fused, True
     else:   # two passes: the write phase = k_emit + k_sparse<..., true>
