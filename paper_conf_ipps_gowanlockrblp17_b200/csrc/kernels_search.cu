@@ -68,6 +68,10 @@ struct SArgs {
     const uint32_t* ord;
     const uint2* sql;
     const uint32_t* spre;
+    // k_fused (f64 modes): the count phase stages each chunk's candidate pairs in shared
+    // memory with cp.async one chunk ahead (the natural-order launches of large point sets,
+    // whose candidates come from the L2 / DRAM rather than the L1)
+    int pf;
 };
 
 __device__ __forceinline__ void dense_range(const SArgs& a, uint32_t& i0, uint32_t& i1) {
@@ -128,7 +132,7 @@ __device__ __forceinline__ void stg_if_bit(uint32_t* p, uint32_t v, uint32_t m, 
 #define HDB_LD_EL 1
 #endif
 #ifndef HDB_PF
-#define HDB_PF 0
+#define HDB_PF 0   // 1: stage the natural-order launches' candidates via cp.async (A/B: C5 +0.4%, profiles/r2q)
 #endif
 __device__ __forceinline__ double2 ld_cand(const double2* p) {
 #if HDB_LD_EL
@@ -967,9 +971,7 @@ struct FusedCount {
     uint2 swin[32][kWinPad];
     ulonglong2 sq[32];
     double2 sqd[32];
-#if HDB_PF
-    double2 cand[2 * 32 * 2];   // count phase: 2-stage cp.async buffer of the candidate pairs
-#endif
+    double2 cand[2 * 32 * 2];   // count phase: 2-stage cp.async buffer of the candidate pairs (a.pf)
 };
 struct FusedEmit {
     uint2 raw[32][kWin + 2];
@@ -997,11 +999,7 @@ __global__ void __launch_bounds__(kFusedThreads, kFusedMinBlocks)
         __syncwarp();   // the previous group's readers of the warp's buffers are done
         uint2* gmask = masks + (m.ma >> 1);
         uint32_t nch = 0;
-#if HDB_PF
-        double2* cbuf = my_sm.c.cand;
-#else
-        double2* cbuf = nullptr;
-#endif
+        double2* cbuf = a.pf ? my_sm.c.cand : nullptr;   // stage the candidates with cp.async
         const uint32_t my = count_group<MODE>(a, m.qs, m.c, m.nq, my_sm.c.swin, vsp[w], my_sm.c.sq, my_sm.c.sqd,
                                               gmask, tests, lane, true, &nch, cbuf);
         // reserve the group's output
@@ -1376,6 +1374,7 @@ SArgs args_of(const DevGrid& g) {
     a.ord = nullptr;   // set by the whole-range count / write launches
     a.sql = g.sql;
     a.spre = g.spre;
+    a.pf = 0;
     return a;
 }
 
@@ -1582,6 +1581,7 @@ void launch_fused(const DevGrid& g, uint64_t g0, uint64_t g1, uint32_t* cnt, uns
     SArgs a = args_of(g);
     // heavy groups first (whole ranges only: ord lists every group): C2 eps 0.45 2.50 -> 2.10 ms
     if (g0 == 0 && g1 == g.n_groups && use_cost_order(g)) a.ord = g.ord;
+    a.pf = HDB_PF && !a.ord && g.dtype == HDB_F64;   // the natural order: point sets beyond the L2
     unsigned int* ctr = g.counters;
     cudaMemsetAsync(ctr, 0, sizeof(unsigned int), s);
     const int mode = g.dtype == HDB_F32 ? kF32 : (g.filter_l ? kF64Filter : kF64Exact);
