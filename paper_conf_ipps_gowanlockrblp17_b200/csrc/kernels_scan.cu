@@ -18,9 +18,17 @@ constexpr unsigned FULL = 0xffffffffu;
 #ifndef HDB_SC_ITEMS
 #define HDB_SC_ITEMS 16   // tiles of 4,096: C5 run-length encoding 354 -> 258 us, 7 plain scans 273 -> 198 us
 #endif
+#ifndef HDB_SC_ITEMS32
+#define HDB_SC_ITEMS32 16  // 32 (tiles of 8,192): C5 / C2 unchanged, C3 -2% (A/B profiles/r2q) -- kept at 16
+#endif
 constexpr int SC_THREADS = 256;
-constexpr int SC_ITEMS = HDB_SC_ITEMS;
-constexpr int SC_TILE = SC_THREADS * SC_ITEMS;
+// items per thread: fewer, longer tiles shorten the look-back chains (latency-bound)
+template <typename Tout>
+struct Sc {
+    static constexpr int ITEMS = sizeof(Tout) == 4 ? HDB_SC_ITEMS32 : HDB_SC_ITEMS;
+    static constexpr int TILE = SC_THREADS * ITEMS;
+};
+constexpr int SC_TILE_MIN = SC_THREADS * (HDB_SC_ITEMS < HDB_SC_ITEMS32 ? HDB_SC_ITEMS : HDB_SC_ITEMS32);
 
 // Single-pass scan with decoupled look-back (Merrill & Garland 2016): tile t
 // publishes its aggregate, then its inclusive prefix once known, as one packed
@@ -67,6 +75,7 @@ template <typename Tout, typename Op>
 __global__ void __launch_bounds__(SC_THREADS) k_scan_lookback(Op op, uint64_t n, unsigned long long* __restrict__ tiles,
                                                               uint64_t ep, unsigned long long* __restrict__ ctr,
                                                               uint64_t ctr_base) {
+    constexpr int SC_ITEMS = Sc<Tout>::ITEMS, SC_TILE = Sc<Tout>::TILE;
     // one pad word per 32: the per-thread runs (stride SC_ITEMS) are bank-conflict free
     __shared__ Tout buf[SC_TILE + SC_TILE / 32];
     auto bi = [](int j) { return j + (j >> 5); };
@@ -165,6 +174,7 @@ __global__ void __launch_bounds__(SC_THREADS) k_scan_lookback(Op op, uint64_t n,
 
 template <typename Tout, typename Op>
 void scan_impl(const Op& op, uint64_t n, void* temp, cudaStream_t s) {
+    constexpr int SC_TILE = Sc<Tout>::TILE;
     const uint64_t nb = (n + SC_TILE - 1) / SC_TILE;
     unsigned long long* tiles = nullptr;
     unsigned long long* ctr = nullptr;   // tile-id counter (null: one tile, id 0)
@@ -197,7 +207,7 @@ void scan_impl(const Op& op, uint64_t n, void* temp, cudaStream_t s) {
 thread_local ScanEpochs* t_scan_epochs = nullptr;
 
 size_t scan_temp_bytes(uint64_t n) {
-    return ((n + SC_TILE - 1) / SC_TILE + 2) * sizeof(unsigned long long) + 64;   // tile words + counter
+    return ((n + SC_TILE_MIN - 1) / SC_TILE_MIN + 2) * sizeof(unsigned long long) + 64;   // tile words + counter
 }
 
 void scan_u32_to_u32(const uint32_t* in, uint32_t* out, uint64_t n, void* temp, cudaStream_t s) {
