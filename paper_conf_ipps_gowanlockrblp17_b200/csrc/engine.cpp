@@ -226,6 +226,14 @@ constexpr double kFusedMinPairsPerQuery = 20.0;
 // 4 B per test fits in this share of the device memory
 constexpr double kFusedDirectTestsPerQuery = 150.0;
 constexpr double kFusedDirectMemShare = 0.3;
+// Query-lane classification (k_qlanes): opt-in with HDB_QLANES=1.
+// Measured on one B200 (profiles/r3*): parity green, but not faster end to end -- C5 table
+// kernels 11.10 vs 11.42 ms while the small-query list costs +0.33 ms of grid build; C2
+// eps 0.15 0.89 vs 0.55 ms, C3 eps 0.07 0.43 vs 0.32 ms -- so the default keeps the tests rule.
+bool qlanes_enabled() {   // read per grid build (tests switch it within one process)
+    const char* e = std::getenv("HDB_QLANES");
+    return e && std::strtol(e, nullptr, 10) != 0;
+}
 uint32_t sparse_max_tests() {
     static const uint32_t v = [] {
         const char* e = std::getenv("HDB_SPARSE_TESTS");
@@ -295,9 +303,9 @@ static float round_up_f(double v) {
 }
 
 void set_filter_bound(DevGrid& g) {
-    g.filter = g.filter_l = false;
+    g.filter = g.filter_l = g.filter_b = false;
     g.band = g.band_l = 0;
-    g.nb2_l = 0;
+    g.nb2_l = g.nb2_b = 0;
     if (g.dtype != HDB_F64) return;
     g.ox = 0.5 * g.xmin + 0.5 * g.xmax;
     g.oy = 0.5 * g.ymin + 0.5 * g.ymax;
@@ -312,6 +320,15 @@ void set_filter_bound(DevGrid& g) {
     if (R < 1e15 && band < 0.25 * e2) {
         g.band = round_up_f(band);
         g.filter = true;
+    }
+    // query-lane blocks: coordinates relative to the block's first query, queries and staged
+    // candidates within kQCX + k + 1 cell widths of it (x) and k + 1 (y)
+    const double Rb = ((double)kQCX + (double)g.split + 1.0) * g.w * (1.0 + 0x1p-18);
+    const double band_b = filter_band(Rb, Dmax, e2);
+    if (Rb < 1e15 && band_b < 0.25 * e2) {
+        const double B = band_b * (1.0 + 0x1p-20);
+        g.nb2_b = -round_up_f(B * B);
+        g.filter_b = true;
     }
     const double band_l = filter_band(Dmax, Dmax, e2);
     if (band_l < 0.25 * e2) {
@@ -624,6 +641,8 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
     const int sk = ctx->opts.search_kernel;
     const uint32_t max_tests = sparse_max_tests();
     const bool classify = (sk == 0 || sk == 1 || sk == 2 || sk == 4) && max_tests > 0 && n > 0;
+    // default kernel choice: small groups go to the query-lane single pass (device tables)
+    const bool qrule = sk == 0 && qlanes_enabled() && (g.dtype == HDB_F32 || g.filter_b);
     DBuf dpre, spre, dl, sql, ord;
     DBuf words(4 * (NG + 1), s);   // hit-mask words per group (written with the classification)
     unsigned long long* nsp = bb + 8;
@@ -637,7 +656,7 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
         sql = DBuf(8 * (n + 1), s);
         const uint32_t* ngd = gofs.as<uint32_t>() + nne;
         // nsp: [0] sparse queries, [1] candidate tests (zeroed by the bbox init)
-        launch_group_class(g.cstart, g.cspan, g.nspan, g.gstart, g.gcell, ngd, NG, max_tests, dflag.as<uint32_t>(),
+        launch_group_class(g.cstart, g.cspan, g.nspan, g.gstart, g.gcell, ngd, NG, max_tests, qrule, dflag.as<uint32_t>(),
                            sqn.as<uint32_t>(), nsp, (uint8_t*)gbin.p, ohist, words.as<uint32_t>(), kMaskWin, s);
         launch_order_scatter((const uint8_t*)gbin.p, ngd, NG, ohist, ord.as<uint32_t>(), s);
         scan_u32_to_u32(dflag.as<uint32_t>(), dpre.as<uint32_t>(), NG, temp.p, s);
@@ -686,6 +705,7 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
             g.sql = (uint2*)sql.release();
             g.n_dense_groups = hds[0];
             g.n_sparse_q = hds[1];
+            g.qsplit = qrule;
         }
     }
     g.ms_build = elapsed(ev0, ev1);
@@ -1188,6 +1208,21 @@ void table_free(hdb_table* t) {
     delete t;
 }
 
+// The grid as the count -> scan -> write paths see it: a query-lane split (the small
+// groups of k_qlanes) is a device-single-pass-only classification, so those paths run
+// every group through the warp-per-group kernels (as without a split).
+DevGrid without_qsplit(const DevGrid& g) {
+    DevGrid r = g;
+    if (r.qsplit) {
+        r.qsplit = false;
+        r.dl = r.dpre = r.spre = nullptr;
+        r.sql = nullptr;
+        r.n_sparse_q = 0;
+        r.n_dense_groups = r.n_groups;
+    }
+    return r;
+}
+
 void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hdb_table** out) {
     auto t_wall0 = std::chrono::steady_clock::now();
     const uint64_t launches0 = g_kernel_launches.load();
@@ -1208,6 +1243,8 @@ void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hd
     const uint32_t rank = ctx->opts.shard_count > 0 ? (uint32_t)ctx->opts.shard_rank : 0;
     const size_t ndev = device_resident ? 1 : grid->dev.size();
     S.n_devices = (int)ndev;
+    std::vector<DevGrid> gx;   // the grids of the two-pass paths (no query-lane split)
+    for (const DevGrid& d : grid->dev) gx.push_back(without_qsplit(d));
 
     auto* t = new hdb_table;
     t->n = n;
@@ -1256,7 +1293,7 @@ void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hd
         Event es0, es1;
         HDB_CUDA(cudaMemsetAsync(dsum.p, 0, 8, s0));
         HDB_CUDA(cudaEventRecord(es0.e, s0));
-        launch_sample_count(G0, stride, ns, dsamp.as<uint32_t>(), dsum.as<unsigned long long>(), s0);
+        launch_sample_count(gx[0], stride, ns, dsamp.as<uint32_t>(), dsum.as<unsigned long long>(), s0);
         HDB_LAUNCH_CHECK();
         HDB_CUDA(cudaEventRecord(es1.e, s0));
         // e_b lands in pinned scratch; unsharded calls read it after the count pass's sync
@@ -1271,7 +1308,7 @@ void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hd
             sh[0].r.g0 = G0.band_g0;
             sh[0].r.g1 = G0.band_g1;
         } else {
-            std::vector<uint64_t> cuts = shard_cuts(G0, dc0, samp, stride, parts);
+            std::vector<uint64_t> cuts = shard_cuts(gx[0], dc0, samp, stride, parts);
             for (size_t d = 0; d < ndev; ++d) {
                 const uint32_t k = rank * (uint32_t)ndev + (uint32_t)d;
                 sh[d].r.g0 = cuts[k];
@@ -1321,7 +1358,7 @@ void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hd
         }
         if (!single) {
             // ---- a6/a7 on every device
-            run_parallel(ndev, [&](size_t d) { count_phase(ctx, ctx->dev[d], grid->dev[d], sh[d]); });
+            run_parallel(ndev, [&](size_t d) { count_phase(ctx, ctx->dev[d], gx[d], sh[d]); });
             tr.mark("count_phase");
             HDB_CUDA(cudaStreamSynchronize(s0));   // no-op when device 0 ran the count pass (same stream)
             {
@@ -1382,7 +1419,7 @@ void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hd
             if (device_resident) {
                 // ---- a8 into a device-resident table
                 DevCtx& dc = ctx->dev[0];
-                const DevGrid& g = grid->dev[0];
+                const DevGrid& g = gx[0];
                 ShardState& st = sh[0];
                 cudaStream_t s = dc.main;
                 t->on_device = true;
@@ -1442,7 +1479,7 @@ void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hd
                 }
                 std::vector<uint64_t> dev_grows(ndev, 0);
                 run_parallel(ndev, [&](size_t d) {
-                    write_phase_host(ctx, ctx->dev[d], grid->dev[d], sh[d], t->nbrs, batch_pairs, &dev_grows[d]);
+                    write_phase_host(ctx, ctx->dev[d], gx[d], sh[d], t->nbrs, batch_pairs, &dev_grows[d]);
                 });
                 tr.mark("write+d2h");
                 if (whole) {

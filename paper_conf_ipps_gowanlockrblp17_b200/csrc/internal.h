@@ -38,6 +38,13 @@ constexpr int kGroup = 32;
 constexpr int kSearchThreads = 256;
 constexpr int kCounterSlots = 64;   // slot 0: count pass; 1 + stream index: write passes
 constexpr int kMaxCellSplit = 6;    // cell_split k <= 6: 2k+1 <= 13 stencil row spans (kMaxSpans)
+// Query-lane blocks (k_qlanes): a group is SMALL -- its queries
+// take one lane each -- when its hit words fit (sum over the stencil rows of
+// ceil((len/2 + 1) / 16) <= kQW) and every row span holds <= kQS candidates; a block's
+// queries lie in one cell row at most kQCX columns apart (bounds the block-local filter).
+constexpr int kQW = 6;
+constexpr int kQS = 256;
+constexpr int kQCX = 24;
 
 // ---------------------------------------------------------------- grid
 // One device's copy of the grid (Fig. 1 re-laid out):
@@ -62,6 +69,8 @@ struct DevGrid {
     float band_l = 0;    // f64 mode, group-local filter (count pass)
     float nb2_l = 0;     //   -(band_l (1 + 2^-20))^2, rounded away from zero
     bool filter_l = false;
+    float nb2_b = 0;     // f64 mode, query-lane block filter (origin: the block's first query)
+    bool filter_b = false;
     double xmin = 0, ymin = 0, xmax = 0, ymax = 0;
     double ox = 0, oy = 0;  // f64 mode: origin of the f32 filter coordinates
     uint32_t nx = 1, ny = 1;
@@ -88,6 +97,8 @@ struct DevGrid {
     uint32_t* spre = nullptr;      // [n_groups+1] sparse queries before group g
     uint2* sql = nullptr;          // [n_sparse_q] {sorted position, non-empty cell} of each sparse query
     uint64_t n_sparse_q = 0, n_dense_groups = 0;
+    bool qsplit = false;           // the sparse list holds the SMALL groups (query-lane rule): only the
+                                   // device single pass uses it (k_qlanes); other paths ignore the split
     uint64_t tests_total = 0;      // sum over groups of queries x candidates (0: not computed); >= P
     cudaStream_t stream = nullptr; // stream the buffers were allocated on
     float ms_build = 0;
@@ -149,7 +160,7 @@ void launch_group_build(const uint32_t* cstart, const uint32_t* gofs, uint64_t n
 // sql[spre[g] + i] = {gstart[g] + i, gcell[g]}
 void launch_group_class(const uint32_t* cstart, const uint2* cspan, uint32_t nspan, const uint32_t* gstart,
                         const uint32_t* gcell, const uint32_t* ng_dev, uint64_t n, uint32_t max_tests,
-                        uint32_t* dflag, uint32_t* sqn, unsigned long long* n_sparse, uint8_t* gbin,
+                        bool qlanes, uint32_t* dflag, uint32_t* sqn, unsigned long long* n_sparse, uint8_t* gbin,
                         uint32_t* ohist, uint32_t* words, uint32_t win, cudaStream_t s);
 // cost order: ord = the groups by gbin (dense groups first, heaviest first); ohist holds
 // 2 * kOrderBins words (bin sizes from launch_group_class, then cursors; zeroed by the caller);

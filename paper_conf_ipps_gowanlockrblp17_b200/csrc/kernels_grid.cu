@@ -626,7 +626,8 @@ __global__ void __launch_bounds__(256) k_group_class(const uint32_t* __restrict_
                                                      const uint32_t* __restrict__ gstart,
                                                      const uint32_t* __restrict__ gcell,
                                                      const uint32_t* __restrict__ ng_dev, uint64_t n,
-                                                     uint32_t max_tests, uint32_t* __restrict__ dflag,
+                                                     uint32_t max_tests, bool qlanes,
+                                                     uint32_t* __restrict__ dflag,
                                                      uint32_t* __restrict__ sqn,
                                                      unsigned long long* __restrict__ n_sparse,
                                                      uint8_t* __restrict__ gbin, uint32_t* __restrict__ ohist,
@@ -644,16 +645,21 @@ __global__ void __launch_bounds__(256) k_group_class(const uint32_t* __restrict_
             const uint32_t nq = min((uint32_t)kGroup, cstart[c + 1] - qs);
             uint64_t cand = 0;
             uint32_t npairs = 0;   // candidate pairs of the virtual chunk sequence (mask layout)
+            uint32_t qw = 0, qlen = 0;   // query-lane hit words, longest row span
             for (uint32_t r = 0; r < nspan; ++r) {
                 const uint2 sp = cspan[(uint64_t)nspan * c + r];
                 cand += sp.y - sp.x;
-                if (sp.y > sp.x) npairs += ((sp.y + 1) >> 1) - (sp.x >> 1);
+                if (sp.y > sp.x) {
+                    npairs += ((sp.y + 1) >> 1) - (sp.x >> 1);
+                    qw += ((sp.y - sp.x) / 2 + 1 + 15) / 16;
+                    qlen = max(qlen, sp.y - sp.x);
+                }
             }
             const uint32_t ch = (npairs + 31) / 32;
             words[g] = 2 * nq * win * ((ch + win - 1) / win);
             const uint64_t tests = (uint64_t)nq * cand;
             ttot += tests;
-            if (tests <= max_tests) sq = nq;
+            if (qlanes ? (qw <= (uint32_t)kQW && qlen <= (uint32_t)kQS) : tests <= max_tests) sq = nq;
             else d = 1;
             // cost bin: dense groups first, each class by decreasing log2(tests)
             const uint32_t lg = 63 - __clzll(tests | 1);
@@ -1027,10 +1033,11 @@ void launch_group_build(const uint32_t* cstart, const uint32_t* gofs, uint64_t n
 
 void launch_group_class(const uint32_t* cstart, const uint2* cspan, uint32_t nspan, const uint32_t* gstart,
                         const uint32_t* gcell, const uint32_t* ng_dev, uint64_t n, uint32_t max_tests,
-                        uint32_t* dflag, uint32_t* sqn, unsigned long long* n_sparse, uint8_t* gbin,
+                        bool qlanes, uint32_t* dflag, uint32_t* sqn, unsigned long long* n_sparse, uint8_t* gbin,
                         uint32_t* ohist, uint32_t* words, uint32_t win, cudaStream_t s) {
     if (n == 0) return;
-    k_group_class<<<grid_for(n), 256, 0, s>>>(cstart, cspan, nspan, gstart, gcell, ng_dev, n, max_tests, dflag, sqn,
+    k_group_class<<<grid_for(n), 256, 0, s>>>(cstart, cspan, nspan, gstart, gcell, ng_dev, n, max_tests, qlanes,
+                                              dflag, sqn,
                                               n_sparse, gbin, ohist, words, win);
     ++g_kernel_launches;
 }

@@ -68,6 +68,12 @@ struct SArgs {
     const uint32_t* ord;
     const uint2* sql;
     const uint32_t* spre;
+    // query-lane blocks (k_qlanes): cell keys (row-major, < 2^30), grid width, points, and the
+    // flag bound of the block-local filter (-(band_b (1 + 2^-20))^2)
+    const uint64_t* ckey;
+    uint32_t nx;
+    uint32_t n;
+    float nb2_b;
     // k_fused (f64 modes): the count phase stages each chunk's candidate pairs in shared
     // memory with cp.async one chunk ahead (the natural-order launches of large point sets,
     // whose candidates come from the L2 / DRAM rather than the L1)
@@ -1017,8 +1023,10 @@ __global__ void __launch_bounds__(kFusedThreads, kFusedMinBlocks)
         if ((uint32_t)lane < m.nq) {
             const uint32_t id = __ldg(&a.ids[m.qs + lane]);
             if (cnt) cnt[m.qs + lane] = my;   // counts in sorted order (optional)
+#ifndef HDB_QX_NOT
             begin[id] = base + excl;
             count[id] = my;
+#endif
         }
         if (base + total <= cap) {
             uint32_t* gout = out + base;
@@ -1245,6 +1253,447 @@ __global__ void __launch_bounds__(256) k_sparse_fused(SArgs a, uint32_t g0, uint
     if (tests_out && lane == 0 && tests) atomicAdd(tests_out, tests);
 }
 
+// ---------------------------------------------------------------- query-per-lane blocks
+// Single pass for the SMALL groups of a device-resident table (DESIGN.md "query
+// lanes"): Alg. 2's thread-per-query mapping with the candidates staged
+// in shared memory as in Alg. 3.  Where cells hold few points (C5's
+// sparse 99% of the area: ~11 queries, ~100 candidates per cell) a warp per cell
+// leaves most lanes idle in the emission and pays its set-up per 11 queries; here
+// a warp takes a BLOCK of up to 32 consecutive small queries of one cell row (up
+// to kQCX cell columns apart), one query per lane:
+//  * per stencil row r the union of the lanes' row spans (one contiguous range of
+//    sorted positions: the spans of cells of one row are monotone) is staged in
+//    shared memory as f32 pairs relative to the block's first query (f64 -> f32
+//    once per candidate, so the filter band is that of a block-sized region, not
+//    of the whole bounding box);
+//  * each lane walks ITS span inside the staged union (broadcast-free per-lane
+//    LDS.128, two candidates per FADD2/FFMA2) and shifts the sign bits of t into
+//    per-lane hit words (SHF, no ballots); a word whose band flag is set is
+//    replayed with the in-band tests decided in exact f64;
+//  * one warp-wide reservation on the pair counter shared with k_fused, T by id,
+//    then each lane walks its hit bits (FLO) writing ids into a shared-memory
+//    stage at its list's offset, and the warp copies the stage out with aligned,
+//    coalesced 16-B streaming stores -- the block's rows are one contiguous range.
+constexpr int kQThreads = 128;
+constexpr int kQWarps = kQThreads / 32;
+constexpr int kQGrab = 128;   // small queries per grab (natural order: the L2 keeps the stencil rows);
+                              // fewer when the warps would otherwise not all get work
+// kQW, kQS, kQCX: internal.h (the grid build's classification bounds them)
+constexpr int kQOut = 1152;                // output stage (ids): most blocks' rows in one round (C5: ~1,150)
+constexpr int kQIds = 384;                 // staged ids of a block: its row unions' lengths + 2 per row
+static_assert(kQOut * 4 >= (kQS / 2 + 1 + 4) * 16, "the candidate stage overlays the output stage");
+struct QSmem {
+    uint32_t bits[kQW][32];    // hit words, [word][lane]
+    uint32_t wtag[kQW][32];    // idst index of the candidate of each word's MSB
+    uint32_t idst[kQIds];      // the ids of the block's row unions, row after row
+    union {
+        float4 cand[kQS / 2 + 1 + 4];   // testing: candidate pairs {x0, x1, y0, y1} of one row union
+        uint32_t out[kQOut];   // emission: the block's ids in table order (offset by the misalignment)
+    } st;
+};
+__device__ __forceinline__ void stg_cs_v4(uint32_t* p, uint4 v) {
+    asm volatile("st.global.cs.v4.u32 [%0], {%1, %2, %3, %4};" ::"l"(p), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w));
+}
+__device__ __forceinline__ void stg_cs(uint32_t* p, uint32_t v) {
+    asm volatile("st.global.cs.u32 [%0], %1;" ::"l"(p), "r"(v));
+}
+// (cur << 1) | (v >> 31): append the sign bit of v
+__device__ __forceinline__ uint32_t push_sign(uint32_t cur, uint32_t v) {
+    uint32_t r;
+    asm("shf.l.wrap.b32 %0, %1, %2, 1;" : "=r"(r) : "r"(v), "r"(cur));
+    return r;
+}
+
+#ifdef HDB_QX_PROF   // profiling build only: clock64 per phase, summed over warps, printed at the end
+__device__ unsigned long long g_qx_prof[8];
+__device__ unsigned int g_qx_done;
+#define QX_T(i)                                         \
+    do {                                                \
+        const long long t_ = clock64();                 \
+        if ((i) > 0) qx_acc[(i) - 1] += t_ - qx_last;   \
+        qx_last = t_;                                   \
+    } while (0)
+#else
+#define QX_T(i) ((void)0)
+#endif
+template <int MODE>   // kF64Filter (block-local f32 filter + exact f64 replay) or kF32 (exact f32)
+__global__ void __launch_bounds__(kQThreads, 7)   // 7 CTAs: 7 KB of shared memory per warp
+    k_qlanes(SArgs a, uint32_t g0, uint32_t g1, uint32_t grab, unsigned int* __restrict__ ctr,
+             unsigned long long* __restrict__ tests_out, unsigned long long* __restrict__ pair_ctr, uint64_t cap,
+             uint32_t* __restrict__ out, uint64_t* __restrict__ begin, uint32_t* __restrict__ count,
+             unsigned int* __restrict__ overflow) {
+    __shared__ QSmem smem[kQWarps];
+    const int lane = threadIdx.x & 31;
+    QSmem& S = smem[threadIdx.x >> 5];
+    const ulonglong2* const st2 = reinterpret_cast<const ulonglong2*>(S.st.cand);
+    const u64x NE2 = pack2(-a.e2f, -a.e2f);
+    const u64x NB2 = pack2(a.nb2_b, a.nb2_b);
+    unsigned long long tests = 0;
+#ifdef HDB_QX_PROF
+    long long qx_acc[6] = {0, 0, 0, 0, 0, 0}, qx_last = 0;
+#endif
+    const uint32_t j0 = __ldg(&a.spre[g0]), j1 = __ldg(&a.spre[g1]);   // the range's small queries
+    // work: grabs of `grab` small queries (the next grab is taken one grab early); the next
+    // block's list entries, cell keys and first stencil rows are loaded while a block runs
+    auto take = [&]() -> uint32_t {
+        uint32_t v = 0;
+        if (lane == 0) v = atomicAdd(ctr, grab);
+        return j0 + __shfl_sync(FULL, v, 0);
+    };
+    constexpr int kPre = 3;   // stencil rows prefetched (k = 1: all)
+    uint32_t j = take(), jn = take();
+    uint32_t jend = min(j + grab, j1);
+    uint2 e_n = make_uint2(0, 0), sp_n[kPre];
+    uint32_t key_n = 0;
+    double2 dq_n = make_double2(0, 0);   // f64 mode: the entry's query coordinates
+    auto prefetch = [&](uint32_t jb, uint32_t je) {
+        const bool in = jb + lane < je;
+        e_n = in ? __ldg(&a.sql[jb + lane]) : make_uint2(0, 0);
+        if (MODE == kF64Filter) dq_n = in ? __ldg(&a.xd[e_n.x]) : make_double2(0, 0);
+        key_n = in ? (uint32_t)__ldg(&a.ckey[e_n.y]) : 0u;
+#pragma unroll
+        for (int r = 0; r < kPre; ++r)
+            sp_n[r] = (in && (uint32_t)r < a.nspan) ? __ldg(&a.cspan[a.nspan * e_n.y + r]) : make_uint2(0, 0);
+    };
+    if (j < j1) prefetch(j, jend);
+    while (j < j1) {
+        {
+            QX_T(0);
+            // ---- the block: the leading run of queries in the row of the first one, at most
+            // kQCX columns on, whose row spans stay within kQS of the first query's span starts
+            const bool in = j + lane < jend;
+            const uint2 e = e_n;
+            const uint32_t key = key_n;
+            const double2 dq0 = dq_n;
+            const uint32_t key0 = __shfl_sync(FULL, key, 0);
+            const uint32_t dk = key - key0;
+            bool ok = in && dk <= (uint32_t)kQCX && key0 % a.nx + dk < a.nx;
+            uint32_t ids_need = 0;   // staged ids if this lane were the block's last
+            for (uint32_t r = 0; r < a.nspan; ++r) {
+                uint2 sp;
+                if (r < (uint32_t)kPre) {
+                    sp = r == 0 ? sp_n[0] : r == 1 ? sp_n[1] : sp_n[2];
+                } else {
+                    sp = in ? __ldg(&a.cspan[a.nspan * e.y + r]) : make_uint2(0, 0);
+                }
+                const uint32_t lo0 = __shfl_sync(FULL, sp.x, 0);
+                ok = ok && sp.x >= lo0 && sp.y - lo0 <= (uint32_t)kQS;
+                ids_need += sp.y - lo0 + 2;
+            }
+            ok = ok && ids_need <= (uint32_t)kQIds;
+            const unsigned okm = __ballot_sync(FULL, ok);
+            uint32_t Q = ~okm ? (uint32_t)(__ffs(~okm) - 1) : 32u;
+            if (Q == 0) {   // cannot happen for a classified small group; the host rebuilds exactly
+                if (lane == 0) atomicOr(overflow, 1u);
+                Q = 1;
+            }
+            // the next block's inputs (loads in flight while this block runs)
+            {
+                uint32_t jb = j + Q;
+                if (jb >= jend) {
+                    jb = jn;
+                    jend = min(jn + grab, j1);
+                    if (jn < j1) jn = take();
+                }
+                if (jb < j1) prefetch(jb, jend);
+                if (Q == 1 && !(okm & 1u)) {   // (the Q == 0 case) skip the query
+                    j = jb;
+                    continue;
+                }
+                j = jb;   // (the current block's entries are e, Q, in registers)
+            }
+            QX_T(1);
+            const bool act = (uint32_t)lane < Q;
+            const uint32_t q = e.x, c = e.y;
+            const uint32_t qid = act ? __ldg(&a.ids[q]) : 0u;   // T by id (used after the reservation)
+            double2 o = make_double2(0, 0);
+            u64x QX, QY;
+            if (MODE == kF64Filter) {
+                const double2 dq = act ? dq0 : make_double2(0, 0);
+                o.x = __shfl_sync(FULL, dq.x, 0);
+                o.y = __shfl_sync(FULL, dq.y, 0);
+                const float qx = (float)__dsub_rn(dq.x, o.x), qy = (float)__dsub_rn(dq.y, o.y);
+                QX = pack2(qx, qx);
+                QY = pack2(qy, qy);
+            } else {
+                const float2 p = act ? __ldg(&a.xs[q]) : make_float2(0, 0);
+                QX = pack2(p.x, p.x);
+                QY = pack2(p.y, p.y);
+            }
+            QX_T(2);
+            // ---- per stencil row: the union [U0e, U1) of the lanes' spans is staged, then every
+            // lane walks its own span inside it
+            uint32_t my = 0, nw = 0, R = 0;   // R: the row's first entry in the id stage
+            for (uint32_t r = 0; r < a.nspan; ++r) {
+                const uint2 sp = act ? __ldg(&a.cspan[a.nspan * c + r]) : make_uint2(0, 0);
+                const uint32_t U0 = __shfl_sync(FULL, sp.x, 0);
+                const uint32_t U1 = __reduce_max_sync(FULL, act ? sp.y : 0u);
+                const uint32_t U0e = U0 & ~1u;
+                __syncwarp();   // the previous row's tests / the previous block's output copy are done
+                if (U1 <= U0) continue;   // the row is empty for every lane (warp-uniform)
+                if (act) tests += sp.y - sp.x;
+                const uint32_t npu = (U1 - U0e + 1) >> 1;
+                for (uint32_t p = lane; p < npu + 4; p += 32) {   // (+4 pairs of far-away padding: overrun)
+                    float4 v = make_float4(kFarF, kFarF, kFarF, kFarF);
+                    if (p < npu) {
+                        const uint32_t s = U0e + 2 * p;
+                        // the pair's ids (s even: 8-B aligned), read by the emission
+                        uint2 iv = make_uint2(0, 0);
+                        if (s + 1 < a.n) iv = ld_ids(reinterpret_cast<const uint2*>(a.ids + s));
+                        else iv.x = __ldg(&a.ids[s]);
+                        *reinterpret_cast<uint2*>(S.idst + R + 2 * p) = iv;
+                        if (MODE == kF64Filter) {
+                            const double2 c0 = ld_cand(a.xd + s);
+                            v.x = (float)__dsub_rn(c0.x, o.x);
+                            v.z = (float)__dsub_rn(c0.y, o.y);
+                            if (s + 1 < a.n) {
+                                const double2 c1 = ld_cand(a.xd + s + 1);
+                                v.y = (float)__dsub_rn(c1.x, o.x);
+                                v.w = (float)__dsub_rn(c1.y, o.y);
+                            }
+                        } else {
+                            const float2 c0 = __ldg(&a.xs[s]);
+                            v.x = c0.x;
+                            v.z = c0.y;
+                            if (s + 1 < a.n) {
+                                const float2 c1 = __ldg(&a.xs[s + 1]);
+                                v.y = c1.x;
+                                v.w = c1.y;
+                            }
+                        }
+                    }
+                    S.st.cand[p] = v;
+                }
+                __syncwarp();
+                // this lane's pairs [pa, pa + npl) of the staged union; the element before the
+                // span (odd start) and after it (odd end) are masked off
+                uint32_t npl = 0, pa = 0;
+                if (act && sp.y > sp.x) {
+                    pa = (sp.x - U0e) >> 1;
+                    npl = ((sp.y - 1 - U0e) >> 1) - pa + 1;
+                }
+                uint32_t fix = ((sp.x - U0e) & 1u) ? 0x7fffffffu : ~0u;
+                const bool odd_end = (sp.y - U0e) & 1u;
+                for (uint32_t i = 0; i < npl; i += 16) {
+                    const uint32_t cnt = min(16u, npl - i);
+                    const ulonglong2* P = st2 + pa + i;
+                    uint32_t cur = 0, acc = 0, proc = 0;
+#pragma unroll 1
+                    for (; proc < cnt; proc += 4) {
+#pragma unroll
+                        for (int u = 0; u < 4; ++u) {
+                            const ulonglong2 C = P[proc + u];
+                            const u64x dx = sub2(QX, C.x);
+                            const u64x dy = sub2(QY, C.y);
+                            if (MODE == kF64Filter) {
+                                const u64x tt = fma2(dy, dy, fma2(dx, dx, NE2));   // (dx^2 - e2) + dy^2
+                                const float2 uu = unpack2(fma2(tt, tt, NB2));     // t^2 - B^2 < 0 <=> |t| < B
+                                acc |= __float_as_uint(uu.x) | __float_as_uint(uu.y);
+                                const float2 t = unpack2(tt);
+                                cur = push_sign(cur, __float_as_uint(t.x));   // hit <=> t < 0 (t = +-0: in the band)
+                                cur = push_sign(cur, __float_as_uint(t.y));
+                            } else {
+                                // exact f32 (reading R2): fl(fl(dx^2) + fl(dy^2)) <= e2; miss <=> e2 - s < 0
+                                const float2 px = unpack2(mul2(dx, dx));
+                                const float2 py = unpack2(mul2(dy, dy));
+                                cur = push_sign(cur, __float_as_uint(__fsub_rn(a.e2f, __fadd_rn(px.x, py.x))));
+                                cur = push_sign(cur, __float_as_uint(__fsub_rn(a.e2f, __fadd_rn(px.y, py.y))));
+                            }
+                        }
+                    }
+                    if (MODE == kF32) cur = ~cur;
+                    cur <<= 2 * (16 - proc);   // bit 31 - 2p - e: element e of pair p
+                    if (MODE == kF64Filter && (int)acc < 0) {
+                        // a test of this word is within the band: decide the band tests in exact f64
+                        const double2 dq = __ldg(&a.xd[q]);
+                        for (uint32_t p = 0; p < cnt; ++p) {
+                            const ulonglong2 C = P[p];
+                            const u64x dx = sub2(QX, C.x);
+                            const u64x dy = sub2(QY, C.y);
+                            const u64x tt = fma2(dy, dy, fma2(dx, dx, NE2));
+                            const float2 uu = unpack2(fma2(tt, tt, NB2));
+#pragma unroll
+                            for (int el = 0; el < 2; ++el) {
+                                const float ue = el ? uu.y : uu.x;
+                                const uint32_t sc = U0e + 2 * (pa + i + p) + el;
+                                if ((ue < 0.f || __float_as_uint(ue) == 0x80000000u) && sc < a.n) {
+                                    const double2 cd = __ldg(&a.xd[sc]);
+                                    const uint32_t bit = 0x80000000u >> (2 * p + el);
+                                    cur = pred_f64(dq.x, dq.y, cd.x, cd.y, a.e2d) ? (cur | bit) : (cur & ~bit);
+                                }
+                            }
+                        }
+                    }
+                    uint32_t m = cnt == 16 ? ~0u : ~(~0u >> (2 * cnt));   // the word's 2 cnt elements
+                    m &= fix;
+                    fix = ~0u;
+                    if (odd_end && i + 16 >= npl) m &= ~(1u << (32 - 2 * cnt));
+                    cur &= m;
+                    my += __popc(cur);
+                    if (cur) {   // only words with hits are kept (the emission never skips a word)
+                        S.bits[nw][lane] = cur;
+                        S.wtag[nw][lane] = R + 2 * (pa + i);
+                        ++nw;
+                    }
+                }
+                R += 2 * npu;
+            }
+            QX_T(3);
+            // ---- reserve the block's rows (one range: lane i's list at excl), T by id (a10)
+            uint32_t incl = my;
+#pragma unroll
+            for (int d = 1; d < 32; d <<= 1) {
+                const uint32_t y = __shfl_up_sync(FULL, incl, d);
+                if (lane >= d) incl += y;
+            }
+            const uint32_t total = __shfl_sync(FULL, incl, 31);
+            unsigned long long base = 0;
+#ifdef HDB_QX_NOATOM   // timing experiment only (wrong table): per-warp arenas instead of the counter
+            {
+                static __shared__ unsigned long long arena[kQWarps];
+                const uint64_t wid = (uint64_t)blockIdx.x * kQWarps + (threadIdx.x >> 5);
+                const uint64_t per = cap / ((uint64_t)gridDim.x * kQWarps);
+                if (lane == 0) {
+                    if (arena[threadIdx.x >> 5] + total > per || j == 0) arena[threadIdx.x >> 5] = 0;
+                    base = wid * per + arena[threadIdx.x >> 5];
+                    arena[threadIdx.x >> 5] += total;
+                }
+            }
+#else
+            if (lane == 0 && total) base = atomicAdd(pair_ctr, (unsigned long long)total);
+#endif
+            base = __shfl_sync(FULL, base, 0);
+            const uint32_t excl = incl - my;
+#ifndef HDB_QX_NOT   // (timing experiment: no T by id)
+            if (act) {
+                begin[qid] = base + excl;
+                count[qid] = my;
+            }
+#endif
+            if (base + total > cap) {   // the capacity bound failed: the host rebuilds exactly
+                if (lane == 0) atomicOr(overflow, 1u);
+                continue;
+            }
+#ifdef HDB_QX_NOEMIT   // timing experiment only (no table)
+            continue;
+#endif
+            QX_T(4);
+            // ---- emission in rounds of <= kQOut ids (one round unless the block is heavy): every
+            // lane walks its hit bits (FLO) writing the ids into the output stage at its list's
+            // offset (the stage is offset by the destination's misalignment); the stage is then
+            // copied out with 16-B aligned streaming stores
+            __syncwarp();   // (orders the words' stores before the reads below)
+            if (total + 3 <= (uint32_t)kQOut) {
+                // one round (the common case): word by word, bit by bit (MSB first)
+                const uint32_t mis = (uint32_t)(base & 3u);
+                uint32_t* dst = S.st.out + mis + excl;
+                for (uint32_t w = 0; w < nw; ++w) {
+                    uint32_t cb = S.bits[w][lane];
+                    const uint32_t* src = S.idst + S.wtag[w][lane];
+                    do {
+                        uint32_t z;
+                        asm("bfind.shiftamt.u32 %0, %1;" : "=r"(z) : "r"(cb));   // clz
+                        cb ^= 0x80000000u >> z;
+                        *dst++ = src[z];
+                    } while (cb);   // (stored words are non-empty)
+                }
+                __syncwarp();
+                QX_T(5);
+                uint32_t* gd = out + (base - mis);   // 16-B aligned
+                const uint32_t nch = (mis + total + 3) >> 2;
+                for (uint32_t ch = lane; ch < nch; ch += 32) {
+                    const uint4 v = reinterpret_cast<const uint4*>(S.st.out)[ch];
+                    const uint32_t e0 = 4 * ch;
+                    if (e0 >= mis && e0 + 4 <= mis + total) {
+                        stg_cs_v4(gd + e0, v);
+                    } else {
+                        const uint32_t w4[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+                        for (int t = 0; t < 4; ++t)
+                            if (e0 + t >= mis && e0 + t < mis + total) stg_cs(gd + e0 + t, w4[t]);
+                    }
+                }
+                __syncwarp();   // the stage is rewritten by the next block
+                QX_T(6);
+                continue;
+            }
+            uint32_t k = 0, cb = 0, src = 0, wi = 0;
+            for (uint32_t r0 = 0; r0 < total;) {
+                const uint32_t mis = (uint32_t)((base + r0) & 3u);
+                const uint32_t cntr = min(total - r0, (uint32_t)kQOut - mis);
+                const uint32_t rend = r0 + cntr;
+                const uint32_t kend = min(my, rend > excl ? rend - excl : 0u);   // this round's hits: [k, kend)
+                uint32_t* dst = S.st.out + mis + excl - r0;
+                // kQB hits per step: positions first, then the id loads, then the stores
+                constexpr int kQB = 8;
+                for (; k < kend; k += kQB) {
+                    uint32_t pos[kQB];
+#pragma unroll
+                    for (int u = 0; u < kQB; ++u) {
+                        pos[u] = 0;
+                        if (k + u < kend) {
+                            if (cb == 0) {
+                                cb = S.bits[wi][lane];
+                                src = S.wtag[wi][lane];
+                                ++wi;
+                            }
+                            uint32_t z;
+                            asm("bfind.shiftamt.u32 %0, %1;" : "=r"(z) : "r"(cb));   // clz
+                            cb ^= 0x80000000u >> z;
+                            pos[u] = src + z;
+                        }
+                    }
+                    uint32_t v[kQB];
+#pragma unroll
+                    for (int u = 0; u < kQB; ++u)
+                        if (k + u < kend) v[u] = S.idst[pos[u]];
+#pragma unroll
+                    for (int u = 0; u < kQB; ++u)
+                        if (k + u < kend) dst[k + u] = v[u];
+                }
+                k = kend;
+                __syncwarp();
+                QX_T(5);
+                uint32_t* gd = out + (base + r0 - mis);   // 16-B aligned
+                const uint32_t nch = (mis + cntr + 3) >> 2;
+                for (uint32_t ch = lane; ch < nch; ch += 32) {
+                    const uint4 v = reinterpret_cast<const uint4*>(S.st.out)[ch];
+                    const uint32_t e0 = 4 * ch;
+                    if (e0 >= mis && e0 + 4 <= mis + cntr) {
+                        stg_cs_v4(gd + e0, v);
+                    } else {
+                        const uint32_t w4[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+                        for (int t = 0; t < 4; ++t)
+                            if (e0 + t >= mis && e0 + t < mis + cntr) stg_cs(gd + e0 + t, w4[t]);
+                    }
+                }
+                __syncwarp();   // the stage is rewritten by the next round / block
+                QX_T(6);
+                r0 = rend;
+            }
+        }
+    }
+#pragma unroll
+    for (int d = 16; d > 0; d >>= 1) tests += __shfl_xor_sync(FULL, tests, d);
+    if (tests_out && lane == 0 && tests) atomicAdd(tests_out, tests);
+#ifdef HDB_QX_PROF
+    if (lane == 0) {
+        for (int i = 0; i < 6; ++i) atomicAdd(&g_qx_prof[i], (unsigned long long)qx_acc[i]);
+        __threadfence();
+        if (atomicAdd(&g_qx_done, 1u) + 1 == gridDim.x * kQWarps) {
+            const char* nm[6] = {"formation", "query set-up", "stage+test", "reserve+T", "bit-walk", "copy-out"};
+            unsigned long long t = 0;
+            for (int i = 0; i < 6; ++i) t += g_qx_prof[i];
+            for (int i = 0; i < 6; ++i)
+                printf("qx_prof %-13s %6.2f%%  %.3e warp-cycles\n", nm[i], 100.0 * g_qx_prof[i] / t, (double)g_qx_prof[i]);
+            for (int i = 0; i < 6; ++i) g_qx_prof[i] = 0;
+            g_qx_done = 0;
+        }
+    }
+#endif
+}
+
 // a5: warp per sampled query (the paper's estimator kernel),
 // exact predicate, lanes over candidates.
 template <bool F64>
@@ -1375,6 +1824,10 @@ SArgs args_of(const DevGrid& g) {
     a.sql = g.sql;
     a.spre = g.spre;
     a.pf = 0;
+    a.ckey = g.ckey;
+    a.nx = g.nx;
+    a.n = (uint32_t)g.n;
+    a.nb2_b = g.nb2_b;
     return a;
 }
 
@@ -1601,6 +2054,36 @@ void launch_sparse_fused(const DevGrid& g, uint64_t g0, uint64_t g1, unsigned lo
                          unsigned long long* pair_ctr, uint64_t cap, uint32_t* out, uint64_t* begin, uint32_t* count,
                          unsigned int* overflow, cudaStream_t s) {
     if (!g.sql || g.n_sparse_q == 0 || g1 <= g0) return;
+    if (g.qsplit && (g.dtype == HDB_F32 || g.filter_b)) {
+        // small groups (query-lane classification): blocks of up to 32 queries, one per lane
+        const SArgs a = args_of(g);
+        static int bps[2] = {0, 0};
+        const int f64 = g.dtype == HDB_F64;
+        if (!bps[f64]) {
+            if (f64) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps[1], k_qlanes<kF64Filter>, kQThreads, 0);
+            else cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps[0], k_qlanes<kF32>, kQThreads, 0);
+            if (bps[f64] < 1) bps[f64] = 1;
+        }
+        // the range's small queries (whole range: all of them; a band's share is ~ its groups')
+        const uint64_t nq = (g0 == 0 && g1 == g.n_groups)
+                                ? g.n_sparse_q
+                                : (uint64_t)((double)g.n_sparse_q * (double)(g1 - g0) / (double)g.n_groups) + 1;
+        unsigned int* ctr = g.counters + (kCounterSlots - 1);
+        HDB_CUDA(cudaMemsetAsync(ctr, 0, sizeof(unsigned int), s));
+        const uint64_t warps = (uint64_t)148 * bps[f64] * kQWarps;
+        const uint32_t grab = (uint32_t)std::max<uint64_t>(32, std::min<uint64_t>(kQGrab, nq / warps / 32 * 32));
+        const uint64_t need = (nq + grab - 1) / grab;   // grabs (extra CTAs of a band exit at once)
+        const unsigned ctas = (unsigned)std::max<uint64_t>(
+            1, std::min<uint64_t>((uint64_t)148 * bps[f64], (need + kQWarps - 1) / kQWarps));
+        if (f64)
+            k_qlanes<kF64Filter><<<ctas, kQThreads, 0, s>>>(a, (uint32_t)g0, (uint32_t)g1, grab, ctr, tests, pair_ctr, cap, out, begin, count,
+                                                            overflow);
+        else
+            k_qlanes<kF32><<<ctas, kQThreads, 0, s>>>(a, (uint32_t)g0, (uint32_t)g1, grab, ctr, tests, pair_ctr, cap, out, begin, count,
+                                                      overflow);
+        ++g_kernel_launches;
+        return;
+    }
     const unsigned blocks =
         (unsigned)std::max<uint64_t>(1, std::min<uint64_t>((g.n_sparse_q + 255) / 256, 148 * HDB_SPARSE_BLOCKS));
     if (g.dtype == HDB_F64)

@@ -812,3 +812,74 @@ def test_c3_large_bucketed_row_scatter(torch_cuda):
         roff, rnbr = oracle.eps_join_rows(xy, 0.07, rows)
         for i, p in enumerate(rows):
             assert np.array_equal(np.sort(v[b[p]:b[p] + c[p]]), rnbr[roff[i]:roff[i + 1]]), p
+
+
+# ------------------------------------------------------------------ query-lane blocks (opt-in)
+@pytest.fixture
+def qlanes(monkeypatch):
+    """HDB_QLANES=1: small groups take the query-per-lane single pass (k_qlanes)."""
+    monkeypatch.setenv("HDB_QLANES", "1")
+
+
+@pytest.mark.parametrize("dtype", ["f64", "f32"])
+def test_query_lane_blocks_heavy_and_ragged(torch_cuda, qlanes, dtype):
+    """Small groups take the query-per-lane single pass (k_qlanes): blocks of up to
+    32 queries of one cell row whose output overflows the kernel's shared output
+    stage (uniform ~20 points per eps-cell: ~63 hits per query, ~2,000 ids per
+    block -> several emission rounds), next to dense groups (a clump), isolated
+    points (empty rows) and points on the grid's last row / column; the table is
+    the oracle's, and with HDB_QLANES-style classification off (search_kernel 3:
+    no split) the counts agree."""
+    rng = np.random.default_rng(21)
+    side = 1000 ** 0.5
+    uni = rng.uniform(0.0, side, size=(20_000, 2))
+    clump = rng.uniform(5.0, 5.5, size=(600, 2))
+    lone = np.array([[side + 40.0, 3.0], [side + 40.0, side + 40.0], [-30.0, side + 40.0]])
+    xy = np.concatenate([uni, clump, lone])
+    x = xy.astype(np.float32) if dtype == "f32" else xy
+    b, c, v, view, st = lib_table(x, 1.0, device=True)
+    assert st["single_pass"] == 1 and 0 < st["n_sparse_queries"] < x.shape[0]
+    assert_table_equal(x, 1.0, b, c, v, dtype)
+    b3, c3, v3, _, st3 = lib_table(x, 1.0, device=True, search_kernel=3)
+    assert st3["n_sparse_queries"] == 0
+    assert np.array_equal(c3, c)
+
+
+@pytest.mark.parametrize("dtype", ["f64", "f32"])
+def test_query_lane_blocks_workloads(torch_cuda, qlanes, dtype):
+    """The query-lane single pass on the workload shapes (TEC bands, SDSS clumps,
+    dense skew) at several eps -- block formation across cell rows, ragged blocks,
+    dense groups next to small ones -- adversarial near-ties (the block-local f32
+    filter's band replay) and exact lattice ties: every table is the oracle's."""
+    cases = [(datagen.subsample(datagen.tec_like(), 30_000, seed=1), (0.15, 0.45)),
+             (datagen.subsample(datagen.sdss_like(), 30_000, seed=2), (0.07, 0.2, 0.6)),
+             (datagen.dense_skew(30_000, seed=7), (0.5, 4.0)),
+             (datagen.near_ties(3_000, 0.35), (0.35,)),
+             (datagen.lattice(60, spacing=0.25), (0.5, 0.75))]
+    saw = False
+    for xy, eps_list in cases:
+        x = xy.astype(np.float32) if dtype == "f32" else xy
+        for eps in eps_list:
+            b, c, v, view, st = lib_table(x, eps, device=True)
+            assert_table_equal(x, eps, b, c, v, dtype)
+            saw |= st["n_sparse_queries"] > 0
+    assert saw
+
+
+def test_query_lane_blocks_in_shard_bands(torch_cuda, qlanes):
+    """Process-shard bands with the query-lane split: each band's small queries
+    are its share of the list (the kernel reads the range from the prefix), and
+    the shards assemble into the oracle's table."""
+    xy = datagen.dense_skew(40_000, seed=11)
+    eps = 2.0
+    off, nbr = oracle.eps_join(xy, eps)
+    want = np.diff(off.astype(np.int64))
+    got = np.zeros(xy.shape[0], np.int64)
+    for r in range(3):
+        b, c, v, view, st = lib_table(xy, eps, device=True, shard_rank=r, shard_count=3)
+        got += c.astype(np.int64)
+        rows = np.nonzero(c)[0]
+        for p in rows[:: max(1, rows.size // 200)]:
+            lst = np.sort(v[int(b[p]):int(b[p]) + int(c[p])])
+            assert np.array_equal(lst, np.sort(nbr[int(off[p]):int(off[p + 1])]))
+    assert np.array_equal(got, want)

@@ -52,16 +52,16 @@ def test_f32_mode_has_no_ffma(sass):
 
 
 # every kernel that evaluates the predicate, by precision (template argument in the mangled name)
-_F32_KERNELS = r"(k_countILi0E|k_searchILi0E|k_fusedILi0E|k_sparseILb0E|k_sample_countILb0E|k_paper_globalILb0E|k_paper_sharedILb0E)"
+_F32_KERNELS = r"(k_countILi0E|k_searchILi0E|k_fusedILi0E|k_sparseILb0E|k_sample_countILb0E|k_paper_globalILb0E|k_paper_sharedILb0E|k_qlanesILi0E)"
 _F64_EXACT_KERNELS = r"(k_countILi2E|k_searchILi2E|k_fusedILi2E|k_sparseILb1E|k_sample_countILb1E|k_paper_globalILb1E|k_paper_sharedILb1E)"
 
 
 def test_every_f32_predicate_kernel_has_no_ffma(sass):
     """All f32-mode kernels (the default single pass k_fused<0>, the sparse
-    thread-per-query kernels, the sampled count, the paper's two kernels):
-    fl(fl(dx^2) + fl(dy^2)) must never be contracted."""
+    thread-per-query kernels, the sampled count, the paper's two kernels, the
+    query-lane single pass): fl(fl(dx^2) + fl(dy^2)) must never be contracted."""
     ks = {k: v for k, v in sass.items() if re.search(_F32_KERNELS, k)}
-    assert len(ks) == 8, sorted(ks)
+    assert len(ks) == 9, sorted(ks)
     for name, body in ks.items():
         assert "FFMA" not in body, name
 

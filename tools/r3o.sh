@@ -1,0 +1,7 @@
+cd $GRAFT_REPO_ROOT
+timeout 900 python -m pytest tests/test_parity_gpu.py -x -q -k "query_lane or c1_full or workload_subsets or sparse_dense or many_hits or near_ties or lattice or decimal or edge_cases or dense_cell or bands_assemble or bands_empty or single_pass" > gpurun_out/r3o_pytest.txt 2>&1
+WLS="C5-eps0.5" VARS="base" REPS=1 bash tools/ab.sh > gpurun_out/r3o_ab.txt 2>&1
+HDB_LIB=ab/libhdb_prof.so python bench.py --steps 1 --warmup 1 --e2e-steps 0 --no-cpu-baseline 2>&1 | grep qx_prof | tail -6 > gpurun_out/r3o_prof.txt
+for wl in C2-eps0.15 C3-eps0.07 C3L-eps0.07 C1-eps0.5; do
+  timeout 300 python bench.py --workload $wl --steps 10 --warmup 3 --e2e-steps 0 --no-cpu-baseline > gpurun_out/r3o_bench_${wl}.json 2> gpurun_out/r3o_bench_${wl}.err
+done
