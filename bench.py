@@ -368,7 +368,7 @@ def run_sweep(args, wl, ws, rank, local):
     if rank == 0 and ws == 1:
         # e2e: same call from pinned host points into host labels
         xy_pin = torch.from_numpy(xy_np).pin_memory()
-        lab_host = np.empty((len(eps_all), len(mp), n), np.int32)
+        lab_host = torch.empty((len(eps_all), len(mp), n), dtype=torch.int32).pin_memory().numpy()
         hdb.hdb_sweep(ctx, xy_pin, eps_all, mp, labels=lab_host)
         ts = []
         for _ in range(max(1, min(args.steps, 3))):
@@ -575,8 +575,9 @@ def main():
     if rank == 0 and ws == 1 and args.e2e_steps > 0 and not paper:
         hdb.hdb_ctx_set_stream(ctx, None)
         xy_pin = torch.from_numpy(xy_np).pin_memory()
-        labels = np.empty(n, np.int32)
-        core = np.empty(n, np.uint8)
+        # the step's results land in pinned host buffers, like its inputs come from them
+        labels = torch.empty(n, dtype=torch.int32).pin_memory().numpy()
+        core = torch.empty(n, dtype=torch.uint8).pin_memory().numpy()
 
         def table_to_host():
             g = hdb.hdb_grid_build(ctx, xy_pin, eps)

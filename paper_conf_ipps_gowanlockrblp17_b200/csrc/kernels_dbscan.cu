@@ -98,7 +98,21 @@ __device__ __forceinline__ bool reaches(const uint32_t* __restrict__ parent, uin
     return x == r;
 }
 
-constexpr uint32_t kRowsPerGrab = 4;      // consecutive (cell-sorted) rows per warp grab
+// Walk order of the per-point passes (sampled links, labels).  The id-indexed arrays
+// (begin, count, parent: 16 B per point) are read at u in either order; in the table's
+// production (cell-sorted) order u is a random id but the lists stream, in id order u
+// streams but the sampled list entry is a random read.  When those arrays fit in the L2
+// the random id accesses are L2 hits and the production order wins (C2, 1.86M points:
+// sampled links 0.93 vs 1.30 ms); beyond it (C5, 50M points, 800 MB) id order makes
+// three of the four accesses coalesced (sampled links 17 -> 8.3 ms, labels 3.3 -> 0.26 ms).
+constexpr double kIdOrderBytes = 48e6;// Consecutive (cell-sorted) rows per warp grab (<= 32: one per lane for the skip test --
+// rows in A and non-core rows add no edge).  Short lists (mostly rows that are skipped,
+// C5: 79 pairs per row, one giant): 32 rows, so the skip tests run 32 at a time; long lists
+// (C2: 700-4,600 pairs per row, edge-bound): 4 rows, so the rows in flight on an SM stay
+// few and their neighbours' parent entries stay in its L1.  Measured on one B200
+// (device DBSCAN ms, grab 4 / 32): C5 16.6 / 12.4, C2 eps 0.45 3.8 / 7.1, eps 1.40 12.9 / 19.4.
+constexpr uint32_t kGrabShort = 32, kGrabLong = 4;
+constexpr double kLongListPairs = 256.0;
 constexpr int kUnionThreads = 1024;       // one CTA per SM
 
 // first row r in [0, n) with pre[r] >= x (pre = exclusive prefix of the list
@@ -255,7 +269,8 @@ __global__ void k_sched_init(const uint64_t* __restrict__ pre, uint32_t n, uint6
 __global__ void __launch_bounds__(kUnionThreads, 1)
     k_union(const uint64_t* __restrict__ begin, const uint32_t* __restrict__ count, const uint32_t* __restrict__ nbrs,
             const uint32_t* __restrict__ rows, uint32_t* __restrict__ parent, const uint32_t* __restrict__ giant,
-            const uint32_t* __restrict__ bits_a, const uint32_t* __restrict__ bits_b, uint32_t* __restrict__ sched) {
+            const uint32_t* __restrict__ bits_a, const uint32_t* __restrict__ bits_b, uint32_t* __restrict__ sched,
+            uint32_t kRowsPerGrab) {
     const bool have_a = giant[0] != kNonCore, have_b = giant[1] != kNonCore;
     const uint32_t G = gridDim.x;
     const int lane = threadIdx.x & 31;
@@ -272,10 +287,18 @@ __global__ void __launch_bounds__(kUnionThreads, 1)
                 continue;
             }
             const uint32_t r1 = min(end, r0 + kRowsPerGrab);
-            for (uint32_t r = r0; r < r1; ++r) {
-                const uint32_t u = rows ? __ldg(&rows[r]) : r;
-                if (have_a && bit_of(bits_a, u)) continue;                 // uniform
-                if (__ldca(&parent[u]) == kNonCore) continue;              // uniform: non-core rows add no edge
+            // the skip test for all 32 rows at once (one row per lane), then the warp walks the
+            // lists of the rows that remain -- at C5 (one giant component) nearly every row is
+            // in A, and testing them one after the other was a chain of dependent loads per row
+            const uint32_t rl = r0 + lane;
+            uint32_t ul = 0;
+            bool keep = false;
+            if (rl < r1) {
+                ul = rows ? __ldg(&rows[rl]) : rl;
+                keep = !(have_a && bit_of(bits_a, ul)) && __ldca(&parent[ul]) != kNonCore;
+            }
+            for (unsigned todo = __ballot_sync(FULL, keep); todo; todo &= todo - 1) {
+                const uint32_t u = __shfl_sync(FULL, ul, __ffs(todo) - 1);
                 const bool in_b = have_b && bit_of(bits_b, u);
                 const uint32_t* L = nbrs + begin[u];
                 const uint32_t m = count[u];
@@ -365,8 +388,9 @@ void launch_dbscan_device(const uint64_t* begin, const uint32_t* count, const ui
                           uint64_t* pre, void* scan_temp, int32_t* labels, cudaStream_t s) {
     if (n == 0) return;
     k_core_init<<<blocks_for(n), 256, 0, s>>>(count, n, minpts, core, parent);
+    const uint32_t* walk = 16.0 * (double)n > kIdOrderBytes ? nullptr : rows;   // null: id order
     for (uint32_t k = 1; k <= kSampleLinks; ++k) {
-        k_sample_link<<<blocks_for(n), 256, 0, s>>>(begin, count, nbrs, rows, n, k, parent);
+        k_sample_link<<<blocks_for(n), 256, 0, s>>>(begin, count, nbrs, walk, n, k, parent);
         k_compress<<<blocks_for(n), 256, 0, s>>>(n, parent);
     }
     k_giant<<<1, kGiantSamples, 0, s>>>(rows, n, parent, giant);
@@ -383,10 +407,12 @@ void launch_dbscan_device(const uint64_t* begin, const uint32_t* count, const ui
     k_row_counts<<<blocks_for(n), 256, 0, s>>>(count, rows, n, (uint32_t*)root);   // root[] is free until k_flatten
     scan_u32_to_u64((const uint32_t*)root, pre, n, scan_temp, s);
     k_sched_init<<<1, 256, 0, s>>>(pre, (uint32_t)n, npairs, (uint32_t)sms, sched);
-    k_union<<<sms, kUnionThreads, 0, s>>>(begin, count, nbrs, rows, parent, giant, bits, bits + (n + 31) / 32, sched);
+    const uint32_t grab = (double)npairs >= kLongListPairs * (double)n ? kGrabLong : kGrabShort;
+    k_union<<<sms, kUnionThreads, 0, s>>>(begin, count, nbrs, rows, parent, giant, bits, bits + (n + 31) / 32, sched,
+                                          grab);
     k_flatten<<<blocks_for(n), 256, 0, s>>>(core, n, parent, root, is_root);
     scan_u32_to_u32(is_root, rank, n, scan_temp, s);
-    k_labels<<<blocks_for(n), 256, 0, s>>>(begin, count, nbrs, rows, core, root, rank, n, labels);
+    k_labels<<<blocks_for(n), 256, 0, s>>>(begin, count, nbrs, walk, core, root, rank, n, labels);
     g_kernel_launches += 8 + 2 * kSampleLinks;
 }
 
