@@ -548,7 +548,8 @@ def main():
                          "kernel": ({7: "k_paper_global (GPUCalcGlobal, Alg. 2)",
                                      8: "k_paper_shared (GPUCalcShared, Alg. 3)"}[args.kernel] if paper else
                                     ("k_fused (single pass: count + reserve + emit, a6-a8)"
-                                     + (" + k_sparse_fused (the sparse queries)" if st["n_sparse_queries"] else ""))
+                                     + ((" + k_qlanes (the small groups' queries, one per lane)" if st["query_lanes"]
+                                         else " + k_sparse_fused (the sparse queries)") if st["n_sparse_queries"] else ""))
                                     if single
                                     else "k_emit (neighbour write, a8)"),
                          "kernel_ms": wms, "alg_bytes": alg_bytes},
@@ -566,7 +567,8 @@ def main():
                         "table_kernels_ms": wms, "table_wall_ms": st["ms_table_wall"]},
             "stats": {k: st[k] for k in ("n_nonempty", "n_groups", "candidate_tests", "ms_grid", "ms_sample",
                                          "ms_count", "ms_scan", "ms_write_kernel", "kernel_launches",
-                                         "single_pass", "est_pairs", "ms_sort", "n_sparse_queries")}}
+                                         "single_pass", "est_pairs", "ms_sort", "n_sparse_queries",
+                                         "query_lanes")}}
 
     # ---- e2e through the C-ABI from pinned HOST points (H2D inside the timed region):
     #   value: the same metric (pairs/s) with the table delivered to a HOST table (D2H inside);

@@ -171,6 +171,9 @@ typedef struct {
                                     ms_write_kernel is then the search kernel's time                   */
     uint64_t n_sparse_queries;   /* queries of the grid's sparse groups, handled thread-per-query (the
                                     dense/sparse hybrid); 0 = none       */
+    int query_lanes;             /* 1: those are the SMALL groups' queries, taken one per lane by the
+                                    query-lane single pass (k_qlanes; the
+                                    default for point sets beyond the L2, HDB_QLANES=0/1 forces it) */
 } hdb_stats;
 
 /* ---- context ------------------------------------------------------------- */

@@ -226,13 +226,16 @@ constexpr double kFusedMinPairsPerQuery = 20.0;
 // 4 B per test fits in this share of the device memory
 constexpr double kFusedDirectTestsPerQuery = 150.0;
 constexpr double kFusedDirectMemShare = 0.3;
-// Query-lane classification (k_qlanes): opt-in with HDB_QLANES=1.
-// Measured on one B200 (profiles/r3*): parity green, but not faster end to end -- C5 table
-// kernels 11.10 vs 11.42 ms while the small-query list costs +0.33 ms of grid build; C2
-// eps 0.15 0.89 vs 0.55 ms, C3 eps 0.07 0.43 vs 0.32 ms -- so the default keeps the tests rule.
-bool qlanes_enabled() {   // read per grid build (tests switch it within one process)
+// Query-lane classification (k_qlanes): small groups' queries one
+// per lane.  Default: on for point sets beyond the L2 -- the regime in which k_fused visits
+// groups in the natural order (coordinates + ids > 256 MB, use_cost_order), where the warp
+// per 11-query group of C5's sparse area is latency-bound; below it (C2 eps 0.15, C3, C1)
+// k_fused / k_sparse_fused stay faster (profiles/r2x).  HDB_QLANES=1 / 0 forces it on / off.
+bool qlanes_enabled(uint64_t n, hdb_dtype dt) {   // read per grid build (tests switch it within one process)
     const char* e = std::getenv("HDB_QLANES");
-    return e && std::strtol(e, nullptr, 10) != 0;
+    if (e && *e) return std::strtol(e, nullptr, 10) != 0;
+    const uint64_t esz = dt == HDB_F64 ? 16 : 8;
+    return n * (esz + 4) > (256ull << 20);
 }
 uint32_t sparse_max_tests() {
     static const uint32_t v = [] {
@@ -642,7 +645,7 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
     const uint32_t max_tests = sparse_max_tests();
     const bool classify = (sk == 0 || sk == 1 || sk == 2 || sk == 4) && max_tests > 0 && n > 0;
     // default kernel choice: small groups go to the query-lane single pass (device tables)
-    const bool qrule = sk == 0 && qlanes_enabled() && (g.dtype == HDB_F32 || g.filter_b);
+    const bool qrule = sk == 0 && qlanes_enabled(n, g.dtype) && (g.dtype == HDB_F32 || g.filter_b);
     DBuf dpre, spre, dl, sql, ord;
     DBuf words(4 * (NG + 1), s);   // hit-mask words per group (written with the classification)
     unsigned long long* nsp = bb + 8;
@@ -791,6 +794,7 @@ void grid_build(hdb_ctx* ctx, const void* xy, uint64_t n, hdb_dtype dt, double e
     ctx->stats.n_nonempty = g0.n_nonempty;
     ctx->stats.n_groups = g0.n_groups;
     ctx->stats.n_sparse_queries = g0.n_sparse_q;
+    ctx->stats.query_lanes = g0.qsplit ? 1 : 0;
     ctx->stats.ms_grid = g0.ms_build;
     ctx->stats.kernel_launches = (uint32_t)(g_kernel_launches.load() - launches0);
     ctx->live_objects++;
@@ -1236,6 +1240,7 @@ void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hd
     S.n_nonempty = G0.n_nonempty;
     S.n_groups = G0.n_groups;
     S.n_sparse_queries = G0.n_sparse_q;
+    S.query_lanes = G0.qsplit ? 1 : 0;
     S.bytes_d2h = 0;
     S.pool_grows = 0;
     S.n_streams = ctx->opts.n_streams;

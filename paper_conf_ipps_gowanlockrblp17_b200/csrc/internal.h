@@ -42,7 +42,7 @@ constexpr int kMaxCellSplit = 6;    // cell_split k <= 6: 2k+1 <= 13 stencil row
 // take one lane each -- when its hit words fit (sum over the stencil rows of
 // ceil((len/2 + 1) / 16) <= kQW) and every row span holds <= kQS candidates; a block's
 // queries lie in one cell row at most kQCX columns apart (bounds the block-local filter).
-constexpr int kQW = 6;
+constexpr int kQW = 8;
 constexpr int kQS = 256;
 constexpr int kQCX = 24;
 

@@ -1279,13 +1279,11 @@ constexpr int kQWarps = kQThreads / 32;
 constexpr int kQGrab = 128;   // small queries per grab (natural order: the L2 keeps the stencil rows);
                               // fewer when the warps would otherwise not all get work
 // kQW, kQS, kQCX: internal.h (the grid build's classification bounds them)
-constexpr int kQOut = 1152;                // output stage (ids): most blocks' rows in one round (C5: ~1,150)
-constexpr int kQIds = 384;                 // staged ids of a block: its row unions' lengths + 2 per row
+constexpr int kQOut = 1280;                // output stage (ids): a block's rows in one round (C5: ~1,150)
 static_assert(kQOut * 4 >= (kQS / 2 + 1 + 4) * 16, "the candidate stage overlays the output stage");
 struct QSmem {
     uint32_t bits[kQW][32];    // hit words, [word][lane]
-    uint32_t wtag[kQW][32];    // idst index of the candidate of each word's MSB
-    uint32_t idst[kQIds];      // the ids of the block's row unions, row after row
+    uint32_t wtag[kQW][32];    // sorted position of the candidate of each word's MSB
     union {
         float4 cand[kQS / 2 + 1 + 4];   // testing: candidate pairs {x0, x1, y0, y1} of one row union
         uint32_t out[kQOut];   // emission: the block's ids in table order (offset by the misalignment)
@@ -1368,7 +1366,6 @@ __global__ void __launch_bounds__(kQThreads, 7)   // 7 CTAs: 7 KB of shared memo
             const uint32_t key0 = __shfl_sync(FULL, key, 0);
             const uint32_t dk = key - key0;
             bool ok = in && dk <= (uint32_t)kQCX && key0 % a.nx + dk < a.nx;
-            uint32_t ids_need = 0;   // staged ids if this lane were the block's last
             for (uint32_t r = 0; r < a.nspan; ++r) {
                 uint2 sp;
                 if (r < (uint32_t)kPre) {
@@ -1378,9 +1375,7 @@ __global__ void __launch_bounds__(kQThreads, 7)   // 7 CTAs: 7 KB of shared memo
                 }
                 const uint32_t lo0 = __shfl_sync(FULL, sp.x, 0);
                 ok = ok && sp.x >= lo0 && sp.y - lo0 <= (uint32_t)kQS;
-                ids_need += sp.y - lo0 + 2;
             }
-            ok = ok && ids_need <= (uint32_t)kQIds;
             const unsigned okm = __ballot_sync(FULL, ok);
             uint32_t Q = ~okm ? (uint32_t)(__ffs(~okm) - 1) : 32u;
             if (Q == 0) {   // cannot happen for a classified small group; the host rebuilds exactly
@@ -1423,7 +1418,7 @@ __global__ void __launch_bounds__(kQThreads, 7)   // 7 CTAs: 7 KB of shared memo
             QX_T(2);
             // ---- per stencil row: the union [U0e, U1) of the lanes' spans is staged, then every
             // lane walks its own span inside it
-            uint32_t my = 0, nw = 0, R = 0;   // R: the row's first entry in the id stage
+            uint32_t my = 0, nw = 0;
             for (uint32_t r = 0; r < a.nspan; ++r) {
                 const uint2 sp = act ? __ldg(&a.cspan[a.nspan * c + r]) : make_uint2(0, 0);
                 const uint32_t U0 = __shfl_sync(FULL, sp.x, 0);
@@ -1437,11 +1432,7 @@ __global__ void __launch_bounds__(kQThreads, 7)   // 7 CTAs: 7 KB of shared memo
                     float4 v = make_float4(kFarF, kFarF, kFarF, kFarF);
                     if (p < npu) {
                         const uint32_t s = U0e + 2 * p;
-                        // the pair's ids (s even: 8-B aligned), read by the emission
-                        uint2 iv = make_uint2(0, 0);
-                        if (s + 1 < a.n) iv = ld_ids(reinterpret_cast<const uint2*>(a.ids + s));
-                        else iv.x = __ldg(&a.ids[s]);
-                        *reinterpret_cast<uint2*>(S.idst + R + 2 * p) = iv;
+                        asm volatile("prefetch.global.L1 [%0];" ::"l"(a.ids + s));   // read by the emission
                         if (MODE == kF64Filter) {
                             const double2 c0 = ld_cand(a.xd + s);
                             v.x = (float)__dsub_rn(c0.x, o.x);
@@ -1532,11 +1523,10 @@ __global__ void __launch_bounds__(kQThreads, 7)   // 7 CTAs: 7 KB of shared memo
                     my += __popc(cur);
                     if (cur) {   // only words with hits are kept (the emission never skips a word)
                         S.bits[nw][lane] = cur;
-                        S.wtag[nw][lane] = R + 2 * (pa + i);
+                        S.wtag[nw][lane] = U0e + 2 * (pa + i);
                         ++nw;
                     }
                 }
-                R += 2 * npu;
             }
             QX_T(3);
             // ---- reserve the block's rows (one range: lane i's list at excl), T by id (a10)
@@ -1579,44 +1569,10 @@ __global__ void __launch_bounds__(kQThreads, 7)   // 7 CTAs: 7 KB of shared memo
 #endif
             QX_T(4);
             // ---- emission in rounds of <= kQOut ids (one round unless the block is heavy): every
-            // lane walks its hit bits (FLO) writing the ids into the output stage at its list's
+            // lane walks its hit bits (FLO) writing the ids (L1) into the output stage at its list's
             // offset (the stage is offset by the destination's misalignment); the stage is then
             // copied out with 16-B aligned streaming stores
             __syncwarp();   // (orders the words' stores before the reads below)
-            if (total + 3 <= (uint32_t)kQOut) {
-                // one round (the common case): word by word, bit by bit (MSB first)
-                const uint32_t mis = (uint32_t)(base & 3u);
-                uint32_t* dst = S.st.out + mis + excl;
-                for (uint32_t w = 0; w < nw; ++w) {
-                    uint32_t cb = S.bits[w][lane];
-                    const uint32_t* src = S.idst + S.wtag[w][lane];
-                    do {
-                        uint32_t z;
-                        asm("bfind.shiftamt.u32 %0, %1;" : "=r"(z) : "r"(cb));   // clz
-                        cb ^= 0x80000000u >> z;
-                        *dst++ = src[z];
-                    } while (cb);   // (stored words are non-empty)
-                }
-                __syncwarp();
-                QX_T(5);
-                uint32_t* gd = out + (base - mis);   // 16-B aligned
-                const uint32_t nch = (mis + total + 3) >> 2;
-                for (uint32_t ch = lane; ch < nch; ch += 32) {
-                    const uint4 v = reinterpret_cast<const uint4*>(S.st.out)[ch];
-                    const uint32_t e0 = 4 * ch;
-                    if (e0 >= mis && e0 + 4 <= mis + total) {
-                        stg_cs_v4(gd + e0, v);
-                    } else {
-                        const uint32_t w4[4] = {v.x, v.y, v.z, v.w};
-#pragma unroll
-                        for (int t = 0; t < 4; ++t)
-                            if (e0 + t >= mis && e0 + t < mis + total) stg_cs(gd + e0 + t, w4[t]);
-                    }
-                }
-                __syncwarp();   // the stage is rewritten by the next block
-                QX_T(6);
-                continue;
-            }
             uint32_t k = 0, cb = 0, src = 0, wi = 0;
             for (uint32_t r0 = 0; r0 < total;) {
                 const uint32_t mis = (uint32_t)((base + r0) & 3u);
@@ -1646,7 +1602,7 @@ __global__ void __launch_bounds__(kQThreads, 7)   // 7 CTAs: 7 KB of shared memo
                     uint32_t v[kQB];
 #pragma unroll
                     for (int u = 0; u < kQB; ++u)
-                        if (k + u < kend) v[u] = S.idst[pos[u]];
+                        if (k + u < kend) v[u] = __ldg(&a.ids[pos[u]]);   // (L1: prefetched by the staging)
 #pragma unroll
                     for (int u = 0; u < kQB; ++u)
                         if (k + u < kend) dst[k + u] = v[u];

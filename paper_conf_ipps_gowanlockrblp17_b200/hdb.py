@@ -58,7 +58,7 @@ class hdb_stats(ctypes.Structure):
                                     "bytes_d2h", "pool_grows")] + \
         [("n_streams", _int), ("n_devices", _int), ("kernel_launches", _u32), ("write_launches", _u32)] + \
         [(k, _dbl) for k in ("ms_grid", "ms_sample", "ms_count", "ms_scan", "ms_write_kernel", "ms_table_wall")] + \
-        [("single_pass", _int), ("ms_sort", _dbl), ("n_sparse_queries", _u64)]
+        [("single_pass", _int), ("ms_sort", _dbl), ("n_sparse_queries", _u64), ("query_lanes", _int)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}

@@ -95,6 +95,10 @@ def test_full_size_device_table_every_row(torch_cuda, name, eps, dtype):
         try:
             view = hdb.hdb_table_view_get(t)
             assert view.on_device and view.first_query == 0 and view.end_query == xy.shape[0]
+            # the default kernel choice: query lanes for the small groups beyond the L2 (C5's 800 MB
+            # point set, its sparse 99% of the area), the warp-per-group kernels below it
+            st = hdb.hdb_stats_get(ctx)
+            assert st["query_lanes"] == (1 if name == "C5" else 0), st
             _rows_equal(torch, xy, eps, dtype, view)
         finally:
             hdb.hdb_table_free(t)

@@ -25,7 +25,7 @@ METRICS = "dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum"
 def capture(wl, dtype="f64", kernel=0, split=0):
     log = f"/tmp/traffic_{wl}.csv"
     cmd = ["ncu", "--metrics", METRICS, "--clock-control", "none", "--csv", "--log-file", log,
-           "-k", "regex:k_fused|k_emit|k_sparse", sys.executable, os.path.join(ROOT, "bench.py"),
+           "-k", "regex:k_fused|k_emit|k_sparse|k_qlanes", sys.executable, os.path.join(ROOT, "bench.py"),
            "--workload", wl, "--steps", "1", "--warmup", "0", "--e2e-steps", "0", "--no-cpu-baseline",
            "--dtype", dtype, "--kernel", str(kernel), "--cell-split", str(split)]
     subprocess.run(cmd, check=True, capture_output=True)
@@ -42,8 +42,9 @@ def capture(wl, dtype="f64", kernel=0, split=0):
         d = per.setdefault(r[iid], {"kernel": r[ik]})
         d[r[im]] = float(r[iv].replace(",", "")) * scale
     launches = list(per.values())
-    # single pass: k_fused (+ k_sparse_fused for the sparse queries of the dense/sparse split)
-    fused = [d for d in launches if "k_fused" in d["kernel"] or "k_sparse_fused" in d["kernel"]]
+    # single pass: k_fused (+ k_sparse_fused / k_qlanes for the sparse / small groups of the split)
+    fused = [d for d in launches if "k_fused" in d["kernel"] or "k_sparse_fused" in d["kernel"]
+             or "k_qlanes" in d["kernel"]]
     if fused:
         pick, single = fused, True
     else:   # two passes: the write phase = k_emit + k_sparse<..., true>
