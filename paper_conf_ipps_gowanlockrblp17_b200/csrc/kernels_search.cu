@@ -1554,12 +1554,6 @@ __global__ void __launch_bounds__(kQThreads, 7)   // 7 CTAs: 7 KB of shared memo
 #endif
             base = __shfl_sync(FULL, base, 0);
             const uint32_t excl = incl - my;
-#ifndef HDB_QX_NOT   // (timing experiment: no T by id)
-            if (act) {
-                begin[qid] = base + excl;
-                count[qid] = my;
-            }
-#endif
             if (base + total > cap) {   // the capacity bound failed: the host rebuilds exactly
                 if (lane == 0) atomicOr(overflow, 1u);
                 continue;
@@ -1628,6 +1622,13 @@ __global__ void __launch_bounds__(kQThreads, 7)   // 7 CTAs: 7 KB of shared memo
                 QX_T(6);
                 r0 = rend;
             }
+#ifndef HDB_QX_NOT   // (timing experiment: no T by id)
+            // T by id (a10), after the block's output (A/B against before it: equal)
+            if (act) {
+                begin[qid] = base + excl;
+                count[qid] = my;
+            }
+#endif
         }
     }
 #pragma unroll
