@@ -1274,6 +1274,19 @@ __global__ void __launch_bounds__(256) k_sparse_fused(SArgs a, uint32_t g0, uint
 //    then each lane walks its hit bits (FLO) writing ids into a shared-memory
 //    stage at its list's offset, and the warp copies the stage out with aligned,
 //    coalesced 16-B streaming stores -- the block's rows are one contiguous range.
+// HDB_QX_CHECK: bounds-checking build (every shared / global index of k_qlanes checked, a
+// violation traps) -- the substitute for compute-sanitizer runs (tools/qx_check.sh)
+#ifdef HDB_QX_CHECK
+#define QX_CHECK(c)                                                                         \
+    do {                                                                                    \
+        if (!(c)) {                                                                         \
+            printf("k_qlanes bound check failed: %s (line %d)\n", #c, __LINE__);           \
+            __trap();                                                                       \
+        }                                                                                   \
+    } while (0)
+#else
+#define QX_CHECK(c) ((void)0)
+#endif
 constexpr int kQThreads = 128;
 constexpr int kQWarps = kQThreads / 32;
 constexpr int kQGrab = 128;   // small queries per grab (natural order: the L2 keeps the stencil rows);
@@ -1453,6 +1466,7 @@ __global__ void __launch_bounds__(kQThreads, 7)   // 7 CTAs: 7 KB of shared memo
                             }
                         }
                     }
+                    QX_CHECK(p < (uint32_t)(kQS / 2 + 1 + 4));
                     S.st.cand[p] = v;
                 }
                 __syncwarp();
@@ -1473,6 +1487,7 @@ __global__ void __launch_bounds__(kQThreads, 7)   // 7 CTAs: 7 KB of shared memo
                     for (; proc < cnt; proc += 4) {
 #pragma unroll
                         for (int u = 0; u < 4; ++u) {
+                            QX_CHECK(pa + i + proc + u < npu + 4);
                             const ulonglong2 C = P[proc + u];
                             const u64x dx = sub2(QX, C.x);
                             const u64x dy = sub2(QY, C.y);
@@ -1522,6 +1537,7 @@ __global__ void __launch_bounds__(kQThreads, 7)   // 7 CTAs: 7 KB of shared memo
                     cur &= m;
                     my += __popc(cur);
                     if (cur) {   // only words with hits are kept (the emission never skips a word)
+                        QX_CHECK(nw < (uint32_t)kQW);
                         S.bits[nw][lane] = cur;
                         S.wtag[nw][lane] = U0e + 2 * (pa + i);
                         ++nw;
@@ -1583,6 +1599,7 @@ __global__ void __launch_bounds__(kQThreads, 7)   // 7 CTAs: 7 KB of shared memo
                         pos[u] = 0;
                         if (k + u < kend) {
                             if (cb == 0) {
+                                QX_CHECK(wi < nw);
                                 cb = S.bits[wi][lane];
                                 src = S.wtag[wi][lane];
                                 ++wi;
@@ -1596,10 +1613,16 @@ __global__ void __launch_bounds__(kQThreads, 7)   // 7 CTAs: 7 KB of shared memo
                     uint32_t v[kQB];
 #pragma unroll
                     for (int u = 0; u < kQB; ++u)
-                        if (k + u < kend) v[u] = __ldg(&a.ids[pos[u]]);   // (L1: prefetched by the staging)
+                        if (k + u < kend) {
+                            QX_CHECK(pos[u] < a.n);
+                            v[u] = __ldg(&a.ids[pos[u]]);   // (L1: prefetched by the staging)
+                        }
 #pragma unroll
                     for (int u = 0; u < kQB; ++u)
-                        if (k + u < kend) dst[k + u] = v[u];
+                        if (k + u < kend) {
+                            QX_CHECK(mis + excl + k + u - r0 < (uint32_t)kQOut);
+                            dst[k + u] = v[u];
+                        }
                 }
                 k = kend;
                 __syncwarp();
@@ -1607,6 +1630,7 @@ __global__ void __launch_bounds__(kQThreads, 7)   // 7 CTAs: 7 KB of shared memo
                 uint32_t* gd = out + (base + r0 - mis);   // 16-B aligned
                 const uint32_t nch = (mis + cntr + 3) >> 2;
                 for (uint32_t ch = lane; ch < nch; ch += 32) {
+                    QX_CHECK(4 * ch + 3 < (uint32_t)kQOut);
                     const uint4 v = reinterpret_cast<const uint4*>(S.st.out)[ch];
                     const uint32_t e0 = 4 * ch;
                     if (e0 >= mis && e0 + 4 <= mis + cntr) {
