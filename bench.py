@@ -609,18 +609,21 @@ def main():
             hdb.hdb_table_free(t)
             return k
 
+        # the device path through the public clustering call: hdb_sweep with one (eps, minpts) on a
+        # sweep_on_device context -- grid, device table (position space) and GPU DBSCAN, labels D2H
+        ctx_dev = hdb.hdb_ctx_create(sweep_on_device=1, cell_split=args.cell_split, search_kernel=args.kernel)
+        lab_sweep = labels.reshape(1, 1, n)
+
         def e2e_device():
-            g = hdb.hdb_grid_build(ctx, xy_pin, eps)
-            t = hdb.hdb_neighbor_table_device(ctx, g)
-            hdb.hdb_grid_free(g)
-            _, _, k = hdb.hdb_dbscan(t, MINPTS, labels=labels, is_core=core)
-            hdb.hdb_table_free(t)
-            return k
+            return int(hdb.hdb_sweep(ctx_dev, xy_pin, [eps], [MINPTS], labels=lab_sweep)[1][0, 0])
 
         te, Pe = timed(e2e_table, args.e2e_steps)
         d2h_peak = pcie_d2h_peak(torch, dev)
         th, kh = timed(e2e_hybrid, max(1, args.e2e_steps - 1))
+        lab_hybrid = labels.copy()
         td, kd = timed(e2e_device, args.e2e_steps)
+        same_labels = bool(np.array_equal(lab_hybrid, labels))
+        hdb.hdb_ctx_destroy(ctx_dev)
         line["e2e"] = {"value": Pe / te, "unit": "pairs/s", "h2d_bytes_per_step": esz * n,
                        "d2h_bytes_per_step": 4 * Pe + 12 * n, "s_per_step": te,
                        "includes": "pinned host points -> H2D -> grid -> count -> batched write + D2H on 3 streams "
@@ -628,8 +631,9 @@ def main():
                        "points_clustered_per_sec_hybrid": n / th, "s_per_step_hybrid": th,
                        "hybrid": "e2e + host DBSCAN on T (minpts=4, all host cores) -- the paper's split",
                        "points_clustered_per_sec_device": n / td, "s_per_step_device": td,
-                       "device": "pinned host points -> device table -> GPU DBSCAN -> labels D2H (NEXT-4)",
-                       "n_clusters": kh, "n_clusters_device": kd,
+                       "device": "pinned host points -> hdb_sweep(sweep_on_device, one eps / minpts): grid, device "
+                                 "table in position space, GPU DBSCAN -> labels D2H (NEXT-4)",
+                       "n_clusters": kh, "n_clusters_device": kd, "labels_equal_hybrid_device": same_labels,
                        "pcie": {"d2h_peak_gbs": d2h_peak, "e2e_d2h_gbs": (4 * Pe + 12 * n) / te / 1e9,
                                 "frac": (4 * Pe + 12 * n) / te / 1e9 / d2h_peak,
                                 "peak_how": "pinned host <- device copy of 1 GiB, best of 5, measured in this run"}}

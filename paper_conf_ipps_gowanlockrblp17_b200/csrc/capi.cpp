@@ -471,7 +471,7 @@ hdb_status hdb_sweep(hdb_ctx* c, const void* xy, uint64_t n, hdb_dtype dt, const
             hdb_table* t = nullptr;
             try {
                 grid_build(c, xy, n, dt, eps[i], &g);
-                neighbor_table(c, g, true, &t);
+                neighbor_table(c, g, true, &t, /*pos_space=*/true);   // internal: clustered in position space
                 grid_free(g);
                 g = nullptr;
                 for (uint32_t j = 0; j < n_minpts; ++j) {

@@ -929,7 +929,7 @@ void count_phase(hdb_ctx* ctx, DevCtx& dc, const DevGrid& g, ShardState& st) {
 // then runs the exact two-pass path (a6-a8) -- if the mask table or the table
 // cannot be allocated or a reservation passed the capacity.
 bool single_pass_table(hdb_ctx* ctx, const DevGrid& g, hdb_table* t, hdb_stats& S, uint64_t est,
-                       bool exact_bound = false) {
+                       bool exact_bound = false, bool pos_space = false) {
     DevCtx& dc = ctx->dev[0];
     cudaStream_t s = dc.main;
     const uint64_t n = g.n_ids;   // rows of T (a banded grid holds fewer points)
@@ -954,11 +954,12 @@ bool single_pass_table(hdb_ctx* ctx, const DevGrid& g, hdb_table* t, hdb_stats& 
     Event e0, e1;
     HDB_CUDA(cudaEventRecord(e0.e, s));
     const uint64_t g0 = g.banded ? g.band_g0 : 0, g1 = g.banded ? g.band_g1 : g.n_groups;
+    pos_space = pos_space && !g.banded && n == g.n;   // whole, unsharded tables only
     launch_fused(g, g0, g1, nullptr, sc, masks.as<uint2>(), sc + 1, cap, nb.as<uint32_t>(), beg.as<uint64_t>(),
-                 cnt_id.as<uint32_t>(), (unsigned int*)(sc + 2), s);
+                 cnt_id.as<uint32_t>(), (unsigned int*)(sc + 2), s, pos_space);
     if (g.dl)   // dense/sparse split: the range's sparse queries reserve on the same counter
         launch_sparse_fused(g, g0, g1, sc, sc + 1, cap, nb.as<uint32_t>(), beg.as<uint64_t>(), cnt_id.as<uint32_t>(),
-                            (unsigned int*)(sc + 2), s);
+                            (unsigned int*)(sc + 2), s, pos_space);
     HDB_LAUNCH_CHECK();
     HDB_CUDA(cudaEventRecord(e1.e, s));
     HDB_CUDA(cudaMemcpyAsync(dc.pin + 4, sc, 24, cudaMemcpyDeviceToHost, s));
@@ -970,6 +971,7 @@ bool single_pass_table(hdb_ctx* ctx, const DevGrid& g, hdb_table* t, hdb_stats& 
     t->device = dc.device;
     t->dstream = s;
     t->npairs = P;
+    t->pos_space = pos_space;
     t->first_query = g.banded ? g.band_q0 : 0;
     t->end_query = g.banded ? g.band_q1 : n;
     if (!g.banded && n) {
@@ -1180,15 +1182,29 @@ uint32_t dbscan_device(const hdb_table* t, uint32_t minpts, int32_t* labels, uin
         dlab = DBuf(4 * n, s);
         L = dlab.as<int32_t>();
     }
-    uint8_t* C = core_dev ? core : dcore.as<uint8_t>();
+    // id space: the core flags are computed in the caller's array (or a device copy of it);
+    // position space: by position in dcore, then written out by id (into core / its copy)
+    DBuf ccopy;
+    uint8_t* C = (core_dev && !t->pos_space) ? core : dcore.as<uint8_t>();
+    uint8_t* Cout = nullptr;
+    if (t->pos_space && core) {
+        if (core_dev) {
+            Cout = core;
+        } else {
+            ccopy = DBuf(n, s);
+            Cout = ccopy.as<uint8_t>();
+        }
+    }
     launch_dbscan_device(t->begin, t->count, t->nbrs, t->rows, n, t->npairs, minpts, C, parent.as<uint32_t>(),
                          root.as<uint32_t>(), is_root.as<uint32_t>(), rank.as<uint32_t>(), giant.as<uint32_t>(),
-                         bits.as<uint32_t>(), sched.as<uint32_t>(), pre.as<uint64_t>(), temp.p, L, s);
+                         bits.as<uint32_t>(), sched.as<uint32_t>(), pre.as<uint64_t>(), temp.p, L, s, t->pos_space,
+                         Cout);
+    if (t->pos_space) C = Cout;   // the by-id flags (null when not asked for)
     HDB_LAUNCH_CHECK();
     uint32_t k = 0;
     HDB_CUDA(cudaMemcpyAsync(&k, rank.as<uint32_t>() + n, 4, cudaMemcpyDeviceToHost, s));
     if (!lab_dev) HDB_CUDA(cudaMemcpyAsync(labels, L, 4 * n, cudaMemcpyDeviceToHost, s));
-    if (core && !core_dev) HDB_CUDA(cudaMemcpyAsync(core, C, n, cudaMemcpyDeviceToHost, s));
+    if (core && !core_dev) HDB_CUDA(cudaMemcpyAsync(core, C, n, cudaMemcpyDeviceToHost, s));   // (by id)
     HDB_CUDA(cudaStreamSynchronize(s));
     return k;
 }
@@ -1227,7 +1243,7 @@ DevGrid without_qsplit(const DevGrid& g) {
     return r;
 }
 
-void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hdb_table** out) {
+void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hdb_table** out, bool pos_space) {
     auto t_wall0 = std::chrono::steady_clock::now();
     const uint64_t launches0 = g_kernel_launches.load();
     hdb_stats& S = ctx->stats;
@@ -1277,7 +1293,7 @@ void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hd
             S.ms_sample = 0;
             S.ms_sort = 0;
             S.planned_batch_pairs = S.planned_batches = 0;
-            if (single_pass_table(ctx, G0, t, S, G0.tests_total, true)) {   // (cannot overflow)
+            if (single_pass_table(ctx, G0, t, S, G0.tests_total, true, pos_space)) {   // (cannot overflow)
                 tr.mark("single-pass (exact bound)");
                 S.kernel_launches = (uint32_t)(g_kernel_launches.load() - launches0);
                 S.ms_table_wall =
@@ -1350,7 +1366,7 @@ void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hd
                 S.sample_pairs = eb;
                 S.est_pairs = eb * stride;
                 S.ms_sample = elapsed(es0, es1);
-                single = single_pass_table(ctx, G0, t, S, eb * stride);
+                single = single_pass_table(ctx, G0, t, S, eb * stride, false, pos_space);
             }
             if (single) {
                 double bb = 0;

@@ -216,12 +216,12 @@ void launch_count(const DevGrid& g, uint64_t g0, uint64_t g1, uint32_t* cnt, uns
 // over the query groups [g0, g1) (a process shard's band: its range); cnt may be null
 void launch_fused(const DevGrid& g, uint64_t g0, uint64_t g1, uint32_t* cnt, unsigned long long* tests, uint2* masks,
                   unsigned long long* pair_ctr, uint64_t cap, uint32_t* out, uint64_t* begin, uint32_t* count,
-                  unsigned int* overflow, cudaStream_t s);
+                  unsigned int* overflow, cudaStream_t s, bool pos_out = false);
 // single pass for the sparse queries (dense/sparse split): thread per query, rows reserved
 // on the same pair counter as launch_fused (run both on one stream)
 void launch_sparse_fused(const DevGrid& g, uint64_t g0, uint64_t g1, unsigned long long* tests,
                          unsigned long long* pair_ctr, uint64_t cap, uint32_t* out, uint64_t* begin, uint32_t* count,
-                         unsigned int* overflow, cudaStream_t s);
+                         unsigned int* overflow, cudaStream_t s, bool pos_out = false);
 void launch_write(const DevGrid& g, uint64_t g0, uint64_t g1, const uint64_t* off, uint64_t out_base,
                   uint32_t* out, int variant, int slot, const uint2* masks, cudaStream_t s,
                   uint64_t* begin = nullptr, uint32_t* count = nullptr);
@@ -240,7 +240,8 @@ void launch_dbscan_device(const uint64_t* begin, const uint32_t* count, const ui
                           uint64_t n, uint64_t npairs, uint32_t minpts, uint8_t* core, uint32_t* parent,
                           uint32_t* root, uint32_t* is_root, uint32_t* rank, uint32_t* giant, uint32_t* bits,
                           uint32_t* sched /* 2 x SM count */, uint64_t* pre /* n + 1 */, void* scan_temp,
-                          int32_t* labels, cudaStream_t s);
+                          int32_t* labels, cudaStream_t s, bool pos_space = false,
+                          uint8_t* core_out = nullptr);
 
 // the paper's kernels (kernels_paper.cu; search_kernel 7 / 8):
 // the key/value result set R of GPUCalcGlobal (Alg. 2) or GPUCalcShared (Alg. 3),
@@ -310,6 +311,9 @@ struct hdb_table {
     uint32_t* count = nullptr;
     uint32_t* nbrs = nullptr;
     uint32_t* rows = nullptr;   // device tables only: query ids in production (cell-sorted) order
+    // position space (internal tables of the device sweep only, never handed to the caller):
+    // nbrs hold sorted POSITIONS and begin / count are indexed by position; rows[pos] = id
+    bool pos_space = false;
     // ownership
     std::shared_ptr<hdb::PinnedPool> pool;   // non-null: begin/count/nbrs are pinned pool blocks
     size_t cap_begin = 0, cap_count = 0, cap_nbrs = 0;
@@ -324,7 +328,10 @@ int resolve_threads(int requested);
 // engine.cpp
 void grid_build(hdb_ctx* ctx, const void* xy, uint64_t n, hdb_dtype dt, double eps, hdb_grid** out);
 void grid_free(hdb_grid* g);
-void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hdb_table** out);
+// pos_space: a device-resident table in position space if the single pass builds it (DESIGN.md
+// "position space"); otherwise (two-pass fallback) an ordinary id-space table
+void neighbor_table(hdb_ctx* ctx, const hdb_grid* grid, bool device_resident, hdb_table** out,
+                    bool pos_space = false);
 void table_free(hdb_table* t);
 // dbscan.cpp
 uint32_t dbscan_host(const hdb_table* t, uint32_t minpts, int n_threads, int32_t* labels, uint8_t* core);

@@ -57,12 +57,15 @@ __device__ __forceinline__ uint32_t find_fast(const uint32_t* __restrict__ paren
     return x;
 }
 
-__device__ __forceinline__ void unite(uint32_t* __restrict__ parent, uint32_t a, uint32_t b) {
+// key: null in id space (an element's id is its index); in position space the ids of the
+// positions, so that a root is always its component's minimum core ID either way
+__device__ __forceinline__ void unite(uint32_t* __restrict__ parent, uint32_t a, uint32_t b,
+                                      const uint32_t* __restrict__ key) {
     while (true) {
         a = find_root(parent, a);
         b = find_root(parent, b);
         if (a == b) return;
-        if (a < b) {
+        if (key ? __ldg(&key[a]) < __ldg(&key[b]) : a < b) {
             const uint32_t t = a;
             a = b;
             b = t;
@@ -147,14 +150,14 @@ __global__ void __launch_bounds__(256) k_sample_link(const uint64_t* __restrict_
                                                      const uint32_t* __restrict__ count,
                                                      const uint32_t* __restrict__ nbrs,
                                                      const uint32_t* __restrict__ rows, uint64_t n, uint32_t k,
-                                                     uint32_t* __restrict__ parent) {
+                                                     uint32_t* __restrict__ parent, const uint32_t* __restrict__ key) {
     for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
         const uint32_t u = rows ? rows[i] : (uint32_t)i;
         const uint32_t pu = __ldcg(&parent[u]);
         if (pu == kNonCore) continue;
         const uint32_t v = nbrs[begin[u] + (uint64_t)count[u] * k / (kSampleLinks + 1)];
         const uint32_t pv = __ldcg(&parent[v]);
-        if (v != u && pv != kNonCore && pv != pu) unite(parent, u, v);
+        if (v != u && pv != kNonCore && pv != pu) unite(parent, u, v, key);
     }
 }
 
@@ -270,7 +273,7 @@ __global__ void __launch_bounds__(kUnionThreads, 1)
     k_union(const uint64_t* __restrict__ begin, const uint32_t* __restrict__ count, const uint32_t* __restrict__ nbrs,
             const uint32_t* __restrict__ rows, uint32_t* __restrict__ parent, const uint32_t* __restrict__ giant,
             const uint32_t* __restrict__ bits_a, const uint32_t* __restrict__ bits_b, uint32_t* __restrict__ sched,
-            uint32_t kRowsPerGrab) {
+            uint32_t kRowsPerGrab, const uint32_t* __restrict__ key) {
     const bool have_a = giant[0] != kNonCore, have_b = giant[1] != kNonCore;
     const uint32_t G = gridDim.x;
     const int lane = threadIdx.x & 31;
@@ -323,7 +326,7 @@ __global__ void __launch_bounds__(kUnionThreads, 1)
                     for (int k = 0; k < 4; ++k) {
                         // skip non-cores and v hanging directly under u's root; else follow the chain
                         if (p[k] != kNonCore && p[k] != ru && !(p[k] != v[k] && reaches(parent, p[k], ru))) {
-                            unite(parent, u, v[k]);
+                            unite(parent, u, v[k], key);
                             ru = find_fast(parent, u);
                         }
                     }
@@ -375,6 +378,48 @@ __global__ void __launch_bounds__(256) k_labels(const uint64_t* __restrict__ beg
     }
 }
 
+// Position space: roots are positions whose id is their
+// component's minimum core id; the root flags and the labels / core flags go out by id.
+__global__ void __launch_bounds__(256) k_flatten_pos(const uint8_t* __restrict__ core, uint64_t n,
+                                                     const uint32_t* __restrict__ parent, const uint32_t* __restrict__ key,
+                                                     uint32_t* __restrict__ root, uint32_t* __restrict__ is_root_id) {
+    for (uint64_t p = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; p < n; p += (uint64_t)gridDim.x * blockDim.x) {
+        uint32_t rt = (uint32_t)p;
+        if (core[p]) {
+            rt = find_fast(parent, (uint32_t)p);
+            if (rt == (uint32_t)p) is_root_id[key[p]] = 1u;   // (is_root_id zeroed before)
+        }
+        root[p] = rt;
+    }
+}
+__global__ void __launch_bounds__(256) k_labels_pos(const uint64_t* __restrict__ begin,
+                                                    const uint32_t* __restrict__ count,
+                                                    const uint32_t* __restrict__ nbrs, const uint8_t* __restrict__ core,
+                                                    const uint32_t* __restrict__ root, const uint32_t* __restrict__ rank,
+                                                    const uint32_t* __restrict__ key, uint64_t n,
+                                                    int32_t* __restrict__ labels, uint8_t* __restrict__ core_out) {
+    for (uint64_t p = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; p < n; p += (uint64_t)gridDim.x * blockDim.x) {
+        int32_t lab = -1;
+        const bool c = core[p];
+        if (c) {
+            lab = (int32_t)rank[key[root[p]]];
+        } else {
+            const uint32_t* L = nbrs + begin[p];
+            const uint32_t m = count[p];
+            for (uint32_t j = 0; j < m; ++j) {
+                const uint32_t v = L[j];
+                if (core[v]) {
+                    const int32_t cl = (int32_t)rank[key[root[v]]];
+                    if (lab < 0 || cl < lab) lab = cl;
+                }
+            }
+        }
+        const uint32_t id = key[p];
+        labels[id] = lab;
+        if (core_out) core_out[id] = c ? 1 : 0;
+    }
+}
+
 inline unsigned blocks_for(uint64_t n, unsigned cap = 148u * 16u) {
     uint64_t b = (n + 255) / 256;
     return (unsigned)(b < 1 ? 1 : (b < cap ? b : cap));
@@ -385,12 +430,17 @@ inline unsigned blocks_for(uint64_t n, unsigned cap = 148u * 16u) {
 void launch_dbscan_device(const uint64_t* begin, const uint32_t* count, const uint32_t* nbrs, const uint32_t* rows,
                           uint64_t n, uint64_t npairs, uint32_t minpts, uint8_t* core, uint32_t* parent, uint32_t* root,
                           uint32_t* is_root, uint32_t* rank, uint32_t* giant, uint32_t* bits, uint32_t* sched,
-                          uint64_t* pre, void* scan_temp, int32_t* labels, cudaStream_t s) {
+                          uint64_t* pre, void* scan_temp, int32_t* labels, cudaStream_t s, bool pos_space,
+                          uint8_t* core_out) {
     if (n == 0) return;
+    // position space: every per-point pass walks positions (the production order itself), roots
+    // are hooked by id (key = rows: position -> id)
+    const uint32_t* key = pos_space ? rows : nullptr;
+    if (pos_space) rows = nullptr;
     k_core_init<<<blocks_for(n), 256, 0, s>>>(count, n, minpts, core, parent);
-    const uint32_t* walk = 16.0 * (double)n > kIdOrderBytes ? nullptr : rows;   // null: id order
+    const uint32_t* walk = 16.0 * (double)n > kIdOrderBytes ? nullptr : rows;   // null: index order
     for (uint32_t k = 1; k <= kSampleLinks; ++k) {
-        k_sample_link<<<blocks_for(n), 256, 0, s>>>(begin, count, nbrs, walk, n, k, parent);
+        k_sample_link<<<blocks_for(n), 256, 0, s>>>(begin, count, nbrs, walk, n, k, parent, key);
         k_compress<<<blocks_for(n), 256, 0, s>>>(n, parent);
     }
     k_giant<<<1, kGiantSamples, 0, s>>>(rows, n, parent, giant);
@@ -409,10 +459,17 @@ void launch_dbscan_device(const uint64_t* begin, const uint32_t* count, const ui
     k_sched_init<<<1, 256, 0, s>>>(pre, (uint32_t)n, npairs, (uint32_t)sms, sched);
     const uint32_t grab = (double)npairs >= kLongListPairs * (double)n ? kGrabLong : kGrabShort;
     k_union<<<sms, kUnionThreads, 0, s>>>(begin, count, nbrs, rows, parent, giant, bits, bits + (n + 31) / 32, sched,
-                                          grab);
-    k_flatten<<<blocks_for(n), 256, 0, s>>>(core, n, parent, root, is_root);
-    scan_u32_to_u32(is_root, rank, n, scan_temp, s);
-    k_labels<<<blocks_for(n), 256, 0, s>>>(begin, count, nbrs, walk, core, root, rank, n, labels);
+                                          grab, key);
+    if (pos_space) {
+        cudaMemsetAsync(is_root, 0, 4 * n, s);
+        k_flatten_pos<<<blocks_for(n), 256, 0, s>>>(core, n, parent, key, root, is_root);
+        scan_u32_to_u32(is_root, rank, n, scan_temp, s);
+        k_labels_pos<<<blocks_for(n), 256, 0, s>>>(begin, count, nbrs, core, root, rank, key, n, labels, core_out);
+    } else {
+        k_flatten<<<blocks_for(n), 256, 0, s>>>(core, n, parent, root, is_root);
+        scan_u32_to_u32(is_root, rank, n, scan_temp, s);
+        k_labels<<<blocks_for(n), 256, 0, s>>>(begin, count, nbrs, walk, core, root, rank, n, labels);
+    }
     g_kernel_launches += 8 + 2 * kSampleLinks;
 }
 

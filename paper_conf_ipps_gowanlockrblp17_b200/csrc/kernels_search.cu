@@ -78,7 +78,13 @@ struct SArgs {
     // memory with cp.async one chunk ahead (the natural-order launches of large point sets,
     // whose candidates come from the L2 / DRAM rather than the L1)
     int pf;
+    // position-space output (internal tables of the device sweep):
+    // the single-pass kernels emit sorted positions instead of ids and write T by position
+    int pos_out;
 };
+
+// the table entry for the point at sorted position s: its original id, or s itself
+__device__ __forceinline__ uint32_t out_id(const SArgs& a, uint32_t s) { return a.pos_out ? s : __ldg(&a.ids[s]); }
 
 __device__ __forceinline__ void dense_range(const SArgs& a, uint32_t& i0, uint32_t& i1) {
     if (a.dl) {
@@ -845,7 +851,7 @@ __device__ __forceinline__ void window_ids(const SArgs& a, const VSpan* vsp, VCu
         if ((uint32_t)kk < nck) {
             bool v0, v1;
             const uint32_t s0 = vc_pair(cur, vsp, a.nspan, 32 * (v * kWin + kk) + lane, v0, v1);
-            if (v0 | v1) ids[kk] = ld_ids((const uint2*)(a.ids + s0));
+            if (v0 | v1) ids[kk] = a.pos_out ? make_uint2(s0, s0 + 1) : ld_ids((const uint2*)(a.ids + s0));
         }
     }
 }
@@ -1021,7 +1027,7 @@ __global__ void __launch_bounds__(kFusedThreads, kFusedMinBlocks)
         base = __shfl_sync(FULL, base, 0);
         const uint32_t excl = incl - my;
         if ((uint32_t)lane < m.nq) {
-            const uint32_t id = __ldg(&a.ids[m.qs + lane]);
+            const uint32_t id = out_id(a, m.qs + lane);
             if (cnt) cnt[m.qs + lane] = my;   // counts in sorted order (optional)
 #ifndef HDB_QX_NOT
             begin[id] = base + excl;
@@ -1204,14 +1210,14 @@ __global__ void __launch_bounds__(256) k_sparse_fused(SArgs a, uint32_t g0, uint
                 uint32_t k = sp.x;
                 for (; k + 4 <= sp.y; k += 4) {   // four loads in flight (latency-bound thread)
                     const bool h0 = test(k), h1 = test(k + 1), h2 = test(k + 2), h3 = test(k + 3);
-                    if (h0) { if (m < kSparseBuf) buf[m] = __ldg(&a.ids[k]); ++m; }
-                    if (h1) { if (m < kSparseBuf) buf[m] = __ldg(&a.ids[k + 1]); ++m; }
-                    if (h2) { if (m < kSparseBuf) buf[m] = __ldg(&a.ids[k + 2]); ++m; }
-                    if (h3) { if (m < kSparseBuf) buf[m] = __ldg(&a.ids[k + 3]); ++m; }
+                    if (h0) { if (m < kSparseBuf) buf[m] = out_id(a, k); ++m; }
+                    if (h1) { if (m < kSparseBuf) buf[m] = out_id(a, k + 1); ++m; }
+                    if (h2) { if (m < kSparseBuf) buf[m] = out_id(a, k + 2); ++m; }
+                    if (h3) { if (m < kSparseBuf) buf[m] = out_id(a, k + 3); ++m; }
                 }
                 for (; k < sp.y; ++k)
                     if (test(k)) {
-                        if (m < kSparseBuf) buf[m] = __ldg(&a.ids[k]);
+                        if (m < kSparseBuf) buf[m] = out_id(a, k);
                         ++m;
                     }
             }
@@ -1229,7 +1235,7 @@ __global__ void __launch_bounds__(256) k_sparse_fused(SArgs a, uint32_t g0, uint
         base = __shfl_sync(FULL, base, 31);
         const uint64_t b = base + (incl - m);
         if (!act) continue;
-        const uint32_t id = __ldg(&a.ids[q]);
+        const uint32_t id = out_id(a, q);
         begin[id] = b;
         count[id] = m;
         if (base + total > cap) {   // the capacity bound failed: the host rebuilds exactly
@@ -1244,7 +1250,7 @@ __global__ void __launch_bounds__(256) k_sparse_fused(SArgs a, uint32_t g0, uint
             for (uint32_t r = 0; r < a.nspan; ++r) {
                 const uint2 sp = __ldg(&a.cspan[a.nspan * c + r]);
                 for (uint32_t k = sp.x; k < sp.y; ++k)
-                    if (test(k)) o[w++] = __ldg(&a.ids[k]);
+                    if (test(k)) o[w++] = out_id(a, k);
             }
         }
     }
@@ -1413,7 +1419,7 @@ __global__ void __launch_bounds__(kQThreads, 7)   // 7 CTAs: 7 KB of shared memo
             QX_T(1);
             const bool act = (uint32_t)lane < Q;
             const uint32_t q = e.x, c = e.y;
-            const uint32_t qid = act ? __ldg(&a.ids[q]) : 0u;   // T by id (used after the reservation)
+            const uint32_t qid = act ? out_id(a, q) : 0u;   // T by id (used after the reservation)
             double2 o = make_double2(0, 0);
             u64x QX, QY;
             if (MODE == kF64Filter) {
@@ -1615,7 +1621,7 @@ __global__ void __launch_bounds__(kQThreads, 7)   // 7 CTAs: 7 KB of shared memo
                     for (int u = 0; u < kQB; ++u)
                         if (k + u < kend) {
                             QX_CHECK(pos[u] < a.n);
-                            v[u] = __ldg(&a.ids[pos[u]]);   // (L1: prefetched by the staging)
+                            v[u] = out_id(a, pos[u]);   // (L1: prefetched by the staging)
                         }
 #pragma unroll
                     for (int u = 0; u < kQB; ++u)
@@ -1809,6 +1815,7 @@ SArgs args_of(const DevGrid& g) {
     a.nx = g.nx;
     a.n = (uint32_t)g.n;
     a.nb2_b = g.nb2_b;
+    a.pos_out = 0;
     return a;
 }
 
@@ -2010,9 +2017,10 @@ void launch_fused_mode(const SArgs& a, uint64_t g0, uint64_t g1, uint64_t ngd, u
 
 void launch_fused(const DevGrid& g, uint64_t g0, uint64_t g1, uint32_t* cnt, unsigned long long* tests, uint2* masks,
                   unsigned long long* pair_ctr, uint64_t cap, uint32_t* out, uint64_t* begin, uint32_t* count,
-                  unsigned int* overflow, cudaStream_t s) {
+                  unsigned int* overflow, cudaStream_t s, bool pos_out) {
     if (g1 <= g0) return;
     SArgs a = args_of(g);
+    a.pos_out = pos_out ? 1 : 0;
     // heavy groups first (whole ranges only: ord lists every group): C2 eps 0.45 2.50 -> 2.10 ms
     if (g0 == 0 && g1 == g.n_groups && use_cost_order(g)) a.ord = g.ord;
     a.pf = HDB_PF && !a.ord && g.dtype == HDB_F64;   // the natural order: point sets beyond the L2
@@ -2033,11 +2041,12 @@ void launch_fused(const DevGrid& g, uint64_t g0, uint64_t g1, uint32_t* cnt, uns
 
 void launch_sparse_fused(const DevGrid& g, uint64_t g0, uint64_t g1, unsigned long long* tests,
                          unsigned long long* pair_ctr, uint64_t cap, uint32_t* out, uint64_t* begin, uint32_t* count,
-                         unsigned int* overflow, cudaStream_t s) {
+                         unsigned int* overflow, cudaStream_t s, bool pos_out) {
     if (!g.sql || g.n_sparse_q == 0 || g1 <= g0) return;
     if (g.qsplit && (g.dtype == HDB_F32 || g.filter_b)) {
         // small groups (query-lane classification): blocks of up to 32 queries, one per lane
-        const SArgs a = args_of(g);
+        SArgs a = args_of(g);
+        a.pos_out = pos_out ? 1 : 0;
         static int bps[2] = {0, 0};
         const int f64 = g.dtype == HDB_F64;
         if (!bps[f64]) {
@@ -2065,13 +2074,15 @@ void launch_sparse_fused(const DevGrid& g, uint64_t g0, uint64_t g1, unsigned lo
         ++g_kernel_launches;
         return;
     }
+    SArgs as = args_of(g);
+    as.pos_out = pos_out ? 1 : 0;
     const unsigned blocks =
         (unsigned)std::max<uint64_t>(1, std::min<uint64_t>((g.n_sparse_q + 255) / 256, 148 * HDB_SPARSE_BLOCKS));
     if (g.dtype == HDB_F64)
-        k_sparse_fused<true><<<blocks, 256, 0, s>>>(args_of(g), (uint32_t)g0, (uint32_t)g1, tests, pair_ctr, cap, out,
+        k_sparse_fused<true><<<blocks, 256, 0, s>>>(as, (uint32_t)g0, (uint32_t)g1, tests, pair_ctr, cap, out,
                                                     begin, count, overflow);
     else
-        k_sparse_fused<false><<<blocks, 256, 0, s>>>(args_of(g), (uint32_t)g0, (uint32_t)g1, tests, pair_ctr, cap, out,
+        k_sparse_fused<false><<<blocks, 256, 0, s>>>(as, (uint32_t)g0, (uint32_t)g1, tests, pair_ctr, cap, out,
                                                      begin, count, overflow);
     ++g_kernel_launches;
 }
