@@ -433,6 +433,40 @@ def test_sweep_matches_oracle(torch_cuda, on_device):
             assert np.array_equal(labels[i, j], want[0])
 
 
+@pytest.mark.parametrize("case", ["sparse_split", "query_lanes", "f32"])
+def test_device_sweep_position_space(torch_cuda, monkeypatch, case):
+    """The device sweep clusters in position space (tables of sorted positions, T by
+    position, union-find over positions with roots hooked by original id): through
+    the single pass's three kernels -- k_fused with k_sparse_fused on SDSS-like
+    sparse groups, with k_qlanes (forced) on dense-skew small groups, and f32 input
+    -- the labels equal the oracle's canonical labelling (and the host sweep's)."""
+    if case == "sparse_split":
+        xy, eps_list = datagen.subsample(datagen.sdss_like(), 25_000, seed=12), (0.2, 0.6)
+    elif case == "query_lanes":
+        monkeypatch.setenv("HDB_QLANES", "1")
+        xy, eps_list = datagen.dense_skew(25_000, seed=13), (4.0, 9.0)
+    else:
+        xy, eps_list = datagen.subsample(datagen.tec_like(), 20_000, seed=14).astype(np.float32), (0.3, 0.9)
+    mp = (4, 12)
+    ctx = _ctx(sweep_on_device=1)
+    try:
+        labels, k = hdb.hdb_sweep(ctx, xy, eps_list, mp)
+        st = hdb.hdb_stats_get(ctx)
+    finally:
+        hdb.hdb_ctx_destroy(ctx)
+    if case == "sparse_split":
+        assert st["n_sparse_queries"] > 0 and not st["query_lanes"]
+    if case == "query_lanes":
+        assert st["n_sparse_queries"] > 0 and st["query_lanes"]
+    dt = "f32" if case == "f32" else "f64"
+    for i, eps in enumerate(eps_list):
+        off, nbr = oracle.eps_join(xy, eps, dtype=dt)
+        for j, m in enumerate(mp):
+            want = oracle.dbscan(off, nbr, m)
+            assert k[i, j] == want[2]
+            assert np.array_equal(labels[i, j], want[0])
+
+
 # ------------------------------------------------------------------ full-size sampled rows
 def _sampled_rows_check(xy, eps, m_rows=1500, seed=0, dtype="f64", **opts):
     b, c, v, view, st = lib_table(xy, eps, device=True, **opts)
