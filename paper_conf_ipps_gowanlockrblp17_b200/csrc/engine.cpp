@@ -665,7 +665,7 @@ void build_dev(hdb_ctx* ctx, DevCtx& dc, const void* xy, PtrInfo where, uint64_t
         scan_u32_to_u32(dflag.as<uint32_t>(), dpre.as<uint32_t>(), NG, temp.p, s);
         scan_u32_to_u32(sqn.as<uint32_t>(), spre.as<uint32_t>(), NG, temp.p, s);
         launch_group_lists(g.gstart, g.gcell, ngd, NG, dpre.as<uint32_t>(), spre.as<uint32_t>(), dl.as<uint32_t>(),
-                           sql.as<uint2>(), s);
+                           sql.as<uint2>(), qrule, s);
         HDB_LAUNCH_CHECK();
     }
     {

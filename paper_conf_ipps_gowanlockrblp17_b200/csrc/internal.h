@@ -173,7 +173,8 @@ constexpr int kMaskWin = HDB_KWIN;   // chunks per window of the hit-mask layout
 void launch_order_scatter(const uint8_t* gbin, const uint32_t* ng_dev, uint64_t n, uint32_t* ohist, uint32_t* ord,
                           cudaStream_t s);
 void launch_group_lists(const uint32_t* gstart, const uint32_t* gcell, const uint32_t* ng_dev, uint64_t n,
-                        const uint32_t* dpre, const uint32_t* spre, uint32_t* dl, uint2* sql, cudaStream_t s);
+                        const uint32_t* dpre, const uint32_t* spre, uint32_t* dl, uint2* sql, bool qlanes,
+                        cudaStream_t s);
 
 // scans (kernels_scan.cu): exclusive scan of in[0..n) into out[0..n], out[n] = total
 size_t scan_temp_bytes(uint64_t n);

@@ -719,6 +719,24 @@ __global__ void __launch_bounds__(256) k_order_scatter(const uint8_t* __restrict
     }
 }
 
+// dl and sql, thread per group (the tests rule: sparse groups hold 1-2 queries)
+__global__ void __launch_bounds__(256) k_group_lists_tpg(const uint32_t* __restrict__ gstart,
+                                                         const uint32_t* __restrict__ gcell,
+                                                         const uint32_t* __restrict__ ng_dev, uint64_t n,
+                                                         const uint32_t* __restrict__ dpre,
+                                                         const uint32_t* __restrict__ spre, uint32_t* __restrict__ dl,
+                                                         uint2* __restrict__ sql) {
+    const uint64_t ng = *ng_dev;
+    for (uint64_t g = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; g < ng; g += (uint64_t)gridDim.x * blockDim.x) {
+        if (dpre[g + 1] != dpre[g]) {
+            dl[dpre[g]] = (uint32_t)g;
+        } else {
+            const uint32_t j = spre[g], m = spre[g + 1] - j, qs = gstart[g], c = gcell[g];
+            for (uint32_t i = 0; i < m; ++i) sql[j + i] = make_uint2(qs + i, c);
+        }
+    }
+}
+
 // dl (dense groups) and sql (the sparse / small groups' queries).  A warp takes 32
 // consecutive groups: their sql entries form one contiguous range of the list, staged in
 // shared memory by the groups' lanes and written out with coalesced stores (a thread
@@ -1069,9 +1087,15 @@ void launch_order_scatter(const uint8_t* gbin, const uint32_t* ng_dev, uint64_t 
 }
 
 void launch_group_lists(const uint32_t* gstart, const uint32_t* gcell, const uint32_t* ng_dev, uint64_t n,
-                        const uint32_t* dpre, const uint32_t* spre, uint32_t* dl, uint2* sql, cudaStream_t s) {
+                        const uint32_t* dpre, const uint32_t* spre, uint32_t* dl, uint2* sql, bool qlanes,
+                        cudaStream_t s) {
     if (n == 0) return;
-    k_group_lists<<<grid_for(n, 128), 128, 0, s>>>(gstart, gcell, ng_dev, n, dpre, spre, dl, sql);
+    // the query-lane rule's small groups hold ~11 queries each: warp-staged coalesced runs;
+    // the tests rule's sparse groups 1-2: a thread per group (A/B: C2 eps 0.45 step 2.40 vs 2.52 ms)
+    if (qlanes)
+        k_group_lists<<<grid_for(n, 128), 128, 0, s>>>(gstart, gcell, ng_dev, n, dpre, spre, dl, sql);
+    else
+        k_group_lists_tpg<<<grid_for(n), 256, 0, s>>>(gstart, gcell, ng_dev, n, dpre, spre, dl, sql);
     ++g_kernel_launches;
 }
 

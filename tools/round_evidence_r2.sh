@@ -19,7 +19,7 @@ timeout 900 python bench.py --impl reference --steps 5 --warmup 1 > gpurun_out/$
 for wl in C5-eps0.5 C2-eps0.45; do
   ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/${T}_launches_$wl.csv \
     python bench.py --workload $wl --steps 2 --warmup 1 --e2e-steps 0 --no-cpu-baseline > /dev/null 2>&1
-  ncu --set full --clock-control none --import-source on -k regex:"k_fused" -c 1 -o gpurun_out/${T}_prof_$wl \
+  ncu --set full --clock-control none --import-source on -k regex:"k_fused|k_qlanes" -c 2 -o gpurun_out/${T}_prof_$wl \
     python bench.py --workload $wl --steps 1 --warmup 0 --e2e-steps 0 --no-cpu-baseline > /dev/null 2>&1
 done
 timeout 900 python tools/shard_sim.py C5-eps0.5 > gpurun_out/${T}_shards_C5.json 2>> gpurun_out/${T}_bench.err
