@@ -20,6 +20,10 @@
 //                 over core neighbours (NEXT-2; the paper runs variants, not one
 //                 variant, in parallel).
 #include <algorithm>
+#include <chrono>
+#include <cstdio>
+#include <cstdlib>
+#include <string>
 #include <atomic>
 #include <cstring>
 #include <memory>
@@ -105,6 +109,19 @@ void parallel_for(int T, uint64_t n, F&& f) {
 }
 
 uint32_t dbscan_par(const hdb_table* t, uint32_t minpts, int T, int32_t* labels, uint8_t* core) {
+    // HDB_TRACE=1: wall time of each phase, to stderr
+    const char* tre = std::getenv("HDB_TRACE");
+    const bool trace = tre && *tre == '1';
+    auto tlast = std::chrono::steady_clock::now();
+    std::string tlog;
+    auto mark = [&](const char* what) {
+        if (!trace) return;
+        const auto now = std::chrono::steady_clock::now();
+        char buf[96];
+        snprintf(buf, sizeof buf, " %s=%.2f", what, std::chrono::duration<double, std::milli>(now - tlast).count());
+        tlog += buf;
+        tlast = now;
+    };
     const uint64_t n = t->n;
     const uint64_t* B = t->begin;
     const uint32_t* C = t->count;
@@ -116,11 +133,29 @@ uint32_t dbscan_par(const hdb_table* t, uint32_t minpts, int T, int32_t* labels,
             parent[p].store((uint32_t)p, std::memory_order_relaxed);
         }
     });
+    mark("init");
     // Afforest-style pre-pass (as the device code): two rounds of one sampled
     // link per core, each followed by a compression of every core to its root.
+    // The sampled list entry and then its parent / core flag are two dependent random reads
+    // per core (ids are a random permutation of space): software prefetch, the list entry
+    // 2 D iterations ahead and its parent / core flag D ahead, keeps ~2 D misses in flight
+    // per thread instead of one.
+    constexpr uint64_t D = 16;
     for (uint32_t k = 1; k <= 2; ++k) {
         parallel_for(T, n, [&](uint64_t a, uint64_t b, int) {
             for (uint64_t u = a; u < b; ++u) {
+                if (u + 2 * D < b) {
+                    const uint64_t w = u + 2 * D;
+                    __builtin_prefetch(&V[B[w] + (uint64_t)C[w] * k / 3]);
+                }
+                if (u + D < b) {
+                    const uint64_t w = u + D;
+                    if (core[w] && C[w]) {
+                        const uint32_t vw = V[B[w] + (uint64_t)C[w] * k / 3];
+                        __builtin_prefetch(&parent[vw]);
+                        __builtin_prefetch(&core[vw]);
+                    }
+                }
                 if (!core[u] || C[u] == 0) continue;
                 const uint32_t v = V[B[u] + (uint64_t)C[u] * k / 3];
                 if (v != u && core[v]) uf_union(parent.get(), (uint32_t)u, v);
@@ -131,6 +166,7 @@ uint32_t dbscan_par(const hdb_table* t, uint32_t minpts, int T, int32_t* labels,
                 if (core[p]) parent[p].store(uf_find(parent.get(), (uint32_t)p), std::memory_order_relaxed);
         });
     }
+    mark("sample_links");
     // the two most frequent roots among 1024 sampled points (>= 1/8 of them):
     // giant components A and B, with membership bitmaps
     const uint32_t kNone = 0xffffffffu;
@@ -172,6 +208,7 @@ uint32_t dbscan_par(const hdb_table* t, uint32_t minpts, int T, int32_t* labels,
     }
     auto inA = [&](uint32_t v) { return gA != kNone && ((bitA[v >> 6] >> (v & 63)) & 1); };
     auto inB = [&](uint32_t v) { return gB != kNone && ((bitB[v >> 6] >> (v & 63)) & 1); };
+    mark("giants");
     // Main pass.  Each core-core edge not inside A or B is taken once:
     //   u in A: none; u in B: v in A; otherwise: v in A or B, or v < u.
     {
@@ -207,6 +244,7 @@ uint32_t dbscan_par(const hdb_table* t, uint32_t minpts, int T, int32_t* labels,
             for (auto& x : th) x.join();
         }
     }
+    mark("union");
     // roots -> cluster numbers in increasing root (= minimum core) id
     std::vector<uint32_t> root(n ? n : 1);
     std::vector<uint64_t> part_cnt(T + 1, 0);
@@ -240,6 +278,7 @@ uint32_t dbscan_par(const hdb_table* t, uint32_t minpts, int T, int32_t* labels,
         part_cnt[0] = pre[T];
     }
     (void)chunk;
+    mark("roots+ranks");
     const uint32_t nclusters = (uint32_t)part_cnt[0];
     parallel_for(T, n, [&](uint64_t a, uint64_t b, int) {
         for (uint64_t p = a; p < b; ++p) {
@@ -259,6 +298,8 @@ uint32_t dbscan_par(const hdb_table* t, uint32_t minpts, int T, int32_t* labels,
             }
         }
     });
+    mark("labels");
+    if (trace) fprintf(stderr, "[hdb trace] dbscan_par n=%llu threads=%d:%s\n", (unsigned long long)n, T, tlog.c_str());
     return nclusters;
 }
 
