@@ -1,5 +1,5 @@
 #!/bin/bash
-# ncu --set full (with source) of one kernel on one workload: bash tools/r3_ncu_q.sh TAG WORKLOAD KREGEX
+# ncu --set full (with source) of one kernel on one workload: bash tools/ncu_kernel.sh TAG WORKLOAD KREGEX
 cd "$(dirname "$0")/.."
 T=$1; WL=$2; K=$3
 ncu --set full --clock-control none --import-source on -k regex:"$K" -c 1 -o gpurun_out/${T}_prof_$WL \
