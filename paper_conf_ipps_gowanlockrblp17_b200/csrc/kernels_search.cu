@@ -1293,6 +1293,9 @@ __global__ void __launch_bounds__(256) k_sparse_fused(SArgs a, uint32_t g0, uint
 #else
 #define QX_CHECK(c) ((void)0)
 #endif
+#ifndef HDB_QX_FULLB
+#define HDB_QX_FULLB 1
+#endif
 constexpr int kQThreads = 128;
 constexpr int kQWarps = kQThreads / 32;
 constexpr int kQGrab = 128;   // small queries per grab (natural order: the L2 keeps the stencil rows);
@@ -1598,23 +1601,44 @@ __global__ void __launch_bounds__(kQThreads, 7)   // 7 CTAs: 7 KB of shared memo
                 uint32_t* dst = S.st.out + mis + excl - r0;
                 // kQB hits per step: positions first, then the id loads, then the stores
                 constexpr int kQB = 8;
+                // the next hit's sorted position (MSB first), loading the next word when cb runs out
+                auto next_pos = [&]() -> uint32_t {
+                    if (cb == 0) {
+                        QX_CHECK(wi < nw);
+                        cb = S.bits[wi][lane];
+                        src = S.wtag[wi][lane];
+                        ++wi;
+                    }
+                    uint32_t z;
+                    asm("bfind.shiftamt.u32 %0, %1;" : "=r"(z) : "r"(cb));   // clz
+                    cb ^= 0x80000000u >> z;
+                    return src + z;
+                };
+#if HDB_QX_FULLB
+                // whole batches without per-slot bounds, then the remainder one by one
+                for (; k + kQB <= kend; k += kQB) {
+                    uint32_t pos[kQB], v[kQB];
+#pragma unroll
+                    for (int u = 0; u < kQB; ++u) pos[u] = next_pos();
+#pragma unroll
+                    for (int u = 0; u < kQB; ++u) {
+                        QX_CHECK(pos[u] < a.n);
+                        v[u] = out_id(a, pos[u]);   // (L1: prefetched by the staging)
+                    }
+#pragma unroll
+                    for (int u = 0; u < kQB; ++u) {
+                        QX_CHECK(mis + excl + k + u - r0 < (uint32_t)kQOut);
+                        dst[k + u] = v[u];
+                    }
+                }
+                for (; k < kend; ++k) dst[k] = out_id(a, next_pos());
+#else
                 for (; k < kend; k += kQB) {
                     uint32_t pos[kQB];
 #pragma unroll
                     for (int u = 0; u < kQB; ++u) {
                         pos[u] = 0;
-                        if (k + u < kend) {
-                            if (cb == 0) {
-                                QX_CHECK(wi < nw);
-                                cb = S.bits[wi][lane];
-                                src = S.wtag[wi][lane];
-                                ++wi;
-                            }
-                            uint32_t z;
-                            asm("bfind.shiftamt.u32 %0, %1;" : "=r"(z) : "r"(cb));   // clz
-                            cb ^= 0x80000000u >> z;
-                            pos[u] = src + z;
-                        }
+                        if (k + u < kend) pos[u] = next_pos();
                     }
                     uint32_t v[kQB];
 #pragma unroll
@@ -1630,6 +1654,7 @@ __global__ void __launch_bounds__(kQThreads, 7)   // 7 CTAs: 7 KB of shared memo
                             dst[k + u] = v[u];
                         }
                 }
+#endif
                 k = kend;
                 __syncwarp();
                 QX_T(5);
