@@ -85,6 +85,11 @@ struct SArgs {
 
 // the table entry for the point at sorted position s: its original id, or s itself
 __device__ __forceinline__ uint32_t out_id(const SArgs& a, uint32_t s) { return a.pos_out ? s : __ldg(&a.ids[s]); }
+template <bool POS>
+__device__ __forceinline__ uint32_t qout(const SArgs& a, uint32_t s) {
+    if (POS) return s;
+    return __ldg(&a.ids[s]);
+}
 
 __device__ __forceinline__ void dense_range(const SArgs& a, uint32_t& i0, uint32_t& i1) {
     if (a.dl) {
@@ -1336,7 +1341,9 @@ __device__ unsigned int g_qx_done;
 #else
 #define QX_T(i) ((void)0)
 #endif
-template <int MODE>   // kF64Filter (block-local f32 filter + exact f64 replay) or kF32 (exact f32)
+// MODE: kF64Filter (block-local f32 filter + exact f64 replay) or kF32 (exact f32);
+// POS: position-space output (the device sweep's internal tables), a compile-time choice
+template <int MODE, bool POS>
 __global__ void __launch_bounds__(kQThreads, 7)   // 7 CTAs: 7 KB of shared memory per warp
     k_qlanes(SArgs a, uint32_t g0, uint32_t g1, uint32_t grab, unsigned int* __restrict__ ctr,
              unsigned long long* __restrict__ tests_out, unsigned long long* __restrict__ pair_ctr, uint64_t cap,
@@ -1422,7 +1429,7 @@ __global__ void __launch_bounds__(kQThreads, 7)   // 7 CTAs: 7 KB of shared memo
             QX_T(1);
             const bool act = (uint32_t)lane < Q;
             const uint32_t q = e.x, c = e.y;
-            const uint32_t qid = act ? out_id(a, q) : 0u;   // T by id (used after the reservation)
+            const uint32_t qid = act ? qout<POS>(a, q) : 0u;   // T by id (used after the reservation)
             double2 o = make_double2(0, 0);
             u64x QX, QY;
             if (MODE == kF64Filter) {
@@ -1623,7 +1630,7 @@ __global__ void __launch_bounds__(kQThreads, 7)   // 7 CTAs: 7 KB of shared memo
 #pragma unroll
                     for (int u = 0; u < kQB; ++u) {
                         QX_CHECK(pos[u] < a.n);
-                        v[u] = out_id(a, pos[u]);   // (L1: prefetched by the staging)
+                        v[u] = qout<POS>(a, pos[u]);   // (L1: prefetched by the staging)
                     }
 #pragma unroll
                     for (int u = 0; u < kQB; ++u) {
@@ -1631,7 +1638,7 @@ __global__ void __launch_bounds__(kQThreads, 7)   // 7 CTAs: 7 KB of shared memo
                         dst[k + u] = v[u];
                     }
                 }
-                for (; k < kend; ++k) dst[k] = out_id(a, next_pos());
+                for (; k < kend; ++k) dst[k] = qout<POS>(a, next_pos());
 #else
                 for (; k < kend; k += kQB) {
                     uint32_t pos[kQB];
@@ -1645,7 +1652,7 @@ __global__ void __launch_bounds__(kQThreads, 7)   // 7 CTAs: 7 KB of shared memo
                     for (int u = 0; u < kQB; ++u)
                         if (k + u < kend) {
                             QX_CHECK(pos[u] < a.n);
-                            v[u] = out_id(a, pos[u]);   // (L1: prefetched by the staging)
+                            v[u] = qout<POS>(a, pos[u]);   // (L1: prefetched by the staging)
                         }
 #pragma unroll
                     for (int u = 0; u < kQB; ++u)
@@ -2075,8 +2082,8 @@ void launch_sparse_fused(const DevGrid& g, uint64_t g0, uint64_t g1, unsigned lo
         static int bps[2] = {0, 0};
         const int f64 = g.dtype == HDB_F64;
         if (!bps[f64]) {
-            if (f64) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps[1], k_qlanes<kF64Filter>, kQThreads, 0);
-            else cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps[0], k_qlanes<kF32>, kQThreads, 0);
+            if (f64) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps[1], k_qlanes<kF64Filter, false>, kQThreads, 0);
+            else cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps[0], k_qlanes<kF32, false>, kQThreads, 0);
             if (bps[f64] < 1) bps[f64] = 1;
         }
         // the range's small queries (whole range: all of them; a band's share is ~ its groups')
@@ -2090,12 +2097,17 @@ void launch_sparse_fused(const DevGrid& g, uint64_t g0, uint64_t g1, unsigned lo
         const uint64_t need = (nq + grab - 1) / grab;   // grabs (extra CTAs of a band exit at once)
         const unsigned ctas = (unsigned)std::max<uint64_t>(
             1, std::min<uint64_t>((uint64_t)148 * bps[f64], (need + kQWarps - 1) / kQWarps));
-        if (f64)
-            k_qlanes<kF64Filter><<<ctas, kQThreads, 0, s>>>(a, (uint32_t)g0, (uint32_t)g1, grab, ctr, tests, pair_ctr, cap, out, begin, count,
-                                                            overflow);
-        else
-            k_qlanes<kF32><<<ctas, kQThreads, 0, s>>>(a, (uint32_t)g0, (uint32_t)g1, grab, ctr, tests, pair_ctr, cap, out, begin, count,
-                                                      overflow);
+        auto go = [&](auto kern) {
+            kern<<<ctas, kQThreads, 0, s>>>(a, (uint32_t)g0, (uint32_t)g1, grab, ctr, tests, pair_ctr, cap, out, begin,
+                                            count, overflow);
+        };
+        if (f64) {
+            if (pos_out) go(k_qlanes<kF64Filter, true>);
+            else go(k_qlanes<kF64Filter, false>);
+        } else {
+            if (pos_out) go(k_qlanes<kF32, true>);
+            else go(k_qlanes<kF32, false>);
+        }
         ++g_kernel_launches;
         return;
     }

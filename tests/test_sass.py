@@ -61,7 +61,7 @@ def test_every_f32_predicate_kernel_has_no_ffma(sass):
     thread-per-query kernels, the sampled count, the paper's two kernels, the
     query-lane single pass): fl(fl(dx^2) + fl(dy^2)) must never be contracted."""
     ks = {k: v for k, v in sass.items() if re.search(_F32_KERNELS, k)}
-    assert len(ks) == 9, sorted(ks)
+    assert len(ks) == 10, sorted(ks)   # (k_qlanes<0>: id and position output)
     for name, body in ks.items():
         assert "FFMA" not in body, name
 
