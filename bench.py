@@ -46,6 +46,8 @@ WORKLOADS = {
     **{f"C3L-eps{e:.2f}": dict(gen=lambda: datagen.sdss_like(datagen.C3_N_LARGE, seed=4), eps=e,
                                desc=f"SDSS-like n=5,000,000 eps={e:.2f} minpts=4") for e in datagen.C3_EPS},
     "C5-eps0.5": dict(gen=datagen.dense_skew, eps=0.5, desc="dense-skew n=50,000,000 eps=0.5 minpts=4"),
+    # the stretch point of the dense-skew set (BASELINE configs[4]: "large eps"): ~4x the pairs
+    "C5-eps1.0": dict(gen=datagen.dense_skew, eps=1.0, desc="dense-skew n=50,000,000 eps=1.0 minpts=4"),
 }
 MINPTS = 4
 SWEEP_WORKLOADS = {

@@ -549,6 +549,16 @@ def test_c5_full_size_sampled_rows(torch_cuda):
     assert 3.5e9 < view.npairs < 4.5e9
 
 
+def test_c5_eps1_full_size_sampled_rows(torch_cuda):
+    """C5's stretch point, eps 1.0 (~4x the pairs of eps 0.5: a ~63 GB device table;
+    the cells are 4x as full, so the groups are dense and take k_fused): sampled rows
+    (plus the longest lists) against the oracle."""
+    xy = datagen.dense_skew()
+    view, st = _sampled_rows_check(xy, datagen.C5_EPS[1], m_rows=300, seed=6)
+    assert st["single_pass"] == 1
+    assert 1.4e10 < view.npairs < 1.8e10
+
+
 def test_exact_f64_kernel_variant(torch_cuda):
     """search_kernel=1 forces the exact-f64-only kernel, 2 the write pass that
     recomputes the tests instead of replaying stored hit masks; all must equal

@@ -10,7 +10,7 @@ timeout 1500 python -m pytest tests -m gpu -q --timeout 900 > gpurun_out/${T}_py
 echo "PYTEST: $(tail -1 gpurun_out/${T}_pytest.txt)"; grep -E "^FAILED|^E  " gpurun_out/${T}_pytest.txt | head -5
 timeout 900 python bench.py --steps 20 --warmup 5 > gpurun_out/${T}_bench_default.json 2> gpurun_out/${T}_bench.err
 echo "default rc=$?"
-for wl in C1-eps0.5 C2-eps0.45 C2-eps0.15 C2-eps1.40 C3-eps0.07 C3-eps0.20 C3L-eps0.07 C3L-eps0.20; do
+for wl in C1-eps0.5 C2-eps0.45 C2-eps0.15 C2-eps1.40 C3-eps0.07 C3-eps0.20 C3L-eps0.07 C3L-eps0.20 C5-eps1.0; do
   timeout 600 python bench.py --workload $wl --steps 10 --warmup 3 --e2e-steps 2 --no-cpu-baseline > gpurun_out/${T}_bench_$wl.json 2>> gpurun_out/${T}_bench.err
 done
 timeout 600 python bench.py --workload C2-eps0.45 --dtype f32 --steps 10 --warmup 3 --e2e-steps 0 --no-cpu-baseline > gpurun_out/${T}_bench_C2-eps0.45-f32.json 2>> gpurun_out/${T}_bench.err
