@@ -1303,7 +1303,10 @@ __global__ void __launch_bounds__(256) k_sparse_fused(SArgs a, uint32_t g0, uint
 #endif
 constexpr int kQThreads = 128;
 constexpr int kQWarps = kQThreads / 32;
-constexpr int kQGrab = 128;   // small queries per grab (natural order: the L2 keeps the stencil rows);
+#ifndef HDB_QX_GRAB
+#define HDB_QX_GRAB 128
+#endif
+constexpr int kQGrab = HDB_QX_GRAB;   // small queries per grab (natural order: the L2 keeps the stencil rows);
                               // fewer when the warps would otherwise not all get work
 // kQW, kQS, kQCX: internal.h (the grid build's classification bounds them)
 constexpr int kQOut = 1280;                // output stage (ids): a block's rows in one round (C5: ~1,150)
